@@ -1,0 +1,212 @@
+/*
+ * ltpg.h -- C-ABI of the B200-native LTPG per-batch pipeline.
+ *
+ * One call of ltpg_run_batch() runs one batch of LTPG's deterministic
+ * optimistic concurrency control (§IV, Alg. 1):
+ *   execute (readMem / recordTID / recordLS)
+ *   -> conflict detection (rcheck / wcheck)
+ *   -> write-back (getStatus -> writeMem / Abort)
+ * with TID order as the serial order and conflicting txns
+ * returned for re-execution in the next batch with their original TIDs
+ * (P:110-112).  Commit rule (R1): txn of rank r aborts
+ * iff it reads or writes a conflict unit that a smaller rank wrote (RAW/WAW),
+ * or adds to a unit a smaller rank plainly wrote; delayed ADDs commute.
+ * A conflict unit is (table, row, column group) (P:239 row-level splitting).
+ *
+ * Conventions (all functions):
+ *  - Every call returns int: 0 = LTPG_OK, negative = error; no C++ exception
+ *    crosses the ABI.  ltpg_last_error() gives a one-line reason.
+ *  - The caller owns every input and result buffer; the library owns the
+ *    device store, indexes, conflict marks and scratch (plain cudaMalloc).
+ *  - Pointers are HOST pointers unless the corresponding *_on_device flag is
+ *    set, in which case they are device pointers on the db's device (e.g. a
+ *    torch tensor's data_ptr()).  Host pointers should be pinned for speed.
+ *  - Validation happens before any mutation: a malformed batch returns
+ *    LTPG_EINVAL and leaves the database unchanged (batch-level atomicity).
+ *    LTPG_ECAPACITY (append region full) is also detected before write-back.
+ *    A CUDA fault poisons the db: later calls return LTPG_EPOISONED.
+ *  - All integer state: int64 columns with wrap-around (uint64) arithmetic,
+ *    u64 keys (0xFFFFFFFFFFFFFFFF reserved), u32 batch ranks as conflict TIDs.
+ */
+#ifndef LTPG_H
+#define LTPG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define LTPG_API __attribute__((visibility("default")))
+#else
+#define LTPG_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ---------------------------------------------------------- */
+enum {
+  LTPG_OK = 0,
+  LTPG_EINVAL = -1,     /* malformed argument or batch; nothing changed            */
+  LTPG_ENOMEM = -2,     /* device allocation failed                                */
+  LTPG_ECAPACITY = -3,  /* an append region / index would overflow; nothing changed */
+  LTPG_ECUDA = -4,      /* CUDA runtime error (db poisoned)                         */
+  LTPG_ENCCL = -5,      /* NCCL error (multi-GPU exchange; db poisoned)             */
+  LTPG_EPOISONED = -6,  /* an earlier device error poisoned this db: destroy it      */
+  LTPG_EINTERNAL = -7   /* broken invariant (e.g. a required TPC-C row missing)      */
+};
+
+/* ---- OPS mode: one 16-byte record per operation ------------------------------ */
+enum { LTPG_SELECT = 0, LTPG_UPDATE = 1, LTPG_ADD = 2, LTPG_INSERT = 3, LTPG_DELETE = 4, LTPG_SCAN = 5 };
+#define LTPG_COL_COUNT 0xFFFFu      /* SCAN column: return the number of present keys */
+#define LTPG_STATIC 0xFFu           /* col_group value: column never written, reads unmarked */
+#define LTPG_NOT_FOUND INT64_MIN    /* read result for an absent key */
+
+/* Operation semantics (DESIGN.md §"OPS semantics"):
+ *  SELECT(t,key,col)       -> value of col in the pre-batch snapshot, or NOT_FOUND.
+ *  UPDATE(t,key,col,arg)   read-modify-write col <- col + arg; returns the pre-image.
+ *  ADD(t,key,col,arg)      delayed blind add on an ADD column; returns 0.
+ *  INSERT(t,key,arg)       new row, column c = arg + c; returns 1, or 0 and a user
+ *                          abort (status 2) if key is present in the snapshot.
+ *  DELETE(t,key)           returns 1 (deleted) or NOT_FOUND.
+ *  SCAN(t,key,col,aux=len) keys [key, key+len): sum of col over present keys
+ *                          (or their count if col == LTPG_COL_COUNT).
+ * Ops on absent keys return NOT_FOUND and count as a read of the key's row.
+ * Within one txn a key that is written is touched by no other op (EINVAL). */
+typedef struct {
+  uint64_t key;
+  uint8_t kind;
+  uint8_t table;
+  uint16_t col;
+  uint32_t aux;
+} ltpg_op;
+
+/* ---- PROC mode: TPC-C stored procedures, 128-byte parameter blocks ---- */
+enum { LTPG_NEW_ORDER = 0, LTPG_PAYMENT = 1, LTPG_ORDER_STATUS = 2, LTPG_DELIVERY = 3, LTPG_STOCK_LEVEL = 4 };
+#define LTPG_PARAM_BYTES 128
+#define LTPG_PROC_RESULTS 4         /* int64 result slots per PROC txn */
+
+/* TPC-C schema (integer-only): table ids and column order.  Keys:
+ *   W = w;  D = w*10+d;  C = D*3000+c;  I = i;  S = w*100000+i;
+ *   O = NO = (D<<32)|o;  OL = O*16+ol;  HISTORY is keyless.            */
+enum { LTPG_T_WAREHOUSE = 0, LTPG_T_DISTRICT = 1, LTPG_T_CUSTOMER = 2, LTPG_T_HISTORY = 3,
+       LTPG_T_NEW_ORDER = 4, LTPG_T_ORDER = 5, LTPG_T_ORDER_LINE = 6, LTPG_T_ITEM = 7,
+       LTPG_T_STOCK = 8, LTPG_TPCC_TABLES = 9 };
+/* WAREHOUSE  : W_TAX, W_YTD
+ * DISTRICT   : D_TAX, D_YTD, D_NEXT_O_ID, D_NEXT_DELIV_O_ID
+ * CUSTOMER   : C_DISCOUNT, C_CREDIT, C_LAST, C_FIRST, C_INIT_O_ID, C_BALANCE,
+ *              C_YTD_PAYMENT, C_PAYMENT_CNT, C_DELIVERY_CNT
+ * HISTORY    : H_C_ID, H_C_D_ID, H_C_W_ID, H_D_ID, H_W_ID, H_DATE, H_AMOUNT, H_TID, H_SEQ
+ * NEW_ORDER  : NO_O_ID
+ * ORDER      : O_C_ID, O_ENTRY_D, O_OL_CNT, O_ALL_LOCAL, O_CARRIER_ID
+ * ORDER_LINE : OL_I_ID, OL_SUPPLY_W_ID, OL_QUANTITY, OL_AMOUNT, OL_DELIVERY_D
+ * ITEM       : I_PRICE, I_IM_ID
+ * STOCK      : S_QUANTITY, S_YTD, S_ORDER_CNT, S_REMOTE_CNT
+ * Column groups / ADD flags select "strict" or "delayed" mode. */
+
+/* Parameter blocks (little endian, 128 bytes):
+ * NewOrder   : u16 w | u8 d | u8 n_lines | u16 c | u8 rbk | u8 pad |
+ *              15 x { u32 i | u16 supply_w | u8 qty | u8 pad }
+ * Payment    : u16 w | u8 d | u8 by_name | u16 c_w | u8 c_d | u8 pad | u16 c_id |
+ *              u16 c_last | u32 pad | i64 amount | ...
+ * OrderStatus: u16 w | u8 d | u8 by_name | u16 c_id | u16 c_last | ...
+ * Delivery   : u16 w | u8 carrier | ...
+ * StockLevel : u16 w | u8 d | u8 threshold | ...
+ * Results (4 x int64 per txn):
+ * NewOrder [o_id (0 unless committed), total, sum(OL_AMOUNT), 0]
+ * Payment  [c_id, C_BALANCE pre-image (strict) or 0 (delayed), 0, 0]
+ * OrderStatus [c_id, C_BALANCE, O_CARRIER_ID, sum(OL_DELIVERY_D)]
+ * Delivery [districts delivered, sum of delivered OL_AMOUNT, 0, 0]
+ * StockLevel [low-stock count, D_NEXT_O_ID, 0, 0]                               */
+
+/* ---- txn status ------------------------------------------------------------- */
+enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
+
+/* ---- configuration ------------------------------------------------------------ */
+#define LTPG_FLAG_NO_GROUPING   (1u << 0)  /* A/B: disable adaptive warp division (§V-B) */
+#define LTPG_FLAG_NO_MARK_FILTER (1u << 1) /* A/B: always issue the atomicMin mark        */
+#define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
+
+typedef struct {
+  int device;                   /* CUDA device ordinal                                  */
+  int rank, world;              /* partition of this process; world = 1: single GPU     */
+  const void* nccl_unique_id;   /* 128-byte ncclUniqueId (world > 1), else NULL          */
+  uint32_t max_txns;            /* per-batch capacity                                    */
+  uint32_t max_ops;             /* OPS mode per-batch op capacity                         */
+  uint32_t flags;               /* LTPG_FLAG_*                                           */
+  uint32_t n_tables;            /* number of table ids used (<= 16)                      */
+  uint32_t n_warehouses;        /* PROC mode: global TPC-C W (validation, routing)       */
+} ltpg_config;
+
+typedef struct ltpg_db ltpg_db;  /* opaque, library-owned device state */
+
+/* Create a database on config->device.  *out receives the handle. */
+LTPG_API int ltpg_create_db(const ltpg_config* config, ltpg_db** out);
+
+/* Table descriptor.  col_group[c] in [0, n_groups) or LTPG_STATIC; col_is_add[c]
+ * marks a delayed-ADD column (its group may hold ADD columns only).  Tables with
+ * static columns accept no DELETE; tables with n_groups == 0 accept no INSERT. */
+typedef struct {
+  uint32_t n_cols;              /* <= 16                                                 */
+  const uint8_t* col_group;     /* host, n_cols                                          */
+  const uint8_t* col_is_add;    /* host, n_cols                                          */
+  uint32_t n_groups;            /* mutable column groups (conflict units per row)        */
+  uint64_t capacity_rows;       /* rows incl. the append region                          */
+  uint32_t has_pk;              /* 1: u64 primary key + hash index; 0: keyless (append)  */
+  uint32_t owner_rule;          /* multi-GPU: 0 replicated, 1 TPC-C warehouse, 2 key range */
+} ltpg_table_desc;
+
+/* Define table_id and load n_rows rows.  keys: host u64[n_rows] (NULL if keyless);
+ * cols: host int64, column-major [n_cols][n_rows].  Duplicate keys -> EINVAL. */
+LTPG_API int ltpg_load_table(ltpg_db* db, uint32_t table_id, const ltpg_table_desc* desc, uint64_t n_rows,
+                    const uint64_t* keys, const int64_t* cols);
+
+enum { LTPG_MODE_OPS = 0, LTPG_MODE_TPCC = 1 };
+
+typedef struct {
+  uint32_t n_txns;
+  const uint64_t* tid;          /* [n_txns], strictly increasing (arrival order)  */
+  uint32_t mode;                /* LTPG_MODE_OPS or LTPG_MODE_TPCC                       */
+  uint32_t n_ops;               /* OPS: total ops                                         */
+  const uint32_t* op_begin;     /* OPS: CSR [n_txns+1]                                    */
+  const ltpg_op* ops;           /* OPS: [n_ops]                                           */
+  const int64_t* op_arg;        /* OPS: [n_ops]                                           */
+  const uint8_t* proc_type;     /* TPCC: [n_txns]                                         */
+  const uint8_t* proc_params;   /* TPCC: [n_txns][128]                                    */
+  int64_t batch_clock;          /* deterministic "now" for TPC-C dates                    */
+  int inputs_on_device;         /* 1: the pointers above are device pointers             */
+  void* stream;                 /* cudaStream_t to run on (NULL = legacy default)         */
+} ltpg_batch;
+
+typedef struct {
+  float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;
+  uint32_t n_commit, n_conflict, n_user_abort;
+} ltpg_stats;
+
+typedef struct {
+  uint32_t* commit_bits;        /* [ceil(n_txns/32)]: bit r%32 of word r/32 = committed   */
+  uint8_t* status;              /* [n_txns]: LTPG_ST_*                                    */
+  uint32_t* abort_idx;          /* [n_txns] capacity: ranks of conflict aborts, ascending */
+  uint32_t* n_aborted;          /* [1]                                                    */
+  int64_t* reads;               /* OPS: [n_ops]; TPCC: [4*n_txns]; NULL = not returned    */
+  int outputs_on_device;        /* 1: the pointers above are device pointers             */
+  ltpg_stats* stats;            /* optional host struct: per-stage device times           */
+} ltpg_result;
+
+/* Run one batch; synchronous on batch->stream (returns when results are in place). */
+LTPG_API int ltpg_run_batch(ltpg_db* db, const ltpg_batch* batch, ltpg_result* result);
+
+/* Canonical dump (valid rows only): keyed tables sorted by key, keyless tables by
+ * the full column tuple.  Call with keys == cols == NULL to get *n_rows only.
+ * keys: host u64[n_rows]; cols: host int64 [n_cols][n_rows]. */
+LTPG_API int ltpg_dump_table(ltpg_db* db, uint32_t table_id, uint64_t* n_rows, uint64_t* keys, int64_t* cols);
+
+LTPG_API void ltpg_destroy_db(ltpg_db* db);
+LTPG_API const char* ltpg_last_error(const ltpg_db* db);
+/* Library version string, e.g. "ltpg-b200 0.1 sm_100a". */
+LTPG_API const char* ltpg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LTPG_H */

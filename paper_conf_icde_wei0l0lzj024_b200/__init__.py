@@ -1,0 +1,275 @@
+"""Thin Python binding of the B200 LTPG C-ABI (include/ltpg.h).
+
+Argument marshalling only: every step of a batch (validation, warp division,
+execute, marks, conflict detection, write-back, result compaction) runs in the
+CUDA kernels of libltpg.so.  There is no CPU fallback: importing this package
+fails if the shared library is missing, and every call that reaches a device
+fails if there is no CUDA device.
+
+Names follow the C-ABI: ltpg_create_db / ltpg_load_table / ltpg_run_batch /
+ltpg_dump_table / ltpg_destroy_db / ltpg_last_error.  The ``Database`` class is
+a convenience wrapper over them that accepts numpy arrays (host) or torch
+tensors (host pinned or CUDA).
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libltpg.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError("libltpg.so not built: run `python -m paper_conf_icde_wei0l0lzj024_b200.build` "
+                      "(or __graft_entry__.build()); there is no CPU fallback")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+# ---- constants (include/ltpg.h) ------------------------------------------------------
+LTPG_OK, LTPG_EINVAL, LTPG_ENOMEM, LTPG_ECAPACITY = 0, -1, -2, -3
+LTPG_ECUDA, LTPG_ENCCL, LTPG_EPOISONED, LTPG_EINTERNAL = -4, -5, -6, -7
+ERR_NAMES = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECAPACITY", -4: "ECUDA", -5: "ENCCL",
+             -6: "EPOISONED", -7: "EINTERNAL"}
+LTPG_MODE_OPS, LTPG_MODE_TPCC = 0, 1
+LTPG_FLAG_NO_GROUPING = 1 << 0
+LTPG_FLAG_NO_MARK_FILTER = 1 << 1
+LTPG_FLAG_LOOPBACK_SHIFT = 8
+LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
+
+c_u32, c_u64, c_i64, c_int, c_vp = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p
+
+
+class ltpg_config(ctypes.Structure):
+    _fields_ = [("device", c_int), ("rank", c_int), ("world", c_int), ("nccl_unique_id", c_vp),
+                ("max_txns", c_u32), ("max_ops", c_u32), ("flags", c_u32), ("n_tables", c_u32),
+                ("n_warehouses", c_u32)]
+
+
+class ltpg_table_desc(ctypes.Structure):
+    _fields_ = [("n_cols", c_u32), ("col_group", c_vp), ("col_is_add", c_vp), ("n_groups", c_u32),
+                ("capacity_rows", c_u64), ("has_pk", c_u32), ("owner_rule", c_u32)]
+
+
+class ltpg_batch(ctypes.Structure):
+    _fields_ = [("n_txns", c_u32), ("tid", c_vp), ("mode", c_u32), ("n_ops", c_u32), ("op_begin", c_vp),
+                ("ops", c_vp), ("op_arg", c_vp), ("proc_type", c_vp), ("proc_params", c_vp),
+                ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp)]
+
+
+class ltpg_stats(ctypes.Structure):
+    _fields_ = [("ms_upload", ctypes.c_float), ("ms_group", ctypes.c_float), ("ms_exec", ctypes.c_float),
+                ("ms_detect", ctypes.c_float), ("ms_exchange", ctypes.c_float),
+                ("ms_writeback", ctypes.c_float), ("ms_download", ctypes.c_float),
+                ("n_commit", c_u32), ("n_conflict", c_u32), ("n_user_abort", c_u32)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class ltpg_result(ctypes.Structure):
+    _fields_ = [("commit_bits", c_vp), ("status", c_vp), ("abort_idx", c_vp), ("n_aborted", c_vp),
+                ("reads", c_vp), ("outputs_on_device", c_int), ("stats", ctypes.POINTER(ltpg_stats))]
+
+
+_lib.ltpg_create_db.restype = c_int
+_lib.ltpg_create_db.argtypes = [ctypes.POINTER(ltpg_config), ctypes.POINTER(c_vp)]
+_lib.ltpg_load_table.restype = c_int
+_lib.ltpg_load_table.argtypes = [c_vp, c_u32, ctypes.POINTER(ltpg_table_desc), c_u64, c_vp, c_vp]
+_lib.ltpg_run_batch.restype = c_int
+_lib.ltpg_run_batch.argtypes = [c_vp, ctypes.POINTER(ltpg_batch), ctypes.POINTER(ltpg_result)]
+_lib.ltpg_dump_table.restype = c_int
+_lib.ltpg_dump_table.argtypes = [c_vp, c_u32, ctypes.POINTER(c_u64), c_vp, c_vp]
+_lib.ltpg_destroy_db.restype = None
+_lib.ltpg_destroy_db.argtypes = [c_vp]
+_lib.ltpg_last_error.restype = ctypes.c_char_p
+_lib.ltpg_last_error.argtypes = [c_vp]
+_lib.ltpg_version.restype = ctypes.c_char_p
+_lib.ltpg_version.argtypes = []
+
+# C-ABI names, re-exported unchanged
+ltpg_create_db = _lib.ltpg_create_db
+ltpg_load_table = _lib.ltpg_load_table
+ltpg_run_batch = _lib.ltpg_run_batch
+ltpg_dump_table = _lib.ltpg_dump_table
+ltpg_destroy_db = _lib.ltpg_destroy_db
+ltpg_last_error = _lib.ltpg_last_error
+ltpg_version = _lib.ltpg_version
+
+EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_dump_table", "ltpg_destroy_db",
+            "ltpg_last_error", "ltpg_version"]
+
+
+class LtpgError(RuntimeError):
+    def __init__(self, rc, msg):
+        super().__init__("%s (%d): %s" % (ERR_NAMES.get(rc, "?"), rc, msg))
+        self.rc = rc
+
+
+def _is_torch(x):
+    return type(x).__module__.startswith("torch")
+
+
+def _ptr(x):
+    if x is None:
+        return None
+    if _is_torch(x):
+        return c_vp(x.data_ptr())
+    return x.ctypes.data_as(c_vp)
+
+
+def _on_device(x):
+    return _is_torch(x) and x.is_cuda
+
+
+class Database:
+    """One device database (tables + PK indexes + conflict marks) on one GPU."""
+
+    def __init__(self, n_tables, max_txns, max_ops=0, device=0, flags=0, n_warehouses=0, rank=0, world=1,
+                 nccl_unique_id=None):
+        self._keep = []
+        cfg = ltpg_config(device=device, rank=rank, world=world, nccl_unique_id=None, max_txns=max_txns,
+                          max_ops=max_ops, flags=flags, n_tables=n_tables, n_warehouses=n_warehouses)
+        if nccl_unique_id is not None:
+            buf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+            self._keep.append(buf)
+            cfg.nccl_unique_id = ctypes.cast(buf, c_vp)
+        h = c_vp()
+        rc = ltpg_create_db(ctypes.byref(cfg), ctypes.byref(h))
+        self.h = h
+        if rc:
+            msg = ltpg_last_error(h).decode() if h.value else ""
+            self.close()
+            raise LtpgError(rc, msg)
+        self.n_tables = n_tables
+        self.max_txns = max_txns
+        self.max_ops = max_ops
+        self.n_cols = {}
+        self.has_pk = {}
+        self._out = None
+
+    def close(self):
+        if getattr(self, "h", None) is not None and self.h.value:
+            ltpg_destroy_db(self.h)
+        self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, rc):
+        if rc:
+            raise LtpgError(rc, ltpg_last_error(self.h).decode())
+
+    def load_table(self, t, col_group, col_is_add, n_groups, keys, cols, capacity=None, has_pk=True,
+                   owner_rule=0):
+        g = np.ascontiguousarray(col_group, dtype=np.uint8)
+        a = np.ascontiguousarray(col_is_add, dtype=np.uint8)
+        cols = np.ascontiguousarray(cols, dtype=np.int64)
+        n = cols.shape[1] if cols.ndim == 2 else 0
+        k = None if (keys is None or not has_pk) else np.ascontiguousarray(keys, dtype=np.uint64)
+        cap = int(capacity if capacity is not None else max(n, 1))
+        d = ltpg_table_desc(n_cols=len(g), col_group=_ptr(g), col_is_add=_ptr(a), n_groups=n_groups,
+                            capacity_rows=cap, has_pk=int(bool(has_pk)), owner_rule=owner_rule)
+        self._check(ltpg_load_table(self.h, t, ctypes.byref(d), n, _ptr(k), _ptr(cols)))
+        self.n_cols[t] = len(g)
+        self.has_pk[t] = bool(has_pk)
+
+    # -- batches -------------------------------------------------------------------------
+    def _outputs(self, n, n_reads, device_out):
+        if device_out:
+            import torch
+            dev = torch.device("cuda", torch.cuda.current_device())
+            return {"status": torch.empty(n, dtype=torch.uint8, device=dev),
+                    "commit_bits": torch.empty((n + 31) // 32, dtype=torch.int32, device=dev),
+                    "abort_idx": torch.empty(max(n, 1), dtype=torch.int32, device=dev),
+                    "n_aborted": torch.zeros(1, dtype=torch.int32, device=dev),
+                    "reads": torch.empty(max(n_reads, 1), dtype=torch.int64, device=dev)}
+        return {"status": np.empty(n, np.uint8), "commit_bits": np.empty((n + 31) // 32, np.uint32),
+                "abort_idx": np.empty(max(n, 1), np.uint32), "n_aborted": np.zeros(1, np.uint32),
+                "reads": np.empty(max(n_reads, 1), np.int64)}
+
+    def _run(self, bt, n, n_reads, want_reads, device_out, stats, out):
+        if out is None:
+            out = self._outputs(n, n_reads, device_out)
+        st = ltpg_stats() if stats else None
+        res = ltpg_result(commit_bits=_ptr(out["commit_bits"]), status=_ptr(out["status"]),
+                          abort_idx=_ptr(out["abort_idx"]), n_aborted=_ptr(out["n_aborted"]),
+                          reads=_ptr(out["reads"]) if want_reads else None,
+                          outputs_on_device=int(device_out),
+                          stats=ctypes.pointer(st) if st is not None else None)
+        self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))
+        out = dict(out)
+        if not device_out:
+            na = int(out["n_aborted"][0])
+            out["abort_idx"] = out["abort_idx"][:na]
+            out["reads"] = out["reads"][:n_reads] if want_reads else None
+        if st is not None:
+            out["stats"] = st.as_dict()
+        return out
+
+    def run_ops(self, batch, stream=None, want_reads=True, device_out=None, stats=False, out=None):
+        """batch: dict(tid u64[n], op_begin u32[n+1], ops OP_DTYPE/uint8[n_ops*16], args i64[n_ops])."""
+        tid, ob, ops, args = batch["tid"], batch["op_begin"], batch["ops"], batch["args"]
+        n = len(tid)
+        n_ops = len(args)
+        on_dev = _on_device(tid)
+        if device_out is None:
+            device_out = on_dev
+        bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_OPS, n_ops=n_ops, op_begin=_ptr(ob),
+                        ops=_ptr(ops), op_arg=_ptr(args), inputs_on_device=int(on_dev),
+                        stream=c_vp(stream) if stream else None)
+        return self._run(bt, n, n_ops, want_reads, device_out, stats, out)
+
+    def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None):
+        """batch: dict(tid u64[n], type u8[n], params u8[n,128])."""
+        tid, ty, params = batch["tid"], batch["type"], batch["params"]
+        n = len(tid)
+        on_dev = _on_device(tid)
+        if device_out is None:
+            device_out = on_dev
+        bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
+                        proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
+                        stream=c_vp(stream) if stream else None)
+        out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out)
+        if not device_out and want_reads:
+            out["reads"] = out["reads"].reshape(n, 4)
+        return out
+
+    def dump_table(self, t):
+        nr = c_u64(0)
+        self._check(ltpg_dump_table(self.h, t, ctypes.byref(nr), None, None))
+        n = nr.value
+        nc = self.n_cols[t]
+        keys = np.zeros(max(n, 1), np.uint64)
+        cols = np.zeros((nc, max(n, 1)), np.int64) if n else np.zeros((nc, 0), np.int64)
+        colbuf = np.zeros(max(nc * n, 1), np.int64)
+        self._check(ltpg_dump_table(self.h, t, ctypes.byref(nr), _ptr(keys), _ptr(colbuf)))
+        cols = colbuf[:nc * n].reshape(nc, n)
+        return (keys[:n] if self.has_pk[t] else None), cols
+
+
+def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0):
+    db = Database(1, max_txns, max_ops, device=device, flags=flags)
+    g, a, ng, pk = workload.table_desc()
+    keys, cols = workload.initial_table()
+    db.load_table(0, g, a, ng, keys, cols, capacity=capacity or len(keys), has_pk=pk)
+    return db
+
+
+def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None):
+    """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns."""
+    from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
+    db = Database(9, max_txns, 0, device=device, flags=flags, n_warehouses=workload.W)
+    tables = tables if tables is not None else workload.initial_tables()
+    extra = {T_ORDER: 1, T_NEW_ORDER: 1, T_ORDER_LINE: 15, T_HISTORY: 1}
+    for t, (g, a, ng, pk) in workload.table_descs().items():
+        k, c = tables[t]
+        n = c.shape[1]
+        cap = n + extra.get(t, 0) * max_txns * append_batches
+        if capacity and t in capacity:
+            cap = capacity[t]
+        db.load_table(t, g, a, ng, k, c, capacity=max(cap, 1), has_pk=pk,
+                      owner_rule=0)
+    return db

@@ -1,0 +1,201 @@
+// Shared kernels: deterministic exclusive scan, result finalisation (commit
+// bitmask via __ballot_sync, abort-list compaction), index build, capacity and
+// append-cursor bookkeeping.
+#include "ltpg_internal.cuh"
+
+namespace ltpg {
+
+constexpr int SCAN_THREADS = 256;
+constexpr int SCAN_ITEMS = 16;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;  // 4096 elements per block
+
+// Block-wide exclusive scan of one value per thread; returns the block total.
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t& total) {
+  __shared__ uint32_t warp_tot[SCAN_THREADS / 32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_tot[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t t = lane < SCAN_THREADS / 32 ? warp_tot[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, t, o);
+      if (lane >= o) t += y;
+    }
+    if (lane < SCAN_THREADS / 32) warp_tot[lane] = t;  // inclusive
+  }
+  __syncthreads();
+  total = warp_tot[SCAN_THREADS / 32 - 1];
+  uint32_t base = wid ? warp_tot[wid - 1] : 0;
+  __syncthreads();
+  return base + x - v;
+}
+
+__global__ void k_scan_reduce(const uint32_t* __restrict__ in, uint32_t n, uint32_t* __restrict__ sums) {
+  const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE;
+  uint32_t s = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_ITEMS; ++k) {
+    uint64_t i = base + (uint64_t)k * SCAN_THREADS + threadIdx.x;
+    if (i < n) s += in[i];
+  }
+  uint32_t tot;
+  block_excl_scan(s, tot);
+  if (threadIdx.x == 0) sums[blockIdx.x] = tot;
+}
+
+// single block: exclusive scan of the block sums (nb <= SCAN_TILE); sums[nb] = total
+__global__ void k_scan_top(uint32_t* sums, uint32_t nb) {
+  uint32_t v[SCAN_ITEMS];
+  uint32_t s = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_ITEMS; ++k) {
+    uint32_t i = threadIdx.x * SCAN_ITEMS + k;
+    v[k] = i < nb ? sums[i] : 0;
+    s += v[k];
+  }
+  uint32_t tot;
+  uint32_t off = block_excl_scan(s, tot);
+#pragma unroll
+  for (int k = 0; k < SCAN_ITEMS; ++k) {
+    uint32_t i = threadIdx.x * SCAN_ITEMS + k;
+    if (i < nb) sums[i] = off;
+    off += v[k];
+  }
+  if (threadIdx.x == 0) sums[nb] = tot;
+}
+
+__global__ void k_scan_down(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t n,
+                            const uint32_t* __restrict__ sums, uint32_t nb) {
+  // each thread owns SCAN_ITEMS consecutive elements of the tile (stable order)
+  const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE + (uint64_t)threadIdx.x * SCAN_ITEMS;
+  uint32_t v[SCAN_ITEMS];
+  uint32_t s = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_ITEMS; ++k) {
+    uint64_t i = base + k;
+    v[k] = i < n ? in[i] : 0;
+    s += v[k];
+  }
+  uint32_t tot;
+  uint32_t off = block_excl_scan(s, tot) + sums[blockIdx.x];
+#pragma unroll
+  for (int k = 0; k < SCAN_ITEMS; ++k) {
+    uint64_t i = base + k;
+    if (i < n) out[i] = off;
+    off += v[k];
+  }
+  if (blockIdx.x == nb - 1 && threadIdx.x == 0) out[n] = sums[nb];
+}
+
+size_t scan_scratch_words(uint32_t n) { return (n + SCAN_TILE - 1) / SCAN_TILE + 2; }
+
+// out[0..n) = exclusive prefix sums of in, out[n] = total.  Deterministic.
+void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s) {
+  if (n == 0) {
+    cudaMemsetAsync(out, 0, sizeof(uint32_t), s);
+    return;
+  }
+  uint32_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;  // <= SCAN_TILE blocks (n <= 16.7M)
+  k_scan_reduce<<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch);
+  k_scan_top<<<1, SCAN_THREADS, 0, s>>>(scratch, nb);
+  k_scan_down<<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb);
+}
+
+// Result finalisation: commit bitmask (one __ballot_sync word per warp), conflict
+// flags for the abort list, per-status counts.
+__global__ void k_finalize(const uint8_t* __restrict__ status, uint32_t n, uint32_t* __restrict__ commit_bits,
+                           uint32_t* __restrict__ flags, uint32_t* __restrict__ counts,
+                           const uint32_t* __restrict__ err) {
+  if (*err) return;
+  uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  uint8_t st = r < n ? status[r] : 0xFF;
+  uint32_t bits = __ballot_sync(0xffffffffu, st == LTPG_ST_COMMIT);
+  if ((threadIdx.x & 31) == 0 && r < n) commit_bits[r >> 5] = bits;
+  if (r < n) flags[r] = st == LTPG_ST_CONFLICT;
+  uint32_t nc = __popc(bits);
+  uint32_t na = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_CONFLICT));
+  uint32_t nu = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_USER_ABORT));
+  if ((threadIdx.x & 31) == 0) {
+    if (nc) atomicAdd(counts + 0, nc);
+    if (na) atomicAdd(counts + 1, na);
+    if (nu) atomicAdd(counts + 2, nu);
+  }
+}
+
+void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags, uint32_t* counts,
+                     const uint32_t* err, cudaStream_t s) {
+  if (!n) return;
+  k_finalize<<<(n + 255) / 256, 256, 0, s>>>(status, n, commit_bits, flags, counts, err);
+}
+
+// abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
+__global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ offs, uint32_t n,
+                          uint32_t* __restrict__ out) {
+  uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < n && flags[r]) out[offs[r]] = r;
+}
+
+void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s) {
+  if (!n) return;
+  k_compact<<<(n + 255) / 256, 256, 0, s>>>(flags, offs, n, out);
+}
+
+__global__ void k_build_index(const DevTable* __restrict__ tabs, uint32_t t, uint64_t row0, uint64_t n,
+                              uint32_t* err) {
+  const DevTable& T = tabs[t];
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t row = row0 + i;
+    uint64_t key = T.rowkey[row];
+    if (key == KEY_EMPTY) { atomicOr(err, ERR_EINVAL); continue; }
+    IdxSlot* sl = idx_find_or_insert(T, key);
+    if (!sl) { atomicOr(err, ERR_ECAPACITY); continue; }
+    if (atomicCAS(&sl->row, ROW_NONE, (unsigned)row) != ROW_NONE) atomicOr(err, ERR_EINVAL);  // duplicate key
+  }
+}
+
+void launch_build_index(const DevTable* tabs, uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
+                        cudaStream_t s) {
+  if (!n) return;
+  uint64_t blocks = (n + 255) / 256;
+  if (blocks > 148 * 64) blocks = 148 * 64;
+  k_build_index<<<(unsigned)blocks, 256, 0, s>>>(tabs, t, row0, n, err);
+}
+
+// ECAPACITY before anything mutates: provisional rows are n_rows + [0, total)
+__global__ void k_capacity(const DevTable* __restrict__ tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                           const uint32_t* total, uint32_t* err) {
+  uint32_t m = *ins_tables;
+  uint64_t tot = *total;
+  for (uint32_t t = 0; t < n_tables; ++t)
+    if ((m >> t) & 1u) {
+      const DevTable& T = tabs[t];
+      if (*T.n_rows + tot > T.capacity || *T.n_rows + tot > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
+    }
+}
+
+void launch_capacity_check(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                           const uint32_t* total, uint32_t* err, cudaStream_t s) {
+  k_capacity<<<1, 1, 0, s>>>(tabs, n_tables, ins_tables, total, err);
+}
+
+__global__ void k_advance(const DevTable* __restrict__ tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                          const uint32_t* total, const uint32_t* err) {
+  if (*err) return;
+  uint32_t m = *ins_tables;
+  for (uint32_t t = 0; t < n_tables; ++t)
+    if ((m >> t) & 1u) *tabs[t].n_rows += *total;
+}
+
+void launch_advance_cursor(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                           const uint32_t* total, const uint32_t* err, cudaStream_t s) {
+  k_advance<<<1, 1, 0, s>>>(tabs, n_tables, ins_tables, total, err);
+}
+
+}  // namespace ltpg

@@ -1,0 +1,379 @@
+// OPS-mode kernels (YCSB and generic key/value transactions).
+//
+//  K-group   validate the batch (a1) and decompose it into per-kind op lists so
+//            every execute warp runs one op kind (adaptive warp division)
+//  K-claim   INSERT keys claim their index slot with a provisional row (a3)
+//  K-exec    readMem / recordLS / recordTID: snapshot reads, result
+//            slots, epoch-tagged atomicMin marks per conflict unit (a4, a5)
+//  K-detect  rcheck / wcheck: per-txn OR of the RAW/WAW test (a6)
+//  K-wb      getStatus -> writeMem: committed write sets only (a7)
+#include "ltpg_internal.cuh"
+
+namespace ltpg {
+
+constexpr int OPS_MAX_TXN_OPS = 256;
+
+__device__ __forceinline__ ltpg_op load_op(const ltpg_op* ops, uint32_t i) {
+  const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(ops + i);
+  ltpg_op o;
+  o.key = v.x;
+  o.kind = (uint8_t)(v.y);
+  o.table = (uint8_t)(v.y >> 8);
+  o.col = (uint16_t)(v.y >> 16);
+  o.aux = (uint32_t)(v.y >> 32);
+  return o;
+}
+
+__device__ __forceinline__ bool op_valid(const DevTable* tabs, uint32_t n_tables, const ltpg_op& o) {
+  if (o.table >= n_tables) return false;
+  const DevTable& T = tabs[o.table];
+  if (!T.defined || !T.has_pk || o.kind > LTPG_SCAN || o.key == KEY_EMPTY) return false;
+  switch (o.kind) {
+    case LTPG_SELECT: return o.col < T.n_cols;
+    case LTPG_UPDATE: return o.col < T.n_cols && T.group[o.col] != LTPG_STATIC && !T.is_add[o.col];
+    case LTPG_ADD: return o.col < T.n_cols && T.is_add[o.col];
+    case LTPG_INSERT: return T.n_groups > 0;
+    case LTPG_DELETE: return T.n_groups > 0 && !T.has_static;
+    default:  // SCAN
+      if (o.col != LTPG_COL_COUNT && o.col >= T.n_cols) return false;
+      return o.aux == 0 || o.key <= KEY_EMPTY - o.aux;
+  }
+}
+
+__device__ __forceinline__ bool is_write_kind(uint8_t k) {
+  return k == LTPG_UPDATE || k == LTPG_ADD || k == LTPG_INSERT || k == LTPG_DELETE;
+}
+
+// ---- K-group: validation + decomposition into per-kind lists (one thread per txn) ----
+template <bool GROUPED>
+__global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __restrict__ tabs, uint32_t n_tables,
+                                                            BatchDev b) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31;
+  bool bad = false;
+  uint32_t b0 = 0, b1 = 0, cnt[NKINDS] = {0, 0, 0, 0, 0, 0};
+  uint32_t my_ins_tables = 0;
+  if (r < b.n_txns) {
+    if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
+    b0 = b.op_begin[r];
+    b1 = b.op_begin[r + 1];
+    if (r == 0 && b0 != 0) bad = true;
+    if (r == b.n_txns - 1 && b1 != b.n_ops) bad = true;
+    if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS) { bad = true; b1 = b0; }
+    for (uint32_t i = b0; i < b1; ++i) {
+      ltpg_op o = load_op(b.ops, i);
+      if (!op_valid(tabs, n_tables, o)) { bad = true; continue; }
+      cnt[o.kind]++;
+      if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
+    }
+    // R10: a written key is touched by no other op of the txn (no read-your-writes)
+    for (uint32_t i = b0 + 1; i < b1 && !bad; ++i) {
+      ltpg_op a = load_op(b.ops, i);
+      uint64_t alo = a.key, ahi = a.kind == LTPG_SCAN ? a.key + a.aux : a.key + 1;
+      for (uint32_t j = b0; j < i; ++j) {
+        ltpg_op c = load_op(b.ops, j);
+        if (c.table != a.table) continue;
+        uint64_t clo = c.key, chi = c.kind == LTPG_SCAN ? c.key + c.aux : c.key + 1;
+        if (!(alo < chi && clo < ahi)) continue;
+        if (is_write_kind(a.kind) || is_write_kind(c.kind) || (a.kind != LTPG_SCAN && c.kind != LTPG_SCAN)) {
+          bad = true;
+          break;
+        }
+      }
+    }
+    b.txn_ins[r] = cnt[LTPG_INSERT];
+    if (bad) atomicOr(b.err, ERR_EINVAL);
+  }
+  my_ins_tables = __reduce_or_sync(0xffffffffu, my_ins_tables);
+  if (lane == 0 && my_ins_tables) atomicOr(b.ins_tables, my_ins_tables);
+  if (!GROUPED) {
+    // one flat list in op order (region 0); INSERTs are still listed for K-claim
+    if (r < b.n_txns)
+      for (uint32_t i = b0; i < b1; ++i) b.items[i] = (unsigned long long)i | ((unsigned long long)r << 32);
+    if (r == 0) b.kcount[0] = b.n_ops;
+    if (r < b.n_txns && !bad)
+      for (uint32_t i = b0; i < b1; ++i)
+        if (b.ops[i].kind == LTPG_INSERT) {
+          uint32_t p = atomicAdd(b.kcount + LTPG_INSERT, 1u);
+          b.items[(uint64_t)LTPG_INSERT * b.max_ops + p] = (unsigned long long)i | ((unsigned long long)r << 32);
+        }
+    return;
+  }
+  // warp-aggregated append into the per-kind lists: one atomicAdd per warp and kind
+  uint32_t pos[NKINDS];
+#pragma unroll
+  for (int k = 0; k < NKINDS; ++k) {
+    uint32_t x = cnt[k];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
+    uint32_t base = 0;
+    if (lane == 31 && tot) base = atomicAdd(b.kcount + k, tot);
+    base = __shfl_sync(0xffffffffu, base, 31);
+    pos[k] = base + x - cnt[k];
+  }
+  if (r < b.n_txns && !bad)
+    for (uint32_t i = b0; i < b1; ++i) {
+      uint8_t k = b.ops[i].kind;
+      uint32_t p = 0;
+#pragma unroll
+      for (int kk = 0; kk < NKINDS; ++kk)
+        if (kk == k) p = pos[kk]++;
+      b.items[(uint64_t)k * b.max_ops + p] = (unsigned long long)i | ((unsigned long long)r << 32);
+    }
+}
+
+void launch_ops_validate_group(const DevTable* tabs, uint32_t n_tables, const BatchDev& b, bool grouped,
+                               cudaStream_t s) {
+  uint32_t blocks = (b.n_txns + 255) / 256;
+  if (grouped)
+    k_ops_validate_group<true><<<blocks, 256, 0, s>>>(tabs, n_tables, b);
+  else
+    k_ops_validate_group<false><<<blocks, 256, 0, s>>>(tabs, n_tables, b);
+}
+
+// ---- K-claim: INSERT keys claim their slot; provisional row = n_rows + rank of the
+//      insert in (rank, op) order; atomicMin makes the earliest inserter own the unit ----
+__global__ void __launch_bounds__(256) k_ops_claim(const DevTable* __restrict__ tabs, BatchDev b) {
+  if (*b.err) return;
+  const uint32_t n = b.kcount[LTPG_INSERT];
+  const unsigned long long* list = b.items + (uint64_t)LTPG_INSERT * b.max_ops;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    unsigned long long it = list[i];
+    uint32_t oi = (uint32_t)it, r = (uint32_t)(it >> 32);
+    ltpg_op o = load_op(b.ops, oi);
+    const DevTable& T = tabs[o.table];
+    uint32_t j = 0;
+    for (uint32_t q = b.op_begin[r]; q < oi; ++q) j += b.ops[q].kind == LTPG_INSERT;
+    uint32_t prov = (uint32_t)(*T.n_rows + b.txn_ins[r] + j);
+    IdxSlot* sl = idx_find_or_insert(T, o.key);
+    if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
+    if (*reinterpret_cast<volatile unsigned*>(&sl->row) != ROW_NONE) continue;  // present in S
+    atomicMin(&sl->claim, prov);
+  }
+}
+
+void launch_ops_claim(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
+  k_ops_claim<<<148 * 4, 256, 0, s>>>(tabs, b);
+}
+
+// ---- K-exec ---------------------------------------------------------------------------
+__device__ __forceinline__ void exec_one(const DevTable* __restrict__ tabs, const BatchDev& b, uint32_t oi,
+                                         uint32_t r, const ltpg_op& o, bool filter) {
+  const DevTable& T = tabs[o.table];
+  const unsigned long long tag = epoch_tag(b.epoch) | r;
+  uint32_t row, claim;
+  long long res = LTPG_NOT_FOUND;
+  uint64_t uref = 0;
+  if (o.kind == LTPG_SCAN) {  // range of predefined keys; checked again in detect
+    long long cnt = 0;
+    unsigned long long sum = 0;
+    for (uint64_t k = o.key; k < o.key + o.aux; ++k) {
+      idx_find(T, k, row, claim);
+      if (row != ROW_NONE) {
+        ++cnt;
+        if (o.col != LTPG_COL_COUNT) sum += (unsigned long long)*col_ptr(T, o.col, row);
+      }
+    }
+    b.res[oi] = o.col == LTPG_COL_COUNT ? cnt : (long long)sum;
+    b.uref[oi] = make_uref(CHK_SCAN, false, false, o.table, 0, 0);
+    return;
+  }
+  idx_find(T, o.key, row, claim);
+  const bool present = row != ROW_NONE;
+  if (!present && o.kind != LTPG_INSERT) {
+    // absent key: a READ of its existence; only an inserter of this batch can conflict
+    uref = claim != ROW_NONE ? make_uref(CHK_RW, false, false, o.table, 0, claim)
+                             : make_uref(CHK_NONE, false, false, o.table, 0, 0);
+    b.res[oi] = LTPG_NOT_FOUND;
+    b.uref[oi] = uref;
+    return;
+  }
+  switch (o.kind) {
+    case LTPG_SELECT: {
+      res = *col_ptr(T, o.col, row);
+      uint32_t g = T.group[o.col];
+      uref = g == LTPG_STATIC ? make_uref(CHK_NONE, false, true, o.table, 0, row)
+                              : make_uref(CHK_RW, false, true, o.table, g, row);
+      break;
+    }
+    case LTPG_UPDATE: {
+      uint32_t g = T.group[o.col];
+      res = *col_ptr(T, o.col, row);  // pre-image; new value = res + arg at write-back
+      mark_min(mark_ptr(T, g, row), tag, filter);
+      uref = make_uref(CHK_RW, false, true, o.table, g, row);
+      break;
+    }
+    case LTPG_ADD: {
+      uint32_t g = T.group[o.col];
+      res = 0;
+      mark_min(mark_ptr(T, g, row) + 1, tag, filter);
+      uref = make_uref(CHK_A, false, true, o.table, g, row);
+      break;
+    }
+    case LTPG_INSERT:
+      if (present) {  // duplicate key: user abort; a READ of the row
+        res = 0;
+        b.ua[r] = 1;
+        uref = make_uref(CHK_RW, false, true, o.table, 0, row);
+      } else {
+        if (claim == ROW_NONE) {  // every absent INSERT key was claimed by K-claim
+          atomicOr(b.err, ERR_EINTERNAL);
+          return;
+        }
+        res = 1;
+        for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(mark_ptr(T, g, claim), tag, filter);
+        uref = make_uref(CHK_RW, true, false, o.table, 0, claim);
+      }
+      break;
+    case LTPG_DELETE:
+      res = 1;
+      for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(mark_ptr(T, g, row), tag, filter);
+      uref = make_uref(CHK_RW, true, true, o.table, 0, row);
+      break;
+  }
+  b.res[oi] = res;
+  b.uref[oi] = uref;
+}
+
+template <bool GROUPED>
+__global__ void __launch_bounds__(256) k_ops_exec(const DevTable* __restrict__ tabs, BatchDev b, bool filter) {
+  if (*b.err) return;
+  const int lane = threadIdx.x & 31;
+  uint32_t cnt[NKINDS], pref[NKINDS + 1];
+  pref[0] = 0;
+#pragma unroll
+  for (int k = 0; k < NKINDS; ++k) {
+    cnt[k] = GROUPED ? b.kcount[k] : (k == 0 ? b.n_ops : 0);
+    pref[k + 1] = pref[k] + ((cnt[k] + 31) & ~31u);  // each kind padded to whole warps
+  }
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); (uint64_t)w * 32 < pref[NKINDS];
+       w += nwarps) {
+    const uint32_t p = w * 32;
+    int k = 0;
+#pragma unroll
+    for (int kk = 1; kk < NKINDS; ++kk)
+      if (p >= pref[kk]) k = kk;  // warp-uniform op kind
+    const uint32_t idx = p - pref[k] + lane;
+    if (idx >= cnt[k]) continue;
+    const unsigned long long it = b.items[(uint64_t)k * b.max_ops + idx];
+    const uint32_t oi = (uint32_t)it, r = (uint32_t)(it >> 32);
+    const ltpg_op o = load_op(b.ops, oi);
+    exec_one(tabs, b, oi, r, o, filter);
+  }
+}
+
+void launch_ops_exec(const DevTable* tabs, const BatchDev& b, bool grouped, bool filter, cudaStream_t s) {
+  uint64_t warps = (b.n_ops + NKINDS * 32 + 31) / 32;
+  uint64_t blocks = (warps + 7) / 8;
+  if (blocks > 148 * 16) blocks = 148 * 16;
+  if (!blocks) return;
+  if (grouped)
+    k_ops_exec<true><<<(unsigned)blocks, 256, 0, s>>>(tabs, b, filter);
+  else
+    k_ops_exec<false><<<(unsigned)blocks, 256, 0, s>>>(tabs, b, filter);
+}
+
+// ---- K-detect: per txn, OR of the unit tests over its ops ------------------------------
+__global__ void __launch_bounds__(256) k_ops_detect(const DevTable* __restrict__ tabs, BatchDev b) {
+  if (*b.err) return;
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= b.n_txns) return;
+  const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
+  bool bad = false;
+  for (uint32_t i = b0; i < b1 && !bad; ++i) {
+    const uint64_t u = b.uref[i];
+    const uint64_t chk = u >> 62;
+    if (chk == CHK_NONE) continue;
+    const DevTable& T = tabs[(u >> 40) & 0xFF];
+    if (chk == CHK_SCAN) {  // phantom-safe: every key of the range is a read (R8)
+      const ltpg_op o = load_op(b.ops, i);
+      if (!T.n_groups) continue;
+      for (uint64_t k = o.key; k < o.key + o.aux && !bad; ++k) {
+        uint32_t row, claim;
+        idx_find(T, k, row, claim);
+        if (row != ROW_NONE) {
+          uint32_t g = (o.col != LTPG_COL_COUNT && T.group[o.col] != LTPG_STATIC) ? T.group[o.col] : 0;
+          bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);
+        } else if (claim != ROW_NONE) {
+          bad = unit_conflicts(T, 0, claim, CHK_RW, r, b.epoch);
+        }
+      }
+      continue;
+    }
+    const uint32_t row = (uint32_t)u;
+    if ((u >> 61) & 1) {
+      for (uint32_t g = 0; g < T.n_groups && !bad; ++g) bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);
+    } else {
+      bad = unit_conflicts(T, (u >> 32) & 0xFF, row, chk, r, b.epoch);
+    }
+  }
+  b.status[r] = bad ? LTPG_ST_CONFLICT : (b.ua[r] ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+}
+
+void launch_ops_detect(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
+  k_ops_detect<<<(b.n_txns + 255) / 256, 256, 0, s>>>(tabs, b);
+}
+
+// ---- K-wb: apply committed write sets; every INSERT releases its claim ----------------
+__global__ void __launch_bounds__(256) k_ops_writeback(const DevTable* __restrict__ tabs, BatchDev b) {
+  if (*b.err) return;
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= b.n_txns) return;
+  const bool commit = b.status[r] == LTPG_ST_COMMIT;
+  const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
+  for (uint32_t i = b0; i < b1; ++i) {
+    const uint64_t u = b.uref[i];
+    const uint32_t kind = b.ops[i].kind;
+    if (!commit && kind != LTPG_INSERT) continue;
+    if ((u >> 62) == CHK_NONE || (u >> 62) == CHK_SCAN) continue;
+    const bool present = (u >> 60) & 1;
+    const uint32_t row = (uint32_t)u;
+    if (kind == LTPG_INSERT) {
+      if (present) continue;  // duplicate-key user abort: nothing claimed
+      const ltpg_op o = load_op(b.ops, i);
+      const DevTable& T = tabs[o.table];
+      IdxSlot* sl = idx_slot(T, o.key);
+      if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
+      if (commit) {
+        const long long arg = b.args[i];
+        for (uint32_t c = 0; c < T.n_cols; ++c)
+          *col_ptr(T, c, row) = (long long)((unsigned long long)arg + c);
+        T.rowkey[row] = o.key;
+        T.valid[row] = 1;
+        sl->row = row;
+      }
+      sl->claim = ROW_NONE;
+      continue;
+    }
+    if (!present) continue;
+    const ltpg_op o = load_op(b.ops, i);
+    const DevTable& T = tabs[o.table];
+    switch (kind) {
+      case LTPG_UPDATE:
+        *col_ptr(T, o.col, row) = (long long)((unsigned long long)b.res[i] + (unsigned long long)b.args[i]);
+        break;
+      case LTPG_ADD:  // delayed update: commutative, order-free and exact
+        atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr(T, o.col, row)), (unsigned long long)b.args[i]);
+        break;
+      case LTPG_DELETE: {
+        T.valid[row] = 0;
+        IdxSlot* sl = idx_slot(T, o.key);
+        if (sl) sl->row = ROW_NONE;
+        break;
+      }
+      default:
+        break;
+    }
+  }
+}
+
+void launch_ops_writeback(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
+  k_ops_writeback<<<(b.n_txns + 255) / 256, 256, 0, s>>>(tabs, b);
+}
+
+}  // namespace ltpg

@@ -1,0 +1,195 @@
+// Internal device-side definitions of the B200 LTPG pipeline (not part of the ABI).
+//
+// HBM layout (DESIGN.md §"Data layout"):
+//   * columns: int64, one array per column (SoA), `capacity` rows incl. the
+//     append region; hidden `valid` byte and `rowkey` u64 per row;
+//   * PK hash index: open addressing, linear probing, 16-byte slots
+//     {u64 key, u32 row, u32 claim}, power-of-two size >= 2x capacity,
+//     Fibonacci hashing (R6: the bucket function is result-invisible);
+//   * conflict marks ("conflict log"): per (group,row) one 16-byte
+//     record {u64 minW, u64 minA}; each u64 is epoch-tagged
+//     ((0xFFFFFFFF - epoch) << 32 | rank) so a new batch never needs a reset
+//     pass: u64 atomicMin keeps the newest epoch and, within it, the smallest
+//     rank -- the per-unit minimum TID of P:219/P:225.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/ltpg.h"
+
+namespace ltpg {
+
+constexpr int MAXC = 16;
+constexpr int MAXT = 16;
+constexpr uint64_t KEY_EMPTY = ~0ull;
+constexpr uint32_t ROW_NONE = 0xFFFFFFFFu;
+constexpr int NKINDS = 6;
+
+// device error word bits
+constexpr uint32_t ERR_EINVAL = 1u, ERR_ECAPACITY = 2u, ERR_EINTERNAL = 4u;
+
+// check kinds stored in uref bits 62..63 (and bit 61 = "all groups")
+constexpr uint64_t CHK_NONE = 0, CHK_RW = 1, CHK_A = 2, CHK_SCAN = 3;
+
+struct alignas(16) IdxSlot {
+  unsigned long long key;
+  unsigned int row;
+  unsigned int claim;
+};
+
+struct DevTable {
+  long long* col[MAXC];
+  uint32_t stride[MAXC];          // in int64 elements between consecutive rows
+  uint8_t group[MAXC];
+  uint8_t is_add[MAXC];
+  uint32_t n_cols, n_groups;
+  uint32_t has_pk, has_static, defined, owner_rule;
+  uint64_t capacity;
+  uint8_t* valid;
+  unsigned long long* rowkey;
+  unsigned long long* marks;      // [n_groups][capacity] x {minW, minA}
+  IdxSlot* idx;
+  uint64_t idx_mask;
+  uint32_t idx_shift;
+  unsigned long long* n_rows;     // device append cursor
+};
+
+__host__ __device__ inline uint64_t idx_hash(uint64_t key, uint32_t shift) {
+  return (key * 0x9E3779B97F4A7C15ull) >> shift;
+}
+
+__device__ __forceinline__ unsigned long long epoch_tag(uint32_t epoch) {
+  return (unsigned long long)(0xFFFFFFFFu - epoch) << 32;
+}
+
+// Minimum rank recorded for this epoch, or UINT32_MAX.
+__device__ __forceinline__ uint32_t mark_rank(unsigned long long v, uint32_t epoch) {
+  return (uint32_t)(v >> 32) == 0xFFFFFFFFu - epoch ? (uint32_t)v : 0xFFFFFFFFu;
+}
+
+// recordTID: atomicMin of this txn's rank into a mark word.  The
+// plain pre-read skips the atomic when a smaller (or equal) rank is already
+// there -- marks only decrease, so a stale read can only cause a redundant
+// atomic, never a missing one (result-identical).
+__device__ __forceinline__ void mark_min(unsigned long long* p, unsigned long long v, bool filter) {
+  if (filter) {
+    unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(p);
+    if (cur <= v) return;
+  }
+  atomicMin(p, v);
+}
+
+__device__ __forceinline__ unsigned long long* mark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
+  return T.marks + 2ull * ((uint64_t)g * T.capacity + row);
+}
+
+__device__ __forceinline__ long long* col_ptr(const DevTable& T, uint32_t c, uint32_t row) {
+  return T.col[c] + (uint64_t)row * T.stride[c];
+}
+
+// Snapshot lookup: returns true if the key has a slot; row = ROW_NONE if absent
+// in the snapshot (deleted / never inserted), claim = ROW_NONE unless an INSERT of
+// this batch claimed it.
+__device__ __forceinline__ bool idx_find(const DevTable& T, uint64_t key, uint32_t& row, uint32_t& claim) {
+  uint64_t h = idx_hash(key, T.idx_shift);
+  for (uint64_t probes = 0; probes <= T.idx_mask; ++probes) {
+    const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(T.idx + h);
+    if (v.x == key) {
+      row = (uint32_t)v.y;
+      claim = (uint32_t)(v.y >> 32);
+      return true;
+    }
+    if (v.x == KEY_EMPTY) break;
+    h = (h + 1) & T.idx_mask;
+  }
+  row = ROW_NONE;
+  claim = ROW_NONE;
+  return false;
+}
+
+// Find or create the slot of `key` (load / claim paths).
+__device__ __forceinline__ IdxSlot* idx_find_or_insert(const DevTable& T, uint64_t key) {
+  uint64_t h = idx_hash(key, T.idx_shift);
+  for (uint64_t probes = 0; probes <= T.idx_mask; ++probes) {
+    IdxSlot* s = T.idx + h;
+    unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&s->key);
+    if (k == KEY_EMPTY) k = atomicCAS(&s->key, KEY_EMPTY, key);
+    if (k == KEY_EMPTY || k == key) return s;
+    h = (h + 1) & T.idx_mask;
+  }
+  return nullptr;
+}
+
+__device__ __forceinline__ IdxSlot* idx_slot(const DevTable& T, uint64_t key) {
+  uint64_t h = idx_hash(key, T.idx_shift);
+  for (uint64_t probes = 0; probes <= T.idx_mask; ++probes) {
+    IdxSlot* s = T.idx + h;
+    unsigned long long k = s->key;
+    if (k == key) return s;
+    if (k == KEY_EMPTY) return nullptr;
+    h = (h + 1) & T.idx_mask;
+  }
+  return nullptr;
+}
+
+// uref: per-op record written by execute, read by detect / write-back.
+//   bits  0..31 row (or claim row)   bits 32..39 group   bits 40..47 table
+//   bit   60    present in snapshot  bit 61 all groups    bits 62..63 check kind
+__host__ __device__ __forceinline__ uint64_t make_uref(uint64_t chk, bool all, bool present, uint32_t t,
+                                                       uint32_t g, uint32_t row) {
+  return (chk << 62) | ((uint64_t)all << 61) | ((uint64_t)present << 60) | ((uint64_t)t << 40) |
+         ((uint64_t)g << 32) | row;
+}
+
+// Commit test of one unit for rank r (rcheck / wcheck; R1, R7).
+__device__ __forceinline__ bool unit_conflicts(const DevTable& T, uint32_t g, uint32_t row, uint64_t chk,
+                                               uint32_t r, uint32_t epoch) {
+  const ulonglong2 m = *reinterpret_cast<const ulonglong2*>(mark_ptr(T, g, row));
+  uint32_t w = mark_rank(m.x, epoch);
+  if (chk == CHK_A) return w < r;
+  uint32_t a = mark_rank(m.y, epoch);
+  return (w < a ? w : a) < r;
+}
+
+// ---- host-side launchers (defined in the .cu files) ----------------------------------
+struct BatchDev {
+  uint32_t n_txns, n_ops, epoch, flags;
+  int64_t clock;
+  const unsigned long long* tid;
+  const uint32_t* op_begin;
+  const ltpg_op* ops;
+  const long long* args;
+  const uint8_t* ptype;
+  const uint8_t* params;
+  long long* res;            // OPS: [n_ops]   TPCC: [4 n]
+  unsigned long long* uref;  // OPS: [n_ops]
+  unsigned long long* items; // [NKINDS][max_ops]  (op idx | txn << 32)
+  uint32_t* kcount;          // [NKINDS]
+  uint32_t* txn_ins;         // [n_txns + 1] per-txn insert count -> exclusive offsets
+  uint8_t* ua;               // [n_txns] user-abort flags
+  uint8_t* status;           // [n_txns]
+  uint32_t* err;             // device error word
+  uint32_t* ins_tables;      // bitmask of tables receiving inserts
+  uint32_t max_ops;
+};
+
+void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
+size_t scan_scratch_words(uint32_t n);
+
+void launch_ops_validate_group(const DevTable* tabs, uint32_t n_tables, const BatchDev& b, bool grouped,
+                               cudaStream_t s);
+void launch_ops_claim(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
+void launch_ops_exec(const DevTable* tabs, const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
+void launch_ops_detect(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
+void launch_ops_writeback(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
+void launch_capacity_check(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                           const uint32_t* total, uint32_t* err, cudaStream_t s);
+void launch_advance_cursor(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+                           const uint32_t* total, const uint32_t* err, cudaStream_t s);
+void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
+                     uint32_t* counts, const uint32_t* err, cudaStream_t s);
+void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);
+void launch_build_index(const DevTable* tabs, uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
+                        cudaStream_t s);
+
+}  // namespace ltpg
