@@ -1,0 +1,426 @@
+#!/usr/bin/env python
+"""bench.py -- LTPG per-batch DOCC pipeline on B200 (one JSON line on rank 0).
+
+A "step" is one batch through the whole hot path:
+validate + warp division -> claim -> execute + marks -> conflict detection ->
+write-back -> commit bitmask / abort list.  Workloads are BASELINE.json configs
+(synthetic, seeded).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl ours|reference]
+
+value      committed txns/s, inputs resident in HBM (CUDA events per step, L2
+           flushed between steps outside the timed events), max over ranks
+e2e        same metric through the public API with pinned HOST inputs/outputs
+           (H2D + kernels + D2H inside each timed step)
+roofline   dominant kernel: algorithmic bytes / its CUDA-event duration vs the
+           measured HBM copy peak (MEASURED_PEAKS.json)
+cpu_baseline  the CPU oracle (oracle/) as it stands, 1 thread, on a bounded sample
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "committed txns/sec"
+UNIT = "txn/s"
+
+WORKLOADS = {
+    # BASELINE.json configs[i]; seed = 0x17C0 + i
+    "ycsb_c1": dict(kind="ycsb", cfg=0, n_rows=10_000, theta=0.5, ops=4, batch=1024),
+    "tpcc_c2": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="strict"),
+    "ycsb_c3": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=10, batch=1 << 20),
+    "tpcc_c4": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="strict"),
+    "tpcc_c5": dict(kind="tpcc", cfg=4, W=512, mix="no_pay", batch=1 << 20, mode="strict"),
+}
+DEFAULT_WORKLOAD = "ycsb_c3"
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ---- clocks sampler (B200_PROFILING.md "clocks DURING the timed region") ------------------
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.lines = []
+        self.stop = threading.Event()
+
+    def __enter__(self):
+        self.t = threading.Thread(target=self._loop, daemon=True)
+        self.t.start()
+        return self
+
+    def _loop(self):
+        while not self.stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout
+                self.lines += [ln.strip() for ln in out.splitlines() if ln.strip()]
+            except Exception:
+                pass
+            self.stop.wait(0.05)
+
+    def __exit__(self, *a):
+        self.stop.set()
+        self.t.join(timeout=6)
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm),
+                "window": "sampled every ~0.1 s from the first warm-up step to the end of the e2e leg"}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("hbm_gbs", 6469.3), "measured"
+    return 6650.0, "fallback"
+
+
+def ncu_traffic(kernel_substr):
+    """dram read+write bytes per launch of the kernel from the committed `ncu --set full` summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_r01_ycsb_c3.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p))
+        for k, v in d.get("kernels", {}).items():
+            if kernel_substr in k:
+                return v.get("dram_bytes")
+    except Exception:
+        return None
+    return None
+
+
+# ---- workloads ------------------------------------------------------------------------------
+def make_workload(name, rank):
+    w = WORKLOADS[name]
+    seed = 0x17C0 + w["cfg"] + 1000 * rank
+    if w["kind"] == "ycsb":
+        from workloads.ycsb import YcsbWorkload
+        return YcsbWorkload(w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
+    from workloads import tpcc
+    mix = tpcc.MIX_FULL if w["mix"] == "full" else tpcc.MIX_NO_PAY
+    return tpcc.TpccWorkload(w["W"], seed=seed, mode=w["mode"], mix=mix)
+
+
+def exec_algorithmic_bytes(batch):
+    """Algorithmic bytes of the execute kernel for an OPS batch:
+    per op 16 B op record + 32 B index sector + 32 B data sector + 8 B result + 8 B
+    unit reference; per marking op (UPDATE/ADD/INSERT/DELETE) + 64 B (atomic sector RMW)."""
+    kinds = batch["ops"]["kind"]
+    n = len(kinds)
+    marking = int(np.isin(kinds, [1, 2, 3, 4]).sum())
+    return 96 * n + 64 * marking
+
+
+def step_algorithmic_bytes(batch):
+    """Whole-step algorithmic bytes (OPS): exec + detect (8 B uref + 32 B mark sector per op)
+    + group (16 B op + 8 B list entry) + per-txn status/bits/flags (~10 B)."""
+    n = len(batch["ops"])
+    return exec_algorithmic_bytes(batch) + n * (40 + 24) + 10 * len(batch["tid"])
+
+
+# ---- reference arm: the CPU oracle ---------------------------------------------------------------
+def run_reference(args, name):
+    import oracle
+    w = WORKLOADS[name]
+    wl = make_workload(name, 0)
+    t0 = time.time()
+    if w["kind"] == "ycsb":
+        db = oracle.ycsb_db(wl)
+    else:
+        db = oracle.tpcc_db(wl)
+    log("oracle load %.1fs" % (time.time() - t0))
+    sample = min(w["batch"], args.ref_sample)
+    committed, secs = 0, 0.0
+    tid = 1
+    for s in range(args.warmup + args.steps):
+        b = wl.batch(sample, tid, 10_000 + s)
+        tid += sample
+        t = time.perf_counter()
+        if w["kind"] == "ycsb":
+            rc, st, _ = db.run_ops(b)
+        else:
+            rc, st, _ = db.run_tpcc(b, clock=2 + s)
+        dt = time.perf_counter() - t
+        assert rc == 0
+        if s >= args.warmup:
+            committed += int((st == 1).sum())
+            secs += dt
+    v = committed / secs if secs else 0.0
+    desc = "%d-txn batches of %s (full batch %d), %d timed" % (sample, name, w["batch"], args.steps)
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * secs / max(args.steps, 1),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic", "config": config_of(name, sample),
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def config_of(name, batch=None):
+    w = dict(WORKLOADS[name])
+    c = {"workload": name, "baseline_config": w.pop("cfg"), "kind": w.pop("kind")}
+    c.update(w)
+    if batch is not None:
+        c["batch"] = batch
+    c["l2"] = "inputs+state larger than L2 (126 MB) and L2 flushed (256 MB write) between timed steps"
+    return c
+
+
+def cpu_baseline(name, batch_host, wl):
+    """The oracle as it stands, 1 thread, on a bounded sample of the same workload."""
+    import oracle
+    w = WORKLOADS[name]
+    t0 = time.time()
+    db = oracle.ycsb_db(wl) if w["kind"] == "ycsb" else oracle.tpcc_db(wl)
+    load_s = time.time() - t0
+    n = len(batch_host["tid"])
+    budget = 25.0
+    t = time.perf_counter()
+    if w["kind"] == "ycsb":
+        rc, st, _ = db.run_ops(batch_host)
+    else:
+        rc, st, _ = db.run_tpcc(batch_host, clock=2)
+    dt = time.perf_counter() - t
+    del db
+    return {"value": float((st == 1).sum()) / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": "one full %d-txn batch of %s (oracle load %.1fs not timed; %.1fs of batch work)"
+                      % (n, name, load_s, dt), "seconds": dt, "budget_s": budget}
+
+
+# ---- our arm -----------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default=os.environ.get("LTPG_BENCH_WORKLOAD", DEFAULT_WORKLOAD),
+                    choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-sample", type=int, default=1 << 17)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--flags", type=int, default=0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    name = args.workload
+
+    if args.impl == "reference":
+        if rank == 0:
+            run_reference(args, name)
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_icde_wei0l0lzj024_b200 as ltpg
+
+    w = WORKLOADS[name]
+    wl = make_workload(name, rank)
+    B = w["batch"]
+    t0 = time.time()
+    if w["kind"] == "ycsb":
+        db = ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=args.flags)
+    else:
+        db = ltpg.tpcc_database(wl, max_txns=B, append_batches=args.steps + args.warmup + 2, flags=args.flags)
+    log("rank %d: db loaded in %.1fs" % (rank, time.time() - t0))
+
+    # distinct input batches, cycled (inputs only; every step recomputes everything)
+    n_distinct = 2
+    host_batches, dev_batches, pin_batches = [], [], []
+    tid = 1
+    for i in range(n_distinct):
+        b = wl.batch(B, tid, i) if w["kind"] == "ycsb" else wl.batch(B, tid, i)
+        tid += B
+        host_batches.append(b)
+    dev = torch.device("cuda", local)
+
+    def to_t(a, pin):
+        t = torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).copy())
+        return t.pin_memory() if pin else t.to(dev)
+
+    for b in host_batches:
+        dev_batches.append({k: to_t(v, False) for k, v in b.items()})
+        pin_batches.append({k: to_t(v, True) for k, v in b.items()})
+    for db_ in dev_batches:  # keep logical lengths for the binding
+        pass
+
+    def run(bd, bh, clock, device, stats):
+        inputs = bd if device else bp_of(bh)
+        if w["kind"] == "ycsb":
+            return db.run_ops(inputs, stream=torch.cuda.current_stream().cuda_stream, want_reads=True,
+                              device_out=device, stats=stats, n_txns=len(bh["tid"]), n_ops=len(bh["args"]))
+        return db.run_tpcc(inputs, clock, stream=torch.cuda.current_stream().cuda_stream, want_reads=True,
+                           device_out=device, stats=stats, n_txns=len(bh["tid"]))
+
+    pin_of = {id(h): p for h, p in zip(host_batches, pin_batches)}
+
+    def bp_of(bh):
+        return pin_of[id(bh)]
+
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    clock = 2
+    clk = ClockSampler(local).__enter__()  # samples through warm-up, timed and e2e legs
+    for s in range(args.warmup):
+        i = s % n_distinct
+        run(dev_batches[i], host_batches[i], clock, True, False)
+        clock += 1
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+
+    # ---- timed: device-resident inputs ------------------------------------------------------
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    commits, procs, exec_ms, kernels, stage = [], [], [], 0, []
+    torch.cuda.synchronize()
+    for s in range(args.steps):
+        i = (args.warmup + s) % n_distinct
+        flush.fill_(s & 0xFF)  # evict L2 between steps (outside the timed events)
+        ev[s][0].record(stream)
+        out = run(dev_batches[i], host_batches[i], clock, True, True)
+        ev[s][1].record(stream)
+        clock += 1
+        st = out["stats"]
+        commits.append(st["n_commit"])
+        procs.append(len(host_batches[i]["tid"]))
+        exec_ms.append(st["ms_exec"])
+        kernels += st["n_kernels"]
+        stage.append(st)
+    torch.cuda.synchronize()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    total_s = sum(step_ms) / 1000.0
+    if dist:
+        t = torch.tensor([total_s], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_s = float(t.item())
+        c = torch.tensor([float(sum(commits)), float(sum(procs))], device=dev, dtype=torch.float64)
+        dist.all_reduce(c)
+        all_commits, all_procs = c[0].item(), c[1].item()
+    else:
+        all_commits, all_procs = float(sum(commits)), float(sum(procs))
+    value = all_commits / total_s
+
+    # ---- timed: end to end through the public API, pinned host buffers ------------------------
+    e2e = None
+    if not args.no_e2e:
+        e_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                for _ in range(args.steps)]
+        e_commits = []
+        h2d = d2h = 0
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        for s in range(args.steps):
+            i = (args.warmup + s) % n_distinct
+            bh = host_batches[i]
+            flush.fill_(s & 0xFF)
+            e_ev[s][0].record(stream)
+            out = run(None, bh, clock, False, False)
+            e_ev[s][1].record(stream)
+            clock += 1
+            e_commits.append(int((out["status"] == 1).sum()))
+            h2d += sum(v.nbytes for v in bh.values())
+            n = len(bh["tid"])
+            nreads = len(bh["args"]) if w["kind"] == "ycsb" else 4 * n
+            d2h += n + 4 * ((n + 31) // 32) + 4 * len(out["abort_idx"]) + 8 * nreads + 68
+        torch.cuda.synchronize()
+        e_s = sum(a.elapsed_time(b) for a, b in e_ev) / 1000.0
+        if dist:
+            t = torch.tensor([e_s], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_s = float(t.item())
+            c = torch.tensor([float(sum(e_commits))], device=dev, dtype=torch.float64)
+            dist.all_reduce(c)
+            e_c = c[0].item()
+        else:
+            e_c = float(sum(e_commits))
+        e2e = {"value": e_c / e_s, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
+               "d2h_bytes_per_step": d2h // args.steps, "ms_per_step": 1000 * e_s / args.steps}
+
+    clk.__exit__(None, None, None)
+    if rank != 0:
+        if dist:
+            dist.barrier()
+            dist.destroy_process_group()
+        return
+
+    # ---- roofline of the dominant kernel (execute) ------------------------------------------------
+    peak, peak_kind = measured_peaks()
+    roof = None
+    if w["kind"] == "ycsb":
+        bytes_exec = statistics.mean(exec_algorithmic_bytes(host_batches[(args.warmup + s) % n_distinct])
+                                     for s in range(args.steps))
+        ms = statistics.mean(exec_ms)
+        ach = bytes_exec / (ms / 1000.0) / 1e9
+        roof = {"bound": "hbm", "kernel": "k_ops_exec", "achieved": ach, "peak": peak, "unit": "GB/s",
+                "frac": ach / peak, "traffic": ncu_traffic("k_ops_exec"), "peak_source": peak_kind,
+                "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
+                "kernel_share_of_step": ms / statistics.mean(step_ms)}
+    else:
+        ms = statistics.mean(exec_ms)
+        roof = {"bound": "hbm", "kernel": "k_tpcc_exec", "achieved": None, "peak": peak, "unit": "GB/s",
+                "frac": None, "traffic": ncu_traffic("k_tpcc_exec"), "peak_source": peak_kind, "kernel_ms": ms}
+
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": dict(config_of(name), parallelism="dp%d (independent partitions)" % world
+                           if world > 1 else "single GPU"),
+            "clocks": clk.summary(), "e2e": e2e, "gpu_launches": kernels, "roofline": roof,
+            "commit_rate": all_commits / all_procs, "processed_txns_per_s": all_procs / total_s,
+            "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)
+                              for k in ("ms_upload", "ms_group", "ms_exec", "ms_detect", "ms_writeback",
+                                        "ms_download")}}
+    if world == 1 and not args.no_cpu_baseline:
+        try:
+            line["cpu_baseline"] = cpu_baseline(name, host_batches[0], make_workload(name, 0))
+        except Exception as e:  # never lose the GPU number to the baseline leg
+            line["cpu_baseline"] = {"error": repr(e)}
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

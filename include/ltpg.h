@@ -150,7 +150,7 @@ typedef struct {
   uint32_t n_cols;              /* <= 16                                                 */
   const uint8_t* col_group;     /* host, n_cols                                          */
   const uint8_t* col_is_add;    /* host, n_cols                                          */
-  uint32_t n_groups;            /* mutable column groups (conflict units per row)        */
+  uint32_t n_groups;            /* mutable column groups (conflict units per row), <= 15 */
   uint64_t capacity_rows;       /* rows incl. the append region                          */
   uint32_t has_pk;              /* 1: u64 primary key + hash index; 0: keyless (append)  */
   uint32_t owner_rule;          /* multi-GPU: 0 replicated, 1 TPC-C warehouse, 2 key range */
@@ -181,6 +181,7 @@ typedef struct {
 typedef struct {
   float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;
   uint32_t n_commit, n_conflict, n_user_abort;
+  uint32_t n_kernels;           /* kernels this library launched for the batch */
 } ltpg_stats;
 
 typedef struct {

@@ -60,7 +60,7 @@ class ltpg_stats(ctypes.Structure):
     _fields_ = [("ms_upload", ctypes.c_float), ("ms_group", ctypes.c_float), ("ms_exec", ctypes.c_float),
                 ("ms_detect", ctypes.c_float), ("ms_exchange", ctypes.c_float),
                 ("ms_writeback", ctypes.c_float), ("ms_download", ctypes.c_float),
-                ("n_commit", c_u32), ("n_conflict", c_u32), ("n_user_abort", c_u32)]
+                ("n_commit", c_u32), ("n_conflict", c_u32), ("n_user_abort", c_u32), ("n_kernels", c_u32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -105,20 +105,16 @@ class LtpgError(RuntimeError):
         self.rc = rc
 
 
-def _is_torch(x):
-    return type(x).__module__.startswith("torch")
-
-
 def _ptr(x):
     if x is None:
         return None
-    if _is_torch(x):
+    if hasattr(x, "data_ptr"):  # torch tensor (host or CUDA)
         return c_vp(x.data_ptr())
     return x.ctypes.data_as(c_vp)
 
 
 def _on_device(x):
-    return _is_torch(x) and x.is_cuda
+    return bool(getattr(x, "is_cuda", False))
 
 
 class Database:
@@ -209,11 +205,13 @@ class Database:
             out["stats"] = st.as_dict()
         return out
 
-    def run_ops(self, batch, stream=None, want_reads=True, device_out=None, stats=False, out=None):
-        """batch: dict(tid u64[n], op_begin u32[n+1], ops OP_DTYPE/uint8[n_ops*16], args i64[n_ops])."""
+    def run_ops(self, batch, stream=None, want_reads=True, device_out=None, stats=False, out=None,
+                n_txns=None, n_ops=None):
+        """batch: dict(tid u64[n], op_begin u32[n+1], ops OP_DTYPE/uint8[n_ops*16], args i64[n_ops]).
+        Pass n_txns / n_ops when the arrays are raw byte views."""
         tid, ob, ops, args = batch["tid"], batch["op_begin"], batch["ops"], batch["args"]
-        n = len(tid)
-        n_ops = len(args)
+        n = len(tid) if n_txns is None else n_txns
+        n_ops = len(args) if n_ops is None else n_ops
         on_dev = _on_device(tid)
         if device_out is None:
             device_out = on_dev
@@ -222,10 +220,11 @@ class Database:
                         stream=c_vp(stream) if stream else None)
         return self._run(bt, n, n_ops, want_reads, device_out, stats, out)
 
-    def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None):
+    def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
+                 n_txns=None):
         """batch: dict(tid u64[n], type u8[n], params u8[n,128])."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
-        n = len(tid)
+        n = len(tid) if n_txns is None else n_txns
         on_dev = _on_device(tid)
         if device_out is None:
             device_out = on_dev

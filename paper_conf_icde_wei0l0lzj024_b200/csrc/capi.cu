@@ -24,6 +24,7 @@ struct ltpg_db {
   std::string last_error;
   uint32_t epoch = 0;
   uint32_t n_tables = 0;
+  uint64_t tab_version = 0;
   DevTable h_tab[MAXT]{};
   DevTable* d_tab = nullptr;
   unsigned long long* d_nrows = nullptr;  // [MAXT]
@@ -52,6 +53,9 @@ struct ltpg_db {
 };
 
 namespace {
+
+uint64_t g_tab_versions = 0;     // process-wide: every table load gets a new version
+uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __constant__
 
 int fail(ltpg_db* db, int code, const std::string& msg) {
   if (db) {
@@ -159,7 +163,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   if (db->poisoned) return LTPG_EPOISONED;
   if (!d || t >= db->n_tables || d->n_cols > MAXC || (d->n_cols && (!d->col_group || !d->col_is_add)) ||
       n_rows > d->capacity_rows || d->capacity_rows >= 0xFFFFFFF0ull || (n_rows && d->n_cols && !cols) ||
-      (d->has_pk && n_rows && !keys) || d->n_groups > 255)
+      (d->has_pk && n_rows && !keys) || d->n_groups > 15)
     return fail(db, LTPG_EINVAL, "bad table descriptor");
   bool has_static = false;
   for (uint32_t c = 0; c < d->n_cols; ++c) {
@@ -195,6 +199,14 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     T.is_add[c] = d->col_is_add[c] ? 1 : 0;
   }
   if (!d->n_cols) T.col[0] = colmem;
+  T.col0 = colmem;
+  T.group_bits = ~0ull;
+  T.add_bits = 0;
+  for (uint32_t c = 0; c < d->n_cols; ++c) {
+    uint64_t g = d->col_group[c] == LTPG_STATIC ? 15u : d->col_group[c];
+    T.group_bits = (T.group_bits & ~(15ull << (4 * c))) | (g << (4 * c));
+    if (d->col_is_add[c]) T.add_bits |= 1u << c;
+  }
   CK(dmalloc(&T.valid, cap));
   CK(cudaMemset(T.valid, 0, cap));
   CK(dmalloc(&T.rowkey, cap));
@@ -221,9 +233,12 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   unsigned long long nr = n_rows;
   CK(cudaMemcpy(T.n_rows, &nr, sizeof(nr), cudaMemcpyHostToDevice));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
+  db->tab_version = ++g_tab_versions;
   if (d->has_pk && n_rows) {
     CK(cudaMemset(db->d_small, 0, sizeof(uint32_t)));
-    launch_build_index(db->d_tab, t, 0, n_rows, db->d_small, 0);
+    upload_tables_common(db->d_tab, 0);
+    g_uploaded[db->device % 64] = 0;
+    launch_build_index(t, 0, n_rows, db->d_small, 0);
     CK(cudaGetLastError());
     uint32_t err = 0;
     CK(cudaMemcpy(&err, db->d_small, sizeof(err), cudaMemcpyDeviceToHost));
@@ -259,6 +274,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool timing = res->stats != nullptr;
   if (timing) CK(cudaEventRecord(db->ev[0], s));
   ++db->epoch;
+  const uint64_t launches0 = g_kernel_launches;
   BatchDev bd{};
   bd.n_txns = n;
   bd.n_ops = ops_mode ? b->n_ops : 0;
@@ -308,27 +324,35 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   CK(cudaMemsetAsync(db->d_small, 0, 16 * sizeof(uint32_t), s));
   if (n) CK(cudaMemsetAsync(db->d_ua, 0, n, s));
   if (timing) CK(cudaEventRecord(db->ev[1], s));
+  // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
+  // skipped when this device's constant bank already holds this db's current tables
+  if (g_uploaded[db->device % 64] != db->tab_version) {
+    upload_tables_common(db->d_tab, s);
+    upload_tables_ops(db->d_tab, s);
+    upload_tables_tpcc(db->d_tab, s);
+    g_uploaded[db->device % 64] = db->tab_version;
+  }
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
   if (n) {
     if (ops_mode) {
       // ---- a1/a2: validate + adaptive warp division ---------------------------------
-      launch_ops_validate_group(db->d_tab, db->n_tables, bd, grouped, s);
+      launch_ops_validate_group(db->n_tables, bd, grouped, s);
       scan_exclusive_u32(db->d_txn_ins, db->d_txn_ins, n, db->d_scan, s);
-      launch_capacity_check(db->d_tab, db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
+      launch_capacity_check(db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
       // ---- a3: insert claims ----------------------------------------------------------
-      launch_ops_claim(db->d_tab, bd, s);
+      launch_ops_claim(bd, s);
       if (timing) CK(cudaEventRecord(db->ev[2], s));
       // ---- a4/a5: execute + marks -----------------------------------------------------
-      launch_ops_exec(db->d_tab, bd, grouped, filter, s);
+      launch_ops_exec(bd, grouped, filter, s);
       if (timing) CK(cudaEventRecord(db->ev[3], s));
       // ---- a6: conflict detection -------------------------------------------------------
-      launch_ops_detect(db->d_tab, bd, s);
+      launch_ops_detect(bd, s);
       if (timing) CK(cudaEventRecord(db->ev[4], s));
       if (timing) CK(cudaEventRecord(db->ev[5], s));
       // ---- a7: write-back -------------------------------------------------------------
-      launch_ops_writeback(db->d_tab, bd, s);
-      launch_advance_cursor(db->d_tab, db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
+      launch_ops_writeback(bd, s);
+      launch_advance_cursor(db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
     } else {
       int rc = tpcc_run(db->tpcc, db->h_tab, db->d_tab, bd, db->cfg, s, timing ? db->ev : nullptr);
       if (rc) return fail(db, rc, "tpcc launch failed");
@@ -385,6 +409,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     st->n_commit = db->h_small[8];
     st->n_conflict = db->h_small[9];
     st->n_user_abort = db->h_small[10];
+    st->n_kernels = (uint32_t)(g_kernel_launches - launches0);
   }
   return LTPG_OK;
 }

@@ -5,6 +5,9 @@
 
 namespace ltpg {
 
+uint64_t g_kernel_launches = 0;
+LTPG_DEFINE_TABLE_UPLOAD(upload_tables_common)
+
 constexpr int SCAN_THREADS = 256;
 constexpr int SCAN_ITEMS = 16;
 constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;  // 4096 elements per block
@@ -104,8 +107,11 @@ void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t*
   }
   uint32_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;  // <= SCAN_TILE blocks (n <= 16.7M)
   k_scan_reduce<<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch);
+  note_launch();
   k_scan_top<<<1, SCAN_THREADS, 0, s>>>(scratch, nb);
+  note_launch();
   k_scan_down<<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb);
+  note_launch();
 }
 
 // Result finalisation: commit bitmask (one __ballot_sync word per warp), conflict
@@ -133,6 +139,7 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
                      const uint32_t* err, cudaStream_t s) {
   if (!n) return;
   k_finalize<<<(n + 255) / 256, 256, 0, s>>>(status, n, commit_bits, flags, counts, err);
+  note_launch();
 }
 
 // abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
@@ -145,11 +152,12 @@ __global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s) {
   if (!n) return;
   k_compact<<<(n + 255) / 256, 256, 0, s>>>(flags, offs, n, out);
+  note_launch();
 }
 
-__global__ void k_build_index(const DevTable* __restrict__ tabs, uint32_t t, uint64_t row0, uint64_t n,
+__global__ void k_build_index(uint32_t t, uint64_t row0, uint64_t n,
                               uint32_t* err) {
-  const DevTable& T = tabs[t];
+  const DevTable& T = c_tabs[t];
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     uint64_t row = row0 + i;
     uint64_t key = T.rowkey[row];
@@ -160,42 +168,45 @@ __global__ void k_build_index(const DevTable* __restrict__ tabs, uint32_t t, uin
   }
 }
 
-void launch_build_index(const DevTable* tabs, uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
+void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
                         cudaStream_t s) {
   if (!n) return;
   uint64_t blocks = (n + 255) / 256;
   if (blocks > 148 * 64) blocks = 148 * 64;
-  k_build_index<<<(unsigned)blocks, 256, 0, s>>>(tabs, t, row0, n, err);
+  k_build_index<<<(unsigned)blocks, 256, 0, s>>>(t, row0, n, err);
+  note_launch();
 }
 
 // ECAPACITY before anything mutates: provisional rows are n_rows + [0, total)
-__global__ void k_capacity(const DevTable* __restrict__ tabs, uint32_t n_tables, const uint32_t* ins_tables,
+__global__ void k_capacity(uint32_t n_tables, const uint32_t* ins_tables,
                            const uint32_t* total, uint32_t* err) {
   uint32_t m = *ins_tables;
   uint64_t tot = *total;
   for (uint32_t t = 0; t < n_tables; ++t)
     if ((m >> t) & 1u) {
-      const DevTable& T = tabs[t];
+      const DevTable& T = c_tabs[t];
       if (*T.n_rows + tot > T.capacity || *T.n_rows + tot > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
     }
 }
 
-void launch_capacity_check(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables,
                            const uint32_t* total, uint32_t* err, cudaStream_t s) {
-  k_capacity<<<1, 1, 0, s>>>(tabs, n_tables, ins_tables, total, err);
+  k_capacity<<<1, 1, 0, s>>>(n_tables, ins_tables, total, err);
+  note_launch();
 }
 
-__global__ void k_advance(const DevTable* __restrict__ tabs, uint32_t n_tables, const uint32_t* ins_tables,
+__global__ void k_advance(uint32_t n_tables, const uint32_t* ins_tables,
                           const uint32_t* total, const uint32_t* err) {
   if (*err) return;
   uint32_t m = *ins_tables;
   for (uint32_t t = 0; t < n_tables; ++t)
-    if ((m >> t) & 1u) *tabs[t].n_rows += *total;
+    if ((m >> t) & 1u) *c_tabs[t].n_rows += *total;
 }
 
-void launch_advance_cursor(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+void launch_advance_cursor(uint32_t n_tables, const uint32_t* ins_tables,
                            const uint32_t* total, const uint32_t* err, cudaStream_t s) {
-  k_advance<<<1, 1, 0, s>>>(tabs, n_tables, ins_tables, total, err);
+  k_advance<<<1, 1, 0, s>>>(n_tables, ins_tables, total, err);
+  note_launch();
 }
 
 }  // namespace ltpg

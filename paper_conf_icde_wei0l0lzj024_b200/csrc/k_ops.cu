@@ -11,6 +11,8 @@
 
 namespace ltpg {
 
+LTPG_DEFINE_TABLE_UPLOAD(upload_tables_ops)
+
 constexpr int OPS_MAX_TXN_OPS = 256;
 
 __device__ __forceinline__ ltpg_op load_op(const ltpg_op* ops, uint32_t i) {
@@ -24,14 +26,14 @@ __device__ __forceinline__ ltpg_op load_op(const ltpg_op* ops, uint32_t i) {
   return o;
 }
 
-__device__ __forceinline__ bool op_valid(const DevTable* tabs, uint32_t n_tables, const ltpg_op& o) {
+__device__ __forceinline__ bool op_valid(uint32_t n_tables, const ltpg_op& o) {
   if (o.table >= n_tables) return false;
-  const DevTable& T = tabs[o.table];
+  const DevTable& T = c_tabs[o.table];
   if (!T.defined || !T.has_pk || o.kind > LTPG_SCAN || o.key == KEY_EMPTY) return false;
   switch (o.kind) {
     case LTPG_SELECT: return o.col < T.n_cols;
-    case LTPG_UPDATE: return o.col < T.n_cols && T.group[o.col] != LTPG_STATIC && !T.is_add[o.col];
-    case LTPG_ADD: return o.col < T.n_cols && T.is_add[o.col];
+    case LTPG_UPDATE: return o.col < T.n_cols && col_group(T, o.col) != LTPG_STATIC && !col_is_add(T, o.col);
+    case LTPG_ADD: return o.col < T.n_cols && col_is_add(T, o.col);
     case LTPG_INSERT: return T.n_groups > 0;
     case LTPG_DELETE: return T.n_groups > 0 && !T.has_static;
     default:  // SCAN
@@ -46,12 +48,13 @@ __device__ __forceinline__ bool is_write_kind(uint8_t k) {
 
 // ---- K-group: validation + decomposition into per-kind lists (one thread per txn) ----
 template <bool GROUPED>
-__global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __restrict__ tabs, uint32_t n_tables,
+__global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
                                                             BatchDev b) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   const int lane = threadIdx.x & 31;
   bool bad = false;
-  uint32_t b0 = 0, b1 = 0, cnt[NKINDS] = {0, 0, 0, 0, 0, 0};
+  uint32_t b0 = 0, b1 = 0;
+  uint64_t cnt64 = 0;  // per-kind op counts, 10 bits each (no dynamically indexed arrays)
   uint32_t my_ins_tables = 0;
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
@@ -60,10 +63,41 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __re
     if (r == 0 && b0 != 0) bad = true;
     if (r == b.n_txns - 1 && b1 != b.n_ops) bad = true;
     if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS) { bad = true; b1 = b0; }
+    constexpr int FAST = 16;
+    if (b1 - b0 <= FAST) {
+      // short txns (YCSB, micro-cases): ops held in registers, R10 pairs fully unrolled
+      uint64_t lo[FAST], hi[FAST];
+      uint32_t tw[FAST];  // table | is_write << 8 | is_scan << 9 | valid slot << 10
+#pragma unroll
+      for (int i = 0; i < FAST; ++i) {
+        lo[i] = hi[i] = 0;
+        tw[i] = 0;
+        if (b0 + i < b1) {
+          ltpg_op o = load_op(b.ops, b0 + i);
+          if (!op_valid(n_tables, o)) bad = true;
+          else {
+            cnt64 += 1ull << (10 * o.kind);
+            if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
+          }
+          lo[i] = o.key;
+          hi[i] = o.kind == LTPG_SCAN ? o.key + o.aux : o.key + 1;
+          tw[i] = o.table | (uint32_t)is_write_kind(o.kind) << 8 | (uint32_t)(o.kind == LTPG_SCAN) << 9 | 1u << 10;
+        }
+      }
+#pragma unroll
+      for (int i = 1; i < FAST; ++i)
+#pragma unroll
+        for (int j = 0; j < i; ++j) {
+          const bool same = (tw[i] & 0x4FF) == (tw[j] & 0x4FF) && (tw[i] & 0x400);
+          const bool overlap = lo[i] < hi[j] && lo[j] < hi[i];
+          const bool forbid = ((tw[i] | tw[j]) & 0x100) || !((tw[i] | tw[j]) & 0x200);
+          if (same && overlap && forbid) bad = true;
+        }
+    } else {
     for (uint32_t i = b0; i < b1; ++i) {
       ltpg_op o = load_op(b.ops, i);
-      if (!op_valid(tabs, n_tables, o)) { bad = true; continue; }
-      cnt[o.kind]++;
+      if (!op_valid(n_tables, o)) { bad = true; continue; }
+      cnt64 += 1ull << (10 * o.kind);
       if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
     }
     // R10: a written key is touched by no other op of the txn (no read-your-writes)
@@ -81,7 +115,8 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __re
         }
       }
     }
-    b.txn_ins[r] = cnt[LTPG_INSERT];
+    }
+    b.txn_ins[r] = (uint32_t)(cnt64 >> (10 * LTPG_INSERT)) & 1023u;
     if (bad) atomicOr(b.err, ERR_EINVAL);
   }
   my_ins_tables = __reduce_or_sync(0xffffffffu, my_ins_tables);
@@ -103,7 +138,8 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __re
   uint32_t pos[NKINDS];
 #pragma unroll
   for (int k = 0; k < NKINDS; ++k) {
-    uint32_t x = cnt[k];
+    const uint32_t ck = (uint32_t)(cnt64 >> (10 * k)) & 1023u;
+    uint32_t x = ck;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
@@ -113,7 +149,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __re
     uint32_t base = 0;
     if (lane == 31 && tot) base = atomicAdd(b.kcount + k, tot);
     base = __shfl_sync(0xffffffffu, base, 31);
-    pos[k] = base + x - cnt[k];
+    pos[k] = base + x - ck;
   }
   if (r < b.n_txns && !bad)
     for (uint32_t i = b0; i < b1; ++i) {
@@ -126,18 +162,19 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(const DevTable* __re
     }
 }
 
-void launch_ops_validate_group(const DevTable* tabs, uint32_t n_tables, const BatchDev& b, bool grouped,
+void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool grouped,
                                cudaStream_t s) {
   uint32_t blocks = (b.n_txns + 255) / 256;
   if (grouped)
-    k_ops_validate_group<true><<<blocks, 256, 0, s>>>(tabs, n_tables, b);
+    k_ops_validate_group<true><<<blocks, 256, 0, s>>>(n_tables, b);
   else
-    k_ops_validate_group<false><<<blocks, 256, 0, s>>>(tabs, n_tables, b);
+    k_ops_validate_group<false><<<blocks, 256, 0, s>>>(n_tables, b);
+  note_launch();
 }
 
 // ---- K-claim: INSERT keys claim their slot; provisional row = n_rows + rank of the
 //      insert in (rank, op) order; atomicMin makes the earliest inserter own the unit ----
-__global__ void __launch_bounds__(256) k_ops_claim(const DevTable* __restrict__ tabs, BatchDev b) {
+__global__ void __launch_bounds__(256) k_ops_claim(BatchDev b) {
   if (*b.err) return;
   const uint32_t n = b.kcount[LTPG_INSERT];
   const unsigned long long* list = b.items + (uint64_t)LTPG_INSERT * b.max_ops;
@@ -145,7 +182,7 @@ __global__ void __launch_bounds__(256) k_ops_claim(const DevTable* __restrict__ 
     unsigned long long it = list[i];
     uint32_t oi = (uint32_t)it, r = (uint32_t)(it >> 32);
     ltpg_op o = load_op(b.ops, oi);
-    const DevTable& T = tabs[o.table];
+    const DevTable& T = c_tabs[o.table];
     uint32_t j = 0;
     for (uint32_t q = b.op_begin[r]; q < oi; ++q) j += b.ops[q].kind == LTPG_INSERT;
     uint32_t prov = (uint32_t)(*T.n_rows + b.txn_ins[r] + j);
@@ -156,14 +193,15 @@ __global__ void __launch_bounds__(256) k_ops_claim(const DevTable* __restrict__ 
   }
 }
 
-void launch_ops_claim(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
-  k_ops_claim<<<148 * 4, 256, 0, s>>>(tabs, b);
+void launch_ops_claim(const BatchDev& b, cudaStream_t s) {
+  k_ops_claim<<<148 * 4, 256, 0, s>>>(b);
+  note_launch();
 }
 
 // ---- K-exec ---------------------------------------------------------------------------
-__device__ __forceinline__ void exec_one(const DevTable* __restrict__ tabs, const BatchDev& b, uint32_t oi,
+__device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
                                          uint32_t r, const ltpg_op& o, bool filter) {
-  const DevTable& T = tabs[o.table];
+  const DevTable& T = c_tabs[o.table];
   const unsigned long long tag = epoch_tag(b.epoch) | r;
   uint32_t row, claim;
   long long res = LTPG_NOT_FOUND;
@@ -175,7 +213,7 @@ __device__ __forceinline__ void exec_one(const DevTable* __restrict__ tabs, cons
       idx_find(T, k, row, claim);
       if (row != ROW_NONE) {
         ++cnt;
-        if (o.col != LTPG_COL_COUNT) sum += (unsigned long long)*col_ptr(T, o.col, row);
+        if (o.col != LTPG_COL_COUNT) sum += (unsigned long long)*col_ptr_ops(T, o.col, row);
       }
     }
     b.res[oi] = o.col == LTPG_COL_COUNT ? cnt : (long long)sum;
@@ -194,21 +232,21 @@ __device__ __forceinline__ void exec_one(const DevTable* __restrict__ tabs, cons
   }
   switch (o.kind) {
     case LTPG_SELECT: {
-      res = *col_ptr(T, o.col, row);
-      uint32_t g = T.group[o.col];
+      res = *col_ptr_ops(T, o.col, row);
+      uint32_t g = col_group(T, o.col);
       uref = g == LTPG_STATIC ? make_uref(CHK_NONE, false, true, o.table, 0, row)
                               : make_uref(CHK_RW, false, true, o.table, g, row);
       break;
     }
     case LTPG_UPDATE: {
-      uint32_t g = T.group[o.col];
-      res = *col_ptr(T, o.col, row);  // pre-image; new value = res + arg at write-back
+      uint32_t g = col_group(T, o.col);
+      res = *col_ptr_ops(T, o.col, row);  // pre-image; new value = res + arg at write-back
       mark_min(mark_ptr(T, g, row), tag, filter);
       uref = make_uref(CHK_RW, false, true, o.table, g, row);
       break;
     }
     case LTPG_ADD: {
-      uint32_t g = T.group[o.col];
+      uint32_t g = col_group(T, o.col);
       res = 0;
       mark_min(mark_ptr(T, g, row) + 1, tag, filter);
       uref = make_uref(CHK_A, false, true, o.table, g, row);
@@ -240,10 +278,10 @@ __device__ __forceinline__ void exec_one(const DevTable* __restrict__ tabs, cons
 }
 
 template <bool GROUPED>
-__global__ void __launch_bounds__(256) k_ops_exec(const DevTable* __restrict__ tabs, BatchDev b, bool filter) {
+__global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
   if (*b.err) return;
   const int lane = threadIdx.x & 31;
-  uint32_t cnt[NKINDS], pref[NKINDS + 1];
+  uint32_t cnt[NKINDS], pref[NKINDS + 1];  // fully unrolled below: registers only
   pref[0] = 0;
 #pragma unroll
   for (int k = 0; k < NKINDS; ++k) {
@@ -254,32 +292,33 @@ __global__ void __launch_bounds__(256) k_ops_exec(const DevTable* __restrict__ t
   for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); (uint64_t)w * 32 < pref[NKINDS];
        w += nwarps) {
     const uint32_t p = w * 32;
-    int k = 0;
+    uint32_t k = 0, pk = 0, ck = cnt[0];
 #pragma unroll
     for (int kk = 1; kk < NKINDS; ++kk)
-      if (p >= pref[kk]) k = kk;  // warp-uniform op kind
-    const uint32_t idx = p - pref[k] + lane;
-    if (idx >= cnt[k]) continue;
+      if (p >= pref[kk]) { k = kk; pk = pref[kk]; ck = cnt[kk]; }  // warp-uniform op kind
+    const uint32_t idx = p - pk + lane;
+    if (idx >= ck) continue;
     const unsigned long long it = b.items[(uint64_t)k * b.max_ops + idx];
     const uint32_t oi = (uint32_t)it, r = (uint32_t)(it >> 32);
     const ltpg_op o = load_op(b.ops, oi);
-    exec_one(tabs, b, oi, r, o, filter);
+    exec_one(b, oi, r, o, filter);
   }
 }
 
-void launch_ops_exec(const DevTable* tabs, const BatchDev& b, bool grouped, bool filter, cudaStream_t s) {
+void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s) {
   uint64_t warps = (b.n_ops + NKINDS * 32 + 31) / 32;
   uint64_t blocks = (warps + 7) / 8;
   if (blocks > 148 * 16) blocks = 148 * 16;
   if (!blocks) return;
   if (grouped)
-    k_ops_exec<true><<<(unsigned)blocks, 256, 0, s>>>(tabs, b, filter);
+    k_ops_exec<true><<<(unsigned)blocks, 256, 0, s>>>(b, filter);
   else
-    k_ops_exec<false><<<(unsigned)blocks, 256, 0, s>>>(tabs, b, filter);
+    k_ops_exec<false><<<(unsigned)blocks, 256, 0, s>>>(b, filter);
+  note_launch();
 }
 
 // ---- K-detect: per txn, OR of the unit tests over its ops ------------------------------
-__global__ void __launch_bounds__(256) k_ops_detect(const DevTable* __restrict__ tabs, BatchDev b) {
+__global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   if (*b.err) return;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
@@ -289,7 +328,7 @@ __global__ void __launch_bounds__(256) k_ops_detect(const DevTable* __restrict__
     const uint64_t u = b.uref[i];
     const uint64_t chk = u >> 62;
     if (chk == CHK_NONE) continue;
-    const DevTable& T = tabs[(u >> 40) & 0xFF];
+    const DevTable& T = c_tabs[(u >> 40) & 0xFF];
     if (chk == CHK_SCAN) {  // phantom-safe: every key of the range is a read (R8)
       const ltpg_op o = load_op(b.ops, i);
       if (!T.n_groups) continue;
@@ -297,7 +336,7 @@ __global__ void __launch_bounds__(256) k_ops_detect(const DevTable* __restrict__
         uint32_t row, claim;
         idx_find(T, k, row, claim);
         if (row != ROW_NONE) {
-          uint32_t g = (o.col != LTPG_COL_COUNT && T.group[o.col] != LTPG_STATIC) ? T.group[o.col] : 0;
+          uint32_t g = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
           bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);
         } else if (claim != ROW_NONE) {
           bad = unit_conflicts(T, 0, claim, CHK_RW, r, b.epoch);
@@ -315,16 +354,18 @@ __global__ void __launch_bounds__(256) k_ops_detect(const DevTable* __restrict__
   b.status[r] = bad ? LTPG_ST_CONFLICT : (b.ua[r] ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
 }
 
-void launch_ops_detect(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
-  k_ops_detect<<<(b.n_txns + 255) / 256, 256, 0, s>>>(tabs, b);
+void launch_ops_detect(const BatchDev& b, cudaStream_t s) {
+  k_ops_detect<<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
+  note_launch();
 }
 
 // ---- K-wb: apply committed write sets; every INSERT releases its claim ----------------
-__global__ void __launch_bounds__(256) k_ops_writeback(const DevTable* __restrict__ tabs, BatchDev b) {
+__global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b) {
   if (*b.err) return;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
   const bool commit = b.status[r] == LTPG_ST_COMMIT;
+  if (!commit && b.txn_ins[r + 1] == b.txn_ins[r]) return;  // aborted, no claims to release
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
   for (uint32_t i = b0; i < b1; ++i) {
     const uint64_t u = b.uref[i];
@@ -336,13 +377,13 @@ __global__ void __launch_bounds__(256) k_ops_writeback(const DevTable* __restric
     if (kind == LTPG_INSERT) {
       if (present) continue;  // duplicate-key user abort: nothing claimed
       const ltpg_op o = load_op(b.ops, i);
-      const DevTable& T = tabs[o.table];
+      const DevTable& T = c_tabs[o.table];
       IdxSlot* sl = idx_slot(T, o.key);
       if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
       if (commit) {
         const long long arg = b.args[i];
         for (uint32_t c = 0; c < T.n_cols; ++c)
-          *col_ptr(T, c, row) = (long long)((unsigned long long)arg + c);
+          *col_ptr_ops(T, c, row) = (long long)((unsigned long long)arg + c);
         T.rowkey[row] = o.key;
         T.valid[row] = 1;
         sl->row = row;
@@ -352,13 +393,13 @@ __global__ void __launch_bounds__(256) k_ops_writeback(const DevTable* __restric
     }
     if (!present) continue;
     const ltpg_op o = load_op(b.ops, i);
-    const DevTable& T = tabs[o.table];
+    const DevTable& T = c_tabs[o.table];
     switch (kind) {
       case LTPG_UPDATE:
-        *col_ptr(T, o.col, row) = (long long)((unsigned long long)b.res[i] + (unsigned long long)b.args[i]);
+        *col_ptr_ops(T, o.col, row) = (long long)((unsigned long long)b.res[i] + (unsigned long long)b.args[i]);
         break;
       case LTPG_ADD:  // delayed update: commutative, order-free and exact
-        atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr(T, o.col, row)), (unsigned long long)b.args[i]);
+        atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr_ops(T, o.col, row)), (unsigned long long)b.args[i]);
         break;
       case LTPG_DELETE: {
         T.valid[row] = 0;
@@ -372,8 +413,9 @@ __global__ void __launch_bounds__(256) k_ops_writeback(const DevTable* __restric
   }
 }
 
-void launch_ops_writeback(const DevTable* tabs, const BatchDev& b, cudaStream_t s) {
-  k_ops_writeback<<<(b.n_txns + 255) / 256, 256, 0, s>>>(tabs, b);
+void launch_ops_writeback(const BatchDev& b, cudaStream_t s) {
+  k_ops_writeback<<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
+  note_launch();
 }
 
 }  // namespace ltpg

@@ -2,6 +2,7 @@
 #include "tpcc_internal.cuh"
 
 namespace ltpg {
+LTPG_DEFINE_TABLE_UPLOAD(upload_tables_tpcc)
 int tpcc_alloc(TpccDev& t, uint32_t max_txns) { t.max_txns = max_txns; return 0; }
 void tpcc_free(TpccDev& t) { (void)t; }
 int tpcc_build_secondary(TpccDev&, const DevTable*, const DevTable*, uint32_t) { return 0; }

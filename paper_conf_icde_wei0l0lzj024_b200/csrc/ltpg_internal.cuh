@@ -52,7 +52,21 @@ struct DevTable {
   uint64_t idx_mask;
   uint32_t idx_shift;
   unsigned long long* n_rows;     // device append cursor
+  // warp-uniform forms of the per-column metadata (OPS path indexes columns by a
+  // per-lane col id; dynamically indexed __constant__ arrays would serialise)
+  long long* col0;                // SoA base: column c starts at col0 + c * capacity
+  uint64_t group_bits;            // 4 bits per column: group id, 15 = static
+  uint32_t add_bits;              // bit c: column c is a delayed-ADD column
 };
+
+__device__ __forceinline__ uint32_t col_group(const DevTable& T, uint32_t c) {
+  uint32_t g = (uint32_t)(T.group_bits >> (4 * c)) & 15u;
+  return g == 15u ? LTPG_STATIC : g;
+}
+__device__ __forceinline__ bool col_is_add(const DevTable& T, uint32_t c) { return (T.add_bits >> c) & 1u; }
+__device__ __forceinline__ long long* col_ptr_ops(const DevTable& T, uint32_t c, uint32_t row) {
+  return T.col0 + (uint64_t)c * T.capacity + row;
+}
 
 __host__ __device__ inline uint64_t idx_hash(uint64_t key, uint32_t shift) {
   return (key * 0x9E3779B97F4A7C15ull) >> shift;
@@ -73,7 +87,7 @@ __device__ __forceinline__ uint32_t mark_rank(unsigned long long v, uint32_t epo
 // atomic, never a missing one (result-identical).
 __device__ __forceinline__ void mark_min(unsigned long long* p, unsigned long long v, bool filter) {
   if (filter) {
-    unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(p);
+    const unsigned long long cur = __ldcg(p);  // L2-coherent read, no system-scope fence
     if (cur <= v) return;
   }
   atomicMin(p, v);
@@ -151,7 +165,24 @@ __device__ __forceinline__ bool unit_conflicts(const DevTable& T, uint32_t g, ui
   return (w < a ? w : a) < r;
 }
 
+// Table metadata lives in __constant__ memory: warp-uniform table ids broadcast from
+// the constant cache and are never evicted by the random data traffic (an ncu run
+// showed per-op DevTable loads through L1 missing to L2).  Every translation unit
+// has its own copy, uploaded stream-ordered before each batch (upload_tables_*).
+static __constant__ DevTable c_tabs[MAXT];
+#define LTPG_DEFINE_TABLE_UPLOAD(fn)                                                            \
+  void fn(const DevTable* d, cudaStream_t s) { /* d: device copy -> async D2D */                \
+    cudaMemcpyToSymbolAsync(c_tabs, d, sizeof(DevTable) * MAXT, 0, cudaMemcpyDeviceToDevice, s); \
+  }
+void upload_tables_common(const DevTable* h, cudaStream_t s);
+void upload_tables_ops(const DevTable* h, cudaStream_t s);
+void upload_tables_tpcc(const DevTable* h, cudaStream_t s);
+
 // ---- host-side launchers (defined in the .cu files) ----------------------------------
+// number of kernels launched by this library (reported per batch in ltpg_stats)
+extern uint64_t g_kernel_launches;
+inline void note_launch(uint32_t k = 1) { g_kernel_launches += k; }
+
 struct BatchDev {
   uint32_t n_txns, n_ops, epoch, flags;
   int64_t clock;
@@ -176,20 +207,20 @@ struct BatchDev {
 void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
 size_t scan_scratch_words(uint32_t n);
 
-void launch_ops_validate_group(const DevTable* tabs, uint32_t n_tables, const BatchDev& b, bool grouped,
+void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool grouped,
                                cudaStream_t s);
-void launch_ops_claim(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
-void launch_ops_exec(const DevTable* tabs, const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
-void launch_ops_detect(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
-void launch_ops_writeback(const DevTable* tabs, const BatchDev& b, cudaStream_t s);
-void launch_capacity_check(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+void launch_ops_claim(const BatchDev& b, cudaStream_t s);
+void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
+void launch_ops_detect(const BatchDev& b, cudaStream_t s);
+void launch_ops_writeback(const BatchDev& b, cudaStream_t s);
+void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables,
                            const uint32_t* total, uint32_t* err, cudaStream_t s);
-void launch_advance_cursor(const DevTable* tabs, uint32_t n_tables, const uint32_t* ins_tables,
+void launch_advance_cursor(uint32_t n_tables, const uint32_t* ins_tables,
                            const uint32_t* total, const uint32_t* err, cudaStream_t s);
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);
-void launch_build_index(const DevTable* tabs, uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
+void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
                         cudaStream_t s);
 
 }  // namespace ltpg

@@ -103,13 +103,16 @@ class YcsbWorkload:
         k = self.ops_per_txn
         keys = self._draw_keys(rng, (n_txns, k))
         # distinct keys per txn: resample duplicate positions
-        while True:
-            eq = keys[:, :, None] == keys[:, None, :]
-            dup = np.triu(np.ones((k, k), dtype=bool), 1)[None, :, :] & eq  # j<l and equal
-            pos = dup.any(axis=1)  # position l duplicates an earlier j
-            if not pos.any():
-                break
-            keys[pos] = self._draw_keys(rng, int(pos.sum()))
+        upper = np.triu(np.ones((k, k), dtype=bool), 1)[None, :, :]
+        s = np.sort(keys, axis=1)
+        rows = np.nonzero((s[:, 1:] == s[:, :-1]).any(axis=1))[0]  # txns with a repeated key
+        while len(rows):
+            sub = keys[rows]
+            pos = ((sub[:, :, None] == sub[:, None, :]) & upper).any(axis=1)  # l repeats an earlier j
+            sub[pos] = self._draw_keys(rng, int(pos.sum()))
+            keys[rows] = sub
+            s = np.sort(sub, axis=1)
+            rows = rows[(s[:, 1:] == s[:, :-1]).any(axis=1)]
         u = rng.random((n_txns, k))
         kinds = np.where(u < self.read_frac, SELECT, UPDATE).astype(np.uint8)
         ops = np.zeros(n_txns * k, dtype=OP_DTYPE)
