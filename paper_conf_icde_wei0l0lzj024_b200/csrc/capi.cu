@@ -135,8 +135,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaMallocHost(reinterpret_cast<void**>(&db->h_small), 64 * sizeof(uint32_t)));
   for (auto& e : db->ev) CK(cudaEventCreate(&e));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
-  int rc = tpcc_alloc(db->tpcc, cfg->max_txns);
-  if (rc) return fail(db, rc, "tpcc scratch allocation failed");
+  int rc = tpcc_alloc(db->tpcc, cfg->max_txns, cfg->n_warehouses);
+  if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
   return LTPG_OK;
 }
 
@@ -249,7 +249,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     }
   }
   if (t == LTPG_T_CUSTOMER && db->cfg.n_warehouses) {
-    int rc = tpcc_build_secondary(db->tpcc, db->h_tab, db->d_tab, db->cfg.n_warehouses);
+    int rc = tpcc_build_secondary(db->tpcc, keys, cols, n_rows, db->cfg.n_warehouses);
     if (rc) return fail(db, rc, "secondary index build failed");
   }
   CK(cudaDeviceSynchronize());
@@ -354,7 +354,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       launch_ops_writeback(bd, s);
       launch_advance_cursor(db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
     } else {
-      int rc = tpcc_run(db->tpcc, db->h_tab, db->d_tab, bd, db->cfg, s, timing ? db->ev : nullptr);
+      int rc = tpcc_run(db->tpcc, bd, db->d_scan, s, timing ? db->ev : nullptr);
       if (rc) return fail(db, rc, "tpcc launch failed");
     }
     // ---- finalize: commit bitmask, abort list ------------------------------------------

@@ -1,12 +1,793 @@
-// TPC-C PROC mode (placeholder until the procedure kernels land).
+// TPC-C PROC mode: pre-compiled stored procedures decomposed into typed
+// sub-transactions and run by type-homogeneous warps (adaptive warp division,
+// P:195-199, Fig. 3):
+//   NewOrder    16 lanes / txn: lane l < n = order line l (item + stock RMW), lane 15 = header
+//   Payment      1 lane  / txn
+//   OrderStatus 16 lanes / txn: lane 15 = customer + order, lanes < cnt = order lines
+//   Delivery    16 lanes / txn: lane d-1 = district d
+//   StockLevel  32 lanes / txn: lanes over the 20-order window, then over distinct items
+// Every procedure is one template instantiated for the three phases of Alg. 1:
+//   PH_EXEC    readMem / recordLS / recordTID (marks)
+//   PH_DETECT  rcheck / wcheck over the same units
+//   PH_WB      writeMem of committed txns
+// so the unit set checked is by construction the unit set marked.  Rows found by
+// execute are logged (NewOrder / Payment / OrderStatus) and reused; Delivery and
+// StockLevel re-derive their rows (their lookups are static or own-unit reads).
+// NewOrder's fetch-ADD of D_NEXT_O_ID (R12, delayed-update prefix sum P:241) is
+// resolved after detection by a per-district prefix count in rank order.
+#include <algorithm>
+#include <map>
+#include <vector>
+
 #include "tpcc_internal.cuh"
 
 namespace ltpg {
+
 LTPG_DEFINE_TABLE_UPLOAD(upload_tables_tpcc)
-int tpcc_alloc(TpccDev& t, uint32_t max_txns) { t.max_txns = max_txns; return 0; }
-void tpcc_free(TpccDev& t) { (void)t; }
-int tpcc_build_secondary(TpccDev&, const DevTable*, const DevTable*, uint32_t) { return 0; }
-int tpcc_run(TpccDev&, const DevTable*, const DevTable*, BatchDev&, const ltpg_config&, cudaStream_t, cudaEvent_t*) {
-  return LTPG_EINVAL;
+
+enum { PH_EXEC = 0, PH_DETECT = 1, PH_WB = 2 };
+
+__device__ __forceinline__ uint32_t p16(const uint8_t* p, int off) { return *reinterpret_cast<const uint16_t*>(p + off); }
+__device__ __forceinline__ uint32_t p32(const uint8_t* p, int off) { return *reinterpret_cast<const uint32_t*>(p + off); }
+__device__ __forceinline__ long long p64(const uint8_t* p, int off) { return *reinterpret_cast<const long long*>(p + off); }
+
+__device__ __forceinline__ uint64_t kD(uint64_t w, uint64_t d) { return w * 10 + d; }
+__device__ __forceinline__ uint64_t kC(uint64_t w, uint64_t d, uint64_t c) { return kD(w, d) * 3000 + c; }
+__device__ __forceinline__ uint64_t kS(uint64_t w, uint64_t i) { return w * 100000 + i; }
+__device__ __forceinline__ uint64_t kO(uint64_t w, uint64_t d, uint64_t o) { return (kD(w, d) << 32) | o; }
+
+__device__ __forceinline__ uint32_t probe(const DevTable& T, uint64_t key) {
+  uint32_t row, claim;
+  idx_find(T, key, row, claim);
+  return row;
 }
+__device__ __forceinline__ long long rd(const DevTable& T, uint32_t c, uint32_t row) { return *col_ptr(T, c, row); }
+__device__ __forceinline__ void wr(const DevTable& T, uint32_t c, uint32_t row, long long v) { *col_ptr(T, c, row) = v; }
+__device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row, long long v) {
+  atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr(T, c, row)), (unsigned long long)v);
+}
+
+struct Tx {
+  uint32_t r;
+  uint32_t epoch;
+  unsigned long long tag;
+  bool filter;
+  bool bad;
+  uint32_t* err;
+};
+
+__device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINTERNAL); }
+
+// unit actions per phase: plain write (W mark / RW check), delayed add (A mark / A check),
+// marked read (RW check only; reads leave no mark under R1)
+template <int PH>
+__device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
+  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter);
+  if (PH == PH_DETECT) x.bad |= unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+}
+template <int PH>
+__device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
+  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter);
+  if (PH == PH_DETECT) x.bad |= unit_conflicts(T, g, row, CHK_A, x.r, x.epoch);
+}
+template <int PH>
+__device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
+  if (PH == PH_DETECT && g != LTPG_STATIC) x.bad |= unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+}
+// update of column c (strict: WRITE unit of its group; delayed: ADD unit)
+template <int PH>
+__device__ __forceinline__ void col_upd(const DevTable& T, uint32_t c, uint32_t row, Tx& x) {
+  if (col_is_add(T, c)) unit_a<PH>(T, col_group(T, c), row, x);
+  else unit_w<PH>(T, col_group(T, c), row, x);
+}
+// same for columns c1..c3 updated together; a unit shared by several columns is touched once
+template <int PH>
+__device__ __forceinline__ void col_upd3(const DevTable& T, uint32_t c1, uint32_t c2, uint32_t c3, uint32_t row,
+                                         Tx& x) {
+  const uint32_t g1 = col_group(T, c1), g2 = col_group(T, c2), g3 = col_group(T, c3);
+  col_upd<PH>(T, c1, row, x);
+  if (g2 != g1) col_upd<PH>(T, c2, row, x);
+  if (g3 != g1 && g3 != g2) col_upd<PH>(T, c3, row, x);
+}
+
+__device__ __forceinline__ long long seg16_sum(long long v) {
+#pragma unroll
+  for (int o = 8; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o, 16);
+  return v;
+}
+__device__ __forceinline__ uint32_t seg16_or(uint32_t v) {
+#pragma unroll
+  for (int o = 8; o; o >>= 1) v |= __shfl_xor_sync(0xffffffffu, v, o, 16);
+  return v;
+}
+
+// ---- NewOrder (TPC-C 2.4; SURVEY §8(c) procedure table) --------------------------------
+template <int PH>
+__device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active, Tx& x) {
+  const DevTable& TWh = c_tabs[TW];
+  const DevTable& TDi = c_tabs[TD];
+  const DevTable& TCu = c_tabs[TC];
+  const DevTable& TIt = c_tabs[TI];
+  const DevTable& TSt = c_tabs[TS];
+  const uint8_t* p = b.params + 128ull * r;
+  uint32_t w = 0, d = 0, n = 0, c = 0;
+  if (active) {
+    w = p16(p, 0);
+    d = p[2];
+    n = p[3];
+    c = p16(p, 4);
+  }
+  uint32_t* log = tp.log + (uint64_t)r * TLOG;
+  long long amount = 0;
+  uint32_t remote = 0, ua = 0;
+  uint32_t i = 0, sw = 0, qty = 0, row_s = ROW_NONE;
+  const bool line = active && sub < n;
+  if (line) {
+    const uint8_t* L = p + 8 + 8 * sub;
+    i = p32(L, 0);
+    sw = p16(L, 4);
+    qty = L[6];
+    remote = sw != w;
+    if (PH == PH_EXEC || PH == PH_WB) {
+      const uint32_t row_i = probe(TIt, i);
+      if (row_i == ROW_NONE) {
+        ua = 1;  // unused item id: NewOrder rollback (R11)
+      } else {
+        amount = (long long)qty * rd(TIt, I_PRICE, row_i);
+      }
+    }
+    if (PH == PH_EXEC) {
+      if (!ua) {
+        row_s = probe(TSt, kS(sw, i));
+        if (row_s == ROW_NONE) internal_error(x);
+      }
+      log[sub] = row_s;
+    } else {
+      row_s = log[sub];
+    }
+    if (row_s != ROW_NONE) {
+      const uint32_t gq = col_group(TSt, S_QUANTITY);
+      unit_w<PH>(TSt, gq, row_s, x);  // S_QUANTITY: conditional RMW -> WRITE unit
+      if (col_group(TSt, S_YTD) != gq)  // delayed mode: the counters form their own ADD unit
+        col_upd3<PH>(TSt, S_YTD, S_ORDER_CNT, S_REMOTE_CNT, row_s, x);
+      if (PH == PH_WB) {
+        const long long q = rd(TSt, S_QUANTITY, row_s);
+        wr(TSt, S_QUANTITY, row_s, q >= (long long)qty + 10 ? q - qty : q - qty + 91);
+        addv(TSt, S_YTD, row_s, qty);
+        addv(TSt, S_ORDER_CNT, row_s, 1);
+        addv(TSt, S_REMOTE_CNT, row_s, remote);
+      }
+    }
+  }
+  // header lane: warehouse / district / customer reads, fetch-ADD of D_NEXT_O_ID
+  long long w_tax = 0, d_tax = 0, disc = 0;
+  if (active && sub == 15) {
+    uint32_t row_d;
+    if (PH == PH_EXEC) {
+      const uint32_t row_w = probe(TWh, w);
+      row_d = probe(TDi, kD(w, d));
+      const uint32_t row_c = probe(TCu, kC(w, d, c));
+      if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
+        internal_error(x);
+        row_d = ROW_NONE;
+      } else {
+        w_tax = rd(TWh, W_TAX, row_w);  // static reads: unmarked (R4)
+        d_tax = rd(TDi, D_TAX, row_d);
+        disc = rd(TCu, C_DISCOUNT, row_c);
+      }
+      log[15] = row_d;
+    } else {
+      row_d = log[15];
+    }
+    if (row_d != ROW_NONE) unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+  }
+  if (PH == PH_EXEC) {
+    const long long sum = seg16_sum(amount);
+    ua = seg16_or(ua);
+    if (active && sub == 15) {
+      long long* res = b.res + 4ull * r;
+      res[0] = 0;  // o_id: assigned after detection if committed
+      res[1] = sum * (10000 - disc) * (10000 + w_tax + d_tax) / 100000000;
+      res[2] = sum;
+      res[3] = 0;
+      if (ua) b.ua[r] = 1;
+    }
+  }
+  if (PH == PH_WB) {
+    const uint32_t all_local = !seg16_or(remote);
+    if (active) {
+      const long long o = b.res[4ull * r];
+      const uint64_t okey = kO(w, d, (uint64_t)o);
+      const DevTable& TOr = c_tabs[TO];
+      const DevTable& TOL_ = c_tabs[TOL];
+      const DevTable& TNw = c_tabs[TNO];
+      if (line) {  // ORDER_LINE row
+        const uint32_t row = (uint32_t)(*TOL_.n_rows + tp.no_lines[r] + sub);
+        wr(TOL_, OL_I_ID, row, i);
+        wr(TOL_, OL_SUPPLY_W_ID, row, sw);
+        wr(TOL_, OL_QUANTITY, row, qty);
+        wr(TOL_, OL_AMOUNT, row, amount);
+        wr(TOL_, OL_DELIVERY_D, row, 0);
+        const uint64_t k = okey * 16 + sub + 1;
+        TOL_.rowkey[row] = k;
+        TOL_.valid[row] = 1;
+        IdxSlot* sl = idx_find_or_insert(TOL_, k);
+        if (sl) sl->row = row; else internal_error(x);
+      }
+      if (sub == 15) {  // ORDER and NEW_ORDER rows
+        const uint32_t orow = (uint32_t)(*TOr.n_rows + tp.no_flag[r]);
+        wr(TOr, O_C_ID, orow, c);
+        wr(TOr, O_ENTRY_D, orow, b.clock);
+        wr(TOr, O_OL_CNT, orow, n);
+        wr(TOr, O_ALL_LOCAL, orow, all_local);
+        wr(TOr, O_CARRIER_ID, orow, 0);
+        TOr.rowkey[orow] = okey;
+        TOr.valid[orow] = 1;
+        IdxSlot* sl = idx_find_or_insert(TOr, okey);
+        if (sl) sl->row = orow; else internal_error(x);
+        const uint32_t nrow = (uint32_t)(*TNw.n_rows + tp.no_flag[r]);
+        wr(TNw, NO_O_ID, nrow, o);
+        TNw.rowkey[nrow] = okey;
+        TNw.valid[nrow] = 1;
+        sl = idx_find_or_insert(TNw, okey);
+        if (sl) sl->row = nrow; else internal_error(x);
+      }
+    }
+  }
+}
+
+// ---- Payment (TPC-C 2.5) ------------------------------------------------------------------
+template <int PH>
+__device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r, Tx& x) {
+  const DevTable& TWh = c_tabs[TW];
+  const DevTable& TDi = c_tabs[TD];
+  const DevTable& TCu = c_tabs[TC];
+  const uint8_t* p = b.params + 128ull * r;
+  const uint32_t w = p16(p, 0), d = p[2], by_name = p[3], cw = p16(p, 4), cd = p[6];
+  uint32_t cid = p16(p, 8);
+  const uint32_t clast = p16(p, 10);
+  const long long amount = p64(p, 16);
+  uint32_t* log = tp.log + (uint64_t)r * TLOG;
+  uint32_t row_w, row_d, row_c;
+  if (PH == PH_EXEC) {
+    if (by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
+    row_w = probe(TWh, w);
+    row_d = probe(TDi, kD(w, d));
+    row_c = cid ? probe(TCu, kC(cw, cd, cid)) : ROW_NONE;
+    if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
+      internal_error(x);
+      return;
+    }
+    log[0] = row_w;
+    log[1] = row_d;
+    log[2] = row_c;
+    log[3] = cid;
+    long long* res = b.res + 4ull * r;
+    res[0] = cid;
+    res[1] = col_is_add(TCu, C_BALANCE) ? 0 : rd(TCu, C_BALANCE, row_c);  // pre-image (strict only)
+    res[2] = 0;
+    res[3] = 0;
+  } else {
+    row_w = log[0];
+    row_d = log[1];
+    row_c = log[2];
+    cid = log[3];
+  }
+  col_upd<PH>(TWh, W_YTD, row_w, x);
+  col_upd<PH>(TDi, D_YTD, row_d, x);
+  col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, row_c, x);
+  if (PH == PH_WB) {
+    addv(TWh, W_YTD, row_w, amount);
+    addv(TDi, D_YTD, row_d, amount);
+    addv(TCu, C_BALANCE, row_c, -amount);
+    addv(TCu, C_YTD_PAYMENT, row_c, amount);
+    addv(TCu, C_PAYMENT_CNT, row_c, 1);
+    const DevTable& THi = c_tabs[TH];  // keyless append, no marks
+    const uint32_t row = (uint32_t)(*THi.n_rows + atomicAdd(tp.misc + M_HIST, 1u));
+    wr(THi, H_C_ID, row, cid);
+    wr(THi, H_C_D_ID, row, cd);
+    wr(THi, H_C_W_ID, row, cw);
+    wr(THi, H_D_ID, row, d);
+    wr(THi, H_W_ID, row, w);
+    wr(THi, H_DATE, row, b.clock);
+    wr(THi, H_AMOUNT, row, amount);
+    wr(THi, H_TID, row, (long long)b.tid[r]);
+    wr(THi, H_SEQ, row, 0);
+    THi.valid[row] = 1;
+  }
+}
+
+// ---- OrderStatus (TPC-C 2.6) with a predefined order key ----------------------------
+template <int PH>
+__device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active,
+                                 Tx& x) {
+  const DevTable& TCu = c_tabs[TC];
+  const DevTable& TOr = c_tabs[TO];
+  const DevTable& TOL_ = c_tabs[TOL];
+  const uint8_t* p = b.params + 128ull * r;
+  uint32_t* log = tp.log + (uint64_t)r * TLOG;
+  uint32_t w = 0, d = 0, cid = 0, o = 0, cnt = 0, row_c = ROW_NONE, row_o = ROW_NONE;
+  long long bal = 0, carrier = 0;
+  if (active) {
+    w = p16(p, 0);
+    d = p[2];
+  }
+  if (active && sub == 15) {
+    if (PH == PH_EXEC) {
+      cid = p[3] ? (uint32_t)tp.by_name[kD(w, d) * 1000 + p16(p, 6)] : p16(p, 4);
+      row_c = cid ? probe(TCu, kC(w, d, cid)) : ROW_NONE;
+      if (row_c != ROW_NONE) {
+        bal = rd(TCu, C_BALANCE, row_c);
+        o = (uint32_t)rd(TCu, C_INIT_O_ID, row_c);
+        row_o = probe(TOr, kO(w, d, o));
+      }
+      if (row_o == ROW_NONE) {
+        internal_error(x);
+      } else {
+        carrier = rd(TOr, O_CARRIER_ID, row_o);
+        cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
+      }
+      log[15] = row_c;
+      log[16] = row_o;
+    } else {
+      row_c = log[15];
+      row_o = log[16];
+      cnt = row_o != ROW_NONE ? (uint32_t)rd(TOr, O_OL_CNT, row_o) : 0;
+    }
+    if (row_c != ROW_NONE) unit_r<PH>(TCu, col_group(TCu, C_BALANCE), row_c, x);
+    if (row_o != ROW_NONE) unit_r<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x);
+  }
+  o = __shfl_sync(0xffffffffu, o, 15, 16);
+  cnt = __shfl_sync(0xffffffffu, cnt, 15, 16);
+  long long dd = 0;
+  if (active && sub < cnt && sub < 15) {
+    uint32_t row_ol;
+    if (PH == PH_EXEC) {
+      row_ol = probe(TOL_, kO(w, d, o) * 16 + sub + 1);
+      if (row_ol == ROW_NONE) internal_error(x);
+      else dd = rd(TOL_, OL_DELIVERY_D, row_ol);
+      log[sub] = row_ol;
+    } else {
+      row_ol = log[sub];
+    }
+    if (row_ol != ROW_NONE) unit_r<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol, x);
+  }
+  if (PH == PH_EXEC) {
+    dd = seg16_sum(dd);
+    if (active && sub == 15) {
+      long long* res = b.res + 4ull * r;
+      res[0] = cid;
+      res[1] = bal;
+      res[2] = carrier;
+      res[3] = dd;
+    }
+  }
+}
+
+// ---- Delivery (TPC-C 2.7), one lane per district; rows re-derived in every phase ----------------
+template <int PH>
+__device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool active, Tx& x) {
+  const DevTable& TDi = c_tabs[TD];
+  const DevTable& TCu = c_tabs[TC];
+  const DevTable& TOr = c_tabs[TO];
+  const DevTable& TOL_ = c_tabs[TOL];
+  const DevTable& TNw = c_tabs[TNO];
+  const uint8_t* p = b.params + 128ull * r;
+  long long delivered = 0, total = 0;
+  if (active && sub < 10) {
+    const uint32_t w = p16(p, 0);
+    const long long carrier = p[2];
+    const uint32_t d = sub + 1;
+    const uint32_t row_d = probe(TDi, kD(w, d));
+    if (row_d == ROW_NONE) {
+      internal_error(x);
+    } else {
+      const long long o = rd(TDi, D_NEXT_DELIV_O_ID, row_d);
+      unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x);  // RMW of the cursor
+      const uint64_t nok = kO(w, d, (uint64_t)o);
+      const uint32_t row_no = probe(TNw, nok);
+      if (row_no == ROW_NONE) {
+        // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
+        unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+      } else {
+        for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x);  // DELETE
+        const uint32_t row_o = probe(TOr, nok);
+        if (row_o == ROW_NONE) {
+          internal_error(x);
+        } else {
+          unit_w<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x);
+          const uint32_t cid = (uint32_t)rd(TOr, O_C_ID, row_o);
+          const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
+          long long sum = 0;
+          for (uint32_t l = 1; l <= cnt; ++l) {
+            const uint32_t row_ol = probe(TOL_, nok * 16 + l);
+            if (row_ol == ROW_NONE) { internal_error(x); continue; }
+            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol, x);
+            sum += rd(TOL_, OL_AMOUNT, row_ol);
+            if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol, b.clock);
+          }
+          const uint32_t row_c = probe(TCu, kC(w, d, cid));
+          if (row_c == ROW_NONE) {
+            internal_error(x);
+          } else {
+            col_upd3<PH>(TCu, C_BALANCE, C_DELIVERY_CNT, C_DELIVERY_CNT, row_c, x);
+            if (PH == PH_WB) {
+              addv(TCu, C_BALANCE, row_c, sum);
+              addv(TCu, C_DELIVERY_CNT, row_c, 1);
+            }
+          }
+          if (PH == PH_WB) {
+            wr(TOr, O_CARRIER_ID, row_o, carrier);
+            TNw.valid[row_no] = 0;
+            IdxSlot* sl = idx_slot(TNw, nok);
+            if (sl) sl->row = ROW_NONE;
+            wr(TDi, D_NEXT_DELIV_O_ID, row_d, o + 1);
+          }
+          delivered = 1;
+          total = sum;
+        }
+      }
+    }
+  }
+  if (PH == PH_EXEC) {
+    delivered = seg16_sum(delivered);
+    total = seg16_sum(total);
+    if (active && sub == 0) {
+      long long* res = b.res + 4ull * r;
+      res[0] = delivered;
+      res[1] = total;
+      res[2] = 0;
+      res[3] = 0;
+    }
+  }
+}
+
+// ---- StockLevel (TPC-C 2.8): window [nx-20, nx), distinct items, one warp per txn -----------
+constexpr int SL_SLOTS = 20 * 15;
+template <int PH>
+__device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bool active, Tx& x,
+                                uint32_t* items) {
+  const DevTable& TDi = c_tabs[TD];
+  const DevTable& TOr = c_tabs[TO];
+  const DevTable& TOL_ = c_tabs[TOL];
+  const DevTable& TSt = c_tabs[TS];
+  if (!active || PH == PH_WB) return;  // warp-uniform (one txn per warp); read-only: no write-back
+  const uint8_t* p = b.params + 128ull * r;
+  const uint32_t w = p16(p, 0), d = p[2];
+  const long long thr = p[3];
+  const uint32_t row_d = probe(TDi, kD(w, d));
+  if (row_d == ROW_NONE) {
+    internal_error(x);
+    return;
+  }
+  const long long nx = rd(TDi, D_NEXT_O_ID, row_d);
+  if (lane == 0) unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+  for (uint32_t s = lane; s < SL_SLOTS; s += 32) items[s] = 0;
+  __syncwarp();
+  if (lane < 20) {
+    const long long o = nx - 20 + lane;
+    const uint32_t row_o = probe(TOr, kO(w, d, (uint64_t)o));
+    if (row_o == ROW_NONE) {
+      internal_error(x);
+    } else {
+      const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);  // static
+      for (uint32_t l = 0; l < cnt && l < 15; ++l) {
+        const uint32_t row_ol = probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1);
+        if (row_ol == ROW_NONE) { internal_error(x); continue; }
+        items[lane * 15 + l] = (uint32_t)rd(TOL_, OL_I_ID, row_ol);  // static
+      }
+    }
+  }
+  __syncwarp();
+  long long low = 0;
+  for (uint32_t s = lane; s < SL_SLOTS; s += 32) {
+    const uint32_t it = items[s];
+    if (!it) continue;
+    bool dup = false;
+    for (uint32_t s2 = 0; s2 < s && !dup; ++s2) dup = items[s2] == it;
+    if (dup) continue;  // count distinct items
+    const uint32_t row_s = probe(TSt, kS(w, it));
+    if (row_s == ROW_NONE) { internal_error(x); continue; }
+    if (PH == PH_EXEC) low += rd(TSt, S_QUANTITY, row_s) < thr;
+    unit_r<PH>(TSt, col_group(TSt, S_QUANTITY), row_s, x);
+  }
+  if (PH == PH_EXEC) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) low += __shfl_xor_sync(0xffffffffu, low, o);
+    if (lane == 0) {
+      long long* res = b.res + 4ull * r;
+      res[0] = low;
+      res[1] = nx;
+      res[2] = 0;
+      res[3] = 0;
+    }
+  }
+}
+
+// ---- the phase kernel: type-homogeneous warps over the per-type txn lists -------------------------
+
+template <int PH>
+__global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
+  if (*b.err) return;
+  __shared__ uint32_t sl_items[8][SL_SLOTS];
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  uint32_t cnt[NTYPES], pre[NTYPES + 1];
+  pre[0] = 0;
+#pragma unroll
+  for (int t = 0; t < NTYPES; ++t) {
+    cnt[t] = b.kcount[t];
+    const uint32_t per = 32 / (t == 1 ? 1 : (t == 4 ? 32 : 16));
+    pre[t + 1] = pre[t] + (cnt[t] + per - 1) / per;
+  }
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NTYPES]; w += nwarps) {
+    uint32_t t = 0, lw = w, ct = cnt[0];
+#pragma unroll
+    for (int tt = 1; tt < NTYPES; ++tt)
+      if (w >= pre[tt]) { t = tt; lw = w - pre[tt]; ct = cnt[tt]; }  // warp-uniform procedure type
+    const uint32_t L = t == 1 ? 1 : (t == 4 ? 32 : 16);
+    const uint32_t per = 32 / L;
+    const uint32_t k = lw * per + lane / L;
+    const uint32_t sub = lane % L;
+    const bool active = k < ct;
+    const uint32_t r = active ? tp.list[(uint64_t)t * tp.max_txns + k] : 0;
+    Tx x{r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), false, b.err};
+    bool go = active;
+    if (PH == PH_WB) go = active && b.status[r] == LTPG_ST_COMMIT;
+    switch (t) {
+      case 0: proc_neworder<PH>(b, tp, r, sub, go, x); break;
+      case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
+      case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
+      case 3: proc_delivery<PH>(b, r, sub, go, x); break;
+      default: proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib]); break;
+    }
+    if (PH == PH_DETECT) {  // per-txn OR over the txn's lanes, one status write per txn
+      const uint32_t bal = __ballot_sync(0xffffffffu, x.bad);
+      const uint32_t seg = L == 32 ? 0xffffffffu : (L == 1 ? (1u << lane) : (0xffffu << (lane & 16)));
+      if (active && sub == 0)
+        b.status[r] = (bal & seg) ? LTPG_ST_CONFLICT : (b.ua[r] ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+    }
+  }
+}
+
+// ---- K-tgroup: validation + per-type lists (warp-aggregated appends) ----------------------------
+__global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t t = 0xFF, lines = 0;
+  bool bad = false;
+  if (r < b.n_txns) {
+    if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;
+    t = b.ptype[r];
+    const uint8_t* p = b.params + 128ull * r;
+    const uint32_t W = tp.nw;
+    auto okw = [W](uint32_t w) { return w >= 1 && w <= W; };
+    auto okd = [](uint32_t d) { return d >= 1 && d <= 10; };
+    if (!okw(p16(p, 0))) bad = true;
+    switch (t) {
+      case 0: {
+        const uint32_t nl = p[3], c = p16(p, 4);
+        if (!okd(p[2]) || nl < 1 || nl > 15 || c < 1 || c > 3000) { bad = true; break; }
+        for (uint32_t l = 0; l < nl; ++l) {
+          const uint8_t* L = p + 8 + 8 * l;
+          const uint32_t i = p32(L, 0);
+          if (!okw(p16(L, 4)) || L[6] < 1 || L[6] > 10 || i < 1 || i > 100001) bad = true;
+          for (uint32_t m = 0; m < l; ++m)
+            if (p32(p + 8 + 8 * m, 0) == i) bad = true;  // R10: distinct items
+        }
+        lines = nl;
+        break;
+      }
+      case 1:
+        if (!okd(p[2]) || !okw(p16(p, 4)) || !okd(p[6]) || p[3] > 1) bad = true;
+        else if (p[3] ? p16(p, 10) > 999 : (p16(p, 8) < 1 || p16(p, 8) > 3000)) bad = true;
+        break;
+      case 2:
+        if (!okd(p[2]) || p[3] > 1) bad = true;
+        else if (p[3] ? p16(p, 6) > 999 : (p16(p, 4) < 1 || p16(p, 4) > 3000)) bad = true;
+        break;
+      case 3:
+        if (p[2] < 1 || p[2] > 10) bad = true;
+        break;
+      case 4:
+        if (!okd(p[2])) bad = true;
+        break;
+      default:
+        bad = true;
+    }
+    if (bad) atomicOr(b.err, ERR_EINVAL);
+  }
+  const uint32_t lsum = __reduce_add_sync(0xffffffffu, lines);
+  if (lane == 0 && lsum) atomicAdd(tp.misc + M_NO_LINES, lsum);
+#pragma unroll
+  for (uint32_t k = 0; k < NTYPES; ++k) {
+    const uint32_t m = __ballot_sync(0xffffffffu, t == k && !bad);
+    if (!m) continue;
+    uint32_t base = 0;
+    const uint32_t leader = __ffs(m) - 1;
+    if (lane == leader) base = atomicAdd(b.kcount + k, __popc(m));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (t == k && !bad) tp.list[(uint64_t)k * tp.max_txns + base + __popc(m & ((1u << lane) - 1))] = r;
+  }
+}
+
+// ECAPACITY before execution: worst case every NewOrder / Payment commits
+__global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
+  const uint64_t n_no = b.kcount[0], n_pay = b.kcount[1], lines = tp.misc[M_NO_LINES];
+  auto over = [](const DevTable& T, uint64_t add) { return *T.n_rows + add > T.capacity; };
+  if (over(c_tabs[TO], n_no) || over(c_tabs[TNO], n_no) || over(c_tabs[TOL], lines) || over(c_tabs[TH], n_pay))
+    atomicOr(b.err, ERR_ECAPACITY);
+}
+
+// ---- NewOrder o_id: fetch-ADD pre-image = snapshot D_NEXT_O_ID + #committed NewOrders of the
+//      same district with a smaller rank (P:241 prefix sum; R12) -------------------------------
+__global__ void k_no_prep(BatchDev b, TpccParams tp) {
+  if (*b.err) return;
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= b.n_txns) return;
+  const bool c = b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT;
+  const uint8_t* p = b.params + 128ull * r;
+  tp.no_flag[r] = c;
+  tp.no_lines[r] = c ? p[3] : 0;
+  tp.dk_of[r] = c ? (uint32_t)kD(p16(p, 0), p[2]) : ~0u;
+}
+
+__global__ void k_no_hist(BatchDev b, TpccParams tp) {
+  extern __shared__ uint32_t hist[];
+  if (*b.err) return;
+  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  const uint32_t r0 = blockIdx.x * NO_CHUNK;
+  for (uint32_t i = threadIdx.x; i < NO_CHUNK; i += blockDim.x) {
+    const uint32_t r = r0 + i;
+    if (r < b.n_txns) {
+      const uint32_t dk = tp.dk_of[r];
+      if (dk != ~0u) atomicAdd(hist + dk, 1u);
+    }
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i] = hist[i];
+}
+
+__global__ void k_no_colscan(BatchDev b, TpccParams tp) {
+  if (*b.err) return;
+  const uint32_t dk = blockIdx.x * blockDim.x + threadIdx.x;
+  if (dk >= tp.dsz) return;
+  uint32_t run = 0;
+  for (uint32_t ch = 0; ch < tp.n_chunks; ++ch) {
+    uint32_t* c = tp.chunk_cnt + (uint64_t)ch * tp.dsz + dk;
+    const uint32_t v = *c;
+    *c = run;
+    run += v;
+  }
+  if (!run) return;
+  const DevTable& TDi = c_tabs[TD];
+  const uint32_t row_d = probe(TDi, dk);
+  if (row_d == ROW_NONE) {
+    atomicOr(b.err, ERR_EINTERNAL);
+    return;
+  }
+  const long long base = rd(TDi, D_NEXT_O_ID, row_d);
+  tp.dist_base[dk] = base;
+  addv(TDi, D_NEXT_O_ID, row_d, run);  // final value: snapshot + committed NewOrders (delayed add)
+}
+
+__global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk, ranks in order
+  extern __shared__ uint32_t cntd[];
+  if (*b.err) return;
+  const uint32_t lane = threadIdx.x;
+  for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i];
+  __syncwarp();
+  const uint32_t r0 = blockIdx.x * NO_CHUNK;
+  for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {
+    const uint32_t r = r0 + it * 32 + lane;
+    const uint32_t dk = r < b.n_txns ? tp.dk_of[r] : ~0u;
+    const uint32_t m = __match_any_sync(0xffffffffu, dk);
+    if (dk != ~0u) {
+      const uint32_t before = __popc(m & ((1u << lane) - 1));
+      b.res[4ull * r] = tp.dist_base[dk] + cntd[dk] + before;
+    }
+    __syncwarp();
+    if (dk != ~0u && lane == (uint32_t)(__ffs(m) - 1)) cntd[dk] += __popc(m);
+    __syncwarp();
+  }
+}
+
+__global__ void k_tpcc_advance(BatchDev b, TpccParams tp) {
+  if (*b.err) return;
+  const uint32_t n = b.n_txns;
+  *c_tabs[TO].n_rows += tp.no_flag[n];
+  *c_tabs[TNO].n_rows += tp.no_flag[n];
+  *c_tabs[TOL].n_rows += tp.no_lines[n];
+  *c_tabs[TH].n_rows += tp.misc[M_HIST];
+}
+
+// ---- host side ------------------------------------------------------------------------------------
+template <class T>
+static cudaError_t dm(T** p, size_t n) {
+  return cudaMalloc(reinterpret_cast<void**>(p), std::max<size_t>(n, 1) * sizeof(T));
+}
+
+int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw) {
+  t.max_txns = max_txns;
+  t.nw = nw;
+  if (!nw) return 0;
+  if (nw > 1000) return LTPG_EINVAL;
+  t.dsz = nw * 10 + 11;
+  const uint64_t chunks = (max_txns + NO_CHUNK - 1) / NO_CHUNK;
+  if (dm(&t.by_name, (uint64_t)t.dsz * 1000) || dm(&t.list, (uint64_t)NTYPES * max_txns) ||
+      dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_flag, max_txns + 1ull) || dm(&t.no_lines, max_txns + 1ull) ||
+      dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
+    return LTPG_ENOMEM;
+  cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
+  return 0;
+}
+
+void tpcc_free(TpccDev& t) {
+  void* ps[] = {t.by_name, t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
+  for (void* p : ps)
+    if (p) cudaFree(p);
+  t = TpccDev{};
+}
+
+// Static secondary index ("primary and secondary hash tables"): (w, d, C_LAST) ->
+// the customer at position ceil(n/2) when sorted by C_FIRST (TPC-C 2.5.2.2); built at load.
+int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, uint64_t n, uint32_t nw) {
+  if (!t.by_name || !n) return 0;
+  std::map<uint64_t, std::vector<std::pair<int64_t, int64_t>>> g;
+  for (uint64_t r = 0; r < n; ++r) {
+    const uint64_t k = keys[r], dk = (k - 1) / 3000, c = (k - 1) % 3000 + 1;
+    const int64_t last = cols[C_LAST * n + r], first = cols[C_FIRST * n + r];
+    if (dk >= t.dsz || last < 0 || last > 999) continue;
+    g[dk * 1000 + (uint64_t)last].push_back({first, (int64_t)c});
+  }
+  std::vector<int> dense((uint64_t)t.dsz * 1000, 0);
+  for (auto& kv : g) {
+    auto& v = kv.second;
+    std::sort(v.begin(), v.end());
+    dense[kv.first] = (int)v[(v.size() + 1) / 2 - 1].second;
+  }
+  (void)nw;
+  return cudaMemcpy(t.by_name, dense.data(), dense.size() * sizeof(int), cudaMemcpyHostToDevice) == cudaSuccess
+             ? 0
+             : LTPG_ECUDA;
+}
+
+int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cudaEvent_t* ev) {
+  if (!t.nw) return LTPG_EINVAL;
+  const uint32_t n = b.n_txns;
+  TpccParams tp{t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
+                t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
+  cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
+  const uint32_t blocks = (n + 255) / 256;
+  k_tpcc_group<<<blocks, 256, 0, s>>>(b, tp);
+  k_tpcc_capacity<<<1, 1, 0, s>>>(b, tp);
+  note_launch(2);
+  if (ev) cudaEventRecord(ev[2], s);
+  // one warp-slot per txn lane group; grid-stride over the per-type warp ranges
+  const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
+  const uint32_t grid = (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
+  k_tpcc_phase<PH_EXEC><<<grid, 256, 0, s>>>(b, tp);
+  note_launch();
+  if (ev) cudaEventRecord(ev[3], s);
+  k_tpcc_phase<PH_DETECT><<<grid, 256, 0, s>>>(b, tp);
+  note_launch();
+  if (ev) cudaEventRecord(ev[4], s);
+  // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders
+  k_no_prep<<<blocks, 256, 0, s>>>(b, tp);
+  note_launch();
+  scan_exclusive_u32(t.no_flag, t.no_flag, n, scan_scratch, s);
+  scan_exclusive_u32(t.no_lines, t.no_lines, n, scan_scratch, s);
+  const size_t smem = (size_t)t.dsz * sizeof(uint32_t);
+  k_no_hist<<<tp.n_chunks, 256, smem, s>>>(b, tp);
+  k_no_colscan<<<(t.dsz + 255) / 256, 256, 0, s>>>(b, tp);
+  k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
+  note_launch(3);
+  if (ev) cudaEventRecord(ev[5], s);
+  k_tpcc_phase<PH_WB><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_advance<<<1, 1, 0, s>>>(b, tp);
+  note_launch(2);
+  return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
+}
+
 }  // namespace ltpg

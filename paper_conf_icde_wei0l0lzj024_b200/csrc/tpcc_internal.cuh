@@ -1,19 +1,61 @@
-// TPC-C PROC-mode scratch and launchers (stored procedures).
+// TPC-C PROC-mode scratch and launchers (pre-compiled stored procedures).
 #pragma once
 #include "ltpg_internal.cuh"
 
 namespace ltpg {
 
+constexpr int NTYPES = 5;
+constexpr int TLOG = 17;         // u32 row slots logged per txn by execute (NewOrder/Payment/OrderStatus)
+constexpr int NO_CHUNK = 1024;   // ranks per chunk of the o_id prefix computation
+
+// TPC-C schema (include/ltpg.h): table ids and column indices
+enum { TW = 0, TD = 1, TC = 2, TH = 3, TNO = 4, TO = 5, TOL = 6, TI = 7, TS = 8 };
+enum { W_TAX = 0, W_YTD = 1 };
+enum { D_TAX = 0, D_YTD = 1, D_NEXT_O_ID = 2, D_NEXT_DELIV_O_ID = 3 };
+enum { C_DISCOUNT = 0, C_CREDIT = 1, C_LAST = 2, C_FIRST = 3, C_INIT_O_ID = 4, C_BALANCE = 5,
+       C_YTD_PAYMENT = 6, C_PAYMENT_CNT = 7, C_DELIVERY_CNT = 8 };
+enum { H_C_ID = 0, H_C_D_ID, H_C_W_ID, H_D_ID, H_W_ID, H_DATE, H_AMOUNT, H_TID, H_SEQ };
+enum { NO_O_ID = 0 };
+enum { O_C_ID = 0, O_ENTRY_D = 1, O_OL_CNT = 2, O_ALL_LOCAL = 3, O_CARRIER_ID = 4 };
+enum { OL_I_ID = 0, OL_SUPPLY_W_ID = 1, OL_QUANTITY = 2, OL_AMOUNT = 3, OL_DELIVERY_D = 4 };
+enum { I_PRICE = 0, I_IM_ID = 1 };
+enum { S_QUANTITY = 0, S_YTD = 1, S_ORDER_CNT = 2, S_REMOTE_CNT = 3 };
+
+// counters in TpccDev::misc
+enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3 };
+
 struct TpccDev {
   uint32_t max_txns = 0;
-  int* by_name = nullptr;  // dense secondary index [(w*10+d)*1000 + last] -> c_id
-  uint32_t n_by_name = 0;
+  uint32_t nw = 0;              // n_warehouses (global)
+  uint32_t dsz = 0;             // district-key array size = nw*10 + 11
+  int* by_name = nullptr;       // dense secondary index [(w*10+d)*1000 + c_last] -> c_id (0: none)
+  uint32_t* list = nullptr;     // [NTYPES][max_txns] ranks, grouped by procedure type
+  uint32_t* log = nullptr;      // [max_txns][TLOG] rows found by execute
+  uint32_t* no_flag = nullptr;  // [max_txns+1] committed NewOrder -> exclusive scan (row offsets)
+  uint32_t* no_lines = nullptr; // [max_txns+1] committed NewOrder lines -> exclusive scan
+  uint32_t* dk_of = nullptr;    // [max_txns] district key of a committed NewOrder, else ~0
+  uint32_t* chunk_cnt = nullptr;// [chunks][dsz]
+  long long* dist_base = nullptr; // [dsz] snapshot D_NEXT_O_ID
+  uint32_t* misc = nullptr;     // counters (M_*)
 };
 
-int tpcc_alloc(TpccDev& t, uint32_t max_txns);
+struct TpccParams {
+  uint32_t* list;
+  uint32_t* log;
+  uint32_t* no_flag;
+  uint32_t* no_lines;
+  uint32_t* dk_of;
+  uint32_t* chunk_cnt;
+  long long* dist_base;
+  uint32_t* misc;
+  const int* by_name;
+  uint32_t nw, dsz, max_txns, n_chunks;
+};
+
+int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses);
 void tpcc_free(TpccDev& t);
-int tpcc_build_secondary(TpccDev& t, const DevTable* h_tab, const DevTable* d_tab, uint32_t n_warehouses);
-int tpcc_run(TpccDev& t, const DevTable* h_tab, const DevTable* d_tab, BatchDev& b, const ltpg_config& cfg,
-             cudaStream_t s, cudaEvent_t* ev);
+int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, uint64_t n_rows,
+                         uint32_t n_warehouses);
+int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cudaEvent_t* ev);
 
 }  // namespace ltpg

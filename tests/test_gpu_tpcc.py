@@ -1,0 +1,127 @@
+"""GPU parity, TPC-C PROC mode: the CUDA stored procedures through the C-ABI vs
+the CPU oracle -- status, 4 result slots per txn and every table's canonical
+dump, bit-exact; TPC-C consistency conditions on the GPU's own state."""
+import numpy as np
+import pytest
+
+import oracle
+from tests import tpcc_cc
+from workloads import tpcc
+from workloads.formats import ST_COMMIT, ST_CONFLICT, NEW_ORDER, PAYMENT, DELIVERY
+
+pytestmark = pytest.mark.gpu
+
+
+def L():
+    import paper_conf_icde_wei0l0lzj024_b200 as lib
+    return lib
+
+
+def pair(W, mode, mix, max_txns, batches, seed=5):
+    wl = tpcc.TpccWorkload(W, seed=seed, mode=mode, mix=mix)
+    tables = wl.initial_tables()
+    g = L().tpcc_database(wl, max_txns=max_txns, tables=tables, append_batches=batches + 1)
+    o = oracle.tpcc_db(wl, tables)
+    return wl, g, o
+
+
+def compare(g, o, batch, clock):
+    rc, ost, ores = o.run_tpcc(batch, clock)
+    assert rc == 0
+    out = g.run_tpcc(batch, clock)
+    bad = np.nonzero(out["status"] != ost)[0]
+    assert len(bad) == 0, ("status", bad[:10], batch["type"][bad[:10]], out["status"][bad[:10]], ost[bad[:10]])
+    diff = np.nonzero((out["reads"] != ores).any(axis=1))[0]
+    assert len(diff) == 0, ("results", diff[:5], batch["type"][diff[:5]], out["reads"][diff[:5]], ores[diff[:5]])
+    assert (out["abort_idx"] == np.nonzero(ost == ST_CONFLICT)[0]).all()
+    return ost
+
+
+def compare_tables(g, o):
+    dumps = {}
+    for t in range(9):
+        gk, gc = g.dump_table(t)
+        ok, oc = o.dump_table(t)
+        assert gc.shape == oc.shape, (t, gc.shape, oc.shape)
+        if ok is not None:
+            assert (gk == ok).all(), t
+        assert (gc == oc).all(), (t, np.nonzero((gc != oc).any(axis=0))[0][:5])
+        dumps[t] = (gk, gc)
+    return dumps
+
+
+@pytest.mark.parametrize("mode", ["strict", "delayed"])
+@pytest.mark.parametrize("W", [1, 2])
+def test_full_mix_closed_loop(W, mode):
+    B = 3000
+    wl, g, o = pair(W, mode, tpcc.MIX_FULL, B, 6)
+    pending = None
+    tid = 1
+    for bno in range(5):
+        fresh = wl.batch(B - (0 if pending is None else len(pending["tid"])), tid, bno)
+        tid += len(fresh["tid"])
+        batch = fresh if pending is None else {k: np.concatenate([pending[k], fresh[k]]) for k in fresh}
+        st = compare(g, o, batch, 2 + bno)
+        ab = np.nonzero(st == ST_CONFLICT)[0]
+        pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
+    dumps = compare_tables(g, o)
+    cc = tpcc_cc.check(dumps)
+    assert all(cc.values()), cc
+
+
+@pytest.mark.parametrize("mode", ["strict", "delayed"])
+def test_c2_one_warehouse_16k(mode):
+    """BASELINE configs[1]: TPC-C 1 warehouse, NewOrder+Payment, batch 16k."""
+    wl, g, o = pair(1, mode, tpcc.MIX_NO_PAY, 16384, 3, seed=0x17C1)
+    tid = 1
+    for bno in range(2):
+        batch = wl.batch(16384, tid, bno)
+        tid += 16384
+        st = compare(g, o, batch, 2 + bno)
+        if mode == "strict":
+            assert ((batch["type"] == PAYMENT) & (st == ST_COMMIT)).sum() == 1  # Table VI-style: 1 per warehouse
+    compare_tables(g, o)
+
+
+def test_table6_gpu():
+    """Table VI "no" row 8/16,384 reproduced by the GPU path (== oracle)."""
+    wl, g, o = pair(8, "strict", tpcc.MIX_NO_PAY, 16384, 1, seed=0x17C0 + 8)
+    batch = wl.batch(16384, 1, 0)
+    st = compare(g, o, batch, 2)
+    no = batch["type"] == NEW_ORDER
+    rate = 100.0 * (no & (st == ST_COMMIT)).sum() / no.sum()
+    assert ((batch["type"] == PAYMENT) & (st == ST_COMMIT)).sum() == 8
+    assert abs(rate - 63.4) <= 2.0
+
+
+def test_tpcc_validation_and_capacity():
+    lib = L()
+    wl = tpcc.TpccWorkload(1, seed=3, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=512, tables=tables, append_batches=1)
+    b = wl.batch(100, 1, 0)
+    b["params"][5, 0] = 9  # warehouse 9 does not exist
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(b, 2)
+    assert e.value.rc == lib.LTPG_EINVAL
+    # capacity: append region sized for one batch of 512; two full batches of NewOrders overflow
+    o = oracle.tpcc_db(wl, tables)
+    nb = wl.batch(512, 1000, 1, types=[NEW_ORDER] * 512)
+    compare(g, o, nb, 3)
+    nb2 = wl.batch(512, 5000, 2, types=[NEW_ORDER] * 512)
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(nb2, 4)
+    assert e.value.rc == lib.LTPG_ECAPACITY
+    compare_tables(g, o)  # nothing changed by the rejected batch
+
+
+def test_delivery_heavy():
+    """Delivery drains NEW_ORDER queues across batches (cursor, delete, carrier, OL dates, balance)."""
+    wl, g, o = pair(1, "strict", (0.3, 0.0, 0.0, 0.7, 0.0), 256, 12)
+    tid = 1
+    for bno in range(10):
+        batch = wl.batch(200, tid, bno)
+        tid += 200
+        compare(g, o, batch, 2 + bno)
+    dumps = compare_tables(g, o)
+    assert all(tpcc_cc.check(dumps).values())

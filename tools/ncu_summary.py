@@ -37,7 +37,7 @@ def parse_launches(path):
             continue
         v = float(r[vi].replace(",", ""))
         unit = r[ui]
-        ns = v * {"nsecond": 1, "usecond": 1e3, "msecond": 1e6, "second": 1e9}.get(unit, 1)
+        ns = v * TIME_UNITS.get(unit, 1.0)
         name = r[ki].split("(")[0]
         a = agg.setdefault(name, {"launches": 0, "total_ns": 0.0})
         a["launches"] += 1
@@ -49,7 +49,11 @@ def parse_launches(path):
     return dict(sorted(agg.items(), key=lambda kv: -kv[1]["total_ns"])), tot
 
 
-WANT = ["dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__time_duration.sum",
+BYTE_UNITS = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+TIME_UNITS = {"ns": 1.0, "nsecond": 1.0, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6, "s": 1e9, "second": 1e9}
+
+WANT = ["lts__t_sectors.sum", "lts__t_sectors_srcunit_ltcfabric.sum", "dram__sectors_read.sum",
+        "dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__time_duration.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
         "lts__t_bytes.sum", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
         "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
@@ -74,10 +78,9 @@ def parse_full(rep):
                 except ValueError:
                     continue
                 u = units[i]
-                if u in ("Kbyte", "Mbyte", "Gbyte", "byte"):
-                    v *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]
-                if u in ("usecond", "msecond", "nsecond"):
-                    v *= {"nsecond": 1, "usecond": 1e3, "msecond": 1e6}[u]
+                v *= BYTE_UNITS.get(u, 1.0) * TIME_UNITS.get(u, 1.0)
+                if u == "sector":
+                    d[m + ".bytes"] = v * 32
                 d[m] = v
         if "dram__bytes_read.sum" in d:
             d["dram_bytes"] = d["dram__bytes_read.sum"] + d.get("dram__bytes_write.sum", 0.0)
@@ -118,7 +121,7 @@ def main():
                 k, v.get("dram_bytes", float("nan")), v.get("gpu__time_duration.sum", 0) / 1e3,
                 v.get("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
                       v.get("dram__throughput.avg.pct_of_peak_sustained_elapsed", "?")),
-                v.get("lts__t_bytes.sum", float("nan"))))
+                v.get("lts__t_sectors.sum", float("nan")) * 32))
     open(os.path.splitext(a.out)[0] + ".md", "w").write("\n".join(md) + "\n")
     print("\n".join(md))
 
