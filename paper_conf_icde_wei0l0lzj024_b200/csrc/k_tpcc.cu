@@ -63,16 +63,16 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 template <int PH>
 __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
   if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter);
-  if (PH == PH_DETECT) x.bad |= unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
   if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter);
-  if (PH == PH_DETECT) x.bad |= unit_conflicts(T, g, row, CHK_A, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_A, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
-  if (PH == PH_DETECT && g != LTPG_STATIC) x.bad |= unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.bad && g != LTPG_STATIC) x.bad = unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
 }
 // update of column c (strict: WRITE unit of its group; delayed: ADD unit)
 template <int PH>
@@ -385,8 +385,10 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
       const long long o = rd(TDi, D_NEXT_DELIV_O_ID, row_d);
       unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x);  // RMW of the cursor
       const uint64_t nok = kO(w, d, (uint64_t)o);
-      const uint32_t row_no = probe(TNw, nok);
-      if (row_no == ROW_NONE) {
+      const uint32_t row_no = (PH == PH_DETECT && x.bad) ? ROW_NONE : probe(TNw, nok);
+      if (PH == PH_DETECT && x.bad) {
+        // conflict already found: the remaining checks cannot change the verdict
+      } else if (row_no == ROW_NONE) {
         // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
         unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
       } else {
@@ -443,10 +445,13 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
 }
 
 // ---- StockLevel (TPC-C 2.8): window [nx-20, nx), distinct items, one warp per txn -----------
+// Distinct items are found with a per-warp open-addressing set in shared memory (the
+// first inserter of an item handles it); the result is order-independent.
 constexpr int SL_SLOTS = 20 * 15;
+constexpr int SL_HASH = 512;
 template <int PH>
 __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bool active, Tx& x,
-                                uint32_t* items) {
+                                uint32_t* items, uint32_t* set) {
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TOr = c_tabs[TO];
   const DevTable& TOL_ = c_tabs[TOL];
@@ -462,7 +467,9 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
   }
   const long long nx = rd(TDi, D_NEXT_O_ID, row_d);
   if (lane == 0) unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+  if (PH == PH_DETECT && __shfl_sync(0xffffffffu, (uint32_t)x.bad, 0)) return;  // RAW on D_NEXT_O_ID: done
   for (uint32_t s = lane; s < SL_SLOTS; s += 32) items[s] = 0;
+  for (uint32_t s = lane; s < SL_HASH; s += 32) set[s] = 0;
   __syncwarp();
   if (lane < 20) {
     const long long o = nx - 20 + lane;
@@ -471,21 +478,32 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
       internal_error(x);
     } else {
       const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);  // static
-      for (uint32_t l = 0; l < cnt && l < 15; ++l) {
-        const uint32_t row_ol = probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1);
-        if (row_ol == ROW_NONE) { internal_error(x); continue; }
-        items[lane * 15 + l] = (uint32_t)rd(TOL_, OL_I_ID, row_ol);  // static
-      }
+      uint32_t row_ol[15];
+#pragma unroll
+      for (uint32_t l = 0; l < 15; ++l)  // independent probes issued back to back
+        row_ol[l] = l < cnt ? probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1) : ROW_NONE;
+#pragma unroll
+      for (uint32_t l = 0; l < 15; ++l)
+        if (l < cnt) {
+          if (row_ol[l] == ROW_NONE) internal_error(x);
+          else items[lane * 15 + l] = (uint32_t)rd(TOL_, OL_I_ID, row_ol[l]);  // static
+        }
     }
   }
   __syncwarp();
   long long low = 0;
-  for (uint32_t s = lane; s < SL_SLOTS; s += 32) {
+  for (uint32_t s = lane; s < SL_SLOTS && !(PH == PH_DETECT && x.bad); s += 32) {
     const uint32_t it = items[s];
     if (!it) continue;
-    bool dup = false;
-    for (uint32_t s2 = 0; s2 < s && !dup; ++s2) dup = items[s2] == it;
-    if (dup) continue;  // count distinct items
+    uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
+    bool first = false;
+    for (;;) {
+      const uint32_t old = atomicCAS(set + h, 0u, it);
+      if (old == 0u) { first = true; break; }
+      if (old == it) break;
+      h = (h + 1) & (SL_HASH - 1);
+    }
+    if (!first) continue;  // count distinct items
     const uint32_t row_s = probe(TSt, kS(w, it));
     if (row_s == ROW_NONE) { internal_error(x); continue; }
     if (PH == PH_EXEC) low += rd(TSt, S_QUANTITY, row_s) < thr;
@@ -510,6 +528,7 @@ template <int PH>
 __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   __shared__ uint32_t sl_items[8][SL_SLOTS];
+  __shared__ uint32_t sl_set[8][SL_HASH];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   uint32_t cnt[NTYPES], pre[NTYPES + 1];
   pre[0] = 0;
@@ -539,7 +558,7 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
       case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
       case 3: proc_delivery<PH>(b, r, sub, go, x); break;
-      default: proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib]); break;
+      default: proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib], sl_set[wib]); break;
     }
     if (PH == PH_DETECT) {  // per-txn OR over the txn's lanes, one status write per txn
       const uint32_t bal = __ballot_sync(0xffffffffu, x.bad);
@@ -649,18 +668,26 @@ __global__ void k_no_hist(BatchDev b, TpccParams tp) {
   for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i] = hist[i];
 }
 
-__global__ void k_no_colscan(BatchDev b, TpccParams tp) {
+__global__ void k_no_colscan(BatchDev b, TpccParams tp) {  // one warp per district key
   if (*b.err) return;
-  const uint32_t dk = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t dk = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
   uint32_t run = 0;
-  for (uint32_t ch = 0; ch < tp.n_chunks; ++ch) {
+  for (uint32_t ch0 = 0; ch0 < tp.n_chunks; ch0 += 32) {
+    const uint32_t ch = ch0 + lane;
     uint32_t* c = tp.chunk_cnt + (uint64_t)ch * tp.dsz + dk;
-    const uint32_t v = *c;
-    *c = run;
-    run += v;
+    const uint32_t v = ch < tp.n_chunks ? *c : 0;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (ch < tp.n_chunks) *c = run + x - v;  // exclusive prefix over chunks
+    run += __shfl_sync(0xffffffffu, x, 31);
   }
-  if (!run) return;
+  if (!run || lane) return;
   const DevTable& TDi = c_tabs[TD];
   const uint32_t row_d = probe(TDi, dk);
   if (row_d == ROW_NONE) {
@@ -780,7 +807,7 @@ int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cu
   scan_exclusive_u32(t.no_lines, t.no_lines, n, scan_scratch, s);
   const size_t smem = (size_t)t.dsz * sizeof(uint32_t);
   k_no_hist<<<tp.n_chunks, 256, smem, s>>>(b, tp);
-  k_no_colscan<<<(t.dsz + 255) / 256, 256, 0, s>>>(b, tp);
+  k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
   if (ev) cudaEventRecord(ev[5], s);
