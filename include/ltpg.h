@@ -135,8 +135,19 @@ typedef struct {
   uint32_t max_ops;             /* OPS mode per-batch op capacity                         */
   uint32_t flags;               /* LTPG_FLAG_*                                           */
   uint32_t n_tables;            /* number of table ids used (<= 16)                      */
-  uint32_t n_warehouses;        /* PROC mode: global TPC-C W (validation, routing)       */
+  uint32_t n_warehouses;        /* PROC mode: global TPC-C W (validation, routing; <= 1000) */
+  uint64_t key_space;           /* OPS mode: keys [0, key_space) split into contiguous
+                                   ranges over partitions (tables with owner_rule 2)      */
 } ltpg_config;
+
+/* Multi-GPU: world > 1 ranks each own a contiguous range of warehouses
+ * (TPC-C, owner_rule 1) or of keys (OPS, owner_rule 2).  Every rank calls ltpg_run_batch
+ * with the same global batch; each executes, marks and checks only the units it owns,
+ * then the per-txn verdicts are exchanged (one ncclAllReduce(MAX) of a byte per txn over
+ * NVLink) before write-back, so commit_bits / status / abort_idx are identical on all
+ * ranks.  Result slots are filled by the owning rank and summed over ranks
+ * (ncclAllReduce(SUM)).  LTPG_FLAG_LOOPBACK_SHIFT runs P logical partitions inside one
+ * process on one GPU with the same ownership, exchange and result-sum logic. */
 
 typedef struct ltpg_db ltpg_db;  /* opaque, library-owned device state */
 

@@ -42,7 +42,7 @@ c_u32, c_u64, c_i64, c_int, c_vp = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_in
 class ltpg_config(ctypes.Structure):
     _fields_ = [("device", c_int), ("rank", c_int), ("world", c_int), ("nccl_unique_id", c_vp),
                 ("max_txns", c_u32), ("max_ops", c_u32), ("flags", c_u32), ("n_tables", c_u32),
-                ("n_warehouses", c_u32)]
+                ("n_warehouses", c_u32), ("key_space", c_u64)]
 
 
 class ltpg_table_desc(ctypes.Structure):
@@ -121,10 +121,12 @@ class Database:
     """One device database (tables + PK indexes + conflict marks) on one GPU."""
 
     def __init__(self, n_tables, max_txns, max_ops=0, device=0, flags=0, n_warehouses=0, rank=0, world=1,
-                 nccl_unique_id=None):
+                 nccl_unique_id=None, key_space=0, loopback=1):
         self._keep = []
+        flags |= (int(loopback) & 0xF) << LTPG_FLAG_LOOPBACK_SHIFT if loopback > 1 else 0
         cfg = ltpg_config(device=device, rank=rank, world=world, nccl_unique_id=None, max_txns=max_txns,
-                          max_ops=max_ops, flags=flags, n_tables=n_tables, n_warehouses=n_warehouses)
+                          max_ops=max_ops, flags=flags, n_tables=n_tables, n_warehouses=n_warehouses,
+                          key_space=key_space)
         if nccl_unique_id is not None:
             buf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
             self._keep.append(buf)
@@ -249,26 +251,74 @@ class Database:
         return (keys[:n] if self.has_pk[t] else None), cols
 
 
-def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0):
-    db = Database(1, max_txns, max_ops, device=device, flags=flags)
+def part_of_w(w, nw, nparts):
+    """Owning partition of warehouse w (contiguous ranges; mirrors csrc part_of_w)."""
+    return 0 if nparts <= 1 else ((np.asarray(w, dtype=np.int64) - 1) * nparts) // nw
+
+
+def part_of_key(key, key_space, nparts):
+    """Owning partition of a key of an owner_rule-2 table (mirrors csrc part_of_key)."""
+    if nparts <= 1:
+        return np.zeros_like(np.asarray(key, dtype=np.uint64), dtype=np.int64)
+    chunk = (int(key_space) + nparts - 1) // nparts
+    return np.minimum(np.asarray(key, dtype=np.uint64) // np.uint64(chunk), nparts - 1).astype(np.int64)
+
+
+def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0, loopback=1, rank=0, world=1,
+                  nccl_unique_id=None):
+    """YCSB usertable, key-range partitioned (owner_rule 2) when world * loopback > 1; a
+    multi-rank db loads only its own key range."""
+    db = Database(1, max_txns, max_ops, device=device, flags=flags, key_space=workload.n_rows, loopback=loopback,
+                  rank=rank, world=world, nccl_unique_id=nccl_unique_id)
     g, a, ng, pk = workload.table_desc()
     keys, cols = workload.initial_table()
-    db.load_table(0, g, a, ng, keys, cols, capacity=capacity or len(keys), has_pk=pk)
+    if world > 1:
+        own = part_of_key(keys, workload.n_rows, world) == rank
+        keys, cols = keys[own], cols[:, own]
+    db.load_table(0, g, a, ng, keys, cols, capacity=capacity or max(len(keys), 1), has_pk=pk, owner_rule=2)
     return db
 
 
-def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None):
-    """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns."""
-    from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
-    db = Database(9, max_txns, 0, device=device, flags=flags, n_warehouses=workload.W)
+def tpcc_owner_w(t, keys, cols):
+    """Warehouse that owns each row of TPC-C table t (None: replicated ITEM)."""
+    from workloads.formats import (T_WAREHOUSE, T_DISTRICT, T_CUSTOMER, T_HISTORY, T_NEW_ORDER, T_ORDER,
+                                   T_ORDER_LINE, T_STOCK)
+    if t == T_WAREHOUSE:
+        return keys.astype(np.int64)
+    if t == T_DISTRICT:
+        return (keys.astype(np.int64) - 1) // 10
+    if t == T_CUSTOMER:
+        return ((keys.astype(np.int64) - 1) // 3000 - 1) // 10
+    if t == T_HISTORY:
+        return cols[2].astype(np.int64)  # H_C_W_ID: the customer's owner keeps the row
+    if t in (T_NEW_ORDER, T_ORDER):
+        return ((keys >> np.uint64(32)).astype(np.int64) - 1) // 10
+    if t == T_ORDER_LINE:
+        return (((keys >> np.uint64(4)) >> np.uint64(32)).astype(np.int64) - 1) // 10
+    if t == T_STOCK:
+        return (keys.astype(np.int64) - 1) // 100000
+    return None
+
+
+def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None,
+                  loopback=1, rank=0, world=1, nccl_unique_id=None):
+    """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns.
+    A multi-rank db (world > 1) loads only the rows of its warehouses (ITEM replicated)."""
+    from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY, T_ITEM
+    db = Database(9, max_txns, 0, device=device, flags=flags, n_warehouses=workload.W, loopback=loopback,
+                  rank=rank, world=world, nccl_unique_id=nccl_unique_id)
     tables = tables if tables is not None else workload.initial_tables()
     extra = {T_ORDER: 1, T_NEW_ORDER: 1, T_ORDER_LINE: 15, T_HISTORY: 1}
     for t, (g, a, ng, pk) in workload.table_descs().items():
         k, c = tables[t]
+        if world > 1 and t != T_ITEM:
+            own = part_of_w(tpcc_owner_w(t, k, c), workload.W, world) == rank
+            k = None if k is None else k[own]
+            c = c[:, own]
         n = c.shape[1]
         cap = n + extra.get(t, 0) * max_txns * append_batches
         if capacity and t in capacity:
             cap = capacity[t]
         db.load_table(t, g, a, ng, k, c, capacity=max(cap, 1), has_pk=pk,
-                      owner_rule=0)
+                      owner_rule=0 if t == T_ITEM else 1)
     return db

@@ -1,14 +1,17 @@
 // C-ABI implementation (include/ltpg.h): device store management and the
 // per-batch driver.  One ltpg_run_batch enqueues, on the caller's stream:
-//   upload -> K-group -> [scan] -> K-claim -> K-exec -> K-detect -> [exchange]
-//   -> K-wb -> finalize (commit bits, abort list) -> download
+//   upload -> [per partition: K-group -> K-claim -> K-exec -> K-detect]
+//   -> exchange (partitioned only: loopback max / ncclAllReduce MAX)
+//   -> [per partition: K-wb] -> finalize (commit bits, abort list) -> download
 // The paper separates its three kernels with cudaDeviceSynchronize() (P:122,
 // P:137-141); here stream order gives the same global isolation with no host
-// round-trip inside the batch.
+// round trip inside the batch.
+#include <dlfcn.h>
+#include <nccl.h>
+
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
-#include <numeric>
 #include <string>
 #include <vector>
 
@@ -16,6 +19,49 @@
 #include "tpcc_internal.cuh"
 
 using namespace ltpg;
+
+namespace {
+
+// ---- NCCL, loaded lazily (only multi-rank dbs need it) -------------------------------------
+struct Nccl {
+  void* h = nullptr;
+  ncclResult_t (*commInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+  const char* (*getErrorString)(ncclResult_t) = nullptr;
+  bool load() {
+    if (h) return true;
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* n : names)
+      if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+    if (!h) return false;
+    commInitRank = reinterpret_cast<decltype(commInitRank)>(dlsym(h, "ncclCommInitRank"));
+    allReduce = reinterpret_cast<decltype(allReduce)>(dlsym(h, "ncclAllReduce"));
+    commDestroy = reinterpret_cast<decltype(commDestroy)>(dlsym(h, "ncclCommDestroy"));
+    getErrorString = reinterpret_cast<decltype(getErrorString)>(dlsym(h, "ncclGetErrorString"));
+    return commInitRank && allReduce && commDestroy && getErrorString;
+  }
+};
+Nccl g_nccl;
+
+uint64_t g_tab_versions = 0;     // process-wide: every table load gets a new version
+uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __constant__
+
+// per-partition scratch (one per logical partition handled by this process)
+struct Part {
+  long long* res = nullptr;
+  unsigned long long* uref = nullptr;
+  unsigned long long* items = nullptr;
+  uint32_t* txn_ins = nullptr;
+  uint8_t* ua = nullptr;
+  uint8_t* lflag = nullptr;
+  uint32_t* small = nullptr;             // [0] err [1] ins_tables [2..7] kcount
+  unsigned long long* base = nullptr;    // [MAXT]
+  TpccDev tpcc;
+};
+
+}  // namespace
 
 struct ltpg_db {
   ltpg_config cfg{};
@@ -25,37 +71,36 @@ struct ltpg_db {
   uint32_t epoch = 0;
   uint32_t n_tables = 0;
   uint64_t tab_version = 0;
+  uint32_t nparts = 1;     // global logical partitions = world * loopback
+  uint32_t loopback = 1;   // partitions handled by this process
   DevTable h_tab[MAXT]{};
   DevTable* d_tab = nullptr;
-  unsigned long long* d_nrows = nullptr;  // [MAXT]
-  // per-batch buffers
+  unsigned long long* d_nrows = nullptr;   // [MAXT]
+  unsigned long long* d_reserve = nullptr; // [MAXT]
+  std::vector<Part> parts;
+  // shared per-batch buffers
   unsigned long long* d_tid = nullptr;
   uint32_t* d_op_begin = nullptr;
   ltpg_op* d_ops = nullptr;
   long long* d_args = nullptr;
   uint8_t* d_ptype = nullptr;
   uint8_t* d_params = nullptr;
-  long long* d_res = nullptr;
-  unsigned long long* d_uref = nullptr;
-  unsigned long long* d_items = nullptr;
-  uint32_t* d_txn_ins = nullptr;
-  uint8_t* d_ua = nullptr;
+  long long* d_res = nullptr;              // combined results
   uint8_t* d_status = nullptr;
+  uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
+  void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_bits = nullptr;
   uint32_t* d_flags = nullptr;
   uint32_t* d_offs = nullptr;
   uint32_t* d_abort = nullptr;
-  uint32_t* d_small = nullptr;  // [0]=err [1]=ins_tables [2..7] kcount [8..10] counts
+  uint32_t* d_small = nullptr;             // [0] err (combined) [8..10] counts
   uint32_t* d_scan = nullptr;
-  uint32_t* h_small = nullptr;  // pinned mirror of d_small (+ n_aborted)
-  TpccDev tpcc{};
+  uint32_t* h_small = nullptr;             // pinned
+  ncclComm_t comm = nullptr;
   cudaEvent_t ev[8]{};
 };
 
 namespace {
-
-uint64_t g_tab_versions = 0;     // process-wide: every table load gets a new version
-uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __constant__
 
 int fail(ltpg_db* db, int code, const std::string& msg) {
   if (db) {
@@ -79,7 +124,7 @@ cudaError_t dmalloc(T** p, size_t n) {
 }
 
 void free_table(DevTable& T) {
-  if (T.col[0]) cudaFree(T.col[0]);
+  if (T.col0) cudaFree(T.col0);
   if (T.valid) cudaFree(T.valid);
   if (T.rowkey) cudaFree(T.rowkey);
   if (T.marks) cudaFree(T.marks);
@@ -89,30 +134,80 @@ void free_table(DevTable& T) {
   T.n_rows = nr;
 }
 
+// ---- exchange / combine kernels ------------------------------------------------------------
+// loopback: verdict = max over partitions of (conflict*2 | user_abort); the OR of all
+// partitions' errors is written back to every partition so that none writes back
+__global__ void k_combine(void* const* lflags, uint32_t np, uint32_t n, uint8_t* status, void* const* errs,
+                          uint32_t* err_all) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r == 0) {
+    uint32_t e = 0;
+    for (uint32_t p = 0; p < np; ++p) e |= *static_cast<const uint32_t*>(errs[p]);
+    *err_all = e;
+  }
+  if (r >= n) return;
+  uint8_t f = 0;
+  for (uint32_t p = 0; p < np; ++p) f = max(f, static_cast<const uint8_t*>(lflags[p])[r]);
+  status[r] = status_of_flag(f);
+}
+__global__ void k_spread_err(const uint32_t* err_all, void* const* errs, uint32_t np) {
+  for (uint32_t p = 0; p < np; ++p) *static_cast<uint32_t*>(errs[p]) = *err_all;
+}
+// NCCL: pack (flags, error bits as bytes) -> allreduce MAX -> unpack
+__global__ void k_pack(const uint8_t* lflag, const uint32_t* err, uint8_t* x, uint32_t n) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < n) x[r] = lflag[r];
+  if (r < 3) x[n + r] = (*err >> r) & 1u;
+}
+__global__ void k_unpack(const uint8_t* x, uint32_t n, uint8_t* status, uint32_t* err, uint32_t* err_all) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < n) status[r] = status_of_flag(x[r]);
+  if (r == 0) {
+    const uint32_t e = (uint32_t)x[n] | (uint32_t)x[n + 1] << 1 | (uint32_t)x[n + 2] << 2;
+    *err = e;
+    *err_all = e;
+  }
+}
+__global__ void k_sum_res(void* const* res, uint32_t np, uint64_t n, long long* out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    unsigned long long s = 0;
+    for (uint32_t p = 0; p < np; ++p) s += (unsigned long long)static_cast<const long long*>(res[p])[i];
+    out[i] = (long long)s;
+  }
+}
+__global__ void k_copy_err(const uint32_t* src, uint32_t* dst) { *dst = *src; }
+
 }  // namespace
 
 extern "C" {
 
-const char* ltpg_version(void) { return "ltpg-b200 0.1 sm_100a"; }
+const char* ltpg_version(void) { return "ltpg-b200 0.2 sm_100a"; }
 
 const char* ltpg_last_error(const ltpg_db* db) { return db ? db->last_error.c_str() : "null db"; }
 
 int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   ltpg_db* db = nullptr;
   if (!cfg || !out) return LTPG_EINVAL;
+  const uint32_t loop = std::max<uint32_t>(1, (cfg->flags >> LTPG_FLAG_LOOPBACK_SHIFT) & 0xF);
   if (cfg->n_tables == 0 || cfg->n_tables > MAXT || cfg->max_txns == 0 || cfg->world < 1 ||
-      cfg->rank < 0 || cfg->rank >= cfg->world || cfg->max_txns > (1u << 24) || cfg->max_ops > (1u << 24))
+      cfg->rank < 0 || cfg->rank >= cfg->world || cfg->max_txns > (1u << 24) || cfg->max_ops > (1u << 24) ||
+      cfg->n_warehouses > 1000 || (cfg->world > 1 && !cfg->nccl_unique_id) || cfg->world * loop > 64 ||
+      (cfg->world > 1 && loop > 1))
     return LTPG_EINVAL;
   db = new ltpg_db();
   db->cfg = *cfg;
   db->device = cfg->device;
   db->n_tables = cfg->n_tables;
+  db->loopback = loop;
+  db->nparts = (uint32_t)cfg->world * loop;
   *out = db;
   CK(cudaSetDevice(cfg->device));
   const size_t n = cfg->max_txns, m = std::max<uint32_t>(cfg->max_ops, 1);
+  const size_t nres = std::max(m, n * LTPG_PROC_RESULTS);
   CK(dmalloc(&db->d_tab, MAXT));
   CK(dmalloc(&db->d_nrows, MAXT));
   CK(cudaMemset(db->d_nrows, 0, MAXT * sizeof(unsigned long long)));
+  CK(dmalloc(&db->d_reserve, MAXT));
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
   CK(dmalloc(&db->d_tid, n));
   CK(dmalloc(&db->d_op_begin, n + 1));
@@ -120,12 +215,10 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_args, m));
   CK(dmalloc(&db->d_ptype, n));
   CK(dmalloc(&db->d_params, n * LTPG_PARAM_BYTES));
-  CK(dmalloc(&db->d_res, std::max(m, n * LTPG_PROC_RESULTS)));
-  CK(dmalloc(&db->d_uref, m));
-  CK(dmalloc(&db->d_items, m * NKINDS));
-  CK(dmalloc(&db->d_txn_ins, n + 1));
-  CK(dmalloc(&db->d_ua, n));
+  CK(dmalloc(&db->d_res, nres));
   CK(dmalloc(&db->d_status, n));
+  CK(dmalloc(&db->d_xchg, n + 4));
+  CK(dmalloc(&db->d_ptrs, 3 * 64));
   CK(dmalloc(&db->d_bits, (n + 31) / 32 + 1));
   CK(dmalloc(&db->d_flags, n));
   CK(dmalloc(&db->d_offs, n + 1));
@@ -135,8 +228,32 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaMallocHost(reinterpret_cast<void**>(&db->h_small), 64 * sizeof(uint32_t)));
   for (auto& e : db->ev) CK(cudaEventCreate(&e));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
-  int rc = tpcc_alloc(db->tpcc, cfg->max_txns, cfg->n_warehouses);
-  if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
+  db->parts.resize(loop);
+  std::vector<void*> ptrs(3 * 64, nullptr);
+  for (uint32_t p = 0; p < loop; ++p) {
+    Part& P = db->parts[p];
+    CK(dmalloc(&P.res, nres));
+    CK(dmalloc(&P.uref, m));
+    CK(dmalloc(&P.items, m * NKINDS));
+    CK(dmalloc(&P.txn_ins, n + 1));
+    CK(dmalloc(&P.ua, n));
+    CK(dmalloc(&P.lflag, n));
+    CK(dmalloc(&P.small, 64));
+    CK(dmalloc(&P.base, MAXT));
+    int rc = tpcc_alloc(P.tpcc, cfg->max_txns, cfg->n_warehouses, p ? db->parts[0].tpcc.by_name : nullptr);
+    if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
+    ptrs[p] = P.lflag;
+    ptrs[64 + p] = P.small;
+    ptrs[128 + p] = P.res;
+  }
+  CK(cudaMemcpy(db->d_ptrs, ptrs.data(), ptrs.size() * sizeof(void*), cudaMemcpyHostToDevice));
+  if (cfg->world > 1) {
+    if (!g_nccl.load()) return fail(db, LTPG_ENCCL, "libnccl.so.2 not loadable");
+    ncclUniqueId id;
+    std::memcpy(&id, cfg->nccl_unique_id, sizeof(id));
+    ncclResult_t r = g_nccl.commInitRank(&db->comm, cfg->world, id, cfg->rank);
+    if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclCommInitRank: ") + g_nccl.getErrorString(r));
+  }
   return LTPG_OK;
 }
 
@@ -145,15 +262,21 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
-  void* bufs[] = {db->d_tab, db->d_nrows, db->d_tid, db->d_op_begin, db->d_ops, db->d_args, db->d_ptype,
-                  db->d_params, db->d_res, db->d_uref, db->d_items, db->d_txn_ins, db->d_ua, db->d_status,
-                  db->d_bits, db->d_flags, db->d_offs, db->d_abort, db->d_small, db->d_scan};
+  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_tid, db->d_op_begin, db->d_ops, db->d_args,
+                  db->d_ptype, db->d_params, db->d_res, db->d_status, db->d_xchg, db->d_ptrs, db->d_bits,
+                  db->d_flags, db->d_offs, db->d_abort, db->d_small, db->d_scan};
   for (void* p : bufs)
     if (p) cudaFree(p);
+  for (Part& P : db->parts) {
+    void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.small, P.base};
+    for (void* p : pb)
+      if (p) cudaFree(p);
+    tpcc_free(P.tpcc);
+  }
   if (db->h_small) cudaFreeHost(db->h_small);
   for (auto& e : db->ev)
     if (e) cudaEventDestroy(e);
-  tpcc_free(db->tpcc);
+  if (db->comm) g_nccl.commDestroy(db->comm);
   delete db;
 }
 
@@ -163,7 +286,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   if (db->poisoned) return LTPG_EPOISONED;
   if (!d || t >= db->n_tables || d->n_cols > MAXC || (d->n_cols && (!d->col_group || !d->col_is_add)) ||
       n_rows > d->capacity_rows || d->capacity_rows >= 0xFFFFFFF0ull || (n_rows && d->n_cols && !cols) ||
-      (d->has_pk && n_rows && !keys) || d->n_groups > 15)
+      (d->has_pk && n_rows && !keys) || d->n_groups > 15 || d->owner_rule > 2)
     return fail(db, LTPG_EINVAL, "bad table descriptor");
   bool has_static = false;
   for (uint32_t c = 0; c < d->n_cols; ++c) {
@@ -192,18 +315,15 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   T.capacity = cap;
   long long* colmem = nullptr;
   CK(dmalloc(&colmem, cap * std::max<uint32_t>(d->n_cols, 1)));
+  T.col0 = colmem;
+  T.group_bits = ~0ull;
+  T.add_bits = 0;
   for (uint32_t c = 0; c < d->n_cols; ++c) {
     T.col[c] = colmem + c * cap;  // SoA: one contiguous int64 array per column
     T.stride[c] = 1;
     T.group[c] = d->col_group[c];
     T.is_add[c] = d->col_is_add[c] ? 1 : 0;
-  }
-  if (!d->n_cols) T.col[0] = colmem;
-  T.col0 = colmem;
-  T.group_bits = ~0ull;
-  T.add_bits = 0;
-  for (uint32_t c = 0; c < d->n_cols; ++c) {
-    uint64_t g = d->col_group[c] == LTPG_STATIC ? 15u : d->col_group[c];
+    const uint64_t g = d->col_group[c] == LTPG_STATIC ? 15u : d->col_group[c];
     T.group_bits = (T.group_bits & ~(15ull << (4 * c))) | (g << (4 * c));
     if (d->col_is_add[c]) T.add_bits |= 1u << c;
   }
@@ -248,8 +368,8 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
       return fail(db, LTPG_EINVAL, "duplicate or reserved primary key");
     }
   }
-  if (t == LTPG_T_CUSTOMER && db->cfg.n_warehouses) {
-    int rc = tpcc_build_secondary(db->tpcc, keys, cols, n_rows, db->cfg.n_warehouses);
+  if (t == LTPG_T_CUSTOMER && db->cfg.n_warehouses && !db->parts.empty()) {
+    int rc = tpcc_build_secondary(db->parts[0].tpcc, keys, cols, n_rows, db->cfg.n_warehouses);
     if (rc) return fail(db, rc, "secondary index build failed");
   }
   CK(cudaDeviceSynchronize());
@@ -272,17 +392,24 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   CK(cudaSetDevice(db->device));
   cudaStream_t s = static_cast<cudaStream_t>(b->stream);
   const bool timing = res->stats != nullptr;
+  const bool partitioned = db->nparts > 1;
+  const uint32_t L = db->loopback;
   if (timing) CK(cudaEventRecord(db->ev[0], s));
   ++db->epoch;
   const uint64_t launches0 = g_kernel_launches;
+  // ---- a1: upload ---------------------------------------------------------------------
   BatchDev bd{};
+  bd.nparts = db->nparts;
+  bd.nw = db->cfg.n_warehouses;
+  bd.key_space = db->cfg.key_space;
+  bd.reserve = db->d_reserve;
   bd.n_txns = n;
   bd.n_ops = ops_mode ? b->n_ops : 0;
   bd.epoch = db->epoch;
   bd.flags = db->cfg.flags;
   bd.clock = b->batch_clock;
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
-  // ---- a1: upload -----------------------------------------------------------------
+  bd.status = db->d_status;
   const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
   if (b->inputs_on_device) {
     bd.tid = reinterpret_cast<const unsigned long long*>(b->tid);
@@ -310,20 +437,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       bd.params = db->d_params;
     }
   }
+  const size_t n_reads = ops_mode ? b->n_ops : (size_t)n * LTPG_PROC_RESULTS;
   const bool reads_dev = res->reads && res->outputs_on_device;
-  bd.res = reads_dev ? reinterpret_cast<long long*>(res->reads) : db->d_res;
-  bd.uref = db->d_uref;
-  bd.items = db->d_items;
-  bd.txn_ins = db->d_txn_ins;
-  bd.ua = db->d_ua;
-  bd.status = db->d_status;
-  bd.err = db->d_small + 0;
-  bd.ins_tables = db->d_small + 1;
-  bd.kcount = db->d_small + 2;
+  long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : db->d_res;
   uint32_t* counts = db->d_small + 8;
   CK(cudaMemsetAsync(db->d_small, 0, 16 * sizeof(uint32_t), s));
-  if (n) CK(cudaMemsetAsync(db->d_ua, 0, n, s));
-  if (timing) CK(cudaEventRecord(db->ev[1], s));
+  CK(cudaMemsetAsync(db->d_reserve, 0, MAXT * sizeof(unsigned long long), s));
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
   if (g_uploaded[db->device % 64] != db->tab_version) {
@@ -334,47 +453,102 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   }
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
-  if (n) {
-    if (ops_mode) {
-      // ---- a1/a2: validate + adaptive warp division ---------------------------------
-      launch_ops_validate_group(db->n_tables, bd, grouped, s);
-      scan_exclusive_u32(db->d_txn_ins, db->d_txn_ins, n, db->d_scan, s);
-      launch_capacity_check(db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
-      // ---- a3: insert claims ----------------------------------------------------------
-      launch_ops_claim(bd, s);
-      if (timing) CK(cudaEventRecord(db->ev[2], s));
-      // ---- a4/a5: execute + marks -----------------------------------------------------
-      launch_ops_exec(bd, grouped, filter, s);
-      if (timing) CK(cudaEventRecord(db->ev[3], s));
-      // ---- a6: conflict detection -------------------------------------------------------
-      launch_ops_detect(bd, s);
-      if (timing) CK(cudaEventRecord(db->ev[4], s));
-      if (timing) CK(cudaEventRecord(db->ev[5], s));
-      // ---- a7: write-back -------------------------------------------------------------
-      launch_ops_writeback(bd, s);
-      launch_advance_cursor(db->n_tables, bd.ins_tables, db->d_txn_ins + n, bd.err, s);
-    } else {
-      int rc = tpcc_run(db->tpcc, bd, db->d_scan, s, timing ? db->ev : nullptr);
-      if (rc) return fail(db, rc, "tpcc launch failed");
+  std::vector<BatchDev> pb(L, bd);
+  for (uint32_t p = 0; p < L; ++p) {
+    Part& P = db->parts[p];
+    BatchDev& x = pb[p];
+    x.part = (uint32_t)db->cfg.rank * L + p;
+    x.res = (!partitioned && p == 0) ? res_out : P.res;
+    x.uref = P.uref;
+    x.items = P.items;
+    x.txn_ins = P.txn_ins;
+    x.ua = P.ua;
+    x.lflag = P.lflag;
+    x.err = P.small + 0;
+    x.ins_tables = P.small + 1;
+    x.kcount = P.small + 2;
+    x.base = P.base;
+    CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
+    if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
+    if (partitioned && n) {
+      CK(cudaMemsetAsync(P.res, 0, n_reads * sizeof(long long), s));
+      CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
     }
-    // ---- finalize: commit bitmask, abort list ------------------------------------------
-    launch_finalize(db->d_status, n, db->d_bits, db->d_flags, counts, bd.err, s);
+  }
+  if (timing) CK(cudaEventRecord(db->ev[1], s));
+  if (n) {
+    // ---- a1..a6 per partition: validate + warp division, claims, execute + marks, detect --------
+    for (uint32_t p = 0; p < L; ++p) {
+      BatchDev& x = pb[p];
+      cudaEvent_t* evp = (timing && p == L - 1) ? db->ev : nullptr;
+      if (ops_mode) {
+        launch_ops_validate_group(db->n_tables, x, grouped, s);
+        scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
+        launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
+        launch_ops_claim(x, s);
+        if (evp) CK(cudaEventRecord(evp[2], s));
+        launch_ops_exec(x, grouped, filter, s);
+        if (evp) CK(cudaEventRecord(evp[3], s));
+        launch_ops_detect(x, s);
+      } else {
+        int rc = tpcc_front(db->parts[p].tpcc, x, s, evp);
+        if (rc) return fail(db, rc, "tpcc launch failed");
+      }
+    }
+    if (timing) CK(cudaEventRecord(db->ev[4], s));
+    // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
+    if (partitioned) {
+      if (db->cfg.world == 1) {
+        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, db->d_status, db->d_ptrs + 64, db->d_small);
+        k_spread_err<<<1, 1, 0, s>>>(db->d_small, db->d_ptrs + 64, L);
+        note_launch(2);
+      } else {
+        k_pack<<<(n + 255) / 256, 256, 0, s>>>(pb[0].lflag, pb[0].err, db->d_xchg, n);
+        ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, n + 3, ncclUint8, ncclMax, db->comm, s);
+        if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
+        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, db->d_status, pb[0].err, db->d_small);
+        note_launch(2);
+      }
+    } else {
+      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, db->d_small);
+      note_launch();
+    }
+    if (timing) CK(cudaEventRecord(db->ev[5], s));
+    // ---- a7: write-back per partition -------------------------------------------------------
+    for (uint32_t p = 0; p < L; ++p) {
+      if (ops_mode) {
+        launch_ops_writeback(pb[p], s);
+      } else {
+        int rc = tpcc_back(db->parts[p].tpcc, pb[p], db->d_scan, s);
+        if (rc) return fail(db, rc, "tpcc launch failed");
+      }
+    }
+    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, db->d_small, s);
+    // results: summed over partitions (each slot is written by its owning partition only)
+    if (partitioned && res->reads) {
+      if (db->cfg.world == 1) {
+        k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);
+        note_launch();
+      } else {
+        ncclResult_t r = g_nccl.allReduce(pb[0].res, res_out, n_reads, ncclInt64, ncclSum, db->comm, s);
+        if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
+      }
+    }
+    // ---- finalize: commit bitmask, abort list -------------------------------------------------
+    launch_finalize(db->d_status, n, db->d_bits, db->d_flags, counts, db->d_small, s);
     scan_exclusive_u32(db->d_flags, db->d_offs, n, db->d_scan, s);
     launch_compact(db->d_flags, db->d_offs, n, db->d_abort, s);
   }
   CK(cudaGetLastError());
   if (timing) CK(cudaEventRecord(db->ev[6], s));
-  // ---- a8: results --------------------------------------------------------------------
+  // ---- a8: results ------------------------------------------------------------------------
   const cudaMemcpyKind out_kind = res->outputs_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
   CK(cudaMemcpyAsync(db->h_small, db->d_small, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   if (n) {
     CK(cudaMemcpyAsync(db->h_small + 16, db->d_offs + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(res->status, db->d_status, n, out_kind, s));
     CK(cudaMemcpyAsync(res->commit_bits, db->d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, s));
-    if (res->reads && !reads_dev) {
-      size_t nr = ops_mode ? b->n_ops : (size_t)n * LTPG_PROC_RESULTS;
-      CK(cudaMemcpyAsync(res->reads, db->d_res, nr * sizeof(int64_t), out_kind, s));
-    }
+    if (res->reads && !reads_dev) CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, s));
     if (res->outputs_on_device) {
       CK(cudaMemcpyAsync(res->n_aborted, db->d_offs + n, sizeof(uint32_t), out_kind, s));
       CK(cudaMemcpyAsync(res->abort_idx, db->d_abort, n * sizeof(uint32_t), out_kind, s));

@@ -177,35 +177,36 @@ void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
   note_launch();
 }
 
-// ECAPACITY before anything mutates: provisional rows are n_rows + [0, total)
-__global__ void k_capacity(uint32_t n_tables, const uint32_t* ins_tables,
-                           const uint32_t* total, uint32_t* err) {
-  uint32_t m = *ins_tables;
-  uint64_t tot = *total;
-  for (uint32_t t = 0; t < n_tables; ++t)
+// ECAPACITY before anything mutates.  The partition's inserts take provisional rows
+// n_rows + base + [0, total); base is this partition's offset in the batch reservation.
+__global__ void k_capacity(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
+                           unsigned long long* base, unsigned long long* reserve, uint32_t* err) {
+  const uint32_t m = *ins_tables;
+  const uint64_t tot = *total;
+  for (uint32_t t = 0; t < n_tables; ++t) {
+    base[t] = reserve[t];
     if ((m >> t) & 1u) {
       const DevTable& T = c_tabs[t];
-      if (*T.n_rows + tot > T.capacity || *T.n_rows + tot > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
+      reserve[t] += tot;
+      if (*T.n_rows + reserve[t] > T.capacity || *T.n_rows + reserve[t] > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
     }
+  }
 }
 
-void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables,
-                           const uint32_t* total, uint32_t* err, cudaStream_t s) {
-  k_capacity<<<1, 1, 0, s>>>(n_tables, ins_tables, total, err);
+void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
+                           unsigned long long* base, unsigned long long* reserve, uint32_t* err, cudaStream_t s) {
+  k_capacity<<<1, 1, 0, s>>>(n_tables, ins_tables, total, base, reserve, err);
   note_launch();
 }
 
-__global__ void k_advance(uint32_t n_tables, const uint32_t* ins_tables,
-                          const uint32_t* total, const uint32_t* err) {
+__global__ void k_advance(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err) {
   if (*err) return;
-  uint32_t m = *ins_tables;
-  for (uint32_t t = 0; t < n_tables; ++t)
-    if ((m >> t) & 1u) *c_tabs[t].n_rows += *total;
+  for (uint32_t t = 0; t < n_tables; ++t) *c_tabs[t].n_rows += reserve[t];
 }
 
-void launch_advance_cursor(uint32_t n_tables, const uint32_t* ins_tables,
-                           const uint32_t* total, const uint32_t* err, cudaStream_t s) {
-  k_advance<<<1, 1, 0, s>>>(n_tables, ins_tables, total, err);
+void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
+                           cudaStream_t s) {
+  k_advance<<<1, 1, 0, s>>>(n_tables, reserve, err);
   note_launch();
 }
 

@@ -46,6 +46,18 @@ __device__ __forceinline__ bool is_write_kind(uint8_t k) {
   return k == LTPG_UPDATE || k == LTPG_ADD || k == LTPG_INSERT || k == LTPG_DELETE;
 }
 
+// Does this partition handle (part of) op o?  Key ranges are contiguous, so a SCAN touches
+// the partitions between the owners of its first and last key.
+__device__ __forceinline__ bool op_touches(const BatchDev& b, const ltpg_op& o) {
+  if (b.nparts <= 1) return true;
+  const DevTable& T = c_tabs[o.table];
+  if (T.owner_rule != 2) return b.part == 0;
+  const uint32_t p0 = part_of_key(2, o.key, b.key_space, b.nparts);
+  if (o.kind != LTPG_SCAN || o.aux <= 1) return p0 == b.part;
+  const uint32_t p1 = part_of_key(2, o.key + o.aux - 1, b.key_space, b.nparts);
+  return p0 <= b.part && b.part <= p1;
+}
+
 // ---- K-group: validation + decomposition into per-kind lists (one thread per txn) ----
 template <bool GROUPED>
 __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
@@ -75,7 +87,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
         if (b0 + i < b1) {
           ltpg_op o = load_op(b.ops, b0 + i);
           if (!op_valid(n_tables, o)) bad = true;
-          else {
+          else if (op_touches(b, o)) {
             cnt64 += 1ull << (10 * o.kind);
             if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
           }
@@ -97,6 +109,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
     for (uint32_t i = b0; i < b1; ++i) {
       ltpg_op o = load_op(b.ops, i);
       if (!op_valid(n_tables, o)) { bad = true; continue; }
+      if (!op_touches(b, o)) continue;
       cnt64 += 1ull << (10 * o.kind);
       if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
     }
@@ -128,7 +141,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
     if (r == 0) b.kcount[0] = b.n_ops;
     if (r < b.n_txns && !bad)
       for (uint32_t i = b0; i < b1; ++i)
-        if (b.ops[i].kind == LTPG_INSERT) {
+        if (b.ops[i].kind == LTPG_INSERT && op_touches(b, load_op(b.ops, i))) {
           uint32_t p = atomicAdd(b.kcount + LTPG_INSERT, 1u);
           b.items[(uint64_t)LTPG_INSERT * b.max_ops + p] = (unsigned long long)i | ((unsigned long long)r << 32);
         }
@@ -153,7 +166,9 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
   }
   if (r < b.n_txns && !bad)
     for (uint32_t i = b0; i < b1; ++i) {
-      uint8_t k = b.ops[i].kind;
+      const ltpg_op o = load_op(b.ops, i);
+      if (!op_touches(b, o)) continue;
+      const uint8_t k = o.kind;
       uint32_t p = 0;
 #pragma unroll
       for (int kk = 0; kk < NKINDS; ++kk)
@@ -184,8 +199,9 @@ __global__ void __launch_bounds__(256) k_ops_claim(BatchDev b) {
     ltpg_op o = load_op(b.ops, oi);
     const DevTable& T = c_tabs[o.table];
     uint32_t j = 0;
-    for (uint32_t q = b.op_begin[r]; q < oi; ++q) j += b.ops[q].kind == LTPG_INSERT;
-    uint32_t prov = (uint32_t)(*T.n_rows + b.txn_ins[r] + j);
+    for (uint32_t q = b.op_begin[r]; q < oi; ++q)
+      j += b.ops[q].kind == LTPG_INSERT && op_touches(b, load_op(b.ops, q));
+    uint32_t prov = (uint32_t)(*T.n_rows + b.base[o.table] + b.txn_ins[r] + j);
     IdxSlot* sl = idx_find_or_insert(T, o.key);
     if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
     if (*reinterpret_cast<volatile unsigned*>(&sl->row) != ROW_NONE) continue;  // present in S
@@ -206,10 +222,12 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
   uint32_t row, claim;
   long long res = LTPG_NOT_FOUND;
   uint64_t uref = 0;
+  if (!op_touches(b, o)) return;  // another partition's op (flat-list mode)
   if (o.kind == LTPG_SCAN) {  // range of predefined keys; checked again in detect
     long long cnt = 0;
     unsigned long long sum = 0;
     for (uint64_t k = o.key; k < o.key + o.aux; ++k) {
+      if (!owns_key(b, T, k)) continue;  // partitioned: this partition's part of the range
       idx_find(T, k, row, claim);
       if (row != ROW_NONE) {
         ++cnt;
@@ -318,6 +336,9 @@ void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t 
 }
 
 // ---- K-detect: per txn, OR of the unit tests over its ops ------------------------------
+// PART: partitioned -- only this partition's ops / keys are checked and the verdict goes
+// to lflag (conflict*2 | user_abort) for the exchange; otherwise it is final (status).
+template <bool PART>
 __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   if (*b.err) return;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
@@ -325,6 +346,7 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
   bool bad = false;
   for (uint32_t i = b0; i < b1 && !bad; ++i) {
+    if (PART && !op_touches(b, load_op(b.ops, i))) continue;
     const uint64_t u = b.uref[i];
     const uint64_t chk = u >> 62;
     if (chk == CHK_NONE) continue;
@@ -333,6 +355,7 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
       const ltpg_op o = load_op(b.ops, i);
       if (!T.n_groups) continue;
       for (uint64_t k = o.key; k < o.key + o.aux && !bad; ++k) {
+        if (PART && !owns_key(b, T, k)) continue;
         uint32_t row, claim;
         idx_find(T, k, row, claim);
         if (row != ROW_NONE) {
@@ -351,11 +374,16 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
       bad = unit_conflicts(T, (u >> 32) & 0xFF, row, chk, r, b.epoch);
     }
   }
-  b.status[r] = bad ? LTPG_ST_CONFLICT : (b.ua[r] ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+  const uint8_t flag = (uint8_t)(bad ? 2 : 0) | (b.ua[r] ? 1 : 0);
+  if (PART) b.lflag[r] = flag;
+  else b.status[r] = status_of_flag(flag);
 }
 
 void launch_ops_detect(const BatchDev& b, cudaStream_t s) {
-  k_ops_detect<<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
+  if (b.nparts > 1)
+    k_ops_detect<true><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
+  else
+    k_ops_detect<false><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
   note_launch();
 }
 
@@ -364,20 +392,20 @@ __global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b) {
   if (*b.err) return;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
-  const bool commit = b.status[r] == LTPG_ST_COMMIT;
+  const bool commit = b.status[r] == LTPG_ST_COMMIT;  // final verdict (after the exchange)
   if (!commit && b.txn_ins[r + 1] == b.txn_ins[r]) return;  // aborted, no claims to release
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
   for (uint32_t i = b0; i < b1; ++i) {
+    const ltpg_op o = load_op(b.ops, i);
+    if (!commit && o.kind != LTPG_INSERT) continue;
+    if (!op_touches(b, o)) continue;  // another partition's op: its uref is not ours
     const uint64_t u = b.uref[i];
-    const uint32_t kind = b.ops[i].kind;
-    if (!commit && kind != LTPG_INSERT) continue;
     if ((u >> 62) == CHK_NONE || (u >> 62) == CHK_SCAN) continue;
     const bool present = (u >> 60) & 1;
     const uint32_t row = (uint32_t)u;
-    if (kind == LTPG_INSERT) {
+    const DevTable& T = c_tabs[o.table];
+    if (o.kind == LTPG_INSERT) {
       if (present) continue;  // duplicate-key user abort: nothing claimed
-      const ltpg_op o = load_op(b.ops, i);
-      const DevTable& T = c_tabs[o.table];
       IdxSlot* sl = idx_slot(T, o.key);
       if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
       if (commit) {
@@ -392,9 +420,7 @@ __global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b) {
       continue;
     }
     if (!present) continue;
-    const ltpg_op o = load_op(b.ops, i);
-    const DevTable& T = c_tabs[o.table];
-    switch (kind) {
+    switch (o.kind) {
       case LTPG_UPDATE:
         *col_ptr_ops(T, o.col, row) = (long long)((unsigned long long)b.res[i] + (unsigned long long)b.args[i]);
         break;

@@ -121,13 +121,21 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   long long amount = 0;
   uint32_t remote = 0, ua = 0;
   uint32_t i = 0, sw = 0, qty = 0, row_s = ROW_NONE;
-  const bool line = active && sub < n;
+  // partitioned (§8(e)): the home partition owns the header, the order inserts and the
+  // result; each stock line belongs to the owner of its supply warehouse
+  const bool home = active && owns_w(b, w);
+  bool line = active && sub < n;
+  bool own_line = false;
   if (line) {
     const uint8_t* L = p + 8 + 8 * sub;
     i = p32(L, 0);
     sw = p16(L, 4);
     qty = L[6];
     remote = sw != w;
+    own_line = owns_w(b, sw);
+    line = home || own_line;
+  }
+  if (line) {
     if (PH == PH_EXEC || PH == PH_WB) {
       const uint32_t row_i = probe(TIt, i);
       if (row_i == ROW_NONE) {
@@ -137,7 +145,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       }
     }
     if (PH == PH_EXEC) {
-      if (!ua) {
+      if (!ua && own_line) {
         row_s = probe(TSt, kS(sw, i));
         if (row_s == ROW_NONE) internal_error(x);
       }
@@ -161,7 +169,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   }
   // header lane: warehouse / district / customer reads, fetch-ADD of D_NEXT_O_ID
   long long w_tax = 0, d_tax = 0, disc = 0;
-  if (active && sub == 15) {
+  if (home && sub == 15) {
     uint32_t row_d;
     if (PH == PH_EXEC) {
       const uint32_t row_w = probe(TWh, w);
@@ -184,24 +192,24 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   if (PH == PH_EXEC) {
     const long long sum = seg16_sum(amount);
     ua = seg16_or(ua);
-    if (active && sub == 15) {
+    if (active && ua && sub == 15) b.ua[r] = 1;
+    if (home && sub == 15) {
       long long* res = b.res + 4ull * r;
       res[0] = 0;  // o_id: assigned after detection if committed
       res[1] = sum * (10000 - disc) * (10000 + w_tax + d_tax) / 100000000;
       res[2] = sum;
       res[3] = 0;
-      if (ua) b.ua[r] = 1;
     }
   }
   if (PH == PH_WB) {
     const uint32_t all_local = !seg16_or(remote);
-    if (active) {
+    if (home) {
       const long long o = b.res[4ull * r];
       const uint64_t okey = kO(w, d, (uint64_t)o);
       const DevTable& TOr = c_tabs[TO];
       const DevTable& TOL_ = c_tabs[TOL];
       const DevTable& TNw = c_tabs[TNO];
-      if (line) {  // ORDER_LINE row
+      if (active && sub < n) {  // ORDER_LINE row
         const uint32_t row = (uint32_t)(*TOL_.n_rows + tp.no_lines[r] + sub);
         wr(TOL_, OL_I_ID, row, i);
         wr(TOL_, OL_SUPPLY_W_ID, row, sw);
@@ -248,37 +256,46 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   const uint32_t clast = p16(p, 10);
   const long long amount = p64(p, 16);
   uint32_t* log = tp.log + (uint64_t)r * TLOG;
-  uint32_t row_w, row_d, row_c;
+  // partitioned (§8(e)): warehouse + district on the home partition, the customer (its
+  // by-name lookup, result and HISTORY row) on the customer's owner
+  const bool home = owns_w(b, w), cust = owns_w(b, cw);
+  uint32_t row_w = ROW_NONE, row_d = ROW_NONE, row_c = ROW_NONE;
   if (PH == PH_EXEC) {
-    if (by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
-    row_w = probe(TWh, w);
-    row_d = probe(TDi, kD(w, d));
-    row_c = cid ? probe(TCu, kC(cw, cd, cid)) : ROW_NONE;
-    if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
-      internal_error(x);
-      return;
+    if (home) {
+      row_w = probe(TWh, w);
+      row_d = probe(TDi, kD(w, d));
+      if (row_w == ROW_NONE || row_d == ROW_NONE) { internal_error(x); return; }
+    }
+    if (cust) {
+      if (by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
+      row_c = cid ? probe(TCu, kC(cw, cd, cid)) : ROW_NONE;
+      if (row_c == ROW_NONE) { internal_error(x); return; }
+      long long* res = b.res + 4ull * r;
+      res[0] = cid;
+      res[1] = col_is_add(TCu, C_BALANCE) ? 0 : rd(TCu, C_BALANCE, row_c);  // pre-image (strict only)
+      res[2] = 0;
+      res[3] = 0;
     }
     log[0] = row_w;
     log[1] = row_d;
     log[2] = row_c;
     log[3] = cid;
-    long long* res = b.res + 4ull * r;
-    res[0] = cid;
-    res[1] = col_is_add(TCu, C_BALANCE) ? 0 : rd(TCu, C_BALANCE, row_c);  // pre-image (strict only)
-    res[2] = 0;
-    res[3] = 0;
   } else {
     row_w = log[0];
     row_d = log[1];
     row_c = log[2];
     cid = log[3];
   }
-  col_upd<PH>(TWh, W_YTD, row_w, x);
-  col_upd<PH>(TDi, D_YTD, row_d, x);
-  col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, row_c, x);
-  if (PH == PH_WB) {
+  if (home) {
+    col_upd<PH>(TWh, W_YTD, row_w, x);
+    col_upd<PH>(TDi, D_YTD, row_d, x);
+  }
+  if (cust) col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, row_c, x);
+  if (PH == PH_WB && home) {
     addv(TWh, W_YTD, row_w, amount);
     addv(TDi, D_YTD, row_d, amount);
+  }
+  if (PH == PH_WB && cust) {
     addv(TCu, C_BALANCE, row_c, -amount);
     addv(TCu, C_YTD_PAYMENT, row_c, amount);
     addv(TCu, C_PAYMENT_CNT, row_c, 1);
@@ -563,8 +580,11 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
     if (PH == PH_DETECT) {  // per-txn OR over the txn's lanes, one status write per txn
       const uint32_t bal = __ballot_sync(0xffffffffu, x.bad);
       const uint32_t seg = L == 32 ? 0xffffffffu : (L == 1 ? (1u << lane) : (0xffffu << (lane & 16)));
-      if (active && sub == 0)
-        b.status[r] = (bal & seg) ? LTPG_ST_CONFLICT : (b.ua[r] ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+      if (active && sub == 0) {
+        const uint8_t flag = (uint8_t)((bal & seg) ? 2 : 0) | (b.ua[r] ? 1 : 0);
+        if (b.nparts > 1) b.lflag[r] = flag;  // partitioned: exchanged before write-back
+        else b.status[r] = status_of_flag(flag);
+      }
     }
   }
 }
@@ -616,26 +636,55 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     }
     if (bad) atomicOr(b.err, ERR_EINVAL);
   }
+  // partitioned (§8(e)): list the txn only where it touches owned rows; count the appends
+  // this partition may make (ORDER/NEW_ORDER/ORDER_LINE at home, HISTORY at the customer)
+  bool touch = false;
+  uint32_t no_home = 0, pay_cust = 0;
+  if (r < b.n_txns && !bad) {
+    const uint8_t* p = b.params + 128ull * r;
+    const bool home = owns_w(b, p16(p, 0));
+    touch = home;
+    if (t == 0) {
+      for (uint32_t l = 0; l < lines && !touch; ++l) touch = owns_w(b, p16(p + 8 + 8 * l, 4));
+      no_home = home;
+      if (!home) lines = 0;
+    } else if (t == 1) {
+      pay_cust = owns_w(b, p16(p, 4));
+      touch = touch || pay_cust;
+    }
+  } else {
+    lines = 0;
+  }
   const uint32_t lsum = __reduce_add_sync(0xffffffffu, lines);
-  if (lane == 0 && lsum) atomicAdd(tp.misc + M_NO_LINES, lsum);
+  const uint32_t nsum = __reduce_add_sync(0xffffffffu, no_home);
+  const uint32_t psum = __reduce_add_sync(0xffffffffu, pay_cust);
+  if (lane == 0) {
+    if (lsum) atomicAdd(tp.misc + M_NO_LINES, lsum);
+    if (nsum) atomicAdd(tp.misc + M_NO, nsum);
+    if (psum) atomicAdd(tp.misc + M_PAY, psum);
+  }
 #pragma unroll
   for (uint32_t k = 0; k < NTYPES; ++k) {
-    const uint32_t m = __ballot_sync(0xffffffffu, t == k && !bad);
+    const uint32_t m = __ballot_sync(0xffffffffu, t == k && !bad && touch);
     if (!m) continue;
     uint32_t base = 0;
     const uint32_t leader = __ffs(m) - 1;
     if (lane == leader) base = atomicAdd(b.kcount + k, __popc(m));
     base = __shfl_sync(0xffffffffu, base, leader);
-    if (t == k && !bad) tp.list[(uint64_t)k * tp.max_txns + base + __popc(m & ((1u << lane) - 1))] = r;
+    if (t == k && !bad && touch) tp.list[(uint64_t)k * tp.max_txns + base + __popc(m & ((1u << lane) - 1))] = r;
   }
 }
 
-// ECAPACITY before execution: worst case every NewOrder / Payment commits
+// ECAPACITY before execution: worst case every NewOrder / Payment of this partition
+// commits; partitions of one process share the table and reserve in stream order
 __global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
-  const uint64_t n_no = b.kcount[0], n_pay = b.kcount[1], lines = tp.misc[M_NO_LINES];
-  auto over = [](const DevTable& T, uint64_t add) { return *T.n_rows + add > T.capacity; };
-  if (over(c_tabs[TO], n_no) || over(c_tabs[TNO], n_no) || over(c_tabs[TOL], lines) || over(c_tabs[TH], n_pay))
-    atomicOr(b.err, ERR_ECAPACITY);
+  const uint64_t add[4] = {tp.misc[M_NO], tp.misc[M_NO], tp.misc[M_NO_LINES], tp.misc[M_PAY]};
+  const int tabs[4] = {TO, TNO, TOL, TH};
+  for (int k = 0; k < 4; ++k) {
+    const DevTable& T = c_tabs[tabs[k]];
+    b.reserve[tabs[k]] += add[k];
+    if (*T.n_rows + b.reserve[tabs[k]] > T.capacity) atomicOr(b.err, ERR_ECAPACITY);
+  }
 }
 
 // ---- NewOrder o_id: fetch-ADD pre-image = snapshot D_NEXT_O_ID + #committed NewOrders of the
@@ -644,8 +693,8 @@ __global__ void k_no_prep(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
-  const bool c = b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT;
   const uint8_t* p = b.params + 128ull * r;
+  const bool c = b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT && owns_w(b, p16(p, 0));
   tp.no_flag[r] = c;
   tp.no_lines[r] = c ? p[3] : 0;
   tp.dk_of[r] = c ? (uint32_t)kD(p16(p, 0), p[2]) : ~0u;
@@ -735,22 +784,26 @@ static cudaError_t dm(T** p, size_t n) {
   return cudaMalloc(reinterpret_cast<void**>(p), std::max<size_t>(n, 1) * sizeof(T));
 }
 
-int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw) {
+int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) {
   t.max_txns = max_txns;
   t.nw = nw;
   if (!nw) return 0;
   if (nw > 1000) return LTPG_EINVAL;
   t.dsz = nw * 10 + 11;
   const uint64_t chunks = (max_txns + NO_CHUNK - 1) / NO_CHUNK;
-  if (dm(&t.by_name, (uint64_t)t.dsz * 1000) || dm(&t.list, (uint64_t)NTYPES * max_txns) ||
+  t.owns_by_name = shared_by_name == nullptr;
+  if (shared_by_name) t.by_name = shared_by_name;
+  else if (dm(&t.by_name, (uint64_t)t.dsz * 1000)) return LTPG_ENOMEM;
+  if (dm(&t.list, (uint64_t)NTYPES * max_txns) ||
       dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_flag, max_txns + 1ull) || dm(&t.no_lines, max_txns + 1ull) ||
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
     return LTPG_ENOMEM;
-  cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
+  if (t.owns_by_name) cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
   return 0;
 }
 
 void tpcc_free(TpccDev& t) {
+  if (!t.owns_by_name) t.by_name = nullptr;
   void* ps[] = {t.by_name, t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
   for (void* p : ps)
     if (p) cudaFree(p);
@@ -780,28 +833,38 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
              : LTPG_ECUDA;
 }
 
-int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cudaEvent_t* ev) {
+static TpccParams params_of(TpccDev& t, uint32_t n) {
+  return TpccParams{t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
+                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
+}
+static uint32_t phase_grid(uint32_t n) {
+  const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
+  return (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
+}
+
+int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   if (!t.nw) return LTPG_EINVAL;
   const uint32_t n = b.n_txns;
-  TpccParams tp{t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
-                t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
+  const TpccParams tp = params_of(t, n);
   cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
-  const uint32_t blocks = (n + 255) / 256;
-  k_tpcc_group<<<blocks, 256, 0, s>>>(b, tp);
+  k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   k_tpcc_capacity<<<1, 1, 0, s>>>(b, tp);
   note_launch(2);
   if (ev) cudaEventRecord(ev[2], s);
-  // one warp-slot per txn lane group; grid-stride over the per-type warp ranges
-  const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
-  const uint32_t grid = (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
+  const uint32_t grid = phase_grid(n);
   k_tpcc_phase<PH_EXEC><<<grid, 256, 0, s>>>(b, tp);
   note_launch();
   if (ev) cudaEventRecord(ev[3], s);
   k_tpcc_phase<PH_DETECT><<<grid, 256, 0, s>>>(b, tp);
   note_launch();
-  if (ev) cudaEventRecord(ev[4], s);
+  return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
+}
+
+int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
+  const uint32_t n = b.n_txns;
+  const TpccParams tp = params_of(t, n);
   // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders
-  k_no_prep<<<blocks, 256, 0, s>>>(b, tp);
+  k_no_prep<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   note_launch();
   scan_exclusive_u32(t.no_flag, t.no_flag, n, scan_scratch, s);
   scan_exclusive_u32(t.no_lines, t.no_lines, n, scan_scratch, s);
@@ -810,8 +873,7 @@ int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cu
   k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  if (ev) cudaEventRecord(ev[5], s);
-  k_tpcc_phase<PH_WB><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_WB><<<phase_grid(n), 256, 0, s>>>(b, tp);
   k_tpcc_advance<<<1, 1, 0, s>>>(b, tp);
   note_launch(2);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;

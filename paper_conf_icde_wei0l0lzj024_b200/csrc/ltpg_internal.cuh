@@ -184,6 +184,15 @@ extern uint64_t g_kernel_launches;
 inline void note_launch(uint32_t k = 1) { g_kernel_launches += k; }
 
 struct BatchDev {
+  // partitioning (§8(e)): nparts logical partitions (ranks x loopback); this is `part`.
+  // nparts == 1: this partition owns everything and detect writes `status` directly;
+  // otherwise detect writes lflag[r] = conflict*2 | user_abort for the exchange.
+  uint32_t nparts, part;
+  uint32_t nw;                     // TPC-C: number of warehouses (warehouse ownership)
+  uint64_t key_space;              // OPS: key-range ownership of owner_rule-2 tables
+  uint8_t* lflag;                  // [n_txns] partitioned detect output
+  unsigned long long* reserve;     // [MAXT] append rows reserved this batch (all partitions)
+  unsigned long long* base;        // [MAXT] this partition's offset inside the reservation
   uint32_t n_txns, n_ops, epoch, flags;
   int64_t clock;
   const unsigned long long* tid;
@@ -204,6 +213,27 @@ struct BatchDev {
   uint32_t max_ops;
 };
 
+// ---- ownership (contiguous ranges) -------------------------------------------------------
+__host__ __device__ __forceinline__ uint32_t part_of_w(uint32_t w, uint32_t nw, uint32_t np) {
+  return np <= 1 || !nw ? 0u : (uint32_t)(((uint64_t)(w - 1) * np) / nw);
+}
+__host__ __device__ __forceinline__ uint32_t part_of_key(uint32_t owner_rule, uint64_t key, uint64_t ks, uint32_t np) {
+  if (np <= 1 || owner_rule != 2 || !ks) return 0u;  // rule 0/1 tables: partition 0 (OPS mode)
+  const uint64_t chunk = (ks + np - 1) / np;
+  const uint64_t p = key / chunk;
+  return p >= np ? np - 1 : (uint32_t)p;
+}
+__device__ __forceinline__ bool owns_key(const BatchDev& b, const DevTable& T, uint64_t key) {
+  return b.nparts <= 1 || part_of_key(T.owner_rule, key, b.key_space, b.nparts) == b.part;
+}
+__device__ __forceinline__ bool owns_w(const BatchDev& b, uint32_t w) {
+  return b.nparts <= 1 || part_of_w(w, b.nw, b.nparts) == b.part;
+}
+// final verdict from a partition-local or exchanged flag (conflict dominates user abort)
+__device__ __forceinline__ uint8_t status_of_flag(uint8_t f) {
+  return f >= 2 ? LTPG_ST_CONFLICT : (f ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+}
+
 void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
 size_t scan_scratch_words(uint32_t n);
 
@@ -213,10 +243,10 @@ void launch_ops_claim(const BatchDev& b, cudaStream_t s);
 void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
 void launch_ops_detect(const BatchDev& b, cudaStream_t s);
 void launch_ops_writeback(const BatchDev& b, cudaStream_t s);
-void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables,
-                           const uint32_t* total, uint32_t* err, cudaStream_t s);
-void launch_advance_cursor(uint32_t n_tables, const uint32_t* ins_tables,
-                           const uint32_t* total, const uint32_t* err, cudaStream_t s);
+void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
+                           unsigned long long* base, unsigned long long* reserve, uint32_t* err, cudaStream_t s);
+void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
+                           cudaStream_t s);
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);

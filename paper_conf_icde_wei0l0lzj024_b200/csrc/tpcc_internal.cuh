@@ -21,7 +21,7 @@ enum { OL_I_ID = 0, OL_SUPPLY_W_ID = 1, OL_QUANTITY = 2, OL_AMOUNT = 3, OL_DELIV
 enum { I_PRICE = 0, I_IM_ID = 1 };
 enum { S_QUANTITY = 0, S_YTD = 1, S_ORDER_CNT = 2, S_REMOTE_CNT = 3 };
 
-// counters in TpccDev::misc
+// counters in TpccDev::misc (M_NO / M_NO_LINES / M_PAY: inserts this partition may append)
 enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3 };
 
 struct TpccDev {
@@ -29,6 +29,7 @@ struct TpccDev {
   uint32_t nw = 0;              // n_warehouses (global)
   uint32_t dsz = 0;             // district-key array size = nw*10 + 11
   int* by_name = nullptr;       // dense secondary index [(w*10+d)*1000 + c_last] -> c_id (0: none)
+  bool owns_by_name = false;    // loopback partitions share partition 0's index
   uint32_t* list = nullptr;     // [NTYPES][max_txns] ranks, grouped by procedure type
   uint32_t* log = nullptr;      // [max_txns][TLOG] rows found by execute
   uint32_t* no_flag = nullptr;  // [max_txns+1] committed NewOrder -> exclusive scan (row offsets)
@@ -52,10 +53,12 @@ struct TpccParams {
   uint32_t nw, dsz, max_txns, n_chunks;
 };
 
-int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses);
+int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);
 void tpcc_free(TpccDev& t);
 int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, uint64_t n_rows,
                          uint32_t n_warehouses);
-int tpcc_run(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s, cudaEvent_t* ev);
+// front: validate + lists, capacity, execute, detect;  back: o_id prefix, write-back, cursors
+int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev);
+int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s);
 
 }  // namespace ltpg
