@@ -40,8 +40,11 @@ WORKLOADS = {
     "ycsb_c3": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=10, batch=1 << 20),
     "tpcc_c4": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="strict"),
     "tpcc_c5": dict(kind="tpcc", cfg=4, W=512, mix="no_pay", batch=1 << 20, mode="strict"),
+    "tpcc_c4_delayed": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="delayed"),
+    "tpcc_c2_delayed": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed"),
+    "ycsb_c3_4ops": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=4, batch=1 << 20),
 }
-DEFAULT_WORKLOAD = "ycsb_c3"
+DEFAULT_WORKLOAD = "tpcc_c4"
 
 
 def log(*a):
@@ -123,9 +126,10 @@ def ncu_traffic(kernel_substr):
 
 
 # ---- workloads ------------------------------------------------------------------------------
-def make_workload(name, rank):
+def make_workload(name, rank=0):
+    # every rank builds the same global workload (partitioned multi-GPU mode, §8(e))
     w = WORKLOADS[name]
-    seed = 0x17C0 + w["cfg"] + 1000 * rank
+    seed = 0x17C0 + w["cfg"]
     if w["kind"] == "ycsb":
         from workloads.ycsb import YcsbWorkload
         return YcsbWorkload(w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
@@ -202,8 +206,8 @@ def run_reference(args, name):
     desc = "%d-txn batches of %s (full batch %d), %d timed" % (sample, name, w["batch"], args.steps)
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * secs / max(args.steps, 1),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
-            "data": "synthetic", "config": config_of(name, sample),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic", "config": dict(config_of(name), parallelism="CPU oracle, 1 thread"),
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -275,15 +279,20 @@ def main():
     import paper_conf_icde_wei0l0lzj024_b200 as ltpg
 
     w = WORKLOADS[name]
-    wl = make_workload(name, rank)
+    wl = make_workload(name)
     B = w["batch"]
+    uid = None
+    if world > 1:  # one NCCL communicator per db: the per-batch verdict exchange
+        from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id
+        uid = nccl_unique_id()
     t0 = time.time()
     if w["kind"] == "ycsb":
-        db = ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=args.flags)
+        db = ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=args.flags, device=local,
+                                rank=rank, world=world, nccl_unique_id=uid)
     else:
         # append regions: worst case of one batch + ~30% NewOrder commit rate for every batch run
         db = ltpg.tpcc_database(wl, max_txns=B, append_batches=2 + int(0.3 * (args.warmup + 2 * args.steps)),
-                                flags=args.flags)
+                                flags=args.flags, device=local, rank=rank, world=world, nccl_unique_id=uid)
     log("rank %d: db loaded in %.1fs" % (rank, time.time() - t0))
 
     # distinct input batches, cycled (inputs only; every step recomputes everything)
@@ -351,15 +360,13 @@ def main():
     torch.cuda.synchronize()
     step_ms = [a.elapsed_time(b) for a, b in ev]
     total_s = sum(step_ms) / 1000.0
+    # the global batch is partitioned over the ranks and the verdicts are exchanged, so
+    # every rank reports the same commits: count them once; time = max over ranks
+    all_commits, all_procs = float(sum(commits)), float(sum(procs))
     if dist:
         t = torch.tensor([total_s], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_s = float(t.item())
-        c = torch.tensor([float(sum(commits)), float(sum(procs))], device=dev, dtype=torch.float64)
-        dist.all_reduce(c)
-        all_commits, all_procs = c[0].item(), c[1].item()
-    else:
-        all_commits, all_procs = float(sum(commits)), float(sum(procs))
     value = all_commits / total_s
 
     # ---- timed: end to end through the public API, pinned host buffers ------------------------
@@ -387,15 +394,11 @@ def main():
             d2h += n + 4 * ((n + 31) // 32) + 4 * len(out["abort_idx"]) + 8 * nreads + 68
         torch.cuda.synchronize()
         e_s = sum(a.elapsed_time(b) for a, b in e_ev) / 1000.0
+        e_c = float(sum(e_commits))
         if dist:
             t = torch.tensor([e_s], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_s = float(t.item())
-            c = torch.tensor([float(sum(e_commits))], device=dev, dtype=torch.float64)
-            dist.all_reduce(c)
-            e_c = c[0].item()
-        else:
-            e_c = float(sum(e_commits))
         e2e = {"value": e_c / e_s, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                "d2h_bytes_per_step": d2h // args.steps, "ms_per_step": 1000 * e_s / args.steps}
 
@@ -430,9 +433,11 @@ def main():
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-            "config": dict(config_of(name), parallelism="dp%d (independent partitions)" % world
-                           if world > 1 else "single GPU"),
+            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": dict(config_of(name), parallelism=(
+                "%d partitions (%s), same global batch, per-txn verdicts exchanged by ncclAllReduce"
+                % (world, "warehouse ranges" if w["kind"] == "tpcc" else "key ranges")) if world > 1
+                else "single GPU"),
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": kernels, "roofline": roof,
             "commit_rate": all_commits / all_procs, "processed_txns_per_s": all_procs / total_s,
             "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)

@@ -307,14 +307,13 @@ def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, f
     from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY, T_ITEM
     db = Database(9, max_txns, 0, device=device, flags=flags, n_warehouses=workload.W, loopback=loopback,
                   rank=rank, world=world, nccl_unique_id=nccl_unique_id)
+    from .dist import tpcc_rank_tables
     tables = tables if tables is not None else workload.initial_tables()
+    if world > 1:
+        tables = tpcc_rank_tables(tables, workload.W, rank, world)
     extra = {T_ORDER: 1, T_NEW_ORDER: 1, T_ORDER_LINE: 15, T_HISTORY: 1}
     for t, (g, a, ng, pk) in workload.table_descs().items():
         k, c = tables[t]
-        if world > 1 and t != T_ITEM:
-            own = part_of_w(tpcc_owner_w(t, k, c), workload.W, world) == rank
-            k = None if k is None else k[own]
-            c = c[:, own]
         n = c.shape[1]
         cap = n + extra.get(t, 0) * max_txns * append_batches
         if capacity and t in capacity:

@@ -1,0 +1,43 @@
+"""Host-side plumbing for the multi-GPU path; one process per GPU.
+
+torch.distributed is only used to share the 128-byte NCCL unique id and for
+bench-side timing reductions; the per-batch exchange itself is the library's own
+ncclAllReduce on the db's communicator (csrc/capi.cu).
+"""
+import numpy as np
+
+
+def nccl_unique_id(group=None):
+    """Rank 0 creates an ncclUniqueId; every rank of `group` receives the same 128 bytes."""
+    import torch
+    import torch.distributed as dist
+    obj = [torch.cuda.nccl.unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    return obj[0]
+
+
+def warehouse_ranges(n_warehouses, world):
+    """[(lo, hi)) warehouse ids owned by each rank: the inverse of part_of_w (contiguous)."""
+    from . import part_of_w
+    w = np.arange(1, n_warehouses + 1)
+    p = part_of_w(w, n_warehouses, world)
+    return [(int(w[p == r].min()), int(w[p == r].max()) + 1) if (p == r).any() else (0, 0) for r in range(world)]
+
+
+def key_ranges(key_space, world):
+    chunk = (int(key_space) + world - 1) // world
+    return [(min(r * chunk, key_space), min((r + 1) * chunk, key_space)) for r in range(world)]
+
+
+def tpcc_rank_tables(tables, n_warehouses, rank, world):
+    """Rows of every TPC-C table that rank owns (ITEM replicated) -- what a rank loads."""
+    from . import part_of_w, tpcc_owner_w
+    out = {}
+    for t, (k, c) in tables.items():
+        ow = tpcc_owner_w(t, k, c)
+        if ow is None or world == 1:
+            out[t] = (k, c)
+            continue
+        own = part_of_w(ow, n_warehouses, world) == rank
+        out[t] = (None if k is None else k[own], c[:, own])
+    return out
