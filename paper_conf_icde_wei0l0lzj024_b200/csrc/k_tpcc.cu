@@ -41,6 +41,22 @@ __device__ __forceinline__ uint32_t probe(const DevTable& T, uint64_t key) {
   idx_find(T, key, row, claim);
   return row;
 }
+// Two-step probe so independent lookups of one lane are in flight together (the exec
+// kernel is bound by dependent index -> row -> column latency; ncu: ~32% of stall samples
+// sat on the first slot load): issue the first slot loads, then resolve them.
+__device__ __forceinline__ ulonglong2 probe_issue(const DevTable& T, uint64_t key, uint64_t& h) {
+  h = idx_hash(key, T.idx_shift);
+  return *reinterpret_cast<const ulonglong2*>(T.idx + h);
+}
+__device__ __forceinline__ uint32_t probe_finish(const DevTable& T, uint64_t key, uint64_t h, ulonglong2 v) {
+  for (uint64_t probes = 0; probes <= T.idx_mask; ++probes) {
+    if (v.x == key) return (uint32_t)v.y;
+    if (v.x == KEY_EMPTY) return ROW_NONE;
+    h = (h + 1) & T.idx_mask;
+    v = *reinterpret_cast<const ulonglong2*>(T.idx + h);
+  }
+  return ROW_NONE;
+}
 __device__ __forceinline__ long long rd(const DevTable& T, uint32_t c, uint32_t row) { return *col_ptr(T, c, row); }
 __device__ __forceinline__ void wr(const DevTable& T, uint32_t c, uint32_t row, long long v) { *col_ptr(T, c, row) = v; }
 __device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row, long long v) {
@@ -60,14 +76,17 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 
 // unit actions per phase: plain write (W mark / RW check), delayed add (A mark / A check),
 // marked read (RW check only; reads leave no mark under R1)
+// Marks: the read-before-atomicMin filter is applied to the popular tables only (P:215,
+// E = T/D > 1: WAREHOUSE and DISTRICT, thousands of accesses per row and batch); on cold
+// rows it would add a dependent DRAM round trip before a fire-and-forget RED.
 template <int PH>
-__device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
-  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter);
+__device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
+  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
 }
 template <int PH>
-__device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
-  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter);
+__device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
+  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_A, x.r, x.epoch);
 }
 template <int PH>
@@ -76,9 +95,9 @@ __device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t r
 }
 // update of column c (strict: WRITE unit of its group; delayed: ADD unit)
 template <int PH>
-__device__ __forceinline__ void col_upd(const DevTable& T, uint32_t c, uint32_t row, Tx& x) {
-  if (col_is_add(T, c)) unit_a<PH>(T, col_group(T, c), row, x);
-  else unit_w<PH>(T, col_group(T, c), row, x);
+__device__ __forceinline__ void col_upd(const DevTable& T, uint32_t c, uint32_t row, Tx& x, bool hot = false) {
+  if (col_is_add(T, c)) unit_a<PH>(T, col_group(T, c), row, x, hot);
+  else unit_w<PH>(T, col_group(T, c), row, x, hot);
 }
 // same for columns c1..c3 updated together; a unit shared by several columns is touched once
 template <int PH>
@@ -137,20 +156,25 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   }
   if (line) {
     if (PH == PH_EXEC || PH == PH_WB) {
-      const uint32_t row_i = probe(TIt, i);
+      uint64_t hi_ = 0, hs_ = 0;
+      const ulonglong2 vi = probe_issue(TIt, i, hi_);  // item and stock probes in flight together
+      ulonglong2 vs = make_ulonglong2(KEY_EMPTY, 0);
+      if (PH == PH_EXEC && own_line) vs = probe_issue(TSt, kS(sw, i), hs_);
+      const uint32_t row_i = probe_finish(TIt, i, hi_, vi);
       if (row_i == ROW_NONE) {
         ua = 1;  // unused item id: NewOrder rollback (R11)
       } else {
         amount = (long long)qty * rd(TIt, I_PRICE, row_i);
       }
-    }
-    if (PH == PH_EXEC) {
-      if (!ua && own_line) {
-        row_s = probe(TSt, kS(sw, i));
-        if (row_s == ROW_NONE) internal_error(x);
+      if (PH == PH_EXEC) {
+        if (!ua && own_line) {
+          row_s = probe_finish(TSt, kS(sw, i), hs_, vs);
+          if (row_s == ROW_NONE) internal_error(x);
+        }
+        log[sub] = row_s;
       }
-      log[sub] = row_s;
-    } else {
+    }
+    if (PH != PH_EXEC) {
       row_s = log[sub];
     }
     if (row_s != ROW_NONE) {
@@ -172,9 +196,12 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   if (home && sub == 15) {
     uint32_t row_d;
     if (PH == PH_EXEC) {
-      const uint32_t row_w = probe(TWh, w);
-      row_d = probe(TDi, kD(w, d));
-      const uint32_t row_c = probe(TCu, kC(w, d, c));
+      uint64_t hw_, hd_, hc_;
+      const ulonglong2 vw = probe_issue(TWh, w, hw_), vd = probe_issue(TDi, kD(w, d), hd_),
+                       vc = probe_issue(TCu, kC(w, d, c), hc_);
+      const uint32_t row_w = probe_finish(TWh, w, hw_, vw);
+      row_d = probe_finish(TDi, kD(w, d), hd_, vd);
+      const uint32_t row_c = probe_finish(TCu, kC(w, d, c), hc_, vc);
       if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
         internal_error(x);
         row_d = ROW_NONE;
@@ -187,7 +214,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     } else {
       row_d = log[15];
     }
-    if (row_d != ROW_NONE) unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+    if (row_d != ROW_NONE) unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
   }
   if (PH == PH_EXEC) {
     const long long sum = seg16_sum(amount);
@@ -261,13 +288,19 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   const bool home = owns_w(b, w), cust = owns_w(b, cw);
   uint32_t row_w = ROW_NONE, row_d = ROW_NONE, row_c = ROW_NONE;
   if (PH == PH_EXEC) {
+    uint64_t hw_ = 0, hd_ = 0;
+    ulonglong2 vw = make_ulonglong2(KEY_EMPTY, 0), vd = vw;
+    if (home) {  // warehouse + district probes and the by-name lookup in flight together
+      vw = probe_issue(TWh, w, hw_);
+      vd = probe_issue(TDi, kD(w, d), hd_);
+    }
+    if (cust && by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
     if (home) {
-      row_w = probe(TWh, w);
-      row_d = probe(TDi, kD(w, d));
+      row_w = probe_finish(TWh, w, hw_, vw);
+      row_d = probe_finish(TDi, kD(w, d), hd_, vd);
       if (row_w == ROW_NONE || row_d == ROW_NONE) { internal_error(x); return; }
     }
     if (cust) {
-      if (by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
       row_c = cid ? probe(TCu, kC(cw, cd, cid)) : ROW_NONE;
       if (row_c == ROW_NONE) { internal_error(x); return; }
       long long* res = b.res + 4ull * r;
@@ -287,8 +320,8 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     cid = log[3];
   }
   if (home) {
-    col_upd<PH>(TWh, W_YTD, row_w, x);
-    col_upd<PH>(TDi, D_YTD, row_d, x);
+    col_upd<PH>(TWh, W_YTD, row_w, x, true);
+    col_upd<PH>(TDi, D_YTD, row_d, x, true);
   }
   if (cust) col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, row_c, x);
   if (PH == PH_WB && home) {
@@ -400,9 +433,11 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
       internal_error(x);
     } else {
       const long long o = rd(TDi, D_NEXT_DELIV_O_ID, row_d);
-      unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x);  // RMW of the cursor
+      unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x, true);  // RMW of the cursor
       const uint64_t nok = kO(w, d, (uint64_t)o);
-      const uint32_t row_no = (PH == PH_DETECT && x.bad) ? ROW_NONE : probe(TNw, nok);
+      uint64_t hn_, ho_;
+      const ulonglong2 vn = probe_issue(TNw, nok, hn_), vo = probe_issue(TOr, nok, ho_);  // together
+      const uint32_t row_no = (PH == PH_DETECT && x.bad) ? ROW_NONE : probe_finish(TNw, nok, hn_, vn);
       if (PH == PH_DETECT && x.bad) {
         // conflict already found: the remaining checks cannot change the verdict
       } else if (row_no == ROW_NONE) {
@@ -410,7 +445,7 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
         unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
       } else {
         for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x);  // DELETE
-        const uint32_t row_o = probe(TOr, nok);
+        const uint32_t row_o = probe_finish(TOr, nok, ho_, vo);
         if (row_o == ROW_NONE) {
           internal_error(x);
         } else {
@@ -418,14 +453,19 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
           const uint32_t cid = (uint32_t)rd(TOr, O_C_ID, row_o);
           const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
           long long sum = 0;
-          for (uint32_t l = 1; l <= cnt; ++l) {
-            const uint32_t row_ol = probe(TOL_, nok * 16 + l);
-            if (row_ol == ROW_NONE) { internal_error(x); continue; }
-            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol, x);
-            sum += rd(TOL_, OL_AMOUNT, row_ol);
-            if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol, b.clock);
-          }
+          uint32_t row_ol[15];
+#pragma unroll
+          for (uint32_t l = 0; l < 15; ++l)  // all order-line probes in flight together
+            row_ol[l] = l < cnt ? probe(TOL_, nok * 16 + l + 1) : ROW_NONE;
           const uint32_t row_c = probe(TCu, kC(w, d, cid));
+#pragma unroll
+          for (uint32_t l = 0; l < 15; ++l) {
+            if (l >= cnt) continue;
+            if (row_ol[l] == ROW_NONE) { internal_error(x); continue; }
+            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[l], x);
+            sum += rd(TOL_, OL_AMOUNT, row_ol[l]);
+            if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol[l], b.clock);
+          }
           if (row_c == ROW_NONE) {
             internal_error(x);
           } else {
