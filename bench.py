@@ -139,19 +139,22 @@ def make_workload(name, rank=0):
 
 
 def exec_algorithmic_bytes(batch):
-    """Algorithmic bytes of the execute kernel for an OPS batch:
-    per op 16 B op record + 32 B index sector + 32 B data sector + 8 B result + 8 B
-    unit reference; per marking op (UPDATE/ADD/INSERT/DELETE) + 64 B (atomic sector RMW)."""
+    """Algorithmic bytes of the OPS execute kernel: per op 16 B op record +
+    32 B data sector + 8 B result + 8 B unit reference = 64 B; + 64 B per marking op
+    (UPDATE/ADD/INSERT/DELETE: atomic sector RMW).  Dense key ranges map key -> row by
+    arithmetic (identity bucket function), so no index bytes are counted."""
     kinds = batch["ops"]["kind"]
     n = len(kinds)
     marking = int(np.isin(kinds, [1, 2, 3, 4]).sum())
-    return 96 * n + 64 * marking
+    return 64 * n + 64 * marking
 
 
 def tpcc_exec_algorithmic_bytes(batch, mode):
-    """Algorithmic bytes of the TPC-C execute kernel: 128 B parameter
-    block + 32 B per random touch (index probe, column read, mark) + streams (result 32 B,
-    row log 4 B/row).  Delivery / StockLevel use the expected line counts (10 / 200)."""
+    """Algorithmic bytes of the TPC-C execute kernel: 128 B parameter block,
+    32 B per random column read or index probe of a sparse-keyed table, 64 B per mark (atomic
+    sector RMW), contiguous order lines at element size, 32 B result + 4 B per logged row.
+    W/D/C/I/S rows are found by arithmetic (dense keys); ORDER_LINE rows from ORDER.
+    Delivery / StockLevel use the expected line counts (10 / 190 distinct items)."""
     ty = batch["type"]
     p = batch["params"]
     nl = p[:, 3].astype(np.int64)
@@ -159,12 +162,12 @@ def tpcc_exec_algorithmic_bytes(batch, mode):
     by_name = p[:, 3].astype(bool)
     b = np.zeros(len(ty), np.int64)
     no = ty == 0
-    b[no] = 128 + 32 * 7 + nl[no] * (32 * (5 + delayed) + 4) + 32 + 4
+    b[no] = 128 + 3 * 32 + 64 + nl[no] * (32 + 64 * (1 + delayed) + 4) + 32 + 4
     pay = ty == 1
-    b[pay] = 128 + 32 * (6 + (not delayed)) + 4 * by_name[pay] + 16 + 32
-    b[ty == 2] = 128 + 32 * 6 + 10 * 68 + 32
-    b[ty == 3] = 128 + 10 * (32 * 4 + 32 * (8 + 10 * 3) + 32) + 32
-    b[ty == 4] = 128 + 64 + 20 * 64 + 200 * 64 + 180 * 64 + 32
+    b[pay] = 128 + 3 * 64 + 32 * (not delayed) + 4 * by_name[pay] + 16 + 32
+    b[ty == 2] = 128 + 2 * 32 + 32 + 2 * 32 + 4 + 10 * 8 + 32 + 68
+    b[ty == 3] = 128 + 10 * (32 + 64 + 32 + 32 + 3 * 32 + 4 + 64 + 10 * (8 + 16) + 64) + 32
+    b[ty == 4] = 128 + 32 + 20 * (32 + 32 + 4 + 10 * 8) + 190 * 32 + 32
     return int(b.sum())
 
 

@@ -77,6 +77,8 @@ struct ltpg_db {
   DevTable* d_tab = nullptr;
   unsigned long long* d_nrows = nullptr;   // [MAXT]
   unsigned long long* d_reserve = nullptr; // [MAXT]
+  uint32_t* d_dense_live = nullptr;        // bitmask: tables whose dense key->row mapping is valid
+  bool olrow_ready = false;                // TPC-C ORDER -> first ORDER_LINE row map built
   std::vector<Part> parts;
   // shared per-batch buffers
   unsigned long long* d_tid = nullptr;
@@ -129,6 +131,7 @@ void free_table(DevTable& T) {
   if (T.rowkey) cudaFree(T.rowkey);
   if (T.marks) cudaFree(T.marks);
   if (T.idx) cudaFree(T.idx);
+  if (T.aux) cudaFree(T.aux);
   unsigned long long* nr = T.n_rows;
   T = DevTable{};
   T.n_rows = nr;
@@ -208,6 +211,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_nrows, MAXT));
   CK(cudaMemset(db->d_nrows, 0, MAXT * sizeof(unsigned long long)));
   CK(dmalloc(&db->d_reserve, MAXT));
+  CK(dmalloc(&db->d_dense_live, 1));
+  CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
   CK(dmalloc(&db->d_tid, n));
   CK(dmalloc(&db->d_op_begin, n + 1));
@@ -262,7 +267,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
-  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_tid, db->d_op_begin, db->d_ops, db->d_args,
+  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_tid, db->d_op_begin, db->d_ops, db->d_args,
                   db->d_ptype, db->d_params, db->d_res, db->d_status, db->d_xchg, db->d_ptrs, db->d_bits,
                   db->d_flags, db->d_offs, db->d_abort, db->d_small, db->d_scan};
   for (void* p : bufs)
@@ -350,6 +355,20 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     CK(cudaMemset(T.valid, 1, n_rows));
     if (d->has_pk) CK(cudaMemcpy(T.rowkey, keys, n_rows * sizeof(uint64_t), cudaMemcpyHostToDevice));
   }
+  // dense key range: keys[r] == keys[0] + r for every loaded row
+  bool dense = d->has_pk && n_rows > 0;
+  for (uint64_t r = 1; dense && r < n_rows; ++r) dense = keys[r] == keys[0] + r;
+  T.key_base = dense ? keys[0] : 0;
+  T.dense_n = dense ? n_rows : 0;
+  uint32_t live = 0;
+  CK(cudaMemcpy(&live, db->d_dense_live, sizeof(live), cudaMemcpyDeviceToHost));
+  live = dense ? (live | (1u << t)) : (live & ~(1u << t));
+  CK(cudaMemcpy(db->d_dense_live, &live, sizeof(live), cudaMemcpyHostToDevice));
+  if (t == LTPG_T_ORDER && db->cfg.n_warehouses) {
+    CK(dmalloc(&T.aux, cap));
+    CK(cudaMemset(T.aux, 0xFF, cap * sizeof(uint32_t)));
+  }
+  if (t == LTPG_T_ORDER || t == LTPG_T_ORDER_LINE) db->olrow_ready = false;
   unsigned long long nr = n_rows;
   CK(cudaMemcpy(T.n_rows, &nr, sizeof(nr), cudaMemcpyHostToDevice));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
@@ -403,6 +422,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.nw = db->cfg.n_warehouses;
   bd.key_space = db->cfg.key_space;
   bd.reserve = db->d_reserve;
+  bd.dense_live = db->d_dense_live;
   bd.n_txns = n;
   bd.n_ops = ops_mode ? b->n_ops : 0;
   bd.epoch = db->epoch;
@@ -451,6 +471,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     upload_tables_tpcc(db->d_tab, s);
     g_uploaded[db->device % 64] = db->tab_version;
   }
+  if (!ops_mode && !db->olrow_ready) {  // ORDER -> contiguous ORDER_LINE rows (first TPC-C batch)
+    tpcc_build_olrow(s);
+    db->olrow_ready = true;
+  }
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
   std::vector<BatchDev> pb(L, bd);
@@ -468,6 +492,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     x.ins_tables = P.small + 1;
     x.kcount = P.small + 2;
     x.base = P.base;
+    x.insdel = P.small + 12;
     CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
     if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
     if (partitioned && n) {
@@ -523,7 +548,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, db->d_small, s);
+    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, db->d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
     if (partitioned && res->reads) {
       if (db->cfg.world == 1) {

@@ -199,14 +199,16 @@ void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const 
   note_launch();
 }
 
-__global__ void k_advance(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err) {
+__global__ void k_advance(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
+                          uint32_t* dense_live, const uint32_t* insdel) {
   if (*err) return;
   for (uint32_t t = 0; t < n_tables; ++t) *c_tabs[t].n_rows += reserve[t];
+  *dense_live &= ~*insdel;  // a table that saw INSERT/DELETE is looked up by hash from now on
 }
 
 void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
-                           cudaStream_t s) {
-  k_advance<<<1, 1, 0, s>>>(n_tables, reserve, err);
+                           uint32_t* dense_live, const uint32_t* insdel, cudaStream_t s) {
+  k_advance<<<1, 1, 0, s>>>(n_tables, reserve, err, dense_live, insdel);
   note_launch();
 }
 

@@ -67,7 +67,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
   bool bad = false;
   uint32_t b0 = 0, b1 = 0;
   uint64_t cnt64 = 0;  // per-kind op counts, 10 bits each (no dynamically indexed arrays)
-  uint32_t my_ins_tables = 0;
+  uint32_t my_ins_tables = 0, my_insdel = 0;
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
     b0 = b.op_begin[r];
@@ -86,6 +86,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
         tw[i] = 0;
         if (b0 + i < b1) {
           ltpg_op o = load_op(b.ops, b0 + i);
+          if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << (o.table & 31);
           if (!op_valid(n_tables, o)) bad = true;
           else if (op_touches(b, o)) {
             cnt64 += 1ull << (10 * o.kind);
@@ -109,6 +110,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
     for (uint32_t i = b0; i < b1; ++i) {
       ltpg_op o = load_op(b.ops, i);
       if (!op_valid(n_tables, o)) { bad = true; continue; }
+      if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << o.table;
       if (!op_touches(b, o)) continue;
       cnt64 += 1ull << (10 * o.kind);
       if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
@@ -134,6 +136,8 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
   }
   my_ins_tables = __reduce_or_sync(0xffffffffu, my_ins_tables);
   if (lane == 0 && my_ins_tables) atomicOr(b.ins_tables, my_ins_tables);
+  my_insdel = __reduce_or_sync(0xffffffffu, my_insdel);
+  if (lane == 0 && my_insdel) atomicOr(b.insdel, my_insdel);
   if (!GROUPED) {
     // one flat list in op order (region 0); INSERTs are still listed for K-claim
     if (r < b.n_txns)
@@ -216,7 +220,7 @@ void launch_ops_claim(const BatchDev& b, cudaStream_t s) {
 
 // ---- K-exec ---------------------------------------------------------------------------
 __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
-                                         uint32_t r, const ltpg_op& o, bool filter) {
+                                         uint32_t r, const ltpg_op& o, bool filter, uint32_t dmask) {
   const DevTable& T = c_tabs[o.table];
   const unsigned long long tag = epoch_tag(b.epoch) | r;
   uint32_t row, claim;
@@ -228,7 +232,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
     unsigned long long sum = 0;
     for (uint64_t k = o.key; k < o.key + o.aux; ++k) {
       if (!owns_key(b, T, k)) continue;  // partitioned: this partition's part of the range
-      idx_find(T, k, row, claim);
+      lookup(T, o.table, dmask, k, row, claim);
       if (row != ROW_NONE) {
         ++cnt;
         if (o.col != LTPG_COL_COUNT) sum += (unsigned long long)*col_ptr_ops(T, o.col, row);
@@ -238,7 +242,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
     b.uref[oi] = make_uref(CHK_SCAN, false, false, o.table, 0, 0);
     return;
   }
-  idx_find(T, o.key, row, claim);
+  lookup(T, o.table, dmask, o.key, row, claim);
   const bool present = row != ROW_NONE;
   if (!present && o.kind != LTPG_INSERT) {
     // absent key: a READ of its existence; only an inserter of this batch can conflict
@@ -298,6 +302,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
 template <bool GROUPED>
 __global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
   if (*b.err) return;
+  const uint32_t dmask = *b.dense_live & ~*b.insdel;
   const int lane = threadIdx.x & 31;
   uint32_t cnt[NKINDS], pref[NKINDS + 1];  // fully unrolled below: registers only
   pref[0] = 0;
@@ -319,7 +324,7 @@ __global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
     const unsigned long long it = b.items[(uint64_t)k * b.max_ops + idx];
     const uint32_t oi = (uint32_t)it, r = (uint32_t)(it >> 32);
     const ltpg_op o = load_op(b.ops, oi);
-    exec_one(b, oi, r, o, filter);
+    exec_one(b, oi, r, o, filter, dmask);
   }
 }
 
@@ -341,6 +346,7 @@ void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t 
 template <bool PART>
 __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   if (*b.err) return;
+  const uint32_t dmask = *b.dense_live & ~*b.insdel;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
@@ -357,7 +363,7 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
       for (uint64_t k = o.key; k < o.key + o.aux && !bad; ++k) {
         if (PART && !owns_key(b, T, k)) continue;
         uint32_t row, claim;
-        idx_find(T, k, row, claim);
+        lookup(T, (u >> 40) & 0xFF, dmask, k, row, claim);
         if (row != ROW_NONE) {
           uint32_t g = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
           bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);

@@ -57,6 +57,32 @@ __device__ __forceinline__ uint32_t probe_finish(const DevTable& T, uint64_t key
   }
   return ROW_NONE;
 }
+// pending lookup honouring the dense key->row mapping of W/D/C/I/S (no slot access there)
+struct PP {
+  uint64_t key, h;
+  ulonglong2 v;
+  uint32_t row;
+};
+__device__ __forceinline__ PP pp_issue(const DevTable& T, uint32_t t, uint64_t key, uint32_t dmask) {
+  PP p;
+  p.key = key;
+  if (((dmask >> t) & 1u) && key - T.key_base < T.dense_n) {
+    p.row = (uint32_t)(key - T.key_base);
+    p.h = ~0ull;
+  } else {
+    p.row = ROW_NONE;
+    p.v = probe_issue(T, key, p.h);
+  }
+  return p;
+}
+__device__ __forceinline__ uint32_t pp_finish(const DevTable& T, const PP& p) {
+  return p.h == ~0ull ? p.row : probe_finish(T, p.key, p.h, p.v);
+}
+__device__ __forceinline__ uint32_t rowof(const DevTable& T, uint32_t t, uint64_t key, uint32_t dmask) {
+  uint32_t row, claim;
+  lookup(T, t, dmask, key, row, claim);
+  return row;
+}
 __device__ __forceinline__ long long rd(const DevTable& T, uint32_t c, uint32_t row) { return *col_ptr(T, c, row); }
 __device__ __forceinline__ void wr(const DevTable& T, uint32_t c, uint32_t row, long long v) { *col_ptr(T, c, row) = v; }
 __device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row, long long v) {
@@ -64,6 +90,7 @@ __device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row
 }
 
 struct Tx {
+  uint32_t dmask;  // tables with a live dense key->row mapping
   uint32_t r;
   uint32_t epoch;
   unsigned long long tag;
@@ -156,11 +183,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   }
   if (line) {
     if (PH == PH_EXEC || PH == PH_WB) {
-      uint64_t hi_ = 0, hs_ = 0;
-      const ulonglong2 vi = probe_issue(TIt, i, hi_);  // item and stock probes in flight together
-      ulonglong2 vs = make_ulonglong2(KEY_EMPTY, 0);
-      if (PH == PH_EXEC && own_line) vs = probe_issue(TSt, kS(sw, i), hs_);
-      const uint32_t row_i = probe_finish(TIt, i, hi_, vi);
+      const PP pi = pp_issue(TIt, TI, i, x.dmask);  // item and stock lookups in flight together
+      PP ps{};
+      if (PH == PH_EXEC && own_line) ps = pp_issue(TSt, TS, kS(sw, i), x.dmask);
+      const uint32_t row_i = pp_finish(TIt, pi);
       if (row_i == ROW_NONE) {
         ua = 1;  // unused item id: NewOrder rollback (R11)
       } else {
@@ -168,7 +194,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       }
       if (PH == PH_EXEC) {
         if (!ua && own_line) {
-          row_s = probe_finish(TSt, kS(sw, i), hs_, vs);
+          row_s = pp_finish(TSt, ps);
           if (row_s == ROW_NONE) internal_error(x);
         }
         log[sub] = row_s;
@@ -196,12 +222,11 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   if (home && sub == 15) {
     uint32_t row_d;
     if (PH == PH_EXEC) {
-      uint64_t hw_, hd_, hc_;
-      const ulonglong2 vw = probe_issue(TWh, w, hw_), vd = probe_issue(TDi, kD(w, d), hd_),
-                       vc = probe_issue(TCu, kC(w, d, c), hc_);
-      const uint32_t row_w = probe_finish(TWh, w, hw_, vw);
-      row_d = probe_finish(TDi, kD(w, d), hd_, vd);
-      const uint32_t row_c = probe_finish(TCu, kC(w, d, c), hc_, vc);
+      const PP pw = pp_issue(TWh, TW, w, x.dmask), pd = pp_issue(TDi, TD, kD(w, d), x.dmask),
+               pc = pp_issue(TCu, TC, kC(w, d, c), x.dmask);
+      const uint32_t row_w = pp_finish(TWh, pw);
+      row_d = pp_finish(TDi, pd);
+      const uint32_t row_c = pp_finish(TCu, pc);
       if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
         internal_error(x);
         row_d = ROW_NONE;
@@ -251,6 +276,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       }
       if (sub == 15) {  // ORDER and NEW_ORDER rows
         const uint32_t orow = (uint32_t)(*TOr.n_rows + tp.no_flag[r]);
+        if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + tp.no_lines[r]);  // contiguous lines
         wr(TOr, O_C_ID, orow, c);
         wr(TOr, O_ENTRY_D, orow, b.clock);
         wr(TOr, O_OL_CNT, orow, n);
@@ -288,20 +314,19 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   const bool home = owns_w(b, w), cust = owns_w(b, cw);
   uint32_t row_w = ROW_NONE, row_d = ROW_NONE, row_c = ROW_NONE;
   if (PH == PH_EXEC) {
-    uint64_t hw_ = 0, hd_ = 0;
-    ulonglong2 vw = make_ulonglong2(KEY_EMPTY, 0), vd = vw;
-    if (home) {  // warehouse + district probes and the by-name lookup in flight together
-      vw = probe_issue(TWh, w, hw_);
-      vd = probe_issue(TDi, kD(w, d), hd_);
+    PP pw{}, pd{};
+    if (home) {  // warehouse + district lookups and the by-name lookup in flight together
+      pw = pp_issue(TWh, TW, w, x.dmask);
+      pd = pp_issue(TDi, TD, kD(w, d), x.dmask);
     }
     if (cust && by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
     if (home) {
-      row_w = probe_finish(TWh, w, hw_, vw);
-      row_d = probe_finish(TDi, kD(w, d), hd_, vd);
+      row_w = pp_finish(TWh, pw);
+      row_d = pp_finish(TDi, pd);
       if (row_w == ROW_NONE || row_d == ROW_NONE) { internal_error(x); return; }
     }
     if (cust) {
-      row_c = cid ? probe(TCu, kC(cw, cd, cid)) : ROW_NONE;
+      row_c = cid ? rowof(TCu, TC, kC(cw, cd, cid), x.dmask) : ROW_NONE;
       if (row_c == ROW_NONE) { internal_error(x); return; }
       long long* res = b.res + 4ull * r;
       res[0] = cid;
@@ -365,7 +390,7 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
   if (active && sub == 15) {
     if (PH == PH_EXEC) {
       cid = p[3] ? (uint32_t)tp.by_name[kD(w, d) * 1000 + p16(p, 6)] : p16(p, 4);
-      row_c = cid ? probe(TCu, kC(w, d, cid)) : ROW_NONE;
+      row_c = cid ? rowof(TCu, TC, kC(w, d, cid), x.dmask) : ROW_NONE;
       if (row_c != ROW_NONE) {
         bal = rd(TCu, C_BALANCE, row_c);
         o = (uint32_t)rd(TCu, C_INIT_O_ID, row_c);
@@ -387,13 +412,15 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
     if (row_c != ROW_NONE) unit_r<PH>(TCu, col_group(TCu, C_BALANCE), row_c, x);
     if (row_o != ROW_NONE) unit_r<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x);
   }
+  uint32_t olrow = (active && sub == 15 && row_o != ROW_NONE && TOr.aux) ? TOr.aux[row_o] : ROW_NONE;
   o = __shfl_sync(0xffffffffu, o, 15, 16);
   cnt = __shfl_sync(0xffffffffu, cnt, 15, 16);
+  olrow = __shfl_sync(0xffffffffu, olrow, 15, 16);
   long long dd = 0;
   if (active && sub < cnt && sub < 15) {
     uint32_t row_ol;
     if (PH == PH_EXEC) {
-      row_ol = probe(TOL_, kO(w, d, o) * 16 + sub + 1);
+      row_ol = olrow != ROW_NONE ? olrow + sub : probe(TOL_, kO(w, d, o) * 16 + sub + 1);
       if (row_ol == ROW_NONE) internal_error(x);
       else dd = rd(TOL_, OL_DELIVERY_D, row_ol);
       log[sub] = row_ol;
@@ -428,7 +455,7 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
     const uint32_t w = p16(p, 0);
     const long long carrier = p[2];
     const uint32_t d = sub + 1;
-    const uint32_t row_d = probe(TDi, kD(w, d));
+    const uint32_t row_d = rowof(TDi, TD, kD(w, d), x.dmask);
     if (row_d == ROW_NONE) {
       internal_error(x);
     } else {
@@ -454,10 +481,11 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
           const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
           long long sum = 0;
           uint32_t row_ol[15];
+          const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
 #pragma unroll
-          for (uint32_t l = 0; l < 15; ++l)  // all order-line probes in flight together
-            row_ol[l] = l < cnt ? probe(TOL_, nok * 16 + l + 1) : ROW_NONE;
-          const uint32_t row_c = probe(TCu, kC(w, d, cid));
+          for (uint32_t l = 0; l < 15; ++l)  // otherwise all order-line probes in flight together
+            row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, nok * 16 + l + 1)) : ROW_NONE;
+          const uint32_t row_c = rowof(TCu, TC, kC(w, d, cid), x.dmask);
 #pragma unroll
           for (uint32_t l = 0; l < 15; ++l) {
             if (l >= cnt) continue;
@@ -517,7 +545,7 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
   const uint8_t* p = b.params + 128ull * r;
   const uint32_t w = p16(p, 0), d = p[2];
   const long long thr = p[3];
-  const uint32_t row_d = probe(TDi, kD(w, d));
+  const uint32_t row_d = rowof(TDi, TD, kD(w, d), x.dmask);
   if (row_d == ROW_NONE) {
     internal_error(x);
     return;
@@ -535,10 +563,12 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
       internal_error(x);
     } else {
       const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);  // static
+      const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
       uint32_t row_ol[15];
 #pragma unroll
-      for (uint32_t l = 0; l < 15; ++l)  // independent probes issued back to back
-        row_ol[l] = l < cnt ? probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1) : ROW_NONE;
+      for (uint32_t l = 0; l < 15; ++l)  // otherwise independent probes issued back to back
+        row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1))
+                            : ROW_NONE;
 #pragma unroll
       for (uint32_t l = 0; l < 15; ++l)
         if (l < cnt) {
@@ -561,7 +591,7 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
       h = (h + 1) & (SL_HASH - 1);
     }
     if (!first) continue;  // count distinct items
-    const uint32_t row_s = probe(TSt, kS(w, it));
+    const uint32_t row_s = rowof(TSt, TS, kS(w, it), x.dmask);
     if (row_s == ROW_NONE) { internal_error(x); continue; }
     if (PH == PH_EXEC) low += rd(TSt, S_QUANTITY, row_s) < thr;
     unit_r<PH>(TSt, col_group(TSt, S_QUANTITY), row_s, x);
@@ -584,6 +614,7 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
 template <int PH>
 __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
+  const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   __shared__ uint32_t sl_items[8][SL_SLOTS];
   __shared__ uint32_t sl_set[8][SL_HASH];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -607,7 +638,7 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
     const uint32_t sub = lane % L;
     const bool active = k < ct;
     const uint32_t r = active ? tp.list[(uint64_t)t * tp.max_txns + k] : 0;
-    Tx x{r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), false, b.err};
+    Tx x{dmask, r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), false, b.err};
     bool go = active;
     if (PH == PH_WB) go = active && b.status[r] == LTPG_ST_COMMIT;
     switch (t) {
@@ -778,7 +809,7 @@ __global__ void k_no_colscan(BatchDev b, TpccParams tp) {  // one warp per distr
   }
   if (!run || lane) return;
   const DevTable& TDi = c_tabs[TD];
-  const uint32_t row_d = probe(TDi, dk);
+  const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
   if (row_d == ROW_NONE) {
     atomicOr(b.err, ERR_EINTERNAL);
     return;
@@ -816,6 +847,31 @@ __global__ void k_tpcc_advance(BatchDev b, TpccParams tp) {
   *c_tabs[TNO].n_rows += tp.no_flag[n];
   *c_tabs[TOL].n_rows += tp.no_lines[n];
   *c_tabs[TH].n_rows += tp.misc[M_HIST];
+}
+
+// ORDER.aux[row] = first ORDER_LINE row of the order if its cnt lines sit in consecutive rows
+__global__ void k_build_olrow() {
+  const DevTable& TOr = c_tabs[TO];
+  const DevTable& TOL_ = c_tabs[TOL];
+  const uint64_t n = *TOr.n_rows;
+  for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n; r += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t first = ROW_NONE;
+    if (TOr.valid[r]) {
+      const uint64_t okey = TOr.rowkey[r];
+      const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, (uint32_t)r);
+      first = probe(TOL_, okey * 16 + 1);
+      for (uint32_t l = 1; l < cnt && first != ROW_NONE; ++l) {
+        const uint64_t row = (uint64_t)first + l;
+        if (row >= *TOL_.n_rows || !TOL_.valid[row] || TOL_.rowkey[row] != okey * 16 + l + 1) first = ROW_NONE;
+      }
+    }
+    TOr.aux[r] = first;
+  }
+}
+
+void tpcc_build_olrow(cudaStream_t s) {
+  k_build_olrow<<<148 * 8, 256, 0, s>>>();
+  note_launch();
 }
 
 // ---- host side ------------------------------------------------------------------------------------

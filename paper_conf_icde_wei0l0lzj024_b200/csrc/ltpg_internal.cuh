@@ -57,7 +57,18 @@ struct DevTable {
   long long* col0;                // SoA base: column c starts at col0 + c * capacity
   uint64_t group_bits;            // 4 bits per column: group id, 15 = static
   uint32_t add_bits;              // bit c: column c is a delayed-ADD column
+  // Dense key range (detected at load): key k in [key_base, key_base + dense_n) sits at row
+  // k - key_base.  While the table has never seen an INSERT/DELETE (bit in *dense_live) a
+  // lookup there is pure arithmetic -- the identity bucket function h(key) = key mod s_h
+  // of P:217 on a dense key range -- and skips the hash-slot access.  Result-invisible (R6).
+  uint64_t key_base, dense_n;
+  uint32_t* aux;                  // TPC-C ORDER: first ORDER_LINE row of the order (ROW_NONE: probe)
 };
+
+// table lookup honouring the dense mapping: dmask = *dense_live & ~(tables with INSERT/DELETE
+// ops in this batch)
+__device__ __forceinline__ bool lookup(const DevTable& T, uint32_t t, uint32_t dmask, uint64_t key, uint32_t& row,
+                                       uint32_t& claim);
 
 __device__ __forceinline__ uint32_t col_group(const DevTable& T, uint32_t c) {
   uint32_t g = (uint32_t)(T.group_bits >> (4 * c)) & 15u;
@@ -119,6 +130,16 @@ __device__ __forceinline__ bool idx_find(const DevTable& T, uint64_t key, uint32
   row = ROW_NONE;
   claim = ROW_NONE;
   return false;
+}
+
+__device__ __forceinline__ bool lookup(const DevTable& T, uint32_t t, uint32_t dmask, uint64_t key, uint32_t& row,
+                                       uint32_t& claim) {
+  if (((dmask >> t) & 1u) && key - T.key_base < T.dense_n) {
+    row = (uint32_t)(key - T.key_base);
+    claim = ROW_NONE;
+    return true;
+  }
+  return idx_find(T, key, row, claim);
 }
 
 // Find or create the slot of `key` (load / claim paths).
@@ -193,6 +214,8 @@ struct BatchDev {
   uint8_t* lflag;                  // [n_txns] partitioned detect output
   unsigned long long* reserve;     // [MAXT] append rows reserved this batch (all partitions)
   unsigned long long* base;        // [MAXT] this partition's offset inside the reservation
+  uint32_t* dense_live;            // persistent bitmask: tables whose dense mapping is valid
+  uint32_t* insdel;                // this batch: tables receiving INSERT or DELETE ops (OPS)
   uint32_t n_txns, n_ops, epoch, flags;
   int64_t clock;
   const unsigned long long* tid;
@@ -246,7 +269,7 @@ void launch_ops_writeback(const BatchDev& b, cudaStream_t s);
 void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
                            unsigned long long* base, unsigned long long* reserve, uint32_t* err, cudaStream_t s);
 void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
-                           cudaStream_t s);
+                           uint32_t* dense_live, const uint32_t* insdel, cudaStream_t s);
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);

@@ -60,5 +60,7 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
 // front: validate + lists, capacity, execute, detect;  back: o_id prefix, write-back, cursors
 int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev);
 int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s);
+// ORDER.aux[row] = first row of the order's ORDER_LINE rows when they are contiguous
+void tpcc_build_olrow(cudaStream_t s);
 
 }  // namespace ltpg
