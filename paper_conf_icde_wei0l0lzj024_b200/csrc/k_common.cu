@@ -119,26 +119,30 @@ void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t*
 __global__ void k_finalize(const uint8_t* __restrict__ status, uint32_t n, uint32_t* __restrict__ commit_bits,
                            uint32_t* __restrict__ flags, uint32_t* __restrict__ counts,
                            const uint32_t* __restrict__ err) {
+  __shared__ uint32_t red[3];
   if (*err) return;
-  uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  uint8_t st = r < n ? status[r] : 0xFF;
-  uint32_t bits = __ballot_sync(0xffffffffu, st == LTPG_ST_COMMIT);
+  if (threadIdx.x < 3) red[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint8_t st = r < n ? status[r] : 0xFF;
+  const uint32_t bits = __ballot_sync(0xffffffffu, st == LTPG_ST_COMMIT);
   if ((threadIdx.x & 31) == 0 && r < n) commit_bits[r >> 5] = bits;
   if (r < n) flags[r] = st == LTPG_ST_CONFLICT;
-  uint32_t nc = __popc(bits);
-  uint32_t na = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_CONFLICT));
-  uint32_t nu = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_USER_ABORT));
-  if ((threadIdx.x & 31) == 0) {
-    if (nc) atomicAdd(counts + 0, nc);
-    if (na) atomicAdd(counts + 1, na);
-    if (nu) atomicAdd(counts + 2, nu);
+  const uint32_t na = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_CONFLICT));
+  const uint32_t nu = __popc(__ballot_sync(0xffffffffu, st == LTPG_ST_USER_ABORT));
+  if ((threadIdx.x & 31) == 0) {  // block-level totals: one global atomic per block and counter
+    atomicAdd(red + 0, __popc(bits));
+    atomicAdd(red + 1, na);
+    atomicAdd(red + 2, nu);
   }
+  __syncthreads();
+  if (threadIdx.x < 3 && red[threadIdx.x]) atomicAdd(counts + threadIdx.x, red[threadIdx.x]);
 }
 
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags, uint32_t* counts,
                      const uint32_t* err, cudaStream_t s) {
   if (!n) return;
-  k_finalize<<<(n + 255) / 256, 256, 0, s>>>(status, n, commit_bits, flags, counts, err);
+  k_finalize<<<(n + 1023) / 1024, 1024, 0, s>>>(status, n, commit_bits, flags, counts, err);
   note_launch();
 }
 

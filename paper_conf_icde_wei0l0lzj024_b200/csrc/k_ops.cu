@@ -151,23 +151,11 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
         }
     return;
   }
-  // warp-aggregated append into the per-kind lists: one atomicAdd per warp and kind
-  uint32_t pos[NKINDS];
+  // block-aggregated reservation in the per-kind lists: one atomicAdd per block and kind
+  uint32_t ck[NKINDS], pos[NKINDS];
 #pragma unroll
-  for (int k = 0; k < NKINDS; ++k) {
-    const uint32_t ck = (uint32_t)(cnt64 >> (10 * k)) & 1023u;
-    uint32_t x = ck;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
-    uint32_t base = 0;
-    if (lane == 31 && tot) base = atomicAdd(b.kcount + k, tot);
-    base = __shfl_sync(0xffffffffu, base, 31);
-    pos[k] = base + x - ck;
-  }
+  for (int k = 0; k < NKINDS; ++k) ck[k] = (uint32_t)(cnt64 >> (10 * k)) & 1023u;
+  block_reserve<NKINDS>(ck, b.kcount, pos);
   if (r < b.n_txns && !bad)
     for (uint32_t i = b0; i < b1; ++i) {
       const ltpg_op o = load_op(b.ops, i);

@@ -622,7 +622,7 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
   pre[0] = 0;
 #pragma unroll
   for (int t = 0; t < NTYPES; ++t) {
-    cnt[t] = b.kcount[t];
+    cnt[t] = tp.counts[t];
     const uint32_t per = 32 / (t == 1 ? 1 : (t == 4 ? 32 : 16));
     pre[t + 1] = pre[t] + (cnt[t] + per - 1) / per;
   }
@@ -662,14 +662,26 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
 
 // ---- K-tgroup: validation + per-type lists (warp-aggregated appends) ----------------------------
 __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
+  __shared__ __align__(16) uint8_t stage[8][32 * 128];
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  // the warp's 32 parameter blocks (4 KB, contiguous) staged through shared memory with
+  // coalesced 16-byte loads; each lane then parses its own block
+  const uint32_t r0 = r - lane;
+  uint8_t* sw = stage[wib];
+#pragma unroll
+  for (uint32_t k = 0; k < 8; ++k) {
+    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB
+    if (r0 + c / 8 < b.n_txns)
+      *reinterpret_cast<uint4*>(sw + 16 * c) = *reinterpret_cast<const uint4*>(b.params + 128ull * r0 + 16 * c);
+  }
+  __syncwarp();
   uint32_t t = 0xFF, lines = 0;
   bool bad = false;
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;
     t = b.ptype[r];
-    const uint8_t* p = b.params + 128ull * r;
+    const uint8_t* p = sw + 128 * lane;
     const uint32_t W = tp.nw;
     auto okw = [W](uint32_t w) { return w >= 1 && w <= W; };
     auto okd = [](uint32_t d) { return d >= 1 && d <= 10; };
@@ -678,13 +690,18 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
       case 0: {
         const uint32_t nl = p[3], c = p16(p, 4);
         if (!okd(p[2]) || nl < 1 || nl > 15 || c < 1 || c > 3000) { bad = true; break; }
-        for (uint32_t l = 0; l < nl; ++l) {
+        uint32_t it[15];
+#pragma unroll
+        for (uint32_t l = 0; l < 15; ++l) {
           const uint8_t* L = p + 8 + 8 * l;
-          const uint32_t i = p32(L, 0);
-          if (!okw(p16(L, 4)) || L[6] < 1 || L[6] > 10 || i < 1 || i > 100001) bad = true;
-          for (uint32_t m = 0; m < l; ++m)
-            if (p32(p + 8 + 8 * m, 0) == i) bad = true;  // R10: distinct items
+          it[l] = l < nl ? p32(L, 0) : 0xFFFFFFF0u - l;  // unused slots never collide
+          if (l < nl && (!okw(p16(L, 4)) || L[6] < 1 || L[6] > 10 || it[l] < 1 || it[l] > 100001)) bad = true;
         }
+#pragma unroll
+        for (uint32_t l = 1; l < 15; ++l)
+#pragma unroll
+          for (uint32_t m = 0; m < l; ++m)
+            if (it[l] == it[m]) bad = true;  // R10: distinct items (registers, unrolled)
         lines = nl;
         break;
       }
@@ -712,7 +729,7 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   bool touch = false;
   uint32_t no_home = 0, pay_cust = 0;
   if (r < b.n_txns && !bad) {
-    const uint8_t* p = b.params + 128ull * r;
+    const uint8_t* p = sw + 128 * lane;
     const bool home = owns_w(b, p16(p, 0));
     touch = home;
     if (t == 0) {
@@ -726,24 +743,40 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   } else {
     lines = 0;
   }
-  const uint32_t lsum = __reduce_add_sync(0xffffffffu, lines);
-  const uint32_t nsum = __reduce_add_sync(0xffffffffu, no_home);
-  const uint32_t psum = __reduce_add_sync(0xffffffffu, pay_cust);
-  if (lane == 0) {
-    if (lsum) atomicAdd(tp.misc + M_NO_LINES, lsum);
-    if (nsum) atomicAdd(tp.misc + M_NO, nsum);
-    if (psum) atomicAdd(tp.misc + M_PAY, psum);
-  }
+  // block-aggregated counters and per-type list positions (one atomic per block and list)
+  const uint32_t ccnt[3] = {lines, pay_cust, no_home};  // misc[M_NO_LINES], misc[M_PAY], misc[M_NO]
+  uint32_t cbase[3];
+  block_reserve<3>(ccnt, tp.misc + M_NO_LINES, cbase);
+  uint32_t tcnt[NTYPES], tbase[NTYPES];
 #pragma unroll
-  for (uint32_t k = 0; k < NTYPES; ++k) {
-    const uint32_t m = __ballot_sync(0xffffffffu, t == k && !bad && touch);
-    if (!m) continue;
-    uint32_t base = 0;
-    const uint32_t leader = __ffs(m) - 1;
-    if (lane == leader) base = atomicAdd(b.kcount + k, __popc(m));
-    base = __shfl_sync(0xffffffffu, base, leader);
-    if (t == k && !bad && touch) tp.list[(uint64_t)k * tp.max_txns + base + __popc(m & ((1u << lane) - 1))] = r;
-  }
+  for (uint32_t k = 0; k < NTYPES; ++k) tcnt[k] = (t == k && !bad && touch) ? 1u : 0u;
+  block_reserve<NTYPES>(tcnt, b.kcount, tbase);
+#pragma unroll
+  for (uint32_t k = 0; k < NTYPES; ++k)
+    if (tcnt[k]) tp.list[(uint64_t)k * tp.max_txns + tbase[k]] = r;
+}
+
+// committed entries of every per-type list -> clist (order inside a list is irrelevant)
+__global__ void __launch_bounds__(256) k_tpcc_relist(BatchDev b, TpccParams tp) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t pre[NTYPES + 1];
+  pre[0] = 0;
+#pragma unroll
+  for (int t = 0; t < NTYPES; ++t) pre[t + 1] = pre[t] + b.kcount[t];
+  uint32_t t = NTYPES, r = 0;
+#pragma unroll
+  for (int k = 0; k < NTYPES; ++k)
+    if (!*b.err && i >= pre[k] && i < pre[k + 1]) {
+      t = k;
+      r = tp.list[(uint64_t)k * tp.max_txns + (i - pre[k])];
+    }
+  uint32_t cnt[NTYPES], base[NTYPES];
+#pragma unroll
+  for (int k = 0; k < NTYPES; ++k) cnt[k] = (t == (uint32_t)k && b.status[r] == LTPG_ST_COMMIT) ? 1u : 0u;
+  block_reserve<NTYPES>(cnt, tp.misc + M_CCOUNT, base);
+#pragma unroll
+  for (int k = 0; k < NTYPES; ++k)
+    if (cnt[k]) tp.clist[(uint64_t)k * tp.max_txns + base[k]] = r;
 }
 
 // ECAPACITY before execution: worst case every NewOrder / Payment of this partition
@@ -890,7 +923,7 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
   t.owns_by_name = shared_by_name == nullptr;
   if (shared_by_name) t.by_name = shared_by_name;
   else if (dm(&t.by_name, (uint64_t)t.dsz * 1000)) return LTPG_ENOMEM;
-  if (dm(&t.list, (uint64_t)NTYPES * max_txns) ||
+  if (dm(&t.list, (uint64_t)NTYPES * max_txns) || dm(&t.clist, (uint64_t)NTYPES * max_txns) ||
       dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_flag, max_txns + 1ull) || dm(&t.no_lines, max_txns + 1ull) ||
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
     return LTPG_ENOMEM;
@@ -900,7 +933,7 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
 
 void tpcc_free(TpccDev& t) {
   if (!t.owns_by_name) t.by_name = nullptr;
-  void* ps[] = {t.by_name, t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
+  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
   for (void* p : ps)
     if (p) cudaFree(p);
   t = TpccDev{};
@@ -929,8 +962,10 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
              : LTPG_ECUDA;
 }
 
-static TpccParams params_of(TpccDev& t, uint32_t n) {
-  return TpccParams{t.list, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
+static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists) {
+  const uint32_t n = b.n_txns;
+  return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
+                    t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
 }
 static uint32_t phase_grid(uint32_t n) {
@@ -941,7 +976,7 @@ static uint32_t phase_grid(uint32_t n) {
 int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   if (!t.nw) return LTPG_EINVAL;
   const uint32_t n = b.n_txns;
-  const TpccParams tp = params_of(t, n);
+  const TpccParams tp = params_of(t, b, false);
   cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
   k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   k_tpcc_capacity<<<1, 1, 0, s>>>(b, tp);
@@ -958,7 +993,10 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
 
 int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   const uint32_t n = b.n_txns;
-  const TpccParams tp = params_of(t, n);
+  const TpccParams tp = params_of(t, b, false);
+  // committed txns re-listed per type: write-back warps only visit committed txns
+  k_tpcc_relist<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
+  note_launch();
   // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders
   k_no_prep<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   note_launch();
@@ -969,7 +1007,7 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  k_tpcc_phase<PH_WB><<<phase_grid(n), 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_WB><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));
   k_tpcc_advance<<<1, 1, 0, s>>>(b, tp);
   note_launch(2);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;

@@ -22,7 +22,7 @@ enum { I_PRICE = 0, I_IM_ID = 1 };
 enum { S_QUANTITY = 0, S_YTD = 1, S_ORDER_CNT = 2, S_REMOTE_CNT = 3 };
 
 // counters in TpccDev::misc (M_NO / M_NO_LINES / M_PAY: inserts this partition may append)
-enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3 };
+enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3, M_CCOUNT = 8 };
 
 struct TpccDev {
   uint32_t max_txns = 0;
@@ -31,6 +31,7 @@ struct TpccDev {
   int* by_name = nullptr;       // dense secondary index [(w*10+d)*1000 + c_last] -> c_id (0: none)
   bool owns_by_name = false;    // loopback partitions share partition 0's index
   uint32_t* list = nullptr;     // [NTYPES][max_txns] ranks, grouped by procedure type
+  uint32_t* clist = nullptr;    // [NTYPES][max_txns] committed ranks (write-back only)
   uint32_t* log = nullptr;      // [max_txns][TLOG] rows found by execute
   uint32_t* no_flag = nullptr;  // [max_txns+1] committed NewOrder -> exclusive scan (row offsets)
   uint32_t* no_lines = nullptr; // [max_txns+1] committed NewOrder lines -> exclusive scan
@@ -41,7 +42,9 @@ struct TpccDev {
 };
 
 struct TpccParams {
+  uint32_t* clist;              // committed re-list target (k_tpcc_relist)
   uint32_t* list;
+  const uint32_t* counts;       // per-type list lengths of `list` (kcount, or misc + M_CCOUNT)
   uint32_t* log;
   uint32_t* no_flag;
   uint32_t* no_lines;
