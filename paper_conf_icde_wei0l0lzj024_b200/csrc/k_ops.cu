@@ -62,74 +62,73 @@ __device__ __forceinline__ bool op_touches(const BatchDev& b, const ltpg_op& o) 
 template <bool GROUPED>
 __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
                                                             BatchDev b) {
+  constexpr uint32_t STAGE = 352;  // ops per warp staged in shared memory (YCSB: 32 x 10 = 320)
+  __shared__ __align__(16) ltpg_op stage[8][STAGE];
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   const int lane = threadIdx.x & 31;
+  const uint32_t wib = threadIdx.x >> 5;
   bool bad = false;
   uint32_t b0 = 0, b1 = 0;
   uint64_t cnt64 = 0;  // per-kind op counts, 10 bits each (no dynamically indexed arrays)
   uint32_t my_ins_tables = 0, my_insdel = 0;
+  // the warp's ops form one contiguous range: stage it with coalesced 16-byte loads
+  const uint32_t r0 = r - lane;
+  const uint32_t rl = min(r0 + 32, b.n_txns);
+  uint32_t w0 = 0, w1 = 0;
+  if (r0 < b.n_txns) {
+    w0 = b.op_begin[r0];
+    w1 = b.op_begin[rl];
+  }
+  const bool staged = r0 < b.n_txns && w1 >= w0 && w1 - w0 <= STAGE && w1 <= b.n_ops;
+  if (staged)
+    for (uint32_t q = w0 + lane; q < w1; q += 32)
+      *reinterpret_cast<ulonglong2*>(&stage[wib][q - w0]) = *reinterpret_cast<const ulonglong2*>(b.ops + q);
+  __syncwarp();
+  auto get = [&](uint32_t q) -> ltpg_op {
+    if (staged) {
+      const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(&stage[wib][q - w0]);
+      ltpg_op o;
+      o.key = v.x;
+      o.kind = (uint8_t)(v.y);
+      o.table = (uint8_t)(v.y >> 8);
+      o.col = (uint16_t)(v.y >> 16);
+      o.aux = (uint32_t)(v.y >> 32);
+      return o;
+    }
+    return load_op(b.ops, q);
+  };
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
     b0 = b.op_begin[r];
     b1 = b.op_begin[r + 1];
     if (r == 0 && b0 != 0) bad = true;
     if (r == b.n_txns - 1 && b1 != b.n_ops) bad = true;
-    if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS) { bad = true; b1 = b0; }
-    constexpr int FAST = 16;
-    if (b1 - b0 <= FAST) {
-      // short txns (YCSB, micro-cases): ops held in registers, R10 pairs fully unrolled
-      uint64_t lo[FAST], hi[FAST];
-      uint32_t tw[FAST];  // table | is_write << 8 | is_scan << 9 | valid slot << 10
-#pragma unroll
-      for (int i = 0; i < FAST; ++i) {
-        lo[i] = hi[i] = 0;
-        tw[i] = 0;
-        if (b0 + i < b1) {
-          ltpg_op o = load_op(b.ops, b0 + i);
-          if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << (o.table & 31);
-          if (!op_valid(n_tables, o)) bad = true;
-          else if (op_touches(b, o)) {
-            cnt64 += 1ull << (10 * o.kind);
-            if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
-          }
-          lo[i] = o.key;
-          hi[i] = o.kind == LTPG_SCAN ? o.key + o.aux : o.key + 1;
-          tw[i] = o.table | (uint32_t)is_write_kind(o.kind) << 8 | (uint32_t)(o.kind == LTPG_SCAN) << 9 | 1u << 10;
-        }
-      }
-#pragma unroll
-      for (int i = 1; i < FAST; ++i)
-#pragma unroll
-        for (int j = 0; j < i; ++j) {
-          const bool same = (tw[i] & 0x4FF) == (tw[j] & 0x4FF) && (tw[i] & 0x400);
-          const bool overlap = lo[i] < hi[j] && lo[j] < hi[i];
-          const bool forbid = ((tw[i] | tw[j]) & 0x100) || !((tw[i] | tw[j]) & 0x200);
-          if (same && overlap && forbid) bad = true;
-        }
-    } else {
+    if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS || (staged && (b0 < w0 || b1 > w1))) {
+      bad = true;
+      b1 = b0;
+    }
     for (uint32_t i = b0; i < b1; ++i) {
-      ltpg_op o = load_op(b.ops, i);
+      const ltpg_op o = get(i);
+      if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << (o.table & 31);
       if (!op_valid(n_tables, o)) { bad = true; continue; }
-      if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << o.table;
       if (!op_touches(b, o)) continue;
       cnt64 += 1ull << (10 * o.kind);
       if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
     }
     // R10: a written key is touched by no other op of the txn (no read-your-writes)
     for (uint32_t i = b0 + 1; i < b1 && !bad; ++i) {
-      ltpg_op a = load_op(b.ops, i);
-      uint64_t alo = a.key, ahi = a.kind == LTPG_SCAN ? a.key + a.aux : a.key + 1;
+      const ltpg_op a = get(i);
+      const uint64_t alo = a.key, ahi = a.kind == LTPG_SCAN ? a.key + a.aux : a.key + 1;
       for (uint32_t j = b0; j < i; ++j) {
-        ltpg_op c = load_op(b.ops, j);
+        const ltpg_op c = get(j);
         if (c.table != a.table) continue;
-        uint64_t clo = c.key, chi = c.kind == LTPG_SCAN ? c.key + c.aux : c.key + 1;
+        const uint64_t clo = c.key, chi = c.kind == LTPG_SCAN ? c.key + c.aux : c.key + 1;
         if (!(alo < chi && clo < ahi)) continue;
         if (is_write_kind(a.kind) || is_write_kind(c.kind) || (a.kind != LTPG_SCAN && c.kind != LTPG_SCAN)) {
           bad = true;
           break;
         }
       }
-    }
     }
     b.txn_ins[r] = (uint32_t)(cnt64 >> (10 * LTPG_INSERT)) & 1023u;
     if (bad) atomicOr(b.err, ERR_EINVAL);
