@@ -187,7 +187,16 @@ typedef struct {
   int64_t batch_clock;          /* deterministic "now" for TPC-C dates                    */
   int inputs_on_device;         /* 1: the pointers above are device pointers             */
   void* stream;                 /* cudaStream_t to run on (NULL = legacy default)         */
+  uint32_t flags;               /* LTPG_BATCH_*                                           */
 } ltpg_batch;
+
+/* Inter-batch pipeline: with LTPG_BATCH_ASYNC, ltpg_run_batch enqueues the batch and
+ * returns; host inputs are uploaded on an internal copy stream while the previous batch's
+ * kernels run, and host outputs are downloaded on a second copy stream while the next batch's
+ * kernels run.  At most two batches are in flight; ltpg_wait_batch(db, result) completes the
+ * batch submitted with `result` and returns its status code.  Host buffers of an async batch
+ * must stay valid (and unmodified) until then.  Batches still execute in submission order. */
+#define LTPG_BATCH_ASYNC 1u
 
 typedef struct {
   float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;
@@ -205,8 +214,12 @@ typedef struct {
   ltpg_stats* stats;            /* optional host struct: per-stage device times           */
 } ltpg_result;
 
-/* Run one batch; synchronous on batch->stream (returns when results are in place). */
+/* Run one batch; synchronous on batch->stream (returns when results are in place)
+ * unless batch->flags has LTPG_BATCH_ASYNC. */
 LTPG_API int ltpg_run_batch(ltpg_db* db, const ltpg_batch* batch, ltpg_result* result);
+
+/* Complete an asynchronously submitted batch (see LTPG_BATCH_ASYNC). */
+LTPG_API int ltpg_wait_batch(ltpg_db* db, ltpg_result* result);
 
 /* Canonical dump (valid rows only): keyed tables sorted by key, keyless tables by
  * the full column tuple.  Call with keys == cols == NULL to get *n_rows only.

@@ -53,7 +53,7 @@ class ltpg_table_desc(ctypes.Structure):
 class ltpg_batch(ctypes.Structure):
     _fields_ = [("n_txns", c_u32), ("tid", c_vp), ("mode", c_u32), ("n_ops", c_u32), ("op_begin", c_vp),
                 ("ops", c_vp), ("op_arg", c_vp), ("proc_type", c_vp), ("proc_params", c_vp),
-                ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp)]
+                ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp), ("flags", c_u32)]
 
 
 class ltpg_stats(ctypes.Structure):
@@ -83,6 +83,8 @@ _lib.ltpg_destroy_db.restype = None
 _lib.ltpg_destroy_db.argtypes = [c_vp]
 _lib.ltpg_last_error.restype = ctypes.c_char_p
 _lib.ltpg_last_error.argtypes = [c_vp]
+_lib.ltpg_wait_batch.restype = c_int
+_lib.ltpg_wait_batch.argtypes = [c_vp, ctypes.POINTER(ltpg_result)]
 _lib.ltpg_version.restype = ctypes.c_char_p
 _lib.ltpg_version.argtypes = []
 
@@ -94,9 +96,11 @@ ltpg_dump_table = _lib.ltpg_dump_table
 ltpg_destroy_db = _lib.ltpg_destroy_db
 ltpg_last_error = _lib.ltpg_last_error
 ltpg_version = _lib.ltpg_version
+ltpg_wait_batch = _lib.ltpg_wait_batch
+LTPG_BATCH_ASYNC = 1
 
-EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_dump_table", "ltpg_destroy_db",
-            "ltpg_last_error", "ltpg_version"]
+EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
+            "ltpg_destroy_db", "ltpg_last_error", "ltpg_version"]
 
 
 class LtpgError(RuntimeError):
@@ -188,7 +192,7 @@ class Database:
                 "abort_idx": np.empty(max(n, 1), np.uint32), "n_aborted": np.zeros(1, np.uint32),
                 "reads": np.empty(max(n_reads, 1), np.int64)}
 
-    def _run(self, bt, n, n_reads, want_reads, device_out, stats, out):
+    def _run(self, bt, n, n_reads, want_reads, device_out, stats, out, wait=True, keep=None):
         if out is None:
             out = self._outputs(n, n_reads, device_out)
         st = ltpg_stats() if stats else None
@@ -197,7 +201,14 @@ class Database:
                           reads=_ptr(out["reads"]) if want_reads else None,
                           outputs_on_device=int(device_out),
                           stats=ctypes.pointer(st) if st is not None else None)
+        if not wait:
+            bt.flags |= LTPG_BATCH_ASYNC
+            self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))
+            return Pending(self, res, bt, st, out, n, n_reads, want_reads, device_out, keep)
         self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))
+        return self._collect(out, n, n_reads, want_reads, device_out, st)
+
+    def _collect(self, out, n, n_reads, want_reads, device_out, st):
         out = dict(out)
         if not device_out:
             na = int(out["n_aborted"][0])
@@ -208,7 +219,7 @@ class Database:
         return out
 
     def run_ops(self, batch, stream=None, want_reads=True, device_out=None, stats=False, out=None,
-                n_txns=None, n_ops=None):
+                n_txns=None, n_ops=None, wait=True):
         """batch: dict(tid u64[n], op_begin u32[n+1], ops OP_DTYPE/uint8[n_ops*16], args i64[n_ops]).
         Pass n_txns / n_ops when the arrays are raw byte views."""
         tid, ob, ops, args = batch["tid"], batch["op_begin"], batch["ops"], batch["args"]
@@ -220,10 +231,10 @@ class Database:
         bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_OPS, n_ops=n_ops, op_begin=_ptr(ob),
                         ops=_ptr(ops), op_arg=_ptr(args), inputs_on_device=int(on_dev),
                         stream=c_vp(stream) if stream else None)
-        return self._run(bt, n, n_ops, want_reads, device_out, stats, out)
+        return self._run(bt, n, n_ops, want_reads, device_out, stats, out, wait, keep=batch)
 
     def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
-                 n_txns=None):
+                 n_txns=None, wait=True):
         """batch: dict(tid u64[n], type u8[n], params u8[n,128])."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
         n = len(tid) if n_txns is None else n_txns
@@ -233,8 +244,8 @@ class Database:
         bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
                         proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
                         stream=c_vp(stream) if stream else None)
-        out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out)
-        if not device_out and want_reads:
+        out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch)
+        if wait and not device_out and want_reads:
             out["reads"] = out["reads"].reshape(n, 4)
         return out
 
@@ -249,6 +260,19 @@ class Database:
         self._check(ltpg_dump_table(self.h, t, ctypes.byref(nr), _ptr(keys), _ptr(colbuf)))
         cols = colbuf[:nc * n].reshape(nc, n)
         return (keys[:n] if self.has_pk[t] else None), cols
+
+
+class Pending:
+    """An asynchronously submitted batch (LTPG_BATCH_ASYNC): .wait() completes it."""
+
+    def __init__(self, db, res, bt, st, out, n, n_reads, want_reads, device_out, keep):
+        self.db, self.res, self.bt, self.st, self.out = db, res, bt, st, out
+        self.args = (n, n_reads, want_reads, device_out)
+        self.keep = keep  # host buffers must stay alive until the batch completes
+
+    def wait(self):
+        self.db._check(ltpg_wait_batch(self.db.h, ctypes.byref(self.res)))
+        return self.db._collect(self.out, *self.args, self.st)
 
 
 def part_of_w(w, nw, nparts):

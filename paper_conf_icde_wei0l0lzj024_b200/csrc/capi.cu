@@ -61,6 +61,29 @@ struct Part {
   TpccDev tpcc;
 };
 
+// one in-flight batch: input staging, device outputs, pinned small results, events
+struct Slot {
+  unsigned long long* d_tid = nullptr;
+  uint32_t* d_op_begin = nullptr;
+  ltpg_op* d_ops = nullptr;
+  long long* d_args = nullptr;
+  uint8_t* d_ptype = nullptr;
+  uint8_t* d_params = nullptr;
+  long long* d_res = nullptr;              // combined results
+  uint8_t* d_status = nullptr;
+  uint32_t* d_bits = nullptr;
+  uint32_t* d_flags = nullptr;
+  uint32_t* d_offs = nullptr;
+  uint32_t* d_abort = nullptr;
+  uint32_t* d_small = nullptr;             // [0] err (combined) [8..10] counts
+  uint32_t* h_small = nullptr;             // pinned: [0..15] d_small, [16] n_aborted
+  cudaEvent_t ev[8]{};
+  cudaEvent_t h2d_done = nullptr, comp_done = nullptr, out_done = nullptr;
+  bool pending = false, timing = false, host_out = false;
+  ltpg_result* res = nullptr;
+  uint64_t launches0 = 0;
+};
+
 }  // namespace
 
 struct ltpg_db {
@@ -80,26 +103,15 @@ struct ltpg_db {
   uint32_t* d_dense_live = nullptr;        // bitmask: tables whose dense key->row mapping is valid
   bool olrow_ready = false;                // TPC-C ORDER -> first ORDER_LINE row map built
   std::vector<Part> parts;
-  // shared per-batch buffers
-  unsigned long long* d_tid = nullptr;
-  uint32_t* d_op_begin = nullptr;
-  ltpg_op* d_ops = nullptr;
-  long long* d_args = nullptr;
-  uint8_t* d_ptype = nullptr;
-  uint8_t* d_params = nullptr;
-  long long* d_res = nullptr;              // combined results
-  uint8_t* d_status = nullptr;
   uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
-  uint32_t* d_bits = nullptr;
-  uint32_t* d_flags = nullptr;
-  uint32_t* d_offs = nullptr;
-  uint32_t* d_abort = nullptr;
-  uint32_t* d_small = nullptr;             // [0] err (combined) [8..10] counts
   uint32_t* d_scan = nullptr;
-  uint32_t* h_small = nullptr;             // pinned
+  // inter-batch pipeline (NEXT-2): two slots, each with its own input staging and
+  // output buffers, so batch n+1's H2D and batch n-1's D2H overlap batch n's kernels
+  Slot slots[2];
+  uint64_t submitted = 0;
+  cudaStream_t h2d = nullptr, d2h = nullptr;
   ncclComm_t comm = nullptr;
-  cudaEvent_t ev[8]{};
 };
 
 namespace {
@@ -214,24 +226,31 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_dense_live, 1));
   CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
-  CK(dmalloc(&db->d_tid, n));
-  CK(dmalloc(&db->d_op_begin, n + 1));
-  CK(dmalloc(&db->d_ops, m));
-  CK(dmalloc(&db->d_args, m));
-  CK(dmalloc(&db->d_ptype, n));
-  CK(dmalloc(&db->d_params, n * LTPG_PARAM_BYTES));
-  CK(dmalloc(&db->d_res, nres));
-  CK(dmalloc(&db->d_status, n));
+  for (Slot& S : db->slots) {
+    CK(dmalloc(&S.d_tid, n));
+    CK(dmalloc(&S.d_op_begin, n + 1));
+    CK(dmalloc(&S.d_ops, m));
+    CK(dmalloc(&S.d_args, m));
+    CK(dmalloc(&S.d_ptype, n));
+    CK(dmalloc(&S.d_params, n * LTPG_PARAM_BYTES));
+    CK(dmalloc(&S.d_res, nres));
+    CK(dmalloc(&S.d_status, n));
+    CK(dmalloc(&S.d_bits, (n + 31) / 32 + 1));
+    CK(dmalloc(&S.d_flags, n));
+    CK(dmalloc(&S.d_offs, n + 1));
+    CK(dmalloc(&S.d_abort, n));
+    CK(dmalloc(&S.d_small, 64));
+    CK(cudaMallocHost(reinterpret_cast<void**>(&S.h_small), 64 * sizeof(uint32_t)));
+    for (auto& e : S.ev) CK(cudaEventCreate(&e));
+    CK(cudaEventCreate(&S.h2d_done));
+    CK(cudaEventCreate(&S.comp_done));
+    CK(cudaEventCreate(&S.out_done));
+  }
   CK(dmalloc(&db->d_xchg, n + 4));
   CK(dmalloc(&db->d_ptrs, 3 * 64));
-  CK(dmalloc(&db->d_bits, (n + 31) / 32 + 1));
-  CK(dmalloc(&db->d_flags, n));
-  CK(dmalloc(&db->d_offs, n + 1));
-  CK(dmalloc(&db->d_abort, n));
-  CK(dmalloc(&db->d_small, 64));
   CK(dmalloc(&db->d_scan, scan_scratch_words(std::max<size_t>(n, m)) + 16));
-  CK(cudaMallocHost(reinterpret_cast<void**>(&db->h_small), 64 * sizeof(uint32_t)));
-  for (auto& e : db->ev) CK(cudaEventCreate(&e));
+  CK(cudaStreamCreateWithFlags(&db->h2d, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&db->d2h, cudaStreamNonBlocking));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
   db->parts.resize(loop);
   std::vector<void*> ptrs(3 * 64, nullptr);
@@ -267,20 +286,28 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
-  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_tid, db->d_op_begin, db->d_ops, db->d_args,
-                  db->d_ptype, db->d_params, db->d_res, db->d_status, db->d_xchg, db->d_ptrs, db->d_bits,
-                  db->d_flags, db->d_offs, db->d_abort, db->d_small, db->d_scan};
+  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_xchg, db->d_ptrs, db->d_scan};
   for (void* p : bufs)
     if (p) cudaFree(p);
+  for (Slot& S : db->slots) {
+    void* sb[] = {S.d_tid, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_res, S.d_status,
+                  S.d_bits, S.d_flags, S.d_offs, S.d_abort, S.d_small};
+    for (void* p : sb)
+      if (p) cudaFree(p);
+    if (S.h_small) cudaFreeHost(S.h_small);
+    for (auto& e : S.ev)
+      if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : {S.h2d_done, S.comp_done, S.out_done})
+      if (e) cudaEventDestroy(e);
+  }
+  if (db->h2d) cudaStreamDestroy(db->h2d);
+  if (db->d2h) cudaStreamDestroy(db->d2h);
   for (Part& P : db->parts) {
     void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.small, P.base};
     for (void* p : pb)
       if (p) cudaFree(p);
     tpcc_free(P.tpcc);
   }
-  if (db->h_small) cudaFreeHost(db->h_small);
-  for (auto& e : db->ev)
-    if (e) cudaEventDestroy(e);
   if (db->comm) g_nccl.commDestroy(db->comm);
   delete db;
 }
@@ -374,13 +401,14 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
   db->tab_version = ++g_tab_versions;
   if (d->has_pk && n_rows) {
-    CK(cudaMemset(db->d_small, 0, sizeof(uint32_t)));
+    uint32_t* d_err = db->slots[0].d_small;
+    CK(cudaMemset(d_err, 0, sizeof(uint32_t)));
     upload_tables_common(db->d_tab, 0);
     g_uploaded[db->device % 64] = 0;
-    launch_build_index(t, 0, n_rows, db->d_small, 0);
+    launch_build_index(t, 0, n_rows, d_err, 0);
     CK(cudaGetLastError());
     uint32_t err = 0;
-    CK(cudaMemcpy(&err, db->d_small, sizeof(err), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&err, d_err, sizeof(err), cudaMemcpyDeviceToHost));
     if (err) {
       free_table(T);
       cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice);
@@ -393,6 +421,49 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   }
   CK(cudaDeviceSynchronize());
   return LTPG_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+// Complete the batch held by slot S: wait for its outputs, report errors / counts / stages.
+int finish_slot(ltpg_db* db, Slot& S) {
+  S.pending = false;
+  CK(cudaEventSynchronize(S.out_done));
+  const uint32_t err = S.h_small[0];
+  if (err & ERR_EINTERNAL) return fail(db, LTPG_EINTERNAL, "device invariant violated");
+  if (err & ERR_EINVAL) return fail(db, LTPG_EINVAL, "invalid batch (validated on device; nothing changed)");
+  if (err & ERR_ECAPACITY) return fail(db, LTPG_ECAPACITY, "append capacity exceeded (nothing changed)");
+  if (S.host_out) *S.res->n_aborted = S.h_small[16];
+  if (S.timing) {
+    ltpg_stats* st = S.res->stats;
+    float ms[7] = {0};
+    for (int i = 0; i < 6; ++i) CK(cudaEventElapsedTime(&ms[i], S.ev[i], S.ev[i + 1]));
+    CK(cudaEventElapsedTime(&ms[6], S.ev[6], S.out_done));
+    st->ms_upload = ms[0];
+    st->ms_group = ms[1];
+    st->ms_exec = ms[2];
+    st->ms_detect = ms[3];
+    st->ms_exchange = ms[4];
+    st->ms_writeback = ms[5];
+    st->ms_download = ms[6];
+    st->n_commit = S.h_small[8];
+    st->n_conflict = S.h_small[9];
+    st->n_user_abort = S.h_small[10];
+  }
+  return LTPG_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int ltpg_wait_batch(ltpg_db* db, ltpg_result* res) {
+  if (!db || !res) return LTPG_EINVAL;
+  for (Slot& S : db->slots)
+    if (S.pending && S.res == res) return finish_slot(db, S);
+  return fail(db, LTPG_EINVAL, "no batch in flight for this result");
 }
 
 int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
@@ -408,15 +479,21 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     return fail(db, LTPG_EINVAL, "bad OPS batch");
   if (!ops_mode && (!b->proc_type || !b->proc_params || !db->cfg.n_warehouses))
     return fail(db, LTPG_EINVAL, "bad TPCC batch");
+  Slot& S = db->slots[db->submitted & 1];
+  if (S.pending) return fail(db, LTPG_EINVAL, "two batches already in flight: ltpg_wait_batch first");
+  ++db->submitted;
   CK(cudaSetDevice(db->device));
   cudaStream_t s = static_cast<cudaStream_t>(b->stream);
+  const bool async = (b->flags & LTPG_BATCH_ASYNC) != 0;
   const bool timing = res->stats != nullptr;
   const bool partitioned = db->nparts > 1;
   const uint32_t L = db->loopback;
-  if (timing) CK(cudaEventRecord(db->ev[0], s));
+  S.timing = timing;
+  S.res = res;
+  S.host_out = !res->outputs_on_device;
+  S.launches0 = g_kernel_launches;
   ++db->epoch;
-  const uint64_t launches0 = g_kernel_launches;
-  // ---- a1: upload ---------------------------------------------------------------------
+  // ---- a1: upload on the copy stream (overlaps the previous batch's kernels) ------------------
   BatchDev bd{};
   bd.nparts = db->nparts;
   bd.nw = db->cfg.n_warehouses;
@@ -429,7 +506,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.flags = db->cfg.flags;
   bd.clock = b->batch_clock;
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
-  bd.status = db->d_status;
+  bd.status = S.d_status;
   const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
   if (b->inputs_on_device) {
     bd.tid = reinterpret_cast<const unsigned long long*>(b->tid);
@@ -439,29 +516,36 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     bd.ptype = b->proc_type;
     bd.params = b->proc_params;
   } else {
-    CK(cudaMemcpyAsync(db->d_tid, b->tid, n * sizeof(uint64_t), h2d, s));
-    bd.tid = db->d_tid;
+    // the slot's staging buffers are free once its previous batch's kernels are done
+    CK(cudaStreamWaitEvent(db->h2d, S.comp_done, 0));
+    CK(cudaMemcpyAsync(S.d_tid, b->tid, n * sizeof(uint64_t), h2d, db->h2d));
+    bd.tid = S.d_tid;
     if (ops_mode) {
-      CK(cudaMemcpyAsync(db->d_op_begin, b->op_begin, (n + 1) * sizeof(uint32_t), h2d, s));
+      CK(cudaMemcpyAsync(S.d_op_begin, b->op_begin, (n + 1) * sizeof(uint32_t), h2d, db->h2d));
       if (b->n_ops) {
-        CK(cudaMemcpyAsync(db->d_ops, b->ops, b->n_ops * sizeof(ltpg_op), h2d, s));
-        CK(cudaMemcpyAsync(db->d_args, b->op_arg, b->n_ops * sizeof(int64_t), h2d, s));
+        CK(cudaMemcpyAsync(S.d_ops, b->ops, b->n_ops * sizeof(ltpg_op), h2d, db->h2d));
+        CK(cudaMemcpyAsync(S.d_args, b->op_arg, b->n_ops * sizeof(int64_t), h2d, db->h2d));
       }
-      bd.op_begin = db->d_op_begin;
-      bd.ops = db->d_ops;
-      bd.args = db->d_args;
+      bd.op_begin = S.d_op_begin;
+      bd.ops = S.d_ops;
+      bd.args = S.d_args;
     } else {
-      CK(cudaMemcpyAsync(db->d_ptype, b->proc_type, n, h2d, s));
-      CK(cudaMemcpyAsync(db->d_params, b->proc_params, (size_t)n * LTPG_PARAM_BYTES, h2d, s));
-      bd.ptype = db->d_ptype;
-      bd.params = db->d_params;
+      CK(cudaMemcpyAsync(S.d_ptype, b->proc_type, n, h2d, db->h2d));
+      CK(cudaMemcpyAsync(S.d_params, b->proc_params, (size_t)n * LTPG_PARAM_BYTES, h2d, db->h2d));
+      bd.ptype = S.d_ptype;
+      bd.params = S.d_params;
     }
+    CK(cudaEventRecord(S.h2d_done, db->h2d));
   }
+  // kernels of this batch: after its upload and after the slot's previous outputs were read
+  CK(cudaStreamWaitEvent(s, S.out_done, 0));
+  if (timing) CK(cudaEventRecord(S.ev[0], s));
+  if (!b->inputs_on_device) CK(cudaStreamWaitEvent(s, S.h2d_done, 0));
   const size_t n_reads = ops_mode ? b->n_ops : (size_t)n * LTPG_PROC_RESULTS;
   const bool reads_dev = res->reads && res->outputs_on_device;
-  long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : db->d_res;
-  uint32_t* counts = db->d_small + 8;
-  CK(cudaMemsetAsync(db->d_small, 0, 16 * sizeof(uint32_t), s));
+  long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : S.d_res;
+  uint32_t* counts = S.d_small + 8;
+  CK(cudaMemsetAsync(S.d_small, 0, 16 * sizeof(uint32_t), s));
   CK(cudaMemsetAsync(db->d_reserve, 0, MAXT * sizeof(unsigned long long), s));
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
@@ -500,12 +584,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
     }
   }
-  if (timing) CK(cudaEventRecord(db->ev[1], s));
+  if (timing) CK(cudaEventRecord(S.ev[1], s));
   if (n) {
     // ---- a1..a6 per partition: validate + warp division, claims, execute + marks, detect --------
     for (uint32_t p = 0; p < L; ++p) {
       BatchDev& x = pb[p];
-      cudaEvent_t* evp = (timing && p == L - 1) ? db->ev : nullptr;
+      cudaEvent_t* evp = (timing && p == L - 1) ? S.ev : nullptr;
       if (ops_mode) {
         launch_ops_validate_group(db->n_tables, x, grouped, s);
         scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
@@ -520,27 +604,28 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (timing) CK(cudaEventRecord(db->ev[4], s));
+    if (timing) CK(cudaEventRecord(S.ev[4], s));
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
       if (db->cfg.world == 1) {
-        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, db->d_status, db->d_ptrs + 64, db->d_small);
-        k_spread_err<<<1, 1, 0, s>>>(db->d_small, db->d_ptrs + 64, L);
+        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, S.d_status, db->d_ptrs + 64, S.d_small);
+        k_spread_err<<<1, 1, 0, s>>>(S.d_small, db->d_ptrs + 64, L);
         note_launch(2);
       } else {
         k_pack<<<(n + 255) / 256, 256, 0, s>>>(pb[0].lflag, pb[0].err, db->d_xchg, n);
         ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, n + 3, ncclUint8, ncclMax, db->comm, s);
         if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
-        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, db->d_status, pb[0].err, db->d_small);
+        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, S.d_status, pb[0].err, S.d_small);
         note_launch(2);
       }
     } else {
-      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, db->d_small);
+      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, S.d_small);
       note_launch();
     }
-    if (timing) CK(cudaEventRecord(db->ev[5], s));
+    if (timing) CK(cudaEventRecord(S.ev[5], s));
     // ---- a7: write-back per partition -------------------------------------------------------
     for (uint32_t p = 0; p < L; ++p) {
+      pb[p].status = S.d_status;
       if (ops_mode) {
         launch_ops_writeback(pb[p], s);
       } else {
@@ -548,7 +633,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, db->d_small, db->d_dense_live, pb[0].insdel, s);
+    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
     if (partitioned && res->reads) {
       if (db->cfg.world == 1) {
@@ -560,57 +645,35 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       }
     }
     // ---- finalize: commit bitmask, abort list -------------------------------------------------
-    launch_finalize(db->d_status, n, db->d_bits, db->d_flags, counts, db->d_small, s);
-    scan_exclusive_u32(db->d_flags, db->d_offs, n, db->d_scan, s);
-    launch_compact(db->d_flags, db->d_offs, n, db->d_abort, s);
+    launch_finalize(S.d_status, n, S.d_bits, S.d_flags, counts, S.d_small, s);
+    scan_exclusive_u32(S.d_flags, S.d_offs, n, db->d_scan, s);
+    launch_compact(S.d_flags, S.d_offs, n, S.d_abort, s);
   }
   CK(cudaGetLastError());
-  if (timing) CK(cudaEventRecord(db->ev[6], s));
-  // ---- a8: results ------------------------------------------------------------------------
-  const cudaMemcpyKind out_kind = res->outputs_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
-  CK(cudaMemcpyAsync(db->h_small, db->d_small, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+  if (timing) CK(cudaEventRecord(S.ev[6], s));
+  CK(cudaEventRecord(S.comp_done, s));
+  // ---- a8: results: D2H on the copy stream (overlaps the next batch's kernels) ------------------
+  cudaStream_t os = S.host_out ? db->d2h : s;
+  if (S.host_out) CK(cudaStreamWaitEvent(db->d2h, S.comp_done, 0));
+  const cudaMemcpyKind out_kind = S.host_out ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  CK(cudaMemcpyAsync(S.h_small, S.d_small, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
   if (n) {
-    CK(cudaMemcpyAsync(db->h_small + 16, db->d_offs + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(res->status, db->d_status, n, out_kind, s));
-    CK(cudaMemcpyAsync(res->commit_bits, db->d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, s));
-    if (res->reads && !reads_dev) CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, s));
-    if (res->outputs_on_device) {
-      CK(cudaMemcpyAsync(res->n_aborted, db->d_offs + n, sizeof(uint32_t), out_kind, s));
-      CK(cudaMemcpyAsync(res->abort_idx, db->d_abort, n * sizeof(uint32_t), out_kind, s));
-    }
+    CK(cudaMemcpyAsync(S.h_small + 16, S.d_offs + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
+    CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));
+    CK(cudaMemcpyAsync(res->commit_bits, S.d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, os));
+    if (res->reads && !reads_dev) CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
+    CK(cudaMemcpyAsync(res->abort_idx, S.d_abort, n * sizeof(uint32_t), out_kind, os));
+    if (!S.host_out) CK(cudaMemcpyAsync(res->n_aborted, S.d_offs + n, sizeof(uint32_t), out_kind, os));
   } else {
-    db->h_small[16] = 0;
+    CK(cudaMemsetAsync(S.d_offs, 0, sizeof(uint32_t), s));
+    CK(cudaMemcpyAsync(S.h_small + 16, S.d_offs, sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
+    if (!S.host_out) CK(cudaMemcpyAsync(res->n_aborted, S.d_offs, sizeof(uint32_t), out_kind, os));
   }
-  CK(cudaStreamSynchronize(s));
-  const uint32_t err = db->h_small[0];
-  if (err & ERR_EINTERNAL) return fail(db, LTPG_EINTERNAL, "device invariant violated");
-  if (err & ERR_EINVAL) return fail(db, LTPG_EINVAL, "invalid batch (validated on device; nothing changed)");
-  if (err & ERR_ECAPACITY) return fail(db, LTPG_ECAPACITY, "append capacity exceeded (nothing changed)");
-  const uint32_t n_ab = db->h_small[16];
-  if (!res->outputs_on_device) {
-    *res->n_aborted = n_ab;
-    if (n_ab) CK(cudaMemcpyAsync(res->abort_idx, db->d_abort, n_ab * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-  }
-  if (timing) {
-    CK(cudaEventRecord(db->ev[7], s));
-    CK(cudaEventSynchronize(db->ev[7]));
-    ltpg_stats* st = res->stats;
-    float ms[7] = {0};
-    for (int i = 0; i < 7; ++i) CK(cudaEventElapsedTime(&ms[i], db->ev[i], db->ev[i + 1]));
-    st->ms_upload = ms[0];
-    st->ms_group = ms[1];
-    st->ms_exec = ms[2];
-    st->ms_detect = ms[3];
-    st->ms_exchange = ms[4];
-    st->ms_writeback = ms[5];
-    st->ms_download = ms[6];
-    st->n_commit = db->h_small[8];
-    st->n_conflict = db->h_small[9];
-    st->n_user_abort = db->h_small[10];
-    st->n_kernels = (uint32_t)(g_kernel_launches - launches0);
-  }
-  return LTPG_OK;
+  CK(cudaEventRecord(S.out_done, os));
+  if (timing) res->stats->n_kernels = (uint32_t)(g_kernel_launches - S.launches0);
+  S.pending = true;
+  if (async) return LTPG_OK;
+  return finish_slot(db, S);
 }
 
 int ltpg_dump_table(ltpg_db* db, uint32_t t, uint64_t* n_rows_out, uint64_t* keys, int64_t* cols) {
