@@ -188,12 +188,16 @@ typedef struct {
   int inputs_on_device;         /* 1: the pointers above are device pointers             */
   void* stream;                 /* cudaStream_t to run on (NULL = legacy default)         */
   uint32_t flags;               /* LTPG_BATCH_*                                           */
+  const uint32_t* proc_offsets; /* TPCC, optional [n_txns+1]: proc_params is PACKED -- txn r's
+                                   block is bytes [off[r], off[r+1]) (<= 128, the used prefix
+                                   of its 128-byte block; the rest reads as zero).  NULL: fixed
+                                   128-byte blocks.  Cuts the host->device bytes ~2x.       */
 } ltpg_batch;
 
 /* Inter-batch pipeline: with LTPG_BATCH_ASYNC, ltpg_run_batch enqueues the batch and
  * returns; host inputs are uploaded on an internal copy stream while the previous batch's
  * kernels run, and host outputs are downloaded on a second copy stream while the next batch's
- * kernels run.  At most two batches are in flight; ltpg_wait_batch(db, result) completes the
+ * kernels run.  At most three batches are in flight; ltpg_wait_batch(db, result) completes the
  * batch submitted with `result` and returns its status code.  Host buffers of an async batch
  * must stay valid (and unmodified) until then.  Batches still execute in submission order. */
 #define LTPG_BATCH_ASYNC 1u

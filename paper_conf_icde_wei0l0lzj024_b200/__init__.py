@@ -53,7 +53,8 @@ class ltpg_table_desc(ctypes.Structure):
 class ltpg_batch(ctypes.Structure):
     _fields_ = [("n_txns", c_u32), ("tid", c_vp), ("mode", c_u32), ("n_ops", c_u32), ("op_begin", c_vp),
                 ("ops", c_vp), ("op_arg", c_vp), ("proc_type", c_vp), ("proc_params", c_vp),
-                ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp), ("flags", c_u32)]
+                ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp), ("flags", c_u32),
+                ("proc_offsets", c_vp)]
 
 
 class ltpg_stats(ctypes.Structure):
@@ -235,15 +236,17 @@ class Database:
 
     def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
                  n_txns=None, wait=True):
-        """batch: dict(tid u64[n], type u8[n], params u8[n,128])."""
+        """batch: dict(tid u64[n], type u8[n], params u8[n,128]) -- or packed blocks:
+        params = used bytes back to back and offsets u32[n+1] (see pack_params)."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
+        offsets = batch.get("offsets")
         n = len(tid) if n_txns is None else n_txns
         on_dev = _on_device(tid)
         if device_out is None:
             device_out = on_dev
         bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
                         proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
-                        stream=c_vp(stream) if stream else None)
+                        stream=c_vp(stream) if stream else None, proc_offsets=_ptr(offsets))
         out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch)
         if wait and not device_out and want_reads:
             out["reads"] = out["reads"].reshape(n, 4)
@@ -260,6 +263,25 @@ class Database:
         self._check(ltpg_dump_table(self.h, t, ctypes.byref(nr), _ptr(keys), _ptr(colbuf)))
         cols = colbuf[:nc * n].reshape(nc, n)
         return (keys[:n] if self.has_pk[t] else None), cols
+
+
+# used prefix of each TPC-C parameter block (include/ltpg.h layouts)
+_USED = {0: None, 1: 24, 2: 8, 3: 4, 4: 4}
+
+
+def pack_params(types, params):
+    """Pack 128-byte TPC-C parameter blocks to their used prefixes (client side).
+    Returns (packed u8[total], offsets u32[n+1]); NewOrder uses 8 + 8 * n_lines bytes."""
+    types = np.asarray(types)
+    params = np.asarray(params, dtype=np.uint8).reshape(len(types), 128)
+    used = np.zeros(len(types), np.int64)
+    for t, u in _USED.items():
+        m = types == t
+        used[m] = 8 + 8 * params[m, 3].astype(np.int64) if u is None else u
+    offs = np.zeros(len(types) + 1, np.int64)
+    np.cumsum(used, out=offs[1:])
+    mask = np.arange(128)[None, :] < used[:, None]
+    return params[mask], offs.astype(np.uint32)
 
 
 class Pending:

@@ -69,6 +69,8 @@ struct Slot {
   long long* d_args = nullptr;
   uint8_t* d_ptype = nullptr;
   uint8_t* d_params = nullptr;
+  uint8_t* d_packed = nullptr;             // packed parameter blocks (proc_offsets)
+  uint32_t* d_offsets = nullptr;
   long long* d_res = nullptr;              // combined results
   uint8_t* d_status = nullptr;
   uint32_t* d_bits = nullptr;
@@ -106,9 +108,9 @@ struct ltpg_db {
   uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_scan = nullptr;
-  // inter-batch pipeline (NEXT-2): two slots, each with its own input staging and
+  // inter-batch pipeline (NEXT-2): three slots, each with its own input staging and
   // output buffers, so batch n+1's H2D and batch n-1's D2H overlap batch n's kernels
-  Slot slots[2];
+  Slot slots[3];
   uint64_t submitted = 0;
   cudaStream_t h2d = nullptr, d2h = nullptr;
   ncclComm_t comm = nullptr;
@@ -233,6 +235,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&S.d_args, m));
     CK(dmalloc(&S.d_ptype, n));
     CK(dmalloc(&S.d_params, n * LTPG_PARAM_BYTES));
+    CK(dmalloc(&S.d_packed, n * LTPG_PARAM_BYTES));
+    CK(dmalloc(&S.d_offsets, n + 1));
     CK(dmalloc(&S.d_res, nres));
     CK(dmalloc(&S.d_status, n));
     CK(dmalloc(&S.d_bits, (n + 31) / 32 + 1));
@@ -290,7 +294,8 @@ void ltpg_destroy_db(ltpg_db* db) {
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
-    void* sb[] = {S.d_tid, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_res, S.d_status,
+    void* sb[] = {S.d_tid, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_packed, S.d_offsets,
+                  S.d_res, S.d_status,
                   S.d_bits, S.d_flags, S.d_offs, S.d_abort, S.d_small};
     for (void* p : sb)
       if (p) cudaFree(p);
@@ -479,8 +484,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     return fail(db, LTPG_EINVAL, "bad OPS batch");
   if (!ops_mode && (!b->proc_type || !b->proc_params || !db->cfg.n_warehouses))
     return fail(db, LTPG_EINVAL, "bad TPCC batch");
-  Slot& S = db->slots[db->submitted & 1];
-  if (S.pending) return fail(db, LTPG_EINVAL, "two batches already in flight: ltpg_wait_batch first");
+  Slot& S = db->slots[db->submitted % 3];
+  if (S.pending) return fail(db, LTPG_EINVAL, "three batches already in flight: ltpg_wait_batch first");
   ++db->submitted;
   CK(cudaSetDevice(db->device));
   cudaStream_t s = static_cast<cudaStream_t>(b->stream);
@@ -531,7 +536,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       bd.args = S.d_args;
     } else {
       CK(cudaMemcpyAsync(S.d_ptype, b->proc_type, n, h2d, db->h2d));
-      CK(cudaMemcpyAsync(S.d_params, b->proc_params, (size_t)n * LTPG_PARAM_BYTES, h2d, db->h2d));
+      if (b->proc_offsets) {  // packed blocks: offsets + used bytes only, expanded on the GPU
+        const uint64_t packed = b->proc_offsets[n];
+        if (packed > (uint64_t)n * LTPG_PARAM_BYTES) return fail(db, LTPG_EINVAL, "packed params too large");
+        CK(cudaMemcpyAsync(S.d_offsets, b->proc_offsets, (n + 1) * sizeof(uint32_t), h2d, db->h2d));
+        CK(cudaMemcpyAsync(S.d_packed, b->proc_params, packed, h2d, db->h2d));
+      } else {
+        CK(cudaMemcpyAsync(S.d_params, b->proc_params, (size_t)n * LTPG_PARAM_BYTES, h2d, db->h2d));
+      }
       bd.ptype = S.d_ptype;
       bd.params = S.d_params;
     }
@@ -540,12 +552,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // kernels of this batch: after its upload and after the slot's previous outputs were read
   CK(cudaStreamWaitEvent(s, S.out_done, 0));
   if (timing) CK(cudaEventRecord(S.ev[0], s));
+  CK(cudaMemsetAsync(S.d_small, 0, 16 * sizeof(uint32_t), s));
   if (!b->inputs_on_device) CK(cudaStreamWaitEvent(s, S.h2d_done, 0));
+  const bool packed_params = !ops_mode && b->proc_offsets;
+  if (packed_params) bd.params = S.d_params;
   const size_t n_reads = ops_mode ? b->n_ops : (size_t)n * LTPG_PROC_RESULTS;
   const bool reads_dev = res->reads && res->outputs_on_device;
   long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : S.d_res;
   uint32_t* counts = S.d_small + 8;
-  CK(cudaMemsetAsync(S.d_small, 0, 16 * sizeof(uint32_t), s));
   CK(cudaMemsetAsync(db->d_reserve, 0, MAXT * sizeof(unsigned long long), s));
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
@@ -582,6 +596,15 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (partitioned && n) {
       CK(cudaMemsetAsync(P.res, 0, n_reads * sizeof(long long), s));
       CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
+    }
+  }
+  if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> every partition)
+    const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
+    const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
+    launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
+    for (uint32_t p = 1; p < L; ++p) {
+      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, pb[p].err);
+      note_launch();
     }
   }
   if (timing) CK(cudaEventRecord(S.ev[1], s));

@@ -146,6 +146,34 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
   note_launch();
 }
 
+// packed TPC-C parameter blocks -> fixed 128-byte blocks (zero-filled tails); one warp per
+// 8 txns, 16-byte lanes
+__global__ void k_unpack_params(const uint8_t* __restrict__ packed, const uint32_t* __restrict__ offs, uint32_t n,
+                                uint8_t* __restrict__ params, uint32_t* err) {
+  const uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const uint32_t r = (uint32_t)(g >> 3), q = (uint32_t)(g & 7);  // txn, 16-byte quarter
+  if (r >= n) return;
+  const uint32_t o0 = offs[r], o1 = offs[r + 1];
+  if (o1 < o0 || o1 - o0 > LTPG_PARAM_BYTES) {
+    if (q == 0) atomicOr(err, ERR_EINVAL);
+    return;
+  }
+  uint8_t v[16];
+#pragma unroll
+  for (int k = 0; k < 16; ++k) {
+    const uint32_t at = q * 16 + k;
+    v[k] = at < o1 - o0 ? packed[o0 + at] : 0;
+  }
+  *reinterpret_cast<uint4*>(params + 128ull * r + 16 * q) = *reinterpret_cast<const uint4*>(v);
+}
+
+void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t n, uint8_t* params, uint32_t* err,
+                          cudaStream_t s) {
+  if (!n) return;
+  k_unpack_params<<<(unsigned)((8ull * n + 255) / 256), 256, 0, s>>>(packed, offs, n, params, err);
+  note_launch();
+}
+
 // abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
 __global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ offs, uint32_t n,
                           uint32_t* __restrict__ out) {

@@ -307,6 +307,8 @@ void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const 
                            unsigned long long* base, unsigned long long* reserve, uint32_t* err, cudaStream_t s);
 void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,
                            uint32_t* dense_live, const uint32_t* insdel, cudaStream_t s);
+void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t n, uint8_t* params, uint32_t* err,
+                          cudaStream_t s);
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);

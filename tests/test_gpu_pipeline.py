@@ -68,14 +68,13 @@ def test_tpcc_pipeline_full_mix():
         assert (gc == oc).all(), t
 
 
-def test_three_in_flight_rejected():
+def test_four_in_flight_rejected():
     wl = YcsbWorkload(1000, theta=0.5, ops_per_txn=4, seed=2)
     g = L().ycsb_database(wl, max_txns=512, max_ops=2048)
-    b = [wl.batch(256, 1 + 256 * i, i) for i in range(3)]
-    p0 = g.run_ops(b[0], wait=False)
-    p1 = g.run_ops(b[1], wait=False)
+    b = [wl.batch(256, 1 + 256 * i, i) for i in range(4)]
+    ps = [g.run_ops(b[i], wait=False) for i in range(3)]
     with pytest.raises(L().LtpgError):
-        g.run_ops(b[2], wait=False)
-    p0.wait()
-    p1.wait()
-    g.run_ops(b[2]).get("status")
+        g.run_ops(b[3], wait=False)
+    for p_ in ps:
+        p_.wait()
+    g.run_ops(b[3]).get("status")

@@ -125,3 +125,27 @@ def test_delivery_heavy():
         compare(g, o, batch, 2 + bno)
     dumps = compare_tables(g, o)
     assert all(tpcc_cc.check(dumps).values())
+
+
+def test_packed_params_equal_fixed_blocks():
+    """proc_offsets: packed parameter blocks (used prefixes only) give the same results."""
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=17, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=2048, tables=tables, append_batches=4)
+    o = oracle.tpcc_db(wl, tables)
+    for bno in range(3):
+        b = wl.batch(2000, 1 + 2000 * bno, bno)
+        packed, offs = lib.pack_params(b["type"], b["params"])
+        assert packed.nbytes < b["params"].nbytes * 0.6
+        pb = {"tid": b["tid"], "type": b["type"], "params": packed, "offsets": offs}
+        out = g.run_tpcc(pb, 2 + bno)
+        rc, st, res = o.run_tpcc(b, 2 + bno)
+        assert (out["status"] == st).all() and (out["reads"] == res).all()
+    compare_tables(g, o)
+    bad = dict(pb)
+    bad["offsets"] = offs.copy()
+    bad["offsets"][1:] += 200  # first block 200+ bytes long
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(bad, 9)
+    assert e.value.rc == lib.LTPG_EINVAL
