@@ -36,6 +36,7 @@ def lib():
         L.orc_create.restype = vp
         L.orc_create.argtypes = [u32, u32]
         L.orc_destroy.argtypes = [vp]
+        L.orc_set_reorder.argtypes = [vp, ip]
         L.orc_define_table.restype = ip
         L.orc_define_table.argtypes = [vp, u32, u32, vp, vp, u32, u32]
         L.orc_load_table.restype = ip
@@ -65,6 +66,10 @@ class OracleDB:
         self.L = lib()
         self.h = self.L.orc_create(n_tables, n_warehouses)
         self.has_pk = {}
+
+    def set_reorder(self, on=True):
+        """NEXT-1 logical reordering: abort iff WAW or (RAW and WAR)."""
+        self.L.orc_set_reorder(self.h, int(bool(on)))
 
     def close(self):
         if self.h:

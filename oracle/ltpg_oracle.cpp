@@ -116,12 +116,20 @@ struct Db {
   std::unordered_map<uint64_t, int64_t> by_name;
   bool by_name_built = false;
   std::vector<double> stage_ns;
+  bool reorder = false;  // NEXT-1 logical reordering
 };
 
 // ---------------------------------------------------------------------------
 // O2 + O3: marks and the commit rule.
 // ---------------------------------------------------------------------------
-void decide(const std::vector<TxnExec>& ex, std::vector<uint8_t>& status) {
+//   reorder = false (hot path, R1):  abort iff WAW or RAW
+//   reorder = true  (NEXT-1, logical reordering P:237 / Aria P:80):  abort iff WAW or (RAW and WAR)
+// with, for txn r:
+//   WAW: a unit r writes was written or added to by a smaller rank, or a unit r adds to was
+//        plainly written by a smaller rank (ADD-ADD commute, R7)
+//   RAW: a unit r reads was written or added to by a smaller rank
+//   WAR: a unit r writes or adds to was read by a smaller rank
+void decide(const std::vector<TxnExec>& ex, std::vector<uint8_t>& status, bool reorder) {
   const uint32_t n = ex.size();
   std::unordered_map<Unit, uint32_t, UnitHash> minR, minW, minA;  // P:219 "two kinds of TIDs"
   auto mark = [](std::unordered_map<Unit, uint32_t, UnitHash>& m, const Unit& u, uint32_t r) {
@@ -141,16 +149,20 @@ void decide(const std::vector<TxnExec>& ex, std::vector<uint8_t>& status) {
   };
   status.assign(n, ST_COMMIT);
   for (uint32_t r = 0; r < n; ++r) {
-    bool abort = false;
+    bool waw = false, raw = false, war = false;
     for (const Access& a : ex[r].acc) {
-      uint32_t w = get(minW, a.u);
-      if (a.acc == ACC_A) {
-        if (w < r) abort = true;                         // WAW against a plain writer
+      const uint32_t w = get(minW, a.u), ad = get(minA, a.u), rd = get(minR, a.u);
+      if (a.acc == ACC_R) {
+        if (std::min(w, ad) < r) raw = true;
+      } else if (a.acc == ACC_W) {
+        if (std::min(w, ad) < r) waw = true;
+        if (rd < r) war = true;
       } else {
-        uint32_t m = std::min(w, get(minA, a.u));
-        if (m < r) abort = true;                         // RAW / WAW (R1)
+        if (w < r) waw = true;
+        if (rd < r) war = true;
       }
     }
+    const bool abort = reorder ? (waw || (raw && war)) : (waw || raw);
     status[r] = abort ? ST_CONFLICT : (ex[r].user_abort ? ST_USER_ABORT : ST_COMMIT);
   }
 }
@@ -632,6 +644,9 @@ void* orc_create(uint32_t n_tables, uint32_t n_warehouses) {
 
 void orc_destroy(void* h) { delete static_cast<Db*>(h); }
 
+// NEXT-1: logical reordering (commit rule WAW or (RAW and WAR) aborts)
+void orc_set_reorder(void* h, int on) { static_cast<Db*>(h)->reorder = on != 0; }
+
 int orc_define_table(void* h, uint32_t t, uint32_t n_cols, const uint8_t* group, const uint8_t* is_add,
                      uint32_t n_groups, uint32_t has_pk) {
   Db& db = *static_cast<Db*>(h);
@@ -683,7 +698,7 @@ int orc_run_ops(void* h, uint32_t n, const uint64_t* tid, const uint32_t* op_beg
     for (uint32_t i = op_begin[r]; i < op_begin[r + 1]; ++i)
       exec_op(db, read_op(ops + 16ull * i), args[i], ex[r], &reads[i]);
   std::vector<uint8_t> st;
-  decide(ex, st);  // O2 + O3
+  decide(ex, st, db.reorder);  // O2 + O3
   for (uint32_t r = 0; r < n; ++r) {  // O4 in TID order
     status[r] = st[r];
     if (st[r] != ST_COMMIT) continue;
@@ -716,9 +731,9 @@ int orc_run_tpcc(void* h, uint32_t n, const uint64_t* tid, const uint8_t* type, 
     if (!x.ok) return ORC_EINTERNAL;
   }
   std::vector<uint8_t> st;
-  decide(ex, st);  // O2 + O3
-  for (uint32_t r = 0; r < n; ++r) {  // O4 in TID order
-    status[r] = st[r];
+  decide(ex, st, db.reorder);  // O2 + O3
+  for (uint32_t r = 0; r < n; ++r) {  // O4: committed write sets (a unit has at most one plain
+    status[r] = st[r];               // writer; adds commute; fetch pre-images in TID order)
     if (st[r] != ST_COMMIT) continue;
     for (const Effect& e : ex[r].eff)
       if (apply_effect(db, e)) return ORC_EINTERNAL;

@@ -38,7 +38,7 @@ def example3(encoding):
     g = json.load(open(os.path.join(GOLDEN, "example3.json")))
     key = g["table"]["key"]
     init = g["table"]["initial"]
-    if encoding == "row_level_no_optimizations":
+    if encoding in ("row_level_no_optimizations", "row_level_reordering"):
         desc = ([0, 0], [0, 0], 1)
         wkind = UPDATE
     elif encoding == "split_only_write":

@@ -120,20 +120,24 @@ class Model:
         return res, R, W, A, eff, ua
 
 
-def brute_force_batch(model, batch):
-    """Pairwise-definition commit decision on snapshot `model`; returns (status, reads, final)."""
+def brute_force_batch(model, batch, reorder=False):
+    """Pairwise-definition commit decision on snapshot `model`; returns (status, reads, final).
+
+    base rule:   abort iff WAW or RAW against a smaller rank;
+    reorder:     abort iff WAW or (RAW and WAR)  (P:237 logical reordering, Aria)."""
     n = len(batch["tid"])
     execs = [model.exec_txn(batch, r) for r in range(n)]  # all against the snapshot
     status = []
     for r in range(n):
         _, Rr, Wr, Ar, _, ua = execs[r]
-        ok = True
+        waw = raw = war = False
         for j in range(r):
             _, Rj, Wj, Aj, _, _ = execs[j]
-            if ((Wj | Aj) & (Rr | Wr)) or (Wj & Ar):
-                ok = False
-                break
-        status.append(ST_CONFLICT if not ok else (ST_USER_ABORT if ua else ST_COMMIT))
+            waw |= bool(((Wj | Aj) & Wr) or (Wj & Ar))
+            raw |= bool((Wj | Aj) & Rr)
+            war |= bool(Rj & (Wr | Ar))
+        bad = (waw or (raw and war)) if reorder else (waw or raw)
+        status.append(ST_CONFLICT if bad else (ST_USER_ABORT if ua else ST_COMMIT))
     final = model.copy()
     for r in range(n):
         if status[r] == ST_COMMIT:
@@ -142,11 +146,43 @@ def brute_force_batch(model, batch):
     return status, reads, final
 
 
-def serial_replay(model, batch, status):
-    """Apply committed txns one at a time in TID order, each seeing its predecessors."""
+def logical_order(model, batch, status):
+    """Committed txns in a serial order consistent with snapshot reads: a txn that read a
+    unit precedes every committed txn that writes or adds to it (Kahn's algorithm, ties by
+    TID).  Raises if the dependency graph has a cycle (the commit rule would be unsound)."""
+    import heapq
+    com = [r for r in range(len(batch["tid"])) if status[r] == ST_COMMIT]
+    sets = {r: model.exec_txn(batch, r) for r in com}
+    succ = {r: set() for r in com}
+    indeg = {r: 0 for r in com}
+    for a in com:
+        for b in com:
+            if a != b and sets[a][1] & (sets[b][2] | sets[b][3]):  # a reads what b changes
+                if b not in succ[a]:
+                    succ[a].add(b)
+                    indeg[b] += 1
+    heap = [r for r in com if indeg[r] == 0]
+    heapq.heapify(heap)
+    order = []
+    while heap:
+        r = heapq.heappop(heap)
+        order.append(r)
+        for b in succ[r]:
+            indeg[b] -= 1
+            if indeg[b] == 0:
+                heapq.heappush(heap, b)
+    if len(order) != len(com):
+        raise AssertionError("cycle among committed txns")
+    return order
+
+
+def serial_replay(model, batch, status, order=None):
+    """Apply committed txns one at a time (TID order, or `order`), each seeing its predecessors."""
     cur = model.copy()
     reads = {}
-    for r in range(len(batch["tid"])):
+    if order is None:
+        order = [r for r in range(len(batch["tid"])) if status[r] == ST_COMMIT]
+    for r in order:
         if status[r] != ST_COMMIT:
             continue
         res, _, _, _, eff, ua = cur.exec_txn(batch, r)

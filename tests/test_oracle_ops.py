@@ -26,10 +26,12 @@ def make_db(descs, tables):
 
 
 @pytest.mark.parametrize("encoding", ["row_level_no_optimizations", "split_only_write",
-                                      "split_and_delayed_update"])
+                                      "split_and_delayed_update", "row_level_reordering"])
 def test_example3(encoding):
     descs, tables, batch, g = opscases.example3(encoding)
     db = make_db(descs, tables)
+    if encoding == "row_level_reordering":
+        db.set_reorder(True)
     rc, status, reads = db.run_ops(batch)
     assert rc == 0
     committed = [i + 1 for i, s in enumerate(status) if s == ST_COMMIT]
@@ -190,3 +192,44 @@ def _concat(a, b):
     return {"tid": np.concatenate([a["tid"], b["tid"]]), "ops": np.concatenate([a["ops"], b["ops"]]),
             "args": np.concatenate([a["args"], b["args"]]),
             "op_begin": np.concatenate([a["op_begin"], b["op_begin"][1:] + a["op_begin"][-1]]).astype(np.uint32)}
+
+
+def test_example3_reordering_logical_order():
+    """with logical reordering the serial order is Tx1, Tx3, Tx5, Tx2."""
+    descs, tables, batch, g = opscases.example3("row_level_reordering")
+    db = make_db(descs, tables)
+    db.set_reorder(True)
+    rc, status, reads = db.run_ops(batch)
+    model = _model_from(descs, tables)
+    order = pymodel.logical_order(model, batch, list(status))
+    assert [r + 1 for r in order] == g["expected_logical_order"]["row_level_reordering"]["value"]
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_brute_force_reordering(seed):
+    """NEXT-1: oracle with logical reordering == pairwise definition (WAW or (RAW and WAR)),
+    and the committed set replays serially in a reader-before-writer topological order."""
+    rng = np.random.default_rng(7000 + seed)
+    tables = opscases.rand_tables(rng)
+    batch = opscases.rand_batch(rng, int(rng.integers(1, 40)))
+    db = make_db(opscases.RAND_DESCS, tables)
+    db.set_reorder(True)
+    rc, status, reads = db.run_ops(batch)
+    assert rc == 0
+    model = _model_from(opscases.RAND_DESCS, tables)
+    bst, breads, bfinal = pymodel.brute_force_batch(model, batch, reorder=True)
+    assert list(status) == bst
+    assert list(reads) == breads
+    order = pymodel.logical_order(model, batch, list(status))
+    sreads, sfinal = pymodel.serial_replay(model, batch, list(status), order)
+    ob = batch["op_begin"]
+    for r, res in sreads.items():
+        assert list(reads[ob[r]:ob[r + 1]]) == res, r
+    for t in opscases.RAND_DESCS:
+        k, c = db.dump_table(t)
+        mk, mc = _dump_model(sfinal, t)
+        assert (k == mk).all() and (c == mc).all()
+    # reordering never commits fewer txns than the base rule on the same batch
+    db2 = make_db(opscases.RAND_DESCS, tables)
+    _, st2, _ = db2.run_ops(batch)
+    assert (status == ST_COMMIT).sum() >= (st2 == ST_COMMIT).sum()
