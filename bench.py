@@ -41,6 +41,9 @@ WORKLOADS = {
     "tpcc_c4": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="strict"),
     "tpcc_c5": dict(kind="tpcc", cfg=4, W=512, mix="no_pay", batch=1 << 20, mode="strict"),
     "tpcc_c4_delayed": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="delayed"),
+    # NEXT-1 "high-contention package": delayed update + logical reordering
+    "tpcc_c4_opt": dict(kind="tpcc", cfg=3, W=64, mix="full", batch=1 << 20, mode="delayed", reorder=True),
+    "tpcc_c2_opt": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed", reorder=True),
     "tpcc_c2_delayed": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed"),
     "ycsb_c3_4ops": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=4, batch=1 << 20),
 }
@@ -188,6 +191,8 @@ def run_reference(args, name):
         db = oracle.ycsb_db(wl)
     else:
         db = oracle.tpcc_db(wl)
+    if w.get("reorder"):
+        db.set_reorder(True)
     log("oracle load %.1fs" % (time.time() - t0))
     sample = min(w["batch"], args.ref_sample)
     committed, secs = 0, 0.0
@@ -232,6 +237,8 @@ def cpu_baseline(name, batch_host, wl):
     w = WORKLOADS[name]
     t0 = time.time()
     db = oracle.ycsb_db(wl) if w["kind"] == "ycsb" else oracle.tpcc_db(wl)
+    if w.get("reorder"):
+        db.set_reorder(True)
     load_s = time.time() - t0
     n = len(batch_host["tid"])
     budget = 25.0
@@ -284,6 +291,8 @@ def main():
     w = WORKLOADS[name]
     wl = make_workload(name)
     B = w["batch"]
+    if w.get("reorder"):
+        args.flags |= ltpg.LTPG_FLAG_REORDER
     uid = None
     if world > 1:  # one NCCL communicator per db: the per-batch verdict exchange
         from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id

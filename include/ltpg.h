@@ -125,6 +125,8 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
 /* ---- configuration ------------------------------------------------------------ */
 #define LTPG_FLAG_NO_GROUPING   (1u << 0)  /* A/B: disable adaptive warp division (§V-B) */
 #define LTPG_FLAG_NO_MARK_FILTER (1u << 1) /* A/B: always issue the atomicMin mark        */
+#define LTPG_FLAG_REORDER       (1u << 2)  /* NEXT-1 logical reordering: abort iff
+                                              WAW or (RAW and WAR); keeps per-unit min reader marks */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
 
 typedef struct {

@@ -33,6 +33,7 @@ ERR_NAMES = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECAPACITY", -4: "ECUDA", 
 LTPG_MODE_OPS, LTPG_MODE_TPCC = 0, 1
 LTPG_FLAG_NO_GROUPING = 1 << 0
 LTPG_FLAG_NO_MARK_FILTER = 1 << 1
+LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_LOOPBACK_SHIFT = 8
 LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
 

@@ -144,6 +144,7 @@ void free_table(DevTable& T) {
   if (T.valid) cudaFree(T.valid);
   if (T.rowkey) cudaFree(T.rowkey);
   if (T.marks) cudaFree(T.marks);
+  if (T.rmarks) cudaFree(T.rmarks);
   if (T.idx) cudaFree(T.idx);
   if (T.aux) cudaFree(T.aux);
   unsigned long long* nr = T.n_rows;
@@ -152,10 +153,12 @@ void free_table(DevTable& T) {
 }
 
 // ---- exchange / combine kernels ------------------------------------------------------------
-// loopback: verdict = max over partitions of (conflict*2 | user_abort); the OR of all
-// partitions' errors is written back to every partition so that none writes back
+// A partition's verdict per txn is a set of conflict bits (CF_UA, CF_WAW, CF_RAW, CF_WAR); the
+// txn's bits are the OR over partitions, then the commit rule applies (R1 or NEXT-1).
+// loopback: OR in one kernel; the OR of all partitions' errors is written back to every
+// partition so that none writes back.
 __global__ void k_combine(void* const* lflags, uint32_t np, uint32_t n, uint8_t* status, void* const* errs,
-                          uint32_t* err_all) {
+                          uint32_t* err_all, bool reorder) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r == 0) {
     uint32_t e = 0;
@@ -163,24 +166,33 @@ __global__ void k_combine(void* const* lflags, uint32_t np, uint32_t n, uint8_t*
     *err_all = e;
   }
   if (r >= n) return;
-  uint8_t f = 0;
-  for (uint32_t p = 0; p < np; ++p) f = max(f, static_cast<const uint8_t*>(lflags[p])[r]);
-  status[r] = status_of_flag(f);
+  uint32_t f = 0;
+  for (uint32_t p = 0; p < np; ++p) f |= static_cast<const uint8_t*>(lflags[p])[r];
+  status[r] = status_of_bits(f, reorder);
 }
 __global__ void k_spread_err(const uint32_t* err_all, void* const* errs, uint32_t np) {
   for (uint32_t p = 0; p < np; ++p) *static_cast<uint32_t*>(errs[p]) = *err_all;
 }
-// NCCL: pack (flags, error bits as bytes) -> allreduce MAX -> unpack
+// NCCL has no bitwise-OR reduction: one byte per conflict bit, allreduce MAX, then unpack.
+// x = [4n bytes: txn r -> bytes 4r..4r+3 = ua, waw, raw, war] [3 error bytes]
 __global__ void k_pack(const uint8_t* lflag, const uint32_t* err, uint8_t* x, uint32_t n) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r < n) x[r] = lflag[r];
-  if (r < 3) x[n + r] = (*err >> r) & 1u;
+  if (r < n) {
+    const uint32_t f = lflag[r];
+    *reinterpret_cast<uchar4*>(x + 4ull * r) = make_uchar4(f & 1u, (f >> 1) & 1u, (f >> 2) & 1u, (f >> 3) & 1u);
+  }
+  if (r < 3) x[4ull * n + r] = (*err >> r) & 1u;
 }
-__global__ void k_unpack(const uint8_t* x, uint32_t n, uint8_t* status, uint32_t* err, uint32_t* err_all) {
+__global__ void k_unpack(const uint8_t* x, uint32_t n, uint8_t* status, uint32_t* err, uint32_t* err_all,
+                         bool reorder) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r < n) status[r] = status_of_flag(x[r]);
+  if (r < n) {
+    const uchar4 v = *reinterpret_cast<const uchar4*>(x + 4ull * r);
+    const uint32_t f = (v.x ? CF_UA : 0u) | (v.y ? CF_WAW : 0u) | (v.z ? CF_RAW : 0u) | (v.w ? CF_WAR : 0u);
+    status[r] = status_of_bits(f, reorder);
+  }
   if (r == 0) {
-    const uint32_t e = (uint32_t)x[n] | (uint32_t)x[n + 1] << 1 | (uint32_t)x[n + 2] << 2;
+    const uint32_t e = (uint32_t)x[4ull * n] | (uint32_t)x[4ull * n + 1] << 1 | (uint32_t)x[4ull * n + 2] << 2;
     *err = e;
     *err_all = e;
   }
@@ -250,7 +262,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(cudaEventCreate(&S.comp_done));
     CK(cudaEventCreate(&S.out_done));
   }
-  CK(dmalloc(&db->d_xchg, n + 4));
+  CK(dmalloc(&db->d_xchg, 4 * n + 4));
   CK(dmalloc(&db->d_ptrs, 3 * 64));
   CK(dmalloc(&db->d_scan, scan_scratch_words(std::max<size_t>(n, m)) + 16));
   CK(cudaStreamCreateWithFlags(&db->h2d, cudaStreamNonBlocking));
@@ -370,6 +382,10 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   if (d->n_groups) {
     CK(dmalloc(&T.marks, 2 * cap * d->n_groups));
     CK(cudaMemset(T.marks, 0xFF, 2 * cap * d->n_groups * sizeof(unsigned long long)));
+    if (db->cfg.flags & LTPG_FLAG_REORDER) {  // NEXT-1: minimum reader rank per unit
+      CK(dmalloc(&T.rmarks, cap * d->n_groups));
+      CK(cudaMemset(T.rmarks, 0xFF, cap * d->n_groups * sizeof(unsigned long long)));
+    }
   }
   if (d->has_pk) {
     uint64_t sz = 1;
@@ -575,6 +591,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   }
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
+  const bool reorder = (db->cfg.flags & LTPG_FLAG_REORDER) != 0;
   std::vector<BatchDev> pb(L, bd);
   for (uint32_t p = 0; p < L; ++p) {
     Part& P = db->parts[p];
@@ -631,14 +648,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
       if (db->cfg.world == 1) {
-        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, S.d_status, db->d_ptrs + 64, S.d_small);
+        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, S.d_status, db->d_ptrs + 64, S.d_small, reorder);
         k_spread_err<<<1, 1, 0, s>>>(S.d_small, db->d_ptrs + 64, L);
         note_launch(2);
       } else {
         k_pack<<<(n + 255) / 256, 256, 0, s>>>(pb[0].lflag, pb[0].err, db->d_xchg, n);
-        ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, n + 3, ncclUint8, ncclMax, db->comm, s);
+        ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, 4ull * n + 3, ncclUint8, ncclMax, db->comm, s);
         if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
-        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, S.d_status, pb[0].err, S.d_small);
+        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, S.d_status, pb[0].err, S.d_small, reorder);
         note_launch(2);
       }
     } else {

@@ -206,6 +206,11 @@ void launch_ops_claim(const BatchDev& b, cudaStream_t s) {
 }
 
 // ---- K-exec ---------------------------------------------------------------------------
+__device__ __forceinline__ void mark_read(const DevTable& T, uint32_t g, uint32_t row, unsigned long long tag,
+                                          bool filter) {
+  if (T.rmarks) mark_min(rmark_ptr(T, g, row), tag, filter);  // NEXT-1 only: min reader rank
+}
+
 __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
                                          uint32_t r, const ltpg_op& o, bool filter, uint32_t dmask) {
   const DevTable& T = c_tabs[o.table];
@@ -217,12 +222,16 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
   if (o.kind == LTPG_SCAN) {  // range of predefined keys; checked again in detect
     long long cnt = 0;
     unsigned long long sum = 0;
+    const uint32_t gs = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
     for (uint64_t k = o.key; k < o.key + o.aux; ++k) {
       if (!owns_key(b, T, k)) continue;  // partitioned: this partition's part of the range
       lookup(T, o.table, dmask, k, row, claim);
       if (row != ROW_NONE) {
         ++cnt;
         if (o.col != LTPG_COL_COUNT) sum += (unsigned long long)*col_ptr_ops(T, o.col, row);
+        if (T.n_groups) mark_read(T, gs, row, tag, filter);
+      } else if (claim != ROW_NONE) {
+        mark_read(T, 0, claim, tag, filter);
       }
     }
     b.res[oi] = o.col == LTPG_COL_COUNT ? cnt : (long long)sum;
@@ -233,6 +242,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
   const bool present = row != ROW_NONE;
   if (!present && o.kind != LTPG_INSERT) {
     // absent key: a READ of its existence; only an inserter of this batch can conflict
+    if (claim != ROW_NONE) mark_read(T, 0, claim, tag, filter);
     uref = claim != ROW_NONE ? make_uref(CHK_RW, false, false, o.table, 0, claim)
                              : make_uref(CHK_NONE, false, false, o.table, 0, 0);
     b.res[oi] = LTPG_NOT_FOUND;
@@ -243,6 +253,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
     case LTPG_SELECT: {
       res = *col_ptr_ops(T, o.col, row);
       uint32_t g = col_group(T, o.col);
+      if (g != LTPG_STATIC) mark_read(T, g, row, tag, filter);
       uref = g == LTPG_STATIC ? make_uref(CHK_NONE, false, true, o.table, 0, row)
                               : make_uref(CHK_RW, false, true, o.table, g, row);
       break;
@@ -251,20 +262,21 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
       uint32_t g = col_group(T, o.col);
       res = *col_ptr_ops(T, o.col, row);  // pre-image; new value = res + arg at write-back
       mark_min(mark_ptr(T, g, row), tag, filter);
-      uref = make_uref(CHK_RW, false, true, o.table, g, row);
+      uref = make_uref(CHK_RW, false, true, o.table, g, row, true);
       break;
     }
     case LTPG_ADD: {
       uint32_t g = col_group(T, o.col);
       res = 0;
       mark_min(mark_ptr(T, g, row) + 1, tag, filter);
-      uref = make_uref(CHK_A, false, true, o.table, g, row);
+      uref = make_uref(CHK_A, false, true, o.table, g, row, true);
       break;
     }
     case LTPG_INSERT:
       if (present) {  // duplicate key: user abort; a READ of the row
         res = 0;
         b.ua[r] = 1;
+        mark_read(T, 0, row, tag, filter);
         uref = make_uref(CHK_RW, false, true, o.table, 0, row);
       } else {
         if (claim == ROW_NONE) {  // every absent INSERT key was claimed by K-claim
@@ -273,13 +285,13 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
         }
         res = 1;
         for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(mark_ptr(T, g, claim), tag, filter);
-        uref = make_uref(CHK_RW, true, false, o.table, 0, claim);
+        uref = make_uref(CHK_RW, true, false, o.table, 0, claim, true);
       }
       break;
     case LTPG_DELETE:
       res = 1;
       for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(mark_ptr(T, g, row), tag, filter);
-      uref = make_uref(CHK_RW, true, true, o.table, 0, row);
+      uref = make_uref(CHK_RW, true, true, o.table, 0, row, true);
       break;
   }
   b.res[oi] = res;
@@ -334,42 +346,42 @@ template <bool PART>
 __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live & ~*b.insdel;
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= b.n_txns) return;
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
-  bool bad = false;
-  for (uint32_t i = b0; i < b1 && !bad; ++i) {
+  uint32_t bits = 0;
+  for (uint32_t i = b0; i < b1 && !conflict_of(bits, reorder); ++i) {
     if (PART && !op_touches(b, load_op(b.ops, i))) continue;
     const uint64_t u = b.uref[i];
     const uint64_t chk = u >> 62;
     if (chk == CHK_NONE) continue;
-    const DevTable& T = c_tabs[(u >> 40) & 0xFF];
+    const uint32_t t = (u >> 40) & 0xFF;
+    const DevTable& T = c_tabs[t];
     if (chk == CHK_SCAN) {  // phantom-safe: every key of the range is a read (R8)
       const ltpg_op o = load_op(b.ops, i);
       if (!T.n_groups) continue;
-      for (uint64_t k = o.key; k < o.key + o.aux && !bad; ++k) {
+      const uint32_t gs = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
+      for (uint64_t k = o.key; k < o.key + o.aux && !(bits & CF_RAW); ++k) {
         if (PART && !owns_key(b, T, k)) continue;
         uint32_t row, claim;
-        lookup(T, (u >> 40) & 0xFF, dmask, k, row, claim);
-        if (row != ROW_NONE) {
-          uint32_t g = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
-          bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);
-        } else if (claim != ROW_NONE) {
-          bad = unit_conflicts(T, 0, claim, CHK_RW, r, b.epoch);
-        }
+        lookup(T, t, dmask, k, row, claim);
+        if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b.epoch);
+        else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b.epoch);
       }
       continue;
     }
     const uint32_t row = (uint32_t)u;
+    const uint32_t acc = chk == CHK_A ? ACC_ADD : (((u >> 59) & 1) ? ACC_WRITE : ACC_READ);
     if ((u >> 61) & 1) {
-      for (uint32_t g = 0; g < T.n_groups && !bad; ++g) bad = unit_conflicts(T, g, row, CHK_RW, r, b.epoch);
+      for (uint32_t g = 0; g < T.n_groups; ++g) bits |= unit_bits(T, g, row, acc, r, b.epoch);
     } else {
-      bad = unit_conflicts(T, (u >> 32) & 0xFF, row, chk, r, b.epoch);
+      bits |= unit_bits(T, (u >> 32) & 0xFF, row, acc, r, b.epoch);
     }
   }
-  const uint8_t flag = (uint8_t)(bad ? 2 : 0) | (b.ua[r] ? 1 : 0);
-  if (PART) b.lflag[r] = flag;
-  else b.status[r] = status_of_flag(flag);
+  const uint32_t flag = bits | (b.ua[r] ? CF_UA : 0u);
+  if (PART) b.lflag[r] = (uint8_t)flag;
+  else b.status[r] = status_of_bits(flag, reorder);
 }
 
 void launch_ops_detect(const BatchDev& b, cudaStream_t s) {

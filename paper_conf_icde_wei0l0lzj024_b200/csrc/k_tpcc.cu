@@ -95,8 +95,11 @@ struct Tx {
   uint32_t epoch;
   unsigned long long tag;
   bool filter;
-  bool bad;
+  uint32_t bits;   // detect: conflict bits found so far (CF_*)
   uint32_t* err;
+  bool reorder;    // NEXT-1 logical reordering
+  // verdict already decided by the bits found (remaining checks cannot change it)
+  __device__ __forceinline__ bool done() const { return conflict_of(bits, reorder); }
 };
 
 __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINTERNAL); }
@@ -109,16 +112,18 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 template <int PH>
 __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
   if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter && hot);
-  if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_WRITE, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
   if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter && hot);
-  if (PH == PH_DETECT && !x.bad) x.bad = unit_conflicts(T, g, row, CHK_A, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_ADD, x.r, x.epoch);
 }
 template <int PH>
-__device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x) {
-  if (PH == PH_DETECT && !x.bad && g != LTPG_STATIC) x.bad = unit_conflicts(T, g, row, CHK_RW, x.r, x.epoch);
+__device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
+  if (g == LTPG_STATIC) return;
+  if (PH == PH_EXEC && T.rmarks) mark_min(rmark_ptr(T, g, row), x.tag, x.filter && hot);  // NEXT-1 minR
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_READ, x.r, x.epoch);
 }
 // update of column c (strict: WRITE unit of its group; delayed: ADD unit)
 template <int PH>
@@ -464,12 +469,12 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
       const uint64_t nok = kO(w, d, (uint64_t)o);
       uint64_t hn_, ho_;
       const ulonglong2 vn = probe_issue(TNw, nok, hn_), vo = probe_issue(TOr, nok, ho_);  // together
-      const uint32_t row_no = (PH == PH_DETECT && x.bad) ? ROW_NONE : probe_finish(TNw, nok, hn_, vn);
-      if (PH == PH_DETECT && x.bad) {
+      const uint32_t row_no = (PH == PH_DETECT && x.done()) ? ROW_NONE : probe_finish(TNw, nok, hn_, vn);
+      if (PH == PH_DETECT && x.done()) {
         // conflict already found: the remaining checks cannot change the verdict
       } else if (row_no == ROW_NONE) {
         // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
-        unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
+        unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
       } else {
         for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x);  // DELETE
         const uint32_t row_o = probe_finish(TOr, nok, ho_, vo);
@@ -551,8 +556,8 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
     return;
   }
   const long long nx = rd(TDi, D_NEXT_O_ID, row_d);
-  if (lane == 0) unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x);
-  if (PH == PH_DETECT && __shfl_sync(0xffffffffu, (uint32_t)x.bad, 0)) return;  // RAW on D_NEXT_O_ID: done
+  if (lane == 0) unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
+  if (PH == PH_DETECT && __shfl_sync(0xffffffffu, (uint32_t)x.done(), 0)) return;  // RAW on D_NEXT_O_ID: done
   for (uint32_t s = lane; s < SL_SLOTS; s += 32) items[s] = 0;
   for (uint32_t s = lane; s < SL_HASH; s += 32) set[s] = 0;
   __syncwarp();
@@ -579,7 +584,7 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
   }
   __syncwarp();
   long long low = 0;
-  for (uint32_t s = lane; s < SL_SLOTS && !(PH == PH_DETECT && x.bad); s += 32) {
+  for (uint32_t s = lane; s < SL_SLOTS && !(PH == PH_DETECT && x.done()); s += 32) {
     const uint32_t it = items[s];
     if (!it) continue;
     uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
@@ -615,6 +620,7 @@ template <int PH>
 __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
   __shared__ uint32_t sl_items[8][SL_SLOTS];
   __shared__ uint32_t sl_set[8][SL_HASH];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -638,9 +644,11 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
     const uint32_t sub = lane % L;
     const bool active = k < ct;
     const uint32_t r = active ? tp.list[(uint64_t)t * tp.max_txns + k] : 0;
-    Tx x{dmask, r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), false, b.err};
+    Tx x{dmask, r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder};
     bool go = active;
     if (PH == PH_WB) go = active && b.status[r] == LTPG_ST_COMMIT;
+    // NEXT-1: read-only procedures (OrderStatus, StockLevel) can never abort under reordering
+    if (PH == PH_DETECT && reorder && (t == 2 || t == 4)) go = false;
     switch (t) {
       case 0: proc_neworder<PH>(b, tp, r, sub, go, x); break;
       case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
@@ -648,13 +656,15 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
       case 3: proc_delivery<PH>(b, r, sub, go, x); break;
       default: proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib], sl_set[wib]); break;
     }
-    if (PH == PH_DETECT) {  // per-txn OR over the txn's lanes, one status write per txn
-      const uint32_t bal = __ballot_sync(0xffffffffu, x.bad);
+    if (PH == PH_DETECT) {  // per-txn OR of the conflict bits over the txn's lanes
       const uint32_t seg = L == 32 ? 0xffffffffu : (L == 1 ? (1u << lane) : (0xffffu << (lane & 16)));
+      const uint32_t bw = __ballot_sync(0xffffffffu, x.bits & CF_WAW) & seg;
+      const uint32_t br = __ballot_sync(0xffffffffu, x.bits & CF_RAW) & seg;
+      const uint32_t bx = __ballot_sync(0xffffffffu, x.bits & CF_WAR) & seg;
       if (active && sub == 0) {
-        const uint8_t flag = (uint8_t)((bal & seg) ? 2 : 0) | (b.ua[r] ? 1 : 0);
-        if (b.nparts > 1) b.lflag[r] = flag;  // partitioned: exchanged before write-back
-        else b.status[r] = status_of_flag(flag);
+        const uint32_t flag = (bw ? CF_WAW : 0u) | (br ? CF_RAW : 0u) | (bx ? CF_WAR : 0u) | (b.ua[r] ? CF_UA : 0u);
+        if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;  // partitioned: exchanged before write-back
+        else b.status[r] = status_of_bits(flag, reorder);
       }
     }
   }

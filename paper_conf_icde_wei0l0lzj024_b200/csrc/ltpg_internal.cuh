@@ -48,6 +48,7 @@ struct DevTable {
   uint8_t* valid;
   unsigned long long* rowkey;
   unsigned long long* marks;      // [n_groups][capacity] x {minW, minA}
+  unsigned long long* rmarks;     // [n_groups][capacity] minR (LTPG_FLAG_REORDER only, else null)
   IdxSlot* idx;
   uint64_t idx_mask;
   uint32_t idx_shift;
@@ -106,6 +107,10 @@ __device__ __forceinline__ void mark_min(unsigned long long* p, unsigned long lo
 
 __device__ __forceinline__ unsigned long long* mark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
   return T.marks + 2ull * ((uint64_t)g * T.capacity + row);
+}
+
+__device__ __forceinline__ unsigned long long* rmark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
+  return T.rmarks + ((uint64_t)g * T.capacity + row);
 }
 
 __device__ __forceinline__ long long* col_ptr(const DevTable& T, uint32_t c, uint32_t row) {
@@ -169,21 +174,42 @@ __device__ __forceinline__ IdxSlot* idx_slot(const DevTable& T, uint64_t key) {
 
 // uref: per-op record written by execute, read by detect / write-back.
 //   bits  0..31 row (or claim row)   bits 32..39 group   bits 40..47 table
-//   bit   60    present in snapshot  bit 61 all groups    bits 62..63 check kind
+//   bit   59 write (CHK_RW: plain write; else a read)     bit 60 present in snapshot
+//   bit   61 all groups              bits 62..63 check kind
 __host__ __device__ __forceinline__ uint64_t make_uref(uint64_t chk, bool all, bool present, uint32_t t,
-                                                       uint32_t g, uint32_t row) {
-  return (chk << 62) | ((uint64_t)all << 61) | ((uint64_t)present << 60) | ((uint64_t)t << 40) |
-         ((uint64_t)g << 32) | row;
+                                                       uint32_t g, uint32_t row, bool write = false) {
+  return (chk << 62) | ((uint64_t)all << 61) | ((uint64_t)present << 60) | ((uint64_t)write << 59) |
+         ((uint64_t)t << 40) | ((uint64_t)g << 32) | row;
 }
 
-// Commit test of one unit for rank r (rcheck / wcheck; R1, R7).
+// per-txn conflict bits (detect) and the verdict (R1; NEXT-1 reordering)
+constexpr uint32_t CF_UA = 1u, CF_WAW = 2u, CF_RAW = 4u, CF_WAR = 8u;
+enum { ACC_READ = 0, ACC_WRITE = 1, ACC_ADD = 2 };
+__device__ __forceinline__ bool conflict_of(uint32_t bits, bool reorder) {
+  return (bits & CF_WAW) || (reorder ? ((bits & CF_RAW) && (bits & CF_WAR)) : (bits & CF_RAW) != 0);
+}
+__device__ __forceinline__ uint8_t status_of_bits(uint32_t bits, bool reorder) {
+  return conflict_of(bits, reorder) ? LTPG_ST_CONFLICT : ((bits & CF_UA) ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
+}
+
+// Conflict bits of one access of rank r to unit (g,row) (rcheck / wcheck; R1, R7):
+//   READ  -> RAW if a smaller rank wrote or added
+//   WRITE -> WAW if a smaller rank wrote or added; WAR if a smaller rank read (reorder only)
+//   ADD   -> WAW if a smaller rank plainly wrote;  WAR if a smaller rank read (reorder only)
+__device__ __forceinline__ uint32_t unit_bits(const DevTable& T, uint32_t g, uint32_t row, uint32_t acc, uint32_t r,
+                                              uint32_t epoch) {
+  const ulonglong2 m = *reinterpret_cast<const ulonglong2*>(mark_ptr(T, g, row));
+  const uint32_t w = mark_rank(m.x, epoch), a = mark_rank(m.y, epoch);
+  const uint32_t wa = w < a ? w : a;
+  uint32_t bits = 0;
+  if (acc == ACC_READ) return wa < r ? CF_RAW : 0u;
+  if ((acc == ACC_WRITE ? wa : w) < r) bits |= CF_WAW;
+  if (T.rmarks && mark_rank(*rmark_ptr(T, g, row), epoch) < r) bits |= CF_WAR;
+  return bits;
+}
 __device__ __forceinline__ bool unit_conflicts(const DevTable& T, uint32_t g, uint32_t row, uint64_t chk,
                                                uint32_t r, uint32_t epoch) {
-  const ulonglong2 m = *reinterpret_cast<const ulonglong2*>(mark_ptr(T, g, row));
-  uint32_t w = mark_rank(m.x, epoch);
-  if (chk == CHK_A) return w < r;
-  uint32_t a = mark_rank(m.y, epoch);
-  return (w < a ? w : a) < r;
+  return unit_bits(T, g, row, chk == CHK_A ? ACC_ADD : ACC_WRITE, r, epoch) & CF_WAW;
 }
 
 // Table metadata lives in __constant__ memory: warp-uniform table ids broadcast from
@@ -207,7 +233,7 @@ inline void note_launch(uint32_t k = 1) { g_kernel_launches += k; }
 struct BatchDev {
   // partitioning (§8(e)): nparts logical partitions (ranks x loopback); this is `part`.
   // nparts == 1: this partition owns everything and detect writes `status` directly;
-  // otherwise detect writes lflag[r] = conflict*2 | user_abort for the exchange.
+  // otherwise detect writes lflag[r] = conflict bits (CF_*) for the exchange (OR over partitions).
   uint32_t nparts, part;
   uint32_t nw;                     // TPC-C: number of warehouses (warehouse ownership)
   uint64_t key_space;              // OPS: key-range ownership of owner_rule-2 tables
@@ -289,10 +315,7 @@ __device__ __forceinline__ bool owns_key(const BatchDev& b, const DevTable& T, u
 __device__ __forceinline__ bool owns_w(const BatchDev& b, uint32_t w) {
   return b.nparts <= 1 || part_of_w(w, b.nw, b.nparts) == b.part;
 }
-// final verdict from a partition-local or exchanged flag (conflict dominates user abort)
-__device__ __forceinline__ uint8_t status_of_flag(uint8_t f) {
-  return f >= 2 ? LTPG_ST_CONFLICT : (f ? LTPG_ST_USER_ABORT : LTPG_ST_COMMIT);
-}
+
 
 void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
 size_t scan_scratch_words(uint32_t n);
