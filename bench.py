@@ -46,6 +46,9 @@ WORKLOADS = {
     "tpcc_c2_opt": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed", reorder=True),
     "tpcc_c2_delayed": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed"),
     "ycsb_c3_4ops": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=4, batch=1 << 20),
+    # NEXT-4: the paper's YCSB suite: Zipf alpha 2.5, 10 ops, 10^7 rows
+    **{"ycsb_%s" % L.lower(): dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=2.5, ops=10, batch=1 << 16,
+                                   letter=L) for L in "ABCDE"},
 }
 DEFAULT_WORKLOAD = "tpcc_c4"
 
@@ -134,7 +137,9 @@ def make_workload(name, rank=0):
     w = WORKLOADS[name]
     seed = 0x17C0 + w["cfg"]
     if w["kind"] == "ycsb":
-        from workloads.ycsb import YcsbWorkload
+        from workloads.ycsb import YcsbWorkload, ycsb_letter
+        if w.get("letter"):
+            return ycsb_letter(w["letter"], w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
         return YcsbWorkload(w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
     from workloads import tpcc
     mix = tpcc.MIX_FULL if w["mix"] == "full" else tpcc.MIX_NO_PAY
@@ -299,8 +304,10 @@ def main():
         uid = nccl_unique_id()
     t0 = time.time()
     if w["kind"] == "ycsb":
+        nb = args.warmup + 2 * args.steps + 2  # inserts (YCSB D/E) of every batch this run makes
         db = ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=args.flags, device=local,
-                                rank=rank, world=world, nccl_unique_id=uid)
+                                rank=rank, world=world, nccl_unique_id=uid,
+                                capacity=w["n_rows"] + nb * B * w["ops"] // 10 + 1024)
     else:
         # append regions: the worst case of one batch (checked before execution) plus the
         # expected appends of every batch this run makes (NewOrder commits <= 30%, Payment <= 100%)

@@ -53,7 +53,7 @@ class YcsbWorkload:
     TABLE = 0
 
     def __init__(self, n_rows, n_fields=10, theta=0.99, ops_per_txn=10, read_frac=0.5,
-                 seed=0x17C0, scan_frac=0.0, insert_frac=0.0, max_scan_len=10):
+                 seed=0x17C0, scan_frac=0.0, insert_frac=0.0, max_scan_len=10, read_latest=False):
         self.n_rows = int(n_rows)
         self.n_fields = int(n_fields)
         self.theta = float(theta)
@@ -66,6 +66,7 @@ class YcsbWorkload:
         self.a = _coprime_multiplier(self.n_rows, self.seed)
         self.b = (self.seed * 7919) % self.n_rows
         self.next_insert_key = self.n_rows
+        self.read_latest = bool(read_latest)
 
     # -- table ------------------------------------------------------------------
     def table_desc(self):
@@ -89,6 +90,32 @@ class YcsbWorkload:
         with np.errstate(over="ignore"):
             k = (np.uint64(self.a) * ranks.astype(np.uint64) + np.uint64(self.b)) % np.uint64(self.n_rows)
         return k
+
+    def _draw_ranks(self, rng, shape):
+        cdf = zipf_cdf(self.n_rows, self.theta)
+        ranks = np.searchsorted(cdf, rng.random(shape), side="right")
+        return np.minimum(ranks, self.n_rows - 1)
+
+    @staticmethod
+    def _dedupe_scans(keys, kinds, aux):
+        """R10: a txn's SCAN range may not cover a key the txn writes (INSERT/UPDATE) or
+        another point key; such SCANs are shortened to length 0 (an empty read)."""
+        n, k = keys.shape
+        lo = keys.astype(np.uint64)
+        for j in range(k):
+            sc = kinds[:, j] == SCAN
+            if not sc.any():
+                continue
+            hi = lo[:, j] + aux[:, j].astype(np.uint64)
+            clash = np.zeros(n, bool)
+            for m in range(k):
+                if m == j:
+                    continue
+                other_hi = lo[:, m] + np.where(kinds[:, m] == SCAN, aux[:, m], 1).astype(np.uint64)
+                ov = (lo[:, m] < hi) & (lo[:, j] < other_hi)
+                writes = np.isin(kinds[:, m], [UPDATE, INSERT])
+                clash |= sc & ov & (writes | (kinds[:, m] != SCAN))
+            aux[clash, j] = 0
 
     def _draw_keys(self, rng, shape):
         cdf = zipf_cdf(self.n_rows, self.theta)
@@ -115,11 +142,36 @@ class YcsbWorkload:
             rows = rows[(s[:, 1:] == s[:, :-1]).any(axis=1)]
         u = rng.random((n_txns, k))
         kinds = np.where(u < self.read_frac, SELECT, UPDATE).astype(np.uint8)
+        aux = np.zeros((n_txns, k), np.uint32)
+        if self.scan_frac > 0 or self.insert_frac > 0:
+            # YCSB D/E: INSERTs of fresh keys N, N+1, ... (unique across batches) and
+            # short SCANs [key, key+len) with len U[1, max_scan_len]
+            u2 = rng.random((n_txns, k))
+            scan = u2 < self.scan_frac
+            ins = (u2 >= self.scan_frac) & (u2 < self.scan_frac + self.insert_frac)
+            kinds = np.where(scan, SCAN, np.where(ins, INSERT, kinds)).astype(np.uint8)
+            aux = np.where(scan, rng.integers(1, self.max_scan_len + 1, (n_txns, k)), 0).astype(np.uint32)
+            n_ins = int(ins.sum())
+            latest = self.next_insert_key - 1  # newest key inserted before this batch
+            keys[ins] = np.arange(self.next_insert_key, self.next_insert_key + n_ins, dtype=np.uint64)
+            self.next_insert_key += n_ins
+            if self.read_latest:  # YCSB D: reads skewed toward the most recently inserted keys
+                off = self._draw_ranks(rng, (n_txns, k)).astype(np.int64)
+                off = np.where(kinds == SELECT, off, 1 << 40)  # non-reads sort last
+                order = np.argsort(off, axis=1, kind="stable")
+                so = np.take_along_axis(off, order, axis=1)
+                idx = np.arange(k)[None, :]
+                so = idx + np.maximum.accumulate(so - idx, axis=1)  # distinct offsets per txn (R10)
+                np.put_along_axis(off, order, so, axis=1)
+                rd = kinds == SELECT
+                keys[rd] = (np.uint64(latest) - (off[rd] % (latest + 1)).astype(np.uint64))
+            self._dedupe_scans(keys, kinds, aux)
         ops = np.zeros(n_txns * k, dtype=OP_DTYPE)
         ops["key"] = keys.reshape(-1)
         ops["kind"] = kinds.reshape(-1)
         ops["table"] = self.TABLE
         ops["col"] = rng.integers(0, self.n_fields, n_txns * k, dtype=np.uint16)
+        ops["aux"] = aux.reshape(-1)
         args = rng.integers(1, 1001, n_txns * k, dtype=np.int64)
         op_begin = (np.arange(n_txns + 1, dtype=np.uint64) * k).astype(np.uint32)
         tid = np.arange(tid_start, tid_start + n_txns, dtype=np.uint64)
@@ -150,3 +202,21 @@ def random_ops_batch(rng, n_txns, n_keys, n_fields=2, max_ops=4, kinds=(SELECT, 
     return {"tid": np.arange(tid_start, tid_start + n_txns, dtype=np.uint64),
             "op_begin": np.array(op_begin, dtype=np.uint32),
             "ops": ops, "args": np.array(args, dtype=np.int64)}
+
+
+# YCSB core workloads A-E (Cooper et al. [7]), as op mixes of this OPS model.
+# Fractions are of ops: read / (update = RMW) / insert / scan.
+YCSB_MIXES = {
+    "A": dict(read_frac=0.50),                                        # update heavy
+    "B": dict(read_frac=0.95),                                        # read heavy
+    "C": dict(read_frac=1.00),                                        # read only
+    "D": dict(read_frac=1.00, insert_frac=0.05, read_latest=True),    # read latest
+    "E": dict(read_frac=1.00, scan_frac=0.95, insert_frac=0.05),      # short ranges
+}
+
+
+def ycsb_letter(letter, n_rows, theta=2.5, ops_per_txn=10, seed=0x17C0, **kw):
+    """YCSB workload `letter` at Zipf theta (the paper's alpha = 2.5)."""
+    args = dict(YCSB_MIXES[letter])
+    args.update(kw)
+    return YcsbWorkload(n_rows, theta=theta, ops_per_txn=ops_per_txn, seed=seed, **args)
