@@ -583,23 +583,55 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
     }
   }
   __syncwarp();
-  long long low = 0;
-  for (uint32_t s = lane; s < SL_SLOTS && !(PH == PH_DETECT && x.done()); s += 32) {
-    const uint32_t it = items[s];
-    if (!it) continue;
-    uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
+  // distinct items: the first inserter of an item into the shared-memory set appends it to a
+  // compact list (the slot array is reused: items were consumed into registers first)
+  uint32_t mine[(SL_SLOTS + 31) / 32];
+#pragma unroll
+  for (uint32_t u = 0; u < (SL_SLOTS + 31) / 32; ++u) {
+    const uint32_t sl = lane + 32 * u;
+    mine[u] = sl < SL_SLOTS ? items[sl] : 0u;
+  }
+  __syncwarp();
+  uint32_t nd = 0;
+#pragma unroll
+  for (uint32_t u = 0; u < (SL_SLOTS + 31) / 32; ++u) {
+    const uint32_t it = mine[u];
     bool first = false;
-    for (;;) {
-      const uint32_t old = atomicCAS(set + h, 0u, it);
-      if (old == 0u) { first = true; break; }
-      if (old == it) break;
-      h = (h + 1) & (SL_HASH - 1);
+    if (it) {
+      uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
+      for (;;) {
+        const uint32_t old = atomicCAS(set + h, 0u, it);
+        if (old == 0u) { first = true; break; }
+        if (old == it) break;
+        h = (h + 1) & (SL_HASH - 1);
+      }
     }
-    if (!first) continue;  // count distinct items
-    const uint32_t row_s = rowof(TSt, TS, kS(w, it), x.dmask);
-    if (row_s == ROW_NONE) { internal_error(x); continue; }
-    if (PH == PH_EXEC) low += rd(TSt, S_QUANTITY, row_s) < thr;
-    unit_r<PH>(TSt, col_group(TSt, S_QUANTITY), row_s, x);
+    const uint32_t m = __ballot_sync(0xffffffffu, first);
+    if (first) items[nd + __popc(m & ((1u << lane) - 1))] = it;
+    nd += __popc(m);
+  }
+  __syncwarp();
+  // stock reads of the distinct items: all of a lane's loads in flight together (dense key
+  // -> row mapping: no index access)
+  long long low = 0;
+  constexpr uint32_t MAXU = (SL_SLOTS + 31) / 32;
+  uint32_t rows[MAXU];
+#pragma unroll
+  for (uint32_t u = 0; u < MAXU; ++u) {
+    const uint32_t j = lane + 32 * u;
+    rows[u] = j < nd ? rowof(TSt, TS, kS(w, items[j]), x.dmask) : ROW_NONE;
+  }
+  long long q[MAXU];
+#pragma unroll
+  for (uint32_t u = 0; u < MAXU; ++u)
+    q[u] = (PH == PH_EXEC && rows[u] != ROW_NONE) ? rd(TSt, S_QUANTITY, rows[u]) : 0;
+#pragma unroll
+  for (uint32_t u = 0; u < MAXU; ++u) {
+    const uint32_t j = lane + 32 * u;
+    if (j >= nd) continue;
+    if (rows[u] == ROW_NONE) { internal_error(x); continue; }
+    if (PH == PH_EXEC) low += q[u] < thr;
+    unit_r<PH>(TSt, col_group(TSt, S_QUANTITY), rows[u], x);
   }
   if (PH == PH_EXEC) {
 #pragma unroll
@@ -616,19 +648,21 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
 
 // ---- the phase kernel: type-homogeneous warps over the per-type txn lists -------------------------
 
-template <int PH>
+// TMASK: procedure types this launch runs.  StockLevel (32 lanes, 26 KB of shared memory per
+// block, many registers) runs in its own launch so it does not cap the occupancy of the
+// others -- each type group gets its own launch configuration.
+constexpr uint32_t TM_MAIN = 0x0Fu, TM_SL = 0x10u;
+template <int PH, uint32_t TMASK>
 __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
-  __shared__ uint32_t sl_items[8][SL_SLOTS];
-  __shared__ uint32_t sl_set[8][SL_HASH];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   uint32_t cnt[NTYPES], pre[NTYPES + 1];
   pre[0] = 0;
 #pragma unroll
   for (int t = 0; t < NTYPES; ++t) {
-    cnt[t] = tp.counts[t];
+    cnt[t] = ((TMASK >> t) & 1u) ? tp.counts[t] : 0u;
     const uint32_t per = 32 / (t == 1 ? 1 : (t == 4 ? 32 : 16));
     pre[t + 1] = pre[t] + (cnt[t] + per - 1) / per;
   }
@@ -645,8 +679,7 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
     const bool active = k < ct;
     const uint32_t r = active ? tp.list[(uint64_t)t * tp.max_txns + k] : 0;
     Tx x{dmask, r, b.epoch, epoch_tag(b.epoch) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder};
-    bool go = active;
-    if (PH == PH_WB) go = active && b.status[r] == LTPG_ST_COMMIT;
+    bool go = active;  // write-back runs over the committed re-list (k_tpcc_relist) only
     // NEXT-1: read-only procedures (OrderStatus, StockLevel) can never abort under reordering
     if (PH == PH_DETECT && reorder && (t == 2 || t == 4)) go = false;
     switch (t) {
@@ -654,7 +687,13 @@ __global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
       case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
       case 3: proc_delivery<PH>(b, r, sub, go, x); break;
-      default: proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib], sl_set[wib]); break;
+      default:
+        if constexpr ((TMASK & TM_SL) != 0) {
+          __shared__ uint32_t sl_items[8][SL_SLOTS];
+          __shared__ uint32_t sl_set[8][SL_HASH];
+          proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib], sl_set[wib]);
+        }
+        break;
     }
     if (PH == PH_DETECT) {  // per-txn OR of the conflict bits over the txn's lanes
       const uint32_t seg = L == 32 ? 0xffffffffu : (L == 1 ? (1u << lane) : (0xffffu << (lane & 16)));
@@ -836,21 +875,34 @@ __global__ void k_no_colscan(BatchDev b, TpccParams tp) {  // one warp per distr
   const uint32_t dk = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
-  uint32_t run = 0;
-  for (uint32_t ch0 = 0; ch0 < tp.n_chunks; ch0 += 32) {
-    const uint32_t ch = ch0 + lane;
-    uint32_t* c = tp.chunk_cnt + (uint64_t)ch * tp.dsz + dk;
-    const uint32_t v = ch < tp.n_chunks ? *c : 0;
-    uint32_t x = v;
+  constexpr uint32_t PER = 32;  // chunks per lane held in registers; 1024 chunks per pass
+  uint32_t run_all = 0;
+  for (uint32_t base = 0; base < tp.n_chunks; base += 32 * PER) {
+    uint32_t v[PER];
+#pragma unroll
+    for (uint32_t k = 0; k < PER; ++k) {  // lane owns chunks base + [lane*PER, lane*PER+PER): loads in flight
+      const uint32_t ch = base + lane * PER + k;
+      v[k] = ch < tp.n_chunks ? tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] : 0u;
+    }
+    uint32_t tot = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < PER; ++k) tot += v[k];
+    uint32_t x = tot;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
+      if (lane >= (uint32_t)o) x += y;
     }
-    if (ch < tp.n_chunks) *c = run + x - v;  // exclusive prefix over chunks
-    run += __shfl_sync(0xffffffffu, x, 31);
+    uint32_t run = run_all + x - tot;  // exclusive prefix of this lane's first chunk
+    run_all += __shfl_sync(0xffffffffu, x, 31);
+#pragma unroll
+    for (uint32_t k = 0; k < PER; ++k) {
+      const uint32_t ch = base + lane * PER + k;
+      if (ch < tp.n_chunks) tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] = run;
+      run += v[k];
+    }
   }
-  if (!run || lane) return;
+  if (!run_all || lane) return;
   const DevTable& TDi = c_tabs[TD];
   const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
   if (row_d == ROW_NONE) {
@@ -859,7 +911,7 @@ __global__ void k_no_colscan(BatchDev b, TpccParams tp) {  // one warp per distr
   }
   const long long base = rd(TDi, D_NEXT_O_ID, row_d);
   tp.dist_base[dk] = base;
-  addv(TDi, D_NEXT_O_ID, row_d, run);  // final value: snapshot + committed NewOrders (delayed add)
+  addv(TDi, D_NEXT_O_ID, row_d, run_all);  // final value: snapshot + committed NewOrders (delayed add)
 }
 
 __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk, ranks in order
@@ -867,11 +919,19 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
   if (*b.err) return;
   const uint32_t lane = threadIdx.x;
   for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i];
-  __syncwarp();
   const uint32_t r0 = blockIdx.x * NO_CHUNK;
+  uint32_t dks[NO_CHUNK / 32];
+#pragma unroll
+  for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {  // all of the chunk's loads in flight first
+    const uint32_t r = r0 + it * 32 + lane;
+    dks[it] = r < b.n_txns ? tp.dk_of[r] : ~0u;
+  }
+  __syncwarp();
+#pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {
     const uint32_t r = r0 + it * 32 + lane;
-    const uint32_t dk = r < b.n_txns ? tp.dk_of[r] : ~0u;
+    const uint32_t dk = dks[it];
+    if (!__any_sync(0xffffffffu, dk != ~0u)) continue;
     const uint32_t m = __match_any_sync(0xffffffffu, dk);
     if (dk != ~0u) {
       const uint32_t before = __popc(m & ((1u << lane) - 1));
@@ -993,10 +1053,14 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   note_launch(2);
   if (ev) cudaEventRecord(ev[2], s);
   const uint32_t grid = phase_grid(n);
-  k_tpcc_phase<PH_EXEC><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_EXEC, TM_SL><<<grid, 256, 0, s>>>(b, tp);
+  note_launch();
   note_launch();
   if (ev) cudaEventRecord(ev[3], s);
-  k_tpcc_phase<PH_DETECT><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_DETECT, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_DETECT, TM_SL><<<grid, 256, 0, s>>>(b, tp);
+  note_launch();
   note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
@@ -1017,7 +1081,7 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  k_tpcc_phase<PH_WB><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));
+  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));
   k_tpcc_advance<<<1, 1, 0, s>>>(b, tp);
   note_launch(2);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
