@@ -998,10 +998,20 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
     return LTPG_ENOMEM;
   if (t.owns_by_name) cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
+  if (cudaStreamCreateWithFlags(&t.side, cudaStreamNonBlocking) != cudaSuccess) return LTPG_ECUDA;
+  for (int k = 0; k < 2; ++k)
+    if (cudaEventCreateWithFlags(&t.fork[k], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&t.join[k], cudaEventDisableTiming) != cudaSuccess)
+      return LTPG_ECUDA;
   return 0;
 }
 
 void tpcc_free(TpccDev& t) {
+  if (t.side) cudaStreamDestroy(t.side);
+  for (int k = 0; k < 2; ++k) {
+    if (t.fork[k]) cudaEventDestroy(t.fork[k]);
+    if (t.join[k]) cudaEventDestroy(t.join[k]);
+  }
   if (!t.owns_by_name) t.by_name = nullptr;
   void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
   for (void* p : ps)
@@ -1053,15 +1063,22 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   note_launch(2);
   if (ev) cudaEventRecord(ev[2], s);
   const uint32_t grid = phase_grid(n);
+  // StockLevel warps on a side stream, concurrently with the other procedures (fork / join)
+  cudaEventRecord(t.fork[0], s);
+  cudaStreamWaitEvent(t.side, t.fork[0], 0);
+  k_tpcc_phase<PH_EXEC, TM_SL><<<grid, 256, 0, t.side>>>(b, tp);
+  cudaEventRecord(t.join[0], t.side);
   k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
-  k_tpcc_phase<PH_EXEC, TM_SL><<<grid, 256, 0, s>>>(b, tp);
-  note_launch();
-  note_launch();
+  cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
+  note_launch(2);
   if (ev) cudaEventRecord(ev[3], s);
+  cudaEventRecord(t.fork[1], s);
+  cudaStreamWaitEvent(t.side, t.fork[1], 0);
+  k_tpcc_phase<PH_DETECT, TM_SL><<<grid, 256, 0, t.side>>>(b, tp);
+  cudaEventRecord(t.join[1], t.side);
   k_tpcc_phase<PH_DETECT, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
-  k_tpcc_phase<PH_DETECT, TM_SL><<<grid, 256, 0, s>>>(b, tp);
-  note_launch();
-  note_launch();
+  cudaStreamWaitEvent(s, t.join[1], 0);
+  note_launch(2);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
 

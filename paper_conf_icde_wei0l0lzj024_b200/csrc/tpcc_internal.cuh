@@ -39,6 +39,8 @@ struct TpccDev {
   uint32_t* chunk_cnt = nullptr;// [chunks][dsz]
   long long* dist_base = nullptr; // [dsz] snapshot D_NEXT_O_ID
   uint32_t* misc = nullptr;     // counters (M_*)
+  cudaStream_t side = nullptr;  // StockLevel phases run here, concurrently with the others
+  cudaEvent_t fork[2]{}, join[2]{};
 };
 
 struct TpccParams {
