@@ -13,58 +13,61 @@ constexpr int SCAN_ITEMS = 16;
 constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;  // 4096 elements per block
 
 // Block-wide exclusive scan of one value per thread; returns the block total.
-__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t& total) {
-  __shared__ uint32_t warp_tot[SCAN_THREADS / 32];
+template <class T>
+__device__ __forceinline__ T block_excl_scan(T v, T& total) {
+  __shared__ T warp_tot[SCAN_THREADS / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  uint32_t x = v;
+  T x = v;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    T y = __shfl_up_sync(0xffffffffu, x, o);
     if (lane >= o) x += y;
   }
   if (lane == 31) warp_tot[wid] = x;
   __syncthreads();
   if (wid == 0) {
-    uint32_t t = lane < SCAN_THREADS / 32 ? warp_tot[lane] : 0;
+    T t = lane < SCAN_THREADS / 32 ? warp_tot[lane] : T(0);
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      uint32_t y = __shfl_up_sync(0xffffffffu, t, o);
+      T y = __shfl_up_sync(0xffffffffu, t, o);
       if (lane >= o) t += y;
     }
     if (lane < SCAN_THREADS / 32) warp_tot[lane] = t;  // inclusive
   }
   __syncthreads();
   total = warp_tot[SCAN_THREADS / 32 - 1];
-  uint32_t base = wid ? warp_tot[wid - 1] : 0;
+  T base = wid ? warp_tot[wid - 1] : T(0);
   __syncthreads();
   return base + x - v;
 }
 
-__global__ void k_scan_reduce(const uint32_t* __restrict__ in, uint32_t n, uint32_t* __restrict__ sums) {
+template <class T>
+__global__ void k_scan_reduce(const T* __restrict__ in, uint32_t n, T* __restrict__ sums) {
   const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE;
-  uint32_t s = 0;
+  T s = 0;
 #pragma unroll
   for (int k = 0; k < SCAN_ITEMS; ++k) {
     uint64_t i = base + (uint64_t)k * SCAN_THREADS + threadIdx.x;
     if (i < n) s += in[i];
   }
-  uint32_t tot;
-  block_excl_scan(s, tot);
+  T tot;
+  block_excl_scan<T>(s, tot);
   if (threadIdx.x == 0) sums[blockIdx.x] = tot;
 }
 
 // single block: exclusive scan of the block sums (nb <= SCAN_TILE); sums[nb] = total
-__global__ void k_scan_top(uint32_t* sums, uint32_t nb) {
-  uint32_t v[SCAN_ITEMS];
-  uint32_t s = 0;
+template <class T>
+__global__ void k_scan_top(T* sums, uint32_t nb) {
+  T v[SCAN_ITEMS];
+  T s = 0;
 #pragma unroll
   for (int k = 0; k < SCAN_ITEMS; ++k) {
     uint32_t i = threadIdx.x * SCAN_ITEMS + k;
-    v[k] = i < nb ? sums[i] : 0;
+    v[k] = i < nb ? sums[i] : T(0);
     s += v[k];
   }
-  uint32_t tot;
-  uint32_t off = block_excl_scan(s, tot);
+  T tot;
+  T off = block_excl_scan<T>(s, tot);
 #pragma unroll
   for (int k = 0; k < SCAN_ITEMS; ++k) {
     uint32_t i = threadIdx.x * SCAN_ITEMS + k;
@@ -74,20 +77,21 @@ __global__ void k_scan_top(uint32_t* sums, uint32_t nb) {
   if (threadIdx.x == 0) sums[nb] = tot;
 }
 
-__global__ void k_scan_down(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t n,
-                            const uint32_t* __restrict__ sums, uint32_t nb) {
+template <class T>
+__global__ void k_scan_down(const T* __restrict__ in, T* __restrict__ out, uint32_t n,
+                            const T* __restrict__ sums, uint32_t nb) {
   // each thread owns SCAN_ITEMS consecutive elements of the tile (stable order)
   const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE + (uint64_t)threadIdx.x * SCAN_ITEMS;
-  uint32_t v[SCAN_ITEMS];
-  uint32_t s = 0;
+  T v[SCAN_ITEMS];
+  T s = 0;
 #pragma unroll
   for (int k = 0; k < SCAN_ITEMS; ++k) {
     uint64_t i = base + k;
-    v[k] = i < n ? in[i] : 0;
+    v[k] = i < n ? in[i] : T(0);
     s += v[k];
   }
-  uint32_t tot;
-  uint32_t off = block_excl_scan(s, tot) + sums[blockIdx.x];
+  T tot;
+  T off = block_excl_scan<T>(s, tot) + sums[blockIdx.x];
 #pragma unroll
   for (int k = 0; k < SCAN_ITEMS; ++k) {
     uint64_t i = base + k;
@@ -97,21 +101,30 @@ __global__ void k_scan_down(const uint32_t* __restrict__ in, uint32_t* __restric
   if (blockIdx.x == nb - 1 && threadIdx.x == 0) out[n] = sums[nb];
 }
 
-size_t scan_scratch_words(uint32_t n) { return (n + SCAN_TILE - 1) / SCAN_TILE + 2; }
+size_t scan_scratch_words(uint32_t n) { return 2 * ((n + SCAN_TILE - 1) / SCAN_TILE + 2); }
 
-// out[0..n) = exclusive prefix sums of in, out[n] = total.  Deterministic.
-void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s) {
+// out[0..n) = exclusive prefix sums of in, out[n] = total.  Deterministic.  scratch holds
+// scan_scratch_words(n) u32 words (enough for 64-bit sums).
+template <class T>
+static void scan_exclusive(const T* in, T* out, uint32_t n, void* scratch_v, cudaStream_t s) {
+  T* scratch = static_cast<T*>(scratch_v);
   if (n == 0) {
-    cudaMemsetAsync(out, 0, sizeof(uint32_t), s);
+    cudaMemsetAsync(out, 0, sizeof(T), s);
     return;
   }
   uint32_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;  // <= SCAN_TILE blocks (n <= 16.7M)
-  k_scan_reduce<<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch);
-  note_launch();
-  k_scan_top<<<1, SCAN_THREADS, 0, s>>>(scratch, nb);
-  note_launch();
-  k_scan_down<<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb);
-  note_launch();
+  k_scan_reduce<T><<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch);
+  k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>(scratch, nb);
+  k_scan_down<T><<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb);
+  note_launch(3);
+}
+
+void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s) {
+  scan_exclusive<uint32_t>(in, out, n, scratch, s);
+}
+void scan_exclusive_u64(const unsigned long long* in, unsigned long long* out, uint32_t n, uint32_t* scratch,
+                        cudaStream_t s) {
+  scan_exclusive<unsigned long long>(in, out, n, scratch, s);
 }
 
 // Result finalisation: commit bitmask (one __ballot_sync word per warp), conflict

@@ -267,7 +267,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const DevTable& TOL_ = c_tabs[TOL];
       const DevTable& TNw = c_tabs[TNO];
       if (active && sub < n) {  // ORDER_LINE row
-        const uint32_t row = (uint32_t)(*TOL_.n_rows + tp.no_lines[r] + sub);
+        const uint32_t row = (uint32_t)(*TOL_.n_rows + (tp.no_pref[r] >> 32) + sub);
         wr(TOL_, OL_I_ID, row, i);
         wr(TOL_, OL_SUPPLY_W_ID, row, sw);
         wr(TOL_, OL_QUANTITY, row, qty);
@@ -280,8 +280,8 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         if (sl) sl->row = row; else internal_error(x);
       }
       if (sub == 15) {  // ORDER and NEW_ORDER rows
-        const uint32_t orow = (uint32_t)(*TOr.n_rows + tp.no_flag[r]);
-        if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + tp.no_lines[r]);  // contiguous lines
+        const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)tp.no_pref[r]);
+        if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + (tp.no_pref[r] >> 32));  // contiguous lines
         wr(TOr, O_C_ID, orow, c);
         wr(TOr, O_ENTRY_D, orow, b.clock);
         wr(TOr, O_OL_CNT, orow, n);
@@ -291,7 +291,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         TOr.valid[orow] = 1;
         IdxSlot* sl = idx_find_or_insert(TOr, okey);
         if (sl) sl->row = orow; else internal_error(x);
-        const uint32_t nrow = (uint32_t)(*TNw.n_rows + tp.no_flag[r]);
+        const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)tp.no_pref[r]);
         wr(TNw, NO_O_ID, nrow, o);
         TNw.rowkey[nrow] = okey;
         TNw.valid[nrow] = 1;
@@ -848,8 +848,7 @@ __global__ void k_no_prep(BatchDev b, TpccParams tp) {
   if (r >= b.n_txns) return;
   const uint8_t* p = b.params + 128ull * r;
   const bool c = b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT && owns_w(b, p16(p, 0));
-  tp.no_flag[r] = c;
-  tp.no_lines[r] = c ? p[3] : 0;
+  tp.no_pref[r] = c ? ((unsigned long long)p[3] << 32 | 1ull) : 0ull;
   tp.dk_of[r] = c ? (uint32_t)kD(p16(p, 0), p[2]) : ~0u;
 }
 
@@ -946,9 +945,9 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
 __global__ void k_tpcc_advance(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t n = b.n_txns;
-  *c_tabs[TO].n_rows += tp.no_flag[n];
-  *c_tabs[TNO].n_rows += tp.no_flag[n];
-  *c_tabs[TOL].n_rows += tp.no_lines[n];
+  *c_tabs[TO].n_rows += (uint32_t)tp.no_pref[n];
+  *c_tabs[TNO].n_rows += (uint32_t)tp.no_pref[n];
+  *c_tabs[TOL].n_rows += tp.no_pref[n] >> 32;
   *c_tabs[TH].n_rows += tp.misc[M_HIST];
 }
 
@@ -994,7 +993,7 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
   if (shared_by_name) t.by_name = shared_by_name;
   else if (dm(&t.by_name, (uint64_t)t.dsz * 1000)) return LTPG_ENOMEM;
   if (dm(&t.list, (uint64_t)NTYPES * max_txns) || dm(&t.clist, (uint64_t)NTYPES * max_txns) ||
-      dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_flag, max_txns + 1ull) || dm(&t.no_lines, max_txns + 1ull) ||
+      dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_pref, max_txns + 1ull) ||
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
     return LTPG_ENOMEM;
   if (t.owns_by_name) cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
@@ -1013,7 +1012,7 @@ void tpcc_free(TpccDev& t) {
     if (t.join[k]) cudaEventDestroy(t.join[k]);
   }
   if (!t.owns_by_name) t.by_name = nullptr;
-  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
+  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
   for (void* p : ps)
     if (p) cudaFree(p);
   t = TpccDev{};
@@ -1045,7 +1044,7 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
 static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists) {
   const uint32_t n = b.n_txns;
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
-                    t.no_flag, t.no_lines, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
+                    t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
 }
 static uint32_t phase_grid(uint32_t n) {
@@ -1091,8 +1090,7 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders
   k_no_prep<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   note_launch();
-  scan_exclusive_u32(t.no_flag, t.no_flag, n, scan_scratch, s);
-  scan_exclusive_u32(t.no_lines, t.no_lines, n, scan_scratch, s);
+  scan_exclusive_u64(t.no_pref, t.no_pref, n, scan_scratch, s);  // row and line offsets at once
   const size_t smem = (size_t)t.dsz * sizeof(uint32_t);
   k_no_hist<<<tp.n_chunks, 256, smem, s>>>(b, tp);
   k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);

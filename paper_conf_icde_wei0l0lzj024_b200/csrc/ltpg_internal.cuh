@@ -318,6 +318,8 @@ __device__ __forceinline__ bool owns_w(const BatchDev& b, uint32_t w) {
 
 
 void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
+void scan_exclusive_u64(const unsigned long long* in, unsigned long long* out, uint32_t n, uint32_t* scratch,
+                        cudaStream_t s);
 size_t scan_scratch_words(uint32_t n);
 
 void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool grouped,

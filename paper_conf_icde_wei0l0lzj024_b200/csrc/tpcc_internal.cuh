@@ -33,8 +33,7 @@ struct TpccDev {
   uint32_t* list = nullptr;     // [NTYPES][max_txns] ranks, grouped by procedure type
   uint32_t* clist = nullptr;    // [NTYPES][max_txns] committed ranks (write-back only)
   uint32_t* log = nullptr;      // [max_txns][TLOG] rows found by execute
-  uint32_t* no_flag = nullptr;  // [max_txns+1] committed NewOrder -> exclusive scan (row offsets)
-  uint32_t* no_lines = nullptr; // [max_txns+1] committed NewOrder lines -> exclusive scan
+  unsigned long long* no_pref = nullptr;  // [max_txns+1] committed NewOrder (lines << 32 | 1) -> exclusive scan
   uint32_t* dk_of = nullptr;    // [max_txns] district key of a committed NewOrder, else ~0
   uint32_t* chunk_cnt = nullptr;// [chunks][dsz]
   long long* dist_base = nullptr; // [dsz] snapshot D_NEXT_O_ID
@@ -48,8 +47,7 @@ struct TpccParams {
   uint32_t* list;
   const uint32_t* counts;       // per-type list lengths of `list` (kcount, or misc + M_CCOUNT)
   uint32_t* log;
-  uint32_t* no_flag;
-  uint32_t* no_lines;
+  unsigned long long* no_pref;  // exclusive prefix: low 32 = committed NewOrders, high 32 = their lines
   uint32_t* dk_of;
   uint32_t* chunk_cnt;
   long long* dist_base;
