@@ -116,9 +116,10 @@ def measured_peaks():
     return 6650.0, "fallback"
 
 
-def ncu_traffic(kernel_substr):
-    """dram read+write bytes per launch of the kernel from the committed `ncu --set full` summary."""
-    p = os.path.join(ROOT, "profiles", "ncu_r01_ycsb_c3.json")
+def ncu_traffic(workload, kernel_substr):
+    """dram read+write bytes per launch of the kernel from the committed `ncu --set full`
+    summary of this workload (profiles/ncu_r01_<workload>.json), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_r01_%s.json" % workload)
     if not os.path.exists(p):
         return None
     try:
@@ -177,6 +178,29 @@ def tpcc_exec_algorithmic_bytes(batch, mode):
     b[ty == 3] = 128 + 10 * (32 + 64 + 32 + 32 + 3 * 32 + 4 + 64 + 10 * (8 + 16) + 64) + 32
     b[ty == 4] = 128 + 32 + 20 * (32 + 32 + 4 + 10 * 8) + 190 * 32 + 32
     return int(b.sum())
+
+
+def fused_algorithmic_bytes(batch):
+    """Algorithmic bytes of the fused OPS kernel (validate + warp-local division + execute):
+    the execute bytes above + 16 B per txn (TID 8 B, op_begin 4 B, txn_ins 4 B)."""
+    return exec_algorithmic_bytes(batch) + 16 * len(batch["tid"])
+
+
+# B200 random-access ceiling measured by tools/randbw.cu (profiles/randbw_r01.txt): independent
+# random 8-byte reads from a >> L2 array retire at ~48.6 G/s whatever the load flavour or the
+# DRAM bytes fetched per access -- a request-rate limit well below the sequential HBM peak.
+RANDOM_READ_CEILING_G = 48.6
+
+
+def ops_random_reads(batch):
+    """Independent random row-sized reads the OPS execute does per batch: one column read per
+    SELECT / UPDATE (dense key -> row by arithmetic), one mark-filter read per UPDATE / ADD
+    (its atomicMin then hits the line in L2), one read per SCANned key; INSERT / DELETE 2."""
+    ops = batch["ops"]
+    kinds = ops["kind"]
+    n = np.bincount(kinds, minlength=6)
+    scan_keys = int(ops["aux"][kinds == 5].astype(np.int64).sum())
+    return int(n[0] + 2 * n[1] + n[2] + 2 * (n[3] + n[4]) + scan_keys)
 
 
 def step_algorithmic_bytes(batch):
@@ -298,6 +322,8 @@ def main():
     B = w["batch"]
     if w.get("reorder"):
         args.flags |= ltpg.LTPG_FLAG_REORDER
+    fused_front = w["kind"] == "ycsb" and not (args.flags & (ltpg.LTPG_FLAG_REORDER | ltpg.LTPG_FLAG_NO_GROUPING
+                                                              | ltpg.LTPG_FLAG_UNFUSED))
     uid = None
     if world > 1:  # one NCCL communicator per db: the per-batch verdict exchange
         from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id
@@ -401,7 +427,7 @@ def main():
         st = out["stats"]
         commits.append(st["n_commit"])
         procs.append(len(host_batches[i]["tid"]))
-        exec_ms.append(st["ms_exec"])
+        exec_ms.append(st["ms_group"] if fused_front else st["ms_exec"])
         kernels += st["n_kernels"]
         stage.append(st)
     torch.cuda.synchronize()
@@ -477,21 +503,30 @@ def main():
     peak, peak_kind = measured_peaks()
     roof = None
     if w["kind"] == "ycsb":
-        bytes_exec = statistics.mean(exec_algorithmic_bytes(host_batches[(args.warmup + s) % n_distinct])
+        model = fused_algorithmic_bytes if fused_front else exec_algorithmic_bytes
+        kname = "k_ops_fused" if fused_front else "k_ops_exec"
+        bytes_exec = statistics.mean(model(host_batches[(args.warmup + s) % n_distinct])
                                      for s in range(args.steps))
         ms = statistics.mean(exec_ms)
         ach = bytes_exec / (ms / 1000.0) / 1e9
-        roof = {"bound": "hbm", "kernel": "k_ops_exec", "achieved": ach, "peak": peak, "unit": "GB/s",
-                "frac": ach / peak, "traffic": ncu_traffic("k_ops_exec"), "peak_source": peak_kind,
+        roof = {"bound": "hbm", "kernel": kname, "achieved": ach, "peak": peak, "unit": "GB/s",
+                "frac": ach / peak, "traffic": ncu_traffic(name, kname), "peak_source": peak_kind,
                 "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
                 "kernel_share_of_step": ms / statistics.mean(step_ms)}
+        nrand = statistics.mean(ops_random_reads(host_batches[(args.warmup + s) % n_distinct])
+                                for s in range(args.steps))
+        roof["random_access"] = {
+            "reads_per_launch": nrand, "ceiling_g_per_s": RANDOM_READ_CEILING_G,
+            "achieved_g_per_s": nrand / (ms / 1000.0) / 1e9,
+            "frac": nrand / (ms / 1000.0) / 1e9 / RANDOM_READ_CEILING_G,
+            "source": "tools/randbw.cu, profiles/randbw_r01.txt"}
     else:
         bytes_exec = statistics.mean(tpcc_exec_algorithmic_bytes(host_batches[(args.warmup + s) % n_distinct],
                                                                   w["mode"]) for s in range(args.steps))
         ms = statistics.mean(exec_ms)
         ach = bytes_exec / (ms / 1000.0) / 1e9
         roof = {"bound": "hbm", "kernel": "k_tpcc_phase<PH_EXEC>", "achieved": ach, "peak": peak, "unit": "GB/s",
-                "frac": ach / peak, "traffic": ncu_traffic("k_tpcc_phase<0>"), "peak_source": peak_kind,
+                "frac": ach / peak, "traffic": ncu_traffic(name, "k_tpcc_phase<0>"), "peak_source": peak_kind,
                 "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
                 "kernel_share_of_step": ms / statistics.mean(step_ms)}
 

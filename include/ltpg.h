@@ -127,6 +127,8 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
 #define LTPG_FLAG_NO_MARK_FILTER (1u << 1) /* A/B: always issue the atomicMin mark        */
 #define LTPG_FLAG_REORDER       (1u << 2)  /* NEXT-1 logical reordering: abort iff
                                               WAW or (RAW and WAR); keeps per-unit min reader marks */
+#define LTPG_FLAG_UNFUSED       (1u << 3)  /* A/B: OPS mode runs validate+division and execute as
+                                              two kernels with global per-kind lists          */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
 
 typedef struct {

@@ -34,6 +34,7 @@ LTPG_MODE_OPS, LTPG_MODE_TPCC = 0, 1
 LTPG_FLAG_NO_GROUPING = 1 << 0
 LTPG_FLAG_NO_MARK_FILTER = 1 << 1
 LTPG_FLAG_REORDER = 1 << 2
+LTPG_FLAG_UNFUSED = 1 << 3
 LTPG_FLAG_LOOPBACK_SHIFT = 8
 LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
 

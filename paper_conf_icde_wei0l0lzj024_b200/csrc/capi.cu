@@ -592,6 +592,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
   const bool reorder = (db->cfg.flags & LTPG_FLAG_REORDER) != 0;
+  // fused OPS front end; NEXT-1 needs min reader marks on claimed keys, so it keeps the lists
+  const bool fused = grouped && !reorder && !(db->cfg.flags & LTPG_FLAG_UNFUSED);
   std::vector<BatchDev> pb(L, bd);
   for (uint32_t p = 0; p < L; ++p) {
     Part& P = db->parts[p];
@@ -631,12 +633,21 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       BatchDev& x = pb[p];
       cudaEvent_t* evp = (timing && p == L - 1) ? S.ev : nullptr;
       if (ops_mode) {
-        launch_ops_validate_group(db->n_tables, x, grouped, s);
-        scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
-        launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
-        launch_ops_claim(x, s);
-        if (evp) CK(cudaEventRecord(evp[2], s));
-        launch_ops_exec(x, grouped, filter, s);
+        if (fused) {  // validate + warp-local division + execute; INSERTs after their claims
+          launch_ops_fused(db->n_tables, x, filter, s);
+          if (evp) CK(cudaEventRecord(evp[2], s));  // ms_group = the fused kernel; ms_exec = INSERT tail
+          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
+          launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
+          launch_ops_claim(x, s);
+          launch_ops_exec_inserts(x, filter, s);
+        } else {
+          launch_ops_validate_group(db->n_tables, x, grouped, s);
+          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
+          launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
+          launch_ops_claim(x, s);
+          if (evp) CK(cudaEventRecord(evp[2], s));
+          launch_ops_exec(x, grouped, filter, s);
+        }
         if (evp) CK(cudaEventRecord(evp[3], s));
         launch_ops_detect(x, s);
       } else {

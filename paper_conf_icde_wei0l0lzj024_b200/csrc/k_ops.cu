@@ -58,6 +58,57 @@ __device__ __forceinline__ bool op_touches(const BatchDev& b, const ltpg_op& o) 
   return p0 <= b.part && b.part <= p1;
 }
 
+// ---- a1: validation of one txn (R2-R4, R10) over a staged or global op accessor --------
+template <class Get>
+__device__ __forceinline__ bool validate_txn(uint32_t n_tables, const BatchDev& b, uint32_t r, bool staged,
+                                             uint32_t w0, uint32_t w1, Get get, uint32_t& b0, uint32_t& b1,
+                                             uint64_t& cnt64, uint32_t& ins_tables, uint32_t& insdel) {
+  bool bad = false;
+  if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
+  b0 = b.op_begin[r];
+  b1 = b.op_begin[r + 1];
+  if (r == 0 && b0 != 0) bad = true;
+  if (r == b.n_txns - 1 && b1 != b.n_ops) bad = true;
+  if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS || (staged && (b0 < w0 || b1 > w1))) {
+    bad = true;
+    b1 = b0;
+  }
+  for (uint32_t i = b0; i < b1; ++i) {
+    const ltpg_op o = get(i);
+    if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) insdel |= 1u << (o.table & 31);
+    if (!op_valid(n_tables, o)) { bad = true; continue; }
+    if (!op_touches(b, o)) continue;
+    cnt64 += 1ull << (10 * o.kind);
+    if (o.kind == LTPG_INSERT) ins_tables |= 1u << o.table;
+  }
+  // R10: a written key is touched by no other op of the txn (no read-your-writes)
+  for (uint32_t i = b0 + 1; i < b1 && !bad; ++i) {
+    const ltpg_op a = get(i);
+    const uint64_t alo = a.key, ahi = a.kind == LTPG_SCAN ? a.key + a.aux : a.key + 1;
+    for (uint32_t j = b0; j < i; ++j) {
+      const ltpg_op c = get(j);
+      if (c.table != a.table) continue;
+      const uint64_t clo = c.key, chi = c.kind == LTPG_SCAN ? c.key + c.aux : c.key + 1;
+      if (!(alo < chi && clo < ahi)) continue;
+      if (is_write_kind(a.kind) || is_write_kind(c.kind) || (a.kind != LTPG_SCAN && c.kind != LTPG_SCAN)) {
+        bad = true;
+        break;
+      }
+    }
+  }
+  return bad;
+}
+
+__device__ __forceinline__ ltpg_op unpack_op(ulonglong2 v) {
+  ltpg_op o;
+  o.key = v.x;
+  o.kind = (uint8_t)(v.y);
+  o.table = (uint8_t)(v.y >> 8);
+  o.col = (uint16_t)(v.y >> 16);
+  o.aux = (uint32_t)(v.y >> 32);
+  return o;
+}
+
 // ---- K-group: validation + decomposition into per-kind lists (one thread per txn) ----
 template <bool GROUPED>
 __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
@@ -85,51 +136,11 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
       *reinterpret_cast<ulonglong2*>(&stage[wib][q - w0]) = *reinterpret_cast<const ulonglong2*>(b.ops + q);
   __syncwarp();
   auto get = [&](uint32_t q) -> ltpg_op {
-    if (staged) {
-      const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(&stage[wib][q - w0]);
-      ltpg_op o;
-      o.key = v.x;
-      o.kind = (uint8_t)(v.y);
-      o.table = (uint8_t)(v.y >> 8);
-      o.col = (uint16_t)(v.y >> 16);
-      o.aux = (uint32_t)(v.y >> 32);
-      return o;
-    }
+    if (staged) return unpack_op(*reinterpret_cast<const ulonglong2*>(&stage[wib][q - w0]));
     return load_op(b.ops, q);
   };
   if (r < b.n_txns) {
-    if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;  // TIDs strictly increasing
-    b0 = b.op_begin[r];
-    b1 = b.op_begin[r + 1];
-    if (r == 0 && b0 != 0) bad = true;
-    if (r == b.n_txns - 1 && b1 != b.n_ops) bad = true;
-    if (b1 < b0 || b1 > b.n_ops || b1 - b0 > OPS_MAX_TXN_OPS || (staged && (b0 < w0 || b1 > w1))) {
-      bad = true;
-      b1 = b0;
-    }
-    for (uint32_t i = b0; i < b1; ++i) {
-      const ltpg_op o = get(i);
-      if (o.kind == LTPG_INSERT || o.kind == LTPG_DELETE) my_insdel |= 1u << (o.table & 31);
-      if (!op_valid(n_tables, o)) { bad = true; continue; }
-      if (!op_touches(b, o)) continue;
-      cnt64 += 1ull << (10 * o.kind);
-      if (o.kind == LTPG_INSERT) my_ins_tables |= 1u << o.table;
-    }
-    // R10: a written key is touched by no other op of the txn (no read-your-writes)
-    for (uint32_t i = b0 + 1; i < b1 && !bad; ++i) {
-      const ltpg_op a = get(i);
-      const uint64_t alo = a.key, ahi = a.kind == LTPG_SCAN ? a.key + a.aux : a.key + 1;
-      for (uint32_t j = b0; j < i; ++j) {
-        const ltpg_op c = get(j);
-        if (c.table != a.table) continue;
-        const uint64_t clo = c.key, chi = c.kind == LTPG_SCAN ? c.key + c.aux : c.key + 1;
-        if (!(alo < chi && clo < ahi)) continue;
-        if (is_write_kind(a.kind) || is_write_kind(c.kind) || (a.kind != LTPG_SCAN && c.kind != LTPG_SCAN)) {
-          bad = true;
-          break;
-        }
-      }
-    }
+    bad = validate_txn(n_tables, b, r, staged, w0, w1, get, b0, b1, cnt64, my_ins_tables, my_insdel);
     b.txn_ins[r] = (uint32_t)(cnt64 >> (10 * LTPG_INSERT)) & 1023u;
     if (bad) atomicOr(b.err, ERR_EINVAL);
   }
@@ -211,8 +222,11 @@ __device__ __forceinline__ void mark_read(const DevTable& T, uint32_t g, uint32_
   if (T.rmarks) mark_min(rmark_ptr(T, g, row), tag, filter);  // NEXT-1 only: min reader rank
 }
 
-__device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
-                                         uint32_t r, const ltpg_op& o, bool filter, uint32_t dmask) {
+// uref bit 58: absent key read before K-claim ran (fused path); K-detect probes it for a claim
+constexpr uint64_t UREF_RECHECK = 1ull << 58;
+
+__device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi, uint32_t r, const ltpg_op& o,
+                                         bool filter, uint32_t dmask, bool pre_claim = false) {
   const DevTable& T = c_tabs[o.table];
   const unsigned long long tag = epoch_tag(b.epoch) | r;
   uint32_t row, claim;
@@ -244,6 +258,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi,
     // absent key: a READ of its existence; only an inserter of this batch can conflict
     if (claim != ROW_NONE) mark_read(T, 0, claim, tag, filter);
     uref = claim != ROW_NONE ? make_uref(CHK_RW, false, false, o.table, 0, claim)
+           : pre_claim       ? (make_uref(CHK_RW, false, false, o.table, 0, 0) | UREF_RECHECK)
                              : make_uref(CHK_NONE, false, false, o.table, 0, 0);
     b.res[oi] = LTPG_NOT_FOUND;
     b.uref[oi] = uref;
@@ -327,6 +342,119 @@ __global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
   }
 }
 
+// ---- K-fused: a1 + warp-local kind division + a4/a5 in one pass ------------
+// Each warp validates its 32 txns from shared memory, orders its own ops by kind and runs
+// them 32 at a time, so a warp executes one op kind except at the few kind boundaries --
+// the warp-division effect without the global lists' round trip through HBM.  INSERTs go
+// to the INSERT list (K-claim, then K-exec on that list); reads of keys absent from the
+// index carry UREF_RECHECK so K-detect finds claims made after this kernel.
+__global__ void __launch_bounds__(256) k_ops_fused(uint32_t n_tables, BatchDev b, bool filter) {
+  constexpr uint32_t STAGE = 320;  // YCSB: 32 txns x 10 ops; larger warps run unstaged
+  __shared__ __align__(16) ltpg_op stage[8][STAGE];
+  __shared__ uint16_t perm[8][STAGE];  // staged op index | lane << 9, ordered by kind
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t wib = threadIdx.x >> 5;
+  const uint32_t dmask = *b.dense_live;  // INSERT/DELETE take effect at write-back only
+  bool bad = false;
+  uint32_t b0 = 0, b1 = 0;
+  uint64_t cnt64 = 0;
+  uint32_t my_ins_tables = 0, my_insdel = 0;
+  const uint32_t r0 = r - lane;
+  const uint32_t rl = min(r0 + 32, b.n_txns);
+  uint32_t w0 = 0, w1 = 0;
+  if (r0 < b.n_txns) {
+    w0 = b.op_begin[r0];
+    w1 = b.op_begin[rl];
+  }
+  const bool staged = r0 < b.n_txns && w1 >= w0 && w1 - w0 <= STAGE && w1 <= b.n_ops;
+  if (staged)
+    for (uint32_t q = w0 + lane; q < w1; q += 32)
+      *reinterpret_cast<ulonglong2*>(&stage[wib][q - w0]) = *reinterpret_cast<const ulonglong2*>(b.ops + q);
+  __syncwarp();
+  auto get = [&](uint32_t q) -> ltpg_op {
+    if (staged) return unpack_op(*reinterpret_cast<const ulonglong2*>(&stage[wib][q - w0]));
+    return load_op(b.ops, q);
+  };
+  if (r < b.n_txns) {
+    bad = validate_txn(n_tables, b, r, staged, w0, w1, get, b0, b1, cnt64, my_ins_tables, my_insdel);
+    b.txn_ins[r] = (uint32_t)(cnt64 >> (10 * LTPG_INSERT)) & 1023u;
+    if (bad) atomicOr(b.err, ERR_EINVAL);
+  }
+  my_ins_tables = __reduce_or_sync(0xffffffffu, my_ins_tables);
+  if (lane == 0 && my_ins_tables) atomicOr(b.ins_tables, my_ins_tables);
+  my_insdel = __reduce_or_sync(0xffffffffu, my_insdel);
+  if (lane == 0 && my_insdel) atomicOr(b.insdel, my_insdel);
+  if (bad) cnt64 = 0, b1 = b0;  // the batch fails; run nothing of this txn
+  // INSERT list: warp-aggregated reservation
+  const uint32_t nins = (uint32_t)(cnt64 >> (10 * LTPG_INSERT)) & 1023u;
+  uint32_t ins_pos = nins;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, ins_pos, o);
+    if (lane >= (uint32_t)o) ins_pos += y;
+  }
+  uint32_t ins_base = 0;
+  if (lane == 31 && ins_pos) ins_base = atomicAdd(b.kcount + LTPG_INSERT, ins_pos);
+  ins_pos += __shfl_sync(0xffffffffu, ins_base, 31) - nins;
+  unsigned long long* ins_list = b.items + (uint64_t)LTPG_INSERT * b.max_ops;
+  if (!staged) {  // large txns: each lane runs its own ops in op order
+    for (uint32_t i = b0; i < b1; ++i) {
+      const ltpg_op o = load_op(b.ops, i);
+      if (!op_touches(b, o)) continue;
+      if (o.kind == LTPG_INSERT) ins_list[ins_pos++] = (unsigned long long)i | ((unsigned long long)r << 32);
+      else exec_one(b, i, r, o, filter, dmask, true);
+    }
+    return;
+  }
+  // warp-local kind order: inclusive scan of the packed counts (each warp total <= STAGE < 1024)
+  const uint64_t mine = cnt64 & ~(1023ull << (10 * LTPG_INSERT));
+  uint64_t inc = mine;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= (uint32_t)o) inc += y;
+  }
+  const uint64_t tot = __shfl_sync(0xffffffffu, inc, 31);
+  const uint64_t excl = inc - mine;
+  uint32_t pos[NKINDS], run = 0;
+#pragma unroll
+  for (int k = 0; k < NKINDS; ++k) {
+    pos[k] = run + ((uint32_t)(excl >> (10 * k)) & 1023u);
+    run += (uint32_t)(tot >> (10 * k)) & 1023u;
+  }
+  for (uint32_t i = b0; i < b1; ++i) {
+    const ltpg_op o = get(i);
+    if (!op_touches(b, o)) continue;
+    if (o.kind == LTPG_INSERT) {
+      ins_list[ins_pos++] = (unsigned long long)i | ((unsigned long long)r << 32);
+      continue;
+    }
+    uint32_t p = 0;
+#pragma unroll
+    for (int k = 0; k < NKINDS; ++k)
+      if (k == o.kind) p = pos[k]++;
+    perm[wib][p] = (uint16_t)((i - w0) | (lane << 9));
+  }
+  __syncwarp();
+  for (uint32_t q = lane; q < run; q += 32) {
+    const uint32_t e = perm[wib][q];
+    const uint32_t li = e & 511u;
+    const ltpg_op o = unpack_op(*reinterpret_cast<const ulonglong2*>(&stage[wib][li]));
+    exec_one(b, w0 + li, r0 + (e >> 9), o, filter, dmask, true);
+  }
+}
+
+void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStream_t s) {
+  k_ops_fused<<<(b.n_txns + 255) / 256, 256, 0, s>>>(n_tables, b, filter);
+  note_launch();
+}
+
+void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s) {
+  k_ops_exec<true><<<148 * 2, 256, 0, s>>>(b, filter);  // only the INSERT list is populated
+  note_launch();
+}
+
 void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s) {
   uint64_t warps = (b.n_ops + NKINDS * 32 + 31) / 32;
   uint64_t blocks = (warps + 7) / 8;
@@ -369,6 +497,13 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
         if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b.epoch);
         else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b.epoch);
       }
+      continue;
+    }
+    if (u & UREF_RECHECK) {  // absent at execution (fused path): an INSERT may have claimed it since
+      const ltpg_op o = load_op(b.ops, i);
+      uint32_t row, claim;
+      lookup(T, t, dmask, o.key, row, claim);
+      if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b.epoch);
       continue;
     }
     const uint32_t row = (uint32_t)u;

@@ -326,6 +326,8 @@ void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool groupe
                                cudaStream_t s);
 void launch_ops_claim(const BatchDev& b, cudaStream_t s);
 void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
+void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStream_t s);
+void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s);
 void launch_ops_detect(const BatchDev& b, cudaStream_t s);
 void launch_ops_writeback(const BatchDev& b, cudaStream_t s);
 void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,

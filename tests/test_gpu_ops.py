@@ -54,7 +54,7 @@ def test_example3_gpu(encoding):
     assert [i + 1 for i, s in enumerate(st) if s == ST_COMMIT] == gold["expected_commits"][encoding]["value"]
 
 
-@pytest.mark.parametrize("flags", [0, 1, 2, 3])
+@pytest.mark.parametrize("flags", [0, 1, 2, 3, 8, 10])
 @pytest.mark.parametrize("seed", range(12))
 def test_random_tiny_batches_all_kinds(seed, flags):
     """Every op kind incl. INSERT claims, DELETE, SCAN over absent keys; grouping and

@@ -95,9 +95,10 @@ def main():
     ap.add_argument("--out", required=True)
     ap.add_argument("--tag", default="")
     ap.add_argument("--note", default="")
+    ap.add_argument("--fresh", action="store_true", help="drop kernels of an existing summary")
     a = ap.parse_args()
     res = {"tag": a.tag, "note": a.note}
-    if os.path.exists(a.out):
+    if os.path.exists(a.out) and not a.fresh:
         old = json.load(open(a.out))
         res["kernels"] = old.get("kernels", {})
     else:
