@@ -169,7 +169,14 @@ typedef struct {
   uint64_t capacity_rows;       /* rows incl. the append region                          */
   uint32_t has_pk;              /* 1: u64 primary key + hash index; 0: keyless (append)  */
   uint32_t owner_rule;          /* multi-GPU: 0 replicated, 1 TPC-C warehouse, 2 key range */
+  uint32_t layout;              /* LTPG_LAYOUT_*: placement of the columns in HBM          */
 } ltpg_table_desc;
+
+/* Column placement (result-invisible).  ROWBLOCK: per row, the non-static
+ * columns side by side and the static columns side by side (blocks of <= 8 words padded to
+ * a power of two) -- for randomly accessed rows whose columns are used together.
+ * COLUMNAR: one array per column -- for append-heavy tables written by consecutive lanes. */
+enum { LTPG_LAYOUT_ROWBLOCK = 0, LTPG_LAYOUT_COLUMNAR = 1 };
 
 /* Define table_id and load n_rows rows.  keys: host u64[n_rows] (NULL if keyless);
  * cols: host int64, column-major [n_cols][n_rows].  Duplicate keys -> EINVAL. */

@@ -35,6 +35,7 @@ LTPG_FLAG_NO_GROUPING = 1 << 0
 LTPG_FLAG_NO_MARK_FILTER = 1 << 1
 LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_UNFUSED = 1 << 3
+LTPG_LAYOUT_ROWBLOCK, LTPG_LAYOUT_COLUMNAR = 0, 1
 LTPG_FLAG_LOOPBACK_SHIFT = 8
 LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
 
@@ -49,7 +50,7 @@ class ltpg_config(ctypes.Structure):
 
 class ltpg_table_desc(ctypes.Structure):
     _fields_ = [("n_cols", c_u32), ("col_group", c_vp), ("col_is_add", c_vp), ("n_groups", c_u32),
-                ("capacity_rows", c_u64), ("has_pk", c_u32), ("owner_rule", c_u32)]
+                ("capacity_rows", c_u64), ("has_pk", c_u32), ("owner_rule", c_u32), ("layout", c_u32)]
 
 
 class ltpg_batch(ctypes.Structure):
@@ -168,7 +169,7 @@ class Database:
             raise LtpgError(rc, ltpg_last_error(self.h).decode())
 
     def load_table(self, t, col_group, col_is_add, n_groups, keys, cols, capacity=None, has_pk=True,
-                   owner_rule=0):
+                   owner_rule=0, layout=0):
         g = np.ascontiguousarray(col_group, dtype=np.uint8)
         a = np.ascontiguousarray(col_is_add, dtype=np.uint8)
         cols = np.ascontiguousarray(cols, dtype=np.int64)
@@ -176,7 +177,8 @@ class Database:
         k = None if (keys is None or not has_pk) else np.ascontiguousarray(keys, dtype=np.uint64)
         cap = int(capacity if capacity is not None else max(n, 1))
         d = ltpg_table_desc(n_cols=len(g), col_group=_ptr(g), col_is_add=_ptr(a), n_groups=n_groups,
-                            capacity_rows=cap, has_pk=int(bool(has_pk)), owner_rule=owner_rule)
+                            capacity_rows=cap, has_pk=int(bool(has_pk)), owner_rule=owner_rule,
+                            layout=layout)
         self._check(ltpg_load_table(self.h, t, ctypes.byref(d), n, _ptr(k), _ptr(cols)))
         self.n_cols[t] = len(g)
         self.has_pk[t] = bool(has_pk)
@@ -366,6 +368,9 @@ def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, f
         cap = n + extra.get(t, 0) * max_txns * append_batches
         if capacity and t in capacity:
             cap = capacity[t]
+        # append-heavy tables columnar (consecutive lanes append whole sectors); the randomly
+        # accessed ones row-blocked (a STOCK / CUSTOMER update writes one sector)
         db.load_table(t, g, a, ng, k, c, capacity=max(cap, 1), has_pk=pk,
-                      owner_rule=0 if t == T_ITEM else 1)
+                      owner_rule=0 if t == T_ITEM else 1,
+                      layout=LTPG_LAYOUT_COLUMNAR if t in (T_ORDER, T_ORDER_LINE) else LTPG_LAYOUT_ROWBLOCK)
     return db

@@ -140,7 +140,8 @@ cudaError_t dmalloc(T** p, size_t n) {
 }
 
 void free_table(DevTable& T) {
-  if (T.col0) cudaFree(T.col0);
+  if (T.dyn) cudaFree(T.dyn);
+  if (T.stat) cudaFree(T.stat);
   if (T.valid) cudaFree(T.valid);
   if (T.rowkey) cudaFree(T.rowkey);
   if (T.marks) cudaFree(T.marks);
@@ -335,7 +336,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   if (db->poisoned) return LTPG_EPOISONED;
   if (!d || t >= db->n_tables || d->n_cols > MAXC || (d->n_cols && (!d->col_group || !d->col_is_add)) ||
       n_rows > d->capacity_rows || d->capacity_rows >= 0xFFFFFFF0ull || (n_rows && d->n_cols && !cols) ||
-      (d->has_pk && n_rows && !keys) || d->n_groups > 15 || d->owner_rule > 2)
+      (d->has_pk && n_rows && !keys) || d->n_groups > 15 || d->owner_rule > 2 || d->layout > LTPG_LAYOUT_COLUMNAR)
     return fail(db, LTPG_EINVAL, "bad table descriptor");
   bool has_static = false;
   for (uint32_t c = 0; c < d->n_cols; ++c) {
@@ -362,24 +363,51 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   T.defined = 1;
   T.owner_rule = d->owner_rule;
   T.capacity = cap;
-  long long* colmem = nullptr;
-  CK(dmalloc(&colmem, cap * std::max<uint32_t>(d->n_cols, 1)));
-  T.col0 = colmem;
+  // row-block layout: mutable block (non-static columns), static block; marks separate
+  uint32_t n_dyn = 0, n_stat = 0;
+  for (uint32_t c = 0; c < d->n_cols; ++c) (d->col_group[c] == LTPG_STATIC ? n_stat : n_dyn)++;
+  // pad blocks of up to 8 words to a power of two (a row never straddles a 64 B unit); wider
+  // rows stay unpadded so that appends from consecutive lanes fill whole sectors
+  auto pad_words = [](uint32_t w) -> uint32_t {
+    if (w == 0 || w > 8) return w;
+    uint32_t p = 1;
+    while (p < w) p <<= 1;
+    return p;
+  };
+  T.dstride = pad_words(n_dyn);
+  T.sstride = pad_words(n_stat);
+  if (T.dstride) CK(dmalloc(&T.dyn, cap * T.dstride));
+  if (T.sstride) CK(dmalloc(&T.stat, cap * T.sstride));
   T.group_bits = ~0ull;
   T.add_bits = 0;
-  for (uint32_t c = 0; c < d->n_cols; ++c) {
-    T.col[c] = colmem + c * cap;  // SoA: one contiguous int64 array per column
-    T.stride[c] = 1;
+  T.dyn_mask = 0;
+  for (uint32_t c = 0, jd = 0, js = 0; c < d->n_cols; ++c) {
+    const bool st = d->col_group[c] == LTPG_STATIC;
+    T.col[c] = st ? T.stat + js++ : T.dyn + jd++;
+    T.stride[c] = st ? T.sstride : T.dstride;
     T.group[c] = d->col_group[c];
     T.is_add[c] = d->col_is_add[c] ? 1 : 0;
-    const uint64_t g = d->col_group[c] == LTPG_STATIC ? 15u : d->col_group[c];
+    const uint64_t g = st ? 15u : d->col_group[c];
     T.group_bits = (T.group_bits & ~(15ull << (4 * c))) | (g << (4 * c));
     if (d->col_is_add[c]) T.add_bits |= 1u << c;
+    if (!st) T.dyn_mask |= 1u << c;
+  }
+  if (d->layout == LTPG_LAYOUT_COLUMNAR) {
+    if (T.dyn) cudaFree(T.dyn);
+    if (T.stat) cudaFree(T.stat);
+    T.dyn = T.stat = nullptr;
+    T.columnar = 1;
+    T.dstride = T.sstride = 1;
+    CK(dmalloc(&T.dyn, cap * std::max<uint32_t>(d->n_cols, 1)));
+    for (uint32_t c = 0; c < d->n_cols; ++c) {
+      T.col[c] = T.dyn + c * cap;
+      T.stride[c] = 1;
+    }
   }
   CK(dmalloc(&T.valid, cap));
   CK(cudaMemset(T.valid, 0, cap));
   CK(dmalloc(&T.rowkey, cap));
-  if (d->n_groups) {
+  if (d->n_groups) {  // every mark starts "older than any epoch"
     CK(dmalloc(&T.marks, 2 * cap * d->n_groups));
     CK(cudaMemset(T.marks, 0xFF, 2 * cap * d->n_groups * sizeof(unsigned long long)));
     if (db->cfg.flags & LTPG_FLAG_REORDER) {  // NEXT-1: minimum reader rank per unit
@@ -398,8 +426,14 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     T.idx_shift = 64 - bits;
   }
   if (n_rows) {
-    for (uint32_t c = 0; c < d->n_cols; ++c)
-      CK(cudaMemcpy(T.col[c], cols + c * n_rows, n_rows * sizeof(int64_t), cudaMemcpyHostToDevice));
+    long long* tmp = nullptr;  // column-major upload, scattered into the row blocks on the device
+    if (d->n_cols) CK(dmalloc(&tmp, n_rows));
+    for (uint32_t c = 0; c < d->n_cols; ++c) {
+      CK(cudaMemcpy(tmp, cols + c * n_rows, n_rows * sizeof(int64_t), cudaMemcpyHostToDevice));
+      launch_scatter_col(T.col[c], T.stride[c], tmp, n_rows, 0);
+    }
+    CK(cudaDeviceSynchronize());
+    if (tmp) cudaFree(tmp);
     CK(cudaMemset(T.valid, 1, n_rows));
     if (d->has_pk) CK(cudaMemcpy(T.rowkey, keys, n_rows * sizeof(uint64_t), cudaMemcpyHostToDevice));
   }

@@ -200,6 +200,17 @@ void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uin
   note_launch();
 }
 
+__global__ void k_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    dst[i * stride] = src[i];
+}
+
+void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s) {
+  if (!n) return;
+  k_scatter_col<<<148 * 16, 256, 0, s>>>(dst, stride, src, n);
+  note_launch();
+}
+
 __global__ void k_build_index(uint32_t t, uint64_t row0, uint64_t n,
                               uint32_t* err) {
   const DevTable& T = c_tabs[t];

@@ -55,7 +55,17 @@ struct DevTable {
   unsigned long long* n_rows;     // device append cursor
   // warp-uniform forms of the per-column metadata (OPS path indexes columns by a
   // per-lane col id; dynamically indexed __constant__ arrays would serialise)
-  long long* col0;                // SoA base: column c starts at col0 + c * capacity
+  // Row-block layout: each row has a "mutable" block of dstride words holding
+  // its non-static columns in column order and a "static" block of sstride words holding
+  // the static ones (blocks of <= 8 words padded to 1/2/4/8): the columns a procedure reads
+  // or writes together share one sector / line.  The marks stay in their
+  // own dense array: a mark RMW and the row's data read then miss on different lines and
+  // are filled in parallel (measured: co-locating them serialises the two fills).
+  long long* dyn;                 // [capacity][dstride]
+  long long* stat;                // [capacity][sstride]
+  uint32_t dstride, sstride;      // words per row block
+  uint32_t dyn_mask;              // bit c: column c is non-static (lives in the mutable block)
+  uint32_t columnar;              // LTPG_LAYOUT_COLUMNAR: column c at dyn + c * capacity
   uint64_t group_bits;            // 4 bits per column: group id, 15 = static
   uint32_t add_bits;              // bit c: column c is a delayed-ADD column
   // Dense key range (detected at load): key k in [key_base, key_base + dense_n) sits at row
@@ -76,8 +86,13 @@ __device__ __forceinline__ uint32_t col_group(const DevTable& T, uint32_t c) {
   return g == 15u ? LTPG_STATIC : g;
 }
 __device__ __forceinline__ bool col_is_add(const DevTable& T, uint32_t c) { return (T.add_bits >> c) & 1u; }
+// column c of row, from per-table scalars only (OPS lanes index columns by a per-lane id)
 __device__ __forceinline__ long long* col_ptr_ops(const DevTable& T, uint32_t c, uint32_t row) {
-  return T.col0 + (uint64_t)c * T.capacity + row;
+  if (T.columnar) return T.dyn + (uint64_t)c * T.capacity + row;
+  const uint32_t below = (1u << c) - 1u;
+  if ((T.dyn_mask >> c) & 1u)
+    return T.dyn + (uint64_t)row * T.dstride + __popc(T.dyn_mask & below);
+  return T.stat + (uint64_t)row * T.sstride + __popc(~T.dyn_mask & below);
 }
 
 __host__ __device__ inline uint64_t idx_hash(uint64_t key, uint32_t shift) {
@@ -339,6 +354,7 @@ void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t 
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);
+void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
 void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
                         cudaStream_t s);
 

@@ -16,12 +16,13 @@ def L():
     return lib
 
 
-def make_pair(descs, tables, max_txns, max_ops, extra_rows=64, flags=0):
+def make_pair(descs, tables, max_txns, max_ops, extra_rows=64, flags=0, layout=0):
     g = L().Database(max(descs) + 1, max_txns, max_ops, flags=flags)
     o = oracle.OracleDB(max(descs) + 1)
     for t, (grp, add, ng) in descs.items():
         k, c = tables[t]
-        g.load_table(t, grp, add, ng, k, c, capacity=c.shape[1] + extra_rows)
+        lay = layout if isinstance(layout, int) else layout[t % len(layout)]
+        g.load_table(t, grp, add, ng, k, c, capacity=c.shape[1] + extra_rows, layout=lay)
         o.define_table(t, grp, add, ng, True)
         o.load_table(t, k, c)
     return g, o
@@ -62,6 +63,18 @@ def test_random_tiny_batches_all_kinds(seed, flags):
     rng = np.random.default_rng(500 + seed)
     tables = opscases.rand_tables(rng)
     g, o = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048, flags=flags)
+    for b in range(6):
+        batch = opscases.rand_batch(rng, int(rng.integers(1, 60)), tid_start=1 + 100 * b)
+        check_batch(g, o, batch, tables)
+
+
+@pytest.mark.parametrize("layout", [1, (0, 1)])
+@pytest.mark.parametrize("seed", range(4))
+def test_random_tiny_batches_layouts(seed, layout):
+    """Column placement is result-invisible: columnar and mixed row-block/columnar tables."""
+    rng = np.random.default_rng(900 + seed)
+    tables = opscases.rand_tables(rng)
+    g, o = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048, layout=layout)
     for b in range(6):
         batch = opscases.rand_batch(rng, int(rng.integers(1, 60)), tid_start=1 + 100 * b)
         check_batch(g, o, batch, tables)
