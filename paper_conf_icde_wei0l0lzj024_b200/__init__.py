@@ -351,11 +351,11 @@ def tpcc_owner_w(t, keys, cols):
 
 
 def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None,
-                  loopback=1, rank=0, world=1, nccl_unique_id=None):
+                  loopback=1, rank=0, world=1, nccl_unique_id=None, max_ops=0):
     """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns.
     A multi-rank db (world > 1) loads only the rows of its warehouses (ITEM replicated)."""
     from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY, T_ITEM
-    db = Database(9, max_txns, 0, device=device, flags=flags, n_warehouses=workload.W, loopback=loopback,
+    db = Database(9, max_txns, max_ops, device=device, flags=flags, n_warehouses=workload.W, loopback=loopback,
                   rank=rank, world=world, nccl_unique_id=nccl_unique_id)
     from .dist import tpcc_rank_tables
     tables = tables if tables is not None else workload.initial_tables()

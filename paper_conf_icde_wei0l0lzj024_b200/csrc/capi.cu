@@ -104,6 +104,12 @@ struct ltpg_db {
   unsigned long long* d_reserve = nullptr; // [MAXT]
   uint32_t* d_dense_live = nullptr;        // bitmask: tables whose dense key->row mapping is valid
   bool olrow_ready = false;                // TPC-C ORDER -> first ORDER_LINE row map built
+  // Deferred PK index maintenance: TPC-C reaches new ORDER_LINE rows through ORDER.aux only,
+  // so their write-back skips the hash insert; rows >= d_idx_from[t] of a table in idx_lag
+  // are indexed in one pass before anything else could look them up by key (an OPS batch,
+  // the ORDER -> ORDER_LINE map rebuild).
+  uint32_t idx_lag = 0;
+  unsigned long long* d_idx_from = nullptr;  // [MAXT]
   std::vector<Part> parts;
   uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
@@ -238,6 +244,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_nrows, MAXT));
   CK(cudaMemset(db->d_nrows, 0, MAXT * sizeof(unsigned long long)));
   CK(dmalloc(&db->d_reserve, MAXT));
+  CK(dmalloc(&db->d_idx_from, MAXT));
   CK(dmalloc(&db->d_dense_live, 1));
   CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
@@ -303,7 +310,8 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
-  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_xchg, db->d_ptrs, db->d_scan};
+  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_xchg, db->d_ptrs, db->d_scan,
+                  db->d_idx_from};
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
@@ -451,6 +459,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     CK(cudaMemset(T.aux, 0xFF, cap * sizeof(uint32_t)));
   }
   if (t == LTPG_T_ORDER || t == LTPG_T_ORDER_LINE) db->olrow_ready = false;
+  db->idx_lag &= ~(1u << t);  // the index is rebuilt from every loaded row below
   unsigned long long nr = n_rows;
   CK(cudaMemcpy(T.n_rows, &nr, sizeof(nr), cudaMemcpyHostToDevice));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
@@ -619,9 +628,18 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     upload_tables_tpcc(db->d_tab, s);
     g_uploaded[db->device % 64] = db->tab_version;
   }
+  if (db->idx_lag && (ops_mode || !db->olrow_ready)) {  // key lookups ahead: catch the indexes up
+    for (uint32_t t = 0; t < db->n_tables; ++t)
+      if ((db->idx_lag >> t) & 1u) launch_build_index_tail(t, db->d_idx_from + t, S.d_small, s);
+    db->idx_lag = 0;
+  }
   if (!ops_mode && !db->olrow_ready) {  // ORDER -> contiguous ORDER_LINE rows (first TPC-C batch)
     tpcc_build_olrow(s);
     db->olrow_ready = true;
+  }
+  if (!ops_mode && !((db->idx_lag >> LTPG_T_ORDER_LINE) & 1u) && db->h_tab[LTPG_T_ORDER_LINE].idx) {
+    launch_note_rows(LTPG_T_ORDER_LINE, db->d_idx_from + LTPG_T_ORDER_LINE, s);  // first unindexed row
+    db->idx_lag |= 1u << LTPG_T_ORDER_LINE;
   }
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);

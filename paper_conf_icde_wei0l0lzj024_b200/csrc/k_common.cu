@@ -224,6 +224,31 @@ __global__ void k_build_index(uint32_t t, uint64_t row0, uint64_t n,
   }
 }
 
+// deferred index maintenance: index the valid rows [*from, n_rows) of table t
+__global__ void k_build_index_tail(uint32_t t, const unsigned long long* from, uint32_t* err) {
+  const DevTable& T = c_tabs[t];
+  const uint64_t r0 = *from, r1 = *T.n_rows;
+  for (uint64_t row = r0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; row < r1;
+       row += (uint64_t)gridDim.x * blockDim.x) {
+    if (!T.valid[row]) continue;
+    IdxSlot* sl = idx_find_or_insert(T, T.rowkey[row]);
+    if (!sl) { atomicOr(err, ERR_EINTERNAL); continue; }
+    sl->row = (uint32_t)row;
+  }
+}
+
+__global__ void k_note_rows(uint32_t t, unsigned long long* dst) { *dst = *c_tabs[t].n_rows; }
+
+void launch_build_index_tail(uint32_t t, const unsigned long long* from, uint32_t* err, cudaStream_t s) {
+  k_build_index_tail<<<148 * 8, 256, 0, s>>>(t, from, err);
+  note_launch();
+}
+
+void launch_note_rows(uint32_t t, unsigned long long* dst, cudaStream_t s) {
+  k_note_rows<<<1, 1, 0, s>>>(t, dst);
+  note_launch();
+}
+
 void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
                         cudaStream_t s) {
   if (!n) return;

@@ -85,8 +85,12 @@ __device__ __forceinline__ uint32_t rowof(const DevTable& T, uint32_t t, uint64_
 }
 __device__ __forceinline__ long long rd(const DevTable& T, uint32_t c, uint32_t row) { return *col_ptr(T, c, row); }
 __device__ __forceinline__ void wr(const DevTable& T, uint32_t c, uint32_t row, long long v) { *col_ptr(T, c, row) = v; }
+// write-back increment: an ADD-unit column may have several committed adders (atomic); a
+// WRITE-unit column has exactly one committed writer per batch (R1: WAW) -> plain RMW
 __device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row, long long v) {
-  atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr(T, c, row)), (unsigned long long)v);
+  long long* p = col_ptr(T, c, row);
+  if (col_is_add(T, c)) atomicAdd(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);
+  else *p = (long long)((unsigned long long)*p + (unsigned long long)v);
 }
 
 struct Tx {
@@ -273,11 +277,8 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         wr(TOL_, OL_QUANTITY, row, qty);
         wr(TOL_, OL_AMOUNT, row, amount);
         wr(TOL_, OL_DELIVERY_D, row, 0);
-        const uint64_t k = okey * 16 + sub + 1;
-        TOL_.rowkey[row] = k;
+        TOL_.rowkey[row] = okey * 16 + sub + 1;  // PK index entry deferred (capi.cu idx_lag)
         TOL_.valid[row] = 1;
-        IdxSlot* sl = idx_find_or_insert(TOL_, k);
-        if (sl) sl->row = row; else internal_error(x);
       }
       if (sub == 15) {  // ORDER and NEW_ORDER rows
         const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)tp.no_pref[r]);

@@ -149,3 +149,30 @@ def test_packed_params_equal_fixed_blocks():
     with pytest.raises(lib.LtpgError) as e:
         g.run_tpcc(bad, 9)
     assert e.value.rc == lib.LTPG_EINVAL
+
+
+def test_deferred_orderline_index_then_ops_lookup():
+    """New ORDER_LINE rows skip the PK-index insert at write-back (reached via ORDER.aux); an
+    OPS batch afterwards must still find them by key (the index is caught up first)."""
+    from tests.opscases import make_batch
+    from workloads.formats import T_ORDER_LINE, SELECT, SCAN, tpcc_col
+    lib = L()
+    wl = tpcc.TpccWorkload(1, seed=21, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=2048, tables=tables, append_batches=5, max_ops=4096)
+    o = oracle.tpcc_db(wl, tables)
+    for bno in range(3):
+        compare(g, o, wl.batch(2000, 1 + 2000 * bno, bno), 2 + bno)
+    keys, _ = o.dump_table(T_ORDER_LINE)
+    rng = np.random.default_rng(3)
+    pick = np.concatenate([keys[-300:], rng.choice(keys, 200)])  # newest lines + old ones
+    amt = tpcc_col(T_ORDER_LINE, "OL_AMOUNT")
+    txns = [[(int(k), SELECT, T_ORDER_LINE, amt, 0, 0)] for k in pick]
+    txns.append([(int(keys[-1]) + 1, SELECT, T_ORDER_LINE, amt, 0, 0)])  # absent
+    txns.append([(int(keys[-20]), SCAN, T_ORDER_LINE, amt, 40, 0)])
+    batch = make_batch(txns, tid_start=100000)
+    rc, ost, ord_ = o.run_ops(batch)
+    out = g.run_ops(batch)
+    assert rc == 0 and (out["status"] == ost).all() and (out["reads"] == ord_).all()
+    compare(g, o, wl.batch(2000, 200000, 7), 9)
+    compare_tables(g, o)
