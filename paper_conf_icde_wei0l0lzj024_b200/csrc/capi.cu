@@ -150,7 +150,8 @@ void free_table(DevTable& T) {
   if (T.stat) cudaFree(T.stat);
   if (T.valid) cudaFree(T.valid);
   if (T.rowkey) cudaFree(T.rowkey);
-  if (T.marks) cudaFree(T.marks);
+  if (T.wmarks) cudaFree(T.wmarks);
+  if (T.amarks) cudaFree(T.amarks);
   if (T.rmarks) cudaFree(T.rmarks);
   if (T.idx) cudaFree(T.idx);
   if (T.aux) cudaFree(T.aux);
@@ -415,12 +416,19 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   CK(dmalloc(&T.valid, cap));
   CK(cudaMemset(T.valid, 0, cap));
   CK(dmalloc(&T.rowkey, cap));
-  if (d->n_groups) {  // every mark starts "older than any epoch"
-    CK(dmalloc(&T.marks, 2 * cap * d->n_groups));
-    CK(cudaMemset(T.marks, 0xFF, 2 * cap * d->n_groups * sizeof(unsigned long long)));
+  if (d->n_groups) {  // every mark starts "unmarked" (0xFF tag byte: no live epoch)
+    T.add_groups = 0;
+    for (uint32_t c = 0; c < d->n_cols; ++c)
+      if (d->col_is_add[c] && d->col_group[c] != LTPG_STATIC) T.add_groups |= 1u << d->col_group[c];
+    CK(dmalloc(&T.wmarks, cap * d->n_groups));
+    CK(cudaMemset(T.wmarks, 0xFF, cap * d->n_groups * sizeof(mark_t)));
+    if (const uint32_t na = __builtin_popcount(T.add_groups)) {
+      CK(dmalloc(&T.amarks, cap * na));
+      CK(cudaMemset(T.amarks, 0xFF, cap * na * sizeof(mark_t)));
+    }
     if (db->cfg.flags & LTPG_FLAG_REORDER) {  // NEXT-1: minimum reader rank per unit
       CK(dmalloc(&T.rmarks, cap * d->n_groups));
-      CK(cudaMemset(T.rmarks, 0xFF, cap * d->n_groups * sizeof(unsigned long long)));
+      CK(cudaMemset(T.rmarks, 0xFF, cap * d->n_groups * sizeof(mark_t)));
     }
   }
   if (d->has_pk) {
@@ -627,6 +635,15 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     upload_tables_ops(db->d_tab, s);
     upload_tables_tpcc(db->d_tab, s);
     g_uploaded[db->device % 64] = db->tab_version;
+  }
+  if (db->epoch % 255 == 0) {  // the epoch tag byte wraps 0 -> 254: clear every mark
+    for (uint32_t t = 0; t < db->n_tables; ++t) {
+      const DevTable& T = db->h_tab[t];
+      const size_t units = T.capacity * T.n_groups * sizeof(mark_t);
+      if (T.wmarks) CK(cudaMemsetAsync(T.wmarks, 0xFF, units, s));
+      if (T.rmarks) CK(cudaMemsetAsync(T.rmarks, 0xFF, units, s));
+      if (T.amarks) CK(cudaMemsetAsync(T.amarks, 0xFF, T.capacity * __builtin_popcount(T.add_groups) * sizeof(mark_t), s));
+    }
   }
   if (db->idx_lag && (ops_mode || !db->olrow_ready)) {  // key lookups ahead: catch the indexes up
     for (uint32_t t = 0; t < db->n_tables; ++t)

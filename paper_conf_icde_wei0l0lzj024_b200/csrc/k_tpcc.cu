@@ -97,7 +97,7 @@ struct Tx {
   uint32_t dmask;  // tables with a live dense key->row mapping
   uint32_t r;
   uint32_t epoch;
-  unsigned long long tag;
+  mark_t tag;
   bool filter;
   uint32_t bits;   // detect: conflict bits found so far (CF_*)
   uint32_t* err;
@@ -115,12 +115,12 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 // rows it would add a dependent DRAM round trip before a fire-and-forget RED.
 template <int PH>
 __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row), x.tag, x.filter && hot);
+  if (PH == PH_EXEC) mark_min(wmark_ptr(T, g, row), x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_WRITE, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_min(mark_ptr(T, g, row) + 1, x.tag, x.filter && hot);
+  if (PH == PH_EXEC) mark_min(amark_ptr(T, g, row), x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_ADD, x.r, x.epoch);
 }
 template <int PH>

@@ -20,6 +20,8 @@
 namespace ltpg {
 
 constexpr int MAXC = 16;
+typedef uint32_t mark_t;
+constexpr uint32_t MARK_RANK_BITS = 24;
 constexpr int MAXT = 16;
 constexpr uint64_t KEY_EMPTY = ~0ull;
 constexpr uint32_t ROW_NONE = 0xFFFFFFFFu;
@@ -47,8 +49,12 @@ struct DevTable {
   uint64_t capacity;
   uint8_t* valid;
   unsigned long long* rowkey;
-  unsigned long long* marks;      // [n_groups][capacity] x {minW, minA}
-  unsigned long long* rmarks;     // [n_groups][capacity] minR (LTPG_FLAG_REORDER only, else null)
+  // conflict marks, 32-bit epoch-tagged (mark_t): minW of every group, minA of the ADD
+  // groups only (a plain group never receives an add), minR under NEXT-1 only
+  mark_t* wmarks;                 // [n_groups][capacity]
+  mark_t* amarks;                 // [popcount(add_groups)][capacity] or null
+  mark_t* rmarks;                 // [n_groups][capacity] (LTPG_FLAG_REORDER only, else null)
+  uint32_t add_groups;            // bit g: group g holds ADD columns
   IdxSlot* idx;
   uint64_t idx_mask;
   uint32_t idx_shift;
@@ -99,32 +105,40 @@ __host__ __device__ inline uint64_t idx_hash(uint64_t key, uint32_t shift) {
   return (key * 0x9E3779B97F4A7C15ull) >> shift;
 }
 
-__device__ __forceinline__ unsigned long long epoch_tag(uint32_t epoch) {
-  return (unsigned long long)(0xFFFFFFFFu - epoch) << 32;
-}
+// Mark word = epoch tag (high 8 bits) | rank (low 24 bits; max_txns <= 2^24).  Batch e uses
+// the tag byte 254 - (e mod 255): a later epoch has a smaller tag, so atomicMin overwrites
+// older marks without a reset pass and mark_rank ignores them; the byte 0xFF (the
+// "unmarked" value) never names a live epoch.  The byte wraps from 0 back to 254 every 255
+// batches, so all marks are reset to 0xFF..FF before each such batch (capi.cu) -- 4 bytes per unit keep the
+// mark arrays of the randomly touched tables L2-resident (126 MB) within a batch.
+__host__ __device__ __forceinline__ uint32_t epoch_byte(uint32_t epoch) { return 254u - epoch % 255u; }
+__device__ __forceinline__ mark_t epoch_tag(uint32_t epoch) { return epoch_byte(epoch) << MARK_RANK_BITS; }
 
 // Minimum rank recorded for this epoch, or UINT32_MAX.
-__device__ __forceinline__ uint32_t mark_rank(unsigned long long v, uint32_t epoch) {
-  return (uint32_t)(v >> 32) == 0xFFFFFFFFu - epoch ? (uint32_t)v : 0xFFFFFFFFu;
+__device__ __forceinline__ uint32_t mark_rank(mark_t v, uint32_t epoch) {
+  return (v >> MARK_RANK_BITS) == epoch_byte(epoch) ? (v & ((1u << MARK_RANK_BITS) - 1)) : 0xFFFFFFFFu;
 }
 
 // recordTID: atomicMin of this txn's rank into a mark word.  The
 // plain pre-read skips the atomic when a smaller (or equal) rank is already
 // there -- marks only decrease, so a stale read can only cause a redundant
 // atomic, never a missing one (result-identical).
-__device__ __forceinline__ void mark_min(unsigned long long* p, unsigned long long v, bool filter) {
+__device__ __forceinline__ void mark_min(mark_t* p, mark_t v, bool filter) {
   if (filter) {
-    const unsigned long long cur = __ldcg(p);  // L2-coherent read, no system-scope fence
+    const mark_t cur = __ldcg(p);  // L2-coherent read, no system-scope fence
     if (cur <= v) return;
   }
   atomicMin(p, v);
 }
 
-__device__ __forceinline__ unsigned long long* mark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
-  return T.marks + 2ull * ((uint64_t)g * T.capacity + row);
+__device__ __forceinline__ mark_t* wmark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
+  return T.wmarks + ((uint64_t)g * T.capacity + row);
 }
-
-__device__ __forceinline__ unsigned long long* rmark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
+// only for ADD groups (validated at load: ADD ops and ADD columns live in ADD groups)
+__device__ __forceinline__ mark_t* amark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
+  return T.amarks + ((uint64_t)__popc(T.add_groups & ((1u << g) - 1u)) * T.capacity + row);
+}
+__device__ __forceinline__ mark_t* rmark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
   return T.rmarks + ((uint64_t)g * T.capacity + row);
 }
 
@@ -213,8 +227,8 @@ __device__ __forceinline__ uint8_t status_of_bits(uint32_t bits, bool reorder) {
 //   ADD   -> WAW if a smaller rank plainly wrote;  WAR if a smaller rank read (reorder only)
 __device__ __forceinline__ uint32_t unit_bits(const DevTable& T, uint32_t g, uint32_t row, uint32_t acc, uint32_t r,
                                               uint32_t epoch) {
-  const ulonglong2 m = *reinterpret_cast<const ulonglong2*>(mark_ptr(T, g, row));
-  const uint32_t w = mark_rank(m.x, epoch), a = mark_rank(m.y, epoch);
+  const uint32_t w = mark_rank(*wmark_ptr(T, g, row), epoch);
+  const uint32_t a = ((T.add_groups >> g) & 1u) ? mark_rank(*amark_ptr(T, g, row), epoch) : 0xFFFFFFFFu;
   const uint32_t wa = w < a ? w : a;
   uint32_t bits = 0;
   if (acc == ACC_READ) return wa < r ? CF_RAW : 0u;

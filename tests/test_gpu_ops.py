@@ -80,6 +80,25 @@ def test_random_tiny_batches_layouts(seed, layout):
         check_batch(g, o, batch, tables)
 
 
+def test_epoch_tag_wrap_600_batches():
+    """Mark words carry an 8-bit epoch tag that repeats every 255 batches (all marks are
+    reset at the wrap): 600 consecutive small batches on hot keys stay oracle-identical."""
+    wl = YcsbWorkload(64, theta=0.9, ops_per_txn=4, seed=77)
+    keys, cols = wl.initial_table()
+    descs = {0: tuple(wl.table_desc()[:3])}
+    g, o = make_pair(descs, {0: (keys, cols)}, 64, 256)
+    tid = 1
+    for bno in range(600):
+        batch = wl.batch(int(1 + bno % 48), tid, bno)
+        tid += len(batch["tid"])
+        rc, ost, ord_ = o.run_ops(batch)
+        out = g.run_ops(batch)
+        assert rc == 0 and (out["status"] == ost).all() and (out["reads"] == ord_).all(), bno
+    gk, gc = g.dump_table(0)
+    ok, oc = o.dump_table(0)
+    assert (gc == oc).all()
+
+
 def test_ycsb_c1_closed_loop():
     """BASELINE configs[0]: YCSB-A 10k rows, 1024 txns x 4 ops, zipf 0.5, retries."""
     wl = YcsbWorkload(10_000, theta=0.5, ops_per_txn=4, seed=0x17C0)
