@@ -654,7 +654,10 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
 // others -- each type group gets its own launch configuration.
 constexpr uint32_t TM_MAIN = 0x0Fu, TM_SL = 0x10u;
 template <int PH, uint32_t TMASK>
-__global__ void __launch_bounds__(256) k_tpcc_phase(BatchDev b, TpccParams tp) {
+// minimum resident blocks per phase (register cap): detection is a chain of dependent
+// loads (params -> log -> marks) and gains most from occupancy (measured: 8 -> 32 regs)
+__global__ void __launch_bounds__(256, (PH == PH_EXEC ? 4 : PH == PH_DETECT ? 8 : 6))
+    k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
