@@ -59,13 +59,22 @@ def log(*a):
 
 # ---- clocks sampler (B200_PROFILING.md "clocks DURING the timed region") ------------------
 class ClockSampler:
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock + throttle reasons sampled every ~2 ms through NVML (nvidia-smi is the
+    fallback) on a background thread; the summary covers the samples taken inside the
+    windows bench.py marks as timed (device-resident leg and e2e leg)."""
+    SMI_Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    # NVML clocks-event reason bits (nvml.h)
+    REASONS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20,
+               "hw_thermal_slowdown": 0x40}
 
     def __init__(self, index):
         self.index = index
-        self.lines = []
+        self.samples = []   # (t, sm_mhz, reason_bits)
+        self.windows = []
+        self.max_mhz = None
+        self.source = None
         self.stop = threading.Event()
 
     def __enter__(self):
@@ -73,13 +82,49 @@ class ClockSampler:
         self.t.start()
         return self
 
+    def mark(self, t0, t1):
+        self.windows.append((t0, t1))
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        try:
+            import torch
+            uuid = str(torch.cuda.get_device_properties(self.index).uuid)
+            return pynvml, pynvml.nvmlDeviceGetHandleByUUID(("GPU-" + uuid) if not uuid.startswith("GPU-") else uuid)
+        except Exception:
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.index)
+
     def _loop(self):
+        try:
+            nv, h = self._nvml_handle()
+            self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+            self.source = "nvml"
+            while not self.stop.is_set():
+                sm = float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM))
+                try:
+                    rb = int(nv.nvmlDeviceGetCurrentClocksEventReasons(h))
+                except Exception:
+                    rb = int(nv.nvmlDeviceGetCurrentClocksThrottleReasons(h))
+                self.samples.append((time.time(), sm, rb))
+                self.stop.wait(0.002)
+            return
+        except Exception:
+            pass
+        self.source = "nvidia-smi"
         while not self.stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.SMI_Q,
                                       "--format=csv,noheader,nounits"], capture_output=True, text=True,
                                      timeout=5).stdout
-                self.lines += [ln.strip() for ln in out.splitlines() if ln.strip()]
+                for ln in out.splitlines():
+                    f = [x.strip() for x in ln.split(",")]
+                    if len(f) < 9:
+                        continue
+                    names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+                    rb = sum(self.REASONS[n] for n, v in zip(names, f[5:9]) if v.lower() == "active")
+                    self.max_mhz = float(f[2])
+                    self.samples.append((time.time(), float(f[1]), rb))
             except Exception:
                 pass
             self.stop.wait(0.05)
@@ -89,23 +134,13 @@ class ClockSampler:
         self.t.join(timeout=6)
 
     def summary(self):
-        sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            f = [x.strip() for x in ln.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                sm.append(float(f[1]))
-                mx = float(f[2])
-            except ValueError:
-                continue
-            for n, v in zip(names, f[5:9]):
-                if v.lower() == "active":
-                    reasons.add(n)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sm),
-                "window": "sampled every ~0.1 s from the first warm-up step to the end of the e2e leg"}
+        inside = [x for x in self.samples if any(t0 <= x[0] <= t1 for t0, t1 in self.windows)]
+        use = inside or self.samples
+        reasons = sorted(n for n, bit in self.REASONS.items() if any(x[2] & bit for x in use))
+        return {"sm_mhz": statistics.median(x[1] for x in use) if use else None, "sm_max_mhz": self.max_mhz,
+                "reasons": reasons, "samples": len(use), "source": self.source,
+                "window": ("samples inside the timed legs" if inside else
+                           "all samples (warm-up .. e2e): timed legs shorter than one sample")}
 
 
 def measured_peaks():
@@ -417,6 +452,7 @@ def main():
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     commits, procs, exec_ms, kernels, stage = [], [], [], 0, []
     torch.cuda.synchronize()
+    tw0 = time.time()
     for s in range(args.steps):
         i = (args.warmup + s) % n_distinct
         flush.fill_(s & 0xFF)  # evict L2 between steps (outside the timed events)
@@ -431,6 +467,7 @@ def main():
         kernels += st["n_kernels"]
         stage.append(st)
     torch.cuda.synchronize()
+    clk.mark(tw0, time.time())
     step_ms = [a.elapsed_time(b) for a, b in ev]
     if os.environ.get("LTPG_BENCH_DEBUG"):
         log("step ms:", ["%.3f" % x for x in step_ms])
@@ -458,13 +495,14 @@ def main():
         if dist:
             dist.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tw0 = time.time()
         e0.record(stream)
         inflight = []
 
         def collect(p):
             nonlocal d2h
             out = p.wait()
-            e_commits.append(int((out["status"] == 1).sum()))
+            e_commits.append(out["stats"]["n_commit"])  # the library's counter: no host pass
             n = len(out["status"])
             nreads = n_reads if w["kind"] == "ycsb" else 4 * B
             d2h += n + 4 * ((n + 31) // 32) + 4 * n + 8 * nreads + 68
@@ -472,7 +510,7 @@ def main():
         for s in range(args.steps):
             i = (args.warmup + s) % n_distinct
             bh = host_batches[i]
-            inflight.append(run(None, bh, clock, False, False, wait=False, slot=s % 3))
+            inflight.append(run(None, bh, clock, False, True, wait=False, slot=s % 3))
             clock += 1
             h2d += sum(v.nbytes for v in bp_of(bh).values())
             if len(inflight) == 3:  # keep two batches queued behind the one completing
@@ -481,6 +519,7 @@ def main():
             collect(inflight.pop(0))
         e1.record(stream)
         torch.cuda.synchronize()
+        clk.mark(tw0, time.time())
         e_s = e0.elapsed_time(e1) / 1000.0
         e_c = float(sum(e_commits))
         if dist:
