@@ -371,13 +371,14 @@ def main():
                                 capacity=w["n_rows"] + nb * B * w["ops"] // 10 + 1024)
     else:
         # append regions: the worst case of one batch (checked before execution) plus the
-        # expected appends of every batch this run makes (NewOrder commits <= 30%, Payment <= 100%)
+        # appends of every batch this run makes (every NewOrder / Payment committing; 10.5 lines
+        # per NewOrder on average)
         from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
         tabs = wl.initial_tables()
         nb = args.warmup + 2 * args.steps + 2
         no, pay = B * wl.mix[0], B * wl.mix[1]
-        cap = {T_ORDER: no * (1 + 0.3 * nb), T_NEW_ORDER: no * (1 + 0.3 * nb),
-               T_ORDER_LINE: 15 * no * (1 + 0.3 * nb), T_HISTORY: pay * (1 + nb)}
+        cap = {T_ORDER: no * (1 + nb), T_NEW_ORDER: no * (1 + nb),
+               T_ORDER_LINE: 15 * no + 10.5 * no * nb, T_HISTORY: pay * (1 + nb)}
         cap = {t: int(tabs[t][1].shape[1] + v) + 1024 for t, v in cap.items()}
         db = ltpg.tpcc_database(wl, max_txns=B, tables=tabs, capacity=cap, flags=args.flags, device=local,
                                 rank=rank, world=world, nccl_unique_id=uid)
