@@ -535,115 +535,221 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
   }
 }
 
-// ---- StockLevel (TPC-C 2.8): window [nx-20, nx), distinct items, one warp per txn -----------
-// Distinct items are found with a per-warp open-addressing set in shared memory (the
-// first inserter of an item handles it); the result is order-independent.
+// ---- StockLevel (TPC-C 2.8): shared per district ---------------------------------------------
+// Every StockLevel of a district reads the same snapshot: D_NEXT_O_ID, the last 20 orders, their
+// distinct items and those items' S_QUANTITY.  So the window is evaluated once per district with
+// StockLevels in the batch (one warp each) into a prefix table low[t] = #distinct items with
+// S_QUANTITY < t (t = 0..256); a txn's result is low[threshold].  Its read set is the district's
+// unit set, so its RAW test (R1: any smaller rank wrote/added a unit) reduces to one comparison
+// with M = the smallest mark rank over that set.  Result- and verdict-identical to one warp per
+// txn; the work drops from per-txn to per-district (~66x at 64 warehouses, 2^20 txns).
 constexpr int SL_SLOTS = 20 * 15;
 constexpr int SL_HASH = 512;
-template <int PH>
-__device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bool active, Tx& x,
-                                uint32_t* items, uint32_t* set) {
+constexpr int SL_T = 257;
+
+__device__ __forceinline__ uint32_t sl_dk_of(const BatchDev& b, uint32_t r) {
+  const uint8_t* p = b.params + 128ull * r;
+  return (uint32_t)kD(p16(p, 0), p[2]);
+}
+
+// every StockLevel: minimum rank per district; the first one lists the district
+__global__ void __launch_bounds__(256) k_sl_claim(BatchDev b, TpccParams tp, SlScratch sl) {
+  if (*b.err) return;
+  const uint32_t n = tp.counts[4];
+  const uint32_t* list = tp.list + 4ull * tp.max_txns;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t r = list[i];
+    const uint32_t dk = sl_dk_of(b, r);
+    if (atomicMin(sl.minr + dk, r) == 0xFFFFFFFFu) {
+      const uint32_t idx = atomicAdd(sl.cnt, 1u);
+      sl.dk[idx] = dk;
+      sl.slot[dk] = idx;
+    }
+  }
+}
+
+// one warp per listed district: window, distinct items, S_QUANTITY prefix table; NEXT-1 minR
+__global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
+  if (*b.err) return;
+  __shared__ uint32_t items_s[8][SL_SLOTS];
+  __shared__ uint32_t set_s[8][SL_HASH];
+  __shared__ uint32_t hist_s[8][SL_T + 1];
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TOr = c_tabs[TO];
   const DevTable& TOL_ = c_tabs[TOL];
   const DevTable& TSt = c_tabs[TS];
-  if (!active || PH == PH_WB) return;  // warp-uniform (one txn per warp); read-only: no write-back
-  const uint8_t* p = b.params + 128ull * r;
-  const uint32_t w = p16(p, 0), d = p[2];
-  const long long thr = p[3];
-  const uint32_t row_d = rowof(TDi, TD, kD(w, d), x.dmask);
-  if (row_d == ROW_NONE) {
-    internal_error(x);
-    return;
-  }
-  const long long nx = rd(TDi, D_NEXT_O_ID, row_d);
-  if (lane == 0) unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
-  if (PH == PH_DETECT && __shfl_sync(0xffffffffu, (uint32_t)x.done(), 0)) return;  // RAW on D_NEXT_O_ID: done
-  for (uint32_t s = lane; s < SL_SLOTS; s += 32) items[s] = 0;
-  for (uint32_t s = lane; s < SL_HASH; s += 32) set[s] = 0;
-  __syncwarp();
-  if (lane < 20) {
-    const long long o = nx - 20 + lane;
-    const uint32_t row_o = probe(TOr, kO(w, d, (uint64_t)o));
-    if (row_o == ROW_NONE) {
-      internal_error(x);
-    } else {
-      const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);  // static
-      const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
-      uint32_t row_ol[15];
-#pragma unroll
-      for (uint32_t l = 0; l < 15; ++l)  // otherwise independent probes issued back to back
-        row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1))
-                            : ROW_NONE;
-#pragma unroll
-      for (uint32_t l = 0; l < 15; ++l)
-        if (l < cnt) {
-          if (row_ol[l] == ROW_NONE) internal_error(x);
-          else items[lane * 15 + l] = (uint32_t)rd(TOL_, OL_I_ID, row_ol[l]);  // static
-        }
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  uint32_t* items = items_s[wib];
+  uint32_t* set = set_s[wib];
+  uint32_t* hist = hist_s[wib];
+  const uint32_t dmask = *b.dense_live;
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
+  const uint32_t nd_total = *sl.cnt;
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t idx = blockIdx.x * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
+    const uint32_t dk = sl.dk[idx];
+    uint32_t w = dk / 10, d = dk % 10;
+    if (d == 0) { d = 10; w -= 1; }  // kD(w, 10) == kD(w + 1, 0)
+    const uint32_t row_d = rowof(TDi, TD, dk, dmask);
+    if (row_d == ROW_NONE) {
+      if (lane == 0) atomicOr(b.err, ERR_EINTERNAL);
+      continue;
     }
-  }
-  __syncwarp();
-  // distinct items: the first inserter of an item into the shared-memory set appends it to a
-  // compact list (the slot array is reused: items were consumed into registers first)
-  uint32_t mine[(SL_SLOTS + 31) / 32];
+    const long long nx = rd(TDi, D_NEXT_O_ID, row_d);
+    for (uint32_t s2 = lane; s2 < SL_SLOTS; s2 += 32) items[s2] = 0;
+    for (uint32_t s2 = lane; s2 < SL_HASH; s2 += 32) set[s2] = 0;
+    for (uint32_t s2 = lane; s2 <= SL_T; s2 += 32) hist[s2] = 0;
+    __syncwarp();
+    if (lane < 20) {
+      const long long o = nx - 20 + lane;
+      const uint32_t row_o = probe(TOr, kO(w, d, (uint64_t)o));
+      if (row_o == ROW_NONE) {
+        atomicOr(b.err, ERR_EINTERNAL);
+      } else {
+        const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);  // static
+        const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
+        uint32_t row_ol[15];
 #pragma unroll
-  for (uint32_t u = 0; u < (SL_SLOTS + 31) / 32; ++u) {
-    const uint32_t sl = lane + 32 * u;
-    mine[u] = sl < SL_SLOTS ? items[sl] : 0u;
-  }
-  __syncwarp();
-  uint32_t nd = 0;
+        for (uint32_t l = 0; l < 15; ++l)  // otherwise independent probes issued back to back
+          row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, kO(w, d, (uint64_t)o) * 16 + l + 1))
+                              : ROW_NONE;
 #pragma unroll
-  for (uint32_t u = 0; u < (SL_SLOTS + 31) / 32; ++u) {
-    const uint32_t it = mine[u];
-    bool first = false;
-    if (it) {
-      uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
-      for (;;) {
-        const uint32_t old = atomicCAS(set + h, 0u, it);
-        if (old == 0u) { first = true; break; }
-        if (old == it) break;
-        h = (h + 1) & (SL_HASH - 1);
+        for (uint32_t l = 0; l < 15; ++l)
+          if (l < cnt) {
+            if (row_ol[l] == ROW_NONE) atomicOr(b.err, ERR_EINTERNAL);
+            else items[lane * 15 + l] = (uint32_t)rd(TOL_, OL_I_ID, row_ol[l]);  // static
+          }
       }
     }
-    const uint32_t m = __ballot_sync(0xffffffffu, first);
-    if (first) items[nd + __popc(m & ((1u << lane) - 1))] = it;
-    nd += __popc(m);
-  }
-  __syncwarp();
-  // stock reads of the distinct items: all of a lane's loads in flight together (dense key
-  // -> row mapping: no index access)
-  long long low = 0;
-  constexpr uint32_t MAXU = (SL_SLOTS + 31) / 32;
-  uint32_t rows[MAXU];
+    __syncwarp();
+    // distinct items: the first inserter of an item into the shared-memory set appends it to a
+    // compact list (the slot array is reused: items were consumed into registers first)
+    constexpr uint32_t MAXU = (SL_SLOTS + 31) / 32;
+    uint32_t mine[MAXU];
 #pragma unroll
-  for (uint32_t u = 0; u < MAXU; ++u) {
-    const uint32_t j = lane + 32 * u;
-    rows[u] = j < nd ? rowof(TSt, TS, kS(w, items[j]), x.dmask) : ROW_NONE;
-  }
-  long long q[MAXU];
-#pragma unroll
-  for (uint32_t u = 0; u < MAXU; ++u)
-    q[u] = (PH == PH_EXEC && rows[u] != ROW_NONE) ? rd(TSt, S_QUANTITY, rows[u]) : 0;
-#pragma unroll
-  for (uint32_t u = 0; u < MAXU; ++u) {
-    const uint32_t j = lane + 32 * u;
-    if (j >= nd) continue;
-    if (rows[u] == ROW_NONE) { internal_error(x); continue; }
-    if (PH == PH_EXEC) low += q[u] < thr;
-    unit_r<PH>(TSt, col_group(TSt, S_QUANTITY), rows[u], x);
-  }
-  if (PH == PH_EXEC) {
-#pragma unroll
-    for (int o = 16; o; o >>= 1) low += __shfl_xor_sync(0xffffffffu, low, o);
-    if (lane == 0) {
-      long long* res = b.res + 4ull * r;
-      res[0] = low;
-      res[1] = nx;
-      res[2] = 0;
-      res[3] = 0;
+    for (uint32_t u = 0; u < MAXU; ++u) {
+      const uint32_t j = lane + 32 * u;
+      mine[u] = j < SL_SLOTS ? items[j] : 0u;
     }
+    __syncwarp();
+    uint32_t nd = 0;
+#pragma unroll
+    for (uint32_t u = 0; u < MAXU; ++u) {
+      const uint32_t it = mine[u];
+      bool first = false;
+      if (it) {
+        uint32_t h = (it * 2654435761u) >> 23;  // 9 bits
+        for (;;) {
+          const uint32_t old = atomicCAS(set + h, 0u, it);
+          if (old == 0u) { first = true; break; }
+          if (old == it) break;
+          h = (h + 1) & (SL_HASH - 1);
+        }
+      }
+      const uint32_t m = __ballot_sync(0xffffffffu, first);
+      if (first) items[nd + __popc(m & ((1u << lane) - 1))] = it;
+      nd += __popc(m);
+    }
+    __syncwarp();
+    // stock rows and quantities of the distinct items (dense key -> row: no index access)
+    uint32_t rows[MAXU];
+#pragma unroll
+    for (uint32_t u = 0; u < MAXU; ++u) {
+      const uint32_t j = lane + 32 * u;
+      rows[u] = j < nd ? rowof(TSt, TS, kS(w, items[j]), dmask) : ROW_NONE;
+    }
+    long long q[MAXU];
+#pragma unroll
+    for (uint32_t u = 0; u < MAXU; ++u) q[u] = rows[u] != ROW_NONE ? rd(TSt, S_QUANTITY, rows[u]) : 0;
+    const mark_t rtag = epoch_tag(b.epoch) | sl.minr[dk];
+    const uint32_t gq = col_group(TSt, S_QUANTITY);
+#pragma unroll
+    for (uint32_t u = 0; u < MAXU; ++u) {
+      const uint32_t j = lane + 32 * u;
+      if (j >= nd) continue;
+      if (rows[u] == ROW_NONE) { atomicOr(b.err, ERR_EINTERNAL); continue; }
+      sl.rows[(uint64_t)idx * SL_SLOTS + j] = rows[u];
+      // bucket q + 1 (clamped): q < t  <=>  bucket <= t
+      const long long bq = q[u] + 1 < 0 ? 0 : (q[u] + 1 > SL_T ? SL_T : q[u] + 1);
+      atomicAdd(hist + bq, 1u);
+      if (reorder && TSt.rmarks) mark_min(rmark_ptr(TSt, gq, rows[u]), rtag, true);  // NEXT-1 minR
+    }
+    if (lane == 0 && reorder && TDi.rmarks)
+      mark_min(rmark_ptr(TDi, col_group(TDi, D_NEXT_O_ID), row_d), rtag, true);
+    __syncwarp();
+    // low[t] = sum of hist[0..t]: 9 buckets per lane, then a warp scan of the lane sums
+    constexpr uint32_t PER = (SL_T + 31) / 32;
+    uint32_t v[PER], run = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < PER; ++k) {
+      const uint32_t t = lane * PER + k;
+      run += t < SL_T ? hist[t] : 0u;
+      v[k] = run;
+    }
+    uint32_t incl = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= (uint32_t)o) incl += y;
+    }
+    const uint32_t base = incl - run;
+#pragma unroll
+    for (uint32_t k = 0; k < PER; ++k) {
+      const uint32_t t = lane * PER + k;
+      if (t < SL_T) sl.low[(uint64_t)idx * SL_T + t] = base + v[k];
+    }
+    if (lane == 0) {
+      sl.nx[idx] = nx;
+      sl.nd[idx] = nd;
+      sl.rowd[idx] = row_d;
+    }
+    __syncwarp();
+  }
+}
+
+// detection, one warp per listed district: M = smallest write / add rank over its unit set
+__global__ void __launch_bounds__(256) k_sl_detect(BatchDev b, SlScratch sl) {
+  if (*b.err) return;
+  const DevTable& TDi = c_tabs[TD];
+  const DevTable& TSt = c_tabs[TS];
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t nd_total = *sl.cnt;
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  const uint32_t gq = col_group(TSt, S_QUANTITY), gd = col_group(TDi, D_NEXT_O_ID);
+  for (uint32_t idx = blockIdx.x * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
+    const uint32_t nd = sl.nd[idx];
+    uint32_t m = 0xFFFFFFFFu;
+    auto wa = [&](const DevTable& T, uint32_t g, uint32_t row) {
+      const uint32_t w = mark_rank(*wmark_ptr(T, g, row), b.epoch);
+      const uint32_t a = ((T.add_groups >> g) & 1u) ? mark_rank(*amark_ptr(T, g, row), b.epoch) : 0xFFFFFFFFu;
+      return w < a ? w : a;
+    };
+    if (lane == 0) m = wa(TDi, gd, sl.rowd[idx]);
+    for (uint32_t j = lane; j < nd; j += 32) m = min(m, wa(TSt, gq, sl.rows[(uint64_t)idx * SL_SLOTS + j]));
+    m = __reduce_min_sync(0xffffffffu, m);
+    if (lane == 0) sl.m[idx] = m;
+  }
+}
+
+// per StockLevel txn: result from the district's table, RAW verdict from its M
+__global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScratch sl) {
+  if (*b.err) return;
+  const uint32_t n = tp.counts[4];
+  const uint32_t* list = tp.list + 4ull * tp.max_txns;
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t r = list[i];
+    const uint8_t* p = b.params + 128ull * r;
+    const uint32_t idx = sl.slot[kD(p16(p, 0), p[2])];
+    long long* res = b.res + 4ull * r;
+    res[0] = sl.low[(uint64_t)idx * SL_T + p[3]];
+    res[1] = sl.nx[idx];
+    res[2] = 0;
+    res[3] = 0;
+    // NEXT-1: read-only procedures never abort under reordering
+    const uint32_t flag = (!reorder && sl.m[idx] < r ? CF_RAW : 0u) | (b.ua[r] ? CF_UA : 0u);
+    if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;
+    else b.status[r] = status_of_bits(flag, reorder);
   }
 }
 
@@ -652,7 +758,7 @@ __device__ void proc_stocklevel(const BatchDev& b, uint32_t r, uint32_t lane, bo
 // TMASK: procedure types this launch runs.  StockLevel (32 lanes, 26 KB of shared memory per
 // block, many registers) runs in its own launch so it does not cap the occupancy of the
 // others -- each type group gets its own launch configuration.
-constexpr uint32_t TM_MAIN = 0x0Fu, TM_SL = 0x10u;
+constexpr uint32_t TM_MAIN = 0x0Fu;  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
 template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
 // loads (params -> log -> marks) and gains most from occupancy (measured: 8 -> 32 regs)
@@ -692,12 +798,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? 4 : PH == PH_DETECT ? 8 
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
       case 3: proc_delivery<PH>(b, r, sub, go, x); break;
       default:
-        if constexpr ((TMASK & TM_SL) != 0) {
-          __shared__ uint32_t sl_items[8][SL_SLOTS];
-          __shared__ uint32_t sl_set[8][SL_HASH];
-          proc_stocklevel<PH>(b, r, lane, go, x, sl_items[wib], sl_set[wib]);
-        }
-        break;
+        break;  // StockLevel: shared per district (k_sl_*)
     }
     if (PH == PH_DETECT) {  // per-txn OR of the conflict bits over the txn's lanes
       const uint32_t seg = L == 32 ? 0xffffffffu : (L == 1 ? (1u << lane) : (0xffffu << (lane & 16)));
@@ -1009,6 +1110,11 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
       dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_pref, max_txns + 1ull) ||
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
     return LTPG_ENOMEM;
+  SlScratch& sl = t.sl;
+  if (dm(&sl.minr, t.dsz) || dm(&sl.slot, t.dsz) || dm(&sl.dk, t.dsz) || dm(&sl.cnt, 1) ||
+      dm(&sl.low, (uint64_t)t.dsz * SL_T) || dm(&sl.nx, t.dsz) || dm(&sl.rows, (uint64_t)t.dsz * SL_SLOTS) ||
+      dm(&sl.nd, t.dsz) || dm(&sl.rowd, t.dsz) || dm(&sl.m, t.dsz))
+    return LTPG_ENOMEM;
   if (t.owns_by_name) cudaMemset(t.by_name, 0, (uint64_t)t.dsz * 1000 * sizeof(int));
   if (cudaStreamCreateWithFlags(&t.side, cudaStreamNonBlocking) != cudaSuccess) return LTPG_ECUDA;
   for (int k = 0; k < 2; ++k)
@@ -1025,7 +1131,8 @@ void tpcc_free(TpccDev& t) {
     if (t.join[k]) cudaEventDestroy(t.join[k]);
   }
   if (!t.owns_by_name) t.by_name = nullptr;
-  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc};
+  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc,
+                t.sl.minr, t.sl.slot, t.sl.dk, t.sl.cnt, t.sl.low, t.sl.nx, t.sl.rows, t.sl.nd, t.sl.rowd, t.sl.m};
   for (void* p : ps)
     if (p) cudaFree(p);
   t = TpccDev{};
@@ -1075,22 +1182,27 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   note_launch(2);
   if (ev) cudaEventRecord(ev[2], s);
   const uint32_t grid = phase_grid(n);
-  // StockLevel warps on a side stream, concurrently with the other procedures (fork / join)
+  // StockLevel (shared per district) on a side stream, concurrently with the other procedures
+  const SlScratch sl = t.sl;
   cudaEventRecord(t.fork[0], s);
   cudaStreamWaitEvent(t.side, t.fork[0], 0);
-  k_tpcc_phase<PH_EXEC, TM_SL><<<grid, 256, 0, t.side>>>(b, tp);
+  cudaMemsetAsync(sl.minr, 0xFF, (size_t)t.dsz * sizeof(uint32_t), t.side);
+  cudaMemsetAsync(sl.cnt, 0, sizeof(uint32_t), t.side);
+  k_sl_claim<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
+  k_sl_district<<<148 * 2, 256, 0, t.side>>>(b, sl);
   cudaEventRecord(t.join[0], t.side);
   k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
-  note_launch(2);
+  note_launch(3);
   if (ev) cudaEventRecord(ev[3], s);
   cudaEventRecord(t.fork[1], s);
   cudaStreamWaitEvent(t.side, t.fork[1], 0);
-  k_tpcc_phase<PH_DETECT, TM_SL><<<grid, 256, 0, t.side>>>(b, tp);
+  k_sl_detect<<<148 * 2, 256, 0, t.side>>>(b, sl);
+  k_sl_txn<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   cudaEventRecord(t.join[1], t.side);
   k_tpcc_phase<PH_DETECT, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[1], 0);
-  note_launch(2);
+  note_launch(3);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
 

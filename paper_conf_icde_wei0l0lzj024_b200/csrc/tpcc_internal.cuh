@@ -24,6 +24,21 @@ enum { S_QUANTITY = 0, S_YTD = 1, S_ORDER_CNT = 2, S_REMOTE_CNT = 3 };
 // counters in TpccDev::misc (M_NO / M_NO_LINES / M_PAY: inserts this partition may append)
 enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3, M_CCOUNT = 8 };
 
+// StockLevel shared per district (k_sl_*): per-batch scratch indexed by district key (dk) or by
+// the compact index of a district with StockLevels in the batch (idx)
+struct SlScratch {
+  uint32_t* minr = nullptr;     // [dsz] by dk: smallest StockLevel rank (0xFFFFFFFF: none)
+  uint32_t* slot = nullptr;     // [dsz] by dk: idx
+  uint32_t* dk = nullptr;       // [dsz] by idx
+  uint32_t* cnt = nullptr;      // [1] listed districts
+  uint32_t* low = nullptr;      // [dsz][257] by idx: #distinct items with S_QUANTITY < t
+  long long* nx = nullptr;      // [dsz] by idx: D_NEXT_O_ID
+  uint32_t* rows = nullptr;     // [dsz][300] by idx: stock rows of the distinct items
+  uint32_t* nd = nullptr;       // [dsz] by idx: distinct items
+  uint32_t* rowd = nullptr;     // [dsz] by idx: district row
+  uint32_t* m = nullptr;        // [dsz] by idx: smallest write/add mark rank over the unit set
+};
+
 struct TpccDev {
   uint32_t max_txns = 0;
   uint32_t nw = 0;              // n_warehouses (global)
@@ -38,6 +53,7 @@ struct TpccDev {
   uint32_t* chunk_cnt = nullptr;// [chunks][dsz]
   long long* dist_base = nullptr; // [dsz] snapshot D_NEXT_O_ID
   uint32_t* misc = nullptr;     // counters (M_*)
+  SlScratch sl;
   cudaStream_t side = nullptr;  // StockLevel phases run here, concurrently with the others
   cudaEvent_t fork[2]{}, join[2]{};
 };

@@ -176,3 +176,22 @@ def test_deferred_orderline_index_then_ops_lookup():
     assert rc == 0 and (out["status"] == ost).all() and (out["reads"] == ord_).all()
     compare(g, o, wl.batch(2000, 200000, 7), 9)
     compare_tables(g, o)
+
+
+def test_stocklevel_shared_per_district_any_threshold():
+    """StockLevel is evaluated once per district (prefix table over S_QUANTITY) and shared by
+    the batch's StockLevels of that district: every threshold 0..255, mixed with NewOrders
+    that write the stock rows (RAW for larger ranks), equals the oracle."""
+    from workloads.formats import STOCK_LEVEL
+    wl, g, o = pair(2, "strict", tpcc.MIX_FULL, 4096, 4, seed=31)
+    compare(g, o, wl.batch(3000, 1, 0), 2)
+    rng = np.random.default_rng(5)
+    types = [STOCK_LEVEL] * 1500 + [NEW_ORDER] * 300
+    rng.shuffle(types)
+    b = wl.batch(1800, 10000, 1, types=types)
+    sl = b["type"] == STOCK_LEVEL
+    b["params"][sl, 3] = rng.integers(0, 256, sl.sum()).astype(np.uint8)
+    st = compare(g, o, b, 3)
+    assert (st[sl] == ST_COMMIT).any() and (st[sl] == ST_CONFLICT).any()
+    compare(g, o, wl.batch(2000, 20000, 2), 4)
+    compare_tables(g, o)
