@@ -165,6 +165,23 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   const DevTable& TIt = c_tabs[TI];
   const DevTable& TSt = c_tabs[TS];
   const uint8_t* p = b.params + 128ull * r;
+  uint32_t* log = tp.log + (uint64_t)r * TLOG;
+  if (PH == PH_DETECT && b.nparts <= 1) {
+    // unpartitioned detection needs no parameters: execute logged every line slot (ROW_NONE
+    // when unused) and the district row
+    if (!active) return;
+    const uint32_t row = log[sub];
+    if (row == ROW_NONE) return;
+    const DevTable& TSt = c_tabs[TS];
+    if (sub < 15) {  // same units as the general path below
+      const uint32_t gq = col_group(TSt, S_QUANTITY);
+      unit_w<PH>(TSt, gq, row, x);
+      if (col_group(TSt, S_YTD) != gq) col_upd3<PH>(TSt, S_YTD, S_ORDER_CNT, S_REMOTE_CNT, row, x);
+    } else {
+      unit_a<PH>(c_tabs[TD], col_group(c_tabs[TD], D_NEXT_O_ID), row, x, true);
+    }
+    return;
+  }
   uint32_t w = 0, d = 0, n = 0, c = 0;
   if (active) {
     w = p16(p, 0);
@@ -172,10 +189,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     n = p[3];
     c = p16(p, 4);
   }
-  uint32_t* log = tp.log + (uint64_t)r * TLOG;
   long long amount = 0;
   uint32_t remote = 0, ua = 0;
   uint32_t i = 0, sw = 0, qty = 0, row_s = ROW_NONE;
+  if (PH == PH_EXEC && active && sub < 15 && sub >= n) log[sub] = ROW_NONE;  // unused line slot
   // partitioned (§8(e)): the home partition owns the header, the order inserts and the
   // result; each stock line belongs to the owner of its supply warehouse
   const bool home = active && owns_w(b, w);
@@ -309,12 +326,18 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   const DevTable& TWh = c_tabs[TW];
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TCu = c_tabs[TC];
+  uint32_t* log = tp.log + (uint64_t)r * TLOG;
+  if (PH == PH_DETECT && b.nparts <= 1) {  // unpartitioned detection: the logged rows suffice
+    col_upd<PH>(TWh, W_YTD, log[0], x, true);
+    col_upd<PH>(TDi, D_YTD, log[1], x, true);
+    col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, log[2], x);
+    return;
+  }
   const uint8_t* p = b.params + 128ull * r;
   const uint32_t w = p16(p, 0), d = p[2], by_name = p[3], cw = p16(p, 4), cd = p[6];
   uint32_t cid = p16(p, 8);
   const uint32_t clast = p16(p, 10);
   const long long amount = p64(p, 16);
-  uint32_t* log = tp.log + (uint64_t)r * TLOG;
   // partitioned (§8(e)): warehouse + district on the home partition, the customer (its
   // by-name lookup, result and HISTORY row) on the customer's owner
   const bool home = owns_w(b, w), cust = owns_w(b, cw);
