@@ -119,6 +119,11 @@ struct ltpg_db {
   Slot slots[3];
   uint64_t submitted = 0;
   cudaStream_t h2d = nullptr, d2h = nullptr;
+  // a8 (commit bitmask, abort list) runs on its own stream once the verdicts are final,
+  // concurrently with write-back; it has its own scan scratch
+  cudaStream_t fin = nullptr;
+  cudaEvent_t status_ready = nullptr, fin_done = nullptr;
+  uint32_t* d_scan_fin = nullptr;
   ncclComm_t comm = nullptr;
 };
 
@@ -213,6 +218,9 @@ __global__ void k_sum_res(void* const* res, uint32_t np, uint64_t n, long long* 
   }
 }
 __global__ void k_copy_err(const uint32_t* src, uint32_t* dst) { *dst = *src; }
+__global__ void k_or_err(const uint32_t* src, uint32_t* dst) {
+  if (*src) *dst |= *src;
+}
 
 }  // namespace
 
@@ -276,6 +284,10 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_scan, scan_scratch_words(std::max<size_t>(n, m)) + 16));
   CK(cudaStreamCreateWithFlags(&db->h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&db->d2h, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&db->fin, cudaStreamNonBlocking));
+  CK(cudaEventCreateWithFlags(&db->status_ready, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&db->fin_done, cudaEventDisableTiming));
+  CK(dmalloc(&db->d_scan_fin, scan_scratch_words(n) + 16));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
   db->parts.resize(loop);
   std::vector<void*> ptrs(3 * 64, nullptr);
@@ -329,6 +341,10 @@ void ltpg_destroy_db(ltpg_db* db) {
   }
   if (db->h2d) cudaStreamDestroy(db->h2d);
   if (db->d2h) cudaStreamDestroy(db->d2h);
+  if (db->fin) cudaStreamDestroy(db->fin);
+  if (db->status_ready) cudaEventDestroy(db->status_ready);
+  if (db->fin_done) cudaEventDestroy(db->fin_done);
+  if (db->d_scan_fin) cudaFree(db->d_scan_fin);
   for (Part& P : db->parts) {
     void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.small, P.base};
     for (void* p : pb)
@@ -743,6 +759,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       note_launch();
     }
     if (timing) CK(cudaEventRecord(S.ev[5], s));
+    // ---- a8 on the finalize stream: commit bitmask, counts, abort list (status is final) ------
+    CK(cudaEventRecord(db->status_ready, s));
+    CK(cudaStreamWaitEvent(db->fin, db->status_ready, 0));
+    launch_finalize(S.d_status, n, S.d_bits, S.d_flags, counts, S.d_small, db->fin);
+    scan_exclusive_u32(S.d_flags, S.d_offs, n, db->d_scan_fin, db->fin);
+    launch_compact(S.d_flags, S.d_offs, n, S.d_abort, db->fin);
+    CK(cudaEventRecord(db->fin_done, db->fin));
     // ---- a7: write-back per partition -------------------------------------------------------
     for (uint32_t p = 0; p < L; ++p) {
       pb[p].status = S.d_status;
@@ -764,10 +787,11 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
       }
     }
-    // ---- finalize: commit bitmask, abort list -------------------------------------------------
-    launch_finalize(S.d_status, n, S.d_bits, S.d_flags, counts, S.d_small, s);
-    scan_exclusive_u32(S.d_flags, S.d_offs, n, db->d_scan, s);
-    launch_compact(S.d_flags, S.d_offs, n, S.d_abort, s);
+    for (uint32_t p = 0; p < L; ++p) {  // errors raised during write-back reach the caller too
+      k_or_err<<<1, 1, 0, s>>>(pb[p].err, S.d_small);
+      note_launch();
+    }
+    CK(cudaStreamWaitEvent(s, db->fin_done, 0));
   }
   CK(cudaGetLastError());
   if (timing) CK(cudaEventRecord(S.ev[6], s));
