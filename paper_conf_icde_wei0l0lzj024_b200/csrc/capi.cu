@@ -78,7 +78,8 @@ struct Slot {
   uint32_t* d_offs = nullptr;
   uint32_t* d_abort = nullptr;
   uint32_t* d_small = nullptr;             // [0] err (combined) [8..10] counts
-  uint32_t* h_small = nullptr;             // pinned: [0..15] d_small, [16] n_aborted
+  uint32_t* h_small = nullptr;             // pinned + mapped: [0..15] d_small, [16] n_aborted
+  uint32_t* h_small_dev = nullptr;         // its device-side address (written by k_publish)
   cudaEvent_t ev[8]{};
   cudaEvent_t h2d_done = nullptr, comp_done = nullptr, out_done = nullptr;
   bool pending = false, timing = false, host_out = false;
@@ -218,6 +219,9 @@ __global__ void k_sum_res(void* const* res, uint32_t np, uint64_t n, long long* 
   }
 }
 __global__ void k_copy_err(const uint32_t* src, uint32_t* dst) { *dst = *src; }
+__global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint32_t n) {
+  if (threadIdx.x < n) host_dst[threadIdx.x] = src[threadIdx.x];
+}
 __global__ void k_or_err(const uint32_t* src, uint32_t* dst) {
   if (*src) *dst |= *src;
 }
@@ -273,7 +277,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&S.d_offs, n + 1));
     CK(dmalloc(&S.d_abort, n));
     CK(dmalloc(&S.d_small, 64));
-    CK(cudaMallocHost(reinterpret_cast<void**>(&S.h_small), 64 * sizeof(uint32_t)));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&S.h_small), 64 * sizeof(uint32_t), cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S.h_small_dev), S.h_small, 0));
     for (auto& e : S.ev) CK(cudaEventCreate(&e));
     CK(cudaEventCreate(&S.h2d_done));
     CK(cudaEventCreate(&S.comp_done));
@@ -594,7 +599,11 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.flags = db->cfg.flags;
   bd.clock = b->batch_clock;
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
-  bd.status = S.d_status;
+  // verdict outputs: written in place when the caller's buffers are on the device
+  uint8_t* st_out = S.host_out ? S.d_status : res->status;
+  uint32_t* bits_out = S.host_out ? S.d_bits : res->commit_bits;
+  uint32_t* abort_out = S.host_out ? S.d_abort : res->abort_idx;
+  bd.status = st_out;
   const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
   if (b->inputs_on_device) {
     bd.tid = reinterpret_cast<const unsigned long long*>(b->tid);
@@ -635,7 +644,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // kernels of this batch: after its upload and after the slot's previous outputs were read
   CK(cudaStreamWaitEvent(s, S.out_done, 0));
   if (timing) CK(cudaEventRecord(S.ev[0], s));
-  CK(cudaMemsetAsync(S.d_small, 0, 16 * sizeof(uint32_t), s));
+  CK(cudaMemsetAsync(S.d_small, 0, 17 * sizeof(uint32_t), s));
+  if (!n && !S.host_out) CK(cudaMemsetAsync(res->n_aborted, 0, sizeof(uint32_t), s));
   if (!b->inputs_on_device) CK(cudaStreamWaitEvent(s, S.h2d_done, 0));
   const bool packed_params = !ops_mode && b->proc_offsets;
   if (packed_params) bd.params = S.d_params;
@@ -744,14 +754,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
       if (db->cfg.world == 1) {
-        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, S.d_status, db->d_ptrs + 64, S.d_small, reorder);
+        k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, st_out, db->d_ptrs + 64, S.d_small, reorder);
         k_spread_err<<<1, 1, 0, s>>>(S.d_small, db->d_ptrs + 64, L);
         note_launch(2);
       } else {
         k_pack<<<(n + 255) / 256, 256, 0, s>>>(pb[0].lflag, pb[0].err, db->d_xchg, n);
         ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, 4ull * n + 3, ncclUint8, ncclMax, db->comm, s);
         if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
-        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, S.d_status, pb[0].err, S.d_small, reorder);
+        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, st_out, pb[0].err, S.d_small, reorder);
         note_launch(2);
       }
     } else {
@@ -762,13 +772,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     // ---- a8 on the finalize stream: commit bitmask, counts, abort list (status is final) ------
     CK(cudaEventRecord(db->status_ready, s));
     CK(cudaStreamWaitEvent(db->fin, db->status_ready, 0));
-    launch_finalize(S.d_status, n, S.d_bits, S.d_flags, counts, S.d_small, db->fin);
+    launch_finalize(st_out, n, bits_out, S.d_flags, counts, S.d_small, db->fin);
     scan_exclusive_u32(S.d_flags, S.d_offs, n, db->d_scan_fin, db->fin);
-    launch_compact(S.d_flags, S.d_offs, n, S.d_abort, db->fin);
+    launch_compact(S.d_flags, S.d_offs, n, abort_out, S.d_small + 16, S.host_out ? nullptr : res->n_aborted,
+                   db->fin);
     CK(cudaEventRecord(db->fin_done, db->fin));
     // ---- a7: write-back per partition -------------------------------------------------------
     for (uint32_t p = 0; p < L; ++p) {
-      pb[p].status = S.d_status;
+      pb[p].status = st_out;
       if (ops_mode) {
         launch_ops_writeback(pb[p], s);
       } else {
@@ -800,18 +811,17 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   cudaStream_t os = S.host_out ? db->d2h : s;
   if (S.host_out) CK(cudaStreamWaitEvent(db->d2h, S.comp_done, 0));
   const cudaMemcpyKind out_kind = S.host_out ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
-  CK(cudaMemcpyAsync(S.h_small, S.d_small, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
-  if (n) {
-    CK(cudaMemcpyAsync(S.h_small + 16, S.d_offs + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
+  // error word, counters and abort count: one tiny kernel stores them into mapped host memory
+  // (cheaper than a D2H copy in stream order); device outputs were written in place
+  k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17);
+  note_launch();
+  if (n && S.host_out) {
     CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));
     CK(cudaMemcpyAsync(res->commit_bits, S.d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, os));
     if (res->reads && !reads_dev) CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
     CK(cudaMemcpyAsync(res->abort_idx, S.d_abort, n * sizeof(uint32_t), out_kind, os));
-    if (!S.host_out) CK(cudaMemcpyAsync(res->n_aborted, S.d_offs + n, sizeof(uint32_t), out_kind, os));
-  } else {
-    CK(cudaMemsetAsync(S.d_offs, 0, sizeof(uint32_t), s));
-    CK(cudaMemcpyAsync(S.h_small + 16, S.d_offs, sizeof(uint32_t), cudaMemcpyDeviceToHost, os));
-    if (!S.host_out) CK(cudaMemcpyAsync(res->n_aborted, S.d_offs, sizeof(uint32_t), out_kind, os));
+  } else if (n && res->reads && !reads_dev) {
+    CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
   }
   CK(cudaEventRecord(S.out_done, os));
   if (timing) res->stats->n_kernels = (uint32_t)(g_kernel_launches - S.launches0);

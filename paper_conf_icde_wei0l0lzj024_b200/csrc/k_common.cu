@@ -188,15 +188,21 @@ void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t 
 }
 
 // abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
+// abort list (ascending ranks) and its length (n_out[0], and n_out2[0] when not null)
 __global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ offs, uint32_t n,
-                          uint32_t* __restrict__ out) {
+                          uint32_t* __restrict__ out, uint32_t* n_out, uint32_t* n_out2) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r < n && flags[r]) out[offs[r]] = r;
+  if (r == 0) {
+    const uint32_t tot = n ? offs[n] : 0u;
+    *n_out = tot;
+    if (n_out2) *n_out2 = tot;
+  }
 }
 
-void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s) {
-  if (!n) return;
-  k_compact<<<(n + 255) / 256, 256, 0, s>>>(flags, offs, n, out);
+void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
+                    uint32_t* n_out2, cudaStream_t s) {
+  k_compact<<<n ? (n + 255) / 256 : 1, 256, 0, s>>>(flags, offs, n, out, n_out, n_out2);
   note_launch();
 }
 

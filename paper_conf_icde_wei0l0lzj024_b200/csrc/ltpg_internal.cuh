@@ -367,7 +367,8 @@ void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t 
                           cudaStream_t s);
 void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* flags,
                      uint32_t* counts, const uint32_t* err, cudaStream_t s);
-void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, cudaStream_t s);
+void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
+                    uint32_t* n_out2, cudaStream_t s);
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
 void launch_build_index_tail(uint32_t t, const unsigned long long* from, uint32_t* err, cudaStream_t s);
 void launch_note_rows(uint32_t t, unsigned long long* dst, cudaStream_t s);
