@@ -20,7 +20,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libltpg.so")
 
 if not os.path.exists(LIB_PATH):
-    raise ImportError("libltpg.so not built: run `python -m paper_conf_icde_wei0l0lzj024_b200.build` "
+    raise ImportError("libltpg.so not built: run `python paper_conf_icde_wei0l0lzj024_b200/build.py` "
                       "(or __graft_entry__.build()); there is no CPU fallback")
 
 _lib = ctypes.CDLL(LIB_PATH)

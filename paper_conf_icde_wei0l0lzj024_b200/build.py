@@ -1,6 +1,6 @@
 """Build libltpg.so (sm_100a) in-tree with nvcc.
 
-    python -m paper_conf_icde_wei0l0lzj024_b200.build [--force]
+    python paper_conf_icde_wei0l0lzj024_b200/build.py [--force]
 """
 import concurrent.futures
 import os
