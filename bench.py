@@ -331,6 +331,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flags", type=int, default=0)
+    ap.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
+                    help="N>1: peer-memory verdict exchange (default) or the ncclAllReduce baseline")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -360,7 +362,8 @@ def main():
     fused_front = w["kind"] == "ycsb" and not (args.flags & (ltpg.LTPG_FLAG_REORDER | ltpg.LTPG_FLAG_NO_GROUPING
                                                               | ltpg.LTPG_FLAG_UNFUSED))
     uid = None
-    if world > 1:  # one NCCL communicator per db: the per-batch verdict exchange
+    if world > 1 and args.exchange == "nccl":  # baseline: one NCCL communicator per db
+        args.flags |= ltpg.LTPG_FLAG_NCCL_EXCHANGE
         from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id
         uid = nccl_unique_id()
     t0 = time.time()
@@ -574,8 +577,10 @@ def main():
             "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": dict(config_of(name), parallelism=(
-                "%d partitions (%s), same global batch, per-txn verdicts exchanged by ncclAllReduce"
-                % (world, "warehouse ranges" if w["kind"] == "tpcc" else "key ranges")) if world > 1
+                "%d partitions (%s), same global batch, per-txn verdicts exchanged by %s"
+                % (world, "warehouse ranges" if w["kind"] == "tpcc" else "key ranges",
+                   "ncclAllReduce" if args.exchange == "nccl" else "peer-memory stores + signals (csrc/xchg.cu)"))
+                if world > 1
                 else "single GPU"),
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": kernels, "roofline": roof,
             "commit_rate": all_commits / all_procs, "processed_txns_per_s": all_procs / total_s,

@@ -129,6 +129,8 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
                                               WAW or (RAW and WAR); keeps per-unit min reader marks */
 #define LTPG_FLAG_UNFUSED       (1u << 3)  /* A/B: OPS mode runs validate+division and execute as
                                               two kernels with global per-kind lists          */
+#define LTPG_FLAG_NCCL_EXCHANGE (1u << 4)  /* world > 1, A/B baseline: exchange verdicts and result
+                                              sums with ncclAllReduce instead of peer memory   */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
 
 typedef struct {
@@ -147,16 +149,34 @@ typedef struct {
 /* Multi-GPU: world > 1 ranks each own a contiguous range of warehouses
  * (TPC-C, owner_rule 1) or of keys (OPS, owner_rule 2).  Every rank calls ltpg_run_batch
  * with the same global batch; each executes, marks and checks only the units it owns,
- * then the per-txn verdicts are exchanged (one ncclAllReduce(MAX) of a byte per txn over
- * NVLink) before write-back, so commit_bits / status / abort_idx are identical on all
- * ranks.  Result slots are filled by the owning rank and summed over ranks
- * (ncclAllReduce(SUM)).  LTPG_FLAG_LOOPBACK_SHIFT runs P logical partitions inside one
- * process on one GPU with the same ownership, exchange and result-sum logic. */
+ * then the per-txn conflict bits are exchanged before write-back, so commit_bits / status /
+ * abort_idx are identical on all ranks.  Result slots are filled by the owning rank and
+ * summed over ranks.  The exchange runs over peer memory (default, world <= 32): each rank
+ * stores 4 bit planes per 32 txns into every peer's exchange region over NVLink and raises a
+ * signal; the combine kernel waits for all signals (no host round trip).  Bootstrap: every
+ * rank calls ltpg_peer_handle, the caller all-gathers the handles (e.g. torch.distributed)
+ * and passes them, in rank order, to ltpg_connect_peers before the first batch.  With
+ * LTPG_FLAG_NCCL_EXCHANGE the exchange is ncclAllReduce(MAX / SUM) on a communicator built
+ * from nccl_unique_id instead.  Every rank must run the same sequence of batches, and
+ * ltpg_destroy_db only after every rank finished its last batch (a barrier): peers read
+ * this rank's region during their batches.  A peer that never arrives fails the batch
+ * after 20 s (LTPG_EINTERNAL).  LTPG_FLAG_LOOPBACK_SHIFT runs P logical partitions inside
+ * one process on one GPU with the same ownership, combine and result-sum logic. */
+#define LTPG_PEER_HANDLE_BYTES 128
 
 typedef struct ltpg_db ltpg_db;  /* opaque, library-owned device state */
 
 /* Create a database on config->device.  *out receives the handle. */
 LTPG_API int ltpg_create_db(const ltpg_config* config, ltpg_db** out);
+
+/* Peer-memory exchange bootstrap (world > 1 without LTPG_FLAG_NCCL_EXCHANGE).
+ * ltpg_peer_handle writes this rank's LTPG_PEER_HANDLE_BYTES-byte handle (a CUDA IPC handle of
+ * its exchange region plus the configuration it must match) to host memory `handle`.
+ * ltpg_connect_peers takes all world handles back to back in rank order (host memory), checks
+ * that every rank has the same max_txns / max_ops / flags (else EINVAL) and maps the peers'
+ * regions.  Ranks on the same GPU are allowed (CUDA IPC within one device). */
+LTPG_API int ltpg_peer_handle(ltpg_db* db, void* handle);
+LTPG_API int ltpg_connect_peers(ltpg_db* db, const void* handles);
 
 /* Table descriptor.  col_group[c] in [0, n_groups) or LTPG_STATIC; col_is_add[c]
  * marks a delayed-ADD column (its group may hold ADD columns only).  Tables with

@@ -35,6 +35,8 @@ LTPG_FLAG_NO_GROUPING = 1 << 0
 LTPG_FLAG_NO_MARK_FILTER = 1 << 1
 LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_UNFUSED = 1 << 3
+LTPG_FLAG_NCCL_EXCHANGE = 1 << 4
+LTPG_PEER_HANDLE_BYTES = 128
 LTPG_LAYOUT_ROWBLOCK, LTPG_LAYOUT_COLUMNAR = 0, 1
 LTPG_FLAG_LOOPBACK_SHIFT = 8
 LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
@@ -89,6 +91,10 @@ _lib.ltpg_last_error.restype = ctypes.c_char_p
 _lib.ltpg_last_error.argtypes = [c_vp]
 _lib.ltpg_wait_batch.restype = c_int
 _lib.ltpg_wait_batch.argtypes = [c_vp, ctypes.POINTER(ltpg_result)]
+_lib.ltpg_peer_handle.restype = c_int
+_lib.ltpg_peer_handle.argtypes = [c_vp, c_vp]
+_lib.ltpg_connect_peers.restype = c_int
+_lib.ltpg_connect_peers.argtypes = [c_vp, c_vp]
 _lib.ltpg_version.restype = ctypes.c_char_p
 _lib.ltpg_version.argtypes = []
 
@@ -101,10 +107,12 @@ ltpg_destroy_db = _lib.ltpg_destroy_db
 ltpg_last_error = _lib.ltpg_last_error
 ltpg_version = _lib.ltpg_version
 ltpg_wait_batch = _lib.ltpg_wait_batch
+ltpg_peer_handle = _lib.ltpg_peer_handle
+ltpg_connect_peers = _lib.ltpg_connect_peers
 LTPG_BATCH_ASYNC = 1
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
-            "ltpg_destroy_db", "ltpg_last_error", "ltpg_version"]
+            "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers"]
 
 
 class LtpgError(RuntimeError):
@@ -152,6 +160,19 @@ class Database:
         self.n_cols = {}
         self.has_pk = {}
         self._out = None
+
+    # -- multi-rank peer-memory exchange bootstrap (include/ltpg.h) ----------------------------
+    def peer_handle(self):
+        """This rank's LTPG_PEER_HANDLE_BYTES-byte exchange handle (bytes)."""
+        buf = ctypes.create_string_buffer(LTPG_PEER_HANDLE_BYTES)
+        self._check(ltpg_peer_handle(self.h, ctypes.cast(buf, c_vp)))
+        return buf.raw
+
+    def connect_peers(self, handles):
+        """handles: every rank's peer_handle(), in rank order."""
+        blob = b"".join(bytes(h) for h in handles)
+        buf = ctypes.create_string_buffer(blob, len(blob))
+        self._check(ltpg_connect_peers(self.h, ctypes.cast(buf, c_vp)))
 
     def close(self):
         if getattr(self, "h", None) is not None and self.h.value:
@@ -315,7 +336,7 @@ def part_of_key(key, key_space, nparts):
 
 
 def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0, loopback=1, rank=0, world=1,
-                  nccl_unique_id=None):
+                  nccl_unique_id=None, peer_group=None):
     """YCSB usertable, key-range partitioned (owner_rule 2) when world * loopback > 1; a
     multi-rank db loads only its own key range."""
     db = Database(1, max_txns, max_ops, device=device, flags=flags, key_space=workload.n_rows, loopback=loopback,
@@ -326,7 +347,15 @@ def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0,
         own = part_of_key(keys, workload.n_rows, world) == rank
         keys, cols = keys[own], cols[:, own]
     db.load_table(0, g, a, ng, keys, cols, capacity=capacity or max(len(keys), 1), has_pk=pk, owner_rule=2)
+    _connect(db, world, flags, peer_group)
     return db
+
+
+def _connect(db, world, flags, group):
+    """Multi-rank db with the peer-memory exchange: all-gather the handles (torch.distributed)."""
+    if world > 1 and not (flags & LTPG_FLAG_NCCL_EXCHANGE):
+        from .dist import connect_peers
+        connect_peers(db, group)
 
 
 def tpcc_owner_w(t, keys, cols):
@@ -351,7 +380,7 @@ def tpcc_owner_w(t, keys, cols):
 
 
 def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None,
-                  loopback=1, rank=0, world=1, nccl_unique_id=None, max_ops=0):
+                  loopback=1, rank=0, world=1, nccl_unique_id=None, max_ops=0, peer_group=None):
     """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns.
     A multi-rank db (world > 1) loads only the rows of its warehouses (ITEM replicated)."""
     from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY, T_ITEM
@@ -373,4 +402,5 @@ def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, f
         db.load_table(t, g, a, ng, k, c, capacity=max(cap, 1), has_pk=pk,
                       owner_rule=0 if t == T_ITEM else 1,
                       layout=LTPG_LAYOUT_COLUMNAR if t in (T_ORDER, T_ORDER_LINE) else LTPG_LAYOUT_ROWBLOCK)
+    _connect(db, world, flags, peer_group)
     return db

@@ -17,6 +17,7 @@
 
 #include "ltpg_internal.cuh"
 #include "tpcc_internal.cuh"
+#include "xchg.cuh"
 
 using namespace ltpg;
 
@@ -126,7 +127,24 @@ struct ltpg_db {
   cudaEvent_t status_ready = nullptr, fin_done = nullptr;
   uint32_t* d_scan_fin = nullptr;
   ncclComm_t comm = nullptr;
+  // peer-memory exchange (world > 1 without LTPG_FLAG_NCCL_EXCHANGE; xchg.cuh)
+  bool p2p = false, connected = false;
+  XLayout xl;
+  XPeers xpeers{};
+  char* xregion = nullptr;
+  uint32_t* d_xdone = nullptr;
+  std::vector<void*> opened;  // peer regions mapped with cudaIpcOpenMemHandle
 };
+
+// what ltpg_peer_handle exports (LTPG_PEER_HANDLE_BYTES)
+struct PeerHandle {
+  cudaIpcMemHandle_t h;
+  uint64_t bytes;
+  uint32_t magic, rank, world, max_txns, max_ops, flags;
+  uint8_t pad[LTPG_PEER_HANDLE_BYTES - sizeof(cudaIpcMemHandle_t) - 8 - 24];
+};
+static_assert(sizeof(PeerHandle) == LTPG_PEER_HANDLE_BYTES, "peer handle size");
+constexpr uint32_t PEER_MAGIC = 0x4C545047u;  // "LTPG"
 
 namespace {
 
@@ -240,7 +258,9 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   const uint32_t loop = std::max<uint32_t>(1, (cfg->flags >> LTPG_FLAG_LOOPBACK_SHIFT) & 0xF);
   if (cfg->n_tables == 0 || cfg->n_tables > MAXT || cfg->max_txns == 0 || cfg->world < 1 ||
       cfg->rank < 0 || cfg->rank >= cfg->world || cfg->max_txns > (1u << 24) || cfg->max_ops > (1u << 24) ||
-      cfg->n_warehouses > 1000 || (cfg->world > 1 && !cfg->nccl_unique_id) || cfg->world * loop > 64 ||
+      cfg->n_warehouses > 1000 || cfg->world * loop > 64 ||
+      (cfg->world > 1 && (cfg->flags & LTPG_FLAG_NCCL_EXCHANGE) && !cfg->nccl_unique_id) ||
+      (cfg->world > 32 && !(cfg->flags & LTPG_FLAG_NCCL_EXCHANGE)) ||
       (cfg->world > 1 && loop > 1))
     return LTPG_EINVAL;
   db = new ltpg_db();
@@ -313,7 +333,15 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     ptrs[128 + p] = P.res;
   }
   CK(cudaMemcpy(db->d_ptrs, ptrs.data(), ptrs.size() * sizeof(void*), cudaMemcpyHostToDevice));
-  if (cfg->world > 1) {
+  if (cfg->world > 1 && !(cfg->flags & LTPG_FLAG_NCCL_EXCHANGE)) {  // peer-memory exchange region
+    db->p2p = true;
+    db->xl.init(cfg->max_txns, nres, (uint32_t)cfg->world);
+    CK(cudaMalloc(reinterpret_cast<void**>(&db->xregion), db->xl.bytes));
+    CK(cudaMemset(db->xregion, 0, db->xl.bytes));
+    CK(dmalloc(&db->d_xdone, 1));
+    CK(cudaMemset(db->d_xdone, 0, sizeof(uint32_t)));
+    db->xpeers.base[cfg->rank] = db->xregion;
+  } else if (cfg->world > 1) {
     if (!g_nccl.load()) return fail(db, LTPG_ENCCL, "libnccl.so.2 not loadable");
     ncclUniqueId id;
     std::memcpy(&id, cfg->nccl_unique_id, sizeof(id));
@@ -357,6 +385,9 @@ void ltpg_destroy_db(ltpg_db* db) {
     tpcc_free(P.tpcc);
   }
   if (db->comm) g_nccl.commDestroy(db->comm);
+  for (void* p : db->opened) cudaIpcCloseMemHandle(p);
+  if (db->xregion) cudaFree(db->xregion);
+  if (db->d_xdone) cudaFree(db->d_xdone);
   delete db;
 }
 
@@ -572,6 +603,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     return fail(db, LTPG_EINVAL, "bad OPS batch");
   if (!ops_mode && (!b->proc_type || !b->proc_params || !db->cfg.n_warehouses))
     return fail(db, LTPG_EINVAL, "bad TPCC batch");
+  if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
   Slot& S = db->slots[db->submitted % 3];
   if (S.pending) return fail(db, LTPG_EINVAL, "three batches already in flight: ltpg_wait_batch first");
   ++db->submitted;
@@ -695,6 +727,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     BatchDev& x = pb[p];
     x.part = (uint32_t)db->cfg.rank * L + p;
     x.res = (!partitioned && p == 0) ? res_out : P.res;
+    if (db->p2p)  // own result slots live in the exchange region (peers pull them), by parity
+      x.res = reinterpret_cast<long long*>(db->xregion + db->xl.off_res) + (uint64_t)(db->epoch & 1u) * db->xl.nres;
     x.uref = P.uref;
     x.items = P.items;
     x.txn_ins = P.txn_ins;
@@ -708,7 +742,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
     if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
     if (partitioned && n) {
-      CK(cudaMemsetAsync(P.res, 0, n_reads * sizeof(long long), s));
+      CK(cudaMemsetAsync(x.res, 0, n_reads * sizeof(long long), s));
       CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
     }
   }
@@ -753,7 +787,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (timing) CK(cudaEventRecord(S.ev[4], s));
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
-      if (db->cfg.world == 1) {
+      if (db->p2p) {  // planes stored into every rank's region, signal, wait + OR (xchg.cuh)
+        launch_xput(pb[0].lflag, pb[0].err, n, db->xpeers, db->xl, (uint32_t)db->cfg.rank, db->epoch, db->d_xdone, s);
+        launch_xcombine(db->xregion, db->xl, n, db->epoch, reorder, st_out, pb[0].err, S.d_small, s);
+      } else if (db->cfg.world == 1) {
         k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, st_out, db->d_ptrs + 64, S.d_small, reorder);
         k_spread_err<<<1, 1, 0, s>>>(S.d_small, db->d_ptrs + 64, L);
         note_launch(2);
@@ -789,7 +826,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     }
     if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
-    if (partitioned && res->reads) {
+    if (db->p2p) {  // every rank publishes (the protocol needs it); the sum is pulled on demand
+      launch_xsig_res(db->xpeers, (uint32_t)db->cfg.rank, (uint32_t)db->cfg.world, db->epoch, s);
+      if (res->reads) launch_xsum(db->xpeers, db->xl, n_reads, db->epoch, res_out, S.d_small, (uint32_t)db->cfg.rank, s);
+    } else if (partitioned && res->reads) {
       if (db->cfg.world == 1) {
         k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);
         note_launch();
@@ -828,6 +868,48 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   S.pending = true;
   if (async) return LTPG_OK;
   return finish_slot(db, S);
+}
+
+int ltpg_peer_handle(ltpg_db* db, void* out) {
+  if (!db || !out) return LTPG_EINVAL;
+  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1 or LTPG_FLAG_NCCL_EXCHANGE)");
+  CK(cudaSetDevice(db->device));
+  PeerHandle h{};
+  CK(cudaIpcGetMemHandle(&h.h, db->xregion));
+  h.bytes = db->xl.bytes;
+  h.magic = PEER_MAGIC;
+  h.rank = (uint32_t)db->cfg.rank;
+  h.world = (uint32_t)db->cfg.world;
+  h.max_txns = db->cfg.max_txns;
+  h.max_ops = db->cfg.max_ops;
+  h.flags = db->cfg.flags;
+  std::memcpy(out, &h, sizeof(h));
+  return LTPG_OK;
+}
+
+int ltpg_connect_peers(ltpg_db* db, const void* handles) {
+  if (!db || !handles) return LTPG_EINVAL;
+  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1 or LTPG_FLAG_NCCL_EXCHANGE)");
+  if (db->connected) return fail(db, LTPG_EINVAL, "peers already connected");
+  CK(cudaSetDevice(db->device));
+  const uint32_t world = (uint32_t)db->cfg.world;
+  std::vector<PeerHandle> hs(world);
+  std::memcpy(hs.data(), handles, world * sizeof(PeerHandle));
+  for (uint32_t q = 0; q < world; ++q) {
+    const PeerHandle& h = hs[q];
+    if (h.magic != PEER_MAGIC || h.rank != q || h.world != world || h.bytes != db->xl.bytes ||
+        h.max_txns != db->cfg.max_txns || h.max_ops != db->cfg.max_ops || h.flags != db->cfg.flags)
+      return fail(db, LTPG_EINVAL, "peer handle " + std::to_string(q) + " does not match this db's configuration");
+  }
+  for (uint32_t q = 0; q < world; ++q) {
+    if (q == (uint32_t)db->cfg.rank) continue;
+    void* p = nullptr;
+    CK(cudaIpcOpenMemHandle(&p, hs[q].h, cudaIpcMemLazyEnablePeerAccess));
+    db->opened.push_back(p);
+    db->xpeers.base[q] = static_cast<char*>(p);
+  }
+  db->connected = true;
+  return LTPG_OK;
 }
 
 int ltpg_dump_table(ltpg_db* db, uint32_t t, uint64_t* n_rows_out, uint64_t* keys, int64_t* cols) {

@@ -1,0 +1,60 @@
+// Peer-memory verdict / result exchange between ranks.
+//
+// Every rank owns one "exchange region" (cudaMalloc, exported with cudaIpcGetMemHandle and
+// mapped by every peer with cudaIpcOpenMemHandle; over NVLink 5 / NVSwitch on an 8xB200 box).
+// Regions have the same layout on every rank:
+//
+//   sig  [2 parity][2 kind][64 src] u64      kind 0: verdict planes of epoch e are in place
+//                                            kind 1: result slots of epoch e are final
+//   board[2 parity][world src][nwords] uint4  per 32 txns: conflict-bit planes {UA,WAW,RAW,WAR}
+//   res  [2 parity][nres] i64                the rank's own result slots (peers pull them)
+//
+// Rank q's batch e: detect -> k_xput stores its planes into board[e&1][q] of EVERY region
+// (its own included) and, after a system-scope fence, sig[e&1][0][q] = e<<3 | err bits.
+// k_xcombine waits until all world signals of epoch e are in ITS region, ORs the planes and
+// writes the final status (identical on all ranks).  After write-back, k_xsig_res publishes
+// sig[e&1][1][q] = e and k_xsum pulls and sums every rank's result slots.
+//
+// Buffer reuse is safe with two parities: rank q can only write parity (e&1) again in batch
+// e+2, which it reaches after its combine of batch e+1, which waited for every peer's
+// verdict signal of e+1 -- sent by each peer after it finished its combine / sum of batch e.
+#pragma once
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace ltpg {
+
+struct XLayout {
+  uint64_t nwords = 0, nres = 0;
+  uint32_t world = 1;
+  uint64_t off_board = 0, off_res = 0, bytes = 0;
+  void init(uint32_t max_txns, uint64_t nres_, uint32_t world_) {
+    world = world_;
+    nwords = (max_txns + 31) / 32;
+    nres = nres_;
+    off_board = 2 * 2 * 64 * sizeof(uint64_t);
+    off_res = off_board + 2ull * world * nwords * 16;
+    off_res = (off_res + 255) & ~255ull;
+    bytes = off_res + 2ull * nres * sizeof(long long);
+  }
+};
+
+struct XPeers {
+  char* base[64];  // region of each rank, mapped into this process (own region included)
+};
+
+// after detect: local per-txn conflict bits -> planes in every region, then the signal
+void launch_xput(const uint8_t* lflag, const uint32_t* err, uint32_t n, const XPeers& peers, const XLayout& L,
+                 uint32_t rank, uint32_t epoch, uint32_t* done_counter, cudaStream_t s);
+// wait for every rank's verdict of `epoch`, OR the planes -> status; OR of the error bits
+// -> *err (this rank's partition word) and *err_all
+void launch_xcombine(char* own, const XLayout& L, uint32_t n, uint32_t epoch, bool reorder, uint8_t* status,
+                     uint32_t* err, uint32_t* err_all, cudaStream_t s);
+// after write-back: publish "my result slots of `epoch` are final"
+void launch_xsig_res(const XPeers& peers, uint32_t rank, uint32_t world, uint32_t epoch, cudaStream_t s);
+// wait for every rank's result signal, out[i] = sum over ranks of their slot i
+void launch_xsum(const XPeers& peers, const XLayout& L, uint64_t n_reads, uint32_t epoch, long long* out,
+                 uint32_t* err, uint32_t rank, cudaStream_t s);
+
+}  // namespace ltpg

@@ -1,8 +1,10 @@
 """Host-side plumbing for the multi-GPU path; one process per GPU.
 
-torch.distributed is only used to share the 128-byte NCCL unique id and for
-bench-side timing reductions; the per-batch exchange itself is the library's own
-ncclAllReduce on the db's communicator (csrc/capi.cu).
+torch.distributed (any backend: nccl on the GPU box, gloo in CPU tests) only carries the
+bootstrap -- the ranks' 128-byte exchange handles (CUDA IPC handles of their exchange
+regions), or the NCCL unique id of the LTPG_FLAG_NCCL_EXCHANGE baseline -- and bench-side
+timing reductions.  The per-batch exchange itself is the library's own peer-memory kernels
+(csrc/xchg.cu) or ncclAllReduce (csrc/capi.cu).
 """
 import numpy as np
 
@@ -14,6 +16,19 @@ def nccl_unique_id(group=None):
     obj = [torch.cuda.nccl.unique_id() if dist.get_rank(group) == 0 else None]
     dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
     return obj[0]
+
+
+def gather_handles(handle, group=None):
+    """All ranks' exchange handles (bytes), in rank order of `group`."""
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, bytes(handle), group=group)
+    return out
+
+
+def connect_peers(db, group=None):
+    """Bootstrap a multi-rank db's peer-memory exchange: every rank of `group` calls this."""
+    db.connect_peers(gather_handles(db.peer_handle(), group))
 
 
 def warehouse_ranges(n_warehouses, world):

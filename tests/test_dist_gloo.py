@@ -84,3 +84,36 @@ def test_key_ranges_match_part_of_key():
         p = L.part_of_key(keys, ks, world)
         for r, (lo, hi) in enumerate(D.key_ranges(ks, world)):
             assert ((keys >= lo) & (keys < hi) == (p == r)).all()
+
+
+def _handles_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch.distributed as dist
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_icde_wei0l0lzj024_b200 import dist as D
+        mine = bytes([rank]) * 128  # stands in for ltpg_peer_handle's 128 bytes
+        q.put((rank, D.gather_handles(mine)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_peer_handle_allgather_rank_order():
+    """Peer-memory bootstrap: every rank receives all handles, in rank order (what
+    ltpg_connect_peers requires)."""
+    world = 3
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_handles_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=300) for _ in range(world)], key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, hs in res:
+        assert hs == [bytes([r]) * 128 for r in range(world)]
