@@ -347,11 +347,20 @@ def main():
         return
 
     import torch
+    # one rank per GPU; with fewer GPUs than ranks (a functional check on a 1-GPU box) ranks
+    # share devices, the library's exchange then runs over CUDA IPC on one device and the
+    # bench plumbing uses gloo (NCCL refuses two ranks on one GPU)
+    ndev = torch.cuda.device_count()
+    shared = world > ndev
+    local = local % ndev
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     import paper_conf_icde_wei0l0lzj024_b200 as ltpg
 
     w = WORKLOADS[name]
@@ -481,7 +490,7 @@ def main():
     # every rank reports the same commits: count them once; time = max over ranks
     all_commits, all_procs = float(sum(commits)), float(sum(procs))
     if dist:
-        t = torch.tensor([total_s], device=dev)
+        t = torch.tensor([total_s], device="cpu" if shared else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_s = float(t.item())
     value = all_commits / total_s
@@ -527,7 +536,7 @@ def main():
         e_s = e0.elapsed_time(e1) / 1000.0
         e_c = float(sum(e_commits))
         if dist:
-            t = torch.tensor([e_s], device=dev)
+            t = torch.tensor([e_s], device="cpu" if shared else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_s = float(t.item())
         e2e = {"value": e_c / e_s, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
@@ -587,6 +596,9 @@ def main():
             "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)
                               for k in ("ms_upload", "ms_group", "ms_exec", "ms_detect", "ms_writeback",
                                         "ms_download")}}
+    if shared:
+        line["config"]["devices"] = ("%d ranks on %d GPU(s): functional check of the multi-rank path, "
+                                     "not a scaling number" % (world, ndev))
     if world == 1 and not args.no_cpu_baseline:
         try:
             line["cpu_baseline"] = cpu_baseline(name, host_batches[0], make_workload(name, 0))
