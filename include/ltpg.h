@@ -131,6 +131,10 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
                                               two kernels with global per-kind lists          */
 #define LTPG_FLAG_NCCL_EXCHANGE (1u << 4)  /* world > 1, A/B baseline: exchange verdicts and result
                                               sums with ncclAllReduce instead of peer memory   */
+#define LTPG_FLAG_LARGE_BUCKETS (1u << 5)  /* NEXT-3: tables with E = max_txns/rows > 1
+                                              record marks in large-sized buckets of
+                                              ceil(E/32)*32 sub-slots (TID mod s_u), folded per
+                                              unit before detection; result-identical          */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
 
 typedef struct {

@@ -10,6 +10,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -179,6 +180,8 @@ void free_table(DevTable& T) {
   if (T.rmarks) cudaFree(T.rmarks);
   if (T.idx) cudaFree(T.idx);
   if (T.aux) cudaFree(T.aux);
+  for (mark_t* p : T.sub)
+    if (p) cudaFree(p);
   unsigned long long* nr = T.n_rows;
   T = DevTable{};
   T.n_rows = nr;
@@ -328,6 +331,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&P.base, MAXT));
     int rc = tpcc_alloc(P.tpcc, cfg->max_txns, cfg->n_warehouses, p ? db->parts[0].tpcc.by_name : nullptr);
     if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
+    P.tpcc.h_tab = db->h_tab;
+    P.tpcc.n_tab = cfg->n_tables;
     ptrs[p] = P.lflag;
     ptrs[64 + p] = P.small;
     ptrs[128 + p] = P.res;
@@ -481,6 +486,19 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
     if (db->cfg.flags & LTPG_FLAG_REORDER) {  // NEXT-1: minimum reader rank per unit
       CK(dmalloc(&T.rmarks, cap * d->n_groups));
       CK(cudaMemset(T.rmarks, 0xFF, cap * d->n_groups * sizeof(mark_t)));
+    }
+    // NEXT-3: a popular table -- E = T/D > 1 with T bounded by the batch capacity
+    // and D the loaded rows -- gets large-sized buckets of su = ceil(E/32)*32 sub-slots per unit
+    const double E = (double)db->cfg.max_txns / (double)std::max<uint64_t>(n_rows, 1);
+    if ((db->cfg.flags & LTPG_FLAG_LARGE_BUCKETS) && E > 1.0) {
+      T.su = (uint32_t)std::min<double>(std::ceil(E / 32.0) * 32.0, 1u << 20);
+      const uint64_t units[3] = {cap * d->n_groups, cap * __builtin_popcount(T.add_groups),
+                                 T.rmarks ? cap * d->n_groups : 0};
+      for (int k = 0; k < 3; ++k) {
+        if (!units[k]) continue;
+        CK(dmalloc(&T.sub[k], units[k] * T.su));
+        CK(cudaMemset(T.sub[k], 0xFF, units[k] * T.su * sizeof(mark_t)));
+      }
     }
   }
   if (d->has_pk) {
@@ -701,6 +719,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       if (T.wmarks) CK(cudaMemsetAsync(T.wmarks, 0xFF, units, s));
       if (T.rmarks) CK(cudaMemsetAsync(T.rmarks, 0xFF, units, s));
       if (T.amarks) CK(cudaMemsetAsync(T.amarks, 0xFF, T.capacity * __builtin_popcount(T.add_groups) * sizeof(mark_t), s));
+      const uint64_t su_units[3] = {T.capacity * T.n_groups, T.capacity * __builtin_popcount(T.add_groups),
+                                    T.capacity * T.n_groups};
+      for (int k = 0; k < 3; ++k)
+        if (T.sub[k]) CK(cudaMemsetAsync(T.sub[k], 0xFF, su_units[k] * T.su * sizeof(mark_t), s));
     }
   }
   if (db->idx_lag && (ops_mode || !db->olrow_ready)) {  // key lookups ahead: catch the indexes up
@@ -777,6 +799,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
           if (evp) CK(cudaEventRecord(evp[2], s));
           launch_ops_exec(x, grouped, filter, s);
         }
+        launch_bucket_reduce(db->h_tab, db->n_tables, s);  // NEXT-3 large-sized buckets (if any)
         if (evp) CK(cudaEventRecord(evp[3], s));
         launch_ops_detect(x, s);
       } else {

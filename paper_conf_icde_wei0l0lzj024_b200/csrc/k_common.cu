@@ -1,6 +1,8 @@
 // Shared kernels: deterministic exclusive scan, result finalisation (commit
 // bitmask via __ballot_sync, abort-list compaction), index build, capacity and
 // append-cursor bookkeeping.
+#include <algorithm>
+
 #include "ltpg_internal.cuh"
 
 namespace ltpg {
@@ -204,6 +206,48 @@ void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uin
                     uint32_t* n_out2, cudaStream_t s) {
   k_compact<<<n ? (n + 255) / 256 : 1, 256, 0, s>>>(flags, offs, n, out, n_out, n_out2);
   note_launch();
+}
+
+// ---- NEXT-3: large-sized bucket -> unit mark (min over the bucket's su sub-slots) ----------
+// One block per (unit, chunk of 1024 sub-slots); the chunk minima meet in the unit's word with
+// atomicMin.  Older epochs carry larger tag bytes, so a stale word or sub-slot never hides a
+// mark of this batch, and mark_rank ignores it when nothing of this batch is there.
+__global__ void __launch_bounds__(256) k_bucket_reduce(const mark_t* __restrict__ sub, mark_t* word, uint64_t units,
+                                                       uint32_t su) {
+  __shared__ mark_t wmin[8];
+  const uint32_t per = (su + 1023) / 1024;
+  for (uint64_t c = blockIdx.x; c < units * per; c += gridDim.x) {
+    const uint64_t u = c / per;
+    const uint32_t j0 = (uint32_t)(c % per) * 1024u;
+    mark_t m = 0xFFFFFFFFu;
+    for (uint32_t j = j0 + threadIdx.x; j < su && j < j0 + 1024u; j += blockDim.x) m = min(m, sub[u * su + j]);
+    m = __reduce_min_sync(0xffffffffu, m);
+    if ((threadIdx.x & 31) == 0) wmin[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (int w = 1; w < 8; ++w) m = min(m, wmin[w]);
+      if (m != 0xFFFFFFFFu) atomicMin(word + u, m);
+    }
+    __syncthreads();
+  }
+}
+
+void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s) {
+  for (uint32_t t = 0; t < n_tables; ++t) {
+    const DevTable& T = h_tab[t];
+    if (T.su <= 1) continue;
+    const mark_t* sub[3] = {T.sub[0], T.sub[1], T.sub[2]};
+    mark_t* word[3] = {T.wmarks, T.amarks, T.rmarks};
+    const uint64_t units[3] = {(uint64_t)T.n_groups * T.capacity,
+                               (uint64_t)__builtin_popcount(T.add_groups) * T.capacity,
+                               (uint64_t)T.n_groups * T.capacity};
+    for (int k = 0; k < 3; ++k) {
+      if (!sub[k] || !word[k] || !units[k]) continue;
+      const uint64_t chunks = units[k] * ((T.su + 1023) / 1024);
+      k_bucket_reduce<<<(unsigned)std::min<uint64_t>(chunks, 148 * 8), 256, 0, s>>>(sub[k], word[k], units[k], T.su);
+      note_launch();
+    }
+  }
 }
 
 __global__ void k_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n) {

@@ -219,7 +219,7 @@ void launch_ops_claim(const BatchDev& b, cudaStream_t s) {
 // ---- K-exec ---------------------------------------------------------------------------
 __device__ __forceinline__ void mark_read(const DevTable& T, uint32_t g, uint32_t row, mark_t tag,
                                           bool filter) {
-  if (T.rmarks) mark_min(rmark_ptr(T, g, row), tag, filter);  // NEXT-1 only: min reader rank
+  if (T.rmarks) mark_unit(T, MK_R, g, row, tag, filter);  // NEXT-1 only: min reader rank
 }
 
 // uref bit 58: absent key read before K-claim ran (fused path); K-detect probes it for a claim
@@ -276,14 +276,14 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi, uint32_
     case LTPG_UPDATE: {
       uint32_t g = col_group(T, o.col);
       res = *col_ptr_ops(T, o.col, row);  // pre-image; new value = res + arg at write-back
-      mark_min(wmark_ptr(T, g, row), tag, filter);
+      mark_unit(T, MK_W, g, row, tag, filter);
       uref = make_uref(CHK_RW, false, true, o.table, g, row, true);
       break;
     }
     case LTPG_ADD: {
       uint32_t g = col_group(T, o.col);
       res = 0;
-      mark_min(amark_ptr(T, g, row), tag, filter);
+      mark_unit(T, MK_A, g, row, tag, filter);
       uref = make_uref(CHK_A, false, true, o.table, g, row, true);
       break;
     }
@@ -299,13 +299,13 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi, uint32_
           return;
         }
         res = 1;
-        for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(wmark_ptr(T, g, claim), tag, filter);
+        for (uint32_t g = 0; g < T.n_groups; ++g) mark_unit(T, MK_W, g, claim, tag, filter);
         uref = make_uref(CHK_RW, true, false, o.table, 0, claim, true);
       }
       break;
     case LTPG_DELETE:
       res = 1;
-      for (uint32_t g = 0; g < T.n_groups; ++g) mark_min(wmark_ptr(T, g, row), tag, filter);
+      for (uint32_t g = 0; g < T.n_groups; ++g) mark_unit(T, MK_W, g, row, tag, filter);
       uref = make_uref(CHK_RW, true, true, o.table, 0, row, true);
       break;
   }

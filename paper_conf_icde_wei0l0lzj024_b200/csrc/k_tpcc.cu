@@ -115,18 +115,18 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 // rows it would add a dependent DRAM round trip before a fire-and-forget RED.
 template <int PH>
 __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_min(wmark_ptr(T, g, row), x.tag, x.filter && hot);
+  if (PH == PH_EXEC) mark_unit(T, MK_W, g, row, x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_WRITE, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_min(amark_ptr(T, g, row), x.tag, x.filter && hot);
+  if (PH == PH_EXEC) mark_unit(T, MK_A, g, row, x.tag, x.filter && hot);
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_ADD, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
   if (g == LTPG_STATIC) return;
-  if (PH == PH_EXEC && T.rmarks) mark_min(rmark_ptr(T, g, row), x.tag, x.filter && hot);  // NEXT-1 minR
+  if (PH == PH_EXEC && T.rmarks) mark_unit(T, MK_R, g, row, x.tag, x.filter && hot);  // NEXT-1 minR
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_READ, x.r, x.epoch);
 }
 // update of column c (strict: WRITE unit of its group; delayed: ADD unit)
@@ -695,10 +695,10 @@ __global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
       // bucket q + 1 (clamped): q < t  <=>  bucket <= t
       const long long bq = q[u] + 1 < 0 ? 0 : (q[u] + 1 > SL_T ? SL_T : q[u] + 1);
       atomicAdd(hist + bq, 1u);
-      if (reorder && TSt.rmarks) mark_min(rmark_ptr(TSt, gq, rows[u]), rtag, true);  // NEXT-1 minR
+      if (reorder && TSt.rmarks) mark_unit(TSt, MK_R, gq, rows[u], rtag, true);  // NEXT-1 minR
     }
     if (lane == 0 && reorder && TDi.rmarks)
-      mark_min(rmark_ptr(TDi, col_group(TDi, D_NEXT_O_ID), row_d), rtag, true);
+      mark_unit(TDi, MK_R, col_group(TDi, D_NEXT_O_ID), row_d, rtag, true);
     __syncwarp();
     // low[t] = sum of hist[0..t]: 9 buckets per lane, then a warp scan of the lane sums
     constexpr uint32_t PER = (SL_T + 31) / 32;
@@ -1217,6 +1217,7 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
   note_launch(3);
+  if (t.h_tab) launch_bucket_reduce(t.h_tab, t.n_tab, s);  // NEXT-3 large-sized buckets (if any)
   if (ev) cudaEventRecord(ev[3], s);
   cudaEventRecord(t.fork[1], s);
   cudaStreamWaitEvent(t.side, t.fork[1], 0);

@@ -80,6 +80,12 @@ struct DevTable {
   // of P:217 on a dense key range -- and skips the hash-slot access.  Result-invisible (R6).
   uint64_t key_base, dense_n;
   uint32_t* aux;                  // TPC-C ORDER: first ORDER_LINE row of the order (ROW_NONE: probe)
+  // NEXT-3 large-sized hash buckets (LTPG_FLAG_LARGE_BUCKETS): a popular table
+  // (E = T/D > 1) records each mark in sub-slot (rank mod su) of its unit's bucket of su =
+  // ceil(E/32)*32 sub-slots; k_bucket_reduce folds every bucket into the unit's mark word
+  // before detection.  su <= 1: standard-sized (one slot per unit).
+  mark_t* sub[3];                 // [MK_W / MK_A / MK_R][units of that kind][su]
+  uint32_t su;
 };
 
 // table lookup honouring the dense mapping: dmask = *dense_live & ~(tables with INSERT/DELETE
@@ -140,6 +146,22 @@ __device__ __forceinline__ mark_t* amark_ptr(const DevTable& T, uint32_t g, uint
 }
 __device__ __forceinline__ mark_t* rmark_ptr(const DevTable& T, uint32_t g, uint32_t row) {
   return T.rmarks + ((uint64_t)g * T.capacity + row);
+}
+
+// recordTID into a unit's mark of kind k (write / add / read).  Standard-sized bucket: the
+// mark word itself.  Large-sized bucket (NEXT-3): sub-slot h = TID mod s_u of the
+// unit's bucket -- threads of different ranks mostly hit different words, so their atomics no
+// longer serialise; k_bucket_reduce then takes the minimum over the bucket ("reads out
+// all the TIDs in the hash bucket and selects ... the smallest TID").  Result-identical.
+enum { MK_W = 0, MK_A = 1, MK_R = 2 };
+__device__ __forceinline__ void mark_unit(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag,
+                                          bool filter) {
+  mark_t* p = k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
+  if (T.su > 1) {
+    const mark_t* base = k == MK_W ? T.wmarks : (k == MK_A ? T.amarks : T.rmarks);
+    p = T.sub[k] + (uint64_t)(p - base) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
+  }
+  mark_min(p, tag, filter);
 }
 
 __device__ __forceinline__ long long* col_ptr(const DevTable& T, uint32_t c, uint32_t row) {
@@ -370,6 +392,9 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
                     uint32_t* n_out2, cudaStream_t s);
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
+// NEXT-3: fold the large-sized buckets of every popular table into their units' mark words
+// (host copies of the tables; nothing is launched when no table has su > 1)
+void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s);
 void launch_build_index_tail(uint32_t t, const unsigned long long* from, uint32_t* err, cudaStream_t s);
 void launch_note_rows(uint32_t t, unsigned long long* dst, cudaStream_t s);
 void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,

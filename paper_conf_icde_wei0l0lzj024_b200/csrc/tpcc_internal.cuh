@@ -56,6 +56,8 @@ struct TpccDev {
   SlScratch sl;
   cudaStream_t side = nullptr;  // StockLevel phases run here, concurrently with the others
   cudaEvent_t fork[2]{}, join[2]{};
+  const DevTable* h_tab = nullptr; // host table copies (NEXT-3 bucket reduce between exec and detect)
+  uint32_t n_tab = 0;
 };
 
 struct TpccParams {
