@@ -596,6 +596,8 @@ def main():
             "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)
                               for k in ("ms_upload", "ms_group", "ms_exec", "ms_detect", "ms_writeback",
                                         "ms_download")}}
+    if args.flags:
+        line["config"]["flags"] = args.flags
     if shared:
         line["config"]["devices"] = ("%d ranks on %d GPU(s): functional check of the multi-rank path, "
                                      "not a scaling number" % (world, ndev))
