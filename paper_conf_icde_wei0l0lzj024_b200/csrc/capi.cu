@@ -47,7 +47,8 @@ struct Nccl {
 };
 Nccl g_nccl;
 
-uint64_t g_tab_versions = 0;     // process-wide: every table load gets a new version
+uint64_t g_tab_versions = 0;
+constexpr uint64_t LARGE_BUCKET_BYTES = 64ull << 20;  // NEXT-3 bucket memory cap per table     // process-wide: every table load gets a new version
 uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __constant__
 
 // per-partition scratch (one per logical partition handled by this process)
@@ -488,16 +489,23 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
       CK(cudaMemset(T.rmarks, 0xFF, cap * d->n_groups * sizeof(mark_t)));
     }
     // NEXT-3: a popular table -- E = T/D > 1 with T bounded by the batch capacity
-    // and D the loaded rows -- gets large-sized buckets of su = ceil(E/32)*32 sub-slots per unit
+    // and D the loaded rows -- gets large-sized buckets of su = ceil(E/32)*32 sub-slots for each
+    // unit of its loaded rows (appended rows keep standard slots).  Buckets are only for
+    // "limited" popular data: a table whose buckets would exceed LARGE_BUCKET_BYTES
+    // stays standard-sized.
     const double E = (double)db->cfg.max_txns / (double)std::max<uint64_t>(n_rows, 1);
-    if ((db->cfg.flags & LTPG_FLAG_LARGE_BUCKETS) && E > 1.0) {
-      T.su = (uint32_t)std::min<double>(std::ceil(E / 32.0) * 32.0, 1u << 20);
-      const uint64_t units[3] = {cap * d->n_groups, cap * __builtin_popcount(T.add_groups),
-                                 T.rmarks ? cap * d->n_groups : 0};
-      for (int k = 0; k < 3; ++k) {
-        if (!units[k]) continue;
-        CK(dmalloc(&T.sub[k], units[k] * T.su));
-        CK(cudaMemset(T.sub[k], 0xFF, units[k] * T.su * sizeof(mark_t)));
+    const uint32_t na = __builtin_popcount(T.add_groups);
+    if ((db->cfg.flags & LTPG_FLAG_LARGE_BUCKETS) && E > 1.0 && n_rows) {
+      const uint64_t su = (uint64_t)std::ceil(E / 32.0) * 32;
+      const uint64_t units[3] = {n_rows * d->n_groups, n_rows * na, T.rmarks ? n_rows * d->n_groups : 0};
+      if ((units[0] + units[1] + units[2]) * su * sizeof(mark_t) <= LARGE_BUCKET_BYTES) {
+        T.su = (uint32_t)su;
+        T.sub_rows = (uint32_t)n_rows;
+        for (int k = 0; k < 3; ++k) {
+          if (!units[k]) continue;
+          CK(dmalloc(&T.sub[k], units[k] * su));
+          CK(cudaMemset(T.sub[k], 0xFF, units[k] * su * sizeof(mark_t)));
+        }
       }
     }
   }
@@ -719,8 +727,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       if (T.wmarks) CK(cudaMemsetAsync(T.wmarks, 0xFF, units, s));
       if (T.rmarks) CK(cudaMemsetAsync(T.rmarks, 0xFF, units, s));
       if (T.amarks) CK(cudaMemsetAsync(T.amarks, 0xFF, T.capacity * __builtin_popcount(T.add_groups) * sizeof(mark_t), s));
-      const uint64_t su_units[3] = {T.capacity * T.n_groups, T.capacity * __builtin_popcount(T.add_groups),
-                                    T.capacity * T.n_groups};
+      const uint64_t su_units[3] = {(uint64_t)T.sub_rows * T.n_groups,
+                                    (uint64_t)T.sub_rows * __builtin_popcount(T.add_groups),
+                                    (uint64_t)T.sub_rows * T.n_groups};
       for (int k = 0; k < 3; ++k)
         if (T.sub[k]) CK(cudaMemsetAsync(T.sub[k], 0xFF, su_units[k] * T.su * sizeof(mark_t), s));
     }

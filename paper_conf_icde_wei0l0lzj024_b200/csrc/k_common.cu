@@ -209,26 +209,24 @@ void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uin
 }
 
 // ---- NEXT-3: large-sized bucket -> unit mark (min over the bucket's su sub-slots) ----------
-// One block per (unit, chunk of 1024 sub-slots); the chunk minima meet in the unit's word with
-// atomicMin.  Older epochs carry larger tag bytes, so a stale word or sub-slot never hides a
-// mark of this batch, and mark_rank ignores it when nothing of this batch is there.
-__global__ void __launch_bounds__(256) k_bucket_reduce(const mark_t* __restrict__ sub, mark_t* word, uint64_t units,
-                                                       uint32_t su) {
-  __shared__ mark_t wmin[8];
+// One warp per (unit, chunk of 1024 sub-slots) -- each lane reads 32 sub-slots, coalesced --
+// and the chunk minima meet in the unit's word with atomicMin.  Older epochs carry larger tag
+// bytes, so a stale word or sub-slot never hides a mark of this batch, and mark_rank ignores
+// it when nothing of this batch is there.  Bucket (gi, row) belongs to word gi*capacity + row.
+__global__ void __launch_bounds__(256) k_bucket_reduce(const mark_t* __restrict__ sub, mark_t* word, uint32_t groups,
+                                                       uint32_t rows, uint64_t capacity, uint32_t su) {
   const uint32_t per = (su + 1023) / 1024;
-  for (uint64_t c = blockIdx.x; c < units * per; c += gridDim.x) {
+  const uint64_t units = (uint64_t)groups * rows;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  for (uint64_t c = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); c < units * per; c += nwarps) {
     const uint64_t u = c / per;
     const uint32_t j0 = (uint32_t)(c % per) * 1024u;
+    const uint32_t j1 = min(su, j0 + 1024u);
     mark_t m = 0xFFFFFFFFu;
-    for (uint32_t j = j0 + threadIdx.x; j < su && j < j0 + 1024u; j += blockDim.x) m = min(m, sub[u * su + j]);
+    for (uint32_t j = j0 + lane; j < j1; j += 32) m = min(m, __ldcg(sub + u * su + j));
     m = __reduce_min_sync(0xffffffffu, m);
-    if ((threadIdx.x & 31) == 0) wmin[threadIdx.x >> 5] = m;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      for (int w = 1; w < 8; ++w) m = min(m, wmin[w]);
-      if (m != 0xFFFFFFFFu) atomicMin(word + u, m);
-    }
-    __syncthreads();
+    if (lane == 0 && m != 0xFFFFFFFFu) atomicMin(word + (u / rows) * capacity + u % rows, m);
   }
 }
 
@@ -238,13 +236,12 @@ void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t
     if (T.su <= 1) continue;
     const mark_t* sub[3] = {T.sub[0], T.sub[1], T.sub[2]};
     mark_t* word[3] = {T.wmarks, T.amarks, T.rmarks};
-    const uint64_t units[3] = {(uint64_t)T.n_groups * T.capacity,
-                               (uint64_t)__builtin_popcount(T.add_groups) * T.capacity,
-                               (uint64_t)T.n_groups * T.capacity};
+    const uint32_t groups[3] = {T.n_groups, (uint32_t)__builtin_popcount(T.add_groups), T.n_groups};
     for (int k = 0; k < 3; ++k) {
-      if (!sub[k] || !word[k] || !units[k]) continue;
-      const uint64_t chunks = units[k] * ((T.su + 1023) / 1024);
-      k_bucket_reduce<<<(unsigned)std::min<uint64_t>(chunks, 148 * 8), 256, 0, s>>>(sub[k], word[k], units[k], T.su);
+      if (!sub[k] || !word[k] || !groups[k] || !T.sub_rows) continue;
+      const uint64_t warps = (uint64_t)groups[k] * T.sub_rows * ((T.su + 1023) / 1024);
+      const unsigned blocks = (unsigned)std::min<uint64_t>((warps + 7) / 8, 148 * 8);
+      k_bucket_reduce<<<blocks, 256, 0, s>>>(sub[k], word[k], groups[k], T.sub_rows, T.capacity, T.su);
       note_launch();
     }
   }

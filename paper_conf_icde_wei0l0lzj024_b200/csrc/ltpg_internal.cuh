@@ -84,8 +84,9 @@ struct DevTable {
   // (E = T/D > 1) records each mark in sub-slot (rank mod su) of its unit's bucket of su =
   // ceil(E/32)*32 sub-slots; k_bucket_reduce folds every bucket into the unit's mark word
   // before detection.  su <= 1: standard-sized (one slot per unit).
-  mark_t* sub[3];                 // [MK_W / MK_A / MK_R][units of that kind][su]
+  mark_t* sub[3];                 // [MK_W / MK_A / MK_R][group of that kind][sub_rows][su]
   uint32_t su;
+  uint32_t sub_rows;              // rows with buckets (the rows loaded; appended rows: standard)
 };
 
 // table lookup honouring the dense mapping: dmask = *dense_live & ~(tables with INSERT/DELETE
@@ -156,10 +157,12 @@ __device__ __forceinline__ mark_t* rmark_ptr(const DevTable& T, uint32_t g, uint
 enum { MK_W = 0, MK_A = 1, MK_R = 2 };
 __device__ __forceinline__ void mark_unit(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag,
                                           bool filter) {
-  mark_t* p = k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
-  if (T.su > 1) {
-    const mark_t* base = k == MK_W ? T.wmarks : (k == MK_A ? T.amarks : T.rmarks);
-    p = T.sub[k] + (uint64_t)(p - base) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
+  mark_t* p;
+  if (T.su > 1 && row < T.sub_rows) {
+    const uint32_t gi = k == MK_A ? __popc(T.add_groups & ((1u << g) - 1u)) : g;
+    p = T.sub[k] + ((uint64_t)gi * T.sub_rows + row) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
+  } else {
+    p = k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
   }
   mark_min(p, tag, filter);
 }
