@@ -849,10 +849,24 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = r - lane;
   uint8_t* sw = stage[wib];
+  // only the used prefix of each block is read (include/ltpg.h layouts): the first 16 bytes of
+  // every block, then NewOrder's line records -- a Payment costs one sector instead of four
+  uint32_t need = 0;
+  if (r < b.n_txns) {
+    const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r);
+    uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * lane);
+    d[0] = v.x;
+    d[1] = v.y;
+    d[2] = v.z;
+    d[3] = v.w;
+    const uint32_t ty = b.ptype[r], nl = (v.x >> 24) & 0xFFu;
+    need = ty == 0 ? 8 + 8 * min(nl, 15u) : (ty == 1 ? 24u : 16u);
+  }
 #pragma unroll
   for (uint32_t k = 0; k < 8; ++k) {
-    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB
-    if (r0 + c / 8 < b.n_txns) {
+    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB: txn c / 8, part c % 8
+    const uint32_t nj = __shfl_sync(0xffffffffu, need, c / 8);
+    if ((c % 8) && 16 * (c % 8) < nj) {
       const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r0 + 16 * c);
       uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * (c / 8) + 16 * (c % 8));
       d[0] = v.x;
@@ -979,35 +993,98 @@ __global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
 
 // ---- NewOrder o_id: fetch-ADD pre-image = snapshot D_NEXT_O_ID + #committed NewOrders of the
 //      same district with a smaller rank (P:241 prefix sum; R12) -------------------------------
-__global__ void k_no_prep(BatchDev b, TpccParams tp) {
-  if (*b.err) return;
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= b.n_txns) return;
-  const uint8_t* p = b.params + 128ull * r;
-  const bool c = b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT && owns_w(b, p16(p, 0));
-  tp.no_pref[r] = c ? ((unsigned long long)p[3] << 32 | 1ull) : 0ull;
-  tp.dk_of[r] = c ? (uint32_t)kD(p16(p, 0), p[2]) : ~0u;
-}
-
-__global__ void k_no_hist(BatchDev b, TpccParams tp) {
+// One block per NO_CHUNK ranks (4 consecutive ranks per thread): committed NewOrders of this
+// partition -> their district histogram (chunk_cnt), the in-chunk exclusive prefix of
+// (lines << 32 | 1) in rank order (no_pref; k_no_assign adds the chunk's base) and the chunk
+// total (chunk_tot; scanned by the last block of k_no_colscan).
+__global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
   extern __shared__ uint32_t hist[];
+  __shared__ unsigned long long wsum[8];
   if (*b.err) return;
   for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) hist[i] = 0;
   __syncthreads();
-  const uint32_t r0 = blockIdx.x * NO_CHUNK;
-  for (uint32_t i = threadIdx.x; i < NO_CHUNK; i += blockDim.x) {
-    const uint32_t r = r0 + i;
-    if (r < b.n_txns) {
-      const uint32_t dk = tp.dk_of[r];
-      if (dk != ~0u) atomicAdd(hist + dk, 1u);
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t r0 = blockIdx.x * NO_CHUNK + 4 * threadIdx.x;
+  unsigned long long v[4], tsum = 0;
+  uint32_t dk[4];
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j) {
+    const uint32_t r = r0 + j;
+    bool c = r < b.n_txns && b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT;
+    uint32_t hdr = 0;
+    if (c) {
+      hdr = *reinterpret_cast<const uint32_t*>(b.params + 128ull * r);  // u16 w | u8 d | u8 n_lines
+      c = owns_w(b, hdr & 0xFFFFu);
     }
+    v[j] = c ? ((unsigned long long)(hdr >> 24) << 32 | 1ull) : 0ull;
+    dk[j] = c ? (uint32_t)kD(hdr & 0xFFFFu, (hdr >> 16) & 0xFFu) : ~0u;
+    if (c) atomicAdd(hist + dk[j], 1u);
+    tsum += v[j];
   }
+  unsigned long long x = tsum;  // block-wide exclusive scan of the per-thread sums, rank order
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  if (lane == 31) wsum[wib] = x;
+  __syncthreads();
+  unsigned long long before = 0, total = 0;
+#pragma unroll
+  for (uint32_t w = 0; w < 8; ++w) {
+    if (w < wib) before += wsum[w];
+    total += wsum[w];
+  }
+  unsigned long long ex = before + x - tsum;
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j) {
+    const uint32_t r = r0 + j;
+    if (r < b.n_txns) {
+      tp.no_pref[r] = ex;
+      tp.dk_of[r] = dk[j];
+    }
+    ex += v[j];
+  }
+  if (threadIdx.x == 0) tp.chunk_tot[blockIdx.x] = total;
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i] = hist[i];
 }
 
+// chunk totals -> exclusive chunk bases (in place) and the batch total in no_pref[n]
+__device__ void chunk_total_scan(const BatchDev& b, const TpccParams& tp) {
+  __shared__ unsigned long long wsum[8];
+  const uint32_t nc = tp.n_chunks, per = (nc + blockDim.x - 1) / blockDim.x;
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t c0 = threadIdx.x * per;
+  unsigned long long tsum = 0;
+  for (uint32_t c = c0; c < c0 + per && c < nc; ++c) tsum += tp.chunk_tot[c];
+  unsigned long long x = tsum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  if (lane == 31) wsum[wib] = x;
+  __syncthreads();
+  unsigned long long ex = x - tsum, total = 0;
+  for (uint32_t w = 0; w < (blockDim.x >> 5); ++w) {
+    if (w < wib) ex += wsum[w];
+    total += wsum[w];
+  }
+  for (uint32_t c = c0; c < c0 + per && c < nc; ++c) {
+    const unsigned long long t = tp.chunk_tot[c];
+    tp.chunk_tot[c] = ex;
+    ex += t;
+  }
+  if (threadIdx.x == 0) tp.no_pref[b.n_txns] = total;
+}
+
 __global__ void k_no_colscan(BatchDev b, TpccParams tp) {  // one warp per district key
   if (*b.err) return;
+  if (blockIdx.x == gridDim.x - 1) {  // the extra last block: chunk bases
+    chunk_total_scan(b, tp);
+    return;
+  }
   const uint32_t dk = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
@@ -1056,6 +1133,7 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
   const uint32_t lane = threadIdx.x;
   for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i];
   const uint32_t r0 = blockIdx.x * NO_CHUNK;
+  const unsigned long long cbase = tp.chunk_tot[blockIdx.x];
   uint32_t dks[NO_CHUNK / 32];
 #pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {  // all of the chunk's loads in flight first
@@ -1072,6 +1150,7 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
     if (dk != ~0u) {
       const uint32_t before = __popc(m & ((1u << lane) - 1));
       b.res[4ull * r] = tp.dist_base[dk] + cntd[dk] + before;
+      tp.no_pref[r] += cbase;  // append positions: chunk base + in-chunk prefix
     }
     __syncwarp();
     if (dk != ~0u && lane == (uint32_t)(__ffs(m) - 1)) cntd[dk] += __popc(m);
@@ -1131,7 +1210,8 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
   else if (dm(&t.by_name, (uint64_t)t.dsz * 1000)) return LTPG_ENOMEM;
   if (dm(&t.list, (uint64_t)NTYPES * max_txns) || dm(&t.clist, (uint64_t)NTYPES * max_txns) ||
       dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_pref, max_txns + 1ull) ||
-      dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16))
+      dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16) ||
+      dm(&t.chunk_tot, chunks + 1))
     return LTPG_ENOMEM;
   SlScratch& sl = t.sl;
   if (dm(&sl.minr, t.dsz) || dm(&sl.slot, t.dsz) || dm(&sl.dk, t.dsz) || dm(&sl.cnt, 1) ||
@@ -1154,7 +1234,7 @@ void tpcc_free(TpccDev& t) {
     if (t.join[k]) cudaEventDestroy(t.join[k]);
   }
   if (!t.owns_by_name) t.by_name = nullptr;
-  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc,
+  void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.chunk_tot,
                 t.sl.minr, t.sl.slot, t.sl.dk, t.sl.cnt, t.sl.low, t.sl.nx, t.sl.rows, t.sl.nd, t.sl.rowd, t.sl.m};
   for (void* p : ps)
     if (p) cudaFree(p);
@@ -1188,7 +1268,7 @@ static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists)
   const uint32_t n = b.n_txns;
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
-                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK};
+                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -1231,18 +1311,17 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
 }
 
 int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
+  (void)scan_scratch;  // the o_id prefix scans inside k_no_chunk / k_no_colscan
   const uint32_t n = b.n_txns;
   const TpccParams tp = params_of(t, b, false);
   // committed txns re-listed per type: write-back warps only visit committed txns
   k_tpcc_relist<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   note_launch();
-  // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders
-  k_no_prep<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
-  note_launch();
-  scan_exclusive_u64(t.no_pref, t.no_pref, n, scan_scratch, s);  // row and line offsets at once
+  // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders: per-chunk
+  // histograms + in-chunk prefixes, column scans (+ chunk bases), assignment in rank order
   const size_t smem = (size_t)t.dsz * sizeof(uint32_t);
-  k_no_hist<<<tp.n_chunks, 256, smem, s>>>(b, tp);
-  k_no_colscan<<<(t.dsz + 7) / 8, 256, 0, s>>>(b, tp);
+  k_no_chunk<<<tp.n_chunks, 256, smem, s>>>(b, tp);
+  k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
   k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));
