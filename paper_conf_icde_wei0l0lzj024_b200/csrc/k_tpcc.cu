@@ -849,24 +849,10 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = r - lane;
   uint8_t* sw = stage[wib];
-  // only the used prefix of each block is read (include/ltpg.h layouts): the first 16 bytes of
-  // every block, then NewOrder's line records -- a Payment costs one sector instead of four
-  uint32_t need = 0;
-  if (r < b.n_txns) {
-    const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r);
-    uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * lane);
-    d[0] = v.x;
-    d[1] = v.y;
-    d[2] = v.z;
-    d[3] = v.w;
-    const uint32_t ty = b.ptype[r], nl = (v.x >> 24) & 0xFFu;
-    need = ty == 0 ? 8 + 8 * min(nl, 15u) : (ty == 1 ? 24u : 16u);
-  }
 #pragma unroll
   for (uint32_t k = 0; k < 8; ++k) {
-    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB: txn c / 8, part c % 8
-    const uint32_t nj = __shfl_sync(0xffffffffu, need, c / 8);
-    if ((c % 8) && 16 * (c % 8) < nj) {
+    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB
+    if (r0 + c / 8 < b.n_txns) {
       const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r0 + 16 * c);
       uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * (c / 8) + 16 * (c % 8));
       d[0] = v.x;
