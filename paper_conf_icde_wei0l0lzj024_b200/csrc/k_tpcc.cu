@@ -287,8 +287,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const DevTable& TOr = c_tabs[TO];
       const DevTable& TOL_ = c_tabs[TOL];
       const DevTable& TNw = c_tabs[TNO];
+      // append position: chunk base + in-chunk prefix of committed NewOrders (k_no_chunk)
+      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
       if (active && sub < n) {  // ORDER_LINE row
-        const uint32_t row = (uint32_t)(*TOL_.n_rows + (tp.no_pref[r] >> 32) + sub);
+        const uint32_t row = (uint32_t)(*TOL_.n_rows + (pref >> 32) + sub);
         wr(TOL_, OL_I_ID, row, i);
         wr(TOL_, OL_SUPPLY_W_ID, row, sw);
         wr(TOL_, OL_QUANTITY, row, qty);
@@ -298,8 +300,8 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         TOL_.valid[row] = 1;
       }
       if (sub == 15) {  // ORDER and NEW_ORDER rows
-        const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)tp.no_pref[r]);
-        if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + (tp.no_pref[r] >> 32));  // contiguous lines
+        const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)pref);
+        if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + (pref >> 32));  // contiguous lines
         wr(TOr, O_C_ID, orow, c);
         wr(TOr, O_ENTRY_D, orow, b.clock);
         wr(TOr, O_OL_CNT, orow, n);
@@ -309,7 +311,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         TOr.valid[orow] = 1;
         IdxSlot* sl = idx_find_or_insert(TOr, okey);
         if (sl) sl->row = orow; else internal_error(x);
-        const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)tp.no_pref[r]);
+        const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)pref);
         wr(TNw, NO_O_ID, nrow, o);
         TNw.rowkey[nrow] = okey;
         TNw.valid[nrow] = 1;
@@ -981,7 +983,7 @@ __global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
 //      same district with a smaller rank (P:241 prefix sum; R12) -------------------------------
 // One block per NO_CHUNK ranks (4 consecutive ranks per thread): committed NewOrders of this
 // partition -> their district histogram (chunk_cnt), the in-chunk exclusive prefix of
-// (lines << 32 | 1) in rank order (no_pref; k_no_assign adds the chunk's base) and the chunk
+// (lines << 32 | 1) in rank order (no_pref; write-back adds the chunk base) and the chunk
 // total (chunk_tot; scanned by the last block of k_no_colscan).
 __global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
   extern __shared__ uint32_t hist[];
@@ -1119,7 +1121,6 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
   const uint32_t lane = threadIdx.x;
   for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i];
   const uint32_t r0 = blockIdx.x * NO_CHUNK;
-  const unsigned long long cbase = tp.chunk_tot[blockIdx.x];
   uint32_t dks[NO_CHUNK / 32];
 #pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {  // all of the chunk's loads in flight first
@@ -1136,7 +1137,6 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
     if (dk != ~0u) {
       const uint32_t before = __popc(m & ((1u << lane) - 1));
       b.res[4ull * r] = tp.dist_base[dk] + cntd[dk] + before;
-      tp.no_pref[r] += cbase;  // append positions: chunk base + in-chunk prefix
     }
     __syncwarp();
     if (dk != ~0u && lane == (uint32_t)(__ffs(m) - 1)) cntd[dk] += __popc(m);
