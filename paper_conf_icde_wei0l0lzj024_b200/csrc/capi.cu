@@ -128,6 +128,8 @@ struct ltpg_db {
   cudaStream_t fin = nullptr;
   cudaEvent_t status_ready = nullptr, fin_done = nullptr;
   uint32_t* d_scan_fin = nullptr;
+  unsigned long long* d_fc_state = nullptr;  // a8 look-back tile states; [0] of d_fc_ctr: tile counter
+  uint32_t* d_fc_ctr = nullptr;
   ncclComm_t comm = nullptr;
   // peer-memory exchange (world > 1 without LTPG_FLAG_NCCL_EXCHANGE; xchg.cuh)
   bool p2p = false, connected = false;
@@ -317,6 +319,9 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaEventCreateWithFlags(&db->status_ready, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&db->fin_done, cudaEventDisableTiming));
   CK(dmalloc(&db->d_scan_fin, scan_scratch_words(n) + 16));
+  CK(dmalloc(&db->d_fc_state, (n + 1023) / 1024 + 1));
+  CK(cudaMemset(db->d_fc_state, 0, ((n + 1023) / 1024 + 1) * sizeof(unsigned long long)));
+  CK(dmalloc(&db->d_fc_ctr, 1));
   CK(cudaMemcpy(db->d_tab, db->h_tab, sizeof(db->h_tab), cudaMemcpyHostToDevice));
   db->parts.resize(loop);
   std::vector<void*> ptrs(3 * 64, nullptr);
@@ -384,6 +389,8 @@ void ltpg_destroy_db(ltpg_db* db) {
   if (db->status_ready) cudaEventDestroy(db->status_ready);
   if (db->fin_done) cudaEventDestroy(db->fin_done);
   if (db->d_scan_fin) cudaFree(db->d_scan_fin);
+  if (db->d_fc_state) cudaFree(db->d_fc_state);
+  if (db->d_fc_ctr) cudaFree(db->d_fc_ctr);
   for (Part& P : db->parts) {
     void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.small, P.base};
     for (void* p : pb)
@@ -841,10 +848,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     // ---- a8 on the finalize stream: commit bitmask, counts, abort list (status is final) ------
     CK(cudaEventRecord(db->status_ready, s));
     CK(cudaStreamWaitEvent(db->fin, db->status_ready, 0));
-    launch_finalize(st_out, n, bits_out, S.d_flags, counts, S.d_small, db->fin);
-    scan_exclusive_u32(S.d_flags, S.d_offs, n, db->d_scan_fin, db->fin);
-    launch_compact(S.d_flags, S.d_offs, n, abort_out, S.d_small + 16, S.host_out ? nullptr : res->n_aborted,
-                   db->fin);
+    launch_finalize_compact(st_out, n, bits_out, counts, S.d_small, abort_out, S.d_small + 16,
+                            S.host_out ? nullptr : res->n_aborted, db->d_fc_state, db->d_fc_ctr, db->epoch, db->fin);
     CK(cudaEventRecord(db->fin_done, db->fin));
     // ---- a7: write-back per partition -------------------------------------------------------
     for (uint32_t p = 0; p < L; ++p) {

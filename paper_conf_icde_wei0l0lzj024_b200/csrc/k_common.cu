@@ -161,6 +161,110 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
   note_launch();
 }
 
+// a8 in one pass: commit bitmask, per-status counts and the abort list (ascending ranks) with
+// a decoupled look-back scan over 1024-txn tiles.  Tile ids come from a counter (reset per
+// batch), so every tile a block waits for belongs to a block that is already running.  Tile
+// state word: [63:32] batch epoch | [31:30] 1 = aggregate, 2 = inclusive prefix | [29:0] value.
+constexpr uint32_t FC_TILE = 1024;
+__global__ void __launch_bounds__(256) k_finalize_compact(const uint8_t* __restrict__ status, uint32_t n,
+                                                          uint32_t* __restrict__ commit_bits, uint32_t* counts,
+                                                          const uint32_t* err, uint32_t* __restrict__ out,
+                                                          uint32_t* n_out, uint32_t* n_out2,
+                                                          unsigned long long* tile_state, uint32_t* tile_ctr,
+                                                          uint32_t epoch) {
+  __shared__ uint32_t tile_s, wsum[8], red[3], base_s;
+  (void)err;  // no early exit: write-back may raise the error word concurrently, and a block
+              // that skipped its tile would leave its successors waiting forever
+  if (threadIdx.x == 0) tile_s = atomicAdd(tile_ctr, 1u);
+  if (threadIdx.x < 3) red[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t tile = tile_s, lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t r0 = tile * FC_TILE + 4 * threadIdx.x;
+  uint8_t st[4];
+  if (r0 + 3 < n) {
+    const uchar4 v = *reinterpret_cast<const uchar4*>(status + r0);
+    st[0] = v.x, st[1] = v.y, st[2] = v.z, st[3] = v.w;
+  } else {
+#pragma unroll
+    for (uint32_t j = 0; j < 4; ++j) st[j] = r0 + j < n ? status[r0 + j] : 0xFF;
+  }
+  uint32_t nib = 0, nc = 0, nu = 0;
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j) {
+    nib |= (st[j] == LTPG_ST_COMMIT ? 1u : 0u) << j;
+    nc += st[j] == LTPG_ST_CONFLICT;
+    nu += st[j] == LTPG_ST_USER_ABORT;
+  }
+  // commit bits: 8 lanes (32 txns) per word
+  uint32_t word = nib << (4 * (lane & 7));
+  word |= __shfl_xor_sync(0xffffffffu, word, 1);
+  word |= __shfl_xor_sync(0xffffffffu, word, 2);
+  word |= __shfl_xor_sync(0xffffffffu, word, 4);
+  if ((lane & 7) == 0 && r0 < n) commit_bits[r0 >> 5] = word;
+  // block-wide exclusive scan of the per-thread conflict counts (rank order)
+  uint32_t x = nc;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  const uint32_t ncw = __reduce_add_sync(0xffffffffu, nc), nuw = __reduce_add_sync(0xffffffffu, nu);
+  const uint32_t nbw = __reduce_add_sync(0xffffffffu, __popc(nib));
+  if (lane == 31) wsum[wib] = x;
+  if (lane == 0) {
+    atomicAdd(red + 0, nbw);
+    atomicAdd(red + 1, ncw);
+    atomicAdd(red + 2, nuw);
+  }
+  __syncthreads();
+  uint32_t before = 0, agg = 0;
+#pragma unroll
+  for (uint32_t w = 0; w < 8; ++w) {
+    if (w < wib) before += wsum[w];
+    agg += wsum[w];
+  }
+  if (threadIdx.x < 3 && red[threadIdx.x]) atomicAdd(counts + threadIdx.x, red[threadIdx.x]);
+  if (threadIdx.x == 0) {  // decoupled look-back
+    const unsigned long long tag = (unsigned long long)epoch << 32;
+    volatile unsigned long long* vs = tile_state;
+    uint32_t base = 0;
+    if (tile == 0) {
+      vs[0] = tag | (2ull << 30) | agg;
+    } else {
+      vs[tile] = tag | (1ull << 30) | agg;
+      for (int64_t j = (int64_t)tile - 1; j >= 0;) {
+        const unsigned long long v = vs[j];
+        const uint32_t fl = (v >> 32) == epoch ? (uint32_t)(v >> 30) & 3u : 0u;
+        if (!fl) continue;  // predecessor not published yet
+        base += (uint32_t)v & 0x3FFFFFFFu;
+        if (fl == 2) break;
+        --j;
+      }
+      vs[tile] = tag | (2ull << 30) | (base + agg);
+    }
+    base_s = base;
+    if ((tile + 1) * FC_TILE >= n) {  // the last tile knows the total
+      *n_out = base + agg;
+      if (n_out2) *n_out2 = base + agg;
+    }
+  }
+  __syncthreads();
+  uint32_t o = base_s + before + x - nc;
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j)
+    if (st[j] == LTPG_ST_CONFLICT) out[o++] = r0 + j;
+}
+
+void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* counts,
+                             const uint32_t* err, uint32_t* out, uint32_t* n_out, uint32_t* n_out2,
+                             unsigned long long* tile_state, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t s) {
+  if (!n) return;
+  cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), s);
+  k_finalize_compact<<<(n + FC_TILE - 1) / FC_TILE, 256, 0, s>>>(status, n, commit_bits, counts, err, out, n_out,
+                                                                 n_out2, tile_state, tile_ctr, epoch);
+  note_launch();
+}
+
 // packed TPC-C parameter blocks -> fixed 128-byte blocks (zero-filled tails); one warp per
 // 8 txns, 16-byte lanes
 __global__ void k_unpack_params(const uint8_t* __restrict__ packed, const uint32_t* __restrict__ offs, uint32_t n,

@@ -395,6 +395,11 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
                     uint32_t* n_out2, cudaStream_t s);
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
+// a8 in one kernel: commit bitmask, counts, abort list (decoupled look-back over 1024-txn tiles;
+// tile_state[ceil(n/1024)] persists across batches, tile_ctr is reset on `s`)
+void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* counts,
+                             const uint32_t* err, uint32_t* out, uint32_t* n_out, uint32_t* n_out2,
+                             unsigned long long* tile_state, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t s);
 // NEXT-3: fold the large-sized buckets of every popular table into their units' mark words
 // (host copies of the tables; nothing is launched when no table has su > 1)
 void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s);
