@@ -803,13 +803,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (fused) {  // validate + warp-local division + execute; INSERTs after their claims
           launch_ops_fused(db->n_tables, x, filter, s);
           if (evp) CK(cudaEventRecord(evp[2], s));  // ms_group = the fused kernel; ms_exec = INSERT tail
-          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
+          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
           launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
           launch_ops_claim(x, s);
           launch_ops_exec_inserts(x, filter, s);
         } else {
           launch_ops_validate_group(db->n_tables, x, grouped, s);
-          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s);
+          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
           launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
           launch_ops_claim(x, s);
           if (evp) CK(cudaEventRecord(evp[2], s));

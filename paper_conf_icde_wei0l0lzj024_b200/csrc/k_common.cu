@@ -44,7 +44,8 @@ __device__ __forceinline__ T block_excl_scan(T v, T& total) {
 }
 
 template <class T>
-__global__ void k_scan_reduce(const T* __restrict__ in, uint32_t n, T* __restrict__ sums) {
+__global__ void k_scan_reduce(const T* __restrict__ in, uint32_t n, T* __restrict__ sums, const uint32_t* skip) {
+  if (skip && !*skip) return;
   const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE;
   T s = 0;
 #pragma unroll
@@ -59,7 +60,8 @@ __global__ void k_scan_reduce(const T* __restrict__ in, uint32_t n, T* __restric
 
 // single block: exclusive scan of the block sums (nb <= SCAN_TILE); sums[nb] = total
 template <class T>
-__global__ void k_scan_top(T* sums, uint32_t nb) {
+__global__ void k_scan_top(T* sums, uint32_t nb, const uint32_t* skip) {
+  if (skip && !*skip) return;
   T v[SCAN_ITEMS];
   T s = 0;
 #pragma unroll
@@ -81,7 +83,11 @@ __global__ void k_scan_top(T* sums, uint32_t nb) {
 
 template <class T>
 __global__ void k_scan_down(const T* __restrict__ in, T* __restrict__ out, uint32_t n,
-                            const T* __restrict__ sums, uint32_t nb) {
+                            const T* __restrict__ sums, uint32_t nb, const uint32_t* skip) {
+  if (skip && !*skip) {  // every input is zero (in-place scan): only the total is missing
+    if (blockIdx.x == 0 && threadIdx.x == 0) out[n] = 0;
+    return;
+  }
   // each thread owns SCAN_ITEMS consecutive elements of the tile (stable order)
   const uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE + (uint64_t)threadIdx.x * SCAN_ITEMS;
   T v[SCAN_ITEMS];
@@ -108,21 +114,23 @@ size_t scan_scratch_words(uint32_t n) { return 2 * ((n + SCAN_TILE - 1) / SCAN_T
 // out[0..n) = exclusive prefix sums of in, out[n] = total.  Deterministic.  scratch holds
 // scan_scratch_words(n) u32 words (enough for 64-bit sums).
 template <class T>
-static void scan_exclusive(const T* in, T* out, uint32_t n, void* scratch_v, cudaStream_t s) {
+static void scan_exclusive(const T* in, T* out, uint32_t n, void* scratch_v, cudaStream_t s,
+                           const uint32_t* skip = nullptr) {
   T* scratch = static_cast<T*>(scratch_v);
   if (n == 0) {
     cudaMemsetAsync(out, 0, sizeof(T), s);
     return;
   }
   uint32_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;  // <= SCAN_TILE blocks (n <= 16.7M)
-  k_scan_reduce<T><<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch);
-  k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>(scratch, nb);
-  k_scan_down<T><<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb);
+  k_scan_reduce<T><<<nb, SCAN_THREADS, 0, s>>>(in, n, scratch, skip);
+  k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>(scratch, nb, skip);
+  k_scan_down<T><<<nb, SCAN_THREADS, 0, s>>>(in, out, n, scratch, nb, skip);
   note_launch(3);
 }
 
-void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s) {
-  scan_exclusive<uint32_t>(in, out, n, scratch, s);
+void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s,
+                        const uint32_t* skip_if_zero) {
+  scan_exclusive<uint32_t>(in, out, n, scratch, s, skip_if_zero);
 }
 void scan_exclusive_u64(const unsigned long long* in, unsigned long long* out, uint32_t n, uint32_t* scratch,
                         cudaStream_t s) {

@@ -371,7 +371,9 @@ __device__ __forceinline__ bool owns_w(const BatchDev& b, uint32_t w) {
 }
 
 
-void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s);
+// skip_if_zero (in-place scans only): when *skip_if_zero == 0 every input is 0, only out[n] = 0 is written
+void scan_exclusive_u32(const uint32_t* in, uint32_t* out, uint32_t n, uint32_t* scratch, cudaStream_t s,
+                        const uint32_t* skip_if_zero = nullptr);
 void scan_exclusive_u64(const unsigned long long* in, unsigned long long* out, uint32_t n, uint32_t* scratch,
                         cudaStream_t s);
 size_t scan_scratch_words(uint32_t n);
