@@ -578,7 +578,7 @@ def main():
         ms = statistics.mean(exec_ms)
         ach = bytes_exec / (ms / 1000.0) / 1e9
         roof = {"bound": "hbm", "kernel": "k_tpcc_phase<PH_EXEC>", "achieved": ach, "peak": peak, "unit": "GB/s",
-                "frac": ach / peak, "traffic": ncu_traffic(name, "k_tpcc_phase<0>"), "peak_source": peak_kind,
+                "frac": ach / peak, "traffic": ncu_traffic(name, "k_tpcc_phase<0,"), "peak_source": peak_kind,
                 "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
                 "kernel_share_of_step": ms / statistics.mean(step_ms)}
 

@@ -168,18 +168,30 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   uint32_t* log = tp.log + (uint64_t)r * TLOG;
   if (PH == PH_DETECT && b.nparts <= 1) {
     // unpartitioned detection needs no parameters: execute logged every line slot (ROW_NONE
-    // when unused) and the district row
+    // when unused) and the district row.  One thread per NewOrder (lanes_of): its 16 log
+    // words and then all of its mark words are loaded together -- 32 txns per warp with every
+    // load of a txn in flight, instead of 2 txns per warp and a dependent chain per unit
     if (!active) return;
-    const uint32_t row = log[sub];
-    if (row == ROW_NONE) return;
-    const DevTable& TSt = c_tabs[TS];
-    if (sub < 15) {  // same units as the general path below
-      const uint32_t gq = col_group(TSt, S_QUANTITY);
-      unit_w<PH>(TSt, gq, row, x);
-      if (col_group(TSt, S_YTD) != gq) col_upd3<PH>(TSt, S_YTD, S_ORDER_CNT, S_REMOTE_CNT, row, x);
-    } else {
-      unit_a<PH>(c_tabs[TD], col_group(c_tabs[TD], D_NEXT_O_ID), row, x, true);
+    (void)sub;
+    uint32_t rows[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) rows[k] = log[k];
+    const uint32_t gq = col_group(TSt, S_QUANTITY), gy = col_group(TSt, S_YTD);
+    const uint32_t go = col_group(TSt, S_ORDER_CNT), gr = col_group(TSt, S_REMOTE_CNT);
+    const uint32_t ay = col_is_add(TSt, S_YTD) ? ACC_ADD : ACC_WRITE;
+    const uint32_t ao = col_is_add(TSt, S_ORDER_CNT) ? ACC_ADD : ACC_WRITE;
+    const uint32_t ar = col_is_add(TSt, S_REMOTE_CNT) ? ACC_ADD : ACC_WRITE;
+    uint32_t bits = 0;
+#pragma unroll
+    for (int k = 0; k < 15; ++k) {  // same units as the general path below (unit_w / col_upd3)
+      if (rows[k] == ROW_NONE) continue;
+      bits |= unit_bits(TSt, gq, rows[k], ACC_WRITE, x.r, x.epoch);
+      if (gy != gq) bits |= unit_bits(TSt, gy, rows[k], ay, x.r, x.epoch);
+      if (go != gq && go != gy) bits |= unit_bits(TSt, go, rows[k], ao, x.r, x.epoch);
+      if (gr != gq && gr != gy && gr != go) bits |= unit_bits(TSt, gr, rows[k], ar, x.r, x.epoch);
     }
+    if (rows[15] != ROW_NONE) bits |= unit_bits(TDi, col_group(TDi, D_NEXT_O_ID), rows[15], ACC_ADD, x.r, x.epoch);
+    x.bits |= bits;
     return;
   }
   uint32_t w = 0, d = 0, n = 0, c = 0;
@@ -783,11 +795,25 @@ __global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScr
 // TMASK: procedure types this launch runs.  StockLevel (32 lanes, 26 KB of shared memory per
 // block, many registers) runs in its own launch so it does not cap the occupancy of the
 // others -- each type group gets its own launch configuration.
-constexpr uint32_t TM_MAIN = 0x0Fu;  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
+constexpr uint32_t TM_MAIN = 0x0Fu;
+// lanes per txn of a procedure type: Payment 1, StockLevel 32, others 16 -- NewOrder detection
+// of an unpartitioned batch 1 (all of a txn's units from one thread, see proc_neworder)
+__device__ __forceinline__ uint32_t lanes_of(uint32_t t, int PH, uint32_t nparts) {
+  return t == 1 ? 1u : (t == 4 ? 32u : ((t == 0 && PH == PH_DETECT && nparts <= 1) ? 1u : 16u));
+}  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
 template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
 // loads (params -> log -> marks) and gains most from occupancy (measured: 8 -> 32 regs)
-__global__ void __launch_bounds__(256, (PH == PH_EXEC ? 4 : PH == PH_DETECT ? 8 : 6))
+#ifndef LTPG_EXEC_MINB
+#define LTPG_EXEC_MINB 4
+#endif
+#ifndef LTPG_DETECT_MINB
+#define LTPG_DETECT_MINB 8
+#endif
+#ifndef LTPG_WB_MINB
+#define LTPG_WB_MINB 6
+#endif
+__global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
     k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
@@ -798,7 +824,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? 4 : PH == PH_DETECT ? 8 
 #pragma unroll
   for (int t = 0; t < NTYPES; ++t) {
     cnt[t] = ((TMASK >> t) & 1u) ? tp.counts[t] : 0u;
-    const uint32_t per = 32 / (t == 1 ? 1 : (t == 4 ? 32 : 16));
+    const uint32_t per = 32 / lanes_of(t, PH, b.nparts);
     pre[t + 1] = pre[t] + (cnt[t] + per - 1) / per;
   }
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
@@ -807,7 +833,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? 4 : PH == PH_DETECT ? 8 
 #pragma unroll
     for (int tt = 1; tt < NTYPES; ++tt)
       if (w >= pre[tt]) { t = tt; lw = w - pre[tt]; ct = cnt[tt]; }  // warp-uniform procedure type
-    const uint32_t L = t == 1 ? 1 : (t == 4 ? 32 : 16);
+    const uint32_t L = lanes_of(t, PH, b.nparts);
     const uint32_t per = 32 / L;
     const uint32_t k = lw * per + lane / L;
     const uint32_t sub = lane % L;
