@@ -166,7 +166,20 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
   const DevTable& TSt = c_tabs[TS];
   const uint8_t* p = b.params + 128ull * r;
   uint32_t* log = tp.log + (uint64_t)r * TLOG;
-  if (PH == PH_DETECT && b.nparts <= 1 && !x.reorder) {
+  if (PH == PH_DETECT && b.nparts <= 1 && x.reorder) {  // 16 lanes, one logged slot each
+    if (!active) return;
+    const uint32_t row = log[sub];
+    if (row == ROW_NONE) return;
+    if (sub < 15) {  // same units as the general path below
+      const uint32_t gq = col_group(TSt, S_QUANTITY);
+      unit_w<PH>(TSt, gq, row, x);
+      if (col_group(TSt, S_YTD) != gq) col_upd3<PH>(TSt, S_YTD, S_ORDER_CNT, S_REMOTE_CNT, row, x);
+    } else {
+      unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row, x, true);
+    }
+    return;
+  }
+  if (PH == PH_DETECT && b.nparts <= 1) {
     // unpartitioned detection needs no parameters: execute logged every line slot (ROW_NONE
     // when unused) and the district row.  4 lanes per NewOrder (lanes_of), 4 log slots per
     // lane: a lane's log words and then all of their mark words are loaded together -- 8 txns
