@@ -262,9 +262,16 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       if (PH == PH_WB) {
         const long long q = rd(TSt, S_QUANTITY, row_s);
         wr(TSt, S_QUANTITY, row_s, q >= (long long)qty + 10 ? q - qty : q - qty + 91);
-        addv(TSt, S_YTD, row_s, qty);
-        addv(TSt, S_ORDER_CNT, row_s, 1);
-        addv(TSt, S_REMOTE_CNT, row_s, remote);
+        // the counters may be ADD columns (delayed mode), but only NewOrder touches STOCK and
+        // every NewOrder writes the row's S_QUANTITY unit (WAW): this txn is the row's only
+        // committed toucher in the batch, so plain read-modify-writes are exact (no atomics)
+        const auto inc = [&](uint32_t c, long long v) {
+          long long* pc = col_ptr(TSt, c, row_s);
+          *pc = (long long)((unsigned long long)*pc + (unsigned long long)v);
+        };
+        inc(S_YTD, qty);
+        inc(S_ORDER_CNT, 1);
+        inc(S_REMOTE_CNT, remote);
       }
     }
   }
@@ -414,7 +421,13 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     addv(TCu, C_YTD_PAYMENT, row_c, amount);
     addv(TCu, C_PAYMENT_CNT, row_c, 1);
     const DevTable& THi = c_tabs[TH];  // keyless append, no marks
-    const uint32_t row = (uint32_t)(*THi.n_rows + atomicAdd(tp.misc + M_HIST, 1u));
+    // warp-aggregated append: one counter atomic per warp (every committed Payment appends;
+    // per-lane atomics on the single counter serialised), consecutive rows per warp
+    const uint32_t am = __activemask(), lane = threadIdx.x & 31, lead = __ffs(am) - 1;
+    uint32_t hb = 0;
+    if (lane == lead) hb = atomicAdd(tp.misc + M_HIST, (uint32_t)__popc(am));
+    hb = __shfl_sync(am, hb, lead) + __popc(am & ((1u << lane) - 1u));
+    const uint32_t row = (uint32_t)(*THi.n_rows + hb);
     wr(THi, H_C_ID, row, cid);
     wr(THi, H_C_D_ID, row, cd);
     wr(THi, H_C_W_ID, row, cw);
