@@ -136,7 +136,8 @@ struct ltpg_db {
   XLayout xl;
   XPeers xpeers{};
   char* xregion = nullptr;
-  uint32_t* d_xdone = nullptr;
+  uint32_t* d_xdone = nullptr;              // [0] k_xput, [1] k_xrs block counters
+  long long* d_xsink = nullptr;             // all-gather target when the caller wants no reads
   std::vector<void*> opened;  // peer regions mapped with cudaIpcOpenMemHandle
 };
 
@@ -349,8 +350,9 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     db->xl.init(cfg->max_txns, nres, (uint32_t)cfg->world);
     CK(cudaMalloc(reinterpret_cast<void**>(&db->xregion), db->xl.bytes));
     CK(cudaMemset(db->xregion, 0, db->xl.bytes));
-    CK(dmalloc(&db->d_xdone, 1));
-    CK(cudaMemset(db->d_xdone, 0, sizeof(uint32_t)));
+    CK(dmalloc(&db->d_xdone, 2));
+    CK(cudaMemset(db->d_xdone, 0, 2 * sizeof(uint32_t)));
+    CK(dmalloc(&db->d_xsink, nres));
     db->xpeers.base[cfg->rank] = db->xregion;
   } else if (cfg->world > 1) {
     if (!g_nccl.load()) return fail(db, LTPG_ENCCL, "libnccl.so.2 not loadable");
@@ -401,6 +403,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   for (void* p : db->opened) cudaIpcCloseMemHandle(p);
   if (db->xregion) cudaFree(db->xregion);
   if (db->d_xdone) cudaFree(db->d_xdone);
+  if (db->d_xsink) cudaFree(db->d_xsink);
   delete db;
 }
 
@@ -863,9 +866,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     }
     if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
-    if (db->p2p) {  // every rank publishes (the protocol needs it); the sum is pulled on demand
+    if (db->p2p) {  // every rank publishes and reduces its slice (the protocol needs it)
       launch_xsig_res(db->xpeers, (uint32_t)db->cfg.rank, (uint32_t)db->cfg.world, db->epoch, s);
-      if (res->reads) launch_xsum(db->xpeers, db->xl, n_reads, db->epoch, res_out, S.d_small, (uint32_t)db->cfg.rank, s);
+      launch_xsum(db->xpeers, db->xl, n_reads, db->epoch, res->reads ? res_out : db->d_xsink, S.d_small,
+                  (uint32_t)db->cfg.rank, db->d_xdone + 1, s);
     } else if (partitioned && res->reads) {
       if (db->cfg.world == 1) {
         k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);

@@ -27,7 +27,7 @@ __device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
 }
 
 __device__ __forceinline__ uint64_t* sig_ptr(char* region, uint32_t par, uint32_t kind, uint32_t src) {
-  return reinterpret_cast<uint64_t*>(region) + (par * 2 + kind) * 64 + src;
+  return reinterpret_cast<uint64_t*>(region) + (par * NSIG + kind) * 64 + src;
 }
 __device__ __forceinline__ uint4* board_ptr(char* region, const XLayout& L, uint32_t par, uint32_t src) {
   return reinterpret_cast<uint4*>(region + L.off_board) + ((uint64_t)par * L.world + src) * L.nwords;
@@ -126,20 +126,54 @@ __global__ void k_xsig_res(XPeers peers, uint32_t rank, uint32_t world, uint32_t
   if (threadIdx.x < world) st_release_sys(sig_ptr(peers.base[threadIdx.x], par, 1, rank), (uint64_t)epoch << 3);
 }
 
-__global__ void __launch_bounds__(256) k_xsum(XPeers peers, XLayout L, uint64_t n, uint32_t epoch, long long* out,
-                                              uint32_t* err, uint32_t rank) {
+// slice q of the slot array (rank q sums it): [q*S, min((q+1)*S, n)), S = ceil(n / world)
+__device__ __forceinline__ void slice_of(uint64_t n, uint32_t world, uint32_t q, uint64_t& lo, uint64_t& hi) {
+  const uint64_t S = (n + world - 1) / world;
+  lo = min(n, (uint64_t)q * S);
+  hi = min(n, lo + S);
+}
+
+// reduce-scatter: rsum[i] = sum over ranks of res[i] for i in this rank's slice; the last block
+// to finish raises kind 2 in every region
+__global__ void __launch_bounds__(256) k_xrs(XPeers peers, XLayout L, uint64_t n, uint32_t epoch, uint32_t* err,
+                                             uint32_t rank, uint32_t* done) {
   const uint32_t par = epoch & 1u;
-  if (!wait_all(peers.base[rank], par, 1, L.world, epoch, 3, nullptr, err)) {
+  const bool ok = wait_all(peers.base[rank], par, 1, L.world, epoch, 3, nullptr, err);
+  if (ok) {
+    const uint64_t off = L.off_res + (uint64_t)par * L.nres * sizeof(long long);
+    long long* rsum = reinterpret_cast<long long*>(peers.base[rank] + L.off_rsum) + (uint64_t)par * L.nres;
+    uint64_t lo, hi;
+    slice_of(n, L.world, rank, lo, hi);
+    for (uint64_t i = lo + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < hi; i += (uint64_t)gridDim.x * blockDim.x) {
+      unsigned long long s = 0;
+      for (uint32_t q = 0; q < L.world; ++q)
+        s += (unsigned long long)__ldcg(reinterpret_cast<const long long*>(peers.base[q] + off) + i);
+      rsum[i] = (long long)s;
+    }
+  } else if (threadIdx.x == 0) {
+    atomicOr(err, ERR_EINTERNAL);
+  }
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0 && atomicAdd(done, 1u) == gridDim.x - 1) {  // every block's sums are fenced
+    __threadfence_system();
+    for (uint32_t q = 0; q < L.world; ++q) st_release_sys(sig_ptr(peers.base[q], par, 2, rank), (uint64_t)epoch << 3);
+    *done = 0;
+  }
+}
+
+// all-gather: out[i] = rsum of slice owner(i), pulled from the owner's region
+__global__ void __launch_bounds__(256) k_xag(XPeers peers, XLayout L, uint64_t n, uint32_t epoch, long long* out,
+                                             uint32_t* err, uint32_t rank) {
+  const uint32_t par = epoch & 1u;
+  if (!wait_all(peers.base[rank], par, 2, L.world, epoch, 3, nullptr, err)) {
     if (threadIdx.x == 0) atomicOr(err, ERR_EINTERNAL);
     return;
   }
-  const uint64_t off = L.off_res + (uint64_t)par * L.nres * sizeof(long long);
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    unsigned long long s = 0;
-    for (uint32_t q = 0; q < L.world; ++q)
-      s += (unsigned long long)__ldcg(reinterpret_cast<const long long*>(peers.base[q] + off) + i);
-    out[i] = (long long)s;
-  }
+  const uint64_t S = (n + L.world - 1) / L.world;
+  const uint64_t off = L.off_rsum + (uint64_t)par * L.nres * sizeof(long long);
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = __ldcg(reinterpret_cast<const long long*>(peers.base[i / S] + off) + i);
 }
 
 }  // namespace
@@ -164,10 +198,11 @@ void launch_xsig_res(const XPeers& peers, uint32_t rank, uint32_t world, uint32_
 }
 
 void launch_xsum(const XPeers& peers, const XLayout& L, uint64_t n_reads, uint32_t epoch, long long* out,
-                 uint32_t* err, uint32_t rank, cudaStream_t s) {
-  // every block waits for the signals itself, so the grid is kept to one wave
-  k_xsum<<<148 * 4, 256, 0, s>>>(peers, L, n_reads, epoch, out, err, rank);
-  note_launch();
+                 uint32_t* err, uint32_t rank, uint32_t* done, cudaStream_t s) {
+  // every block waits for the signals itself, so the grids are kept to one wave
+  k_xrs<<<148 * 4, 256, 0, s>>>(peers, L, n_reads, epoch, err, rank, done);
+  k_xag<<<148 * 4, 256, 0, s>>>(peers, L, n_reads, epoch, out, err, rank);
+  note_launch(2);
 }
 
 }  // namespace ltpg
