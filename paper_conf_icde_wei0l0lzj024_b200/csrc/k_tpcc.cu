@@ -138,11 +138,11 @@ __device__ __forceinline__ void col_upd(const DevTable& T, uint32_t c, uint32_t 
 // same for columns c1..c3 updated together; a unit shared by several columns is touched once
 template <int PH>
 __device__ __forceinline__ void col_upd3(const DevTable& T, uint32_t c1, uint32_t c2, uint32_t c3, uint32_t row,
-                                         Tx& x) {
+                                         Tx& x, bool hot = false) {
   const uint32_t g1 = col_group(T, c1), g2 = col_group(T, c2), g3 = col_group(T, c3);
-  col_upd<PH>(T, c1, row, x);
-  if (g2 != g1) col_upd<PH>(T, c2, row, x);
-  if (g3 != g1 && g3 != g2) col_upd<PH>(T, c3, row, x);
+  col_upd<PH>(T, c1, row, x, hot);
+  if (g2 != g1) col_upd<PH>(T, c2, row, x, hot);
+  if (g3 != g1 && g3 != g2) col_upd<PH>(T, c3, row, x, hot);
 }
 
 __device__ __forceinline__ long long seg16_sum(long long v) {
@@ -540,12 +540,15 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
         // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
         unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
       } else {
-        for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x);  // DELETE
+        // every Delivery of a warehouse in the batch reads the same cursor and so delivers the
+        // same order: its NEW_ORDER / ORDER / ORDER_LINE / CUSTOMER units are as hot as the
+        // district's (E >> 1) -- marks take the read-before-atomicMin filter
+        for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x, true);  // DELETE
         const uint32_t row_o = probe_finish(TOr, nok, ho_, vo);
         if (row_o == ROW_NONE) {
           internal_error(x);
         } else {
-          unit_w<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x);
+          unit_w<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x, true);
           const uint32_t cid = (uint32_t)rd(TOr, O_C_ID, row_o);
           const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
           long long sum = 0;
@@ -559,14 +562,14 @@ __device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool 
           for (uint32_t l = 0; l < 15; ++l) {
             if (l >= cnt) continue;
             if (row_ol[l] == ROW_NONE) { internal_error(x); continue; }
-            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[l], x);
+            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[l], x, true);
             sum += rd(TOL_, OL_AMOUNT, row_ol[l]);
             if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol[l], b.clock);
           }
           if (row_c == ROW_NONE) {
             internal_error(x);
           } else {
-            col_upd3<PH>(TCu, C_BALANCE, C_DELIVERY_CNT, C_DELIVERY_CNT, row_c, x);
+            col_upd3<PH>(TCu, C_BALANCE, C_DELIVERY_CNT, C_DELIVERY_CNT, row_c, x, true);
             if (PH == PH_WB) {
               addv(TCu, C_BALANCE, row_c, sum);
               addv(TCu, C_DELIVERY_CNT, row_c, 1);
