@@ -511,8 +511,26 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
 }
 
 // ---- Delivery (TPC-C 2.7), one lane per district; rows re-derived in every phase ----------------
+// Shared per warehouse: every Delivery RMWs the cursors of all ten districts of its warehouse
+// (WRITE units), so of a warehouse's Deliveries in a batch only the smallest rank can commit
+// (R1 and NEXT-1: WAW aborts).  They all read the same snapshot -- same cursors, orders, lines
+// and customers -- so they mark the same units, where the smallest rank's mark is the minimum,
+// and return the same results (the carrier is not part of them).  Only that rank (dl_min[w],
+// from k_tpcc_group) executes, marks and is checked; the others copy its result slots and take
+// the WAW verdict.  Result-identical to running each one (oracle parity).
 template <int PH>
-__device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool active, Tx& x) {
+__device__ void proc_delivery(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active,
+                              Tx& x) {
+  if (active) {
+    const uint32_t rmin = tp.dl_min[p16(b.params + 128ull * r, 0)];
+    if (rmin != r) {
+      if (PH == PH_DETECT) {
+        x.bits |= CF_WAW;  // WAW on the district cursors against rank rmin < r
+        if (sub < 4) b.res[4ull * r + sub] = b.res[4ull * rmin + sub];  // written by rmin's execute
+      }
+      return;  // (never committed: no write-back)
+    }
+  }
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TCu = c_tabs[TC];
   const DevTable& TOr = c_tabs[TO];
@@ -877,7 +895,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
       case 0: proc_neworder<PH>(b, tp, r, sub, go, x); break;
       case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
-      case 3: proc_delivery<PH>(b, r, sub, go, x); break;
+      case 3: proc_delivery<PH>(b, tp, r, sub, go, x); break;
       default:
         break;  // StockLevel: shared per district (k_sl_*)
     }
@@ -986,6 +1004,10 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     }
   } else {
     lines = 0;
+  }
+  if (t == 3 && touch) {  // smallest Delivery rank per warehouse (shared Delivery, proc_delivery)
+    uint32_t* m = tp.dl_min + p16(sw + SROW * lane, 0);
+    if (r < *m) atomicMin(m, r);
   }
   // block-aggregated counters and per-type list positions (one atomic per block and list)
   const uint32_t ccnt[3] = {lines, pay_cust, no_home};  // misc[M_NO_LINES], misc[M_PAY], misc[M_NO]
@@ -1253,7 +1275,7 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
   if (dm(&t.list, (uint64_t)NTYPES * max_txns) || dm(&t.clist, (uint64_t)NTYPES * max_txns) ||
       dm(&t.log, (uint64_t)max_txns * TLOG) || dm(&t.no_pref, max_txns + 1ull) ||
       dm(&t.dk_of, max_txns) || dm(&t.chunk_cnt, chunks * t.dsz) || dm(&t.dist_base, t.dsz) || dm(&t.misc, 16) ||
-      dm(&t.chunk_tot, chunks + 1))
+      dm(&t.chunk_tot, chunks + 1) || dm(&t.dl_min, nw + 1ull))
     return LTPG_ENOMEM;
   SlScratch& sl = t.sl;
   if (dm(&sl.minr, t.dsz) || dm(&sl.slot, t.dsz) || dm(&sl.dk, t.dsz) || dm(&sl.cnt, 1) ||
@@ -1277,6 +1299,7 @@ void tpcc_free(TpccDev& t) {
   }
   if (!t.owns_by_name) t.by_name = nullptr;
   void* ps[] = {t.by_name, t.list, t.clist, t.log, t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.chunk_tot,
+                t.dl_min,
                 t.sl.minr, t.sl.slot, t.sl.dk, t.sl.cnt, t.sl.low, t.sl.nx, t.sl.rows, t.sl.nd, t.sl.rowd, t.sl.m};
   for (void* p : ps)
     if (p) cudaFree(p);
@@ -1310,7 +1333,7 @@ static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists)
   const uint32_t n = b.n_txns;
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
-                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot};
+                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -1322,6 +1345,7 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   const uint32_t n = b.n_txns;
   const TpccParams tp = params_of(t, b, false);
   cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
+  cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
   k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   k_tpcc_capacity<<<1, 1, 0, s>>>(b, tp);
   note_launch(2);

@@ -53,6 +53,7 @@ struct TpccDev {
   uint32_t* chunk_cnt = nullptr;// [chunks][dsz]
   long long* dist_base = nullptr; // [dsz] snapshot D_NEXT_O_ID
   unsigned long long* chunk_tot = nullptr;  // [chunks+1] committed NewOrder (lines << 32 | 1) per chunk -> bases
+  uint32_t* dl_min = nullptr;   // [nw+1] smallest Delivery rank per warehouse this batch (~0: none)
   uint32_t* misc = nullptr;     // counters (M_*)
   SlScratch sl;
   cudaStream_t side = nullptr;  // StockLevel phases run here, concurrently with the others
@@ -74,6 +75,7 @@ struct TpccParams {
   const int* by_name;
   uint32_t nw, dsz, max_txns, n_chunks;
   unsigned long long* chunk_tot;
+  uint32_t* dl_min;
 };
 
 int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);
