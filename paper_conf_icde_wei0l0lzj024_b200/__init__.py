@@ -111,6 +111,7 @@ ltpg_wait_batch = _lib.ltpg_wait_batch
 ltpg_peer_handle = _lib.ltpg_peer_handle
 ltpg_connect_peers = _lib.ltpg_connect_peers
 LTPG_BATCH_ASYNC = 1
+LTPG_BATCH_COMPACT_PARAMS = 2
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
             "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers"]
@@ -263,7 +264,8 @@ class Database:
     def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
                  n_txns=None, wait=True):
         """batch: dict(tid u64[n], type u8[n], params u8[n,128]) -- or packed blocks:
-        params = used bytes back to back and offsets u32[n+1] (see pack_params)."""
+        params = used bytes back to back and offsets u32[n+1] (see pack_params), or compact
+        records with compact=True (see pack_params_compact)."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
         offsets = batch.get("offsets")
         n = len(tid) if n_txns is None else n_txns
@@ -272,7 +274,8 @@ class Database:
             device_out = on_dev
         bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
                         proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
-                        stream=c_vp(stream) if stream else None, proc_offsets=_ptr(offsets))
+                        stream=c_vp(stream) if stream else None, proc_offsets=_ptr(offsets),
+                        flags=LTPG_BATCH_COMPACT_PARAMS if batch.get("compact") else 0)
         out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch)
         if wait and not device_out and want_reads:
             out["reads"] = out["reads"].reshape(n, 4)
@@ -308,6 +311,61 @@ def pack_params(types, params):
     np.cumsum(used, out=offs[1:])
     mask = np.arange(128)[None, :] < used[:, None]
     return params[mask], offs.astype(np.uint32)
+
+
+def pack_params_compact(types, params):
+    """Compact TPC-C records (include/ltpg.h LTPG_BATCH_COMPACT_PARAMS): NewOrder lines as u32
+    (item, qty, remote flag) plus the supply warehouses of remote lines, Payment amounts as u32.
+    Client-side encoding (vectorised); returns (packed u8[total], offsets u32[n+1])."""
+    types = np.asarray(types)
+    params = np.ascontiguousarray(params, dtype=np.uint8).reshape(len(types), 128)
+    n = len(types)
+    comp = np.zeros((n, 128), np.uint8)
+    used = np.zeros(n, np.int64)
+    for t, u in _USED.items():  # other types: the used prefix
+        if u is not None and t != 1:
+            m = types == t
+            comp[m, :u] = params[m, :u]
+            used[m] = u
+    no = np.nonzero(types == 0)[0]
+    if len(no):
+        P = params[no]
+        nl = P[:, 3].astype(np.int64)
+        w = P[:, 0].astype(np.uint32) | (P[:, 1].astype(np.uint32) << 8)
+        L = P[:, 8:128].reshape(len(no), 15, 8)
+        item = L[:, :, :4].copy().view(np.uint32)[:, :, 0]
+        sw = L[:, :, 4:6].copy().view(np.uint16)[:, :, 0].astype(np.uint32)
+        qty = L[:, :, 6].astype(np.uint32)
+        live = np.arange(15)[None, :] < nl[:, None]
+        if (live & ((item >= (1 << 17)) | (qty < 1) | (qty > 16))).any():
+            raise ValueError("NewOrder line not representable compactly (item >= 2^17 or qty outside 1..16)")
+        remote = live & (sw != w[:, None])
+        v = np.where(live, item | ((qty - 1) << 17) | (remote.astype(np.uint32) << 21), 0).astype(np.uint32)
+        C = np.zeros((len(no), 128), np.uint8)
+        C[:, :7] = P[:, :7]
+        nrem = remote.sum(axis=1)
+        C[:, 7] = nrem
+        C[:, 8:68] = v.view(np.uint8).reshape(len(no), 60)
+        # supply warehouses of remote lines at 8 + 4 nl + 2 k (k-th remote line)
+        k = np.cumsum(remote, axis=1) - 1
+        ri, li = np.nonzero(remote)
+        pos = 8 + 4 * nl[ri] + 2 * k[ri, li]
+        C[ri, pos] = (sw[ri, li] & 0xFF).astype(np.uint8)
+        C[ri, pos + 1] = (sw[ri, li] >> 8).astype(np.uint8)
+        comp[no] = C
+        used[no] = 8 + 4 * nl + 2 * nrem
+    pay = np.nonzero(types == 1)[0]
+    if len(pay):
+        amount = params[pay, 16:24].copy().view(np.int64)[:, 0]
+        if ((amount < 0) | (amount >= (1 << 32))).any():
+            raise ValueError("Payment amount not representable compactly (outside [0, 2^32))")
+        comp[pay, :12] = params[pay, :12]
+        comp[pay, 12:16] = amount.astype(np.uint32).view(np.uint8).reshape(len(pay), 4)
+        used[pay] = 16
+    offs = np.zeros(n + 1, np.int64)
+    np.cumsum(used, out=offs[1:])
+    mask = np.arange(128)[None, :] < used[:, None]
+    return comp[mask], offs.astype(np.uint32)
 
 
 class Pending:

@@ -639,6 +639,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     return fail(db, LTPG_EINVAL, "bad OPS batch");
   if (!ops_mode && (!b->proc_type || !b->proc_params || !db->cfg.n_warehouses))
     return fail(db, LTPG_EINVAL, "bad TPCC batch");
+  if ((b->flags & LTPG_BATCH_COMPACT_PARAMS) && (ops_mode || !b->proc_offsets))
+    return fail(db, LTPG_EINVAL, "LTPG_BATCH_COMPACT_PARAMS needs a TPCC batch with proc_offsets");
   if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
   Slot& S = db->slots[db->submitted % 3];
   if (S.pending) return fail(db, LTPG_EINVAL, "three batches already in flight: ltpg_wait_batch first");
@@ -790,7 +792,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> every partition)
     const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
     const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
-    launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
+    if (b->flags & LTPG_BATCH_COMPACT_PARAMS)
+      launch_unpack_compact(packed, offs, bd.ptype, n, S.d_params, pb[0].err, s);
+    else
+      launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
     for (uint32_t p = 1; p < L; ++p) {
       k_copy_err<<<1, 1, 0, s>>>(pb[0].err, pb[p].err);
       note_launch();

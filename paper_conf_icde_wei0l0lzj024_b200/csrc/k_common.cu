@@ -301,6 +301,98 @@ void launch_unpack_params(const uint8_t* packed, const uint32_t* offs, uint32_t 
   note_launch();
 }
 
+// LTPG_BATCH_COMPACT_PARAMS (include/ltpg.h): compact TPC-C records -> fixed 128-byte blocks.
+// One warp per 32 txns: the warp's records (contiguous bytes) are staged in shared memory, each
+// lane decodes its own record into a block in shared memory, and the warp stores its 4 KB of
+// blocks with coalesced 16-byte stores.
+constexpr int UC_WARPS = 4;
+__device__ __forceinline__ uint32_t ld_u16(const uint8_t* p) { return (uint32_t)p[0] | (uint32_t)p[1] << 8; }
+__global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t* __restrict__ packed,
+                                                                  const uint32_t* __restrict__ offs,
+                                                                  const uint8_t* __restrict__ types, uint32_t n,
+                                                                  uint8_t* __restrict__ params, uint32_t* err) {
+  __shared__ __align__(16) uint8_t in[UC_WARPS][32 * 128 + 32];
+  __shared__ __align__(16) uint8_t out[UC_WARPS][32 * 128];
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t r0 = (blockIdx.x * UC_WARPS + wib) * 32;
+  if (r0 >= n) return;
+  const uint32_t cnt = min(32u, n - r0);
+  const uint32_t lo = offs[r0], hi = offs[r0 + cnt], end = offs[n];
+  if (hi < lo || hi - lo > 32 * 128 || hi > end) {
+    if (lane == 0) atomicOr(err, ERR_EINVAL);
+    return;
+  }
+  // stage [a0, hi) with 16-byte loads where aligned and inside the buffer, bytes otherwise
+  const uint32_t a0 = lo & ~15u, nch = (hi - a0 + 15) / 16;
+  const bool vec = ((uintptr_t)packed & 15) == 0;
+  for (uint32_t c = lane; c < nch; c += 32) {
+    const uint32_t at = a0 + 16 * c;
+    if (vec && at + 16 <= end) {
+      *reinterpret_cast<uint4*>(in[wib] + 16 * c) = *reinterpret_cast<const uint4*>(packed + at);
+    } else {
+      for (uint32_t k = 0; k < 16; ++k) in[wib][16 * c + k] = at + k < end ? packed[at + k] : 0;
+    }
+  }
+  uint4* ob = reinterpret_cast<uint4*>(out[wib] + 128 * lane);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) ob[k] = make_uint4(0, 0, 0, 0);
+  __syncwarp();
+  bool bad = false;
+  if (lane < cnt) {
+    const uint32_t r = r0 + lane, b0 = offs[r], b1 = offs[r + 1];
+    const uint8_t* q = in[wib] + (b0 - a0);
+    uint8_t* o = out[wib] + 128 * lane;
+    const uint32_t len = b1 - b0;
+    if (b1 < b0 || b0 < lo || b1 > hi || len > 128) {
+      bad = true;
+    } else if (types[r] == 0) {  // NewOrder: 8-byte header, u32 lines, u16 supply warehouses
+      const uint32_t nl = len >= 8 ? q[3] : 0, nrem = len >= 8 ? q[7] : 0;
+      if (len < 8 || nl > 15 || len != 8 + 4 * nl + 2 * nrem) {
+        bad = true;
+      } else {
+        for (int k = 0; k < 7; ++k) o[k] = q[k];
+        const uint32_t w = ld_u16(q);
+        uint32_t k = 0;
+        for (uint32_t l = 0; l < nl; ++l) {
+          const uint8_t* L = q + 8 + 4 * l;
+          const uint32_t v = ld_u16(L) | ld_u16(L + 2) << 16;
+          uint32_t sw = w;
+          if ((v >> 21) & 1u) {
+            if (k < nrem) sw = ld_u16(q + 8 + 4 * nl + 2 * k);
+            ++k;
+          }
+          const uint32_t i = v & 0x1FFFFu;
+          uint8_t* D = o + 8 + 8 * l;
+          D[0] = i & 0xFF, D[1] = (i >> 8) & 0xFF, D[2] = i >> 16, D[3] = 0;
+          D[4] = sw & 0xFF, D[5] = sw >> 8, D[6] = ((v >> 17) & 15u) + 1, D[7] = 0;
+        }
+        if (k != nrem) bad = true;
+      }
+    } else if (types[r] == 1) {  // Payment: 12 header bytes + u32 amount
+      if (len != 16) {
+        bad = true;
+      } else {
+        for (int k = 0; k < 12; ++k) o[k] = q[k];
+        for (int k = 0; k < 4; ++k) o[16 + k] = q[12 + k];  // zero-extended to the i64 at 16
+      }
+    } else {
+      for (uint32_t k = 0; k < len; ++k) o[k] = q[k];
+    }
+  }
+  if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, ERR_EINVAL);
+  __syncwarp();
+  for (uint32_t c = lane; c < cnt * 8; c += 32)
+    *reinterpret_cast<uint4*>(params + 128ull * r0 + 16 * c) = *reinterpret_cast<const uint4*>(out[wib] + 16 * c);
+}
+
+void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const uint8_t* types, uint32_t n,
+                           uint8_t* params, uint32_t* err, cudaStream_t s) {
+  if (!n) return;
+  const uint32_t warps = (n + 31) / 32;
+  k_unpack_compact<<<(warps + UC_WARPS - 1) / UC_WARPS, 32 * UC_WARPS, 0, s>>>(packed, offs, types, n, params, err);
+  note_launch();
+}
+
 // abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
 // abort list (ascending ranks) and its length (n_out[0], and n_out2[0] when not null)
 __global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ offs, uint32_t n,

@@ -397,6 +397,8 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
                     uint32_t* n_out2, cudaStream_t s);
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
+void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const uint8_t* types, uint32_t n,
+                           uint8_t* params, uint32_t* err, cudaStream_t s);
 // a8 in one kernel: commit bitmask, counts, abort list (decoupled look-back over 1024-txn tiles;
 // tile_state[ceil(n/1024)] persists across batches, tile_ctr is reset on `s`)
 void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* counts,

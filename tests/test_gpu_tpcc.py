@@ -195,3 +195,31 @@ def test_stocklevel_shared_per_district_any_threshold():
     assert (st[sl] == ST_COMMIT).any() and (st[sl] == ST_CONFLICT).any()
     compare(g, o, wl.batch(2000, 20000, 2), 4)
     compare_tables(g, o)
+
+
+def test_compact_params_equal_fixed_blocks():
+    """LTPG_BATCH_COMPACT_PARAMS: compact records (u32 NewOrder lines, remote supply lists,
+    u32 Payment amounts) expanded on the GPU give the oracle's results; a record whose length
+    contradicts its header is EINVAL with nothing changed."""
+    lib = L()
+    wl = tpcc.TpccWorkload(3, seed=19, mix=tpcc.MIX_FULL, remote_line_frac=0.25)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=3000, tables=tables, append_batches=4)
+    o = oracle.tpcc_db(wl, tables)
+    for bno in range(3):
+        b = wl.batch(2999, 1 + 3000 * bno, bno)  # ragged: not a multiple of 32
+        packed, offs = lib.pack_params_compact(b["type"], b["params"])
+        pb = {"tid": b["tid"], "type": b["type"], "params": packed, "offsets": offs, "compact": True}
+        out = g.run_tpcc(pb, 2 + bno)
+        rc, st, res = o.run_tpcc(b, 2 + bno)
+        assert (out["status"] == st).all() and (out["reads"] == res).all()
+    compare_tables(g, o)
+    no = int(np.nonzero(b["type"] == 0)[0][0])
+    bad = dict(pb)
+    bad["offsets"] = offs.copy()
+    bad["offsets"][no + 1:] -= 2  # NewOrder record 2 bytes short of its header
+    bad["params"] = np.delete(packed, offs[no + 1] - 1)[: len(packed) - 1]
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(bad, 9)
+    assert e.value.rc == lib.LTPG_EINVAL
+    compare_tables(g, o)  # nothing changed
