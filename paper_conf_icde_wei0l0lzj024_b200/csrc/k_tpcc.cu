@@ -867,20 +867,27 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
+  // NewOrder, Payment), so that the grid's tail is made of short Payment warps (0.088 -> 0.077
+  // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
+  constexpr uint32_t ORD = PH == PH_DETECT ? (2u | 3u << 4 | 0u << 8 | 1u << 12 | 4u << 16)
+                                           : (0u | 1u << 4 | 2u << 8 | 3u << 12 | 4u << 16);  // slot j -> type
   uint32_t cnt[NTYPES], pre[NTYPES + 1];
   pre[0] = 0;
 #pragma unroll
-  for (int t = 0; t < NTYPES; ++t) {
-    cnt[t] = ((TMASK >> t) & 1u) ? tp.counts[t] : 0u;
+  for (int j = 0; j < NTYPES; ++j) {
+    const uint32_t t = (ORD >> (4 * j)) & 15u;
+    cnt[j] = ((TMASK >> t) & 1u) ? tp.counts[t] : 0u;
     const uint32_t per = 32 / lanes_of(t, PH, b.nparts, reorder);
-    pre[t + 1] = pre[t] + (cnt[t] + per - 1) / per;
+    pre[j + 1] = pre[j] + (cnt[j] + per - 1) / per;
   }
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
   for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NTYPES]; w += nwarps) {
-    uint32_t t = 0, lw = w, ct = cnt[0];
+    uint32_t j = 0, lw = w, ct = cnt[0];
 #pragma unroll
-    for (int tt = 1; tt < NTYPES; ++tt)
-      if (w >= pre[tt]) { t = tt; lw = w - pre[tt]; ct = cnt[tt]; }  // warp-uniform procedure type
+    for (int jj = 1; jj < NTYPES; ++jj)
+      if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }  // warp-uniform procedure type
+    const uint32_t t = (ORD >> (4 * j)) & 15u;
     const uint32_t L = lanes_of(t, PH, b.nparts, reorder);
     const uint32_t per = 32 / L;
     const uint32_t k = lw * per + lane / L;
