@@ -1070,6 +1070,9 @@ __global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
 // partition -> their district histogram (chunk_cnt), the in-chunk exclusive prefix of
 // (lines << 32 | 1) in rank order (no_pref; write-back adds the chunk base) and the chunk
 // total (chunk_tot; scanned by the last block of k_no_colscan).
+// RELIST (unpartitioned batches, where every txn touches this partition): also the committed
+// re-list of k_tpcc_relist, from the same status reads.
+template <bool RELIST>
 __global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
   extern __shared__ uint32_t hist[];
   __shared__ unsigned long long wsum[8];
@@ -1079,11 +1082,32 @@ __global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = blockIdx.x * NO_CHUNK + 4 * threadIdx.x;
   unsigned long long v[4], tsum = 0;
-  uint32_t dk[4];
+  uint32_t dk[4], ty[4], cm[4];
 #pragma unroll
   for (uint32_t j = 0; j < 4; ++j) {
     const uint32_t r = r0 + j;
-    bool c = r < b.n_txns && b.ptype[r] == 0 && b.status[r] == LTPG_ST_COMMIT;
+    ty[j] = r < b.n_txns ? b.ptype[r] : 0xFFu;
+    cm[j] = r < b.n_txns && b.status[r] == LTPG_ST_COMMIT;
+  }
+  if (RELIST) {
+    uint32_t cnt[NTYPES], base[NTYPES];
+#pragma unroll
+    for (uint32_t k = 0; k < NTYPES; ++k) cnt[k] = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < 4; ++j)
+#pragma unroll
+      for (uint32_t k = 0; k < NTYPES; ++k) cnt[k] += (cm[j] && ty[j] == k) ? 1u : 0u;
+    block_reserve<NTYPES>(cnt, tp.misc + M_CCOUNT, base);
+#pragma unroll
+    for (uint32_t j = 0; j < 4; ++j)
+#pragma unroll
+      for (uint32_t k = 0; k < NTYPES; ++k)
+        if (cm[j] && ty[j] == k) tp.clist[(uint64_t)k * tp.max_txns + base[k]++] = r0 + j;
+  }
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j) {
+    const uint32_t r = r0 + j;
+    bool c = ty[j] == 0 && cm[j];
     uint32_t hdr = 0;
     if (c) {
       hdr = *reinterpret_cast<const uint32_t*>(b.params + 128ull * r);  // u16 w | u8 d | u8 n_lines
@@ -1387,13 +1411,18 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   (void)scan_scratch;  // the o_id prefix scans inside k_no_chunk / k_no_colscan
   const uint32_t n = b.n_txns;
   const TpccParams tp = params_of(t, b, false);
-  // committed txns re-listed per type: write-back warps only visit committed txns
-  k_tpcc_relist<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
-  note_launch();
-  // fetch-ADD pre-images of D_NEXT_O_ID and append positions of committed NewOrders: per-chunk
-  // histograms + in-chunk prefixes, column scans (+ chunk bases), assignment in rank order
+  // committed txns re-listed per type (write-back warps only visit committed txns) -- inside
+  // k_no_chunk when every txn touches this partition -- and the fetch-ADD pre-images of
+  // D_NEXT_O_ID and append positions of committed NewOrders: per-chunk histograms + in-chunk
+  // prefixes, column scans (+ chunk bases), assignment in rank order
   const size_t smem = (size_t)t.dsz * sizeof(uint32_t);
-  k_no_chunk<<<tp.n_chunks, 256, smem, s>>>(b, tp);
+  if (b.nparts <= 1) {
+    k_no_chunk<true><<<tp.n_chunks, 256, smem, s>>>(b, tp);
+  } else {
+    k_tpcc_relist<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
+    k_no_chunk<false><<<tp.n_chunks, 256, smem, s>>>(b, tp);
+    note_launch();
+  }
   k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
