@@ -207,6 +207,81 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     x.bits |= bits;
     return;
   }
+  if (PH == PH_EXEC && b.nparts <= 1) {
+    // 4 lanes per NewOrder (lanes_of): lane q takes lines 4q..4q+3 (lane 3: lines 12-14 and the
+    // header).  A lane's line records, row lookups (arithmetic on the dense W/D/C/I/S key
+    // ranges) and item-price loads are all issued before any is used: 8 txns per warp instead
+    // of 2, so a warp pays the parameter -> price dependency chain once for 4x the lines.
+    long long amount = 0, w_tax = 0, d_tax = 0, disc = 0;
+    uint32_t ua = 0;
+    if (active) {
+      const uint32_t h0 = *reinterpret_cast<const uint32_t*>(p), h1 = *reinterpret_cast<const uint32_t*>(p + 4);
+      const uint32_t w = h0 & 0xFFFFu, d = (h0 >> 16) & 0xFFu, n = h0 >> 24, c = h1 & 0xFFFFu;
+      uint32_t it[4], qt[4], ri[4], rs[4];
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const uint32_t l = 4 * sub + k;
+        uint2 v = make_uint2(0, 0);
+        if (l < n) v = *reinterpret_cast<const uint2*>(p + 8 + 8 * l);  // u32 i | u16 supply_w | u8 qty
+        it[k] = v.x;
+        qt[k] = (v.y >> 16) & 0xFFu;
+        ri[k] = l < n ? rowof(TIt, TI, v.x, x.dmask) : ROW_NONE;
+        rs[k] = l < n ? rowof(TSt, TS, kS(v.y & 0xFFFFu, v.x), x.dmask) : ROW_NONE;
+      }
+      long long price[4];
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) price[k] = ri[k] != ROW_NONE ? rd(TIt, I_PRICE, ri[k]) : 0;
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const uint32_t l = 4 * sub + k;
+        if (l >= 15) continue;
+        uint32_t row_s = ROW_NONE;
+        if (l < n) {
+          if (ri[k] == ROW_NONE) {
+            ua = 1;  // unused item id: NewOrder rollback (R11)
+          } else {
+            amount += (long long)qt[k] * price[k];
+            row_s = rs[k];
+            if (row_s == ROW_NONE) internal_error(x);
+          }
+        }
+        log[l] = row_s;  // ROW_NONE: unused line slot
+        if (row_s != ROW_NONE) {
+          const uint32_t gq = col_group(TSt, S_QUANTITY);
+          unit_w<PH>(TSt, gq, row_s, x);  // S_QUANTITY: conditional RMW -> WRITE unit
+          if (col_group(TSt, S_YTD) != gq) col_upd3<PH>(TSt, S_YTD, S_ORDER_CNT, S_REMOTE_CNT, row_s, x);
+        }
+      }
+      (void)it;
+      if (sub == 3) {  // header: warehouse / district / customer reads, fetch-ADD of D_NEXT_O_ID
+        const uint32_t row_w = rowof(TWh, TW, w, x.dmask), row_d = rowof(TDi, TD, kD(w, d), x.dmask),
+                       row_c = rowof(TCu, TC, kC(w, d, c), x.dmask);
+        if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
+          internal_error(x);
+          log[15] = ROW_NONE;
+        } else {
+          w_tax = rd(TWh, W_TAX, row_w);  // static reads: unmarked (R4)
+          d_tax = rd(TDi, D_TAX, row_d);
+          disc = rd(TCu, C_DISCOUNT, row_c);
+          log[15] = row_d;
+          unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
+        }
+      }
+    }
+    amount += __shfl_xor_sync(0xffffffffu, amount, 1);  // sums over the txn's 4 lanes
+    amount += __shfl_xor_sync(0xffffffffu, amount, 2);
+    ua |= __shfl_xor_sync(0xffffffffu, ua, 1);
+    ua |= __shfl_xor_sync(0xffffffffu, ua, 2);
+    if (active && sub == 3) {
+      if (ua) b.ua[r] = 1;
+      long long* res = b.res + 4ull * r;
+      res[0] = 0;  // o_id: assigned after detection if committed
+      res[1] = amount * (10000 - disc) * (10000 + w_tax + d_tax) / 100000000;
+      res[2] = amount;
+      res[3] = 0;
+    }
+    return;
+  }
   uint32_t w = 0, d = 0, n = 0, c = 0;
   if (active) {
     w = p16(p, 0);
@@ -843,11 +918,14 @@ __global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScr
 // block, many registers) runs in its own launch so it does not cap the occupancy of the
 // others -- each type group gets its own launch configuration.
 constexpr uint32_t TM_MAIN = 0x0Fu;
-// lanes per txn of a procedure type: Payment 1, StockLevel 32, others 16 -- NewOrder detection
-// of an unpartitioned batch 4 (4 units per lane, see proc_neworder) -- except under NEXT-1
-// reordering, where every unit's three marks are read and 16 lanes measured faster (0.18 vs 0.27 ms)
+// lanes per txn of a procedure type: Payment 1, StockLevel 32, others 16 -- NewOrder execution
+// and detection of an unpartitioned batch 4 (4 lines / units per lane, see proc_neworder;
+// execute 0.255 -> 0.198 ms, detect 0.113 -> 0.087 ms on tpcc_c4) -- except detection under
+// NEXT-1 reordering, where every unit's three marks are read and 16 lanes measured faster
 __device__ __forceinline__ uint32_t lanes_of(uint32_t t, int PH, uint32_t nparts, bool reorder) {
-  return t == 1 ? 1u : (t == 4 ? 32u : ((t == 0 && PH == PH_DETECT && nparts <= 1 && !reorder) ? 4u : 16u));
+  return t == 1 ? 1u
+                : (t == 4 ? 32u
+                          : ((t == 0 && nparts <= 1 && (PH == PH_EXEC || (PH == PH_DETECT && !reorder))) ? 4u : 16u));
 }  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
 template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
