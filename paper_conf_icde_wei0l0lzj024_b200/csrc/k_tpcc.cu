@@ -282,6 +282,95 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     }
     return;
   }
+  if (PH == PH_WB && b.nparts <= 1) {
+    // 4 lanes per committed NewOrder, lane q takes lines q, q+4, q+8, q+12 (the 4 lanes of a txn
+    // write 4 consecutive ORDER_LINE rows per store); a lane's line records, item prices and
+    // stock rows are all loaded before any is used
+    uint32_t remote = 0, w = 0, d = 0, n = 0, c = 0;
+    if (active) {
+      const uint32_t h0 = *reinterpret_cast<const uint32_t*>(p), h1 = *reinterpret_cast<const uint32_t*>(p + 4);
+      w = h0 & 0xFFFFu, d = (h0 >> 16) & 0xFFu, n = h0 >> 24, c = h1 & 0xFFFFu;
+      uint2 v[4];
+      uint32_t rs[4];
+      long long price[4], sq[4];
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const uint32_t l = sub + 4 * k;
+        v[k] = l < n ? *reinterpret_cast<const uint2*>(p + 8 + 8 * l) : make_uint2(0, 0);
+        rs[k] = l < n ? log[l] : ROW_NONE;
+      }
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const uint32_t ri = sub + 4 * k < n ? rowof(TIt, TI, v[k].x, x.dmask) : ROW_NONE;
+        price[k] = ri != ROW_NONE ? rd(TIt, I_PRICE, ri) : 0;  // committed: every item exists
+        sq[k] = rs[k] != ROW_NONE ? rd(TSt, S_QUANTITY, rs[k]) : 0;
+      }
+      const long long o = b.res[4ull * r];
+      const uint64_t okey = kO(w, d, (uint64_t)o);
+      const DevTable& TOL_ = c_tabs[TOL];
+      // append position: chunk base + in-chunk prefix of committed NewOrders (k_no_chunk)
+      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const uint32_t l = sub + 4 * k;
+        if (l >= n) continue;
+        const uint32_t i = v[k].x, sw = v[k].y & 0xFFFFu, qty = (v[k].y >> 16) & 0xFFu;
+        const uint32_t rem = sw != w;
+        remote |= rem;
+        const uint32_t row_s = rs[k];
+        if (row_s != ROW_NONE) {
+          const long long q = sq[k];
+          wr(TSt, S_QUANTITY, row_s, q >= (long long)qty + 10 ? q - qty : q - qty + 91);
+          // the counters may be ADD columns (delayed mode), but only NewOrder touches STOCK and
+          // every NewOrder writes the row's S_QUANTITY unit (WAW): this txn is the row's only
+          // committed toucher in the batch, so plain read-modify-writes are exact (no atomics)
+          const auto inc = [&](uint32_t cc, long long dv) {
+            long long* pc = col_ptr(TSt, cc, row_s);
+            *pc = (long long)((unsigned long long)*pc + (unsigned long long)dv);
+          };
+          inc(S_YTD, qty);
+          inc(S_ORDER_CNT, 1);
+          inc(S_REMOTE_CNT, rem);
+        }
+        const uint32_t row = (uint32_t)(*TOL_.n_rows + (pref >> 32) + l);  // ORDER_LINE row
+        wr(TOL_, OL_I_ID, row, i);
+        wr(TOL_, OL_SUPPLY_W_ID, row, sw);
+        wr(TOL_, OL_QUANTITY, row, qty);
+        wr(TOL_, OL_AMOUNT, row, (long long)qty * price[k]);
+        wr(TOL_, OL_DELIVERY_D, row, 0);
+        TOL_.rowkey[row] = okey * 16 + l + 1;  // PK index entry deferred (capi.cu idx_lag)
+        TOL_.valid[row] = 1;
+      }
+    }
+    remote |= __shfl_xor_sync(0xffffffffu, remote, 1);
+    remote |= __shfl_xor_sync(0xffffffffu, remote, 2);
+    if (active && sub == 0) {  // ORDER and NEW_ORDER rows
+      const DevTable& TOr = c_tabs[TO];
+      const DevTable& TOL_ = c_tabs[TOL];
+      const DevTable& TNw = c_tabs[TNO];
+      const long long o = b.res[4ull * r];
+      const uint64_t okey = kO(w, d, (uint64_t)o);
+      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
+      const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)pref);
+      if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + (pref >> 32));  // contiguous lines
+      wr(TOr, O_C_ID, orow, c);
+      wr(TOr, O_ENTRY_D, orow, b.clock);
+      wr(TOr, O_OL_CNT, orow, n);
+      wr(TOr, O_ALL_LOCAL, orow, !remote);
+      wr(TOr, O_CARRIER_ID, orow, 0);
+      TOr.rowkey[orow] = okey;
+      TOr.valid[orow] = 1;
+      IdxSlot* sl = idx_find_or_insert(TOr, okey);
+      if (sl) sl->row = orow; else internal_error(x);
+      const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)pref);
+      wr(TNw, NO_O_ID, nrow, o);
+      TNw.rowkey[nrow] = okey;
+      TNw.valid[nrow] = 1;
+      sl = idx_find_or_insert(TNw, okey);
+      if (sl) sl->row = nrow; else internal_error(x);
+    }
+    return;
+  }
   uint32_t w = 0, d = 0, n = 0, c = 0;
   if (active) {
     w = p16(p, 0);
@@ -925,7 +1014,7 @@ constexpr uint32_t TM_MAIN = 0x0Fu;
 __device__ __forceinline__ uint32_t lanes_of(uint32_t t, int PH, uint32_t nparts, bool reorder) {
   return t == 1 ? 1u
                 : (t == 4 ? 32u
-                          : ((t == 0 && nparts <= 1 && (PH == PH_EXEC || (PH == PH_DETECT && !reorder))) ? 4u : 16u));
+                          : ((t == 0 && nparts <= 1 && (PH != PH_DETECT || !reorder)) ? 4u : 16u));
 }  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
 template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
