@@ -76,6 +76,7 @@ class ClockSampler:
         self.max_mhz = None
         self.source = None
         self.stop = threading.Event()
+        self.ready = threading.Event()  # set at the first sample (or when sampling gave up)
 
     def __enter__(self):
         self.t = threading.Thread(target=self._loop, daemon=True)
@@ -107,6 +108,7 @@ class ClockSampler:
                 except Exception:
                     rb = int(nv.nvmlDeviceGetCurrentClocksThrottleReasons(h))
                 self.samples.append((time.time(), sm, rb))
+                self.ready.set()
                 self.stop.wait(0.002)
             return
         except Exception:
@@ -125,22 +127,30 @@ class ClockSampler:
                     rb = sum(self.REASONS[n] for n, v in zip(names, f[5:9]) if v.lower() == "active")
                     self.max_mhz = float(f[2])
                     self.samples.append((time.time(), float(f[1]), rb))
+                    self.ready.set()
             except Exception:
                 pass
             self.stop.wait(0.05)
+        self.ready.set()
 
     def __exit__(self, *a):
         self.stop.set()
         self.t.join(timeout=6)
+        self.ready.set()
 
     def summary(self):
         inside = [x for x in self.samples if any(t0 <= x[0] <= t1 for t0, t1 in self.windows)]
+        if not inside:  # timed legs shorter than the sampling period: the samples bracketing them
+            for t0, t1 in self.windows:
+                before = [x for x in self.samples if x[0] < t0]
+                after = [x for x in self.samples if x[0] > t1]
+                inside += before[-1:] + after[:1]
         use = inside or self.samples
         reasons = sorted(n for n, bit in self.REASONS.items() if any(x[2] & bit for x in use))
         return {"sm_mhz": statistics.median(x[1] for x in use) if use else None, "sm_max_mhz": self.max_mhz,
                 "reasons": reasons, "samples": len(use), "source": self.source,
-                "window": ("samples inside the timed legs" if inside else
-                           "all samples (warm-up .. e2e): timed legs shorter than one sample")}
+                "window": ("samples inside (or, for legs shorter than the sampling period, "
+                           "bracketing) the timed legs" if inside else "all samples")}
 
 
 def measured_peaks():
@@ -180,6 +190,29 @@ def make_workload(name, rank=0):
     from workloads import tpcc
     mix = tpcc.MIX_FULL if w["mix"] == "full" else tpcc.MIX_NO_PAY
     return tpcc.TpccWorkload(w["W"], seed=seed, mode=w["mode"], mix=mix)
+
+
+def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, nccl_unique_id=None, **kw):
+    """The database exactly as the bench times it (also used by the full-size parity tests):
+    append regions sized for the worst case of one batch plus the appends of `n_batches`
+    batches (every NewOrder / Payment committing; 10.5 lines per NewOrder on average)."""
+    import paper_conf_icde_wei0l0lzj024_b200 as ltpg
+    w = WORKLOADS[name]
+    B = w["batch"]
+    if w.get("reorder"):
+        flags |= ltpg.LTPG_FLAG_REORDER
+    if w["kind"] == "ycsb":  # inserts (YCSB D/E) of every batch
+        return ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=flags, device=device,
+                                  rank=rank, world=world, nccl_unique_id=nccl_unique_id,
+                                  capacity=w["n_rows"] + n_batches * B * w["ops"] // 10 + 1024, **kw)
+    from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
+    tabs = wl.initial_tables()
+    no, pay = B * wl.mix[0], B * wl.mix[1]
+    cap = {T_ORDER: no * (1 + n_batches), T_NEW_ORDER: no * (1 + n_batches),
+           T_ORDER_LINE: 15 * no + 10.5 * no * n_batches, T_HISTORY: pay * (1 + n_batches)}
+    cap = {t: int(tabs[t][1].shape[1] + v) + 1024 for t, v in cap.items()}
+    return ltpg.tpcc_database(wl, max_txns=B, tables=tabs, capacity=cap, flags=flags, device=device,
+                              rank=rank, world=world, nccl_unique_id=nccl_unique_id, **kw)
 
 
 def exec_algorithmic_bytes(batch):
@@ -366,6 +399,9 @@ def main():
     shared = world > ndev
     local = local % ndev
     torch.cuda.set_device(local)
+    clk = ClockSampler(local)  # samples through load, warm-up, timed and e2e legs
+    if not os.environ.get("LTPG_NO_CLOCKS"):
+        clk.__enter__()
     dist = None
     if world > 1:
         import torch.distributed as dist
@@ -388,24 +424,8 @@ def main():
         from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id
         uid = nccl_unique_id()
     t0 = time.time()
-    if w["kind"] == "ycsb":
-        nb = args.warmup + 2 * args.steps + 2  # inserts (YCSB D/E) of every batch this run makes
-        db = ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=args.flags, device=local,
-                                rank=rank, world=world, nccl_unique_id=uid,
-                                capacity=w["n_rows"] + nb * B * w["ops"] // 10 + 1024)
-    else:
-        # append regions: the worst case of one batch (checked before execution) plus the
-        # appends of every batch this run makes (every NewOrder / Payment committing; 10.5 lines
-        # per NewOrder on average)
-        from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
-        tabs = wl.initial_tables()
-        nb = args.warmup + 2 * args.steps + 2
-        no, pay = B * wl.mix[0], B * wl.mix[1]
-        cap = {T_ORDER: no * (1 + nb), T_NEW_ORDER: no * (1 + nb),
-               T_ORDER_LINE: 15 * no + 10.5 * no * nb, T_HISTORY: pay * (1 + nb)}
-        cap = {t: int(tabs[t][1].shape[1] + v) + 1024 for t, v in cap.items()}
-        db = ltpg.tpcc_database(wl, max_txns=B, tables=tabs, capacity=cap, flags=args.flags, device=local,
-                                rank=rank, world=world, nccl_unique_id=uid)
+    db = open_database(name, wl, args.warmup + 2 * args.steps + 2, flags=args.flags, device=local,
+                       rank=rank, world=world, nccl_unique_id=uid)
     log("rank %d: db loaded in %.1fs" % (rank, time.time() - t0))
 
     # distinct input batches, cycled (inputs only; every step recomputes everything)
@@ -464,9 +484,8 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
     clock = 2
-    clk = ClockSampler(local)  # samples through warm-up, timed and e2e legs
     if not os.environ.get("LTPG_NO_CLOCKS"):
-        clk.__enter__()
+        clk.ready.wait(30)  # NVML init on a fresh box can take seconds
     for s in range(args.warmup):
         i = s % n_distinct
         run(dev_batches[i], host_batches[i], clock, True, False)
