@@ -135,6 +135,9 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
                                               record marks in large-sized buckets of
                                               ceil(E/32)*32 sub-slots (TID mod s_u), folded per
                                               unit before detection; result-identical          */
+#define LTPG_FLAG_GRAPH         (1u << 6)  /* run each batch's device work as a captured CUDA graph,
+                                              replayed for later batches of the same shape
+                                              (see ltpg_run_batch); result-identical          */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
 
 typedef struct {
@@ -264,7 +267,13 @@ typedef struct {
 } ltpg_result;
 
 /* Run one batch; synchronous on batch->stream (returns when results are in place)
- * unless batch->flags has LTPG_BATCH_ASYNC. */
+ * unless batch->flags has LTPG_BATCH_ASYNC.
+ * With LTPG_FLAG_GRAPH a single-process db (world == 1) runs a batch's device work (a2..a8:
+ * every kernel, memset and intra-batch stream fork/join) as one CUDA graph: the first batch of
+ * a shape is captured and instantiated (slow: ~0.1-2 ms of host time), later batches of the same
+ * shape (n_txns, n_ops, input/output pointers when on the device, flags) replay it; epoch and
+ * clock reach the kernels through device memory.  Up to four shapes are kept per pipeline
+ * slot.  Results are identical either way. */
 LTPG_API int ltpg_run_batch(ltpg_db* db, const ltpg_batch* batch, ltpg_result* result);
 
 /* Complete an asynchronously submitted batch (see LTPG_BATCH_ASYNC). */

@@ -37,6 +37,7 @@ LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_UNFUSED = 1 << 3
 LTPG_FLAG_NCCL_EXCHANGE = 1 << 4
 LTPG_FLAG_LARGE_BUCKETS = 1 << 5
+LTPG_FLAG_GRAPH = 1 << 6
 LTPG_PEER_HANDLE_BYTES = 128
 LTPG_LAYOUT_ROWBLOCK, LTPG_LAYOUT_COLUMNAR = 0, 1
 LTPG_FLAG_LOOPBACK_SHIFT = 8

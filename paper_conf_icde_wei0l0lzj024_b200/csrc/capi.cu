@@ -10,6 +10,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -64,6 +65,23 @@ struct Part {
   TpccDev tpcc;
 };
 
+// What a captured batch graph bakes in: every launch geometry and pointer of the batch's
+// device work.  Two batches with equal keys enqueue identical work except for the BatchVars
+// (epoch, clock), which the graph copies from the slot's pinned host copy when it runs.
+struct GraphKey {
+  uint32_t mode, n, n_ops, bflags, host_out, reads_dev, inputs_dev, packed;
+  uint64_t tab_version;
+  const void* in[7];   // tid, op_begin, ops, args, ptype, params, offsets (device inputs only)
+  const void* out[5];  // status, bits, abort, n_aborted, reads
+  bool operator==(const GraphKey& o) const { return std::memcmp(this, &o, sizeof(*this)) == 0; }
+};
+struct GraphEntry {
+  GraphKey key{};
+  cudaGraphExec_t exec = nullptr;
+  uint64_t launches = 0, last_use = 0;
+};
+constexpr int GRAPHS_PER_SLOT = 4;
+
 // one in-flight batch: input staging, device outputs, pinned small results, events
 struct Slot {
   unsigned long long* d_tid = nullptr;
@@ -88,6 +106,10 @@ struct Slot {
   bool pending = false, timing = false, host_out = false;
   ltpg_result* res = nullptr;
   uint64_t launches0 = 0;
+  BatchVars* d_vars = nullptr;             // this batch's epoch / clock (read by the kernels)
+  BatchVars* h_vars = nullptr;             // pinned + mapped host copy (read by graph replays)
+  BatchVars* h_vars_dev = nullptr;         // its device-side address
+  GraphEntry graphs[GRAPHS_PER_SLOT];
 };
 
 }  // namespace
@@ -123,6 +145,8 @@ struct ltpg_db {
   Slot slots[3];
   uint64_t submitted = 0;
   cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaStream_t cap = nullptr;              // batch graphs are captured here (never executes work)
+  uint64_t graph_uses = 0;
   // a8 (commit bitmask, abort list) runs on its own stream once the verdicts are final,
   // concurrently with write-back; it has its own scan scratch
   cudaStream_t fin = nullptr;
@@ -247,6 +271,17 @@ __global__ void k_copy_err(const uint32_t* src, uint32_t* dst) { *dst = *src; }
 __global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint32_t n) {
   if (threadIdx.x < n) host_dst[threadIdx.x] = src[threadIdx.x];
 }
+// batch start: append reservations cleared and the batch scalars stored where the kernels read
+// them -- from the arguments (direct enqueue) or, in a replayed graph, from the slot's pinned
+// host copy through its mapped address (read when the graph runs, not when it was captured)
+__global__ void k_batch_init(unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host,
+                             uint32_t epoch, long long clock) {
+  if (threadIdx.x < MAXT) reserve[threadIdx.x] = 0;
+  if (threadIdx.x == 0) {
+    vars->epoch = host ? host->epoch : epoch;
+    vars->clock = host ? host->clock : clock;
+  }
+}
 __global__ void k_or_err(const uint32_t* src, uint32_t* dst) {
   if (*src) *dst |= *src;
 }
@@ -310,6 +345,9 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(cudaEventCreate(&S.h2d_done));
     CK(cudaEventCreate(&S.comp_done));
     CK(cudaEventCreate(&S.out_done));
+    CK(dmalloc(&S.d_vars, 1));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&S.h_vars), sizeof(BatchVars), cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S.h_vars_dev), S.h_vars, 0));
   }
   CK(dmalloc(&db->d_xchg, 4 * n + 4));
   CK(dmalloc(&db->d_ptrs, 3 * 64));
@@ -317,6 +355,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaStreamCreateWithFlags(&db->h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&db->d2h, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&db->fin, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&db->cap, cudaStreamNonBlocking));
   CK(cudaEventCreateWithFlags(&db->status_ready, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&db->fin_done, cudaEventDisableTiming));
   CK(dmalloc(&db->d_scan_fin, scan_scratch_words(n) + 16));
@@ -376,10 +415,13 @@ void ltpg_destroy_db(ltpg_db* db) {
   for (Slot& S : db->slots) {
     void* sb[] = {S.d_tid, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_packed, S.d_offsets,
                   S.d_res, S.d_status,
-                  S.d_bits, S.d_flags, S.d_offs, S.d_abort, S.d_small};
+                  S.d_bits, S.d_flags, S.d_offs, S.d_abort, S.d_small, S.d_vars};
     for (void* p : sb)
       if (p) cudaFree(p);
     if (S.h_small) cudaFreeHost(S.h_small);
+    if (S.h_vars) cudaFreeHost(S.h_vars);
+    for (GraphEntry& g : S.graphs)
+      if (g.exec) cudaGraphExecDestroy(g.exec);
     for (auto& e : S.ev)
       if (e) cudaEventDestroy(e);
     for (cudaEvent_t e : {S.h2d_done, S.comp_done, S.out_done})
@@ -388,6 +430,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   if (db->h2d) cudaStreamDestroy(db->h2d);
   if (db->d2h) cudaStreamDestroy(db->d2h);
   if (db->fin) cudaStreamDestroy(db->fin);
+  if (db->cap) cudaStreamDestroy(db->cap);
   if (db->status_ready) cudaEventDestroy(db->status_ready);
   if (db->fin_done) cudaEventDestroy(db->fin_done);
   if (db->d_scan_fin) cudaFree(db->d_scan_fin);
@@ -665,9 +708,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.dense_live = db->d_dense_live;
   bd.n_txns = n;
   bd.n_ops = ops_mode ? b->n_ops : 0;
-  bd.epoch = db->epoch;
   bd.flags = db->cfg.flags;
-  bd.clock = b->batch_clock;
+  bd.vars = S.d_vars;
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
   // verdict outputs: written in place when the caller's buffers are on the device
   uint8_t* st_out = S.host_out ? S.d_status : res->status;
@@ -723,7 +765,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool reads_dev = res->reads && res->outputs_on_device;
   long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : S.d_res;
   uint32_t* counts = S.d_small + 8;
-  CK(cudaMemsetAsync(db->d_reserve, 0, MAXT * sizeof(unsigned long long), s));
+  // ---- work that depends on host-side state, stream-ordered ahead of the batch's device work ----
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
   if (g_uploaded[db->device % 64] != db->tab_version) {
@@ -782,35 +824,53 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     x.kcount = P.small + 2;
     x.base = P.base;
     x.insdel = P.small + 12;
-    CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
-    if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
-    if (partitioned && n) {
-      CK(cudaMemsetAsync(x.res, 0, n_reads * sizeof(long long), s));
-      CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
-    }
   }
-  if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> every partition)
-    const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
-    const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
-    if (b->flags & LTPG_BATCH_COMPACT_PARAMS)
-      launch_unpack_compact(packed, offs, bd.ptype, n, S.d_params, pb[0].err, s);
-    else
-      launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
-    for (uint32_t p = 1; p < L; ++p) {
-      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, pb[p].err);
-      note_launch();
+  S.h_vars->epoch = db->epoch;  // the slot's previous batch (the copy's last reader) is complete
+  S.h_vars->clock = b->batch_clock;
+  std::atomic_thread_fence(std::memory_order_seq_cst);
+  // timing marks inside the batch's device work: event-record nodes when captured (always
+  // recorded there, so one graph serves batches with and without statistics)
+  bool capturing = false;
+  auto tmark = [](cudaEvent_t e, cudaStream_t st) { return record_stage(e, st); };
+
+  // ---- the batch's device work (a2..a8), enqueued on `s` -- or captured into a graph ---------
+  auto enqueue = [&](cudaStream_t s) -> int {
+    static_assert(MAXT <= 32, "k_batch_init clears the reservations with one warp");
+    k_batch_init<<<1, 32, 0, s>>>(db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch,
+                                  b->batch_clock);
+    note_launch();
+    for (uint32_t p = 0; p < L; ++p) {
+      Part& P = db->parts[p];
+      CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
+      if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
+      if (partitioned && n) {
+        CK(cudaMemsetAsync(pb[p].res, 0, n_reads * sizeof(long long), s));
+        CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
+      }
     }
-  }
-  if (timing) CK(cudaEventRecord(S.ev[1], s));
-  if (n) {
+    if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> every partition)
+      const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
+      const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
+      if (b->flags & LTPG_BATCH_COMPACT_PARAMS)
+        launch_unpack_compact(packed, offs, bd.ptype, n, S.d_params, pb[0].err, s);
+      else
+        launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
+      for (uint32_t p = 1; p < L; ++p) {
+        k_copy_err<<<1, 1, 0, s>>>(pb[0].err, pb[p].err);
+        note_launch();
+      }
+    }
+    const bool timed = timing || capturing;
+    if (timed) CK(tmark(S.ev[1], s));
+    if (!n) return LTPG_OK;
     // ---- a1..a6 per partition: validate + warp division, claims, execute + marks, detect --------
     for (uint32_t p = 0; p < L; ++p) {
       BatchDev& x = pb[p];
-      cudaEvent_t* evp = (timing && p == L - 1) ? S.ev : nullptr;
+      cudaEvent_t* evp = (timed && p == L - 1) ? S.ev : nullptr;
       if (ops_mode) {
         if (fused) {  // validate + warp-local division + execute; INSERTs after their claims
           launch_ops_fused(db->n_tables, x, filter, s);
-          if (evp) CK(cudaEventRecord(evp[2], s));  // ms_group = the fused kernel; ms_exec = INSERT tail
+          if (evp) CK(tmark(evp[2], s));  // ms_group = the fused kernel; ms_exec = INSERT tail
           scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
           launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
           launch_ops_claim(x, s);
@@ -820,18 +880,18 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
           scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
           launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
           launch_ops_claim(x, s);
-          if (evp) CK(cudaEventRecord(evp[2], s));
+          if (evp) CK(tmark(evp[2], s));
           launch_ops_exec(x, grouped, filter, s);
         }
         launch_bucket_reduce(db->h_tab, db->n_tables, s);  // NEXT-3 large-sized buckets (if any)
-        if (evp) CK(cudaEventRecord(evp[3], s));
+        if (evp) CK(tmark(evp[3], s));
         launch_ops_detect(x, s);
       } else {
         int rc = tpcc_front(db->parts[p].tpcc, x, s, evp);
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (timing) CK(cudaEventRecord(S.ev[4], s));
+    if (timed) CK(tmark(S.ev[4], s));
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
       if (db->p2p) {  // planes stored into every rank's region, signal, wait + OR (xchg.cuh)
@@ -852,12 +912,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       k_copy_err<<<1, 1, 0, s>>>(pb[0].err, S.d_small);
       note_launch();
     }
-    if (timing) CK(cudaEventRecord(S.ev[5], s));
+    if (timed) CK(tmark(S.ev[5], s));
     // ---- a8 on the finalize stream: commit bitmask, counts, abort list (status is final) ------
     CK(cudaEventRecord(db->status_ready, s));
     CK(cudaStreamWaitEvent(db->fin, db->status_ready, 0));
     launch_finalize_compact(st_out, n, bits_out, counts, S.d_small, abort_out, S.d_small + 16,
-                            S.host_out ? nullptr : res->n_aborted, db->d_fc_state, db->d_fc_ctr, db->epoch, db->fin);
+                            S.host_out ? nullptr : res->n_aborted, db->d_fc_state, db->d_fc_ctr, S.d_vars, db->fin);
     CK(cudaEventRecord(db->fin_done, db->fin));
     // ---- a7: write-back per partition -------------------------------------------------------
     for (uint32_t p = 0; p < L; ++p) {
@@ -889,8 +949,68 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       note_launch();
     }
     CK(cudaStreamWaitEvent(s, db->fin_done, 0));
+    CK(cudaGetLastError());
+    return LTPG_OK;
+  };
+
+  // Graph replay: the same shape's captured graph if this slot has one, else capture, instantiate
+  // and keep it (least recently used of GRAPHS_PER_SLOT replaced).  Multi-rank dbs enqueue
+  // directly (their exchange selects buffers by epoch parity on the host).
+  const bool use_graph = n && db->cfg.world == 1 && (db->cfg.flags & LTPG_FLAG_GRAPH);
+  if (use_graph) {
+    GraphKey k;
+    std::memset(&k, 0, sizeof(k));
+    k.mode = b->mode, k.n = n, k.n_ops = bd.n_ops, k.bflags = b->flags & LTPG_BATCH_COMPACT_PARAMS;
+    k.host_out = S.host_out, k.reads_dev = reads_dev, k.inputs_dev = b->inputs_on_device != 0;
+    k.packed = packed_params;
+    k.tab_version = db->tab_version;
+    if (b->inputs_on_device) {
+      const void* in[7] = {b->tid, b->op_begin, b->ops, b->op_arg, b->proc_type, b->proc_params, b->proc_offsets};
+      std::memcpy(k.in, in, sizeof(in));
+    }
+    const void* outp[5] = {res->status, res->commit_bits, res->abort_idx, res->n_aborted, res->reads};
+    if (!S.host_out) std::memcpy(k.out, outp, sizeof(outp));
+    else k.out[4] = res->reads ? reinterpret_cast<const void*>(1) : nullptr;
+    GraphEntry* E = nullptr;
+    for (GraphEntry& g : S.graphs)
+      if (g.exec && g.key == k) E = &g;
+    if (!E) {  // capture on the private stream (the caller's may be the legacy default stream)
+      E = &S.graphs[0];
+      for (GraphEntry& g : S.graphs)
+        if (!g.exec || g.last_use < E->last_use) E = &g;
+      if (E->exec) {
+        cudaGraphExecDestroy(E->exec);
+        E->exec = nullptr;
+      }
+      const uint64_t l0 = g_kernel_launches;
+      cudaGraph_t graph = nullptr;
+      CK(cudaStreamBeginCapture(db->cap, cudaStreamCaptureModeThreadLocal));
+      capturing = true;
+      const int rc = enqueue(db->cap);
+      capturing = false;
+      const cudaError_t ec = cudaStreamEndCapture(db->cap, &graph);
+      E->launches = g_kernel_launches - l0;
+      g_kernel_launches = l0;
+      if (rc) {
+        if (graph) cudaGraphDestroy(graph);
+        return rc;
+      }
+      if (ec != cudaSuccess) return fail(db, LTPG_ECUDA, std::string("graph capture: ") + cudaGetErrorString(ec));
+      const cudaError_t ei = cudaGraphInstantiate(&E->exec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (ei != cudaSuccess) {
+        E->exec = nullptr;
+        return fail(db, LTPG_ECUDA, std::string("cudaGraphInstantiate: ") + cudaGetErrorString(ei));
+      }
+      E->key = k;
+    }
+    E->last_use = ++db->graph_uses;
+    CK(cudaGraphLaunch(E->exec, s));
+    g_kernel_launches += E->launches;
+  } else {
+    const int rc = enqueue(s);
+    if (rc) return rc;
   }
-  CK(cudaGetLastError());
   if (timing) CK(cudaEventRecord(S.ev[6], s));
   CK(cudaEventRecord(S.comp_done, s));
   // ---- a8: results: D2H on the copy stream (overlaps the next batch's kernels) ------------------

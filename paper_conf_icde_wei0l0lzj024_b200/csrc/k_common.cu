@@ -179,7 +179,7 @@ __global__ void __launch_bounds__(256) k_finalize_compact(const uint8_t* __restr
                                                           const uint32_t* err, uint32_t* __restrict__ out,
                                                           uint32_t* n_out, uint32_t* n_out2,
                                                           unsigned long long* tile_state, uint32_t* tile_ctr,
-                                                          uint32_t epoch) {
+                                                          const BatchVars* __restrict__ vars) {
   __shared__ uint32_t tile_s, wsum[8], red[3], base_s;
   (void)err;  // no early exit: write-back may raise the error word concurrently, and a block
               // that skipped its tile would leave its successors waiting forever
@@ -233,6 +233,7 @@ __global__ void __launch_bounds__(256) k_finalize_compact(const uint8_t* __restr
   }
   if (threadIdx.x < 3 && red[threadIdx.x]) atomicAdd(counts + threadIdx.x, red[threadIdx.x]);
   if (threadIdx.x == 0) {  // decoupled look-back
+    const uint32_t epoch = vars->epoch;
     const unsigned long long tag = (unsigned long long)epoch << 32;
     volatile unsigned long long* vs = tile_state;
     uint32_t base = 0;
@@ -265,11 +266,11 @@ __global__ void __launch_bounds__(256) k_finalize_compact(const uint8_t* __restr
 
 void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* counts,
                              const uint32_t* err, uint32_t* out, uint32_t* n_out, uint32_t* n_out2,
-                             unsigned long long* tile_state, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t s) {
+                             unsigned long long* tile_state, uint32_t* tile_ctr, const BatchVars* vars, cudaStream_t s) {
   if (!n) return;
   cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), s);
   k_finalize_compact<<<(n + FC_TILE - 1) / FC_TILE, 256, 0, s>>>(status, n, commit_bits, counts, err, out, n_out,
-                                                                 n_out2, tile_state, tile_ctr, epoch);
+                                                                 n_out2, tile_state, tile_ctr, vars);
   note_launch();
 }
 

@@ -228,7 +228,7 @@ constexpr uint64_t UREF_RECHECK = 1ull << 58;
 __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi, uint32_t r, const ltpg_op& o,
                                          bool filter, uint32_t dmask, bool pre_claim = false) {
   const DevTable& T = c_tabs[o.table];
-  const mark_t tag = epoch_tag(b.epoch) | r;
+  const mark_t tag = epoch_tag(b_epoch(b)) | r;
   uint32_t row, claim;
   long long res = LTPG_NOT_FOUND;
   uint64_t uref = 0;
@@ -494,8 +494,8 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
         if (PART && !owns_key(b, T, k)) continue;
         uint32_t row, claim;
         lookup(T, t, dmask, k, row, claim);
-        if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b.epoch);
-        else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b.epoch);
+        if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b_epoch(b));
+        else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b));
       }
       continue;
     }
@@ -503,15 +503,15 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
       const ltpg_op o = load_op(b.ops, i);
       uint32_t row, claim;
       lookup(T, t, dmask, o.key, row, claim);
-      if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b.epoch);
+      if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b));
       continue;
     }
     const uint32_t row = (uint32_t)u;
     const uint32_t acc = chk == CHK_A ? ACC_ADD : (((u >> 59) & 1) ? ACC_WRITE : ACC_READ);
     if ((u >> 61) & 1) {
-      for (uint32_t g = 0; g < T.n_groups; ++g) bits |= unit_bits(T, g, row, acc, r, b.epoch);
+      for (uint32_t g = 0; g < T.n_groups; ++g) bits |= unit_bits(T, g, row, acc, r, b_epoch(b));
     } else {
-      bits |= unit_bits(T, (u >> 32) & 0xFF, row, acc, r, b.epoch);
+      bits |= unit_bits(T, (u >> 32) & 0xFF, row, acc, r, b_epoch(b));
     }
   }
   const uint32_t flag = bits | (b.ua[r] ? CF_UA : 0u);

@@ -155,16 +155,16 @@ __device__ __forceinline__ mark_t* rmark_ptr(const DevTable& T, uint32_t g, uint
 // longer serialise; k_bucket_reduce then takes the minimum over the bucket ("reads out
 // all the TIDs in the hash bucket and selects ... the smallest TID").  Result-identical.
 enum { MK_W = 0, MK_A = 1, MK_R = 2 };
-__device__ __forceinline__ void mark_unit(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag,
-                                          bool filter) {
-  mark_t* p;
+__device__ __forceinline__ mark_t* mark_addr(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag) {
   if (T.su > 1 && row < T.sub_rows) {
     const uint32_t gi = k == MK_A ? __popc(T.add_groups & ((1u << g) - 1u)) : g;
-    p = T.sub[k] + ((uint64_t)gi * T.sub_rows + row) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
-  } else {
-    p = k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
+    return T.sub[k] + ((uint64_t)gi * T.sub_rows + row) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
   }
-  mark_min(p, tag, filter);
+  return k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
+}
+__device__ __forceinline__ void mark_unit(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag,
+                                          bool filter) {
+  mark_min(mark_addr(T, k, g, row, tag), tag, filter);
 }
 
 __device__ __forceinline__ long long* col_ptr(const DevTable& T, uint32_t c, uint32_t row) {
@@ -283,6 +283,23 @@ void upload_tables_tpcc(const DevTable* h, cudaStream_t s);
 // number of kernels launched by this library (reported per batch in ltpg_stats)
 extern uint64_t g_kernel_launches;
 inline void note_launch(uint32_t k = 1) { g_kernel_launches += k; }
+// stage-timing event inside a batch's device work: an event-record node when the stream is
+// being captured into a batch graph (a plain record there would only order the capture)
+inline cudaError_t record_stage(cudaEvent_t e, cudaStream_t s) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(s, &cs);
+  return cs == cudaStreamCaptureStatusActive ? cudaEventRecordWithFlags(e, s, cudaEventRecordExternal)
+                                             : cudaEventRecord(e, s);
+}
+
+// Per-batch scalars that change from batch to batch while every pointer and size stays put.
+// They live in device memory (one copy per pipeline slot, refreshed by a stream-ordered H2D
+// copy of the slot's pinned host copy), so that a captured CUDA graph of the batch replays
+// with the new values (capi.cu: graph replay).
+struct BatchVars {
+  uint32_t epoch, pad;
+  long long clock;
+};
 
 struct BatchDev {
   // partitioning (§8(e)): nparts logical partitions (ranks x loopback); this is `part`.
@@ -296,8 +313,8 @@ struct BatchDev {
   unsigned long long* base;        // [MAXT] this partition's offset inside the reservation
   uint32_t* dense_live;            // persistent bitmask: tables whose dense mapping is valid
   uint32_t* insdel;                // this batch: tables receiving INSERT or DELETE ops (OPS)
-  uint32_t n_txns, n_ops, epoch, flags;
-  int64_t clock;
+  uint32_t n_txns, n_ops, flags;
+  const BatchVars* vars;           // epoch (conflict-log tag) and batch clock, in device memory
   const unsigned long long* tid;
   const uint32_t* op_begin;
   const ltpg_op* ops;
@@ -315,6 +332,9 @@ struct BatchDev {
   uint32_t* ins_tables;      // bitmask of tables receiving inserts
   uint32_t max_ops;
 };
+
+__device__ __forceinline__ uint32_t b_epoch(const BatchDev& b) { return __ldg(&b.vars->epoch); }
+__device__ __forceinline__ long long b_clock(const BatchDev& b) { return __ldg(&b.vars->clock); }
 
 // ---- block-aggregated list reservation ------------------------------------------------------
 // Every thread of a 256-thread block contributes cnt[k] items to list k; base[k] receives the
@@ -403,7 +423,7 @@ void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const ui
 // tile_state[ceil(n/1024)] persists across batches, tile_ctr is reset on `s`)
 void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit_bits, uint32_t* counts,
                              const uint32_t* err, uint32_t* out, uint32_t* n_out, uint32_t* n_out2,
-                             unsigned long long* tile_state, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t s);
+                             unsigned long long* tile_state, uint32_t* tile_ctr, const BatchVars* vars, cudaStream_t s);
 // NEXT-3: fold the large-sized buckets of every popular table into their units' mark words
 // (host copies of the tables; nothing is launched when no table has su > 1)
 void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s);
