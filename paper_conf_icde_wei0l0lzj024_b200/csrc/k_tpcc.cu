@@ -314,8 +314,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const long long o = b.res[4ull * r];
       const uint64_t okey = kO(w, d, (uint64_t)o);
       const DevTable& TOL_ = c_tabs[TOL];
-      // append position: chunk base + in-chunk prefix of committed NewOrders (k_no_chunk)
+      // append position: chunk base + in-chunk prefix of committed NewOrders (k_no_chunk); the
+      // row counter is read before any store (a store could alias it and force a reload)
       const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
+      const unsigned long long ol0 = *TOL_.n_rows;
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
         const uint32_t l = sub + 4 * k;
@@ -338,7 +340,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
           wr(TSt, S_ORDER_CNT, row_s, add(so[k], 1));
           wr(TSt, S_REMOTE_CNT, row_s, add(sr[k], rem));
         }
-        const uint32_t row = (uint32_t)(*TOL_.n_rows + (pref >> 32) + l);  // ORDER_LINE row
+        const uint32_t row = (uint32_t)(ol0 + (pref >> 32) + l);  // ORDER_LINE row
         wr(TOL_, OL_I_ID, row, i);
         wr(TOL_, OL_SUPPLY_W_ID, row, sw);
         wr(TOL_, OL_QUANTITY, row, qty);
@@ -357,23 +359,25 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const long long o = b.res[4ull * r];
       const uint64_t okey = kO(w, d, (uint64_t)o);
       const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
-      const uint32_t orow = (uint32_t)(*TOr.n_rows + (uint32_t)pref);
-      if (TOr.aux) TOr.aux[orow] = (uint32_t)(*TOL_.n_rows + (pref >> 32));  // contiguous lines
+      const unsigned long long nr_o = *TOr.n_rows, nr_ol = *TOL_.n_rows, nr_no = *TNw.n_rows;  // before stores
+      const long long clock = b_clock(b);
+      const uint32_t orow = (uint32_t)(nr_o + (uint32_t)pref);
+      if (TOr.aux) TOr.aux[orow] = (uint32_t)(nr_ol + (pref >> 32));  // contiguous lines
       wr(TOr, O_C_ID, orow, c);
-      wr(TOr, O_ENTRY_D, orow, b_clock(b));
+      wr(TOr, O_ENTRY_D, orow, clock);
       wr(TOr, O_OL_CNT, orow, n);
       wr(TOr, O_ALL_LOCAL, orow, !remote);
       wr(TOr, O_CARRIER_ID, orow, 0);
       TOr.rowkey[orow] = okey;
       TOr.valid[orow] = 1;
-      IdxSlot* sl = idx_find_or_insert(TOr, okey);
-      if (sl) sl->row = orow; else internal_error(x);
-      const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)pref);
+      const uint32_t nrow = (uint32_t)(nr_no + (uint32_t)pref);
       wr(TNw, NO_O_ID, nrow, o);
       TNw.rowkey[nrow] = okey;
       TNw.valid[nrow] = 1;
-      sl = idx_find_or_insert(TNw, okey);
-      if (sl) sl->row = nrow; else internal_error(x);
+      IdxSlot *so, *sn;
+      idx_insert2(TOr, okey, so, TNw, okey, sn);
+      if (so) so->row = orow; else internal_error(x);
+      if (sn) sn->row = nrow; else internal_error(x);
     }
     return;
   }
@@ -511,14 +515,14 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         wr(TOr, O_CARRIER_ID, orow, 0);
         TOr.rowkey[orow] = okey;
         TOr.valid[orow] = 1;
-        IdxSlot* sl = idx_find_or_insert(TOr, okey);
-        if (sl) sl->row = orow; else internal_error(x);
         const uint32_t nrow = (uint32_t)(*TNw.n_rows + (uint32_t)pref);
         wr(TNw, NO_O_ID, nrow, o);
         TNw.rowkey[nrow] = okey;
         TNw.valid[nrow] = 1;
-        sl = idx_find_or_insert(TNw, okey);
-        if (sl) sl->row = nrow; else internal_error(x);
+        IdxSlot *so, *sn;
+        idx_insert2(TOr, okey, so, TNw, okey, sn);
+        if (so) so->row = orow; else internal_error(x);
+        if (sn) sn->row = nrow; else internal_error(x);
       }
     }
   }
@@ -582,6 +586,13 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     col_upd<PH>(TDi, D_YTD, row_d, x, true);
   }
   if (cust) col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, row_c, x);
+  // HISTORY row inputs loaded before the balance stores (a store could alias them)
+  const DevTable& THi = c_tabs[TH];  // keyless append, no marks
+  unsigned long long h_tid = 0, h_rows = 0;
+  if (PH == PH_WB && cust) {
+    h_tid = b.tid[r];
+    h_rows = *THi.n_rows;
+  }
   if (PH == PH_WB && home) {
     addv(TWh, W_YTD, row_w, amount);
     addv(TDi, D_YTD, row_d, amount);
@@ -590,14 +601,13 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     addv(TCu, C_BALANCE, row_c, -amount);
     addv(TCu, C_YTD_PAYMENT, row_c, amount);
     addv(TCu, C_PAYMENT_CNT, row_c, 1);
-    const DevTable& THi = c_tabs[TH];  // keyless append, no marks
     // warp-aggregated append: one counter atomic per warp (every committed Payment appends;
     // per-lane atomics on the single counter serialised), consecutive rows per warp
     const uint32_t am = __activemask(), lane = threadIdx.x & 31, lead = __ffs(am) - 1;
     uint32_t hb = 0;
     if (lane == lead) hb = atomicAdd(tp.misc + M_HIST, (uint32_t)__popc(am));
     hb = __shfl_sync(am, hb, lead) + __popc(am & ((1u << lane) - 1u));
-    const uint32_t row = (uint32_t)(*THi.n_rows + hb);
+    const uint32_t row = (uint32_t)(h_rows + hb);
     wr(THi, H_C_ID, row, cid);
     wr(THi, H_C_D_ID, row, cd);
     wr(THi, H_C_W_ID, row, cw);
@@ -605,7 +615,7 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     wr(THi, H_W_ID, row, w);
     wr(THi, H_DATE, row, b_clock(b));
     wr(THi, H_AMOUNT, row, amount);
-    wr(THi, H_TID, row, (long long)b.tid[r]);
+    wr(THi, H_TID, row, (long long)h_tid);
     wr(THi, H_SEQ, row, 0);
     THi.valid[row] = 1;
   }
@@ -1026,8 +1036,8 @@ template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
 // loads (params -> log -> marks) and gains most from occupancy (measured: 8 -> 32 regs);
 // write-back keeps every stock column of a lane's lines in registers (one load wave instead of
-// a read-modify-write chain per column): 4 blocks / 64 regs, 0.165 -> 0.140 ms on tpcc_c4
-// (6 blocks / 40 regs spilled: 0.170)
+// a read-modify-write chain per column): 3 blocks / 80 regs, 0.165 -> 0.138 ms on tpcc_c4
+// (4 blocks / 64 regs: 0.141; 6 blocks / 40 regs spilled: 0.170)
 #ifndef LTPG_EXEC_MINB
 #define LTPG_EXEC_MINB 4
 #endif
@@ -1035,7 +1045,7 @@ template <int PH, uint32_t TMASK>
 #define LTPG_DETECT_MINB 8
 #endif
 #ifndef LTPG_WB_MINB
-#define LTPG_WB_MINB 4
+#define LTPG_WB_MINB 3
 #endif
 __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
     k_tpcc_phase(BatchDev b, TpccParams tp) {

@@ -201,10 +201,10 @@ __device__ __forceinline__ bool lookup(const DevTable& T, uint32_t t, uint32_t d
   return idx_find(T, key, row, claim);
 }
 
-// Find or create the slot of `key` (load / claim paths).
-__device__ __forceinline__ IdxSlot* idx_find_or_insert(const DevTable& T, uint64_t key) {
-  uint64_t h = idx_hash(key, T.idx_shift);
-  for (uint64_t probes = 0; probes <= T.idx_mask; ++probes) {
+// Find or create the slot of `key` (load / claim paths), probing from slot h.
+__device__ __forceinline__ IdxSlot* idx_find_or_insert_from(const DevTable& T, uint64_t key, uint64_t h,
+                                                            uint64_t probes0 = 0) {
+  for (uint64_t probes = probes0; probes <= T.idx_mask; ++probes) {
     IdxSlot* s = T.idx + h;
     unsigned long long k = __ldcg(&s->key);  // hint only; the CAS decides
     if (k == KEY_EMPTY) k = atomicCAS(&s->key, KEY_EMPTY, key);
@@ -212,6 +212,22 @@ __device__ __forceinline__ IdxSlot* idx_find_or_insert(const DevTable& T, uint64
     h = (h + 1) & T.idx_mask;
   }
   return nullptr;
+}
+__device__ __forceinline__ IdxSlot* idx_find_or_insert(const DevTable& T, uint64_t key) {
+  return idx_find_or_insert_from(T, key, idx_hash(key, T.idx_shift));
+}
+// Two fresh keys in two tables (a NewOrder's ORDER and NEW_ORDER rows): both home slots are
+// claimed by CAS straight away -- independent atomics, one round trip instead of a hint read
+// and a CAS per key, one key after the other -- and only a taken home slot falls back to probing.
+__device__ __forceinline__ void idx_insert2(const DevTable& TA, uint64_t ka, IdxSlot*& sa, const DevTable& TB,
+                                            uint64_t kb, IdxSlot*& sb) {
+  const uint64_t ha = idx_hash(ka, TA.idx_shift), hb = idx_hash(kb, TB.idx_shift);
+  sa = TA.idx + ha;
+  sb = TB.idx + hb;
+  const unsigned long long va = atomicCAS(&sa->key, KEY_EMPTY, ka);
+  const unsigned long long vb = atomicCAS(&sb->key, KEY_EMPTY, kb);
+  if (va != KEY_EMPTY && va != ka) sa = idx_find_or_insert_from(TA, ka, (ha + 1) & TA.idx_mask, 1);
+  if (vb != KEY_EMPTY && vb != kb) sb = idx_find_or_insert_from(TB, kb, (hb + 1) & TB.idx_mask, 1);
 }
 
 __device__ __forceinline__ IdxSlot* idx_slot(const DevTable& T, uint64_t key) {
