@@ -908,10 +908,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, st_out, pb[0].err, S.d_small, reorder);
         note_launch(2);
       }
-    } else {
-      k_copy_err<<<1, 1, 0, s>>>(pb[0].err, S.d_small);
-      note_launch();
-    }
+    }  // unpartitioned: the partition's error word reaches S.d_small with k_or_err after write-back
     if (timed) CK(tmark(S.ev[5], s));
     // ---- a8 on the finalize stream: commit bitmask, counts, abort list (status is final) ------
     CK(cudaEventRecord(db->status_ready, s));
@@ -929,7 +926,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (ops_mode) launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
+    if (ops_mode)  // the combined verdict error (partitioned) or the partition's own
+      launch_advance_cursor(db->n_tables, db->d_reserve, partitioned ? S.d_small : pb[0].err, db->d_dense_live,
+                            pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
     if (db->p2p) {  // every rank publishes and reduces its slice (the protocol needs it)
       launch_xsig_res(db->xpeers, (uint32_t)db->cfg.rank, (uint32_t)db->cfg.world, db->epoch, s);

@@ -156,6 +156,47 @@ __device__ __forceinline__ uint32_t seg16_or(uint32_t v) {
   return v;
 }
 
+// "Last block" of a grid: every block calls this once at its end (after all of its threads'
+// global writes); it returns true in exactly one block, the last to arrive, once every other
+// block's writes are visible.  `ctr` is zeroed before the launch.
+__device__ __forceinline__ bool last_block(uint32_t* ctr) {
+  __shared__ bool last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(ctr, 1u) == gridDim.x - 1;
+    if (last) __threadfence();
+  }
+  __syncthreads();
+  return last;
+}
+
+// ECAPACITY before execution: worst case every NewOrder / Payment of this partition
+// commits; partitions of one process share the table and reserve in stream order (one thread
+// of k_tpcc_group's last block)
+__device__ void tpcc_capacity_tail(const BatchDev& b, const TpccParams& tp) {
+  const uint64_t add[4] = {__ldcg(tp.misc + M_NO), __ldcg(tp.misc + M_NO), __ldcg(tp.misc + M_NO_LINES),
+                           __ldcg(tp.misc + M_PAY)};
+  const int tabs[4] = {TO, TNO, TOL, TH};
+  for (int k = 0; k < 4; ++k) {
+    const DevTable& T = c_tabs[tabs[k]];
+    b.reserve[tabs[k]] += add[k];
+    if (*T.n_rows + b.reserve[tabs[k]] > T.capacity) atomicOr(b.err, ERR_ECAPACITY);
+  }
+}
+
+// append-row counters advanced past this batch's committed rows (one thread of the write-back
+// phase's last block)
+__device__ void tpcc_advance_tail(const BatchDev& b, const TpccParams& tp) {
+  if (*(volatile uint32_t*)b.err) return;
+  const uint32_t n = b.n_txns;
+  const unsigned long long tot = __ldcg(tp.no_pref + n);
+  *c_tabs[TO].n_rows += (uint32_t)tot;
+  *c_tabs[TNO].n_rows += (uint32_t)tot;
+  *c_tabs[TOL].n_rows += tot >> 32;
+  *c_tabs[TH].n_rows += __ldcg(tp.misc + M_HIST);
+}
+
 // ---- NewOrder (TPC-C 2.4; SURVEY §8(c) procedure table) --------------------------------
 template <int PH>
 __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active, Tx& x) {
@@ -1049,7 +1090,7 @@ template <int PH, uint32_t TMASK>
 #endif
 __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
     k_tpcc_phase(BatchDev b, TpccParams tp) {
-  if (*b.err) return;
+  if (*b.err) return;  // (write-back: the row counters then stay put -- no last block runs)
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1104,6 +1145,8 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
       }
     }
   }
+  if (PH == PH_WB && TMASK == TM_MAIN && last_block(tp.misc + M_DONE_WB) && threadIdx.x == 0)
+    tpcc_advance_tail(b, tp);
 }
 
 // ---- K-tgroup: validation + per-type lists (warp-aggregated appends) ----------------------------
@@ -1213,6 +1256,7 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
 #pragma unroll
   for (uint32_t k = 0; k < NTYPES; ++k)
     if (tcnt[k]) tp.list[(uint64_t)k * tp.max_txns + tbase[k]] = r;
+  if (last_block(tp.misc + M_DONE_G) && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
 }
 
 // committed entries of every per-type list -> clist (order inside a list is irrelevant)
@@ -1236,18 +1280,6 @@ __global__ void __launch_bounds__(256) k_tpcc_relist(BatchDev b, TpccParams tp) 
 #pragma unroll
   for (int k = 0; k < NTYPES; ++k)
     if (cnt[k]) tp.clist[(uint64_t)k * tp.max_txns + base[k]] = r;
-}
-
-// ECAPACITY before execution: worst case every NewOrder / Payment of this partition
-// commits; partitions of one process share the table and reserve in stream order
-__global__ void k_tpcc_capacity(BatchDev b, TpccParams tp) {
-  const uint64_t add[4] = {tp.misc[M_NO], tp.misc[M_NO], tp.misc[M_NO_LINES], tp.misc[M_PAY]};
-  const int tabs[4] = {TO, TNO, TOL, TH};
-  for (int k = 0; k < 4; ++k) {
-    const DevTable& T = c_tabs[tabs[k]];
-    b.reserve[tabs[k]] += add[k];
-    if (*T.n_rows + b.reserve[tabs[k]] > T.capacity) atomicOr(b.err, ERR_ECAPACITY);
-  }
 }
 
 // ---- NewOrder o_id: fetch-ADD pre-image = snapshot D_NEXT_O_ID + #committed NewOrders of the
@@ -1439,14 +1471,6 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
   }
 }
 
-__global__ void k_tpcc_advance(BatchDev b, TpccParams tp) {
-  if (*b.err) return;
-  const uint32_t n = b.n_txns;
-  *c_tabs[TO].n_rows += (uint32_t)tp.no_pref[n];
-  *c_tabs[TNO].n_rows += (uint32_t)tp.no_pref[n];
-  *c_tabs[TOL].n_rows += tp.no_pref[n] >> 32;
-  *c_tabs[TH].n_rows += tp.misc[M_HIST];
-}
 
 // ORDER.aux[row] = first ORDER_LINE row of the order if its cnt lines sit in consecutive rows
 __global__ void k_build_olrow() {
@@ -1563,9 +1587,8 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
   const TpccParams tp = params_of(t, b, false);
   cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
   cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
-  k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);
-  k_tpcc_capacity<<<1, 1, 0, s>>>(b, tp);
-  note_launch(2);
+  k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);  // + the capacity check (last block)
+  note_launch(1);
   if (ev) record_stage(ev[2], s);
   const uint32_t grid = phase_grid(n);
   // StockLevel (shared per district) on a side stream, concurrently with the other procedures
@@ -1612,9 +1635,8 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));
-  k_tpcc_advance<<<1, 1, 0, s>>>(b, tp);
-  note_launch(2);
+  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));  // + row counters
+  note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
 

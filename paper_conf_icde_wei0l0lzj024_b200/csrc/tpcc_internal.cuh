@@ -22,7 +22,9 @@ enum { I_PRICE = 0, I_IM_ID = 1 };
 enum { S_QUANTITY = 0, S_YTD = 1, S_ORDER_CNT = 2, S_REMOTE_CNT = 3 };
 
 // counters in TpccDev::misc (M_NO / M_NO_LINES / M_PAY: inserts this partition may append)
-enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3, M_CCOUNT = 8 };
+// M_DONE_G / M_DONE_WB: blocks of k_tpcc_group / the write-back phase that finished (the last
+// one runs the capacity check / the row-counter advance)
+enum { M_HIST = 0, M_NO_LINES = 1, M_PAY = 2, M_NO = 3, M_DONE_G = 4, M_DONE_WB = 5, M_CCOUNT = 8 };
 
 // StockLevel shared per district (k_sl_*): per-batch scratch indexed by district key (dk) or by
 // the compact index of a district with StockLevels in the batch (idx)
