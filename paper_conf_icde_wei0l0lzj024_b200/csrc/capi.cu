@@ -824,6 +824,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     x.kcount = P.small + 2;
     x.base = P.base;
     x.insdel = P.small + 12;
+    x.done = P.small + 14;
   }
   S.h_vars->epoch = db->epoch;  // the slot's previous batch (the copy's last reader) is complete
   S.h_vars->clock = b->batch_clock;
@@ -920,15 +921,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     for (uint32_t p = 0; p < L; ++p) {
       pb[p].status = st_out;
       if (ops_mode) {
-        launch_ops_writeback(pb[p], s);
+        launch_ops_writeback(pb[p], db->n_tables, L == 1, s);  // L == 1: + the cursor advance
       } else {
         int rc = tpcc_back(db->parts[p].tpcc, pb[p], db->d_scan, s);
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }
-    if (ops_mode)  // the combined verdict error (partitioned) or the partition's own
-      launch_advance_cursor(db->n_tables, db->d_reserve, partitioned ? S.d_small : pb[0].err, db->d_dense_live,
-                            pb[0].insdel, s);
+    if (ops_mode && L > 1)  // the combined verdict error, after every partition's write-back
+      launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
     if (db->p2p) {  // every rank publishes and reduces its slice (the protocol needs it)
       launch_xsig_res(db->xpeers, (uint32_t)db->cfg.rank, (uint32_t)db->cfg.world, db->epoch, s);

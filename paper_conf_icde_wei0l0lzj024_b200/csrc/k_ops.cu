@@ -528,10 +528,7 @@ void launch_ops_detect(const BatchDev& b, cudaStream_t s) {
 }
 
 // ---- K-wb: apply committed write sets; every INSERT releases its claim ----------------
-__global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b) {
-  if (*b.err) return;
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= b.n_txns) return;
+__device__ __forceinline__ void ops_writeback_txn(const BatchDev& b, uint32_t r) {
   const bool commit = b.status[r] == LTPG_ST_COMMIT;  // final verdict (after the exchange)
   if (!commit && b.txn_ins[r + 1] == b.txn_ins[r]) return;  // aborted, no claims to release
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
@@ -578,9 +575,25 @@ __global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b) {
     }
   }
 }
+// ADV (single-partition batches): the grid's last block also advances the append cursors past
+// this batch's reservations and retires the dense key mapping of tables that saw INSERT or
+// DELETE (what k_advance does after the write-back of every partition otherwise)
+template <bool ADV>
+__global__ void __launch_bounds__(256) k_ops_writeback(BatchDev b, uint32_t n_tables) {
+  if (*b.err) return;  // (no block counts: the cursors stay put)
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < b.n_txns) ops_writeback_txn(b, r);
+  if (ADV && last_block(b.done) && threadIdx.x == 0 && !*(volatile uint32_t*)b.err) {
+    for (uint32_t t = 0; t < n_tables; ++t) *c_tabs[t].n_rows += b.reserve[t];
+    *b.dense_live &= ~*b.insdel;
+  }
+}
 
-void launch_ops_writeback(const BatchDev& b, cudaStream_t s) {
-  k_ops_writeback<<<(b.n_txns + 255) / 256, 256, 0, s>>>(b);
+void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cudaStream_t s) {
+  if (advance)
+    k_ops_writeback<true><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b, n_tables);
+  else
+    k_ops_writeback<false><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b, n_tables);
   note_launch();
 }
 

@@ -156,21 +156,6 @@ __device__ __forceinline__ uint32_t seg16_or(uint32_t v) {
   return v;
 }
 
-// "Last block" of a grid: every block calls this once at its end (after all of its threads'
-// global writes); it returns true in exactly one block, the last to arrive, once every other
-// block's writes are visible.  `ctr` is zeroed before the launch.
-__device__ __forceinline__ bool last_block(uint32_t* ctr) {
-  __shared__ bool last;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    last = atomicAdd(ctr, 1u) == gridDim.x - 1;
-    if (last) __threadfence();
-  }
-  __syncthreads();
-  return last;
-}
-
 // ECAPACITY before execution: worst case every NewOrder / Payment of this partition
 // commits; partitions of one process share the table and reserve in stream order (one thread
 // of k_tpcc_group's last block)
@@ -571,7 +556,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
 
 // ---- Payment (TPC-C 2.5) ------------------------------------------------------------------
 template <int PH>
-__device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r, Tx& x) {
+__device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r, Tx& x, long long* agg = nullptr) {
   const DevTable& TWh = c_tabs[TW];
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TCu = c_tabs[TC];
@@ -635,8 +620,16 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     h_rows = *THi.n_rows;
   }
   if (PH == PH_WB && home) {
-    addv(TWh, W_YTD, row_w, amount);
-    addv(TDi, D_YTD, row_d, amount);
+    if (agg) {  // block-aggregated delayed adds (k_tpcc_phase)
+      atomicAdd(reinterpret_cast<unsigned long long*>(agg + w), (unsigned long long)amount);
+      if (tp.agg_dsz)
+        atomicAdd(reinterpret_cast<unsigned long long*>(agg + tp.nw + 1 + kD(w, d)), (unsigned long long)amount);
+      else
+        addv(TDi, D_YTD, row_d, amount);
+    } else {
+      addv(TWh, W_YTD, row_w, amount);
+      addv(TDi, D_YTD, row_d, amount);
+    }
   }
   if (PH == PH_WB && cust) {
     addv(TCu, C_BALANCE, row_c, -amount);
@@ -1092,6 +1085,15 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     k_tpcc_phase(BatchDev b, TpccParams tp) {
   if (*b.err) return;  // (write-back: the row counters then stay put -- no last block runs)
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
+  // write-back with delayed W_YTD / D_YTD (ADD columns): the block's committed Payments add
+  // into shared-memory deltas per warehouse (and district), flushed with one atomic per touched
+  // row at the end -- hundreds of thousands of same-row atomics at the L2 become a few per block
+  extern __shared__ long long agg[];
+  const bool aggw = PH == PH_WB && col_is_add(c_tabs[TW], W_YTD) && col_is_add(c_tabs[TD], D_YTD);
+  if (aggw) {
+    for (uint32_t i = threadIdx.x; i < tp.nw + 1 + tp.agg_dsz; i += blockDim.x) agg[i] = 0;
+    __syncthreads();
+  }
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
@@ -1127,7 +1129,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     if (PH == PH_DETECT && reorder && (t == 2 || t == 4)) go = false;
     switch (t) {
       case 0: proc_neworder<PH>(b, tp, r, sub, go, x); break;
-      case 1: if (go) proc_payment<PH>(b, tp, r, x); break;
+      case 1: if (go) proc_payment<PH>(b, tp, r, x, aggw ? agg : nullptr); break;
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
       case 3: proc_delivery<PH>(b, tp, r, sub, go, x); break;
       default:
@@ -1143,6 +1145,20 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
         if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;  // partitioned: exchanged before write-back
         else b.status[r] = status_of_bits(flag, reorder);
       }
+    }
+  }
+  if (aggw) {
+    __syncthreads();
+    const DevTable& TWh = c_tabs[TW];
+    const DevTable& TDi = c_tabs[TD];
+    for (uint32_t i = threadIdx.x; i < tp.nw + 1 + tp.agg_dsz; i += blockDim.x) {
+      const long long v = agg[i];
+      if (!v) continue;
+      const bool isw = i <= tp.nw;
+      const DevTable& T = isw ? TWh : TDi;
+      const uint32_t row = rowof(T, isw ? TW : TD, isw ? i : i - tp.nw - 1, dmask);
+      if (row == ROW_NONE) { atomicOr(b.err, ERR_EINTERNAL); continue; }
+      addv(T, isw ? W_YTD : D_YTD, row, v);
     }
   }
   if (PH == PH_WB && TMASK == TM_MAIN && last_block(tp.misc + M_DONE_WB) && threadIdx.x == 0)
@@ -1570,11 +1586,16 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
              : LTPG_ECUDA;
 }
 
+constexpr uint32_t AGG_DSZ_MAX = 4096;  // per-block D_YTD aggregation up to ~400 warehouses (32 KB)
+static size_t wb_smem(const TpccDev& t) {
+  return ((size_t)t.nw + 1 + (t.dsz <= AGG_DSZ_MAX ? t.dsz : 0)) * sizeof(long long);
+}
 static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists) {
   const uint32_t n = b.n_txns;
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
-                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min};
+                    t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min,
+                    committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -1635,7 +1656,7 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
   k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, 0, s>>>(b, params_of(t, b, true));  // + row counters
+  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, wb_smem(t), s>>>(b, params_of(t, b, true));  // + row counters
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }

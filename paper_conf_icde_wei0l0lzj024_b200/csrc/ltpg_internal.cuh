@@ -329,6 +329,7 @@ struct BatchDev {
   unsigned long long* base;        // [MAXT] this partition's offset inside the reservation
   uint32_t* dense_live;            // persistent bitmask: tables whose dense mapping is valid
   uint32_t* insdel;                // this batch: tables receiving INSERT or DELETE ops (OPS)
+  uint32_t* done;                  // zeroed per batch: block counter of the OPS write-back grid
   uint32_t n_txns, n_ops, flags;
   const BatchVars* vars;           // epoch (conflict-log tag) and batch clock, in device memory
   const unsigned long long* tid;
@@ -351,6 +352,21 @@ struct BatchDev {
 
 __device__ __forceinline__ uint32_t b_epoch(const BatchDev& b) { return __ldg(&b.vars->epoch); }
 __device__ __forceinline__ long long b_clock(const BatchDev& b) { return __ldg(&b.vars->clock); }
+
+// "Last block" of a grid: every block calls this once at its end (after all of its threads'
+// global writes); it returns true in exactly one block, the last to arrive, once every other
+// block's writes are visible.  `ctr` is zeroed before the launch.
+__device__ __forceinline__ bool last_block(uint32_t* ctr) {
+  __shared__ bool last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(ctr, 1u) == gridDim.x - 1;
+    if (last) __threadfence();
+  }
+  __syncthreads();
+  return last;
+}
 
 // ---- block-aggregated list reservation ------------------------------------------------------
 // Every thread of a 256-thread block contributes cnt[k] items to list k; base[k] receives the
@@ -421,7 +437,7 @@ void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t 
 void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStream_t s);
 void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s);
 void launch_ops_detect(const BatchDev& b, cudaStream_t s);
-void launch_ops_writeback(const BatchDev& b, cudaStream_t s);
+void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cudaStream_t s);
 void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
                            unsigned long long* base, unsigned long long* reserve, uint32_t* err, cudaStream_t s);
 void launch_advance_cursor(uint32_t n_tables, const unsigned long long* reserve, const uint32_t* err,

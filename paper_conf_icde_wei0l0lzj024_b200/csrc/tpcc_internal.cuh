@@ -78,6 +78,7 @@ struct TpccParams {
   uint32_t nw, dsz, max_txns, n_chunks;
   unsigned long long* chunk_tot;
   uint32_t* dl_min;
+  uint32_t agg_dsz;             // write-back: DISTRICT D_YTD deltas aggregated per block (0: not)
 };
 
 int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);
