@@ -223,3 +223,28 @@ def test_compact_params_equal_fixed_blocks():
         g.run_tpcc(bad, 9)
     assert e.value.rc == lib.LTPG_EINVAL
     compare_tables(g, o)  # nothing changed
+
+
+def test_many_districts_tiled_colscan():
+    """More than 2048 district keys (210 warehouses) switch the o_id column scan to the tiled
+    kernel (k_no_colscan_tiled): verdicts, o_id results and the DISTRICT / ORDER / NEW_ORDER
+    state equal the oracle over a closed loop of NewOrder/Payment batches."""
+    W, B = 210, 8192
+    wl = tpcc.TpccWorkload(W, seed=21, mode="strict", mix=tpcc.MIX_NO_PAY)
+    tables = wl.initial_tables()
+    g = L().tpcc_database(wl, max_txns=B, tables=tables, append_batches=4)
+    o = oracle.tpcc_db(wl, tables)
+    pending, tid = None, 1
+    for bno in range(3):
+        fresh = wl.batch(B - (0 if pending is None else len(pending["tid"])), tid, bno)
+        tid += len(fresh["tid"])
+        batch = fresh if pending is None else {k: np.concatenate([pending[k], fresh[k]]) for k in fresh}
+        st = compare(g, o, batch, 2 + bno)
+        assert (st == 1).sum() > B // 16
+        ab = np.nonzero(st == ST_CONFLICT)[0]
+        pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
+    from workloads.formats import T_WAREHOUSE, T_DISTRICT, T_ORDER, T_NEW_ORDER
+    for t in (T_WAREHOUSE, T_DISTRICT, T_ORDER, T_NEW_ORDER):
+        gk, gc = g.dump_table(t)
+        ok, oc = o.dump_table(t)
+        assert (gk == ok).all() and gc.shape == oc.shape and (gc == oc).all(), t
