@@ -284,6 +284,32 @@ LTPG_API int ltpg_wait_batch(ltpg_db* db, ltpg_result* result);
  * keys: host u64[n_rows]; cols: host int64 [n_cols][n_rows]. */
 LTPG_API int ltpg_dump_table(ltpg_db* db, uint32_t table_id, uint64_t* n_rows, uint64_t* keys, int64_t* cols);
 
+/* ---- a9: the host retry loop ("aborted transactions ... are re-executed in the next
+ * batch", P:120 TID order) ------------------------------------------------------------------
+ * The next batch = the conflict aborts of `prev` (abort_idx as returned by ltpg_run_batch:
+ * ascending ranks), with their original TIDs and inputs, followed by a prefix of `fresh`, as
+ * many fresh txns as fit in out->cap_txns (and, OPS, out->cap_ops).  Because every aborted TID is
+ * smaller than every fresh one, the retried txns take the smallest ranks: the batch's smallest
+ * rank commits unless it user-aborts, so no txn is retried forever.
+ * Host memory only (prev/fresh with inputs_on_device == 0 and fixed 128-byte TPC-C blocks; the
+ * caller owns every buffer).  Needs no db and no GPU.  Errors (EINVAL, nothing written
+ * past the buffers): mode mismatch, device or packed inputs, an abort index out of range or
+ * not ascending, the aborts alone exceeding the capacity, or a fresh TID not larger than the
+ * last retried one. */
+typedef struct {
+  uint32_t cap_txns, cap_ops;   /* in: capacity of the buffers below (txns / OPS ops)       */
+  uint64_t* tid;                /* [cap_txns]                                               */
+  uint32_t* op_begin;           /* OPS: [cap_txns+1]                                        */
+  ltpg_op* ops;                 /* OPS: [cap_ops]                                           */
+  int64_t* op_arg;              /* OPS: [cap_ops]                                           */
+  uint8_t* proc_type;           /* TPCC: [cap_txns]                                         */
+  uint8_t* proc_params;         /* TPCC: [cap_txns][128]                                    */
+  uint32_t n_txns, n_ops;       /* out: the composed batch                                  */
+  uint32_t n_retried, n_fresh;  /* out: aborts carried over, fresh txns taken (a prefix)    */
+} ltpg_batch_buf;
+LTPG_API int ltpg_compose_retry(const ltpg_batch* prev, const uint32_t* abort_idx, uint32_t n_aborted,
+                                const ltpg_batch* fresh, ltpg_batch_buf* out);
+
 LTPG_API void ltpg_destroy_db(ltpg_db* db);
 LTPG_API const char* ltpg_last_error(const ltpg_db* db);
 /* Library version string, e.g. "ltpg-b200 0.1 sm_100a". */

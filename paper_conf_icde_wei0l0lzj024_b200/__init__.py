@@ -39,6 +39,7 @@ LTPG_FLAG_NCCL_EXCHANGE = 1 << 4
 LTPG_FLAG_LARGE_BUCKETS = 1 << 5
 LTPG_FLAG_GRAPH = 1 << 6
 LTPG_PEER_HANDLE_BYTES = 128
+LTPG_PARAM_BYTES = 128
 LTPG_LAYOUT_ROWBLOCK, LTPG_LAYOUT_COLUMNAR = 0, 1
 LTPG_FLAG_LOOPBACK_SHIFT = 8
 LTPG_ST_CONFLICT, LTPG_ST_COMMIT, LTPG_ST_USER_ABORT = 0, 1, 2
@@ -97,6 +98,15 @@ _lib.ltpg_peer_handle.restype = c_int
 _lib.ltpg_peer_handle.argtypes = [c_vp, c_vp]
 _lib.ltpg_connect_peers.restype = c_int
 _lib.ltpg_connect_peers.argtypes = [c_vp, c_vp]
+class ltpg_batch_buf(ctypes.Structure):
+    _fields_ = [("cap_txns", c_u32), ("cap_ops", c_u32), ("tid", c_vp), ("op_begin", c_vp), ("ops", c_vp),
+                ("op_arg", c_vp), ("proc_type", c_vp), ("proc_params", c_vp), ("n_txns", c_u32), ("n_ops", c_u32),
+                ("n_retried", c_u32), ("n_fresh", c_u32)]
+
+
+_lib.ltpg_compose_retry.restype = c_int
+_lib.ltpg_compose_retry.argtypes = [ctypes.POINTER(ltpg_batch), c_vp, c_u32, ctypes.POINTER(ltpg_batch),
+                                    ctypes.POINTER(ltpg_batch_buf)]
 _lib.ltpg_version.restype = ctypes.c_char_p
 _lib.ltpg_version.argtypes = []
 
@@ -111,11 +121,13 @@ ltpg_version = _lib.ltpg_version
 ltpg_wait_batch = _lib.ltpg_wait_batch
 ltpg_peer_handle = _lib.ltpg_peer_handle
 ltpg_connect_peers = _lib.ltpg_connect_peers
+ltpg_compose_retry = _lib.ltpg_compose_retry
 LTPG_BATCH_ASYNC = 1
 LTPG_BATCH_COMPACT_PARAMS = 2
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
-            "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers"]
+            "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers",
+            "ltpg_compose_retry"]
 
 
 class LtpgError(RuntimeError):
@@ -464,3 +476,45 @@ def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, f
                       layout=LTPG_LAYOUT_COLUMNAR if t in (T_ORDER, T_ORDER_LINE) else LTPG_LAYOUT_ROWBLOCK)
     _connect(db, world, flags, peer_group)
     return db
+
+
+def compose_retry(prev, abort_idx, fresh, max_txns, max_ops=0):
+    """a9, the host retry loop (ltpg_compose_retry): the next batch = the conflict aborts of
+    `prev` (ascending ranks from run_ops / run_tpcc, original TIDs) followed by as many txns of
+    `fresh` as fit in max_txns (and max_ops).  Host numpy batches in, a host numpy batch out;
+    returns (batch, n_fresh_taken)."""
+    ops = "op_begin" in prev
+    abort_idx = np.ascontiguousarray(abort_idx, dtype=np.uint32)
+
+    def desc(b):
+        if ops:
+            b = {k: np.ascontiguousarray(v) for k, v in b.items()}
+            return b, ltpg_batch(n_txns=len(b["tid"]), tid=_ptr(b["tid"]), mode=LTPG_MODE_OPS,
+                                 n_ops=len(b["args"]), op_begin=_ptr(b["op_begin"]), ops=_ptr(b["ops"]),
+                                 op_arg=_ptr(b["args"]))
+        b = {k: np.ascontiguousarray(v) for k, v in b.items()}
+        return b, ltpg_batch(n_txns=len(b["tid"]), tid=_ptr(b["tid"]), mode=LTPG_MODE_TPCC,
+                             proc_type=_ptr(b["type"]), proc_params=_ptr(b["params"]))
+
+    pk, pd = desc(prev)
+    fk, fd = desc(fresh)
+    out = {"tid": np.zeros(max_txns, np.uint64)}
+    if ops:
+        out.update(op_begin=np.zeros(max_txns + 1, np.uint32), ops=np.zeros(max(max_ops, 1), pk["ops"].dtype),
+                   args=np.zeros(max(max_ops, 1), np.int64))
+        buf = ltpg_batch_buf(cap_txns=max_txns, cap_ops=max_ops, tid=_ptr(out["tid"]), op_begin=_ptr(out["op_begin"]),
+                             ops=_ptr(out["ops"]), op_arg=_ptr(out["args"]))
+    else:
+        out.update(type=np.zeros(max_txns, np.uint8), params=np.zeros((max_txns, LTPG_PARAM_BYTES), np.uint8))
+        buf = ltpg_batch_buf(cap_txns=max_txns, tid=_ptr(out["tid"]), proc_type=_ptr(out["type"]),
+                             proc_params=_ptr(out["params"]))
+    rc = ltpg_compose_retry(ctypes.byref(pd), abort_idx.ctypes.data_as(c_vp), len(abort_idx), ctypes.byref(fd),
+                            ctypes.byref(buf))
+    if rc:
+        raise LtpgError(rc, "ltpg_compose_retry: invalid arguments")
+    n, m = buf.n_txns, buf.n_ops
+    if ops:
+        res = {"tid": out["tid"][:n], "op_begin": out["op_begin"][:n + 1], "ops": out["ops"][:m], "args": out["args"][:m]}
+    else:
+        res = {"tid": out["tid"][:n], "type": out["type"][:n], "params": out["params"][:n]}
+    return res, buf.n_fresh

@@ -47,6 +47,7 @@ int main(void) {
          sizeof(ltpg_batch), sizeof(ltpg_result), sizeof(ltpg_stats));
   printf("%zu %zu %zu\n", offsetof(ltpg_batch, batch_clock), offsetof(ltpg_batch, stream),
          offsetof(ltpg_result, stats));
+  printf("%zu %zu\n", sizeof(ltpg_batch_buf), offsetof(ltpg_batch_buf, n_txns));
   return 0;
 }
 """
@@ -62,6 +63,7 @@ int main(void) {
     assert sizes == [16, ctypes.sizeof(L.ltpg_config), ctypes.sizeof(L.ltpg_table_desc),
                      ctypes.sizeof(L.ltpg_batch), ctypes.sizeof(L.ltpg_result), ctypes.sizeof(L.ltpg_stats)]
     assert offs == [L.ltpg_batch.batch_clock.offset, L.ltpg_batch.stream.offset, L.ltpg_result.stats.offset]
+    assert [int(x) for x in lines[2].split()] == [ctypes.sizeof(L.ltpg_batch_buf), L.ltpg_batch_buf.n_txns.offset]
 
 
 def test_op_record_matches_generator_format():
@@ -128,3 +130,61 @@ def test_compact_params_roundtrip_and_size():
     used = np.diff(poffs.astype(np.int64))
     for r in range(len(b["type"])):
         assert (dec[r, :used[r]] == b["params"][r, :used[r]]).all(), r
+
+
+# ---- a9: the host retry loop (ltpg_compose_retry; host-only, runs without a GPU) ---------------
+def _np_retry_ops(prev, ab, fresh, cap_txns, cap_ops):
+    """Plain reference: aborted txns (ascending ranks) then the fresh prefix that fits."""
+    ob = prev["op_begin"]
+    txns = [(prev["tid"][r], prev["ops"][ob[r]:ob[r + 1]], prev["args"][ob[r]:ob[r + 1]]) for r in ab]
+    nops = sum(len(t[1]) for t in txns)
+    fb = fresh["op_begin"]
+    for j in range(len(fresh["tid"])):
+        k = fb[j + 1] - fb[j]
+        if len(txns) == cap_txns or nops + k > cap_ops:
+            break
+        txns.append((fresh["tid"][j], fresh["ops"][fb[j]:fb[j + 1]], fresh["args"][fb[j]:fb[j + 1]]))
+        nops += k
+    lens = np.array([len(t[1]) for t in txns], np.uint32)
+    return {"tid": np.array([t[0] for t in txns], np.uint64),
+            "op_begin": np.concatenate([[0], np.cumsum(lens)]).astype(np.uint32),
+            "ops": np.concatenate([t[1] for t in txns]), "args": np.concatenate([t[2] for t in txns])}
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_compose_retry_ops_equals_reference(seed):
+    import paper_conf_icde_wei0l0lzj024_b200 as L
+    from workloads.ycsb import YcsbWorkload
+    wl = YcsbWorkload(5000, theta=0.8, ops_per_txn=3 + seed % 3, seed=seed)
+    prev = wl.batch(300, 1, 0)
+    fresh = wl.batch(400, 301, 1)
+    rng = np.random.default_rng(seed)
+    ab = np.sort(rng.choice(300, size=rng.integers(0, 300), replace=False)).astype(np.uint32)
+    cap_t, cap_o = 350, (350 * (3 + seed % 3)) - 7 * seed
+    got, nf = L.compose_retry(prev, ab, fresh, cap_t, cap_o)
+    exp = _np_retry_ops(prev, ab, fresh, cap_t, cap_o)
+    assert nf == len(exp["tid"]) - len(ab)
+    for k in exp:
+        assert (got[k] == exp[k]).all(), k
+    assert (np.diff(got["tid"].astype(np.int64)) > 0).all()  # TID order preserved (P:120)
+
+
+def test_compose_retry_tpcc_and_errors():
+    import paper_conf_icde_wei0l0lzj024_b200 as L
+    from workloads import tpcc
+    wl = tpcc.TpccWorkload(2, seed=3, mode="strict", mix=tpcc.MIX_FULL)
+    prev = wl.batch(200, 1, 0)
+    fresh = wl.batch(200, 201, 1)
+    ab = np.array([0, 5, 17, 199], np.uint32)
+    got, nf = L.compose_retry(prev, ab, fresh, 150)
+    assert nf == 146 and len(got["tid"]) == 150
+    assert (got["tid"][:4] == prev["tid"][ab]).all() and (got["tid"][4:] == fresh["tid"][:146]).all()
+    assert (got["type"][:4] == prev["type"][ab]).all() and (got["params"][:4] == prev["params"][ab]).all()
+    assert (got["params"][4:] == fresh["params"][:146]).all()
+    for bad in (np.array([5, 5], np.uint32), np.array([7, 3], np.uint32), np.array([200], np.uint32)):
+        with pytest.raises(L.LtpgError):
+            L.compose_retry(prev, bad, fresh, 150)  # not ascending / out of range
+    with pytest.raises(L.LtpgError):
+        L.compose_retry(fresh, np.array([0], np.uint32), prev, 150)  # fresh TIDs must follow the retried
+    with pytest.raises(L.LtpgError):
+        L.compose_retry(prev, np.arange(151, dtype=np.uint32), fresh, 150)  # aborts alone overflow

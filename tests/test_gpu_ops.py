@@ -183,3 +183,23 @@ def concat(a, b):
     return {"tid": np.concatenate([a["tid"], b["tid"]]), "ops": np.concatenate([a["ops"], b["ops"]]),
             "args": np.concatenate([a["args"], b["args"]]),
             "op_begin": np.concatenate([a["op_begin"], b["op_begin"][1:] + a["op_begin"][-1]]).astype(np.uint32)}
+
+
+def test_closed_loop_with_compose_retry():
+    """a9 through the library: every next batch is ltpg_compose_retry(previous batch, its abort
+    list, fresh txns); GPU == oracle on every batch, and the retried txns keep their TIDs."""
+    wl = YcsbWorkload(10_000, theta=0.9, ops_per_txn=4, seed=0x17C0)
+    keys, cols = wl.initial_table()
+    descs = {0: tuple(wl.table_desc()[:3])}
+    tables = {0: (keys, cols)}
+    g, o = make_pair(descs, tables, 1024, 4096)
+    batch = wl.batch(1024, 1, 0)
+    tid = 1025
+    for b in range(12):
+        st = check_batch(g, o, batch, tables)
+        ab = np.nonzero(st == ST_CONFLICT)[0].astype(np.uint32)
+        fresh = wl.batch(1024, tid, b + 1)
+        nxt, nf = L().compose_retry(batch, ab, fresh, 1024, 4096)
+        assert (nxt["tid"][:len(ab)] == batch["tid"][ab]).all() and nf == 1024 - len(ab)
+        tid += nf
+        batch = nxt

@@ -9,8 +9,8 @@ NCU=/usr/local/cuda/bin/ncu
 mkdir -p gpurun_out
 export LTPG_NO_CLOCKS=1
 $NCU --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$W.csv \
-  python bench.py --workload $W --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/launch_$W.log 2>&1
+  python bench.py --workload $W --steps 2 --warmup 3 --no-cpu-baseline --no-closed-loop > gpurun_out/launch_$W.log 2>&1
 echo "launch list rc=$?"
 $NCU --set full --clock-control none --import-source on -k "regex:$K" -s $SKIP -c $CNT -f -o gpurun_out/full_$W \
-  python bench.py --workload $W --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/full_$W.log 2>&1
+  python bench.py --workload $W --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --no-closed-loop > gpurun_out/full_$W.log 2>&1
 echo "full rc=$?"
