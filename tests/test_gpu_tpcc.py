@@ -248,3 +248,34 @@ def test_many_districts_tiled_colscan():
         gk, gc = g.dump_table(t)
         ok, oc = o.dump_table(t)
         assert (gk == ok).all() and gc.shape == oc.shape and (gc == oc).all(), t
+
+
+@pytest.mark.parametrize("mode", ["strict", "delayed"])
+def test_ten_repeated_runs_identical(mode):
+    """PIN-8: the same closed loop run 10 times on fresh databases gives identical verdicts,
+    results and canonical state every time (atomics race in a different order on each run;
+    min marks, commutative adds and rank-ordered appends make the outcome unique, R20)."""
+    W, B = 2, 3000
+    wl = tpcc.TpccWorkload(W, seed=13, mode=mode, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    ref = None
+    for run in range(10):
+        g = L().tpcc_database(wl, max_txns=B, tables=tables, append_batches=5)
+        outs, pending, tid = [], None, 1
+        for bno in range(4):
+            fresh = wl.batch(B - (0 if pending is None else len(pending["tid"])), tid, bno)
+            tid += len(fresh["tid"])
+            batch = fresh if pending is None else {k: np.concatenate([pending[k], fresh[k]]) for k in fresh}
+            out = g.run_tpcc(batch, 2 + bno)
+            outs.append((out["status"].copy(), out["reads"].copy()))
+            ab = np.nonzero(out["status"] == ST_CONFLICT)[0]
+            pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
+        dumps = [g.dump_table(t) for t in range(9)]
+        g.close()
+        if ref is None:
+            ref = (outs, dumps)
+            continue
+        for (s0, r0), (s1, r1) in zip(ref[0], outs):
+            assert (s0 == s1).all() and (r0 == r1).all(), run
+        for (k0, c0), (k1, c1) in zip(ref[1], dumps):
+            assert (k0 is None or (k0 == k1).all()) and (c0 == c1).all(), run
