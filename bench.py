@@ -167,14 +167,13 @@ def ncu_traffic(workload, kernel_substr):
     p = os.path.join(ROOT, "profiles", "ncu_r01_%s.json" % workload)
     if not os.path.exists(p):
         return None
-    try:
+    try:  # summed over every instantiation that matches (the execute stage may be two launches)
         d = json.load(open(p))
-        for k, v in d.get("kernels", {}).items():
-            if kernel_substr in k:
-                return v.get("dram_bytes")
+        vals = [v.get("dram_bytes") for k, v in d.get("kernels", {}).items()
+                if kernel_substr in k and v.get("dram_bytes") is not None]
+        return sum(vals) if vals else None
     except Exception:
         return None
-    return None
 
 
 # ---- workloads ------------------------------------------------------------------------------
