@@ -1262,16 +1262,19 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     if (r < *m) atomicMin(m, r);
   }
   // block-aggregated counters and per-type list positions (one atomic per block and list)
-  const uint32_t ccnt[3] = {lines, pay_cust, no_home};  // misc[M_NO_LINES], misc[M_PAY], misc[M_NO]
-  uint32_t cbase[3];
-  block_reserve<3>(ccnt, tp.misc + M_NO_LINES, cbase);
-  uint32_t tcnt[NTYPES], tbase[NTYPES];
+  // slots 0..4: the per-type list flags (b.kcount), 5..7: misc[M_NO_LINES], misc[M_PAY],
+  // misc[M_NO]; every slot but the line count is a 0/1 flag (ballot scans), one barrier pair
+  uint32_t cnt[NTYPES + 3], base[NTYPES + 3];
 #pragma unroll
-  for (uint32_t k = 0; k < NTYPES; ++k) tcnt[k] = (t == k && !bad && touch) ? 1u : 0u;
-  block_reserve<NTYPES>(tcnt, b.kcount, tbase);
+  for (uint32_t k = 0; k < NTYPES; ++k) cnt[k] = (t == k && !bad && touch) ? 1u : 0u;
+  cnt[NTYPES] = lines;
+  cnt[NTYPES + 1] = pay_cust;
+  cnt[NTYPES + 2] = no_home;
+  block_reserve<NTYPES + 3, ((1u << NTYPES) - 1u) | (3u << (NTYPES + 1)), NTYPES>(cnt, b.kcount, base,
+                                                                                   tp.misc + M_NO_LINES);
 #pragma unroll
   for (uint32_t k = 0; k < NTYPES; ++k)
-    if (tcnt[k]) tp.list[(uint64_t)k * tp.max_txns + tbase[k]] = r;
+    if (cnt[k]) tp.list[(uint64_t)k * tp.max_txns + base[k]] = r;
   if (last_block(tp.misc + M_DONE_G) && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
 }
 
@@ -1292,7 +1295,7 @@ __global__ void __launch_bounds__(256) k_tpcc_relist(BatchDev b, TpccParams tp) 
   uint32_t cnt[NTYPES], base[NTYPES];
 #pragma unroll
   for (int k = 0; k < NTYPES; ++k) cnt[k] = (t == (uint32_t)k && b.status[r] == LTPG_ST_COMMIT) ? 1u : 0u;
-  block_reserve<NTYPES>(cnt, tp.misc + M_CCOUNT, base);
+  block_reserve<NTYPES, (1u << NTYPES) - 1u>(cnt, tp.misc + M_CCOUNT, base);
 #pragma unroll
   for (int k = 0; k < NTYPES; ++k)
     if (cnt[k]) tp.clist[(uint64_t)k * tp.max_txns + base[k]] = r;

@@ -372,22 +372,33 @@ __device__ __forceinline__ bool last_block(uint32_t* ctr) {
 // Every thread of a 256-thread block contributes cnt[k] items to list k; base[k] receives the
 // global position of its first item.  One atomicAdd per block and list (per-warp atomics on
 // a handful of counters serialised: ncu showed ~40% of a grouping kernel on them).
-template <int NK>
-__device__ __forceinline__ void block_reserve(const uint32_t (&cnt)[NK], uint32_t* counters, uint32_t (&base)[NK]) {
+// FLAGS: bit k set = cnt[k] is 0 or 1 for every thread, so the warp scan is one ballot + popc
+// instead of five shuffle steps.  Counters k < SPLIT live at counters0 + k, the others at
+// counters1 + (k - SPLIT): one pair of block barriers for two counter arrays.
+template <int NK, uint32_t FLAGS = 0u, int SPLIT = NK>
+__device__ __forceinline__ void block_reserve(const uint32_t (&cnt)[NK], uint32_t* counters0, uint32_t (&base)[NK],
+                                              uint32_t* counters1 = nullptr) {
   __shared__ uint32_t wsum[NK][8];
   __shared__ uint32_t gbase[NK];
   const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   uint32_t incl[NK];
 #pragma unroll
   for (int k = 0; k < NK; ++k) {
-    uint32_t x = cnt[k];
+    uint32_t x = cnt[k], tot;
+    if ((FLAGS >> k) & 1u) {
+      const uint32_t bal = __ballot_sync(0xffffffffu, x != 0u);
+      x = __popc(bal & (0xffffffffu >> (31 - lane)));
+      tot = __popc(bal);
+      if (lane == 0) wsum[k][wid] = tot;
+    } else {
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= (uint32_t)o) x += y;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      if (lane == 31) wsum[k][wid] = x;
     }
     incl[k] = x;
-    if (lane == 31) wsum[k][wid] = x;
   }
   __syncthreads();
   if (threadIdx.x < NK) {
@@ -398,7 +409,7 @@ __device__ __forceinline__ void block_reserve(const uint32_t (&cnt)[NK], uint32_
       wsum[k][w] = run;
       run += v;
     }
-    gbase[k] = run ? atomicAdd(counters + k, run) : 0u;
+    gbase[k] = run ? atomicAdd(k < SPLIT ? counters0 + k : counters1 + (k - SPLIT), run) : 0u;
   }
   __syncthreads();
 #pragma unroll
