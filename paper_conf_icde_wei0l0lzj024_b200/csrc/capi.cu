@@ -274,13 +274,22 @@ __global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint
 // batch start: append reservations cleared and the batch scalars stored where the kernels read
 // them -- from the arguments (direct enqueue) or, in a replayed graph, from the slot's pinned
 // host copy through its mapped address (read when the graph runs, not when it was captured)
+// + partition 0's small words (error, counters) and user-abort flags, which were two memset
+// nodes of their own ahead of every batch
 __global__ void k_batch_init(unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host,
-                             uint32_t epoch, long long clock) {
-  if (threadIdx.x < MAXT) reserve[threadIdx.x] = 0;
-  if (threadIdx.x == 0) {
-    vars->epoch = host ? host->epoch : epoch;
-    vars->clock = host ? host->clock : clock;
+                             uint32_t epoch, long long clock, uint32_t* small0, uint8_t* ua0, uint32_t n) {
+  if (blockIdx.x == 0) {
+    if (threadIdx.x < MAXT) reserve[threadIdx.x] = 0;
+    if (threadIdx.x < 16) small0[threadIdx.x] = 0;
+    if (threadIdx.x == 0) {
+      vars->epoch = host ? host->epoch : epoch;
+      vars->clock = host ? host->clock : clock;
+    }
   }
+  const uint32_t n16 = n / 16;  // ua0 is 256-byte aligned (cudaMalloc)
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += gridDim.x * blockDim.x)
+    reinterpret_cast<uint4*>(ua0)[i] = make_uint4(0, 0, 0, 0);
+  if (blockIdx.x == 0 && threadIdx.x < n % 16) ua0[16 * n16 + threadIdx.x] = 0;
 }
 __global__ void k_or_err(const uint32_t* src, uint32_t* dst) {
   if (*src) *dst |= *src;
@@ -837,13 +846,16 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // ---- the batch's device work (a2..a8), enqueued on `s` -- or captured into a graph ---------
   auto enqueue = [&](cudaStream_t s) -> int {
     static_assert(MAXT <= 32, "k_batch_init clears the reservations with one warp");
-    k_batch_init<<<1, 32, 0, s>>>(db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch,
-                                  b->batch_clock);
+    const uint32_t ib = std::min<uint32_t>(148u * 4u, std::max<uint32_t>(1u, (n / 16 + 255) / 256));
+    k_batch_init<<<ib, 256, 0, s>>>(db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch,
+                                    b->batch_clock, db->parts[0].small, db->parts[0].ua, n);
     note_launch();
     for (uint32_t p = 0; p < L; ++p) {
       Part& P = db->parts[p];
-      CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
-      if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
+      if (p) {  // partition 0: cleared by k_batch_init
+        CK(cudaMemsetAsync(P.small, 0, 16 * sizeof(uint32_t), s));
+        if (n) CK(cudaMemsetAsync(P.ua, 0, n, s));
+      }
       if (partitioned && n) {
         CK(cudaMemsetAsync(pb[p].res, 0, n_reads * sizeof(long long), s));
         CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
