@@ -277,10 +277,15 @@ __global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint
 // + partition 0's small words (error, counters) and user-abort flags, which were two memset
 // nodes of their own ahead of every batch
 __global__ void k_batch_init(unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host,
-                             uint32_t epoch, long long clock, uint32_t* small0, uint8_t* ua0, uint32_t n) {
+                             uint32_t epoch, long long clock, uint32_t* small0, uint8_t* ua0, uint32_t n,
+                             uint32_t* tmisc, uint32_t* dl_min, uint32_t nw) {
   if (blockIdx.x == 0) {
     if (threadIdx.x < MAXT) reserve[threadIdx.x] = 0;
     if (threadIdx.x < 16) small0[threadIdx.x] = 0;
+    if (tmisc) {  // TPC-C partition 0: batch counters, smallest Delivery rank per warehouse (none)
+      if (threadIdx.x < 16) tmisc[threadIdx.x] = 0;
+      for (uint32_t w = threadIdx.x; w <= nw; w += blockDim.x) dl_min[w] = ~0u;
+    }
     if (threadIdx.x == 0) {
       vars->epoch = host ? host->epoch : epoch;
       vars->clock = host ? host->clock : clock;
@@ -848,7 +853,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     static_assert(MAXT <= 32, "k_batch_init clears the reservations with one warp");
     const uint32_t ib = std::min<uint32_t>(148u * 4u, std::max<uint32_t>(1u, (n / 16 + 255) / 256));
     k_batch_init<<<ib, 256, 0, s>>>(db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch,
-                                    b->batch_clock, db->parts[0].small, db->parts[0].ua, n);
+                                    b->batch_clock, db->parts[0].small, db->parts[0].ua, n,
+                                    (ops_mode || !db->parts[0].tpcc.nw) ? nullptr : db->parts[0].tpcc.misc, db->parts[0].tpcc.dl_min,
+                                    db->parts[0].tpcc.nw);
     note_launch();
     for (uint32_t p = 0; p < L; ++p) {
       Part& P = db->parts[p];
@@ -900,7 +907,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (evp) CK(tmark(evp[3], s));
         launch_ops_detect(x, s);
       } else {
-        int rc = tpcc_front(db->parts[p].tpcc, x, s, evp);
+        int rc = tpcc_front(db->parts[p].tpcc, x, s, evp, p == 0);  // partition 0: cleared by k_batch_init
         if (rc) return fail(db, rc, "tpcc launch failed");
       }
     }

@@ -1672,12 +1672,15 @@ static uint32_t phase_grid(uint32_t n) {
   return (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
 }
 
-int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev) {
+// cleared: misc and dl_min were reset by the batch's first kernel (k_batch_init, partition 0)
+int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cleared) {
   if (!t.nw) return LTPG_EINVAL;
   const uint32_t n = b.n_txns;
   const TpccParams tp = params_of(t, b, false);
-  cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
-  cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
+  if (!cleared) {
+    cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
+    cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
+  }
   k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);  // + the capacity check (last block)
   note_launch(1);
   if (ev) record_stage(ev[2], s);

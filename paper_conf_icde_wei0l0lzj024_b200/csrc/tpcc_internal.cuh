@@ -86,7 +86,7 @@ void tpcc_free(TpccDev& t);
 int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, uint64_t n_rows,
                          uint32_t n_warehouses);
 // front: validate + lists, capacity, execute, detect;  back: o_id prefix, write-back, cursors
-int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev);
+int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cleared);
 int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s);
 // ORDER.aux[row] = first row of the order's ORDER_LINE rows when they are contiguous
 void tpcc_build_olrow(cudaStream_t s);
