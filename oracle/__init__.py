@@ -31,7 +31,8 @@ _lib = None
 def lib():
     global _lib
     if _lib is None:
-        L = ctypes.CDLL(build())
+        # LTPG_ORACLE_LIB: a deliberately mutated build (tools/mutate_oracle.py) -- tests only
+        L = ctypes.CDLL(os.environ.get("LTPG_ORACLE_LIB") or build())
         vp, u32, u64, i64, ip = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int
         L.orc_create.restype = vp
         L.orc_create.argtypes = [u32, u32]
