@@ -289,42 +289,88 @@ def step_algorithmic_bytes(batch):
     return exec_algorithmic_bytes(batch) + n * (40 + 24) + 10 * len(batch["tid"])
 
 
-# ---- reference arm: the CPU oracle ---------------------------------------------------------------
-def run_reference(args, name):
+# ---- host CPU ---------------------------------------------------------------------------------------
+def host_cpu():
+    """CPU model and the cores this process may use (report them)."""
+    model = None
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    try:
+        n = len(os.sched_getaffinity(0))
+    except AttributeError:
+        n = os.cpu_count() or 1
+    return {"model": model, "nproc": n}
+
+
+def _oracle_db(name, wl, threads):
     import oracle
     w = WORKLOADS[name]
-    wl = make_workload(name, 0)
-    t0 = time.time()
-    if w["kind"] == "ycsb":
-        db = oracle.ycsb_db(wl)
-    else:
-        db = oracle.tpcc_db(wl)
+    db = oracle.ycsb_db(wl) if w["kind"] == "ycsb" else oracle.tpcc_db(wl)
     if w.get("reorder"):
         db.set_reorder(True)
-    log("oracle load %.1fs" % (time.time() - t0))
-    sample = min(w["batch"], args.ref_sample)
+    db.set_threads(threads)
+    return db
+
+
+def _oracle_run(db, kind, b, clock):
+    t = time.perf_counter()
+    rc, st, _ = db.run_ops(b) if kind == "ycsb" else db.run_tpcc(b, clock=clock)
+    dt = time.perf_counter() - t
+    assert rc == 0
+    return int((st == 1).sum()), dt
+
+
+# ---- reference arm: the CPU oracle ---------------------------------------------------------------
+REF_BUDGET_S = 150.0   # timed oracle work of the whole reference run (the run must end in minutes)
+
+
+def run_reference(args, name):
+    """The reference arm is the CPU oracle (oracle/) on the box's host cores, on the same workload
+    and metric as our arm: fresh batches of the workload's full size when K of them fit in
+    REF_BUDGET_S on nproc threads (the oracle's SURVEY §8(d) threaded mode), else the largest
+    power-of-two sample that does.  Warm-up steps are small untimed samples."""
+    w = WORKLOADS[name]
+    kind = w["kind"]
+    wl = make_workload(name, 0)
+    cpu = host_cpu()
+    threads = args.ref_threads or cpu["nproc"]
+    t0 = time.time()
+    db = _oracle_db(name, wl, threads)
+    log("oracle load %.1fs (%d threads)" % (time.time() - t0, threads))
+    tid, clock = 1, 2
+    rate = None
+    for s in range(args.warmup):  # untimed; the last one estimates the processing rate
+        n = min(w["batch"], 1 << 14)
+        _, dt = _oracle_run(db, kind, wl.batch(n, tid, 10_000 + s), clock)
+        tid, clock = tid + n, clock + 1
+        rate = n / max(dt, 1e-6)
+    sample = w["batch"]
+    if args.ref_sample:
+        sample = min(sample, args.ref_sample)
+    while sample > 1024 and rate and sample / rate * args.steps > REF_BUDGET_S:
+        sample //= 2
     committed, secs = 0, 0.0
-    tid = 1
-    for s in range(args.warmup + args.steps):
-        b = wl.batch(sample, tid, 10_000 + s)
-        tid += sample
-        t = time.perf_counter()
-        if w["kind"] == "ycsb":
-            rc, st, _ = db.run_ops(b)
-        else:
-            rc, st, _ = db.run_tpcc(b, clock=2 + s)
-        dt = time.perf_counter() - t
-        assert rc == 0
-        if s >= args.warmup:
-            committed += int((st == 1).sum())
-            secs += dt
+    for s in range(args.steps):
+        c, dt = _oracle_run(db, kind, wl.batch(sample, tid, 20_000 + s), clock)
+        tid, clock = tid + sample, clock + 1
+        committed += c
+        secs += dt
     v = committed / secs if secs else 0.0
-    desc = "%d-txn batches of %s (full batch %d), %d timed" % (sample, name, w["batch"], args.steps)
+    desc = ("%d fresh %d-txn batches of %s (full batch %d%s), oracle on %d threads"
+            % (args.steps, sample, name, w["batch"], "" if sample == w["batch"] else ": sample bounded by the time budget",
+               threads))
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * secs / max(args.steps, 1),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64",
-            "data": "synthetic", "config": dict(config_of(name), parallelism="CPU oracle, 1 thread"),
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
+            "data": "synthetic",
+            "config": dict(config_of(name, batch=sample), parallelism="CPU oracle, %d threads" % threads),
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": desc,
+                             "cpu_model": cpu["model"], "nproc": cpu["nproc"]},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -339,27 +385,58 @@ def config_of(name, batch=None):
     return c
 
 
-def cpu_baseline(name, batch_host, wl):
-    """The oracle as it stands, 1 thread, on a bounded sample of the same workload."""
-    import oracle
+def cpu_baseline_child(name):
+    """Runs in a child process (python bench.py --cpu-baseline-child NAME), so the GPU arm's
+    process never maps the oracle: the oracle as it stands, 1 thread, on the first bench batch
+    (the same 2^k-txn batch the GPU times; bounded by the workload's size: ~10-30 s), then the
+    SURVEY §8(d) secondary run on nproc threads on a fresh copy of the same database."""
     w = WORKLOADS[name]
-    t0 = time.time()
-    db = oracle.ycsb_db(wl) if w["kind"] == "ycsb" else oracle.tpcc_db(wl)
-    if w.get("reorder"):
-        db.set_reorder(True)
-    load_s = time.time() - t0
-    n = len(batch_host["tid"])
-    budget = 25.0
-    t = time.perf_counter()
-    if w["kind"] == "ycsb":
-        rc, st, _ = db.run_ops(batch_host)
-    else:
-        rc, st, _ = db.run_tpcc(batch_host, clock=2)
-    dt = time.perf_counter() - t
-    del db
-    return {"value": float((st == 1).sum()) / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": "one full %d-txn batch of %s (oracle load %.1fs not timed; %.1fs of batch work)"
-                      % (n, name, load_s, dt), "seconds": dt, "budget_s": budget}
+    wl = make_workload(name, 0)
+    cpu = host_cpu()
+    out = {}
+    for threads in (1, cpu["nproc"]):
+        t0 = time.time()
+        db = _oracle_db(name, wl, threads)
+        load_s = time.time() - t0
+        c = dt = 0
+        nb = 0
+        while nb == 0 or (dt < 2.0 and nb < 64):  # the bench's batches 0, 1, ... (>= 2 s of work)
+            ci, dti = _oracle_run(db, w["kind"], wl.batch(w["batch"], 1 + nb * w["batch"], nb), 2 + nb)
+            c, dt, nb = c + ci, dt + dti, nb + 1
+        del db
+        out[threads] = (c, dt, load_s, nb)
+    c, dt, load_s, nb = out[1]
+    cn, dtn, _, nbn = out[cpu["nproc"]]
+    assert nb != nbn or c == cn, "threaded oracle disagrees with the single-threaded one"
+    res = {"value": c / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+           "sample": "the first %d full %d-txn batch(es) of %s, as the bench generates them (oracle load %.1fs "
+                     "not timed; %.1fs of batch work)" % (nb, w["batch"], name, load_s, dt),
+           "seconds": dt, "cpu_model": cpu["model"], "nproc": cpu["nproc"], "process": "child (bench.py)",
+           "threaded": {"value": cn / dtn, "unit": UNIT, "cores": cpu["nproc"], "seconds": dtn,
+                        "kind": "oracle, O1-O3 on nproc std::threads (SURVEY §8(d) secondary)"}}
+    print(json.dumps(res), flush=True)
+
+
+def cpu_baseline(name):
+    p = subprocess.run([sys.executable, os.path.abspath(__file__), "--cpu-baseline-child", name],
+                       capture_output=True, text=True, timeout=600)
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    if p.returncode or not lines:
+        return {"error": "cpu baseline child rc=%d: %s" % (p.returncode, p.stderr[-400:])}
+    return json.loads(lines[-1])
+
+
+def relaunch_under_torchrun(args):
+    """`bench.py --gpus N` outside torchrun: re-run this command as N ranks (one per GPU, or
+    sharing the GPUs there are) under torch.distributed.run on 127.0.0.1."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % args.gpus,
+           "--master-addr=127.0.0.1", "--master-port=%d" % port, os.path.abspath(__file__)] + sys.argv[1:]
+    log("relaunching as %d ranks: %s" % (args.gpus, " ".join(cmd)))
+    return subprocess.call(cmd)
 
 
 # ---- our arm -----------------------------------------------------------------------------------------
@@ -371,7 +448,9 @@ def main():
     ap.add_argument("--workload", default=os.environ.get("LTPG_BENCH_WORKLOAD", DEFAULT_WORKLOAD),
                     choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--ref-sample", type=int, default=1 << 17)
+    ap.add_argument("--ref-sample", type=int, default=0, help="cap the reference arm's batch (0: full)")
+    ap.add_argument("--ref-threads", type=int, default=0, help="reference arm oracle threads (0: nproc)")
+    ap.add_argument("--cpu-baseline-child", default=None, help=argparse.SUPPRESS)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-closed-loop", action="store_true")
@@ -380,6 +459,11 @@ def main():
                     help="N>1: peer-memory verdict exchange (default) or the ncclAllReduce baseline")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.cpu_baseline_child:
+        cpu_baseline_child(args.cpu_baseline_child)
+        return
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_under_torchrun(args))
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -452,8 +536,6 @@ def main():
         pin_batches.append({k: to_t(v, True) for k, v in hb.items()})
         if w["kind"] == "tpcc":
             pin_batches[-1]["compact"] = True
-    for db_ in dev_batches:  # keep logical lengths for the binding
-        pass
 
     # result buffers allocated once (device for the resident leg, pinned host for e2e), so no
     # allocation ever lands inside a timed step
@@ -697,12 +779,17 @@ def main():
                                         "ms_download")}}
     if args.flags:
         line["config"]["flags"] = args.flags
+    line["gpus_requested"] = args.gpus
+    line["gpus_active"] = min(world, ndev)
+    line["ranks"] = world
+    line["exchange"] = (None if world == 1 else
+                        "ncclAllReduce" if args.exchange == "nccl" else "peer-memory stores + signals (csrc/xchg.cu)")
     if shared:
         line["config"]["devices"] = ("%d ranks on %d GPU(s): functional check of the multi-rank path, "
                                      "not a scaling number" % (world, ndev))
     if world == 1 and not args.no_cpu_baseline:
         try:
-            line["cpu_baseline"] = cpu_baseline(name, host_batches[0], make_workload(name, 0))
+            line["cpu_baseline"] = cpu_baseline(name)
         except Exception as e:  # never lose the GPU number to the baseline leg
             line["cpu_baseline"] = {"error": repr(e)}
     print(json.dumps(line), flush=True)

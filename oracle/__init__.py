@@ -38,6 +38,7 @@ def lib():
         L.orc_create.argtypes = [u32, u32]
         L.orc_destroy.argtypes = [vp]
         L.orc_set_reorder.argtypes = [vp, ip]
+        L.orc_set_threads.argtypes = [vp, u32]
         L.orc_define_table.restype = ip
         L.orc_define_table.argtypes = [vp, u32, u32, vp, vp, u32, u32]
         L.orc_load_table.restype = ip
@@ -71,6 +72,10 @@ class OracleDB:
     def set_reorder(self, on=True):
         """NEXT-1 logical reordering: abort iff WAW or (RAW and WAR)."""
         self.L.orc_set_reorder(self.h, int(bool(on)))
+
+    def set_threads(self, n):
+        """SURVEY §8(d) secondary baseline: O1-O3 on n threads (1 = the plain oracle)."""
+        self.L.orc_set_threads(self.h, int(n))
 
     def close(self):
         if self.h:

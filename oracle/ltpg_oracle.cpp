@@ -1,6 +1,6 @@
 // LTPG CPU ORACLE -- TEST INFRASTRUCTURE ONLY.
 //
-// A plain, slow, single-threaded implementation of one LTPG batch under
+// A plain, slow implementation of one LTPG batch under
 // deterministic optimistic concurrency control (§IV, Alg. 1
 // P:128-157), written from the paper and the readings in DESIGN.md.  Only
 // tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl
@@ -22,6 +22,12 @@
 //   O5 output    status / reads / canonical table dump.
 // Conflict unit = (table, key, column group) (R4, P:239 row-level splitting).
 //
+// Single-threaded by default.  orc_set_threads(h, T > 1) is the SURVEY §8(d) secondary CPU
+// baseline: O1 runs over txns on T std::threads (every txn reads only the snapshot), O2 / O3
+// shard the conflict units over the threads by hash (each thread builds the min marks of its
+// own units, then tests the txns of a contiguous rank range against them); O4 stays serial.
+// tests/test_oracle_threads.py checks that it equals the single-threaded run.
+//
 // Parity: pinned by tests/test_oracle_*.py (Example 2/3 of the paper, brute
 // force of the pairwise definition, serial replay, TPC-C consistency
 // conditions, Table VI "no" rows, closed forms).
@@ -29,6 +35,7 @@
 #include <cstdint>
 #include <cstring>
 #include <map>
+#include <thread>
 #include <unordered_map>
 #include <unordered_set>
 #include <vector>
@@ -117,7 +124,21 @@ struct Db {
   bool by_name_built = false;
   std::vector<double> stage_ns;
   bool reorder = false;  // NEXT-1 logical reordering
+  unsigned threads = 1;  // SURVEY §8(d) secondary baseline (orc_set_threads)
 };
+
+// Run f(lo, hi) over [0, n) split into T contiguous ranges on T threads.
+template <class F>
+void parallel_ranges(uint32_t n, unsigned T, F f) {
+  if (T <= 1 || n < 2 * T) {
+    f(0u, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (unsigned k = 0; k < T; ++k)
+    th.emplace_back([&, k] { f(uint32_t(uint64_t(n) * k / T), uint32_t(uint64_t(n) * (k + 1) / T)); });
+  for (auto& t : th) t.join();
+}
 
 // ---------------------------------------------------------------------------
 // O2 + O3: marks and the commit rule.
@@ -165,6 +186,54 @@ void decide(const std::vector<TxnExec>& ex, std::vector<uint8_t>& status, bool r
     const bool abort = reorder ? (waw || (raw && war)) : (waw || raw);
     status[r] = abort ? ST_CONFLICT : (ex[r].user_abort ? ST_USER_ABORT : ST_COMMIT);
   }
+}
+
+// The same O2 + O3 with T threads: thread k builds the min marks of the units u with
+// hash(u) % T == k (over all txns, in any order: min is order-free), then every thread tests
+// the txns of its rank range against the shard maps (read-only).  Identical to decide().
+void decide_threads(const std::vector<TxnExec>& ex, std::vector<uint8_t>& status, bool reorder, unsigned T) {
+  const uint32_t n = ex.size();
+  using Map = std::unordered_map<Unit, uint32_t, UnitHash>;
+  std::vector<Map> minR(T), minW(T), minA(T);
+  UnitHash H;
+  std::vector<std::thread> th;
+  for (unsigned k = 0; k < T; ++k)
+    th.emplace_back([&, k] {
+      for (uint32_t r = 0; r < n; ++r)
+        for (const Access& a : ex[r].acc) {
+          if (H(a.u) % T != k) continue;
+          Map& m = a.acc == ACC_R ? minR[k] : (a.acc == ACC_W ? minW[k] : minA[k]);
+          auto it = m.find(a.u);
+          if (it == m.end()) m.emplace(a.u, r);
+          else if (r < it->second) it->second = r;
+        }
+    });
+  for (auto& t : th) t.join();
+  auto get = [&](const std::vector<Map>& ms, const Unit& u) -> uint32_t {
+    const Map& m = ms[H(u) % T];
+    auto it = m.find(u);
+    return it == m.end() ? UINT32_MAX : it->second;
+  };
+  status.assign(n, ST_COMMIT);
+  parallel_ranges(n, T, [&](uint32_t lo, uint32_t hi) {
+    for (uint32_t r = lo; r < hi; ++r) {
+      bool waw = false, raw = false, war = false;
+      for (const Access& a : ex[r].acc) {
+        const uint32_t w = get(minW, a.u), ad = get(minA, a.u), rd = get(minR, a.u);
+        if (a.acc == ACC_R) {
+          if (std::min(w, ad) < r) raw = true;
+        } else if (a.acc == ACC_W) {
+          if (std::min(w, ad) < r) waw = true;
+          if (rd < r) war = true;
+        } else {
+          if (w < r) waw = true;
+          if (rd < r) war = true;
+        }
+      }
+      const bool abort = reorder ? (waw || (raw && war)) : (waw || raw);
+      status[r] = abort ? ST_CONFLICT : (ex[r].user_abort ? ST_USER_ABORT : ST_COMMIT);
+    }
+  });
 }
 
 // O4: apply one buffered effect (writeMem).
@@ -647,6 +716,9 @@ void orc_destroy(void* h) { delete static_cast<Db*>(h); }
 // NEXT-1: logical reordering (commit rule WAW or (RAW and WAR) aborts)
 void orc_set_reorder(void* h, int on) { static_cast<Db*>(h)->reorder = on != 0; }
 
+// SURVEY §8(d) secondary baseline: O1-O3 on `threads` std::threads (1 = the plain oracle)
+void orc_set_threads(void* h, uint32_t threads) { static_cast<Db*>(h)->threads = threads ? threads : 1; }
+
 int orc_define_table(void* h, uint32_t t, uint32_t n_cols, const uint8_t* group, const uint8_t* is_add,
                      uint32_t n_groups, uint32_t has_pk) {
   Db& db = *static_cast<Db*>(h);
@@ -694,11 +766,14 @@ int orc_run_ops(void* h, uint32_t n, const uint64_t* tid, const uint32_t* op_beg
   int rc = validate_ops(db, n, tid, op_begin, ops);
   if (rc) return rc;
   std::vector<TxnExec> ex(n);
-  for (uint32_t r = 0; r < n; ++r)  // O1 (rank order irrelevant: all reads hit S)
-    for (uint32_t i = op_begin[r]; i < op_begin[r + 1]; ++i)
-      exec_op(db, read_op(ops + 16ull * i), args[i], ex[r], &reads[i]);
+  parallel_ranges(n, db.threads, [&](uint32_t lo, uint32_t hi) {
+    for (uint32_t r = lo; r < hi; ++r)  // O1 (rank order irrelevant: all reads hit S)
+      for (uint32_t i = op_begin[r]; i < op_begin[r + 1]; ++i)
+        exec_op(db, read_op(ops + 16ull * i), args[i], ex[r], &reads[i]);
+  });
   std::vector<uint8_t> st;
-  decide(ex, st, db.reorder);  // O2 + O3
+  if (db.threads > 1) decide_threads(ex, st, db.reorder, db.threads);
+  else decide(ex, st, db.reorder);  // O2 + O3
   for (uint32_t r = 0; r < n; ++r) {  // O4 in TID order
     status[r] = st[r];
     if (st[r] != ST_COMMIT) continue;
@@ -717,21 +792,27 @@ int orc_run_tpcc(void* h, uint32_t n, const uint64_t* tid, const uint8_t* type, 
   if (rc) return rc;
   if (!db.by_name_built) build_by_name(db);
   std::vector<TxnExec> ex(n);
-  for (uint32_t r = 0; r < n; ++r) {  // O1
-    ProcCtx x{db, ex[r], clock, tid[r]};
-    const uint8_t* p = params + 128ull * r;
-    int64_t* res = results + 4ull * r;
-    switch (type[r]) {
-      case P_NEWORDER: proc_neworder(x, p, res); break;
-      case P_PAYMENT: proc_payment(x, p, res); break;
-      case P_ORDERSTATUS: proc_orderstatus(x, p, res); break;
-      case P_DELIVERY: proc_delivery(x, p, res); break;
-      case P_STOCKLEVEL: proc_stocklevel(x, p, res); break;
+  std::vector<uint8_t> bad(n, 0);
+  parallel_ranges(n, db.threads, [&](uint32_t lo, uint32_t hi) {
+    for (uint32_t r = lo; r < hi; ++r) {  // O1
+      ProcCtx x{db, ex[r], clock, tid[r]};
+      const uint8_t* p = params + 128ull * r;
+      int64_t* res = results + 4ull * r;
+      switch (type[r]) {
+        case P_NEWORDER: proc_neworder(x, p, res); break;
+        case P_PAYMENT: proc_payment(x, p, res); break;
+        case P_ORDERSTATUS: proc_orderstatus(x, p, res); break;
+        case P_DELIVERY: proc_delivery(x, p, res); break;
+        case P_STOCKLEVEL: proc_stocklevel(x, p, res); break;
+      }
+      bad[r] = !x.ok;
     }
-    if (!x.ok) return ORC_EINTERNAL;
-  }
+  });
+  for (uint32_t r = 0; r < n; ++r)
+    if (bad[r]) return ORC_EINTERNAL;
   std::vector<uint8_t> st;
-  decide(ex, st, db.reorder);  // O2 + O3
+  if (db.threads > 1) decide_threads(ex, st, db.reorder, db.threads);
+  else decide(ex, st, db.reorder);  // O2 + O3
   for (uint32_t r = 0; r < n; ++r) {  // O4: committed write sets (a unit has at most one plain
     status[r] = st[r];               // writer; adds commute; fetch pre-images in TID order)
     if (st[r] != ST_COMMIT) continue;

@@ -51,6 +51,10 @@ Nccl g_nccl;
 uint64_t g_tab_versions = 0;
 constexpr uint64_t LARGE_BUCKET_BYTES = 64ull << 20;  // NEXT-3 bucket memory cap per table     // process-wide: every table load gets a new version
 uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __constant__
+// per device: recorded after every batch's device work (any db).  A db that re-uploads the
+// constant bank (another db's tables were there) first waits on it, so the kernels of the
+// previous owner -- possibly still running on another stream -- never see the new tables.
+cudaEvent_t g_const_users[64] = {nullptr};
 
 // per-partition scratch (one per logical partition handled by this process)
 struct Part {
@@ -103,7 +107,7 @@ struct Slot {
   uint32_t* h_small_dev = nullptr;         // its device-side address (written by k_publish)
   cudaEvent_t ev[8]{};
   cudaEvent_t h2d_done = nullptr, comp_done = nullptr, out_done = nullptr;
-  bool pending = false, timing = false, host_out = false;
+  bool pending = false, timing = false, host_out = false, empty = false;
   ltpg_result* res = nullptr;
   uint64_t launches0 = 0;
   BatchVars* d_vars = nullptr;             // this batch's epoch / clock (read by the kernels)
@@ -120,6 +124,7 @@ struct ltpg_db {
   bool poisoned = false;
   std::string last_error;
   uint32_t epoch = 0;
+  uint32_t mark_window = 0;  // epoch / 255 of the last batch: a new window clears the marks
   uint32_t n_tables = 0;
   uint64_t tab_version = 0;
   uint32_t nparts = 1;     // global logical partitions = world * loopback
@@ -146,6 +151,9 @@ struct ltpg_db {
   uint64_t submitted = 0;
   cudaStream_t h2d = nullptr, d2h = nullptr;
   cudaStream_t cap = nullptr;              // batch graphs are captured here (never executes work)
+  // batches execute in submission order even when the caller passes different streams:
+  // each batch's first kernel waits on the previous batch's compute (they share scratch)
+  cudaEvent_t last_comp = nullptr;
   uint64_t graph_uses = 0;
   // a8 (commit bitmask, abort list) runs on its own stream once the verdicts are final,
   // concurrently with write-back; it has its own scan scratch
@@ -372,6 +380,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaStreamCreateWithFlags(&db->cap, cudaStreamNonBlocking));
   CK(cudaEventCreateWithFlags(&db->status_ready, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&db->fin_done, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&db->last_comp, cudaEventDisableTiming));
+  if (!g_const_users[cfg->device % 64]) CK(cudaEventCreateWithFlags(&g_const_users[cfg->device % 64], cudaEventDisableTiming));
   CK(dmalloc(&db->d_scan_fin, scan_scratch_words(n) + 16));
   CK(dmalloc(&db->d_fc_state, (n + 1023) / 1024 + 1));
   CK(cudaMemset(db->d_fc_state, 0, ((n + 1023) / 1024 + 1) * sizeof(unsigned long long)));
@@ -447,6 +457,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   if (db->cap) cudaStreamDestroy(db->cap);
   if (db->status_ready) cudaEventDestroy(db->status_ready);
   if (db->fin_done) cudaEventDestroy(db->fin_done);
+  if (db->last_comp) cudaEventDestroy(db->last_comp);
   if (db->d_scan_fin) cudaFree(db->d_scan_fin);
   if (db->d_fc_state) cudaFree(db->d_fc_state);
   if (db->d_fc_ctr) cudaFree(db->d_fc_ctr);
@@ -653,7 +664,9 @@ int finish_slot(ltpg_db* db, Slot& S) {
   if (err & ERR_EINVAL) return fail(db, LTPG_EINVAL, "invalid batch (validated on device; nothing changed)");
   if (err & ERR_ECAPACITY) return fail(db, LTPG_ECAPACITY, "append capacity exceeded (nothing changed)");
   if (S.host_out) *S.res->n_aborted = S.h_small[16];
-  if (S.timing) {
+  if (S.timing && S.empty) {  // nothing ran: no stage events were recorded
+    *S.res->stats = ltpg_stats{};
+  } else if (S.timing) {
     ltpg_stats* st = S.res->stats;
     float ms[7] = {0};
     for (int i = 0; i < 6; ++i) CK(cudaEventElapsedTime(&ms[i], S.ev[i], S.ev[i + 1]));
@@ -699,6 +712,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if ((b->flags & LTPG_BATCH_COMPACT_PARAMS) && (ops_mode || !b->proc_offsets))
     return fail(db, LTPG_EINVAL, "LTPG_BATCH_COMPACT_PARAMS needs a TPCC batch with proc_offsets");
   if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
+  if (!ops_mode && b->proc_offsets && !b->inputs_on_device && b->proc_offsets[n] > (uint64_t)n * LTPG_PARAM_BYTES)
+    return fail(db, LTPG_EINVAL, "packed params too large");
+  // every host-side validation is above this line: from here on the batch is submitted
   Slot& S = db->slots[db->submitted % 3];
   if (S.pending) return fail(db, LTPG_EINVAL, "three batches already in flight: ltpg_wait_batch first");
   ++db->submitted;
@@ -712,6 +728,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   S.res = res;
   S.host_out = !res->outputs_on_device;
   S.launches0 = g_kernel_launches;
+  S.empty = n == 0;
   ++db->epoch;
   // ---- a1: upload on the copy stream (overlaps the previous batch's kernels) ------------------
   BatchDev bd{};
@@ -755,8 +772,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     } else {
       CK(cudaMemcpyAsync(S.d_ptype, b->proc_type, n, h2d, db->h2d));
       if (b->proc_offsets) {  // packed blocks: offsets + used bytes only, expanded on the GPU
-        const uint64_t packed = b->proc_offsets[n];
-        if (packed > (uint64_t)n * LTPG_PARAM_BYTES) return fail(db, LTPG_EINVAL, "packed params too large");
+        const uint64_t packed = b->proc_offsets[n];  // <= n * 128 (checked before submission)
         CK(cudaMemcpyAsync(S.d_offsets, b->proc_offsets, (n + 1) * sizeof(uint32_t), h2d, db->h2d));
         CK(cudaMemcpyAsync(S.d_packed, b->proc_params, packed, h2d, db->h2d));
       } else {
@@ -767,8 +783,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     }
     CK(cudaEventRecord(S.h2d_done, db->h2d));
   }
-  // kernels of this batch: after its upload and after the slot's previous outputs were read
+  // kernels of this batch: after its upload, after the slot's previous outputs were read and
+  // after the previous batch's compute (it may have run on another stream)
   CK(cudaStreamWaitEvent(s, S.out_done, 0));
+  if (db->submitted > 1) CK(cudaStreamWaitEvent(s, db->last_comp, 0));
   if (timing) CK(cudaEventRecord(S.ev[0], s));
   CK(cudaMemsetAsync(S.d_small, 0, 17 * sizeof(uint32_t), s));
   if (!n && !S.host_out) CK(cudaMemsetAsync(res->n_aborted, 0, sizeof(uint32_t), s));
@@ -783,12 +801,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
   if (g_uploaded[db->device % 64] != db->tab_version) {
+    CK(cudaStreamWaitEvent(s, g_const_users[db->device % 64], 0));  // the previous owner's kernels
     upload_tables_common(db->d_tab, s);
     upload_tables_ops(db->d_tab, s);
     upload_tables_tpcc(db->d_tab, s);
     g_uploaded[db->device % 64] = db->tab_version;
   }
-  if (db->epoch % 255 == 0) {  // the epoch tag byte wraps 0 -> 254: clear every mark
+  if (db->epoch / 255 != db->mark_window) {  // the epoch tag byte wraps 0 -> 254: clear every mark
+    db->mark_window = db->epoch / 255;
     for (uint32_t t = 0; t < db->n_tables; ++t) {
       const DevTable& T = db->h_tab[t];
       const size_t units = T.capacity * T.n_groups * sizeof(mark_t);
@@ -1031,6 +1051,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   }
   if (timing) CK(cudaEventRecord(S.ev[6], s));
   CK(cudaEventRecord(S.comp_done, s));
+  CK(cudaEventRecord(db->last_comp, s));
+  CK(cudaEventRecord(g_const_users[db->device % 64], s));
   // ---- a8: results: D2H on the copy stream (overlaps the next batch's kernels) ------------------
   cudaStream_t os = S.host_out ? db->d2h : s;
   if (S.host_out) CK(cudaStreamWaitEvent(db->d2h, S.comp_done, 0));
