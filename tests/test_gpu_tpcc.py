@@ -279,3 +279,40 @@ def test_ten_repeated_runs_identical(mode):
             assert (s0 == s1).all() and (r0 == r1).all(), run
         for (k0, c0), (k1, c1) in zip(ref[1], dumps):
             assert (k0 is None or (k0 == k1).all()) and (c0 == c1).all(), run
+
+
+@pytest.mark.parametrize("what", ["item0", "item_big", "qty0", "qty11", "supply_w", "dup_item", "dup_far"])
+def test_neworder_line_validation_in_execute(what):
+    """Unpartitioned batches validate NewOrder lines in execute (the grouping kernel reads only
+    the 16-byte headers): every malformed line is EINVAL with nothing changed, and the database
+    keeps running the next batch == oracle."""
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=23, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3)
+    o = oracle.tpcc_db(wl, tables)
+    b = wl.batch(1000, 1, 0)
+    no = np.nonzero((b["type"] == NEW_ORDER) & (b["params"][:, 3] >= 14))[0][3]
+    p = b["params"][no]
+    line = lambda l: p[8 + 8 * l: 16 + 8 * l]  # noqa: E731
+    if what == "item0":
+        line(2)[:4] = 0
+    elif what == "item_big":
+        line(13)[:4] = np.array([100002], "<u4").view(np.uint8)
+    elif what == "qty0":
+        line(0)[6] = 0
+    elif what == "qty11":
+        line(5)[6] = 11
+    elif what == "supply_w":
+        line(7)[4:6] = np.array([3], "<u2").view(np.uint8)   # W = 2
+    elif what == "dup_item":
+        line(1)[:4] = line(2)[:4]                          # same lane (lines 0..3)
+    elif what == "dup_far":
+        line(13)[:4] = line(0)[:4]                         # lanes 0 and 3
+    assert o.run_tpcc(b, 2)[0] == oracle.ORC_EINVAL
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(b, 2)
+    assert e.value.rc == lib.LTPG_EINVAL
+    compare_tables(g, o)                                   # nothing changed
+    compare(g, o, wl.batch(1000, 5000, 1), 3)              # and the db still works
+    compare_tables(g, o)
