@@ -131,10 +131,14 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
                                               two kernels with global per-kind lists          */
 #define LTPG_FLAG_NCCL_EXCHANGE (1u << 4)  /* world > 1, A/B baseline: exchange verdicts and result
                                               sums with ncclAllReduce instead of peer memory   */
-#define LTPG_FLAG_LARGE_BUCKETS (1u << 5)  /* NEXT-3: tables with E = max_txns/rows > 1
-                                              record marks in large-sized buckets of
-                                              ceil(E/32)*32 sub-slots (TID mod s_u), folded per
-                                              unit before detection; result-identical          */
+#define LTPG_FLAG_LARGE_BUCKETS (1u << 5)  /* NEXT-3: popularity is identified per batch
+                                              ("in real time"): a table with E = T/D > 1
+                                              (T = txns of the batch accessing it, D = its loaded
+                                              rows) records that batch's marks in large-sized
+                                              buckets of ceil(E/32)*32 sub-slots (TID mod s_u),
+                                              folded per unit before detection.  Buckets are
+                                              allocated at load for tables with max_txns/rows > 1
+                                              (at most 64 MB each).  Result-identical          */
 #define LTPG_FLAG_GRAPH         (1u << 6)  /* run each batch's device work as a captured CUDA graph,
                                               replayed for later batches of the same shape
                                               (see ltpg_run_batch); result-identical          */
@@ -254,6 +258,8 @@ typedef struct {
   float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;
   uint32_t n_commit, n_conflict, n_user_abort;
   uint32_t n_kernels;           /* kernels this library launched for the batch */
+  uint32_t popular_tables;      /* NEXT-3 (LTPG_FLAG_LARGE_BUCKETS): bit t = table t was popular in
+                                   this batch (E = T/D > 1) and marked into large buckets */
 } ltpg_stats;
 
 typedef struct {
@@ -278,6 +284,12 @@ LTPG_API int ltpg_run_batch(ltpg_db* db, const ltpg_batch* batch, ltpg_result* r
 
 /* Complete an asynchronously submitted batch (see LTPG_BATCH_ASYNC). */
 LTPG_API int ltpg_wait_batch(ltpg_db* db, ltpg_result* result);
+
+/* NEXT-3 / Table VIII: bytes of table t's conflict marks -- standard-sized (one word per
+ * unit and kind) and large-sized buckets (LTPG_FLAG_LARGE_BUCKETS), as allocated -- and the bucket
+ * size s_u allocated (1: none).  Host outputs; EINVAL for a bad table id. */
+LTPG_API int ltpg_mark_memory(ltpg_db* db, uint32_t table_id, uint64_t* standard_bytes, uint64_t* large_bytes,
+                              uint32_t* su);
 
 /* Canonical dump (valid rows only): keyed tables sorted by key, keyless tables by
  * the full column tuple.  Call with keys == cols == NULL to get *n_rows only.

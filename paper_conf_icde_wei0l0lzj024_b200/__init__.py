@@ -69,7 +69,8 @@ class ltpg_stats(ctypes.Structure):
     _fields_ = [("ms_upload", ctypes.c_float), ("ms_group", ctypes.c_float), ("ms_exec", ctypes.c_float),
                 ("ms_detect", ctypes.c_float), ("ms_exchange", ctypes.c_float),
                 ("ms_writeback", ctypes.c_float), ("ms_download", ctypes.c_float),
-                ("n_commit", c_u32), ("n_conflict", c_u32), ("n_user_abort", c_u32), ("n_kernels", c_u32)]
+                ("n_commit", c_u32), ("n_conflict", c_u32), ("n_user_abort", c_u32), ("n_kernels", c_u32),
+                ("popular_tables", c_u32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -107,6 +108,8 @@ class ltpg_batch_buf(ctypes.Structure):
 _lib.ltpg_compose_retry.restype = c_int
 _lib.ltpg_compose_retry.argtypes = [ctypes.POINTER(ltpg_batch), c_vp, c_u32, ctypes.POINTER(ltpg_batch),
                                     ctypes.POINTER(ltpg_batch_buf)]
+_lib.ltpg_mark_memory.restype = c_int
+_lib.ltpg_mark_memory.argtypes = [c_vp, c_u32, ctypes.POINTER(c_u64), ctypes.POINTER(c_u64), ctypes.POINTER(c_u32)]
 _lib.ltpg_version.restype = ctypes.c_char_p
 _lib.ltpg_version.argtypes = []
 
@@ -122,12 +125,13 @@ ltpg_wait_batch = _lib.ltpg_wait_batch
 ltpg_peer_handle = _lib.ltpg_peer_handle
 ltpg_connect_peers = _lib.ltpg_connect_peers
 ltpg_compose_retry = _lib.ltpg_compose_retry
+ltpg_mark_memory = _lib.ltpg_mark_memory
 LTPG_BATCH_ASYNC = 1
 LTPG_BATCH_COMPACT_PARAMS = 2
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
             "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers",
-            "ltpg_compose_retry"]
+            "ltpg_compose_retry", "ltpg_mark_memory"]
 
 
 class LtpgError(RuntimeError):
@@ -293,6 +297,12 @@ class Database:
         if wait and not device_out and want_reads:
             out["reads"] = out["reads"].reshape(n, 4)
         return out
+
+    def mark_memory(self, t):
+        """(standard bytes, large-bucket bytes, allocated s_u) of table t's conflict marks (Table VIII)."""
+        a, b, su = c_u64(0), c_u64(0), c_u32(0)
+        self._check(ltpg_mark_memory(self.h, t, ctypes.byref(a), ctypes.byref(b), ctypes.byref(su)))
+        return a.value, b.value, su.value
 
     def dump_table(self, t):
         nr = c_u64(0)

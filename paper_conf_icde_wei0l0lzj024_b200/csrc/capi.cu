@@ -141,6 +141,7 @@ struct ltpg_db {
   // the ORDER -> ORDER_LINE map rebuild).
   uint32_t idx_lag = 0;
   unsigned long long* d_idx_from = nullptr;  // [MAXT]
+  uint16_t* d_su = nullptr;                  // [MAXT] NEXT-3: this batch's bucket size per table
   std::vector<Part> parts;
   uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
@@ -342,6 +343,8 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaMemset(db->d_nrows, 0, MAXT * sizeof(unsigned long long)));
   CK(dmalloc(&db->d_reserve, MAXT));
   CK(dmalloc(&db->d_idx_from, MAXT));
+  CK(dmalloc(&db->d_su, MAXT));
+  CK(cudaMemset(db->d_su, 0, MAXT * sizeof(uint16_t)));
   CK(dmalloc(&db->d_dense_live, 1));
   CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
@@ -403,6 +406,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
     P.tpcc.h_tab = db->h_tab;
     P.tpcc.n_tab = cfg->n_tables;
+    P.tpcc.d_su = db->d_su;
     ptrs[p] = P.lflag;
     ptrs[64 + p] = P.small;
     ptrs[128 + p] = P.res;
@@ -433,7 +437,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
   void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_xchg, db->d_ptrs, db->d_scan,
-                  db->d_idx_from};
+                  db->d_idx_from, db->d_su};
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
@@ -508,6 +512,7 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   T.defined = 1;
   T.owner_rule = d->owner_rule;
   T.capacity = cap;
+  T.id = t;
   // row-block layout: mutable block (non-static columns), static block; marks separate
   uint32_t n_dyn = 0, n_stat = 0;
   for (uint32_t c = 0; c < d->n_cols; ++c) (d->col_group[c] == LTPG_STATIC ? n_stat : n_dyn)++;
@@ -681,6 +686,7 @@ int finish_slot(ltpg_db* db, Slot& S) {
     st->n_commit = S.h_small[8];
     st->n_conflict = S.h_small[9];
     st->n_user_abort = S.h_small[10];
+    st->popular_tables = S.h_small[11];
   }
   return LTPG_OK;
 }
@@ -904,9 +910,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (timed) CK(tmark(S.ev[1], s));
     if (!n) return LTPG_OK;
     // ---- a1..a6 per partition: validate + warp division, claims, execute + marks, detect --------
+    // NEXT-3 real-time popularity: OPS batches know T (every txn may access every table)
+    // before their front end marks; TPC-C counts per procedure after grouping (tpcc_front)
+    if (ops_mode) launch_popularity(db->h_tab, db->n_tables, nullptr, n, db->d_su, S.d_small + 11, s);
     for (uint32_t p = 0; p < L; ++p) {
       BatchDev& x = pb[p];
       cudaEvent_t* evp = (timed && p == L - 1) ? S.ev : nullptr;
+      db->parts[p].tpcc.popular = S.d_small + 11;
       if (ops_mode) {
         if (fused) {  // validate + warp-local division + execute; INSERTs after their claims
           launch_ops_fused(db->n_tables, x, filter, s);
@@ -923,7 +933,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
           if (evp) CK(tmark(evp[2], s));
           launch_ops_exec(x, grouped, filter, s);
         }
-        launch_bucket_reduce(db->h_tab, db->n_tables, s);  // NEXT-3 large-sized buckets (if any)
+        launch_bucket_reduce(db->h_tab, db->n_tables, db->d_su, s);  // NEXT-3 large-sized buckets (if any)
         if (evp) CK(tmark(evp[3], s));
         launch_ops_detect(x, s);
       } else {
@@ -1115,6 +1125,19 @@ int ltpg_connect_peers(ltpg_db* db, const void* handles) {
     db->xpeers.base[q] = static_cast<char*>(p);
   }
   db->connected = true;
+  return LTPG_OK;
+}
+
+int ltpg_mark_memory(ltpg_db* db, uint32_t t, uint64_t* standard_bytes, uint64_t* large_bytes, uint32_t* su) {
+  if (!db || t >= db->n_tables || !standard_bytes || !large_bytes) return fail(db, LTPG_EINVAL, "bad mark_memory args");
+  const DevTable& T = db->h_tab[t];
+  const uint64_t na = __builtin_popcount(T.add_groups);
+  *standard_bytes = (T.wmarks ? T.capacity * T.n_groups : 0) * sizeof(mark_t) +
+                    (T.amarks ? T.capacity * na : 0) * sizeof(mark_t) +
+                    (T.rmarks ? T.capacity * T.n_groups : 0) * sizeof(mark_t);
+  const uint64_t units = (T.sub[0] ? (uint64_t)T.n_groups : 0) + (T.sub[1] ? na : 0) + (T.sub[2] ? (uint64_t)T.n_groups : 0);
+  *large_bytes = T.su > 1 ? units * T.sub_rows * T.su * sizeof(mark_t) : 0;
+  if (su) *su = T.su > 1 ? T.su : 1;
   return LTPG_OK;
 }
 

@@ -419,7 +419,10 @@ void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uin
 // bytes, so a stale word or sub-slot never hides a mark of this batch, and mark_rank ignores
 // it when nothing of this batch is there.  Bucket (gi, row) belongs to word gi*capacity + row.
 __global__ void __launch_bounds__(256) k_bucket_reduce(const mark_t* __restrict__ sub, mark_t* word, uint32_t groups,
-                                                       uint32_t rows, uint64_t capacity, uint32_t su) {
+                                                       uint32_t rows, uint64_t capacity, uint32_t stride,
+                                                       const uint16_t* d_su, uint32_t t) {
+  const uint32_t su = d_su[t];  // this batch's bucket size (<= stride, the allocated one)
+  if (su <= 1) return;          // standard-sized this batch: the marks are in the words already
   const uint32_t per = (su + 1023) / 1024;
   const uint64_t units = (uint64_t)groups * rows;
   const uint32_t lane = threadIdx.x & 31;
@@ -429,13 +432,13 @@ __global__ void __launch_bounds__(256) k_bucket_reduce(const mark_t* __restrict_
     const uint32_t j0 = (uint32_t)(c % per) * 1024u;
     const uint32_t j1 = min(su, j0 + 1024u);
     mark_t m = 0xFFFFFFFFu;
-    for (uint32_t j = j0 + lane; j < j1; j += 32) m = min(m, __ldcg(sub + u * su + j));
+    for (uint32_t j = j0 + lane; j < j1; j += 32) m = min(m, __ldcg(sub + u * stride + j));
     m = __reduce_min_sync(0xffffffffu, m);
     if (lane == 0 && m != 0xFFFFFFFFu) atomicMin(word + (u / rows) * capacity + u % rows, m);
   }
 }
 
-void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s) {
+void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, const uint16_t* d_su, cudaStream_t s) {
   for (uint32_t t = 0; t < n_tables; ++t) {
     const DevTable& T = h_tab[t];
     if (T.su <= 1) continue;
@@ -446,10 +449,52 @@ void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t
       if (!sub[k] || !word[k] || !groups[k] || !T.sub_rows) continue;
       const uint64_t warps = (uint64_t)groups[k] * T.sub_rows * ((T.su + 1023) / 1024);
       const unsigned blocks = (unsigned)std::min<uint64_t>((warps + 7) / 8, 148 * 8);
-      k_bucket_reduce<<<blocks, 256, 0, s>>>(sub[k], word[k], groups[k], T.sub_rows, T.capacity, T.su);
+      k_bucket_reduce<<<blocks, 256, 0, s>>>(sub[k], word[k], groups[k], T.sub_rows, T.capacity, T.su, d_su, t);
       note_launch();
     }
   }
+}
+
+// T per table: OPS batches (kcount == null): every txn may access every table (YCSB's one table:
+// exact).  TPC-C: the sum of the per-procedure list lengths of the procedures that access the
+// table (NewOrder: W D C I S + inserts into O NO OL; Payment: W D C H; OrderStatus: C O OL;
+// Delivery: D NO O OL C; StockLevel: D O OL S).
+__global__ void k_popularity(const uint32_t* kcount, uint32_t n_all, uint16_t* d_su, uint32_t* popular,
+                             uint32_t n_tables) {
+  constexpr uint32_t TPCC_ACCESS[5] = {0x1F7u, 0x00Fu, 0x064u, 0x076u, 0x162u};  // table bits per procedure
+  const uint32_t t = threadIdx.x;
+  uint32_t su = 1;
+  if (t < n_tables) {
+    const DevTable& T = c_tabs[t];
+    if (T.su > 1 && T.sub_rows) {  // E = T / D > 1  <=>  T > D
+      uint64_t cnt = n_all;
+      if (kcount) {
+        cnt = 0;
+        for (int k = 0; k < 5; ++k)
+          if ((TPCC_ACCESS[k] >> t) & 1u) cnt += kcount[k];
+      }
+      if (cnt > T.sub_rows) {
+        const uint64_t e = (cnt + T.sub_rows - 1) / T.sub_rows;  // ceil(E); ceil(ceil(E)/32) == ceil(E/32)
+        su = (uint32_t)((e + 31) / 32 * 32 < T.su ? (e + 31) / 32 * 32 : T.su);
+      }
+    }
+    d_su[t] = (uint16_t)su;
+  }
+  const uint32_t m = __ballot_sync(0xffffffffu, su > 1);
+  if (t == 0 && popular) *popular = m;
+}
+
+void launch_popularity(const DevTable* h_tab, uint32_t n_tables, const uint32_t* kcount, uint32_t n_all,
+                       uint16_t* d_su, uint32_t* popular, cudaStream_t s) {
+  bool any = false;
+  for (uint32_t t = 0; t < n_tables; ++t) any |= h_tab[t].su > 1;
+  if (!any) return;
+  static_assert(MAXT <= 32, "one warp");
+  k_popularity<<<1, 32, 0, s>>>(kcount, n_all, d_su, popular, n_tables);
+  note_launch();
+  upload_tables_common_su(d_su, s);
+  upload_tables_ops_su(d_su, s);
+  upload_tables_tpcc_su(d_su, s);
 }
 
 __global__ void k_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n) {

@@ -102,6 +102,8 @@ struct Tx {
   uint32_t bits;   // detect: conflict bits found so far (CF_*)
   uint32_t* err;
   bool reorder;    // NEXT-1 logical reordering
+  mark_t* hm;      // execute: the block's shared-memory marks of the WAREHOUSE / DISTRICT units (or null)
+  uint32_t nw;
   // verdict already decided by the bits found (remaining checks cannot change it)
   __device__ __forceinline__ bool done() const { return conflict_of(bits, reorder); }
 };
@@ -113,14 +115,37 @@ __device__ __forceinline__ void internal_error(Tx& x) { atomicOr(x.err, ERR_EINT
 // Marks: the read-before-atomicMin filter is applied to the popular tables only (P:215,
 // E = T/D > 1: WAREHOUSE and DISTRICT, thousands of accesses per row and batch); on cold
 // rows it would add a dependent DRAM round trip before a fire-and-forget RED.
+// Execute: the hottest units -- WAREHOUSE (W_YTD) and DISTRICT (D_YTD, D_NEXT_O_ID, the
+// Delivery cursor), touched by nearly every txn -- are marked into a per-block shared-memory
+// copy (atomicMin in shared memory, hm) and flushed with one global atomicMin per touched unit
+// when the block ends (k_tpcc_phase): marks are read only by detection, after this kernel, and
+// min is order-free, so the marks are identical; the per-txn filter read of a hot L2 line (a
+// dependent round trip, ~11% of execute's stall samples) disappears.  A unit whose group kind
+// does not match (a W mark on an ADD group) takes the global path.
+__device__ __forceinline__ mark_t* hot_mark(const DevTable& T, uint32_t g, uint32_t row, const Tx& x, bool add) {
+#ifdef LTPG_NO_HOT_MARKS
+  return nullptr;
+#endif
+  if (!x.hm || T.id > TD || (((T.add_groups >> g) & 1u) != (add ? 1u : 0u))) return nullptr;
+  if (T.id == TW) return (g == 0 && row < x.nw) ? x.hm + row : nullptr;
+  return (g < 3 && row < 10 * x.nw) ? x.hm + x.nw + g * 10 * x.nw + row : nullptr;
+}
 template <int PH>
 __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_unit(T, MK_W, g, row, x.tag, x.filter && hot);
+  if (PH == PH_EXEC) {
+    mark_t* h = hot ? hot_mark(T, g, row, x, false) : nullptr;
+    if (h) atomicMin(h, x.tag);
+    else mark_unit(T, MK_W, g, row, x.tag, x.filter && hot);
+  }
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_WRITE, x.r, x.epoch);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
-  if (PH == PH_EXEC) mark_unit(T, MK_A, g, row, x.tag, x.filter && hot);
+  if (PH == PH_EXEC) {
+    mark_t* h = hot ? hot_mark(T, g, row, x, true) : nullptr;
+    if (h) atomicMin(h, x.tag);
+    else mark_unit(T, MK_A, g, row, x.tag, x.filter && hot);
+  }
   if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_ADD, x.r, x.epoch);
 }
 template <int PH>
@@ -156,9 +181,9 @@ __device__ __forceinline__ uint32_t seg16_or(uint32_t v) {
   return v;
 }
 
-// ECAPACITY before execution: worst case every NewOrder / Payment of this partition
+// ECAPACITY before write-back: worst case every NewOrder / Payment of this partition
 // commits; partitions of one process share the table and reserve in stream order (one thread
-// of k_tpcc_group's last block)
+// of the execute grid's first block, after the grouping kernel)
 __device__ void tpcc_capacity_tail(const BatchDev& b, const TpccParams& tp) {
   const uint64_t add[4] = {__ldcg(tp.misc + M_NO), __ldcg(tp.misc + M_NO), __ldcg(tp.misc + M_NO_LINES),
                            __ldcg(tp.misc + M_PAY)};
@@ -240,19 +265,55 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     // of 2, so a warp pays the parameter -> price dependency chain once for 4x the lines.
     long long amount = 0, w_tax = 0, d_tax = 0, disc = 0;
     uint32_t ua = 0;
+    // line validation (k_tpcc_group reads only the 16-byte headers of unpartitioned batches):
+    // item in [1, 100001], quantity in [1, 10], an existing supply warehouse, and the txn's
+    // items distinct (R10) -- the 4 lanes of the txn compare their 4 items each with the 16
+    // the header word and the lane's line records are loaded together (the records of slots past
+    // n_lines are read -- they are inside the 128-byte block -- and ignored)
+    uint32_t it[4];
+    uint2 v[4];
+    uint32_t h0 = 0, h1 = 0;
     if (active) {
-      const uint32_t h0 = *reinterpret_cast<const uint32_t*>(p), h1 = *reinterpret_cast<const uint32_t*>(p + 4);
-      const uint32_t w = h0 & 0xFFFFu, d = (h0 >> 16) & 0xFFu, n = h0 >> 24, c = h1 & 0xFFFFu;
-      uint32_t it[4], qt[4], ri[4], rs[4];
+      h0 = *reinterpret_cast<const uint32_t*>(p);
+      h1 = *reinterpret_cast<const uint32_t*>(p + 4);
+    }
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint32_t l = 4 * sub + k;
+      v[k] = make_uint2(0, 0);
+      if (active && l < 15) v[k] = *reinterpret_cast<const uint2*>(p + 8 + 8 * l);  // u32 i | u16 supply_w | u8 qty
+    }
+    const uint32_t n = h0 >> 24;
+    bool bad = false;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint32_t l = 4 * sub + k;
+      if (l >= n) v[k] = make_uint2(0, 0);
+      // unused slots get ids no item has (and that never collide with each other)
+      it[k] = (active && l < n) ? v[k].x : 0xFFFFFFF0u - l;
+      const uint32_t sw = v[k].y & 0xFFFFu, q = (v[k].y >> 16) & 0xFFu;
+      if (active && l < n && (v[k].x < 1 || v[k].x > 100001 || q < 1 || q > 10 || sw < 1 || sw > b.nw)) bad = true;
+    }
+#pragma unroll
+    for (uint32_t j = 0; j < 4; ++j)
+#pragma unroll
+      for (uint32_t m = 0; m < 4; ++m) {
+        const uint32_t o = __shfl_sync(0xffffffffu, it[m], j, 4);
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k)
+          if (o == it[k] && 4 * j + m != 4 * sub + k) bad = true;
+      }
+    if (bad) atomicOr(b.err, ERR_EINVAL);
+    const bool warp_bad = __any_sync(0xffffffffu, bad);  // the batch is rejected: skip the work
+    if (active && !warp_bad) {
+      const uint32_t w = h0 & 0xFFFFu, d = (h0 >> 16) & 0xFFu, c = h1 & 0xFFFFu;
+      uint32_t qt[4], ri[4], rs[4];
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
         const uint32_t l = 4 * sub + k;
-        uint2 v = make_uint2(0, 0);
-        if (l < n) v = *reinterpret_cast<const uint2*>(p + 8 + 8 * l);  // u32 i | u16 supply_w | u8 qty
-        it[k] = v.x;
-        qt[k] = (v.y >> 16) & 0xFFu;
-        ri[k] = l < n ? rowof(TIt, TI, v.x, x.dmask) : ROW_NONE;
-        rs[k] = l < n ? rowof(TSt, TS, kS(v.y & 0xFFFFu, v.x), x.dmask) : ROW_NONE;
+        qt[k] = (v[k].y >> 16) & 0xFFu;
+        ri[k] = l < n ? rowof(TIt, TI, v[k].x, x.dmask) : ROW_NONE;
+        rs[k] = l < n ? rowof(TSt, TS, kS(v[k].y & 0xFFFFu, v[k].x), x.dmask) : ROW_NONE;
       }
       long long price[4];
 #pragma unroll
@@ -656,6 +717,8 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
 }
 
 // ---- OrderStatus (TPC-C 2.6) with a predefined order key ----------------------------
+// 4 lanes per txn (8 txns per warp): lane 3 finds the customer and its order, then lane q reads
+// order lines 4q..4q+3 (all of a lane's line loads in flight together).
 template <int PH>
 __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active,
                                  Tx& x) {
@@ -670,7 +733,7 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
     w = p16(p, 0);
     d = p[2];
   }
-  if (active && sub == 15) {
+  if (active && sub == 3) {
     if (PH == PH_EXEC) {
       cid = p[3] ? (uint32_t)tp.by_name[kD(w, d) * 1000 + p16(p, 6)] : p16(p, 4);
       row_c = cid ? rowof(TCu, TC, kC(w, d, cid), x.dmask) : ROW_NONE;
@@ -695,26 +758,35 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
     if (row_c != ROW_NONE) unit_r<PH>(TCu, col_group(TCu, C_BALANCE), row_c, x);
     if (row_o != ROW_NONE) unit_r<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x);
   }
-  uint32_t olrow = (active && sub == 15 && row_o != ROW_NONE && TOr.aux) ? TOr.aux[row_o] : ROW_NONE;
-  o = __shfl_sync(0xffffffffu, o, 15, 16);
-  cnt = __shfl_sync(0xffffffffu, cnt, 15, 16);
-  olrow = __shfl_sync(0xffffffffu, olrow, 15, 16);
+  uint32_t olrow = (PH == PH_EXEC && active && sub == 3 && row_o != ROW_NONE && TOr.aux) ? TOr.aux[row_o] : ROW_NONE;
+  o = __shfl_sync(0xffffffffu, o, 3, 4);
+  cnt = __shfl_sync(0xffffffffu, cnt, 3, 4);
+  olrow = __shfl_sync(0xffffffffu, olrow, 3, 4);
   long long dd = 0;
-  if (active && sub < cnt && sub < 15) {
-    uint32_t row_ol;
+  uint32_t row_ol[4];
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) {  // the lane's line rows: from ORDER.aux (contiguous) or probed
+    const uint32_t l = 4 * sub + k;
+    row_ol[k] = ROW_NONE;
+    if (!active || l >= cnt || l >= 15) continue;
     if (PH == PH_EXEC) {
-      row_ol = olrow != ROW_NONE ? olrow + sub : probe(TOL_, kO(w, d, o) * 16 + sub + 1);
-      if (row_ol == ROW_NONE) internal_error(x);
-      else dd = rd(TOL_, OL_DELIVERY_D, row_ol);
-      log[sub] = row_ol;
+      row_ol[k] = olrow != ROW_NONE ? olrow + l : probe(TOL_, kO(w, d, o) * 16 + l + 1);
+      if (row_ol[k] == ROW_NONE) internal_error(x);
+      log[l] = row_ol[k];
     } else {
-      row_ol = log[sub];
+      row_ol[k] = log[l];
     }
-    if (row_ol != ROW_NONE) unit_r<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol, x);
+  }
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) {
+    if (row_ol[k] == ROW_NONE) continue;
+    if (PH == PH_EXEC) dd += rd(TOL_, OL_DELIVERY_D, row_ol[k]);
+    unit_r<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[k], x);
   }
   if (PH == PH_EXEC) {
-    dd = seg16_sum(dd);
-    if (active && sub == 15) {
+    dd += __shfl_xor_sync(0xffffffffu, dd, 1);  // sum over the txn's 4 lanes
+    dd += __shfl_xor_sync(0xffffffffu, dd, 2);
+    if (active && sub == 3) {
       long long* res = b.res + 4ull * r;
       res[0] = cid;
       res[1] = bal;
@@ -724,7 +796,7 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
   }
 }
 
-// ---- Delivery (TPC-C 2.7), one lane per district; rows re-derived in every phase ----------------
+// ---- Delivery (TPC-C 2.7), rows re-derived in every phase -----------------------------------
 // Shared per warehouse: every Delivery RMWs the cursors of all ten districts of its warehouse
 // (WRITE units), so of a warehouse's Deliveries in a batch only the smallest rank can commit
 // (R1 and NEXT-1: WAW aborts).  They all read the same snapshot -- same cursors, orders, lines
@@ -732,94 +804,90 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
 // and return the same results (the carrier is not part of them).  Only that rank (dl_min[w],
 // from k_tpcc_group) executes, marks and is checked; the others copy its result slots and take
 // the WAW verdict.  Result-identical to running each one (oracle parity).
+// The phase kernel runs the leaders by warehouse (slot type SL_DLW: one 16-lane slot per
+// warehouse with a Delivery in the batch, lane d-1 = district d), and detection visits every
+// Delivery txn once more with one lane each (SL_DLT) to give the followers their verdict and
+// results -- the followers, nearly all Deliveries, cost one load each instead of a 16-lane slot.
+
+// one district of leader txn x.r (lane d - 1)
 template <int PH>
-__device__ void proc_delivery(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active,
-                              Tx& x) {
-  if (active) {
-    const uint32_t rmin = tp.dl_min[p16(b.params + 128ull * r, 0)];
-    if (rmin != r) {
-      if (PH == PH_DETECT) {
-        x.bits |= CF_WAW;  // WAW on the district cursors against rank rmin < r
-        if (sub < 4) b.res[4ull * r + sub] = b.res[4ull * rmin + sub];  // written by rmin's execute
-      }
-      return;  // (never committed: no write-back)
-    }
-  }
+__device__ void delivery_district(const BatchDev& b, uint32_t w, uint32_t d, long long carrier, Tx& x,
+                                  long long& delivered, long long& total) {
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TCu = c_tabs[TC];
   const DevTable& TOr = c_tabs[TO];
   const DevTable& TOL_ = c_tabs[TOL];
   const DevTable& TNw = c_tabs[TNO];
-  const uint8_t* p = b.params + 128ull * r;
-  long long delivered = 0, total = 0;
-  if (active && sub < 10) {
-    const uint32_t w = p16(p, 0);
-    const long long carrier = p[2];
-    const uint32_t d = sub + 1;
-    const uint32_t row_d = rowof(TDi, TD, kD(w, d), x.dmask);
-    if (row_d == ROW_NONE) {
-      internal_error(x);
-    } else {
-      const long long o = rd(TDi, D_NEXT_DELIV_O_ID, row_d);
-      unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x, true);  // RMW of the cursor
-      const uint64_t nok = kO(w, d, (uint64_t)o);
-      uint64_t hn_, ho_;
-      const ulonglong2 vn = probe_issue(TNw, nok, hn_), vo = probe_issue(TOr, nok, ho_);  // together
-      const uint32_t row_no = (PH == PH_DETECT && x.done()) ? ROW_NONE : probe_finish(TNw, nok, hn_, vn);
-      if (PH == PH_DETECT && x.done()) {
-        // conflict already found: the remaining checks cannot change the verdict
-      } else if (row_no == ROW_NONE) {
-        // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
-        unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
-      } else {
-        // every Delivery of a warehouse in the batch reads the same cursor and so delivers the
-        // same order: its NEW_ORDER / ORDER / ORDER_LINE / CUSTOMER units are as hot as the
-        // district's (E >> 1) -- marks take the read-before-atomicMin filter
-        for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x, true);  // DELETE
-        const uint32_t row_o = probe_finish(TOr, nok, ho_, vo);
-        if (row_o == ROW_NONE) {
-          internal_error(x);
-        } else {
-          unit_w<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x, true);
-          const uint32_t cid = (uint32_t)rd(TOr, O_C_ID, row_o);
-          const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
-          long long sum = 0;
-          uint32_t row_ol[15];
-          const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
+  const uint32_t row_d = rowof(TDi, TD, kD(w, d), x.dmask);
+  if (row_d == ROW_NONE) {
+    internal_error(x);
+    return;
+  }
+  const long long o = rd(TDi, D_NEXT_DELIV_O_ID, row_d);
+  unit_w<PH>(TDi, col_group(TDi, D_NEXT_DELIV_O_ID), row_d, x, true);  // RMW of the cursor
+  const uint64_t nok = kO(w, d, (uint64_t)o);
+  uint64_t hn_, ho_;
+  const ulonglong2 vn = probe_issue(TNw, nok, hn_), vo = probe_issue(TOr, nok, ho_);  // together
+  if (PH == PH_DETECT && x.done()) return;  // conflict already found: the verdict cannot change
+  const uint32_t row_no = probe_finish(TNw, nok, hn_, vn);
+  if (row_no == ROW_NONE) {
+    // queue empty in S: READ of the D_NEXT_O_ID unit (same-batch NewOrders conflict)
+    unit_r<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
+    return;
+  }
+  // every Delivery of a warehouse in the batch reads the same cursor and so delivers the same
+  // order: its NEW_ORDER / ORDER / ORDER_LINE / CUSTOMER units are as hot as the district's
+  // (E >> 1) -- marks take the read-before-atomicMin filter
+  for (uint32_t g = 0; g < TNw.n_groups; ++g) unit_w<PH>(TNw, g, row_no, x, true);  // DELETE
+  const uint32_t row_o = probe_finish(TOr, nok, ho_, vo);
+  if (row_o == ROW_NONE) {
+    internal_error(x);
+    return;
+  }
+  unit_w<PH>(TOr, col_group(TOr, O_CARRIER_ID), row_o, x, true);
+  const uint32_t cid = (uint32_t)rd(TOr, O_C_ID, row_o);
+  const uint32_t cnt = (uint32_t)rd(TOr, O_OL_CNT, row_o);
+  long long sum = 0;
+  uint32_t row_ol[15];
+  const uint32_t olrow = TOr.aux ? TOr.aux[row_o] : ROW_NONE;  // lines are contiguous rows
 #pragma unroll
-          for (uint32_t l = 0; l < 15; ++l)  // otherwise all order-line probes in flight together
-            row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, nok * 16 + l + 1)) : ROW_NONE;
-          const uint32_t row_c = rowof(TCu, TC, kC(w, d, cid), x.dmask);
+  for (uint32_t l = 0; l < 15; ++l)  // otherwise all order-line probes in flight together
+    row_ol[l] = l < cnt ? (olrow != ROW_NONE ? olrow + l : probe(TOL_, nok * 16 + l + 1)) : ROW_NONE;
+  const uint32_t row_c = rowof(TCu, TC, kC(w, d, cid), x.dmask);
 #pragma unroll
-          for (uint32_t l = 0; l < 15; ++l) {
-            if (l >= cnt) continue;
-            if (row_ol[l] == ROW_NONE) { internal_error(x); continue; }
-            unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[l], x, true);
-            sum += rd(TOL_, OL_AMOUNT, row_ol[l]);
-            if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol[l], b_clock(b));
-          }
-          if (row_c == ROW_NONE) {
-            internal_error(x);
-          } else {
-            col_upd3<PH>(TCu, C_BALANCE, C_DELIVERY_CNT, C_DELIVERY_CNT, row_c, x, true);
-            if (PH == PH_WB) {
-              addv(TCu, C_BALANCE, row_c, sum);
-              addv(TCu, C_DELIVERY_CNT, row_c, 1);
-            }
-          }
-          if (PH == PH_WB) {
-            wr(TOr, O_CARRIER_ID, row_o, carrier);
-            TNw.valid[row_no] = 0;
-            IdxSlot* sl = idx_slot(TNw, nok);
-            if (sl) sl->row = ROW_NONE;
-            wr(TDi, D_NEXT_DELIV_O_ID, row_d, o + 1);
-          }
-          delivered = 1;
-          total = sum;
-        }
-      }
+  for (uint32_t l = 0; l < 15; ++l) {
+    if (l >= cnt) continue;
+    if (row_ol[l] == ROW_NONE) { internal_error(x); continue; }
+    unit_w<PH>(TOL_, col_group(TOL_, OL_DELIVERY_D), row_ol[l], x, true);
+    sum += rd(TOL_, OL_AMOUNT, row_ol[l]);
+    if (PH == PH_WB) wr(TOL_, OL_DELIVERY_D, row_ol[l], b_clock(b));
+  }
+  if (row_c == ROW_NONE) {
+    internal_error(x);
+  } else {
+    col_upd3<PH>(TCu, C_BALANCE, C_DELIVERY_CNT, C_DELIVERY_CNT, row_c, x, true);
+    if (PH == PH_WB) {
+      addv(TCu, C_BALANCE, row_c, sum);
+      addv(TCu, C_DELIVERY_CNT, row_c, 1);
     }
   }
+  if (PH == PH_WB) {
+    wr(TOr, O_CARRIER_ID, row_o, carrier);
+    TNw.valid[row_no] = 0;
+    IdxSlot* sl = idx_slot(TNw, nok);
+    if (sl) sl->row = ROW_NONE;
+    wr(TDi, D_NEXT_DELIV_O_ID, row_d, o + 1);
+  }
+  delivered = 1;
+  total = sum;
+}
+
+// the leader of warehouse w (slot type SL_DLW, 16 lanes: lane d-1 = district d); r = dl_min[w]
+template <int PH>
+__device__ void proc_delivery(const BatchDev& b, uint32_t r, uint32_t sub, bool active, Tx& x) {
+  long long delivered = 0, total = 0;
+  const uint8_t* p = b.params + 128ull * r;
+  if (active && sub < 10) delivery_district<PH>(b, p16(p, 0), sub + 1, p[2], x, delivered, total);
   if (PH == PH_EXEC) {
     delivered = seg16_sum(delivered);
     total = seg16_sum(total);
@@ -831,6 +899,21 @@ __device__ void proc_delivery(const BatchDev& b, const TpccParams& tp, uint32_t 
       res[3] = 0;
     }
   }
+}
+// detection pass over every Delivery txn (slot type SL_DLT, one lane each): a follower (not its
+// warehouse's smallest rank) takes the WAW verdict and copies the leader's results; returns
+// whether r is a follower (a leader's verdict comes from its SL_DLW slot)
+__device__ __forceinline__ bool delivery_follower(const BatchDev& b, const TpccParams& tp, uint32_t r, Tx& x) {
+  const uint32_t rmin = tp.dl_min[p16(b.params + 128ull * r, 0)];
+  if (rmin == r) return false;
+  x.bits |= CF_WAW;  // WAW on the district cursors against rank rmin < r
+  long long* res = b.res + 4ull * r;  // written by rmin's execute
+  const long long* src = b.res + 4ull * rmin;
+  res[0] = src[0];
+  res[1] = src[1];
+  res[2] = src[2];
+  res[3] = src[3];
+  return true;
 }
 
 // ---- StockLevel (TPC-C 2.8): shared per district ---------------------------------------------
@@ -1057,14 +1140,18 @@ __global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScr
 // block, many registers) runs in its own launch so it does not cap the occupancy of the
 // others -- each type group gets its own launch configuration.
 constexpr uint32_t TM_MAIN = 0x0Fu;
-// lanes per txn of a procedure type: Payment 1, StockLevel 32, others 16 -- NewOrder execution
-// and detection of an unpartitioned batch 4 (4 lines / units per lane, see proc_neworder;
-// execute 0.255 -> 0.198 ms, detect 0.113 -> 0.087 ms on tpcc_c4) -- except detection under
-// NEXT-1 reordering, where every unit's three marks are read and 16 lanes measured faster
+// Warp slot types of the phase kernel: the procedure types 0..4 (Delivery's type 3 is the
+// detection-only pass over every Delivery txn) and SL_DLW, the Delivery leader of a warehouse.
+constexpr uint32_t SL_DLT = 3, SL_DLW = 5, NSLOT = 6;
+// lanes per slot: Payment 1; Delivery txn pass 1; Delivery leader 16 (one per district);
+// OrderStatus 4 (4 lines per lane); StockLevel 32 (k_sl_*); NewOrder 16 -- 4 in execution and detection of an unpartitioned
+// batch (4 lines / units per lane, see proc_neworder; execute 0.255 -> 0.198 ms, detect 0.113 ->
+// 0.087 ms on tpcc_c4) except detection under NEXT-1 reordering, where every unit's three marks
+// are read and 16 lanes measured faster
 __device__ __forceinline__ uint32_t lanes_of(uint32_t t, int PH, uint32_t nparts, bool reorder) {
-  return t == 1 ? 1u
-                : (t == 4 ? 32u
-                          : ((t == 0 && nparts <= 1 && (PH != PH_DETECT || !reorder)) ? 4u : 16u));
+  return t == 1 || t == SL_DLT ? 1u
+                          : (t == 4 ? 32u
+                                    : (t == 2 || (t == 0 && nparts <= 1 && (PH != PH_DETECT || !reorder)) ? 4u : 16u));
 }  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
 template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
@@ -1083,7 +1170,15 @@ template <int PH, uint32_t TMASK>
 #endif
 __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
     k_tpcc_phase(BatchDev b, TpccParams tp) {
-  if (*b.err) return;  // (write-back: the row counters then stay put -- no last block runs)
+  // one read of the error word per block: the kernel has block barriers, and the word can be
+  // raised by other blocks of this grid while this one starts
+  __shared__ uint32_t s_err;
+  if (threadIdx.x == 0) s_err = *(volatile uint32_t*)b.err;
+  __syncthreads();
+  if (s_err) return;  // (write-back: the row counters then stay put -- no last block runs)
+  // ECAPACITY before anything is written back: the grouping counts are final here (a block
+  // barrier + fence + counter per grouping block for a "last block" cost 22% of that kernel)
+  if (PH == PH_EXEC && TMASK == TM_MAIN && blockIdx.x == 0 && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
   const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
   // write-back with delayed W_YTD / D_YTD (ADD columns): the block's committed Payments add
   // into shared-memory deltas per warehouse (and district), flushed with one atomic per touched
@@ -1094,44 +1189,61 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     for (uint32_t i = threadIdx.x; i < tp.nw + 1 + tp.agg_dsz; i += blockDim.x) agg[i] = 0;
     __syncthreads();
   }
+  // execute: shared-memory marks of the hot WAREHOUSE / DISTRICT units (hot_mark)
+  mark_t* hm = (PH == PH_EXEC && tp.hot_words) ? reinterpret_cast<mark_t*>(agg) : nullptr;
+  if (hm) {
+    for (uint32_t i = threadIdx.x; i < tp.hot_words; i += blockDim.x) hm[i] = 0xFFFFFFFFu;
+    __syncthreads();
+  }
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
   // NewOrder, Payment), so that the grid's tail is made of short Payment warps (0.088 -> 0.077
   // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
-  constexpr uint32_t ORD = PH == PH_DETECT ? (2u | 3u << 4 | 0u << 8 | 1u << 12 | 4u << 16)
-                                           : (0u | 1u << 4 | 2u << 8 | 3u << 12 | 4u << 16);  // slot j -> type
-  uint32_t cnt[NTYPES], pre[NTYPES + 1];
+  constexpr uint32_t ORD = PH == PH_DETECT ? (2u | SL_DLW << 4 | 0u << 8 | SL_DLT << 12 | 1u << 16 | 4u << 20)
+                                           : (0u | 1u << 4 | 2u << 8 | SL_DLW << 12 | SL_DLT << 16 | 4u << 20);  // slot j -> type
+  uint32_t cnt[NSLOT], pre[NSLOT + 1];
   pre[0] = 0;
 #pragma unroll
-  for (int j = 0; j < NTYPES; ++j) {
+  for (int j = 0; j < NSLOT; ++j) {
     const uint32_t t = (ORD >> (4 * j)) & 15u;
-    cnt[j] = ((TMASK >> t) & 1u) ? tp.counts[t] : 0u;
+    const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
+    cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : tp.counts[t]));
     const uint32_t per = 32 / lanes_of(t, PH, b.nparts, reorder);
     pre[j + 1] = pre[j] + (cnt[j] + per - 1) / per;
   }
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NTYPES]; w += nwarps) {
+  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NSLOT]; w += nwarps) {
     uint32_t j = 0, lw = w, ct = cnt[0];
 #pragma unroll
-    for (int jj = 1; jj < NTYPES; ++jj)
-      if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }  // warp-uniform procedure type
+    for (int jj = 1; jj < NSLOT; ++jj)
+      if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }  // warp-uniform slot type
     const uint32_t t = (ORD >> (4 * j)) & 15u;
     const uint32_t L = lanes_of(t, PH, b.nparts, reorder);
     const uint32_t per = 32 / L;
     const uint32_t k = lw * per + lane / L;
     const uint32_t sub = lane % L;
-    const bool active = k < ct;
-    const uint32_t r = active ? tp.list[(uint64_t)t * tp.max_txns + k] : 0;
-    Tx x{dmask, r, b_epoch(b), epoch_tag(b_epoch(b)) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder};
+    bool active = k < ct;
+    uint32_t r = 0;
+    if (t == SL_DLW) {  // warehouse k + 1's Delivery leader (write-back: only if it committed)
+      r = active ? tp.dl_min[k + 1] : ~0u;
+      active = r != ~0u && (PH != PH_WB || b.status[r] == LTPG_ST_COMMIT);
+      if (!active) r = 0;
+    } else if (active) {
+      r = tp.list[(uint64_t)t * tp.max_txns + k];
+    }
+    Tx x{dmask, r, b_epoch(b), epoch_tag(b_epoch(b)) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder,
+         hm, tp.nw};
     bool go = active;  // write-back runs over the committed re-list (k_tpcc_relist) only
+    bool status_here = true;  // detection: this slot decides txn r's verdict
     // NEXT-1: read-only procedures (OrderStatus, StockLevel) can never abort under reordering
     if (PH == PH_DETECT && reorder && (t == 2 || t == 4)) go = false;
     switch (t) {
       case 0: proc_neworder<PH>(b, tp, r, sub, go, x); break;
       case 1: if (go) proc_payment<PH>(b, tp, r, x, aggw ? agg : nullptr); break;
       case 2: if (PH != PH_WB) proc_orderstatus<PH>(b, tp, r, sub, go, x); break;
-      case 3: proc_delivery<PH>(b, tp, r, sub, go, x); break;
+      case SL_DLW: proc_delivery<PH>(b, r, sub, go, x); break;
+      case SL_DLT: if (go && PH == PH_DETECT) status_here = delivery_follower(b, tp, r, x); break;
       default:
         break;  // StockLevel: shared per district (k_sl_*)
     }
@@ -1140,11 +1252,24 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
       const uint32_t bw = __ballot_sync(0xffffffffu, x.bits & CF_WAW) & seg;
       const uint32_t br = __ballot_sync(0xffffffffu, x.bits & CF_RAW) & seg;
       const uint32_t bx = __ballot_sync(0xffffffffu, x.bits & CF_WAR) & seg;
-      if (active && sub == 0) {
+      if (active && sub == 0 && status_here) {
         const uint32_t flag = (bw ? CF_WAW : 0u) | (br ? CF_RAW : 0u) | (bx ? CF_WAR : 0u) | (b.ua[r] ? CF_UA : 0u);
         if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;  // partitioned: exchanged before write-back
         else b.status[r] = status_of_bits(flag, reorder);
       }
+    }
+  }
+  if (hm) {  // flush: one global atomicMin per unit this block marked
+    __syncthreads();
+    const DevTable& TWh = c_tabs[TW];
+    const DevTable& TDi = c_tabs[TD];
+    for (uint32_t i = threadIdx.x; i < tp.hot_words; i += blockDim.x) {
+      const mark_t v = hm[i];
+      if (v == 0xFFFFFFFFu) continue;
+      const bool isw = i < tp.nw;
+      const DevTable& T = isw ? TWh : TDi;
+      const uint32_t g = isw ? 0u : (i - tp.nw) / (10 * tp.nw), row = isw ? i : (i - tp.nw) % (10 * tp.nw);
+      atomicMin((T.add_groups >> g) & 1u ? amark_ptr(T, g, row) : wmark_ptr(T, g, row), v);
     }
   }
   if (aggw) {
@@ -1166,36 +1291,47 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
 }
 
 // ---- K-tgroup: validation + per-type lists (warp-aggregated appends) ----------------------------
+// FULL (partitioned batches): the whole 128-byte block is parsed here -- a NewOrder's supply
+// warehouses decide whether it touches this partition.  Otherwise (one partition) only the
+// first 16 bytes of each block are read: every field but the NewOrder lines sits there, and the
+// lines are validated by execute, which reads them anyway (proc_neworder; an invalid line
+// raises ERR_EINVAL there, before anything is written back).  134 -> 16 MB read per 2^20 txns.
+template <bool FULL>
 __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
-  // the warp's 32 parameter blocks (4 KB, contiguous) staged through shared memory with
+  // FULL: the warp's 32 parameter blocks (4 KB, contiguous) staged through shared memory with
   // coalesced 16-byte loads; each lane then parses its own block.  Rows are padded to 33
   // words: with a 128-byte stride every lane's field would sit in the same bank (32-way
   // conflicts measured at 45% short-scoreboard stalls)
   constexpr uint32_t SROW = 132;
-  __shared__ __align__(16) uint8_t stage[8][32 * SROW];
+  __shared__ __align__(16) uint8_t stage[FULL ? 8 : 1][FULL ? 32 * SROW : 16];
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = r - lane;
-  uint8_t* sw = stage[wib];
+  uint8_t* sw = stage[FULL ? wib : 0];
+  uint4 head = make_uint4(0, 0, 0, 0);  // !FULL: the block's first 16 bytes, in registers
+  if (FULL) {
 #pragma unroll
-  for (uint32_t k = 0; k < 8; ++k) {
-    const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB
-    if (r0 + c / 8 < b.n_txns) {
-      const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r0 + 16 * c);
-      uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * (c / 8) + 16 * (c % 8));
-      d[0] = v.x;
-      d[1] = v.y;
-      d[2] = v.z;
-      d[3] = v.w;
+    for (uint32_t k = 0; k < 8; ++k) {
+      const uint32_t c = k * 32 + lane;  // 16-byte chunk of the warp's 4 KB
+      if (r0 + c / 8 < b.n_txns) {
+        const uint4 v = *reinterpret_cast<const uint4*>(b.params + 128ull * r0 + 16 * c);
+        uint32_t* d = reinterpret_cast<uint32_t*>(sw + SROW * (c / 8) + 16 * (c % 8));
+        d[0] = v.x;
+        d[1] = v.y;
+        d[2] = v.z;
+        d[3] = v.w;
+      }
     }
+    __syncwarp();
+  } else if (r < b.n_txns) {
+    head = *reinterpret_cast<const uint4*>(b.params + 128ull * r);
   }
-  __syncwarp();
   uint32_t t = 0xFF, lines = 0;
   bool bad = false;
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;
     t = b.ptype[r];
-    const uint8_t* p = sw + SROW * lane;
+    const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
     const uint32_t W = tp.nw;
     auto okw = [W](uint32_t w) { return w >= 1 && w <= W; };
     auto okd = [](uint32_t d) { return d >= 1 && d <= 10; };
@@ -1204,6 +1340,8 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
       case 0: {
         const uint32_t nl = p[3], c = p16(p, 4);
         if (!okd(p[2]) || nl < 1 || nl > 15 || c < 1 || c > 3000) { bad = true; break; }
+        lines = nl;
+        if (!FULL) break;  // lines: validated by execute
         uint32_t it[15];
 #pragma unroll
         for (uint32_t l = 0; l < 15; ++l) {
@@ -1216,7 +1354,6 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
 #pragma unroll
           for (uint32_t m = 0; m < l; ++m)
             if (it[l] == it[m]) bad = true;  // R10: distinct items (registers, unrolled)
-        lines = nl;
         break;
       }
       case 1:
@@ -1243,10 +1380,10 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   bool touch = false;
   uint32_t no_home = 0, pay_cust = 0;
   if (r < b.n_txns && !bad) {
-    const uint8_t* p = sw + SROW * lane;
+    const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
     const bool home = owns_w(b, p16(p, 0));
     touch = home;
-    if (t == 0) {
+    if (FULL && t == 0) {
       for (uint32_t l = 0; l < lines && !touch; ++l) touch = owns_w(b, p16(p + 8 + 8 * l, 4));
       no_home = home;
       if (!home) lines = 0;
@@ -1258,7 +1395,7 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     lines = 0;
   }
   if (t == 3 && touch) {  // smallest Delivery rank per warehouse (shared Delivery, proc_delivery)
-    uint32_t* m = tp.dl_min + p16(sw + SROW * lane, 0);
+    uint32_t* m = tp.dl_min + (FULL ? p16(sw + SROW * lane, 0) : (head.x & 0xFFFFu));
     if (r < *m) atomicMin(m, r);
   }
   // block-aggregated counters and per-type list positions (one atomic per block and list)
@@ -1275,7 +1412,6 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
 #pragma unroll
   for (uint32_t k = 0; k < NTYPES; ++k)
     if (cnt[k]) tp.list[(uint64_t)k * tp.max_txns + base[k]] = r;
-  if (last_block(tp.misc + M_DONE_G) && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
 }
 
 // committed entries of every per-type list -> clist (order inside a list is irrelevant)
@@ -1660,12 +1796,22 @@ constexpr uint32_t COLSCAN_TILED_DSZ = 2048;  // above: k_no_colscan_tiled
 static size_t wb_smem(const TpccDev& t) {
   return ((size_t)t.nw + 1 + (t.dsz <= AGG_DSZ_MAX ? t.dsz : 0)) * sizeof(long long);
 }
+constexpr uint32_t HOT_SMEM_MAX = 24 * 1024;  // execute's shared-memory W / D marks: up to ~190 warehouses
+static uint32_t hot_words(const TpccDev& t, const BatchDev& b) {
+  // off for the A/B and NEXT-3 configurations that measure the global mark path itself
+  if (b.flags & (LTPG_FLAG_NO_MARK_FILTER | LTPG_FLAG_LARGE_BUCKETS)) return 0;
+#ifdef LTPG_NO_HOT_MARKS
+  return 0;
+#endif
+  const uint32_t words = t.nw + 30 * t.nw;
+  return words * sizeof(mark_t) <= HOT_SMEM_MAX ? words : 0;
+}
 static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists) {
   const uint32_t n = b.n_txns;
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min,
-                    committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u};
+                    committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u, committed_lists ? 0u : hot_words(t, b)};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -1681,9 +1827,14 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
     cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
     cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
   }
-  k_tpcc_group<<<(n + 255) / 256, 256, 0, s>>>(b, tp);  // + the capacity check (last block)
+  if (b.nparts > 1)
+    k_tpcc_group<true><<<(n + 255) / 256, 256, 0, s>>>(b, tp);  // + the capacity check (last block)
+  else
+    k_tpcc_group<false><<<(n + 255) / 256, 256, 0, s>>>(b, tp);
   note_launch(1);
   if (ev) record_stage(ev[2], s);
+  // NEXT-3: popularity from this batch's per-procedure counts -> bucket sizes
+  if (t.h_tab) launch_popularity(t.h_tab, t.n_tab, b.kcount, n, t.d_su, t.popular, s);
   const uint32_t grid = phase_grid(n);
   // StockLevel (shared per district) on a side stream, concurrently with the other procedures
   const SlScratch sl = t.sl;
@@ -1694,10 +1845,10 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   k_sl_claim<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   k_sl_district<<<148 * 2, 256, 0, t.side>>>(b, sl);
   cudaEventRecord(t.join[0], t.side);
-  k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, tp.hot_words * sizeof(mark_t), s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
   note_launch(3);
-  if (t.h_tab) launch_bucket_reduce(t.h_tab, t.n_tab, s);  // NEXT-3 large-sized buckets (if any)
+  if (t.h_tab) launch_bucket_reduce(t.h_tab, t.n_tab, t.d_su, s);  // NEXT-3 large-sized buckets (if any)
   if (ev) record_stage(ev[3], s);
   cudaEventRecord(t.fork[1], s);
   cudaStreamWaitEvent(t.side, t.fork[1], 0);

@@ -84,9 +84,13 @@ struct DevTable {
   // (E = T/D > 1) records each mark in sub-slot (rank mod su) of its unit's bucket of su =
   // ceil(E/32)*32 sub-slots; k_bucket_reduce folds every bucket into the unit's mark word
   // before detection.  su <= 1: standard-sized (one slot per unit).
+  // Popularity is identified per batch ("in real-time"): E = T/D with T = txns of the
+  // batch that access the table, so a batch's bucket size c_su[id] = ceil(E/32)*32 (1: standard,
+  // the mark word) is at most the allocated su (E bounded by max_txns / rows loaded).
   mark_t* sub[3];                 // [MK_W / MK_A / MK_R][group of that kind][sub_rows][su]
-  uint32_t su;
+  uint32_t su;                    // allocated sub-slots per unit (the stride); <= 1: no buckets
   uint32_t sub_rows;              // rows with buckets (the rows loaded; appended rows: standard)
+  uint32_t id;                    // table id (index of the batch's bucket size in c_su)
 };
 
 // table lookup honouring the dense mapping: dmask = *dense_live & ~(tables with INSERT/DELETE
@@ -155,10 +159,14 @@ __device__ __forceinline__ mark_t* rmark_ptr(const DevTable& T, uint32_t g, uint
 // longer serialise; k_bucket_reduce then takes the minimum over the bucket ("reads out
 // all the TIDs in the hash bucket and selects ... the smallest TID").  Result-identical.
 enum { MK_W = 0, MK_A = 1, MK_R = 2 };
+static __constant__ uint16_t c_su[MAXT];  // this batch's bucket size per table (per TU copy)
 __device__ __forceinline__ mark_t* mark_addr(const DevTable& T, int k, uint32_t g, uint32_t row, mark_t tag) {
   if (T.su > 1 && row < T.sub_rows) {
-    const uint32_t gi = k == MK_A ? __popc(T.add_groups & ((1u << g) - 1u)) : g;
-    return T.sub[k] + ((uint64_t)gi * T.sub_rows + row) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % T.su;
+    const uint32_t su = c_su[T.id];
+    if (su > 1) {
+      const uint32_t gi = k == MK_A ? __popc(T.add_groups & ((1u << g) - 1u)) : g;
+      return T.sub[k] + ((uint64_t)gi * T.sub_rows + row) * T.su + (tag & ((1u << MARK_RANK_BITS) - 1)) % su;
+    }
   }
   return k == MK_W ? wmark_ptr(T, g, row) : (k == MK_A ? amark_ptr(T, g, row) : rmark_ptr(T, g, row));
 }
@@ -290,10 +298,16 @@ static __constant__ DevTable c_tabs[MAXT];
 #define LTPG_DEFINE_TABLE_UPLOAD(fn)                                                            \
   void fn(const DevTable* d, cudaStream_t s) { /* d: device copy -> async D2D */                \
     cudaMemcpyToSymbolAsync(c_tabs, d, sizeof(DevTable) * MAXT, 0, cudaMemcpyDeviceToDevice, s); \
+  }                                                                                             \
+  void fn##_su(const uint16_t* d_su, cudaStream_t s) { /* the batch's bucket sizes (NEXT-3) */   \
+    cudaMemcpyToSymbolAsync(c_su, d_su, sizeof(uint16_t) * MAXT, 0, cudaMemcpyDeviceToDevice, s); \
   }
 void upload_tables_common(const DevTable* h, cudaStream_t s);
 void upload_tables_ops(const DevTable* h, cudaStream_t s);
 void upload_tables_tpcc(const DevTable* h, cudaStream_t s);
+void upload_tables_ops_su(const uint16_t* d_su, cudaStream_t s);
+void upload_tables_tpcc_su(const uint16_t* d_su, cudaStream_t s);
+void upload_tables_common_su(const uint16_t* d_su, cudaStream_t s);
 
 // ---- host-side launchers (defined in the .cu files) ----------------------------------
 // number of kernels launched by this library (reported per batch in ltpg_stats)
@@ -469,7 +483,14 @@ void launch_finalize_compact(const uint8_t* status, uint32_t n, uint32_t* commit
                              unsigned long long* tile_state, uint32_t* tile_ctr, const BatchVars* vars, cudaStream_t s);
 // NEXT-3: fold the large-sized buckets of every popular table into their units' mark words
 // (host copies of the tables; nothing is launched when no table has su > 1)
-void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, cudaStream_t s);
+void launch_bucket_reduce(const DevTable* h_tab, uint32_t n_tables, const uint16_t* d_su, cudaStream_t s);
+// NEXT-3 real-time popularity: the batch's bucket size per table from T = txns accessing
+// it and D = its loaded rows: su = E > 1 ? ceil(E/32)*32 : 1 with E = T/D, capped by the
+// allocation; then copied into every TU's c_su; *popular = bitmask of tables with su > 1.
+// kcount: TPC-C per-procedure list lengths (device) or null (OPS: T = n_all for every table).
+// Nothing runs when no table has buckets.
+void launch_popularity(const DevTable* h_tab, uint32_t n_tables, const uint32_t* kcount, uint32_t n_all,
+                       uint16_t* d_su, uint32_t* popular, cudaStream_t s);
 void launch_build_index_tail(uint32_t t, const unsigned long long* from, uint32_t* err, cudaStream_t s);
 void launch_note_rows(uint32_t t, unsigned long long* dst, cudaStream_t s);
 void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,

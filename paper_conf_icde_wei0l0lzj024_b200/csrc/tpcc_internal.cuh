@@ -62,6 +62,8 @@ struct TpccDev {
   cudaEvent_t fork[2]{}, join[2]{};
   const DevTable* h_tab = nullptr; // host table copies (NEXT-3 bucket reduce between exec and detect)
   uint32_t n_tab = 0;
+  uint16_t* d_su = nullptr;        // NEXT-3: this batch's bucket size per table (capi.cu)
+  uint32_t* popular = nullptr;     // NEXT-3: bitmask of this batch's popular tables (set per batch)
 };
 
 struct TpccParams {
@@ -79,6 +81,7 @@ struct TpccParams {
   unsigned long long* chunk_tot;
   uint32_t* dl_min;
   uint32_t agg_dsz;             // write-back: DISTRICT D_YTD deltas aggregated per block (0: not)
+  uint32_t hot_words;           // execute: shared-memory marks of the W / D units (nw + 30 nw; 0: off)
 };
 
 int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);

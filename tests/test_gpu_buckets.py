@@ -96,3 +96,36 @@ def test_tpcc_large_buckets(W, mode, reorder):
         pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
     dumps = compare_tables(g, o)
     assert all(tpcc_cc.check(dumps).values())
+
+
+@pytest.mark.parametrize("mode", ["strict", "delayed"])
+def test_realtime_popularity_follows_the_batch(mode):
+    """P:215 "identify such tables in real-time": E = T/D with T = the batch's txns accessing the
+    table.  Batches of 6, 40, 3000, 3400 and 8 txns on one warehouse (D: WAREHOUSE 1 row, DISTRICT
+    10 rows) switch WAREHOUSE / DISTRICT between standard and large buckets
+    from batch to batch (ltpg_stats.popular_tables); every batch == oracle."""
+    lib = L()
+    from workloads.formats import T_WAREHOUSE, T_DISTRICT, T_CUSTOMER, NEW_ORDER, PAYMENT
+    W, B = 1, 4096
+    wl = tpcc.TpccWorkload(W, seed=61, mode=mode, mix=tpcc.MIX_NO_PAY)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=B, tables=tables, append_batches=3, flags=lib.LTPG_FLAG_LARGE_BUCKETS)
+    o = oracle.tpcc_db(wl, tables)
+    std, large, su = g.mark_memory(T_WAREHOUSE)
+    assert su == 4096 and large > 0                       # allocated for E <= 4096 / 1
+    assert g.mark_memory(T_DISTRICT)[2] == 416            # ceil(4096 / 10 / 32) * 32
+    assert g.mark_memory(T_CUSTOMER)[2] == 1              # 30,000 rows > 4096: never popular
+    tid = 1
+    for bno, (n, types) in enumerate([(6, [NEW_ORDER] * 6), (40, None), (3000, [PAYMENT] * 1500 + [NEW_ORDER] * 1500),
+                                      (3400, [PAYMENT] * 3100 + [NEW_ORDER] * 300), (8, None)]):
+        b = wl.batch(n, tid, bno, types=types)
+        tid += n
+        rc, ost, ores = o.run_tpcc(b, 2 + bno)
+        out = g.run_tpcc(b, 2 + bno, stats=True)
+        assert rc == 0 and (out["status"] == ost).all() and (out["reads"] == ores).all()
+        pop = out["stats"]["popular_tables"]
+        T = n  # every NewOrder / Payment accesses WAREHOUSE, DISTRICT and CUSTOMER
+        assert bool(pop >> T_WAREHOUSE & 1) == (T > 1), (n, pop)
+        assert bool(pop >> T_DISTRICT & 1) == (T > 10), (n, pop)
+        assert not pop >> T_CUSTOMER & 1
+    compare_tables(g, o)

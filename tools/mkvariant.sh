@@ -6,7 +6,7 @@ set -e
 N=$1; F=$2
 D=_v$N
 rm -rf $D; mkdir -p $D
-rsync -a --exclude .git --exclude gpurun_out --exclude '_v*' --exclude profiles --exclude '*.o' ./ $D/
+tar --exclude=./.git --exclude=./gpurun_out --exclude='./_v*' --exclude=./profiles --exclude='*.o' -cf - . | tar -xf - -C $D
 (cd $D && python -c "
 import importlib.util, sys
 spec = importlib.util.spec_from_file_location('b', 'paper_conf_icde_wei0l0lzj024_b200/build.py')
