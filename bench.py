@@ -191,7 +191,7 @@ def make_workload(name, rank=0):
     return tpcc.TpccWorkload(w["W"], seed=seed, mode=w["mode"], mix=mix)
 
 
-def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, nccl_unique_id=None, **kw):
+def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, **kw):
     """The database exactly as the bench times it (also used by the full-size parity tests):
     append regions sized for the worst case of one batch plus the appends of `n_batches`
     batches (every NewOrder / Payment committing; 10.5 lines per NewOrder on average)."""
@@ -202,7 +202,7 @@ def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, nccl_
         flags |= ltpg.LTPG_FLAG_REORDER
     if w["kind"] == "ycsb":  # inserts (YCSB D/E) of every batch
         return ltpg.ycsb_database(wl, max_txns=B, max_ops=B * w["ops"], flags=flags, device=device,
-                                  rank=rank, world=world, nccl_unique_id=nccl_unique_id,
+                                  rank=rank, world=world,
                                   capacity=w["n_rows"] + n_batches * B * w["ops"] // 10 + 1024, **kw)
     from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY
     tabs = wl.initial_tables()
@@ -211,7 +211,7 @@ def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, nccl_
            T_ORDER_LINE: 15 * no + 10.5 * no * n_batches, T_HISTORY: pay * (1 + n_batches)}
     cap = {t: int(tabs[t][1].shape[1] + v) + 1024 for t, v in cap.items()}
     return ltpg.tpcc_database(wl, max_txns=B, tables=tabs, capacity=cap, flags=flags, device=device,
-                              rank=rank, world=world, nccl_unique_id=nccl_unique_id, **kw)
+                              rank=rank, world=world, **kw)
 
 
 def exec_algorithmic_bytes(batch):
@@ -455,8 +455,6 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-closed-loop", action="store_true")
     ap.add_argument("--flags", type=int, default=0)
-    ap.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
-                    help="N>1: peer-memory verdict exchange (default) or the ncclAllReduce baseline")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.cpu_baseline_child:
@@ -502,37 +500,48 @@ def main():
         args.flags |= ltpg.LTPG_FLAG_REORDER
     fused_front = w["kind"] == "ycsb" and not (args.flags & (ltpg.LTPG_FLAG_REORDER | ltpg.LTPG_FLAG_NO_GROUPING
                                                               | ltpg.LTPG_FLAG_UNFUSED))
-    uid = None
-    if world > 1 and args.exchange == "nccl":  # baseline: one NCCL communicator per db
-        args.flags |= ltpg.LTPG_FLAG_NCCL_EXCHANGE
-        from paper_conf_icde_wei0l0lzj024_b200.dist import nccl_unique_id
-        uid = nccl_unique_id()
     t0 = time.time()
     db = open_database(name, wl, args.warmup + 4 * args.steps + 2, flags=args.flags, device=local,
-                       rank=rank, world=world, nccl_unique_id=uid)
+                       rank=rank, world=world)
     log("rank %d: db loaded in %.1fs" % (rank, time.time() - t0))
 
     # distinct input batches, cycled (inputs only; every step recomputes everything)
     # (small batches: enough distinct batches that the closed-loop leg's fresh-txn pool lasts)
     n_distinct = 2 if B >= (1 << 18) else min(args.steps + 2, 32)
     host_batches, dev_batches, pin_batches = [], [], []
+    # multi-rank TPC-C runs SHARDED batches (SURVEY §8(e) host routing, ltpg_route_tpcc): every
+    # rank builds the same global batch, routes out its own shard (the txns touching its
+    # warehouses) and uploads only that; it counts the commits of the txns it is home of
+    sharded = world > 1 and w["kind"] == "tpcc"
+    home_masks, shard_sizes = [], []
     tid = 1
     for i in range(n_distinct):
         b = wl.batch(B, tid, i)
         tid += B
+        if sharded:
+            b = ltpg.route_tpcc(b, wl.W, world, rank)
+            p = b["params"]
+            home_masks.append(ltpg.part_of_w(p[:, 0].astype(np.int64) | (p[:, 1].astype(np.int64) << 8),
+                                             wl.W, world) == rank)
+        shard_sizes.append(len(b["tid"]))
         host_batches.append(b)
     dev = torch.device("cuda", local)
 
     def to_t(a, pin):
+        if not isinstance(a, np.ndarray):
+            return a  # scalars (n_global)
         t = torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).copy())
         return t.pin_memory() if pin else t.to(dev)
 
+    home_dev = [torch.from_numpy(m).to(dev) for m in home_masks]
     for b in host_batches:
         dev_batches.append({k: to_t(v, False) for k, v in b.items()})
         hb = b
         if w["kind"] == "tpcc":  # host leg ships compact TPC-C records (LTPG_BATCH_COMPACT_PARAMS)
             packed, offs = ltpg.pack_params_compact(b["type"], b["params"])
             hb = {"tid": b["tid"], "type": b["type"], "params": packed, "offsets": offs}
+            if sharded:
+                hb.update(grank=b["grank"], n_global=b["n_global"])
         pin_batches.append({k: to_t(v, True) for k, v in hb.items()})
         if w["kind"] == "tpcc":
             pin_batches[-1]["compact"] = True
@@ -594,7 +603,10 @@ def main():
         ev[s][1].record(stream)
         clock += 1
         n_s = len(host_batches[i]["tid"])
-        commits.append(int((out["status"][:n_s] == 1).sum()))
+        if sharded:  # the commits of the txns this rank is home of (summed over ranks below)
+            commits.append(int(((out["status"][:n_s] == 1) & home_dev[i]).sum()))
+        else:
+            commits.append(int((out["status"][:n_s] == 1).sum()))
         procs.append(n_s)
     torch.cuda.synchronize()
     clk.mark(tw0, time.time())
@@ -612,9 +624,14 @@ def main():
         log("step ms:", ["%.3f" % x for x in step_ms])
         log("lib ms :", ["%.3f" % sum(st_[k] for k in st_ if k.startswith("ms_")) for st_ in stage])
     total_s = sum(step_ms) / 1000.0
-    # the global batch is partitioned over the ranks and the verdicts are exchanged, so
-    # every rank reports the same commits: count them once; time = max over ranks
+    # global batches: the verdicts are exchanged, every rank reports the same commits -- count
+    # them once; sharded: every rank counts its home txns -- sum; time = max over ranks
     all_commits, all_procs = float(sum(commits)), float(sum(procs))
+    if sharded:
+        t = torch.tensor([all_commits], dtype=torch.float64, device="cpu" if shared else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        all_commits = float(t.item())
+        all_procs = float(B * args.steps)
     if dist:
         t = torch.tensor([total_s], device="cpu" if shared else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -691,18 +708,24 @@ def main():
         def collect(p):
             nonlocal d2h
             out = p.wait()
-            n = len(out["status"])
+            n = shard_sizes[p.i]  # (the pinned output buffers are sized for the full batch)
             # commits: popcount of the returned commit bitmask (no per-stage instrumentation)
             cb = out["commit_bits"]
             cb = cb.numpy() if hasattr(cb, "numpy") else cb
-            e_commits.append(int(np.bitwise_count(cb[:(n + 31) // 32].view(np.uint32)).sum()))
-            nreads = n_reads if w["kind"] == "ycsb" else 4 * B
+            if sharded:  # the commits of this rank's home txns (status is downloaded anyway)
+                st_ = out["status"]
+                st_ = st_.numpy() if hasattr(st_, "numpy") else st_
+                e_commits.append(int(((st_[:n] == 1) & home_masks[p.i]).sum()))
+            else:
+                e_commits.append(int(np.bitwise_count(cb[:(n + 31) // 32].view(np.uint32)).sum()))
+            nreads = n_reads if w["kind"] == "ycsb" else 4 * n
             d2h += n + 4 * ((n + 31) // 32) + 4 * n + 8 * nreads + 68
 
         for s in range(args.steps):
             i = (args.warmup + s) % n_distinct
             bh = host_batches[i]
             inflight.append(run(None, bh, clock, False, False, wait=False, slot=s % 3))
+            inflight[-1].i = i
             clock += 1
             h2d += sum(v.nbytes for v in bp_of(bh).values() if hasattr(v, "nbytes"))
             if len(inflight) == 3:  # keep two batches queued behind the one completing
@@ -714,6 +737,10 @@ def main():
         clk.mark(tw0, time.time())
         e_s = e0.elapsed_time(e1) / 1000.0
         e_c = float(sum(e_commits))
+        if sharded:
+            t = torch.tensor([e_c], dtype=torch.float64, device="cpu" if shared else dev)
+            dist.all_reduce(t, op=dist.ReduceOp.SUM)
+            e_c = float(t.item())
         if dist:
             t = torch.tensor([e_s], device="cpu" if shared else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -767,11 +794,11 @@ def main():
             "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": dict(config_of(name), parallelism=(
-                "%d partitions (%s), same global batch, per-txn verdicts exchanged by %s"
-                % (world, "warehouse ranges" if w["kind"] == "tpcc" else "key ranges",
-                   "ncclAllReduce" if args.exchange == "nccl" else "peer-memory stores + signals (csrc/xchg.cu)"))
-                if world > 1
-                else "single GPU"),
+                ("%d ranks by warehouse range, SHARDED global batch (each rank gets the txns touching its "
+                 "warehouses; verdict bytes of cross-rank txns over peer memory, csrc/xchg.cu)" % world)
+                if sharded else
+                ("%d ranks by key range, same global batch on every rank, per-txn verdict planes over peer "
+                 "memory (csrc/xchg.cu)" % world) if world > 1 else "single GPU")),
             "clocks": clk.summary(), "e2e": e2e, "closed_loop": closed, "gpu_launches": kernels, "roofline": roof,
             "commit_rate": all_commits / all_procs, "processed_txns_per_s": all_procs / total_s,
             "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)
@@ -782,8 +809,10 @@ def main():
     line["gpus_requested"] = args.gpus
     line["gpus_active"] = min(world, ndev)
     line["ranks"] = world
-    line["exchange"] = (None if world == 1 else
-                        "ncclAllReduce" if args.exchange == "nccl" else "peer-memory stores + signals (csrc/xchg.cu)")
+    line["exchange"] = (None if world == 1 else "peer-memory stores + signals (csrc/xchg.cu)" +
+                        (", sharded batches" if sharded else ", global batches"))
+    if sharded:
+        line["shard_txns_rank0"] = statistics.mean(shard_sizes)
     if shared:
         line["config"]["devices"] = ("%d ranks on %d GPU(s): functional check of the multi-rank path, "
                                      "not a scaling number" % (world, ndev))

@@ -51,7 +51,7 @@ enum {
   LTPG_ENOMEM = -2,     /* device allocation failed                                */
   LTPG_ECAPACITY = -3,  /* an append region / index would overflow; nothing changed */
   LTPG_ECUDA = -4,      /* CUDA runtime error (db poisoned)                         */
-  LTPG_ENCCL = -5,      /* NCCL error (multi-GPU exchange; db poisoned)             */
+  LTPG_ERESERVED5 = -5, /* (unused)                                                 */
   LTPG_EPOISONED = -6,  /* an earlier device error poisoned this db: destroy it      */
   LTPG_EINTERNAL = -7   /* broken invariant (e.g. a required TPC-C row missing)      */
 };
@@ -129,8 +129,9 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
                                               WAW or (RAW and WAR); keeps per-unit min reader marks */
 #define LTPG_FLAG_UNFUSED       (1u << 3)  /* A/B: OPS mode runs validate+division and execute as
                                               two kernels with global per-kind lists          */
-#define LTPG_FLAG_NCCL_EXCHANGE (1u << 4)  /* world > 1, A/B baseline: exchange verdicts and result
-                                              sums with ncclAllReduce instead of peer memory   */
+#define LTPG_FLAG_RESERVED_4    (1u << 4)  /* reserved (EINVAL); round 1's ncclAllReduce exchange
+                                              baseline, removed: it could not run with several
+                                              ranks on one GPU, the only multi-rank setup tested */
 #define LTPG_FLAG_LARGE_BUCKETS (1u << 5)  /* NEXT-3: popularity is identified per batch
                                               ("in real time"): a table with E = T/D > 1
                                               (T = txns of the batch accessing it, D = its loaded
@@ -147,7 +148,6 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
 typedef struct {
   int device;                   /* CUDA device ordinal                                  */
   int rank, world;              /* partition of this process; world = 1: single GPU     */
-  const void* nccl_unique_id;   /* 128-byte ncclUniqueId (world > 1), else NULL          */
   uint32_t max_txns;            /* per-batch capacity                                    */
   uint32_t max_ops;             /* OPS mode per-batch op capacity                         */
   uint32_t flags;               /* LTPG_FLAG_*                                           */
@@ -157,18 +157,18 @@ typedef struct {
                                    ranges over partitions (tables with owner_rule 2)      */
 } ltpg_config;
 
-/* Multi-GPU: world > 1 ranks each own a contiguous range of warehouses
- * (TPC-C, owner_rule 1) or of keys (OPS, owner_rule 2).  Every rank calls ltpg_run_batch
- * with the same global batch; each executes, marks and checks only the units it owns,
- * then the per-txn conflict bits are exchanged before write-back, so commit_bits / status /
- * abort_idx are identical on all ranks.  Result slots are filled by the owning rank and
- * summed over ranks.  The exchange runs over peer memory (default, world <= 32): each rank
- * stores 4 bit planes per 32 txns into every peer's exchange region over NVLink and raises a
- * signal; the combine kernel waits for all signals (no host round trip).  Bootstrap: every
- * rank calls ltpg_peer_handle, the caller all-gathers the handles (e.g. torch.distributed)
- * and passes them, in rank order, to ltpg_connect_peers before the first batch.  With
- * LTPG_FLAG_NCCL_EXCHANGE the exchange is ncclAllReduce(MAX / SUM) on a communicator built
- * from nccl_unique_id instead.  Every rank must run the same sequence of batches, and
+/* Multi-GPU: world > 1 (<= 32) ranks each own a contiguous range of warehouses
+ * (TPC-C, owner_rule 1) or of keys (OPS, owner_rule 2).  Global batches: every rank calls
+ * ltpg_run_batch with the same global batch; each executes, marks and checks only the units it
+ * owns, then the per-txn conflict bits are exchanged before write-back, so commit_bits / status
+ * / abort_idx are identical on all ranks; result slots are filled by the owning rank and summed
+ * over ranks.  The exchange runs over peer memory: each rank stores 4 bit planes per 32 txns
+ * into every peer's exchange region over NVLink and raises a signal; the combine kernel waits
+ * for all signals (no host round trip).  TPC-C can instead run SHARDED batches (ltpg_batch.grank,
+ * see "Sharded batches"): each rank gets only the txns touching it, and only the bits of
+ * cross-rank txns travel.  Bootstrap: every rank calls ltpg_peer_handle, the caller all-gathers
+ * the handles (e.g. torch.distributed) and passes them, in rank order, to ltpg_connect_peers
+ * before the first batch.  Every rank must run the same sequence of batches, and
  * ltpg_destroy_db only after every rank finished its last batch (a barrier): peers read
  * this rank's region during their batches.  A peer that never arrives fails the batch
  * after 20 s (LTPG_EINTERNAL).  LTPG_FLAG_LOOPBACK_SHIFT runs P logical partitions inside
@@ -180,7 +180,7 @@ typedef struct ltpg_db ltpg_db;  /* opaque, library-owned device state */
 /* Create a database on config->device.  *out receives the handle. */
 LTPG_API int ltpg_create_db(const ltpg_config* config, ltpg_db** out);
 
-/* Peer-memory exchange bootstrap (world > 1 without LTPG_FLAG_NCCL_EXCHANGE).
+/* Peer-memory exchange bootstrap (world > 1).
  * ltpg_peer_handle writes this rank's LTPG_PEER_HANDLE_BYTES-byte handle (a CUDA IPC handle of
  * its exchange region plus the configuration it must match) to host memory `handle`.
  * ltpg_connect_peers takes all world handles back to back in rank order (host memory), checks
@@ -234,7 +234,23 @@ typedef struct {
                                    block is bytes [off[r], off[r+1]) (<= 128, the used prefix
                                    of its 128-byte block; the rest reads as zero).  NULL: fixed
                                    128-byte blocks.  Cuts the host->device bytes ~2x.       */
+  const uint32_t* grank;        /* TPCC, world > 1, optional [n_txns]: this is rank's SHARD of a
+                                   global batch (see "Sharded batches" below): the global rank of
+                                   each txn, strictly increasing, < n_global.  NULL: the batch is
+                                   the global batch (every rank passes all of it).            */
+  uint32_t n_global;            /* with grank: size of the global batch (<= max_txns)        */
 } ltpg_batch;
+
+/* Sharded batches (SURVEY §8(e) routing; world > 1, TPC-C): each rank receives only the txns
+ * that touch its warehouses -- home warehouse, NewOrder supply warehouses, Payment customer
+ * warehouse -- in global rank order, with their global ranks (ltpg_route_tpcc builds a rank's
+ * shard from the global batch on the host).  The conflict TIDs are the global ranks, so every
+ * unit's minimum marks are those of the whole batch.  Only the verdict bits of txns that touch
+ * several ranks cross NVLink (one byte per txn and peer, stored into the peers' exchange regions),
+ * plus the customer's (c_id, C_BALANCE) of a remote-customer Payment, returned to its home rank.
+ * Outputs are per shard (index i = the shard's i-th txn): status / commit_bits / abort_idx for
+ * every txn of the shard (identical on every rank that holds the txn); the result slots of a
+ * txn are final on its home rank (the rank of its home warehouse). */
 
 /* Inter-batch pipeline: with LTPG_BATCH_ASYNC, ltpg_run_batch enqueues the batch and
  * returns; host inputs are uploaded on an internal copy stream while the previous batch's
@@ -253,6 +269,16 @@ typedef struct {
  * other types: the used prefix of the block (as without this flag).
  * A record whose length does not match its header is LTPG_EINVAL (nothing changed). */
 #define LTPG_BATCH_COMPACT_PARAMS 2u
+/* a9 on the device (TPC-C): the batch is the previous batch's conflict aborts -- kept on the
+ * device with their original TIDs and parameter blocks, ascending ranks, never copied back to
+ * the host -- followed by the n_txns txns given (host inputs, fixed or compact blocks, TIDs
+ * larger than the carried ones).  The previous batch on this db must have completed (it is the
+ * last one submitted; ltpg_wait_batch for an async one); ltpg_pending_aborts tells how many txns
+ * it carries.  Outputs cover n_carried + n_txns txns (the carried ones first).  The previous
+ * batch's device input and abort-list buffers (when they were the caller's) must stay valid until
+ * this batch is submitted.  EINVAL: OPS mode, device inputs, a graph db, or no completed previous
+ * batch, or n_carried + n_txns > max_txns. */
+#define LTPG_BATCH_CARRY_ABORTS 4u
 
 typedef struct {
   float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;
@@ -284,6 +310,10 @@ LTPG_API int ltpg_run_batch(ltpg_db* db, const ltpg_batch* batch, ltpg_result* r
 
 /* Complete an asynchronously submitted batch (see LTPG_BATCH_ASYNC). */
 LTPG_API int ltpg_wait_batch(ltpg_db* db, ltpg_result* result);
+
+/* Number of conflict aborts an LTPG_BATCH_CARRY_ABORTS batch submitted now would carry (those of
+ * the last batch, once it completed; 0 if there is none or it is still in flight). */
+LTPG_API int ltpg_pending_aborts(ltpg_db* db, uint32_t* n_aborted);
 
 /* NEXT-3 / Table VIII: bytes of table t's conflict marks -- standard-sized (one word per
  * unit and kind) and large-sized buckets (LTPG_FLAG_LARGE_BUCKETS), as allocated -- and the bucket
@@ -321,6 +351,15 @@ typedef struct {
 } ltpg_batch_buf;
 LTPG_API int ltpg_compose_retry(const ltpg_batch* prev, const uint32_t* abort_idx, uint32_t n_aborted,
                                 const ltpg_batch* fresh, ltpg_batch_buf* out);
+
+/* Routing (host, no db or GPU needed): the shard of `rank` out of the global TPC-C batch
+ * `global` (host memory, fixed 128-byte blocks) for `world` ranks owning contiguous ranges of
+ * n_warehouses warehouses: the txns whose home / supply / customer warehouse the rank owns, in
+ * order, copied into out (tid, proc_type, proc_params) with their global ranks in grank[cap_txns];
+ * out->n_txns receives the shard size.  EINVAL: bad arguments or capacity too small. */
+LTPG_API int ltpg_route_tpcc(const ltpg_batch* global, uint32_t n_warehouses, uint32_t world, uint32_t rank,
+                             ltpg_batch_buf* out, uint32_t* grank);
+
 
 LTPG_API void ltpg_destroy_db(ltpg_db* db);
 LTPG_API const char* ltpg_last_error(const ltpg_db* db);

@@ -27,15 +27,13 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 # ---- constants (include/ltpg.h) ------------------------------------------------------
 LTPG_OK, LTPG_EINVAL, LTPG_ENOMEM, LTPG_ECAPACITY = 0, -1, -2, -3
-LTPG_ECUDA, LTPG_ENCCL, LTPG_EPOISONED, LTPG_EINTERNAL = -4, -5, -6, -7
-ERR_NAMES = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECAPACITY", -4: "ECUDA", -5: "ENCCL",
-             -6: "EPOISONED", -7: "EINTERNAL"}
+LTPG_ECUDA, LTPG_EPOISONED, LTPG_EINTERNAL = -4, -6, -7
+ERR_NAMES = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ECAPACITY", -4: "ECUDA", -6: "EPOISONED", -7: "EINTERNAL"}
 LTPG_MODE_OPS, LTPG_MODE_TPCC = 0, 1
 LTPG_FLAG_NO_GROUPING = 1 << 0
 LTPG_FLAG_NO_MARK_FILTER = 1 << 1
 LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_UNFUSED = 1 << 3
-LTPG_FLAG_NCCL_EXCHANGE = 1 << 4
 LTPG_FLAG_LARGE_BUCKETS = 1 << 5
 LTPG_FLAG_GRAPH = 1 << 6
 LTPG_PEER_HANDLE_BYTES = 128
@@ -48,7 +46,7 @@ c_u32, c_u64, c_i64, c_int, c_vp = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_in
 
 
 class ltpg_config(ctypes.Structure):
-    _fields_ = [("device", c_int), ("rank", c_int), ("world", c_int), ("nccl_unique_id", c_vp),
+    _fields_ = [("device", c_int), ("rank", c_int), ("world", c_int),
                 ("max_txns", c_u32), ("max_ops", c_u32), ("flags", c_u32), ("n_tables", c_u32),
                 ("n_warehouses", c_u32), ("key_space", c_u64)]
 
@@ -62,7 +60,7 @@ class ltpg_batch(ctypes.Structure):
     _fields_ = [("n_txns", c_u32), ("tid", c_vp), ("mode", c_u32), ("n_ops", c_u32), ("op_begin", c_vp),
                 ("ops", c_vp), ("op_arg", c_vp), ("proc_type", c_vp), ("proc_params", c_vp),
                 ("batch_clock", c_i64), ("inputs_on_device", c_int), ("stream", c_vp), ("flags", c_u32),
-                ("proc_offsets", c_vp)]
+                ("proc_offsets", c_vp), ("grank", c_vp), ("n_global", c_u32)]
 
 
 class ltpg_stats(ctypes.Structure):
@@ -108,6 +106,10 @@ class ltpg_batch_buf(ctypes.Structure):
 _lib.ltpg_compose_retry.restype = c_int
 _lib.ltpg_compose_retry.argtypes = [ctypes.POINTER(ltpg_batch), c_vp, c_u32, ctypes.POINTER(ltpg_batch),
                                     ctypes.POINTER(ltpg_batch_buf)]
+_lib.ltpg_pending_aborts.restype = c_int
+_lib.ltpg_pending_aborts.argtypes = [c_vp, ctypes.POINTER(c_u32)]
+_lib.ltpg_route_tpcc.restype = c_int
+_lib.ltpg_route_tpcc.argtypes = [ctypes.POINTER(ltpg_batch), c_u32, c_u32, c_u32, ctypes.POINTER(ltpg_batch_buf), c_vp]
 _lib.ltpg_mark_memory.restype = c_int
 _lib.ltpg_mark_memory.argtypes = [c_vp, c_u32, ctypes.POINTER(c_u64), ctypes.POINTER(c_u64), ctypes.POINTER(c_u32)]
 _lib.ltpg_version.restype = ctypes.c_char_p
@@ -126,12 +128,15 @@ ltpg_peer_handle = _lib.ltpg_peer_handle
 ltpg_connect_peers = _lib.ltpg_connect_peers
 ltpg_compose_retry = _lib.ltpg_compose_retry
 ltpg_mark_memory = _lib.ltpg_mark_memory
+ltpg_route_tpcc = _lib.ltpg_route_tpcc
+ltpg_pending_aborts = _lib.ltpg_pending_aborts
 LTPG_BATCH_ASYNC = 1
 LTPG_BATCH_COMPACT_PARAMS = 2
+LTPG_BATCH_CARRY_ABORTS = 4
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
             "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers",
-            "ltpg_compose_retry", "ltpg_mark_memory"]
+            "ltpg_compose_retry", "ltpg_mark_memory", "ltpg_route_tpcc", "ltpg_pending_aborts"]
 
 
 class LtpgError(RuntimeError):
@@ -156,16 +161,12 @@ class Database:
     """One device database (tables + PK indexes + conflict marks) on one GPU."""
 
     def __init__(self, n_tables, max_txns, max_ops=0, device=0, flags=0, n_warehouses=0, rank=0, world=1,
-                 nccl_unique_id=None, key_space=0, loopback=1):
+                 key_space=0, loopback=1):
         self._keep = []
         flags |= (int(loopback) & 0xF) << LTPG_FLAG_LOOPBACK_SHIFT if loopback > 1 else 0
-        cfg = ltpg_config(device=device, rank=rank, world=world, nccl_unique_id=None, max_txns=max_txns,
+        cfg = ltpg_config(device=device, rank=rank, world=world, max_txns=max_txns,
                           max_ops=max_ops, flags=flags, n_tables=n_tables, n_warehouses=n_warehouses,
                           key_space=key_space)
-        if nccl_unique_id is not None:
-            buf = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
-            self._keep.append(buf)
-            cfg.nccl_unique_id = ctypes.cast(buf, c_vp)
         h = c_vp()
         rc = ltpg_create_db(ctypes.byref(cfg), ctypes.byref(h))
         self.h = h
@@ -278,21 +279,34 @@ class Database:
                         stream=c_vp(stream) if stream else None)
         return self._run(bt, n, n_ops, want_reads, device_out, stats, out, wait, keep=batch)
 
+    def pending_aborts(self):
+        """Conflict aborts a carry=True batch would lead with (ltpg_pending_aborts)."""
+        n = c_u32(0)
+        self._check(ltpg_pending_aborts(self.h, ctypes.byref(n)))
+        return n.value
+
     def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
-                 n_txns=None, wait=True):
+                 n_txns=None, wait=True, carry=False):
         """batch: dict(tid u64[n], type u8[n], params u8[n,128]) -- or packed blocks:
         params = used bytes back to back and offsets u32[n+1] (see pack_params), or compact
-        records with compact=True (see pack_params_compact)."""
+        records with compact=True (see pack_params_compact).  A rank's shard of a global batch
+        (route_tpcc) also carries grank u32[n] and n_global.  carry=True: the batch is the previous
+        batch's conflict aborts (kept on the device) followed by these txns
+        (LTPG_BATCH_CARRY_ABORTS); the outputs cover pending_aborts() + n txns."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
         offsets = batch.get("offsets")
-        n = len(tid) if n_txns is None else n_txns
+        grank = batch.get("grank")
+        nf = len(tid) if n_txns is None else n_txns
+        n = nf + (self.pending_aborts() if carry else 0)
         on_dev = _on_device(tid)
         if device_out is None:
             device_out = on_dev
-        bt = ltpg_batch(n_txns=n, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
+        bt = ltpg_batch(n_txns=nf, tid=_ptr(tid), mode=LTPG_MODE_TPCC, proc_type=_ptr(ty),
                         proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
                         stream=c_vp(stream) if stream else None, proc_offsets=_ptr(offsets),
-                        flags=LTPG_BATCH_COMPACT_PARAMS if batch.get("compact") else 0)
+                        flags=(LTPG_BATCH_COMPACT_PARAMS if batch.get("compact") else 0) |
+                        (LTPG_BATCH_CARRY_ABORTS if carry else 0),
+                        grank=_ptr(grank), n_global=int(batch.get("n_global", 0)))
         out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch)
         if wait and not device_out and want_reads:
             out["reads"] = out["reads"].reshape(n, 4)
@@ -418,11 +432,11 @@ def part_of_key(key, key_space, nparts):
 
 
 def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0, loopback=1, rank=0, world=1,
-                  nccl_unique_id=None, peer_group=None):
+                  peer_group=None):
     """YCSB usertable, key-range partitioned (owner_rule 2) when world * loopback > 1; a
     multi-rank db loads only its own key range."""
     db = Database(1, max_txns, max_ops, device=device, flags=flags, key_space=workload.n_rows, loopback=loopback,
-                  rank=rank, world=world, nccl_unique_id=nccl_unique_id)
+                  rank=rank, world=world)
     g, a, ng, pk = workload.table_desc()
     keys, cols = workload.initial_table()
     if world > 1:
@@ -435,7 +449,7 @@ def ycsb_database(workload, max_txns, max_ops, capacity=None, device=0, flags=0,
 
 def _connect(db, world, flags, group):
     """Multi-rank db with the peer-memory exchange: all-gather the handles (torch.distributed)."""
-    if world > 1 and not (flags & LTPG_FLAG_NCCL_EXCHANGE):
+    if world > 1:
         from .dist import connect_peers
         connect_peers(db, group)
 
@@ -462,12 +476,12 @@ def tpcc_owner_w(t, keys, cols):
 
 
 def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, flags=0, capacity=None,
-                  loopback=1, rank=0, world=1, nccl_unique_id=None, max_ops=0, peer_group=None):
+                  loopback=1, rank=0, world=1, max_ops=0, peer_group=None):
     """Load the TPC-C schema; append regions sized for ``append_batches`` batches of max_txns.
     A multi-rank db (world > 1) loads only the rows of its warehouses (ITEM replicated)."""
     from workloads.formats import T_ORDER, T_NEW_ORDER, T_ORDER_LINE, T_HISTORY, T_ITEM
     db = Database(9, max_txns, max_ops, device=device, flags=flags, n_warehouses=workload.W, loopback=loopback,
-                  rank=rank, world=world, nccl_unique_id=nccl_unique_id)
+                  rank=rank, world=world)
     from .dist import tpcc_rank_tables
     tables = tables if tables is not None else workload.initial_tables()
     if world > 1:
@@ -486,6 +500,27 @@ def tpcc_database(workload, max_txns, tables=None, append_batches=4, device=0, f
                       layout=LTPG_LAYOUT_COLUMNAR if t in (T_ORDER, T_ORDER_LINE) else LTPG_LAYOUT_ROWBLOCK)
     _connect(db, world, flags, peer_group)
     return db
+
+
+def route_tpcc(batch, n_warehouses, world, rank):
+    """SURVEY §8(e) host routing (ltpg_route_tpcc): rank's shard of a global TPC-C batch -- the
+    txns touching its warehouses, in order -- as a batch dict with grank (global ranks) and
+    n_global, ready for Database.run_tpcc."""
+    b = {k: np.ascontiguousarray(batch[k]) for k in ("tid", "type", "params")}
+    n = len(b["tid"])
+    gb = ltpg_batch(n_txns=n, tid=_ptr(b["tid"]), mode=LTPG_MODE_TPCC, proc_type=_ptr(b["type"]),
+                    proc_params=_ptr(b["params"]))
+    out = {"tid": np.zeros(max(n, 1), np.uint64), "type": np.zeros(max(n, 1), np.uint8),
+           "params": np.zeros((max(n, 1), LTPG_PARAM_BYTES), np.uint8)}
+    grank = np.zeros(max(n, 1), np.uint32)
+    buf = ltpg_batch_buf(cap_txns=n, tid=_ptr(out["tid"]), proc_type=_ptr(out["type"]),
+                         proc_params=_ptr(out["params"]))
+    rc = ltpg_route_tpcc(ctypes.byref(gb), n_warehouses, world, rank, ctypes.byref(buf), grank.ctypes.data_as(c_vp))
+    if rc:
+        raise LtpgError(rc, "ltpg_route_tpcc: invalid arguments")
+    m = buf.n_txns
+    return {"tid": out["tid"][:m], "type": out["type"][:m], "params": out["params"][:m], "grank": grank[:m],
+            "n_global": n}
 
 
 def compose_retry(prev, abort_idx, fresh, max_txns, max_ops=0):

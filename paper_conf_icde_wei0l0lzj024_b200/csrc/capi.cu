@@ -1,14 +1,11 @@
 // C-ABI implementation (include/ltpg.h): device store management and the
 // per-batch driver.  One ltpg_run_batch enqueues, on the caller's stream:
 //   upload -> [per partition: K-group -> K-claim -> K-exec -> K-detect]
-//   -> exchange (partitioned only: loopback max / ncclAllReduce MAX)
+//   -> exchange (partitioned only: loopback OR / peer-memory stores between ranks)
 //   -> [per partition: K-wb] -> finalize (commit bits, abort list) -> download
 // The paper separates its three kernels with cudaDeviceSynchronize() (P:122,
 // P:137-141); here stream order gives the same global isolation with no host
 // round trip inside the batch.
-#include <dlfcn.h>
-#include <nccl.h>
-
 #include <algorithm>
 #include <atomic>
 #include <cmath>
@@ -24,29 +21,6 @@
 using namespace ltpg;
 
 namespace {
-
-// ---- NCCL, loaded lazily (only multi-rank dbs need it) -------------------------------------
-struct Nccl {
-  void* h = nullptr;
-  ncclResult_t (*commInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
-  ncclResult_t (*allReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
-                            cudaStream_t) = nullptr;
-  ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
-  const char* (*getErrorString)(ncclResult_t) = nullptr;
-  bool load() {
-    if (h) return true;
-    const char* names[] = {"libnccl.so.2", "libnccl.so"};
-    for (const char* n : names)
-      if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
-    if (!h) return false;
-    commInitRank = reinterpret_cast<decltype(commInitRank)>(dlsym(h, "ncclCommInitRank"));
-    allReduce = reinterpret_cast<decltype(allReduce)>(dlsym(h, "ncclAllReduce"));
-    commDestroy = reinterpret_cast<decltype(commDestroy)>(dlsym(h, "ncclCommDestroy"));
-    getErrorString = reinterpret_cast<decltype(getErrorString)>(dlsym(h, "ncclGetErrorString"));
-    return commInitRank && allReduce && commDestroy && getErrorString;
-  }
-};
-Nccl g_nccl;
 
 uint64_t g_tab_versions = 0;
 constexpr uint64_t LARGE_BUCKET_BYTES = 64ull << 20;  // NEXT-3 bucket memory cap per table     // process-wide: every table load gets a new version
@@ -64,6 +38,7 @@ struct Part {
   uint32_t* txn_ins = nullptr;
   uint8_t* ua = nullptr;
   uint8_t* lflag = nullptr;
+  uint32_t* pmask = nullptr;             // sharded batches: partitions each shard txn touches
   uint32_t* small = nullptr;             // [0] err [1] ins_tables [2..7] kcount
   unsigned long long* base = nullptr;    // [MAXT]
   TpccDev tpcc;
@@ -89,6 +64,7 @@ constexpr int GRAPHS_PER_SLOT = 4;
 // one in-flight batch: input staging, device outputs, pinned small results, events
 struct Slot {
   unsigned long long* d_tid = nullptr;
+  uint32_t* d_grank = nullptr;             // sharded batches: global ranks of the shard's txns
   uint32_t* d_op_begin = nullptr;
   ltpg_op* d_ops = nullptr;
   long long* d_args = nullptr;
@@ -114,6 +90,13 @@ struct Slot {
   BatchVars* h_vars = nullptr;             // pinned + mapped host copy (read by graph replays)
   BatchVars* h_vars_dev = nullptr;         // its device-side address
   GraphEntry graphs[GRAPHS_PER_SLOT];
+  // the batch's effective device inputs and abort list (LTPG_BATCH_CARRY_ABORTS of the next one)
+  const unsigned long long* eff_tid = nullptr;
+  const uint8_t* eff_ptype = nullptr;
+  const uint8_t* eff_params = nullptr;
+  const uint32_t* eff_abort = nullptr;
+  uint64_t seq = 0;
+  bool carry_src = false;  // a TPC-C batch of a single-rank db: its aborts can be carried
 };
 
 }  // namespace
@@ -143,13 +126,17 @@ struct ltpg_db {
   unsigned long long* d_idx_from = nullptr;  // [MAXT]
   uint16_t* d_su = nullptr;                  // [MAXT] NEXT-3: this batch's bucket size per table
   std::vector<Part> parts;
-  uint8_t* d_xchg = nullptr;               // [n + 4] exchange buffer (flags + error bytes)
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_scan = nullptr;
   // inter-batch pipeline (NEXT-2): three slots, each with its own input staging and
   // output buffers, so batch n+1's H2D and batch n-1's D2H overlap batch n's kernels
   Slot slots[3];
   uint64_t submitted = 0;
+  // LTPG_BATCH_CARRY_ABORTS: the last completed batch's conflict aborts, still on the device
+  bool carry_ok = false;
+  uint64_t carry_seq = 0;
+  uint32_t carry_n = 0;
+  int carry_slot = -1;
   cudaStream_t h2d = nullptr, d2h = nullptr;
   cudaStream_t cap = nullptr;              // batch graphs are captured here (never executes work)
   // batches execute in submission order even when the caller passes different streams:
@@ -163,8 +150,7 @@ struct ltpg_db {
   uint32_t* d_scan_fin = nullptr;
   unsigned long long* d_fc_state = nullptr;  // a8 look-back tile states; [0] of d_fc_ctr: tile counter
   uint32_t* d_fc_ctr = nullptr;
-  ncclComm_t comm = nullptr;
-  // peer-memory exchange (world > 1 without LTPG_FLAG_NCCL_EXCHANGE; xchg.cuh)
+  // peer-memory exchange between ranks (world > 1; xchg.cuh)
   bool p2p = false, connected = false;
   XLayout xl;
   XPeers xpeers{};
@@ -189,7 +175,7 @@ namespace {
 int fail(ltpg_db* db, int code, const std::string& msg) {
   if (db) {
     db->last_error = msg;
-    if (code == LTPG_ECUDA || code == LTPG_ENCCL || code == LTPG_EINTERNAL) db->poisoned = true;
+    if (code == LTPG_ECUDA || code == LTPG_EINTERNAL) db->poisoned = true;
   }
   return code;
 }
@@ -245,30 +231,6 @@ __global__ void k_combine(void* const* lflags, uint32_t np, uint32_t n, uint8_t*
 __global__ void k_spread_err(const uint32_t* err_all, void* const* errs, uint32_t np) {
   for (uint32_t p = 0; p < np; ++p) *static_cast<uint32_t*>(errs[p]) = *err_all;
 }
-// NCCL has no bitwise-OR reduction: one byte per conflict bit, allreduce MAX, then unpack.
-// x = [4n bytes: txn r -> bytes 4r..4r+3 = ua, waw, raw, war] [3 error bytes]
-__global__ void k_pack(const uint8_t* lflag, const uint32_t* err, uint8_t* x, uint32_t n) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r < n) {
-    const uint32_t f = lflag[r];
-    *reinterpret_cast<uchar4*>(x + 4ull * r) = make_uchar4(f & 1u, (f >> 1) & 1u, (f >> 2) & 1u, (f >> 3) & 1u);
-  }
-  if (r < 3) x[4ull * n + r] = (*err >> r) & 1u;
-}
-__global__ void k_unpack(const uint8_t* x, uint32_t n, uint8_t* status, uint32_t* err, uint32_t* err_all,
-                         bool reorder) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r < n) {
-    const uchar4 v = *reinterpret_cast<const uchar4*>(x + 4ull * r);
-    const uint32_t f = (v.x ? CF_UA : 0u) | (v.y ? CF_WAW : 0u) | (v.z ? CF_RAW : 0u) | (v.w ? CF_WAR : 0u);
-    status[r] = status_of_bits(f, reorder);
-  }
-  if (r == 0) {
-    const uint32_t e = (uint32_t)x[4ull * n] | (uint32_t)x[4ull * n + 1] << 1 | (uint32_t)x[4ull * n + 2] << 2;
-    *err = e;
-    *err_all = e;
-  }
-}
 __global__ void k_sum_res(void* const* res, uint32_t np, uint64_t n, long long* out) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     unsigned long long s = 0;
@@ -323,9 +285,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   const uint32_t loop = std::max<uint32_t>(1, (cfg->flags >> LTPG_FLAG_LOOPBACK_SHIFT) & 0xF);
   if (cfg->n_tables == 0 || cfg->n_tables > MAXT || cfg->max_txns == 0 || cfg->world < 1 ||
       cfg->rank < 0 || cfg->rank >= cfg->world || cfg->max_txns > (1u << 24) || cfg->max_ops > (1u << 24) ||
-      cfg->n_warehouses > 1000 || cfg->world * loop > 64 ||
-      (cfg->world > 1 && (cfg->flags & LTPG_FLAG_NCCL_EXCHANGE) && !cfg->nccl_unique_id) ||
-      (cfg->world > 32 && !(cfg->flags & LTPG_FLAG_NCCL_EXCHANGE)) ||
+      cfg->n_warehouses > 1000 || cfg->world * loop > 64 || cfg->world > 32 || (cfg->flags & LTPG_FLAG_RESERVED_4) ||
       (cfg->world > 1 && loop > 1))
     return LTPG_EINVAL;
   db = new ltpg_db();
@@ -350,6 +310,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   for (int t = 0; t < MAXT; ++t) db->h_tab[t].n_rows = db->d_nrows + t;
   for (Slot& S : db->slots) {
     CK(dmalloc(&S.d_tid, n));
+    CK(dmalloc(&S.d_grank, n));
     CK(dmalloc(&S.d_op_begin, n + 1));
     CK(dmalloc(&S.d_ops, m));
     CK(dmalloc(&S.d_args, m));
@@ -374,7 +335,6 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(cudaHostAlloc(reinterpret_cast<void**>(&S.h_vars), sizeof(BatchVars), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S.h_vars_dev), S.h_vars, 0));
   }
-  CK(dmalloc(&db->d_xchg, 4 * n + 4));
   CK(dmalloc(&db->d_ptrs, 3 * 64));
   CK(dmalloc(&db->d_scan, scan_scratch_words(std::max<size_t>(n, m)) + 16));
   CK(cudaStreamCreateWithFlags(&db->h2d, cudaStreamNonBlocking));
@@ -400,6 +360,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&P.txn_ins, n + 1));
     CK(dmalloc(&P.ua, n));
     CK(dmalloc(&P.lflag, n));
+    CK(dmalloc(&P.pmask, n));
     CK(dmalloc(&P.small, 64));
     CK(dmalloc(&P.base, MAXT));
     int rc = tpcc_alloc(P.tpcc, cfg->max_txns, cfg->n_warehouses, p ? db->parts[0].tpcc.by_name : nullptr);
@@ -412,7 +373,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     ptrs[128 + p] = P.res;
   }
   CK(cudaMemcpy(db->d_ptrs, ptrs.data(), ptrs.size() * sizeof(void*), cudaMemcpyHostToDevice));
-  if (cfg->world > 1 && !(cfg->flags & LTPG_FLAG_NCCL_EXCHANGE)) {  // peer-memory exchange region
+  if (cfg->world > 1) {  // peer-memory exchange region
     db->p2p = true;
     db->xl.init(cfg->max_txns, nres, (uint32_t)cfg->world);
     CK(cudaMalloc(reinterpret_cast<void**>(&db->xregion), db->xl.bytes));
@@ -421,12 +382,6 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(cudaMemset(db->d_xdone, 0, 2 * sizeof(uint32_t)));
     CK(dmalloc(&db->d_xsink, nres));
     db->xpeers.base[cfg->rank] = db->xregion;
-  } else if (cfg->world > 1) {
-    if (!g_nccl.load()) return fail(db, LTPG_ENCCL, "libnccl.so.2 not loadable");
-    ncclUniqueId id;
-    std::memcpy(&id, cfg->nccl_unique_id, sizeof(id));
-    ncclResult_t r = g_nccl.commInitRank(&db->comm, cfg->world, id, cfg->rank);
-    if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclCommInitRank: ") + g_nccl.getErrorString(r));
   }
   return LTPG_OK;
 }
@@ -436,12 +391,12 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
-  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_xchg, db->d_ptrs, db->d_scan,
+  void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_ptrs, db->d_scan,
                   db->d_idx_from, db->d_su};
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
-    void* sb[] = {S.d_tid, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_packed, S.d_offsets,
+    void* sb[] = {S.d_tid, S.d_grank, S.d_op_begin, S.d_ops, S.d_args, S.d_ptype, S.d_params, S.d_packed, S.d_offsets,
                   S.d_res, S.d_status,
                   S.d_bits, S.d_flags, S.d_offs, S.d_abort, S.d_small, S.d_vars};
     for (void* p : sb)
@@ -466,12 +421,11 @@ void ltpg_destroy_db(ltpg_db* db) {
   if (db->d_fc_state) cudaFree(db->d_fc_state);
   if (db->d_fc_ctr) cudaFree(db->d_fc_ctr);
   for (Part& P : db->parts) {
-    void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.small, P.base};
+    void* pb[] = {P.res, P.uref, P.items, P.txn_ins, P.ua, P.lflag, P.pmask, P.small, P.base};
     for (void* p : pb)
       if (p) cudaFree(p);
     tpcc_free(P.tpcc);
   }
-  if (db->comm) g_nccl.commDestroy(db->comm);
   for (void* p : db->opened) cudaIpcCloseMemHandle(p);
   if (db->xregion) cudaFree(db->xregion);
   if (db->d_xdone) cudaFree(db->d_xdone);
@@ -663,12 +617,19 @@ namespace {
 // Complete the batch held by slot S: wait for its outputs, report errors / counts / stages.
 int finish_slot(ltpg_db* db, Slot& S) {
   S.pending = false;
+  db->carry_ok = false;
   CK(cudaEventSynchronize(S.out_done));
   const uint32_t err = S.h_small[0];
   if (err & ERR_EINTERNAL) return fail(db, LTPG_EINTERNAL, "device invariant violated");
   if (err & ERR_EINVAL) return fail(db, LTPG_EINVAL, "invalid batch (validated on device; nothing changed)");
   if (err & ERR_ECAPACITY) return fail(db, LTPG_ECAPACITY, "append capacity exceeded (nothing changed)");
   if (S.host_out) *S.res->n_aborted = S.h_small[16];
+  if (S.carry_src) {  // its conflict aborts can lead the next batch (LTPG_BATCH_CARRY_ABORTS)
+    db->carry_ok = true;
+    db->carry_seq = S.seq;
+    db->carry_n = S.h_small[16];
+    db->carry_slot = (int)(&S - db->slots);
+  }
   if (S.timing && S.empty) {  // nothing ran: no stage events were recorded
     *S.res->stats = ltpg_stats{};
   } else if (S.timing) {
@@ -695,6 +656,12 @@ int finish_slot(ltpg_db* db, Slot& S) {
 
 extern "C" {
 
+int ltpg_pending_aborts(ltpg_db* db, uint32_t* n) {
+  if (!db || !n) return LTPG_EINVAL;
+  *n = (db->carry_ok && db->carry_seq == db->submitted) ? db->carry_n : 0u;
+  return LTPG_OK;
+}
+
 int ltpg_wait_batch(ltpg_db* db, ltpg_result* res) {
   if (!db || !res) return LTPG_EINVAL;
   for (Slot& S : db->slots)
@@ -707,9 +674,16 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (db->poisoned) return LTPG_EPOISONED;
   if (!b || !res || !b->tid || !res->status || !res->commit_bits || !res->abort_idx || !res->n_aborted)
     return fail(db, LTPG_EINVAL, "null argument");
-  const uint32_t n = b->n_txns;
-  if (n > db->cfg.max_txns) return fail(db, LTPG_EINVAL, "n_txns > max_txns");
+  const uint32_t nf = b->n_txns;  // txns given (LTPG_BATCH_CARRY_ABORTS: after the carried ones)
   const bool ops_mode = b->mode == LTPG_MODE_OPS;
+  const bool carry = (b->flags & LTPG_BATCH_CARRY_ABORTS) != 0;
+  if (carry && (ops_mode || b->inputs_on_device || db->cfg.world > 1 || (db->cfg.flags & LTPG_FLAG_GRAPH) ||
+                !db->carry_ok || db->carry_seq != db->submitted))
+    return fail(db, LTPG_EINVAL, "LTPG_BATCH_CARRY_ABORTS: TPCC host inputs on a single-rank, non-graph db, after "
+                                 "the previous batch completed");
+  const uint32_t nc = carry ? db->carry_n : 0u;  // carried conflict aborts of the previous batch
+  const uint32_t n = nc + nf;
+  if ((uint64_t)nc + nf > db->cfg.max_txns) return fail(db, LTPG_EINVAL, "n_txns > max_txns"); 
   if (!ops_mode && b->mode != LTPG_MODE_TPCC) return fail(db, LTPG_EINVAL, "bad mode");
   if (ops_mode && (b->n_ops > db->cfg.max_ops || !b->op_begin || (b->n_ops && (!b->ops || !b->op_arg))))
     return fail(db, LTPG_EINVAL, "bad OPS batch");
@@ -718,8 +692,11 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if ((b->flags & LTPG_BATCH_COMPACT_PARAMS) && (ops_mode || !b->proc_offsets))
     return fail(db, LTPG_EINVAL, "LTPG_BATCH_COMPACT_PARAMS needs a TPCC batch with proc_offsets");
   if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
-  if (!ops_mode && b->proc_offsets && !b->inputs_on_device && b->proc_offsets[n] > (uint64_t)n * LTPG_PARAM_BYTES)
+  if (!ops_mode && b->proc_offsets && !b->inputs_on_device && b->proc_offsets[nf] > (uint64_t)nf * LTPG_PARAM_BYTES)
     return fail(db, LTPG_EINVAL, "packed params too large");
+  const bool sharded = b->grank != nullptr;
+  if (sharded && (ops_mode || !db->p2p || b->n_global > db->cfg.max_txns || n > b->n_global))
+    return fail(db, LTPG_EINVAL, "sharded batches: TPCC on a multi-rank peer-memory db, n_txns <= n_global <= max_txns");
   // every host-side validation is above this line: from here on the batch is submitted
   Slot& S = db->slots[db->submitted % 3];
   if (S.pending) return fail(db, LTPG_EINVAL, "three batches already in flight: ltpg_wait_batch first");
@@ -748,6 +725,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.flags = db->cfg.flags;
   bd.vars = S.d_vars;
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
+  bd.n_global = sharded ? b->n_global : n;
   // verdict outputs: written in place when the caller's buffers are on the device
   uint8_t* st_out = S.host_out ? S.d_status : res->status;
   uint32_t* bits_out = S.host_out ? S.d_bits : res->commit_bits;
@@ -755,6 +733,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.status = st_out;
   const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
   if (b->inputs_on_device) {
+    bd.grank = b->grank;
     bd.tid = reinterpret_cast<const unsigned long long*>(b->tid);
     bd.op_begin = b->op_begin;
     bd.ops = b->ops;
@@ -764,8 +743,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   } else {
     // the slot's staging buffers are free once its previous batch's kernels are done
     CK(cudaStreamWaitEvent(db->h2d, S.comp_done, 0));
-    CK(cudaMemcpyAsync(S.d_tid, b->tid, n * sizeof(uint64_t), h2d, db->h2d));
+    // (carried txns: positions [0, nc) are filled on the device by k_carry; the given ones follow)
+    CK(cudaMemcpyAsync(S.d_tid + nc, b->tid, nf * sizeof(uint64_t), h2d, db->h2d));
     bd.tid = S.d_tid;
+    if (sharded) {
+      CK(cudaMemcpyAsync(S.d_grank, b->grank, n * sizeof(uint32_t), h2d, db->h2d));
+      bd.grank = S.d_grank;
+    }
     if (ops_mode) {
       CK(cudaMemcpyAsync(S.d_op_begin, b->op_begin, (n + 1) * sizeof(uint32_t), h2d, db->h2d));
       if (b->n_ops) {
@@ -776,13 +760,14 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       bd.ops = S.d_ops;
       bd.args = S.d_args;
     } else {
-      CK(cudaMemcpyAsync(S.d_ptype, b->proc_type, n, h2d, db->h2d));
+      CK(cudaMemcpyAsync(S.d_ptype + nc, b->proc_type, nf, h2d, db->h2d));
       if (b->proc_offsets) {  // packed blocks: offsets + used bytes only, expanded on the GPU
-        const uint64_t packed = b->proc_offsets[n];  // <= n * 128 (checked before submission)
-        CK(cudaMemcpyAsync(S.d_offsets, b->proc_offsets, (n + 1) * sizeof(uint32_t), h2d, db->h2d));
+        const uint64_t packed = b->proc_offsets[nf];  // <= nf * 128 (checked before submission)
+        CK(cudaMemcpyAsync(S.d_offsets, b->proc_offsets, (nf + 1) * sizeof(uint32_t), h2d, db->h2d));
         CK(cudaMemcpyAsync(S.d_packed, b->proc_params, packed, h2d, db->h2d));
       } else {
-        CK(cudaMemcpyAsync(S.d_params, b->proc_params, (size_t)n * LTPG_PARAM_BYTES, h2d, db->h2d));
+        CK(cudaMemcpyAsync(S.d_params + (size_t)nc * LTPG_PARAM_BYTES, b->proc_params, (size_t)nf * LTPG_PARAM_BYTES,
+                           h2d, db->h2d));
       }
       bd.ptype = S.d_ptype;
       bd.params = S.d_params;
@@ -852,8 +837,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     BatchDev& x = pb[p];
     x.part = (uint32_t)db->cfg.rank * L + p;
     x.res = (!partitioned && p == 0) ? res_out : P.res;
-    if (db->p2p)  // own result slots live in the exchange region (peers pull them), by parity
+    if (db->p2p && !sharded)  // own result slots live in the exchange region (peers pull them), by parity
       x.res = reinterpret_cast<long long*>(db->xregion + db->xl.off_res) + (uint64_t)(db->epoch & 1u) * db->xl.nres;
+    if (sharded) x.res = res_out;  // every result slot is final on its home rank: written in place
+    x.pmask = sharded ? P.pmask : nullptr;
     x.uref = P.uref;
     x.items = P.items;
     x.txn_ins = P.txn_ins;
@@ -894,13 +881,20 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
       }
     }
+    if (nc) {  // a9 on the device: the previous batch's conflict aborts lead this batch
+      const Slot& P = db->slots[db->carry_slot];
+      launch_carry(P.eff_tid, P.eff_ptype, P.eff_params, P.eff_abort, nc, S.d_tid, S.d_ptype, S.d_params, s);
+      // the source slot's staging is reused only after this read (its next upload waits on it)
+      CK(cudaEventRecord(db->slots[db->carry_slot].comp_done, s));
+    }
     if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> every partition)
       const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
       const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
+      uint8_t* dst = S.d_params + (size_t)nc * LTPG_PARAM_BYTES;
       if (b->flags & LTPG_BATCH_COMPACT_PARAMS)
-        launch_unpack_compact(packed, offs, bd.ptype, n, S.d_params, pb[0].err, s);
+        launch_unpack_compact(packed, offs, bd.ptype + nc, nf, dst, pb[0].err, s);
       else
-        launch_unpack_params(packed, offs, n, S.d_params, pb[0].err, s);
+        launch_unpack_params(packed, offs, nf, dst, pb[0].err, s);
       for (uint32_t p = 1; p < L; ++p) {
         k_copy_err<<<1, 1, 0, s>>>(pb[0].err, pb[p].err);
         note_launch();
@@ -944,18 +938,18 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (timed) CK(tmark(S.ev[4], s));
     // ---- exchange of per-txn verdicts (partitioned only) ---------------------------------------
     if (partitioned) {
-      if (db->p2p) {  // planes stored into every rank's region, signal, wait + OR (xchg.cuh)
+      if (sharded) {  // bytes of cross-rank txns + remote-customer results, signal, wait + OR (xchg.cuh)
+        launch_xput_sharded(pb[0].lflag, pb[0].pmask, bd.grank, bd.ptype, bd.params, pb[0].res, pb[0].err, n,
+                            db->xpeers, db->xl, (uint32_t)db->cfg.rank, db->cfg.n_warehouses, db->epoch, db->d_xdone, s);
+        launch_xcombine_sharded(db->xregion, db->xl, n, db->epoch, reorder, st_out, pb[0].lflag, pb[0].pmask,
+                                bd.grank, bd.ptype, bd.params, pb[0].res, (uint32_t)db->cfg.rank, db->cfg.n_warehouses,
+                                pb[0].err, S.d_small, s);
+      } else if (db->p2p) {  // planes stored into every rank's region, signal, wait + OR (xchg.cuh)
         launch_xput(pb[0].lflag, pb[0].err, n, db->xpeers, db->xl, (uint32_t)db->cfg.rank, db->epoch, db->d_xdone, s);
         launch_xcombine(db->xregion, db->xl, n, db->epoch, reorder, st_out, pb[0].err, S.d_small, s);
-      } else if (db->cfg.world == 1) {
+      } else {  // loopback partitions of one process
         k_combine<<<(n + 255) / 256, 256, 0, s>>>(db->d_ptrs, L, n, st_out, db->d_ptrs + 64, S.d_small, reorder);
         k_spread_err<<<1, 1, 0, s>>>(S.d_small, db->d_ptrs + 64, L);
-        note_launch(2);
-      } else {
-        k_pack<<<(n + 255) / 256, 256, 0, s>>>(pb[0].lflag, pb[0].err, db->d_xchg, n);
-        ncclResult_t r = g_nccl.allReduce(db->d_xchg, db->d_xchg, 4ull * n + 3, ncclUint8, ncclMax, db->comm, s);
-        if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
-        k_unpack<<<(n + 255) / 256, 256, 0, s>>>(db->d_xchg, n, st_out, pb[0].err, S.d_small, reorder);
         note_launch(2);
       }
     }  // unpartitioned: the partition's error word reaches S.d_small with k_or_err after write-back
@@ -979,18 +973,15 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (ops_mode && L > 1)  // the combined verdict error, after every partition's write-back
       launch_advance_cursor(db->n_tables, db->d_reserve, S.d_small, db->d_dense_live, pb[0].insdel, s);
     // results: summed over partitions (each slot is written by its owning partition only)
-    if (db->p2p) {  // every rank publishes and reduces its slice (the protocol needs it)
+    if (sharded) {
+      // result slots final in place (home rank); nothing to sum
+    } else if (db->p2p) {  // every rank publishes and reduces its slice (the protocol needs it)
       launch_xsig_res(db->xpeers, (uint32_t)db->cfg.rank, (uint32_t)db->cfg.world, db->epoch, s);
       launch_xsum(db->xpeers, db->xl, n_reads, db->epoch, res->reads ? res_out : db->d_xsink, S.d_small,
                   (uint32_t)db->cfg.rank, db->d_xdone + 1, s);
-    } else if (partitioned && res->reads) {
-      if (db->cfg.world == 1) {
-        k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);
-        note_launch();
-      } else {
-        ncclResult_t r = g_nccl.allReduce(pb[0].res, res_out, n_reads, ncclInt64, ncclSum, db->comm, s);
-        if (r != ncclSuccess) return fail(db, LTPG_ENCCL, std::string("ncclAllReduce: ") + g_nccl.getErrorString(r));
-      }
+    } else if (partitioned && res->reads) {  // loopback partitions: sum of the partitions' slots
+      k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);
+      note_launch();
     }
     for (uint32_t p = 0; p < L; ++p) {  // errors raised during write-back reach the caller too
       k_or_err<<<1, 1, 0, s>>>(pb[p].err, S.d_small);
@@ -1081,6 +1072,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   }
   CK(cudaEventRecord(S.out_done, os));
   if (timing) res->stats->n_kernels = (uint32_t)(g_kernel_launches - S.launches0);
+  S.eff_tid = bd.tid;
+  S.eff_ptype = bd.ptype;
+  S.eff_params = bd.params;
+  S.eff_abort = abort_out;
+  S.seq = db->submitted;
+  S.carry_src = !ops_mode && db->cfg.world == 1 && db->loopback == 1;
   S.pending = true;
   if (async) return LTPG_OK;
   return finish_slot(db, S);
@@ -1088,7 +1085,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
 
 int ltpg_peer_handle(ltpg_db* db, void* out) {
   if (!db || !out) return LTPG_EINVAL;
-  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1 or LTPG_FLAG_NCCL_EXCHANGE)");
+  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1)");
   CK(cudaSetDevice(db->device));
   PeerHandle h{};
   CK(cudaIpcGetMemHandle(&h.h, db->xregion));
@@ -1105,7 +1102,7 @@ int ltpg_peer_handle(ltpg_db* db, void* out) {
 
 int ltpg_connect_peers(ltpg_db* db, const void* handles) {
   if (!db || !handles) return LTPG_EINVAL;
-  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1 or LTPG_FLAG_NCCL_EXCHANGE)");
+  if (!db->p2p) return fail(db, LTPG_EINVAL, "no peer-memory exchange (world == 1)");
   if (db->connected) return fail(db, LTPG_EINVAL, "peers already connected");
   CK(cudaSetDevice(db->device));
   const uint32_t world = (uint32_t)db->cfg.world;

@@ -394,6 +394,33 @@ void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const ui
   note_launch();
 }
 
+// LTPG_BATCH_CARRY_ABORTS: the previous batch's conflict aborts (abort[0..nc), ascending ranks) ->
+// the first nc txns of this batch, with their original TIDs, types and 128-byte blocks.  One
+// warp per carried txn: lanes move the block as 32 coalesced 4-byte words.
+__global__ void __launch_bounds__(256) k_carry(const unsigned long long* __restrict__ ptid,
+                                               const uint8_t* __restrict__ ptype, const uint8_t* __restrict__ pparams,
+                                               const uint32_t* __restrict__ abort, uint32_t nc,
+                                               unsigned long long* __restrict__ tid, uint8_t* __restrict__ type,
+                                               uint8_t* __restrict__ params) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < nc; w += nwarps) {
+    const uint32_t r = abort[w];
+    reinterpret_cast<uint32_t*>(params + 128ull * w)[lane] = reinterpret_cast<const uint32_t*>(pparams + 128ull * r)[lane];
+    if (lane == 0) {
+      tid[w] = ptid[r];
+      type[w] = ptype[r];
+    }
+  }
+}
+
+void launch_carry(const unsigned long long* ptid, const uint8_t* ptype, const uint8_t* pparams, const uint32_t* abort,
+                  uint32_t nc, unsigned long long* tid, uint8_t* type, uint8_t* params, cudaStream_t s) {
+  if (!nc) return;
+  k_carry<<<std::min<uint32_t>((nc + 7) / 8, 148 * 16), 256, 0, s>>>(ptid, ptype, pparams, abort, nc, tid, type, params);
+  note_launch();
+}
+
 // abort list: ranks of conflict-aborted txns in ascending order (stable compaction)
 // abort list (ascending ranks) and its length (n_out[0], and n_out2[0] when not null)
 __global__ void k_compact(const uint32_t* __restrict__ flags, const uint32_t* __restrict__ offs, uint32_t n,

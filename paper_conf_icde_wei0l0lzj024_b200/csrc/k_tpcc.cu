@@ -294,6 +294,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const uint32_t sw = v[k].y & 0xFFFFu, q = (v[k].y >> 16) & 0xFFu;
       if (active && l < n && (v[k].x < 1 || v[k].x > 100001 || q < 1 || q > 10 || sw < 1 || sw > b.nw)) bad = true;
     }
+#ifdef LTPG_DISTINCT_ALL16
 #pragma unroll
     for (uint32_t j = 0; j < 4; ++j)
 #pragma unroll
@@ -303,6 +304,22 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         for (uint32_t k = 0; k < 4; ++k)
           if (o == it[k] && 4 * j + m != 4 * sub + k) bad = true;
       }
+#else
+#pragma unroll
+    for (uint32_t k = 1; k < 4; ++k)  // pairs inside the lane
+#pragma unroll
+      for (uint32_t m = 0; m < k; ++m)
+        if (it[k] == it[m]) bad = true;
+#pragma unroll
+    for (uint32_t j = 1; j <= 2; ++j)  // pairs across lanes: partners sub+1 and sub+2 (mod 4) cover all
+#pragma unroll
+      for (uint32_t m = 0; m < 4; ++m) {
+        const uint32_t o = __shfl_sync(0xffffffffu, it[m], (sub + j) & 3u, 4);
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k)
+          if (o == it[k]) bad = true;
+      }
+#endif
     if (bad) atomicOr(b.err, ERR_EINVAL);
     const bool warp_bad = __any_sync(0xffffffffu, bad);  // the batch is rejected: skip the work
     if (active && !warp_bad) {
@@ -1042,7 +1059,7 @@ __global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
     long long q[MAXU];
 #pragma unroll
     for (uint32_t u = 0; u < MAXU; ++u) q[u] = rows[u] != ROW_NONE ? rd(TSt, S_QUANTITY, rows[u]) : 0;
-    const mark_t rtag = epoch_tag(b_epoch(b)) | sl.minr[dk];
+    const mark_t rtag = epoch_tag(b_epoch(b)) | grank_of(b, sl.minr[dk]);
     const uint32_t gq = col_group(TSt, S_QUANTITY);
 #pragma unroll
     for (uint32_t u = 0; u < MAXU; ++u) {
@@ -1128,7 +1145,7 @@ __global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScr
     res[2] = 0;
     res[3] = 0;
     // NEXT-1: read-only procedures never abort under reordering
-    const uint32_t flag = (!reorder && sl.m[idx] < r ? CF_RAW : 0u) | (b.ua[r] ? CF_UA : 0u);
+    const uint32_t flag = (!reorder && sl.m[idx] < grank_of(b, r) ? CF_RAW : 0u) | (b.ua[r] ? CF_UA : 0u);
     if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;
     else b.status[r] = status_of_bits(flag, reorder);
   }
@@ -1209,8 +1226,8 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     const uint32_t t = (ORD >> (4 * j)) & 15u;
     const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
     cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : tp.counts[t]));
-    const uint32_t per = 32 / lanes_of(t, PH, b.nparts, reorder);
-    pre[j + 1] = pre[j] + (cnt[j] + per - 1) / per;
+    const uint32_t lp = 5 - (__ffs(lanes_of(t, PH, b.nparts, reorder)) - 1);  // log2(txns per warp slot)
+    pre[j + 1] = pre[j] + ((cnt[j] + (1u << lp) - 1) >> lp);
   }
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
   for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NSLOT]; w += nwarps) {
@@ -1219,10 +1236,10 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     for (int jj = 1; jj < NSLOT; ++jj)
       if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }  // warp-uniform slot type
     const uint32_t t = (ORD >> (4 * j)) & 15u;
-    const uint32_t L = lanes_of(t, PH, b.nparts, reorder);
-    const uint32_t per = 32 / L;
-    const uint32_t k = lw * per + lane / L;
-    const uint32_t sub = lane % L;
+    const uint32_t L = lanes_of(t, PH, b.nparts, reorder);  // a power of two
+    const uint32_t ll = __ffs(L) - 1;
+    const uint32_t k = (lw << (5 - ll)) + (lane >> ll);
+    const uint32_t sub = lane & (L - 1);
     bool active = k < ct;
     uint32_t r = 0;
     if (t == SL_DLW) {  // warehouse k + 1's Delivery leader (write-back: only if it committed)
@@ -1232,7 +1249,8 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     } else if (active) {
       r = tp.list[(uint64_t)t * tp.max_txns + k];
     }
-    Tx x{dmask, r, b_epoch(b), epoch_tag(b_epoch(b)) | r, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder,
+    const uint32_t gr = active ? grank_of(b, r) : 0u;  // conflict TID (global rank of a sharded batch)
+    Tx x{dmask, gr, b_epoch(b), epoch_tag(b_epoch(b)) | gr, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder,
          hm, tp.nw};
     bool go = active;  // write-back runs over the committed re-list (k_tpcc_relist) only
     bool status_here = true;  // detection: this slot decides txn r's verdict
@@ -1263,13 +1281,18 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     __syncthreads();
     const DevTable& TWh = c_tabs[TW];
     const DevTable& TDi = c_tabs[TD];
-    for (uint32_t i = threadIdx.x; i < tp.hot_words; i += blockDim.x) {
+    for (uint32_t i = threadIdx.x; i < tp.nw; i += blockDim.x) {  // WAREHOUSE group 0
       const mark_t v = hm[i];
-      if (v == 0xFFFFFFFFu) continue;
-      const bool isw = i < tp.nw;
-      const DevTable& T = isw ? TWh : TDi;
-      const uint32_t g = isw ? 0u : (i - tp.nw) / (10 * tp.nw), row = isw ? i : (i - tp.nw) % (10 * tp.nw);
-      atomicMin((T.add_groups >> g) & 1u ? amark_ptr(T, g, row) : wmark_ptr(T, g, row), v);
+      if (v != 0xFFFFFFFFu) atomicMin((TWh.add_groups & 1u) ? amark_ptr(TWh, 0, i) : wmark_ptr(TWh, 0, i), v);
+    }
+#pragma unroll
+    for (uint32_t g = 0; g < 3; ++g) {  // DISTRICT groups 0..2
+      const mark_t* hg = hm + tp.nw + g * 10 * tp.nw;
+      const bool add = (TDi.add_groups >> g) & 1u;
+      for (uint32_t row = threadIdx.x; row < 10 * tp.nw; row += blockDim.x) {
+        const mark_t v = hg[row];
+        if (v != 0xFFFFFFFFu) atomicMin(add ? amark_ptr(TDi, g, row) : wmark_ptr(TDi, g, row), v);
+      }
     }
   }
   if (aggw) {
@@ -1330,6 +1353,7 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   bool bad = false;
   if (r < b.n_txns) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;
+    if (b.grank && (b.grank[r] >= b.n_global || (r > 0 && b.grank[r] <= b.grank[r - 1]))) bad = true;
     t = b.ptype[r];
     const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
     const uint32_t W = tp.nw;
@@ -1383,14 +1407,20 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
     const bool home = owns_w(b, p16(p, 0));
     touch = home;
+    // partitions the txn touches (bit q; the sharded exchange needs them, world <= 32)
+    const auto pbit = [&](uint32_t w) { const uint32_t q = part_of_w(w, b.nw, b.nparts); return q < 32 ? 1u << q : 0u; };
+    uint32_t pm = pbit(p16(p, 0));
     if (FULL && t == 0) {
-      for (uint32_t l = 0; l < lines && !touch; ++l) touch = owns_w(b, p16(p + 8 + 8 * l, 4));
+      for (uint32_t l = 0; l < lines; ++l) pm |= pbit(p16(p + 8 + 8 * l, 4));
+      touch = (pm >> b.part) & 1u;
       no_home = home;
       if (!home) lines = 0;
     } else if (t == 1) {
+      pm |= pbit(p16(p, 4));
       pay_cust = owns_w(b, p16(p, 4));
       touch = touch || pay_cust;
     }
+    if (FULL && b.pmask) b.pmask[r] = pm;
   } else {
     lines = 0;
   }
@@ -1817,6 +1847,21 @@ static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
   return (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
 }
+// execute with shared-memory hot marks: one wave of resident blocks (the grid-stride warp loop
+// covers every slot), so each block's mark-array init and flush is paid 148 x (blocks / SM)
+// times per batch instead of once per 8 warp slots
+static uint32_t exec_grid(uint32_t n, uint32_t hot_words) {
+  static int per_sm[2] = {0, 0};  // by hot_words != 0 (the dynamic shared memory differs)
+  const int h = hot_words ? 1 : 0;
+  if (!hot_words) return phase_grid(n);
+  if (!per_sm[h] && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[h], k_tpcc_phase<PH_EXEC, TM_MAIN>, 256,
+                                                                  hot_words * sizeof(mark_t)) != cudaSuccess)
+    per_sm[h] = 4;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return std::min<uint32_t>(phase_grid(n), (uint32_t)(std::max(per_sm[h], 1) * sms));
+}
 
 // cleared: misc and dl_min were reset by the batch's first kernel (k_batch_init, partition 0)
 int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cleared) {
@@ -1845,7 +1890,7 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   k_sl_claim<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   k_sl_district<<<148 * 2, 256, 0, t.side>>>(b, sl);
   cudaEventRecord(t.join[0], t.side);
-  k_tpcc_phase<PH_EXEC, TM_MAIN><<<grid, 256, tp.hot_words * sizeof(mark_t), s>>>(b, tp);
+  k_tpcc_phase<PH_EXEC, TM_MAIN><<<exec_grid(n, tp.hot_words), 256, tp.hot_words * sizeof(mark_t), s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
   note_launch(3);
   if (t.h_tab) launch_bucket_reduce(t.h_tab, t.n_tab, t.d_su, s);  // NEXT-3 large-sized buckets (if any)

@@ -362,7 +362,16 @@ struct BatchDev {
   uint32_t* err;             // device error word
   uint32_t* ins_tables;      // bitmask of tables receiving inserts
   uint32_t max_ops;
+  // sharded TPC-C batches (include/ltpg.h): this rank's shard of a global batch.  Per-txn arrays
+  // are indexed by the shard index i; the conflict TID (marks, checks) is the global rank
+  // grank[i].  pmask[i]: the partitions txn i touches (k_tpcc_group, partitioned batches).
+  const uint32_t* grank;           // null: the batch is the global batch (rank = index)
+  uint32_t n_global;
+  uint32_t* pmask;
 };
+
+// conflict TID of the batch's txn i (its global rank in a sharded batch)
+__device__ __forceinline__ uint32_t grank_of(const BatchDev& b, uint32_t i) { return b.grank ? __ldg(b.grank + i) : i; }
 
 __device__ __forceinline__ uint32_t b_epoch(const BatchDev& b) { return __ldg(&b.vars->epoch); }
 __device__ __forceinline__ long long b_clock(const BatchDev& b) { return __ldg(&b.vars->clock); }
@@ -474,6 +483,8 @@ void launch_finalize(const uint8_t* status, uint32_t n, uint32_t* commit_bits, u
 void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uint32_t* out, uint32_t* n_out,
                     uint32_t* n_out2, cudaStream_t s);
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
+void launch_carry(const unsigned long long* ptid, const uint8_t* ptype, const uint8_t* pparams, const uint32_t* abort,
+                  uint32_t nc, unsigned long long* tid, uint8_t* type, uint8_t* params, cudaStream_t s);
 void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const uint8_t* types, uint32_t n,
                            uint8_t* params, uint32_t* err, cudaStream_t s);
 // a8 in one kernel: commit bitmask, counts, abort list (decoupled look-back over 1024-txn tiles;

@@ -91,3 +91,38 @@ extern "C" int ltpg_compose_retry(const ltpg_batch* prev, const uint32_t* abort_
   out->n_fresh = nf;
   return LTPG_OK;
 }
+
+// SURVEY §8(e) routing: the shard of `rank` (txns touching its warehouses, in order, with their
+// global ranks).  Host-side copies only; part_of_w is the device's ownership rule.
+extern "C" int ltpg_route_tpcc(const ltpg_batch* g, uint32_t nw, uint32_t world, uint32_t rank, ltpg_batch_buf* out,
+                               uint32_t* grank) {
+  if (!g || !out || !grank || g->mode != LTPG_MODE_TPCC || g->inputs_on_device || g->proc_offsets || !world ||
+      rank >= world || !nw || (g->n_txns && (!g->tid || !g->proc_type || !g->proc_params)) || !out->tid ||
+      (out->cap_txns && (!out->proc_type || !out->proc_params)))
+    return LTPG_EINVAL;
+  auto part = [&](uint32_t w) { return ltpg::part_of_w(w, nw, world); };
+  uint32_t n = 0;
+  for (uint32_t r = 0; r < g->n_txns; ++r) {
+    const uint8_t* p = g->proc_params + (size_t)r * LTPG_PARAM_BYTES;
+    const uint32_t w = p[0] | (uint32_t)p[1] << 8;
+    bool mine = part(w) == rank;
+    if (!mine && g->proc_type[r] == LTPG_NEW_ORDER)
+      for (uint32_t l = 0; l < p[3] && l < 15 && !mine; ++l) {
+        const uint8_t* L = p + 8 + 8 * l;
+        mine = part(L[4] | (uint32_t)L[5] << 8) == rank;
+      }
+    if (!mine && g->proc_type[r] == LTPG_PAYMENT) mine = part(p[4] | (uint32_t)p[5] << 8) == rank;
+    if (!mine) continue;
+    if (n >= out->cap_txns) return LTPG_EINVAL;
+    out->tid[n] = g->tid[r];
+    out->proc_type[n] = g->proc_type[r];
+    std::memcpy(out->proc_params + (size_t)n * LTPG_PARAM_BYTES, p, LTPG_PARAM_BYTES);
+    grank[n] = r;
+    ++n;
+  }
+  out->n_txns = n;
+  out->n_ops = 0;
+  out->n_retried = 0;
+  out->n_fresh = n;
+  return LTPG_OK;
+}

@@ -1,8 +1,10 @@
-// Peer-memory exchange kernels (protocol and layout: xchg.cuh).  These replace the
-// pack -> ncclAllReduce(MAX) -> unpack sequence of the NCCL baseline (LTPG_FLAG_NCCL_EXCHANGE):
-// a rank's verdicts cross NVLink as 4 bit planes per 32 txns (16 B) stored straight
-// into every peer's region, i.e. (world-1) * n/2 bytes per rank instead of a 4n-byte ring
-// allreduce, and the waiting side needs no host involvement.
+// Peer-memory exchange kernels (protocol and layout: xchg.cuh), fused with the conflict test
+// instead of a collective library's allreduce: global batches send a rank's verdicts as 4 bit
+// planes per 32 txns (16 B) stored straight into every peer's region, i.e. (world-1) * n/2
+// bytes per rank instead of a 4n-byte ring allreduce; sharded batches send one byte per
+// cross-rank txn and peer.  The waiting side needs no host involvement.
+#include <algorithm>
+
 #include "ltpg_internal.cuh"
 #include "xchg.cuh"
 
@@ -120,6 +122,93 @@ __global__ void __launch_bounds__(256) k_xcombine(char* own, XLayout L, uint32_t
   status[r] = status_of_bits(f, reorder);
 }
 
+// ---- sharded TPC-C batches -------------------------------------------------------------------
+__device__ __forceinline__ uint8_t* b8_ptr(char* region, const XLayout& L, uint32_t par, uint32_t src) {
+  return reinterpret_cast<uint8_t*>(region + L.off_b8) + ((uint64_t)par * L.world + src) * L.max_txns;
+}
+__device__ __forceinline__ longlong2* rb_ptr(char* region, const XLayout& L, uint32_t par) {
+  return reinterpret_cast<longlong2*>(region + L.off_rb) + (uint64_t)par * L.max_txns;
+}
+__device__ __forceinline__ uint32_t u16_at(const uint8_t* p, int off) {
+  return p[off] | (uint32_t)p[off + 1] << 8;
+}
+// a Payment whose customer lives on another rank: (home rank, customer rank)
+__device__ __forceinline__ bool remote_customer(const uint8_t* ptype, const uint8_t* params, uint32_t i, uint32_t nw,
+                                                uint32_t world, uint32_t& home, uint32_t& cust) {
+  if (ptype[i] != LTPG_PAYMENT) return false;
+  const uint8_t* p = params + 128ull * i;
+  home = part_of_w(u16_at(p, 0), nw, world);
+  cust = part_of_w(u16_at(p, 4), nw, world);
+  return home != cust;
+}
+
+__global__ void __launch_bounds__(256) k_xput_sharded(const uint8_t* __restrict__ lflag, const uint32_t* __restrict__ pmask,
+                                                      const uint32_t* __restrict__ grank, const uint8_t* ptype,
+                                                      const uint8_t* params, const long long* res, const uint32_t* err,
+                                                      uint32_t n, XPeers peers, XLayout L, uint32_t rank, uint32_t nw,
+                                                      uint32_t epoch, uint32_t* done) {
+  const uint32_t par = epoch & 1u;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t others = pmask[i] & ~(1u << rank);
+    if (!others) continue;  // a txn of this rank only: its verdict is local
+    const uint32_t g = grank[i];
+    const uint8_t f = lflag[i];
+    for (uint32_t m = others; m; m &= m - 1) b8_ptr(peers.base[__ffs(m) - 1], L, par, rank)[g] = f;
+    uint32_t home, cust;
+    if (remote_customer(ptype, params, i, nw, L.world, home, cust) && cust == rank)
+      rb_ptr(peers.base[home], L, par)[g] = make_longlong2(res[4ull * i], res[4ull * i + 1]);
+  }
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t prev = atomicAdd(done, 1u);
+    if (prev == gridDim.x - 1) {  // every block's stores are fenced: publish
+      __threadfence_system();
+      const uint64_t v = ((uint64_t)epoch << 3) | (*err & 7u);
+      for (uint32_t q = 0; q < L.world; ++q) st_release_sys(sig_ptr(peers.base[q], par, 0, rank), v);
+      *done = 0;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_xcombine_sharded(char* own, XLayout L, uint32_t n, uint32_t epoch,
+                                                          bool reorder, uint8_t* status, const uint8_t* lflag,
+                                                          const uint32_t* pmask, const uint32_t* grank,
+                                                          const uint8_t* ptype, const uint8_t* params, long long* res,
+                                                          uint32_t rank, uint32_t nw, uint32_t* err, uint32_t* err_all) {
+  const uint32_t par = epoch & 1u;
+  uint32_t e = 0;
+  const bool ok = wait_all(own, par, 0, L.world, epoch, 3, &e, err_all);
+  if (!ok) {
+    if (threadIdx.x == 0) {
+      atomicOr(err, ERR_EINTERNAL);
+      atomicOr(err_all, ERR_EINTERNAL);
+    }
+    return;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    *err = e;
+    *err_all = e;
+  }
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    uint32_t f = lflag[i];
+    const uint32_t others = pmask[i] & ~(1u << rank);
+    if (others) {
+      const uint32_t g = grank[i];
+      for (uint32_t m = others; m; m &= m - 1) f |= __ldcg(b8_ptr(own, L, par, __ffs(m) - 1) + g);
+      uint32_t home, cust;
+      if (remote_customer(ptype, params, i, nw, L.world, home, cust) && home == rank) {
+        const longlong2 v = __ldcg(rb_ptr(own, L, par) + g);
+        res[4ull * i] = v.x;
+        res[4ull * i + 1] = v.y;
+        res[4ull * i + 2] = 0;
+        res[4ull * i + 3] = 0;
+      }
+    }
+    status[i] = status_of_bits(f, reorder);
+  }
+}
+
 __global__ void k_xsig_res(XPeers peers, uint32_t rank, uint32_t world, uint32_t epoch) {
   __threadfence_system();
   const uint32_t par = epoch & 1u;
@@ -189,6 +278,28 @@ void launch_xcombine(char* own, const XLayout& L, uint32_t n, uint32_t epoch, bo
                      uint32_t* err, uint32_t* err_all, cudaStream_t s) {
   const uint32_t blocks = (n + 255) / 256 ? (n + 255) / 256 : 1;
   k_xcombine<<<blocks, 256, 0, s>>>(own, L, n, epoch, reorder, status, err, err_all);
+  note_launch();
+}
+
+void launch_xput_sharded(const uint8_t* lflag, const uint32_t* pmask, const uint32_t* grank, const uint8_t* ptype,
+                         const uint8_t* params, const long long* res, const uint32_t* err, uint32_t n,
+                         const XPeers& peers, const XLayout& L, uint32_t rank, uint32_t nw, uint32_t epoch,
+                         uint32_t* done, cudaStream_t s) {
+  // grid-stride over the shard; the last block to finish raises the signals
+  const uint32_t blocks = std::max<uint32_t>(1, std::min<uint32_t>((n + 255) / 256, 148 * 4));
+  k_xput_sharded<<<blocks, 256, 0, s>>>(lflag, pmask, grank, ptype, params, res, err, n, peers, L, rank, nw, epoch,
+                                        done);
+  note_launch();
+}
+
+void launch_xcombine_sharded(char* own, const XLayout& L, uint32_t n, uint32_t epoch, bool reorder, uint8_t* status,
+                             const uint8_t* lflag, const uint32_t* pmask, const uint32_t* grank, const uint8_t* ptype,
+                             const uint8_t* params, long long* res, uint32_t rank, uint32_t nw, uint32_t* err,
+                             uint32_t* err_all, cudaStream_t s) {
+  // every block waits for the signals itself, so the grid is kept to one wave
+  const uint32_t blocks = std::max<uint32_t>(1, std::min<uint32_t>((n + 255) / 256, 148 * 4));
+  k_xcombine_sharded<<<blocks, 256, 0, s>>>(own, L, n, epoch, reorder, status, lflag, pmask, grank, ptype, params, res,
+                                            rank, nw, err, err_all);
   note_launch();
 }
 

@@ -2,20 +2,11 @@
 
 torch.distributed (any backend: nccl on the GPU box, gloo in CPU tests) only carries the
 bootstrap -- the ranks' 128-byte exchange handles (CUDA IPC handles of their exchange
-regions), or the NCCL unique id of the LTPG_FLAG_NCCL_EXCHANGE baseline -- and bench-side
-timing reductions.  The per-batch exchange itself is the library's own peer-memory kernels
-(csrc/xchg.cu) or ncclAllReduce (csrc/capi.cu).
+regions) -- and bench-side timing reductions.  The per-batch exchange itself is the library's
+own peer-memory kernels (csrc/xchg.cu).  Host routing of sharded TPC-C batches:
+paper_conf_icde_wei0l0lzj024_b200.route_tpcc (ltpg_route_tpcc).
 """
 import numpy as np
-
-
-def nccl_unique_id(group=None):
-    """Rank 0 creates an ncclUniqueId; every rank of `group` receives the same 128 bytes."""
-    import torch
-    import torch.distributed as dist
-    obj = [torch.cuda.nccl.unique_id() if dist.get_rank(group) == 0 else None]
-    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
-    return obj[0]
 
 
 def gather_handles(handle, group=None):

@@ -1,5 +1,5 @@
-"""Multi-rank host plumbing on CPU (world_size 2, gloo, 127.0.0.1): NCCL unique-id
-broadcast, per-rank partition loading (disjoint + complete, ITEM replicated), and
+"""Multi-rank host plumbing on CPU (world_size 2, gloo, 127.0.0.1): per-rank routing of a
+global TPC-C batch into shards (ltpg_route_tpcc), per-rank partition loading (disjoint + complete, ITEM replicated), and
 the verdict exchange semantics (max of conflict*2 | user_abort)."""
 import multiprocessing as mp
 import os
@@ -28,8 +28,12 @@ def _worker(rank, world, port, q):
     try:
         from paper_conf_icde_wei0l0lzj024_b200 import dist as D
         from workloads import tpcc
-        uid = D.nccl_unique_id()
+        import paper_conf_icde_wei0l0lzj024_b200 as L
         wl = tpcc.TpccWorkload(4, seed=1)
+        shard = L.route_tpcc(wl.batch(2000, 1, 0), 4, world, rank)
+        parts = [None] * world
+        dist.all_gather_object(parts, shard["grank"].tolist())
+        uid = parts
         tables = wl.initial_tables()
         mine = D.tpcc_rank_tables(tables, 4, rank, world)
         keysets = {t: (None if k is None else k.tolist(), c.shape[1]) for t, (k, c) in mine.items()}
@@ -56,7 +60,9 @@ def test_two_rank_gloo_plumbing():
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    assert res[0][1] == res[1][1] and len(res[0][1]) == 128            # same NCCL unique id
+    assert res[0][1] == res[1][1]                                      # every rank saw every shard
+    covered = sorted(set(res[0][1][0]) | set(res[0][1][1]))
+    assert covered == list(range(2000)) and len(res[0][1][0]) < 2000     # shards cover the batch
     assert res[0][5] == [(1, 3), (3, 5)]                               # warehouses 1-2 | 3-4
     from workloads import tpcc
     from workloads.formats import T_ITEM, T_HISTORY

@@ -1,6 +1,6 @@
 """Multi-partition path on one GPU: LTPG_FLAG_LOOPBACK runs P logical
 partitions (contiguous key / warehouse ranges) with the same ownership gating,
-per-txn verdict exchange (max of conflict*2|user_abort) and result sums as the NCCL
+per-txn verdict exchange (OR of the conflict bits) and result sums as the multi-rank
 path; every output must equal the 1-partition run, i.e. the oracle (PIN-8)."""
 import numpy as np
 import pytest
