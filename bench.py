@@ -693,6 +693,58 @@ def main():
                   "note": "next batch = aborts (original TIDs) + fresh txns (ltpg_compose_retry); device time "
                           "per batch, composition and upload outside the timed region"}
 
+    # ---- closed loop END TO END (batches back to back, aborts re-run in the next batch):
+    # every step = the previous step's conflict aborts, carried on the device
+    # (LTPG_BATCH_CARRY_ABORTS, a9 without a host round trip) + as many fresh txns as fit, taken
+    # from a pool of pinned compact client records.  Timed per step (CUDA events on the stream +
+    # wall clock): the host's submission (slice of the pool, its offsets rebased into a pinned
+    # buffer), H2D of the fresh records, every kernel, D2H of status / bitmask / abort list / all
+    # result slots.  TPC-C, single GPU. ----
+    closed_e2e = None
+    if world == 1 and w["kind"] == "tpcc" and not args.no_closed_loop and not args.no_e2e:
+        pool = {k: np.concatenate([hb[k] for hb in host_batches]) for k in ("tid", "type", "params")}
+        ppk, poffs = ltpg.pack_params_compact(pool["type"], pool["params"])
+        pin = {"tid": to_t(pool["tid"], True), "type": to_t(pool["type"], True), "params": to_t(ppk, True)}
+        offs_pin = torch.empty(B + 1, dtype=torch.int32).pin_memory()
+        offs_np = offs_pin.numpy().view(np.uint32)
+        out_c = pin_outs[0]
+        torch.cuda.synchronize()
+        cursor, c_commit, c_carried, c_steps, h2d_c, d2h_c = 0, 0, 0, 0, 0, 0
+        ce0, ce1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tw0 = time.time()
+        ce0.record(stream)
+        for s_ in range(args.steps):
+            nc = db.pending_aborts() if s_ else 0
+            m = min(B - nc, len(pool["tid"]) - cursor)
+            if m <= 0:
+                break
+            np.subtract(poffs[cursor:cursor + m + 1], poffs[cursor], out=offs_np[:m + 1])
+            p0, p1 = int(poffs[cursor]), int(poffs[cursor + m])
+            inp = {"tid": pin["tid"][8 * cursor:8 * (cursor + m)], "type": pin["type"][cursor:cursor + m],
+                   "params": pin["params"][p0:p1], "offsets": offs_pin[:m + 1], "compact": True}
+            outc = db.run_tpcc(inp, clock, stream=stream.cuda_stream, want_reads=True, device_out=False,
+                               n_txns=m, out=out_c, carry=s_ > 0)
+            clock += 1
+            n_s = nc + m
+            c_commit += int(np.bitwise_count(outc["commit_bits"][:(n_s + 31) // 32].numpy().view(np.uint32)).sum())
+            c_carried += nc
+            c_steps += 1
+            h2d_c += 8 * m + m + (p1 - p0) + 4 * (m + 1)
+            d2h_c += n_s + 4 * ((n_s + 31) // 32) + 4 * int(outc["n_aborted"][0]) + 32 * n_s + 68
+            cursor += m
+        ce1.record(stream)
+        torch.cuda.synchronize()
+        wall = time.time() - tw0
+        clk.mark(tw0, time.time())
+        c_s = ce0.elapsed_time(ce1) / 1000.0
+        closed_e2e = {"value": c_commit / c_s, "unit": UNIT, "steps": c_steps, "ms_per_step": 1000 * c_s / c_steps,
+                      "wall_ms_per_step": 1000 * wall / c_steps, "commit_rate": c_commit / (c_steps * B),
+                      "carried_per_step": c_carried / max(c_steps - 1, 1),
+                      "h2d_bytes_per_step": h2d_c // c_steps, "d2h_bytes_per_step": d2h_c // c_steps,
+                      "note": "closed loop end to end: previous step's aborts carried on the device "
+                              "(LTPG_BATCH_CARRY_ABORTS) + fresh compact records from pinned host memory; "
+                              "H2D, kernels, D2H and host submission inside the timed region"}
+
     e2e = None
     if not args.no_e2e:
         e_commits = []
@@ -799,7 +851,7 @@ def main():
                 if sharded else
                 ("%d ranks by key range, same global batch on every rank, per-txn verdict planes over peer "
                  "memory (csrc/xchg.cu)" % world) if world > 1 else "single GPU")),
-            "clocks": clk.summary(), "e2e": e2e, "closed_loop": closed, "gpu_launches": kernels, "roofline": roof,
+            "clocks": clk.summary(), "e2e": e2e, "closed_loop": closed, "closed_loop_e2e": closed_e2e, "gpu_launches": kernels, "roofline": roof,
             "commit_rate": all_commits / all_procs, "processed_txns_per_s": all_procs / total_s,
             "stage_ms_mean": {k: statistics.mean(s_[k] for s_ in stage)
                               for k in ("ms_upload", "ms_group", "ms_exec", "ms_detect", "ms_writeback",

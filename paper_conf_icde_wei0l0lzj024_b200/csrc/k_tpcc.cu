@@ -294,7 +294,9 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const uint32_t sw = v[k].y & 0xFFFFu, q = (v[k].y >> 16) & 0xFFu;
       if (active && l < n && (v[k].x < 1 || v[k].x > 100001 || q < 1 || q > 10 || sw < 1 || sw > b.nw)) bad = true;
     }
-#ifdef LTPG_DISTINCT_ALL16
+#ifndef LTPG_DISTINCT_PAIRS  // each lane compares its 4 items with all 16 of the txn (measured
+                             // faster than the fewer-compare pair scheme below: 0.185 vs 0.190 ms
+                             // execute on tpcc_c4, profiles/ab_r02_distinct.txt -- register use)
 #pragma unroll
     for (uint32_t j = 0; j < 4; ++j)
 #pragma unroll
@@ -335,6 +337,21 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       long long price[4];
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) price[k] = ri[k] != ROW_NONE ? rd(TIt, I_PRICE, ri[k]) : 0;
+#ifndef LTPG_NO_HDR_EARLY
+      // header lane: the static W / D / C reads go out with the item prices (one load wave);
+      // issued after the line stores below they would wait behind them (possible aliasing)
+      uint32_t row_w = ROW_NONE, row_d = ROW_NONE, row_c = ROW_NONE;
+      if (sub == 3) {
+        row_w = rowof(TWh, TW, w, x.dmask);
+        row_d = rowof(TDi, TD, kD(w, d), x.dmask);
+        row_c = rowof(TCu, TC, kC(w, d, c), x.dmask);
+        if (row_w != ROW_NONE && row_d != ROW_NONE && row_c != ROW_NONE) {
+          w_tax = rd(TWh, W_TAX, row_w);  // static reads: unmarked (R4)
+          d_tax = rd(TDi, D_TAX, row_d);
+          disc = rd(TCu, C_DISCOUNT, row_c);
+        }
+      }
+#endif
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
         const uint32_t l = 4 * sub + k;
@@ -358,15 +375,19 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       }
       (void)it;
       if (sub == 3) {  // header: warehouse / district / customer reads, fetch-ADD of D_NEXT_O_ID
+#ifdef LTPG_NO_HDR_EARLY
         const uint32_t row_w = rowof(TWh, TW, w, x.dmask), row_d = rowof(TDi, TD, kD(w, d), x.dmask),
                        row_c = rowof(TCu, TC, kC(w, d, c), x.dmask);
+#endif
         if (row_w == ROW_NONE || row_d == ROW_NONE || row_c == ROW_NONE) {
           internal_error(x);
           log[15] = ROW_NONE;
         } else {
+#ifdef LTPG_NO_HDR_EARLY
           w_tax = rd(TWh, W_TAX, row_w);  // static reads: unmarked (R4)
           d_tax = rd(TDi, D_TAX, row_d);
           disc = rd(TCu, C_DISCOUNT, row_c);
+#endif
           log[15] = row_d;
           unit_a<PH>(TDi, col_group(TDi, D_NEXT_O_ID), row_d, x, true);
         }
@@ -1847,20 +1868,21 @@ static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
   return (uint32_t)std::min<uint64_t>((warps + 7) / 8, 148 * 16);
 }
-// execute with shared-memory hot marks: one wave of resident blocks (the grid-stride warp loop
-// covers every slot), so each block's mark-array init and flush is paid 148 x (blocks / SM)
-// times per batch instead of once per 8 warp slots
-static uint32_t exec_grid(uint32_t n, uint32_t hot_words) {
-  static int per_sm[2] = {0, 0};  // by hot_words != 0 (the dynamic shared memory differs)
-  const int h = hot_words ? 1 : 0;
-  if (!hot_words) return phase_grid(n);
-  if (!per_sm[h] && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[h], k_tpcc_phase<PH_EXEC, TM_MAIN>, 256,
-                                                                  hot_words * sizeof(mark_t)) != cudaSuccess)
-    per_sm[h] = 4;
+// One wave of resident blocks per phase (the grid-stride warp loop covers every slot): the
+// per-block fixed costs -- the error-word barrier, execute's shared-memory mark init and flush,
+// write-back's last-block counter -- are paid 148 x (blocks / SM) times per batch instead of
+// once per 8 warp slots (write-back visits only the committed txns: most of a full-size grid
+// had nothing to do but those fixed costs)
+template <int PH>
+static uint32_t resident_grid(uint32_t n, size_t smem) {
+  static int per_sm[3][2] = {{0, 0}, {0, 0}, {0, 0}};  // by phase, by dynamic shared memory or not
+  int& b = per_sm[PH][smem ? 1 : 0];
+  if (!b && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_tpcc_phase<PH, TM_MAIN>, 256, smem) != cudaSuccess)
+    b = 2;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  return std::min<uint32_t>(phase_grid(n), (uint32_t)(std::max(per_sm[h], 1) * sms));
+  return std::min<uint32_t>(phase_grid(n), (uint32_t)(std::max(b, 1) * sms));
 }
 
 // cleared: misc and dl_min were reset by the batch's first kernel (k_batch_init, partition 0)
@@ -1880,7 +1902,6 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   if (ev) record_stage(ev[2], s);
   // NEXT-3: popularity from this batch's per-procedure counts -> bucket sizes
   if (t.h_tab) launch_popularity(t.h_tab, t.n_tab, b.kcount, n, t.d_su, t.popular, s);
-  const uint32_t grid = phase_grid(n);
   // StockLevel (shared per district) on a side stream, concurrently with the other procedures
   const SlScratch sl = t.sl;
   cudaEventRecord(t.fork[0], s);
@@ -1890,7 +1911,8 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   k_sl_claim<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   k_sl_district<<<148 * 2, 256, 0, t.side>>>(b, sl);
   cudaEventRecord(t.join[0], t.side);
-  k_tpcc_phase<PH_EXEC, TM_MAIN><<<exec_grid(n, tp.hot_words), 256, tp.hot_words * sizeof(mark_t), s>>>(b, tp);
+  k_tpcc_phase<PH_EXEC, TM_MAIN><<<resident_grid<PH_EXEC>(n, tp.hot_words * sizeof(mark_t)), 256,
+                                   tp.hot_words * sizeof(mark_t), s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
   note_launch(3);
   if (t.h_tab) launch_bucket_reduce(t.h_tab, t.n_tab, t.d_su, s);  // NEXT-3 large-sized buckets (if any)
@@ -1900,7 +1922,7 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   k_sl_detect<<<148 * 2, 256, 0, t.side>>>(b, sl);
   k_sl_txn<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   cudaEventRecord(t.join[1], t.side);
-  k_tpcc_phase<PH_DETECT, TM_MAIN><<<grid, 256, 0, s>>>(b, tp);
+  k_tpcc_phase<PH_DETECT, TM_MAIN><<<resident_grid<PH_DETECT>(n, 0), 256, 0, s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[1], 0);
   note_launch(3);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
@@ -1928,7 +1950,7 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
     k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
   note_launch(3);
-  k_tpcc_phase<PH_WB, TM_MAIN><<<phase_grid(n), 256, wb_smem(t), s>>>(b, params_of(t, b, true));  // + row counters
+  k_tpcc_phase<PH_WB, TM_MAIN><<<resident_grid<PH_WB>(n, wb_smem(t)), 256, wb_smem(t), s>>>(b, params_of(t, b, true));  // + row counters
   note_launch(1);
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
