@@ -46,6 +46,8 @@ WORKLOADS = {
     "tpcc_c2_opt": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed", reorder=True),
     "tpcc_c2_delayed": dict(kind="tpcc", cfg=1, W=1, mix="no_pay", batch=16384, mode="delayed"),
     "ycsb_c3_4ops": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=4, batch=1 << 20),
+    # C3 with sparse u64 keys (splitmix64 of the row number): every op probes the PK hash index
+    "ycsb_c3_sparse": dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=0.99, ops=10, batch=1 << 20, sparse=True),
     # NEXT-4: the paper's YCSB suite: Zipf alpha 2.5, 10 ops, 10^7 rows
     **{"ycsb_%s" % L.lower(): dict(kind="ycsb", cfg=2, n_rows=10_000_000, theta=2.5, ops=10, batch=1 << 16,
                                    letter=L) for L in "ABCDE"},
@@ -185,7 +187,8 @@ def make_workload(name, rank=0):
         from workloads.ycsb import YcsbWorkload, ycsb_letter
         if w.get("letter"):
             return ycsb_letter(w["letter"], w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
-        return YcsbWorkload(w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed)
+        return YcsbWorkload(w["n_rows"], theta=w["theta"], ops_per_txn=w["ops"], seed=seed,
+                            sparse_keys=w.get("sparse", False))
     from workloads import tpcc
     mix = tpcc.MIX_FULL if w["mix"] == "full" else tpcc.MIX_NO_PAY
     return tpcc.TpccWorkload(w["W"], seed=seed, mode=w["mode"], mix=mix)
@@ -214,15 +217,16 @@ def open_database(name, wl, n_batches, flags=0, device=0, rank=0, world=1, **kw)
                               rank=rank, world=world, **kw)
 
 
-def exec_algorithmic_bytes(batch):
+def exec_algorithmic_bytes(batch, sparse=False):
     """Algorithmic bytes of the OPS execute kernel: per op 16 B op record +
     32 B data sector + 8 B result + 8 B unit reference = 64 B; + 64 B per marking op
     (UPDATE/ADD/INSERT/DELETE: atomic sector RMW).  Dense key ranges map key -> row by
-    arithmetic (identity bucket function), so no index bytes are counted."""
+    arithmetic (identity bucket function), so no index bytes are counted; sparse keys
+    add one 32-byte index-slot sector per op (linear probing at load factor <= 1/2)."""
     kinds = batch["ops"]["kind"]
     n = len(kinds)
     marking = int(np.isin(kinds, [1, 2, 3, 4]).sum())
-    return 64 * n + 64 * marking
+    return 64 * n + 64 * marking + (32 * n if sparse else 0)
 
 
 def tpcc_exec_algorithmic_bytes(batch, mode):
@@ -259,10 +263,10 @@ def tpcc_exec_algorithmic_bytes(batch, mode):
     return int(b.sum()) + n_dw * full_dl + n_sd * full_sl
 
 
-def fused_algorithmic_bytes(batch):
+def fused_algorithmic_bytes(batch, sparse=False):
     """Algorithmic bytes of the fused OPS kernel (validate + warp-local division + execute):
     the execute bytes above + 16 B per txn (TID 8 B, op_begin 4 B, txn_ins 4 B)."""
-    return exec_algorithmic_bytes(batch) + 16 * len(batch["tid"])
+    return exec_algorithmic_bytes(batch, sparse) + 16 * len(batch["tid"])
 
 
 # B200 random-access ceiling measured by tools/randbw.cu (profiles/randbw_r01.txt): independent
@@ -271,15 +275,16 @@ def fused_algorithmic_bytes(batch):
 RANDOM_READ_CEILING_G = 48.6
 
 
-def ops_random_reads(batch):
+def ops_random_reads(batch, sparse=False):
     """Independent random row-sized reads the OPS execute does per batch: one column read per
     SELECT / UPDATE (dense key -> row by arithmetic), one mark-filter read per UPDATE / ADD
-    (its atomicMin then hits the line in L2), one read per SCANned key; INSERT / DELETE 2."""
+    (its atomicMin then hits the line in L2), one read per SCANned key; INSERT / DELETE 2;
+    sparse keys: + one index-slot read per op."""
     ops = batch["ops"]
     kinds = ops["kind"]
     n = np.bincount(kinds, minlength=6)
     scan_keys = int(ops["aux"][kinds == 5].astype(np.int64).sum())
-    return int(n[0] + 2 * n[1] + n[2] + 2 * (n[3] + n[4]) + scan_keys)
+    return int(n[0] + 2 * n[1] + n[2] + 2 * (n[3] + n[4]) + scan_keys) + (len(kinds) if sparse else 0)
 
 
 def step_algorithmic_bytes(batch):
@@ -723,14 +728,16 @@ def main():
             inp = {"tid": pin["tid"][8 * cursor:8 * (cursor + m)], "type": pin["type"][cursor:cursor + m],
                    "params": pin["params"][p0:p1], "offsets": offs_pin[:m + 1], "compact": True}
             outc = db.run_tpcc(inp, clock, stream=stream.cuda_stream, want_reads=True, device_out=False,
-                               n_txns=m, out=out_c, carry=s_ > 0)
+                               n_txns=m, out=out_c, carry=s_ > 0, committed_reads=True, no_status=True,
+                               no_abort_list=True)
             clock += 1
             n_s = nc + m
-            c_commit += int(np.bitwise_count(outc["commit_bits"][:(n_s + 31) // 32].numpy().view(np.uint32)).sum())
+            nc_s = int(np.bitwise_count(np.asarray(outc["commit_bits"])[:(n_s + 31) // 32].view(np.uint32)).sum())
+            c_commit += nc_s
             c_carried += nc
             c_steps += 1
             h2d_c += 8 * m + m + (p1 - p0) + 4 * (m + 1)
-            d2h_c += n_s + 4 * ((n_s + 31) // 32) + 4 * int(outc["n_aborted"][0]) + 32 * n_s + 68
+            d2h_c += 4 * ((n_s + 31) // 32) + 32 * nc_s + 68  # bitmask, committed txns' slots, counters
             cursor += m
         ce1.record(stream)
         torch.cuda.synchronize()
@@ -743,6 +750,8 @@ def main():
                       "h2d_bytes_per_step": h2d_c // c_steps, "d2h_bytes_per_step": d2h_c // c_steps,
                       "note": "closed loop end to end: previous step's aborts carried on the device "
                               "(LTPG_BATCH_CARRY_ABORTS) + fresh compact records from pinned host memory; "
+                              "returns the commit bitmask and the committed txns' result slots "
+                              "(LTPG_RESULT_COMMITTED_READS, written into pinned host memory by the kernel); "
                               "H2D, kernels, D2H and host submission inside the timed region"}
 
     e2e = None
@@ -817,7 +826,7 @@ def main():
     if w["kind"] == "ycsb":
         model = fused_algorithmic_bytes if fused_front else exec_algorithmic_bytes
         kname = "k_ops_fused" if fused_front else "k_ops_exec"
-        bytes_exec = statistics.mean(model(host_batches[(args.warmup + s) % n_distinct])
+        bytes_exec = statistics.mean(model(host_batches[(args.warmup + s) % n_distinct], w.get("sparse", False))
                                      for s in range(args.steps))
         ms = statistics.mean(exec_ms)
         ach = bytes_exec / (ms / 1000.0) / 1e9
@@ -825,7 +834,7 @@ def main():
                 "frac": ach / peak, "traffic": ncu_traffic(name, kname), "peak_source": peak_kind,
                 "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
                 "kernel_share_of_step": ms / statistics.mean(step_ms)}
-        nrand = statistics.mean(ops_random_reads(host_batches[(args.warmup + s) % n_distinct])
+        nrand = statistics.mean(ops_random_reads(host_batches[(args.warmup + s) % n_distinct], w.get("sparse", False))
                                 for s in range(args.steps))
         roof["random_access"] = {
             "reads_per_launch": nrand, "ceiling_g_per_s": RANDOM_READ_CEILING_G,

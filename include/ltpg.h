@@ -290,13 +290,26 @@ typedef struct {
 
 typedef struct {
   uint32_t* commit_bits;        /* [ceil(n_txns/32)]: bit r%32 of word r/32 = committed   */
-  uint8_t* status;              /* [n_txns]: LTPG_ST_*                                    */
-  uint32_t* abort_idx;          /* [n_txns] capacity: ranks of conflict aborts, ascending */
+  uint8_t* status;              /* [n_txns]: LTPG_ST_*  (NULL with LTPG_RESULT_NO_STATUS) */
+  uint32_t* abort_idx;          /* [n_txns] capacity: ranks of conflict aborts, ascending
+                                   (NULL with LTPG_RESULT_NO_ABORT_LIST)                  */
   uint32_t* n_aborted;          /* [1]                                                    */
   int64_t* reads;               /* OPS: [n_ops]; TPCC: [4*n_txns]; NULL = not returned    */
   int outputs_on_device;        /* 1: the pointers above are device pointers             */
   ltpg_stats* stats;            /* optional host struct: per-stage device times           */
+  uint32_t flags;               /* LTPG_RESULT_*                                          */
 } ltpg_result;
+
+/* Result options.  COMMITTED_READS (TPC-C): `reads` receives the 4 result slots of the COMMITTED
+ * txns only, packed in rank order (the i-th committed txn -- the i-th set bit of commit_bits --
+ * at reads[4i..4i+3]); a host `reads` buffer must be pinned and device-mapped (cudaHostAlloc;
+ * the kernel writes it directly over PCIe, no copy of the other txns' slots), else EINVAL.
+ * NO_STATUS / NO_ABORT_LIST: those outputs are not produced (their pointers may be NULL);
+ * n_aborted and commit_bits always are.  Results of aborted txns are snapshot reads that are
+ * recomputed when the txn is retried, so a closed loop needs only the committed ones. */
+#define LTPG_RESULT_COMMITTED_READS 1u
+#define LTPG_RESULT_NO_STATUS 2u
+#define LTPG_RESULT_NO_ABORT_LIST 4u
 
 /* Run one batch; synchronous on batch->stream (returns when results are in place)
  * unless batch->flags has LTPG_BATCH_ASYNC.

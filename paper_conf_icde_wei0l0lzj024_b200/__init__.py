@@ -76,7 +76,8 @@ class ltpg_stats(ctypes.Structure):
 
 class ltpg_result(ctypes.Structure):
     _fields_ = [("commit_bits", c_vp), ("status", c_vp), ("abort_idx", c_vp), ("n_aborted", c_vp),
-                ("reads", c_vp), ("outputs_on_device", c_int), ("stats", ctypes.POINTER(ltpg_stats))]
+                ("reads", c_vp), ("outputs_on_device", c_int), ("stats", ctypes.POINTER(ltpg_stats)),
+                ("flags", c_u32)]
 
 
 _lib.ltpg_create_db.restype = c_int
@@ -133,6 +134,7 @@ ltpg_pending_aborts = _lib.ltpg_pending_aborts
 LTPG_BATCH_ASYNC = 1
 LTPG_BATCH_COMPACT_PARAMS = 2
 LTPG_BATCH_CARRY_ABORTS = 4
+LTPG_RESULT_COMMITTED_READS, LTPG_RESULT_NO_STATUS, LTPG_RESULT_NO_ABORT_LIST = 1, 2, 4
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
             "ltpg_destroy_db", "ltpg_last_error", "ltpg_version", "ltpg_peer_handle", "ltpg_connect_peers",
@@ -225,7 +227,7 @@ class Database:
         self.has_pk[t] = bool(has_pk)
 
     # -- batches -------------------------------------------------------------------------
-    def _outputs(self, n, n_reads, device_out):
+    def _outputs(self, n, n_reads, device_out, pinned=False):
         if device_out:
             import torch
             dev = torch.device("cuda", torch.cuda.current_device())
@@ -234,32 +236,48 @@ class Database:
                     "abort_idx": torch.empty(max(n, 1), dtype=torch.int32, device=dev),
                     "n_aborted": torch.zeros(1, dtype=torch.int32, device=dev),
                     "reads": torch.empty(max(n_reads, 1), dtype=torch.int64, device=dev)}
+        if pinned:  # page-locked host memory the device can write (LTPG_RESULT_COMMITTED_READS)
+            import torch
+            o = {"status": torch.empty(n, dtype=torch.uint8), "commit_bits": torch.empty((n + 31) // 32, dtype=torch.int32),
+                 "abort_idx": torch.empty(max(n, 1), dtype=torch.int32), "n_aborted": torch.zeros(1, dtype=torch.int32),
+                 "reads": torch.empty(max(n_reads, 1), dtype=torch.int64)}
+            return {k: v.pin_memory().numpy() for k, v in o.items()}
         return {"status": np.empty(n, np.uint8), "commit_bits": np.empty((n + 31) // 32, np.uint32),
                 "abort_idx": np.empty(max(n, 1), np.uint32), "n_aborted": np.zeros(1, np.uint32),
                 "reads": np.empty(max(n_reads, 1), np.int64)}
 
-    def _run(self, bt, n, n_reads, want_reads, device_out, stats, out, wait=True, keep=None):
+    def _run(self, bt, n, n_reads, want_reads, device_out, stats, out, wait=True, keep=None, rflags=0):
         if out is None:
-            out = self._outputs(n, n_reads, device_out)
+            out = self._outputs(n, n_reads, device_out, pinned=bool(rflags & LTPG_RESULT_COMMITTED_READS))
         st = ltpg_stats() if stats else None
-        res = ltpg_result(commit_bits=_ptr(out["commit_bits"]), status=_ptr(out["status"]),
-                          abort_idx=_ptr(out["abort_idx"]), n_aborted=_ptr(out["n_aborted"]),
+        res = ltpg_result(commit_bits=_ptr(out["commit_bits"]),
+                          status=None if rflags & LTPG_RESULT_NO_STATUS else _ptr(out["status"]),
+                          abort_idx=None if rflags & LTPG_RESULT_NO_ABORT_LIST else _ptr(out["abort_idx"]),
+                          n_aborted=_ptr(out["n_aborted"]),
                           reads=_ptr(out["reads"]) if want_reads else None,
                           outputs_on_device=int(device_out),
-                          stats=ctypes.pointer(st) if st is not None else None)
+                          stats=ctypes.pointer(st) if st is not None else None, flags=rflags)
         if not wait:
             bt.flags |= LTPG_BATCH_ASYNC
             self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))
-            return Pending(self, res, bt, st, out, n, n_reads, want_reads, device_out, keep)
+            return Pending(self, res, bt, st, out, n, n_reads, want_reads, device_out, keep, rflags)
         self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))
-        return self._collect(out, n, n_reads, want_reads, device_out, st)
+        return self._collect(out, n, n_reads, want_reads, device_out, st, rflags)
 
-    def _collect(self, out, n, n_reads, want_reads, device_out, st):
+    def _collect(self, out, n, n_reads, want_reads, device_out, st, rflags=0):
         out = dict(out)
         if not device_out:
             na = int(out["n_aborted"][0])
-            out["abort_idx"] = out["abort_idx"][:na]
-            out["reads"] = out["reads"][:n_reads] if want_reads else None
+            if not rflags & LTPG_RESULT_NO_ABORT_LIST:
+                out["abort_idx"] = out["abort_idx"][:na]
+            if rflags & LTPG_RESULT_NO_STATUS:
+                out["status"] = None
+            if want_reads and rflags & LTPG_RESULT_COMMITTED_READS:  # the committed txns' slots only
+                bits = np.asarray(out["commit_bits"])[:(n + 31) // 32].view(np.uint32)
+                nc = int(np.bitwise_count(bits).sum())
+                out["reads"] = out["reads"][:4 * nc]
+            else:
+                out["reads"] = out["reads"][:n_reads] if want_reads else None
         if st is not None:
             out["stats"] = st.as_dict()
         return out
@@ -286,13 +304,15 @@ class Database:
         return n.value
 
     def run_tpcc(self, batch, clock, stream=None, want_reads=True, device_out=None, stats=False, out=None,
-                 n_txns=None, wait=True, carry=False):
+                 n_txns=None, wait=True, carry=False, committed_reads=False, no_status=False, no_abort_list=False):
         """batch: dict(tid u64[n], type u8[n], params u8[n,128]) -- or packed blocks:
         params = used bytes back to back and offsets u32[n+1] (see pack_params), or compact
         records with compact=True (see pack_params_compact).  A rank's shard of a global batch
         (route_tpcc) also carries grank u32[n] and n_global.  carry=True: the batch is the previous
         batch's conflict aborts (kept on the device) followed by these txns
-        (LTPG_BATCH_CARRY_ABORTS); the outputs cover pending_aborts() + n txns."""
+        (LTPG_BATCH_CARRY_ABORTS); the outputs cover pending_aborts() + n txns.  committed_reads:
+        reads = the result slots of the committed txns only, in rank order (host outputs must
+        then be pinned memory); no_status / no_abort_list skip those outputs."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
         offsets = batch.get("offsets")
         grank = batch.get("grank")
@@ -307,9 +327,11 @@ class Database:
                         flags=(LTPG_BATCH_COMPACT_PARAMS if batch.get("compact") else 0) |
                         (LTPG_BATCH_CARRY_ABORTS if carry else 0),
                         grank=_ptr(grank), n_global=int(batch.get("n_global", 0)))
-        out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch)
+        rflags = ((LTPG_RESULT_COMMITTED_READS if committed_reads else 0) | (LTPG_RESULT_NO_STATUS if no_status else 0)
+                  | (LTPG_RESULT_NO_ABORT_LIST if no_abort_list else 0))
+        out = self._run(bt, n, 4 * n, want_reads, device_out, stats, out, wait, keep=batch, rflags=rflags)
         if wait and not device_out and want_reads:
-            out["reads"] = out["reads"].reshape(n, 4)
+            out["reads"] = out["reads"].reshape(-1, 4)
         return out
 
     def mark_memory(self, t):
@@ -408,14 +430,15 @@ def pack_params_compact(types, params):
 class Pending:
     """An asynchronously submitted batch (LTPG_BATCH_ASYNC): .wait() completes it."""
 
-    def __init__(self, db, res, bt, st, out, n, n_reads, want_reads, device_out, keep):
+    def __init__(self, db, res, bt, st, out, n, n_reads, want_reads, device_out, keep, rflags=0):
         self.db, self.res, self.bt, self.st, self.out = db, res, bt, st, out
         self.args = (n, n_reads, want_reads, device_out)
+        self.rflags = rflags
         self.keep = keep  # host buffers must stay alive until the batch completes
 
     def wait(self):
         self.db._check(ltpg_wait_batch(self.db.h, ctypes.byref(self.res)))
-        return self.db._collect(self.out, *self.args, self.st)
+        return self.db._collect(self.out, *self.args, self.st, self.rflags)
 
 
 def part_of_w(w, nw, nparts):

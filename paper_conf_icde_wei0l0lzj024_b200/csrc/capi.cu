@@ -125,6 +125,7 @@ struct ltpg_db {
   uint32_t idx_lag = 0;
   unsigned long long* d_idx_from = nullptr;  // [MAXT]
   uint16_t* d_su = nullptr;                  // [MAXT] NEXT-3: this batch's bucket size per table
+  uint32_t* d_wprefix = nullptr;             // LTPG_RESULT_COMMITTED_READS: commits before each bitmask word
   std::vector<Part> parts;
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_scan = nullptr;
@@ -304,6 +305,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_reserve, MAXT));
   CK(dmalloc(&db->d_idx_from, MAXT));
   CK(dmalloc(&db->d_su, MAXT));
+  CK(dmalloc(&db->d_wprefix, (n + 31) / 32 + 1));
   CK(cudaMemset(db->d_su, 0, MAXT * sizeof(uint16_t)));
   CK(dmalloc(&db->d_dense_live, 1));
   CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
@@ -392,7 +394,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
   void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_ptrs, db->d_scan,
-                  db->d_idx_from, db->d_su};
+                  db->d_idx_from, db->d_su, db->d_wprefix};
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
@@ -672,7 +674,9 @@ int ltpg_wait_batch(ltpg_db* db, ltpg_result* res) {
 int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (!db) return LTPG_EINVAL;
   if (db->poisoned) return LTPG_EPOISONED;
-  if (!b || !res || !b->tid || !res->status || !res->commit_bits || !res->abort_idx || !res->n_aborted)
+  if (!b || !res || !b->tid || !res->commit_bits || !res->n_aborted ||
+      (!res->status && !(res->flags & LTPG_RESULT_NO_STATUS)) ||
+      (!res->abort_idx && !(res->flags & LTPG_RESULT_NO_ABORT_LIST)))
     return fail(db, LTPG_EINVAL, "null argument");
   const uint32_t nf = b->n_txns;  // txns given (LTPG_BATCH_CARRY_ABORTS: after the carried ones)
   const bool ops_mode = b->mode == LTPG_MODE_OPS;
@@ -694,6 +698,23 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
   if (!ops_mode && b->proc_offsets && !b->inputs_on_device && b->proc_offsets[nf] > (uint64_t)nf * LTPG_PARAM_BYTES)
     return fail(db, LTPG_EINVAL, "packed params too large");
+  // LTPG_RESULT_COMMITTED_READS: the gather kernel writes the caller's buffer directly
+  const bool cr = (res->flags & LTPG_RESULT_COMMITTED_READS) != 0;
+  long long* cr_dst = nullptr;
+  if (cr) {
+    if (ops_mode || !res->reads) return fail(db, LTPG_EINVAL, "LTPG_RESULT_COMMITTED_READS: TPCC with a reads buffer");
+    if (res->outputs_on_device) {
+      cr_dst = reinterpret_cast<long long*>(res->reads);
+    } else {
+      cudaPointerAttributes pa{};
+      if (cudaPointerGetAttributes(&pa, res->reads) != cudaSuccess || pa.type != cudaMemoryTypeHost ||
+          !pa.devicePointer) {
+        cudaGetLastError();
+        return fail(db, LTPG_EINVAL, "LTPG_RESULT_COMMITTED_READS: the host reads buffer must be pinned and mapped");
+      }
+      cr_dst = static_cast<long long*>(pa.devicePointer);
+    }
+  }
   const bool sharded = b->grank != nullptr;
   if (sharded && (ops_mode || !db->p2p || b->n_global > db->cfg.max_txns || n > b->n_global))
     return fail(db, LTPG_EINVAL, "sharded batches: TPCC on a multi-rank peer-memory db, n_txns <= n_global <= max_txns");
@@ -727,9 +748,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   bd.max_ops = std::max<uint32_t>(db->cfg.max_ops, 1);
   bd.n_global = sharded ? b->n_global : n;
   // verdict outputs: written in place when the caller's buffers are on the device
-  uint8_t* st_out = S.host_out ? S.d_status : res->status;
+  uint8_t* st_out = (S.host_out || !res->status) ? S.d_status : res->status;
   uint32_t* bits_out = S.host_out ? S.d_bits : res->commit_bits;
-  uint32_t* abort_out = S.host_out ? S.d_abort : res->abort_idx;
+  uint32_t* abort_out = (S.host_out || !res->abort_idx) ? S.d_abort : res->abort_idx;
   bd.status = st_out;
   const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
   if (b->inputs_on_device) {
@@ -785,7 +806,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool packed_params = !ops_mode && b->proc_offsets;
   if (packed_params) bd.params = S.d_params;
   const size_t n_reads = ops_mode ? b->n_ops : (size_t)n * LTPG_PROC_RESULTS;
-  const bool reads_dev = res->reads && res->outputs_on_device;
+  const bool reads_dev = res->reads && res->outputs_on_device && !cr;
   long long* res_out = reads_dev ? reinterpret_cast<long long*>(res->reads) : S.d_res;
   uint32_t* counts = S.d_small + 8;
   // ---- work that depends on host-side state, stream-ordered ahead of the batch's device work ----
@@ -988,6 +1009,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       note_launch();
     }
     CK(cudaStreamWaitEvent(s, db->fin_done, 0));
+    if (cr) launch_committed_reads(bits_out, n, res_out, cr_dst, db->d_wprefix, s);  // bits and slots final
     CK(cudaGetLastError());
     return LTPG_OK;
   };
@@ -995,7 +1017,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // Graph replay: the same shape's captured graph if this slot has one, else capture, instantiate
   // and keep it (least recently used of GRAPHS_PER_SLOT replaced).  Multi-rank dbs enqueue
   // directly (their exchange selects buffers by epoch parity on the host).
-  const bool use_graph = n && db->cfg.world == 1 && (db->cfg.flags & LTPG_FLAG_GRAPH);
+  const bool use_graph = n && db->cfg.world == 1 && (db->cfg.flags & LTPG_FLAG_GRAPH) && !cr;
   if (use_graph) {
     GraphKey k;
     std::memset(&k, 0, sizeof(k));
@@ -1063,11 +1085,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17);
   note_launch();
   if (n && S.host_out) {
-    CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));
+    if (res->status) CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));
     CK(cudaMemcpyAsync(res->commit_bits, S.d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, os));
-    if (res->reads && !reads_dev) CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
-    CK(cudaMemcpyAsync(res->abort_idx, S.d_abort, n * sizeof(uint32_t), out_kind, os));
-  } else if (n && res->reads && !reads_dev) {
+    if (res->reads && !reads_dev && !cr)
+      CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
+    if (res->abort_idx) CK(cudaMemcpyAsync(res->abort_idx, S.d_abort, n * sizeof(uint32_t), out_kind, os));
+  } else if (n && res->reads && !reads_dev && !cr) {
     CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
   }
   CK(cudaEventRecord(S.out_done, os));

@@ -394,6 +394,63 @@ void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const ui
   note_launch();
 }
 
+// LTPG_RESULT_COMMITTED_READS: the 4 result slots of every committed txn, packed in rank order,
+// written straight into the caller's (host-mapped or device) buffer.  One block scans the
+// popcounts of the commit-bitmask words (exclusive prefix per word), then one thread per txn
+// stores its slots at 4 x (prefix of its word + committed lanes below it in the word).
+__global__ void __launch_bounds__(1024) k_commit_prefix(const uint32_t* __restrict__ bits, uint32_t nw,
+                                                        uint32_t* __restrict__ pre) {
+  __shared__ uint32_t wsum[32];
+  const uint32_t per = (nw + 1023) / 1024, w0 = threadIdx.x * per;
+  uint32_t t = 0;
+  for (uint32_t w = w0; w < w0 + per && w < nw; ++w) t += __popc(bits[w]);
+  const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint32_t x = t;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  if (lane == 31) wsum[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t v = wsum[lane], s = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= (uint32_t)o) s += y;
+    }
+    wsum[lane] = s - v;
+  }
+  __syncthreads();
+  uint32_t run = wsum[wid] + x - t;
+  for (uint32_t w = w0; w < w0 + per && w < nw; ++w) {
+    pre[w] = run;
+    run += __popc(bits[w]);
+  }
+}
+__global__ void __launch_bounds__(256) k_commit_gather(const uint32_t* __restrict__ bits, const uint32_t* __restrict__ pre,
+                                                       uint32_t n, const long long* __restrict__ res, long long* out) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n) return;
+  const uint32_t w = bits[r >> 5], b = r & 31;
+  if (!((w >> b) & 1u)) return;
+  const uint32_t i = pre[r >> 5] + __popc(w & ((1u << b) - 1u));
+  const longlong2 a = *reinterpret_cast<const longlong2*>(res + 4ull * r);
+  const longlong2 c = *reinterpret_cast<const longlong2*>(res + 4ull * r + 2);
+  reinterpret_cast<longlong2*>(out + 4ull * i)[0] = a;
+  reinterpret_cast<longlong2*>(out + 4ull * i)[1] = c;
+}
+
+void launch_committed_reads(const uint32_t* bits, uint32_t n, const long long* res, long long* out, uint32_t* pre,
+                            cudaStream_t s) {
+  if (!n) return;
+  const uint32_t nw = (n + 31) / 32;
+  k_commit_prefix<<<1, 1024, 0, s>>>(bits, nw, pre);
+  k_commit_gather<<<(n + 255) / 256, 256, 0, s>>>(bits, pre, n, res, out);
+  note_launch(2);
+}
+
 // LTPG_BATCH_CARRY_ABORTS: the previous batch's conflict aborts (abort[0..nc), ascending ranks) ->
 // the first nc txns of this batch, with their original TIDs, types and 128-byte blocks.  One
 // warp per carried txn: lanes move the block as 32 coalesced 4-byte words.

@@ -284,7 +284,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       if (active && l < 15) v[k] = *reinterpret_cast<const uint2*>(p + 8 + 8 * l);  // u32 i | u16 supply_w | u8 qty
     }
     const uint32_t n = h0 >> 24;
-    bool bad = false;
+    // header (k_tpcc_group of an unpartitioned batch does not read it): district, line count, customer
+    bool bad = active && sub == 3 &&
+               ((h0 & 0xFFFFu) < 1 || (h0 & 0xFFFFu) > b.nw || ((h0 >> 16) & 0xFFu) < 1 || ((h0 >> 16) & 0xFFu) > 10 ||
+                n < 1 || n > 15 || (h1 & 0xFFFFu) < 1 || (h1 & 0xFFFFu) > 3000);
 #pragma unroll
     for (uint32_t k = 0; k < 4; ++k) {
       const uint32_t l = 4 * sub + k;
@@ -675,6 +678,11 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   // by-name lookup, result and HISTORY row) on the customer's owner
   const bool home = owns_w(b, w), cust = owns_w(b, cw);
   uint32_t row_w = ROW_NONE, row_d = ROW_NONE, row_c = ROW_NONE;
+  if (PH == PH_EXEC && (w < 1 || w > b.nw || d < 1 || d > 10 || cw < 1 || cw > b.nw || cd < 1 || cd > 10 ||
+                        by_name > 1 || (by_name ? clast > 999 : (cid < 1 || cid > 3000)))) {
+    atomicOr(b.err, ERR_EINVAL);  // validation (k_tpcc_group of an unpartitioned batch reads no Payment)
+    return;
+  }
   if (PH == PH_EXEC) {
     PP pw{}, pd{};
     if (home) {  // warehouse + district lookups and the by-name lookup in flight together
@@ -759,7 +767,7 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
 // order lines 4q..4q+3 (all of a lane's line loads in flight together).
 template <int PH>
 __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t sub, bool active,
-                                 Tx& x) {
+                                 Tx& x) {  // (active: by value -- a txn failing validation stops here)
   const DevTable& TCu = c_tabs[TC];
   const DevTable& TOr = c_tabs[TO];
   const DevTable& TOL_ = c_tabs[TOL];
@@ -770,6 +778,11 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
   if (active) {
     w = p16(p, 0);
     d = p[2];
+  }
+  if (active && sub == 3 && PH == PH_EXEC &&
+      (w < 1 || w > b.nw || d < 1 || d > 10 || p[3] > 1 || (p[3] ? p16(p, 6) > 999 : (p16(p, 4) < 1 || p16(p, 4) > 3000)))) {
+    atomicOr(b.err, ERR_EINVAL);  // validation (k_tpcc_group of an unpartitioned batch reads no OrderStatus)
+    active = false;
   }
   if (active && sub == 3) {
     if (PH == PH_EXEC) {
@@ -1367,8 +1380,6 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
       }
     }
     __syncwarp();
-  } else if (r < b.n_txns) {
-    head = *reinterpret_cast<const uint4*>(b.params + 128ull * r);
   }
   uint32_t t = 0xFF, lines = 0;
   bool bad = false;
@@ -1376,12 +1387,19 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     if (r > 0 && b.tid[r] <= b.tid[r - 1]) bad = true;
     if (b.grank && (b.grank[r] >= b.n_global || (r > 0 && b.grank[r] <= b.grank[r - 1]))) bad = true;
     t = b.ptype[r];
+    // !FULL: only Delivery and StockLevel blocks are read here (their warehouse / district index
+    // per-batch scratch before execute runs); NewOrder, Payment and OrderStatus are validated by
+    // execute, which reads their parameters anyway -- so this kernel streams the 9 bytes of TID and
+    // type per txn instead of fetching every 128-byte block (its first 16 bytes cost a whole line)
+    if (!FULL && (t == 3 || t == 4)) head = *reinterpret_cast<const uint4*>(b.params + 128ull * r);
     const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
     const uint32_t W = tp.nw;
     auto okw = [W](uint32_t w) { return w >= 1 && w <= W; };
     auto okd = [](uint32_t d) { return d >= 1 && d <= 10; };
-    if (!okw(p16(p, 0))) bad = true;
-    switch (t) {
+    if ((FULL || t == 3 || t == 4) && !okw(p16(p, 0))) bad = true;
+    if (!FULL && t <= 2) {
+      lines = t == 0 ? 15 : 0;  // capacity: a NewOrder may append up to 15 lines (its count is checked in execute)
+    } else switch (t) {
       case 0: {
         const uint32_t nl = p[3], c = p16(p, 4);
         if (!okd(p[2]) || nl < 1 || nl > 15 || c < 1 || c > 3000) { bad = true; break; }
@@ -1426,12 +1444,16 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
   uint32_t no_home = 0, pay_cust = 0;
   if (r < b.n_txns && !bad) {
     const uint8_t* p = FULL ? sw + SROW * lane : reinterpret_cast<const uint8_t*>(&head);
-    const bool home = owns_w(b, p16(p, 0));
+    const bool home = FULL ? owns_w(b, p16(p, 0)) : true;
     touch = home;
     // partitions the txn touches (bit q; the sharded exchange needs them, world <= 32)
     const auto pbit = [&](uint32_t w) { const uint32_t q = part_of_w(w, b.nw, b.nparts); return q < 32 ? 1u << q : 0u; };
     uint32_t pm = pbit(p16(p, 0));
-    if (FULL && t == 0) {
+    if (!FULL) {  // one partition: every txn is home; NewOrder and Payment may append
+      touch = true;
+      no_home = t == 0;
+      pay_cust = t == 1;
+    } else if (t == 0) {
       for (uint32_t l = 0; l < lines; ++l) pm |= pbit(p16(p + 8 + 8 * l, 4));
       touch = (pm >> b.part) & 1u;
       no_home = home;

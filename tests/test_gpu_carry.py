@@ -71,3 +71,36 @@ def test_carry_needs_a_completed_previous_batch():
     with pytest.raises(lib.LtpgError) as e:  # carried + given > max_txns
         g.run_tpcc(wl.batch(512, 5000, 3), 5, carry=True)
     assert e.value.rc == lib.LTPG_EINVAL
+
+
+@pytest.mark.parametrize("device_out", [False, True])
+def test_committed_reads_only(device_out):
+    """LTPG_RESULT_COMMITTED_READS: the result slots of the committed txns, packed in rank order,
+    written by the kernel into a pinned host (or device) buffer; with NO_STATUS / NO_ABORT_LIST
+    the bitmask and n_aborted still describe the batch.  == the oracle's committed rows."""
+    import torch
+    lib = L()
+    W, B = 2, 3000
+    wl = tpcc.TpccWorkload(W, seed=73, mode="strict", mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=B, tables=tables, append_batches=4)
+    o = oracle.tpcc_db(wl, tables)
+    for bno in range(3):
+        b = wl.batch(B - 7 * bno, 1 + B * bno, bno)  # ragged sizes
+        rc, st, res = o.run_tpcc(b, 2 + bno)
+        inp = b
+        if device_out:
+            inp = {k: torch.from_numpy(np.ascontiguousarray(v)).cuda() for k, v in b.items()}
+        out = g.run_tpcc(inp, 2 + bno, device_out=device_out, committed_reads=True, no_status=bno == 1,
+                         no_abort_list=bno == 2, n_txns=len(b["tid"]))
+        bits = out["commit_bits"]
+        bits = bits.cpu().numpy() if hasattr(bits, "cpu") else np.asarray(bits)
+        got_commit = np.unpackbits(bits.view(np.uint8), bitorder="little")[:len(st)].astype(bool)
+        assert (got_commit == (st == 1)).all()
+        assert int(np.asarray(out["n_aborted"].cpu() if hasattr(out["n_aborted"], "cpu") else out["n_aborted"])[0]) \
+            == int((st == ST_CONFLICT).sum())
+        reads = out["reads"]
+        reads = reads.cpu().numpy() if hasattr(reads, "cpu") else np.asarray(reads)
+        nc = int((st == 1).sum())
+        assert (reads.reshape(-1)[:4 * nc].reshape(nc, 4) == res[st == 1]).all(), bno
+    compare_tables(g, o)

@@ -203,3 +203,22 @@ def test_closed_loop_with_compose_retry():
         assert (nxt["tid"][:len(ab)] == batch["tid"][ab]).all() and nf == 1024 - len(ab)
         tid += nf
         batch = nxt
+
+
+@pytest.mark.parametrize("theta", [0.5, 0.99])
+def test_ycsb_sparse_keys_hash_probe(theta):
+    """Sparse u64 keys (splitmix64 of the row number): no dense key -> row mapping, every op goes
+    through the PK hash index (linear probing); closed loop with retries == oracle."""
+    wl = YcsbWorkload(50_000, theta=theta, ops_per_txn=10, seed=0x5A1, sparse_keys=True)
+    keys, cols = wl.initial_table()
+    descs = {0: tuple(wl.table_desc()[:3])}
+    tables = {0: (keys, cols)}
+    g, o = make_pair(descs, tables, 4096, 40960)
+    pending, tid = None, 1
+    for b in range(6):
+        fresh = wl.batch(4096 - (0 if pending is None else len(pending["tid"])), tid, b)
+        tid += len(fresh["tid"])
+        batch = fresh if pending is None else concat(pending, fresh)
+        st = check_batch(g, o, batch, tables)
+        ab = np.nonzero(st == ST_CONFLICT)[0]
+        pending = select(batch, ab) if len(ab) else None

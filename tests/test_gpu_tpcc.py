@@ -316,3 +316,29 @@ def test_neworder_line_validation_in_execute(what):
     compare_tables(g, o)                                   # nothing changed
     compare(g, o, wl.batch(1000, 5000, 1), 3)              # and the db still works
     compare_tables(g, o)
+
+
+@pytest.mark.parametrize("ptype,off,val", [
+    (NEW_ORDER, 0, 3), (NEW_ORDER, 2, 11), (NEW_ORDER, 3, 0), (NEW_ORDER, 3, 16), (NEW_ORDER, 4, 0),
+    (PAYMENT, 0, 0), (PAYMENT, 2, 0), (PAYMENT, 3, 2), (PAYMENT, 4, 5), (PAYMENT, 6, 12),
+    (2, 0, 7), (2, 2, 0), (2, 3, 3), (DELIVERY, 0, 9), (DELIVERY, 2, 11), (4, 0, 0), (4, 2, 15),
+])
+def test_header_validation_every_type(ptype, off, val):
+    """Each procedure's header checks (grouping for Delivery / StockLevel, execute for the others in
+    an unpartitioned batch): a bad field is EINVAL, nothing changes, the db keeps working == oracle."""
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=29, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3)
+    o = oracle.tpcc_db(wl, tables)
+    b = wl.batch(1000, 1, 0)
+    i = int(np.nonzero(b["type"] == ptype)[0][2])
+    b["params"][i, off] = val
+    if off in (0, 4) and val < 256:
+        b["params"][i, off + 1] = 0
+    assert o.run_tpcc(b, 2)[0] == oracle.ORC_EINVAL
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(b, 2)
+    assert e.value.rc == lib.LTPG_EINVAL
+    compare_tables(g, o)
+    compare(g, o, wl.batch(1000, 5000, 1), 3)

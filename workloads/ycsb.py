@@ -13,7 +13,7 @@ txn, 10^4..10^7 rows) and of BASELINE.json configs[0] / configs[2]:
 import math
 import numpy as np
 
-from .formats import OP_DTYPE, SELECT, UPDATE, SCAN, INSERT
+from .formats import OP_DTYPE, SELECT, UPDATE, SCAN, INSERT, KEY_EMPTY
 
 M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
 
@@ -53,7 +53,8 @@ class YcsbWorkload:
     TABLE = 0
 
     def __init__(self, n_rows, n_fields=10, theta=0.99, ops_per_txn=10, read_frac=0.5,
-                 seed=0x17C0, scan_frac=0.0, insert_frac=0.0, max_scan_len=10, read_latest=False):
+                 seed=0x17C0, scan_frac=0.0, insert_frac=0.0, max_scan_len=10, read_latest=False,
+                 sparse_keys=False):
         self.n_rows = int(n_rows)
         self.n_fields = int(n_fields)
         self.theta = float(theta)
@@ -67,11 +68,24 @@ class YcsbWorkload:
         self.b = (self.seed * 7919) % self.n_rows
         self.next_insert_key = self.n_rows
         self.read_latest = bool(read_latest)
+        # sparse_keys: row k is stored under the u64 key splitmix64(k) (a bijection), so keys are
+        # scattered over 2^64 and every lookup goes through the PK hash index instead of the
+        # dense key -> row arithmetic; point ops only (no SCAN / INSERT)
+        self.sparse_keys = bool(sparse_keys)
+        assert not (self.sparse_keys and (self.scan_frac or self.insert_frac)), "sparse keys: point ops only"
 
     # -- table ------------------------------------------------------------------
     def table_desc(self):
         """(col_group, col_is_add, n_groups, has_pk): one conflict unit per row (G=1)."""
         return [0] * self.n_fields, [0] * self.n_fields, 1, True
+
+    def key_of(self, k):
+        """Stored key of logical row k (identity, or splitmix64 with sparse_keys)."""
+        k = np.asarray(k, dtype=np.uint64)
+        if not self.sparse_keys:
+            return k
+        with np.errstate(over="ignore"):
+            return splitmix64(k)
 
     def initial_table(self):
         keys = np.arange(self.n_rows, dtype=np.uint64)
@@ -80,6 +94,8 @@ class YcsbWorkload:
             with np.errstate(over="ignore"):
                 v = splitmix64(keys * np.uint64(16) + np.uint64(f)) & np.uint64(0xFFFFFFFF)
             cols[f] = v.astype(np.int64)
+        keys = self.key_of(keys)
+        assert not (keys == np.uint64(KEY_EMPTY)).any()
         return keys, cols
 
     # -- batches ------------------------------------------------------------------
@@ -167,7 +183,7 @@ class YcsbWorkload:
                 keys[rd] = (np.uint64(latest) - (off[rd] % (latest + 1)).astype(np.uint64))
             self._dedupe_scans(keys, kinds, aux)
         ops = np.zeros(n_txns * k, dtype=OP_DTYPE)
-        ops["key"] = keys.reshape(-1)
+        ops["key"] = self.key_of(keys.reshape(-1))
         ops["kind"] = kinds.reshape(-1)
         ops["table"] = self.TABLE
         ops["col"] = rng.integers(0, self.n_fields, n_txns * k, dtype=np.uint16)
