@@ -165,9 +165,10 @@ def measured_peaks():
 
 def ncu_traffic(workload, kernel_substr):
     """dram read+write bytes per launch of the kernel from the committed `ncu --set full`
-    summary of this workload (profiles/ncu_r01_<workload>.json), or None."""
-    p = os.path.join(ROOT, "profiles", "ncu_r01_%s.json" % workload)
-    if not os.path.exists(p):
+    summary of this workload (profiles/ncu_r02_<workload>.json, else the round-1 one), or None."""
+    p = next((q for q in (os.path.join(ROOT, "profiles", "ncu_r0%d_%s.json" % (k, workload)) for k in (2, 1))
+              if os.path.exists(q)), None)
+    if p is None:
         return None
     try:  # summed over every instantiation that matches (the execute stage may be two launches)
         d = json.load(open(p))
@@ -261,6 +262,28 @@ def tpcc_exec_algorithmic_bytes(batch, mode):
     b[sl] = 32 + 32
     full_sl = 32 + 20 * (32 + 32 + 4 + 10 * 8) + 190 * 32 + 32
     return int(b.sum()) + n_dw * full_dl + n_sd * full_sl
+
+
+def tpcc_random_touches(batch):
+    """Independent random row/mark touches of the TPC-C execute stage per batch (the TPC-C analogue
+    of ops_random_reads): NewOrder 2 per line (item price read, stock mark) + 3 (W / D / C static
+    reads; the district mark is in shared memory); Payment 2 (customer row, customer mark) + 1 by
+    name; OrderStatus 4 + its ~10 lines; a Delivery leader per warehouse ~10 x (cursor, 2 probes,
+    order row, customer row + ~10 lines) = 150; StockLevel once per district ~20 x 3 + ~190 stock
+    rows = 250, + 1 per txn.  Many of these hit L2 (items, marks), so the fraction of the DRAM
+    random-read ceiling is an upper estimate of how hard the stage drives the memory system."""
+    ty = batch["type"]
+    p = batch["params"]
+    nl = p[:, 3].astype(np.int64)
+    w = p[:, 0].astype(np.int64) | (p[:, 1].astype(np.int64) << 8)
+    t = np.zeros(len(ty), np.int64)
+    t[ty == 0] = 2 * nl[ty == 0] + 3
+    t[ty == 1] = 2 + p[ty == 1, 3].astype(np.int64)
+    t[ty == 2] = 14
+    t[ty == 4] = 1
+    n_dw = len(np.unique(w[ty == 3]))
+    n_sd = len(np.unique(w[ty == 4] * 16 + p[ty == 4, 2].astype(np.int64)))
+    return int(t.sum()) + 150 * n_dw + 250 * n_sd
 
 
 def fused_algorithmic_bytes(batch, sparse=False):
@@ -850,6 +873,13 @@ def main():
                 "frac": ach / peak, "traffic": ncu_traffic(name, "k_tpcc_phase<0,"), "peak_source": peak_kind,
                 "algorithmic_bytes_per_launch": bytes_exec, "kernel_ms": ms,
                 "kernel_share_of_step": ms / statistics.mean(step_ms)}
+        ntouch = statistics.mean(tpcc_random_touches(host_batches[(args.warmup + s) % n_distinct])
+                                 for s in range(args.steps))
+        roof["random_access"] = {
+            "touches_per_launch": ntouch, "ceiling_g_per_s": RANDOM_READ_CEILING_G,
+            "achieved_g_per_s": ntouch / (ms / 1000.0) / 1e9,
+            "frac": ntouch / (ms / 1000.0) / 1e9 / RANDOM_READ_CEILING_G,
+            "source": "tools/randbw.cu, profiles/randbw_r01.txt; touches: bench.py tpcc_random_touches"}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps, "higher_is_better": True,

@@ -126,6 +126,7 @@ struct ltpg_db {
   unsigned long long* d_idx_from = nullptr;  // [MAXT]
   uint16_t* d_su = nullptr;                  // [MAXT] NEXT-3: this batch's bucket size per table
   uint32_t* d_wprefix = nullptr;             // LTPG_RESULT_COMMITTED_READS: commits before each bitmask word
+  uint32_t* d_coop = nullptr;                // [4096] per-block partial sums of cooperative kernels
   std::vector<Part> parts;
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_scan = nullptr;
@@ -240,8 +241,10 @@ __global__ void k_sum_res(void* const* res, uint32_t np, uint64_t n, long long* 
   }
 }
 __global__ void k_copy_err(const uint32_t* src, uint32_t* dst) { *dst = *src; }
-__global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint32_t n) {
-  if (threadIdx.x < n) host_dst[threadIdx.x] = src[threadIdx.x];
+// err_extra (single partition): the partition's own error word, ORed into word 0 here instead of
+// a k_or_err launch at the end of every batch
+__global__ void k_publish(const uint32_t* src, volatile uint32_t* host_dst, uint32_t n, const uint32_t* err_extra) {
+  if (threadIdx.x < n) host_dst[threadIdx.x] = src[threadIdx.x] | (threadIdx.x == 0 && err_extra ? *err_extra : 0u);
 }
 // batch start: append reservations cleared and the batch scalars stored where the kernels read
 // them -- from the arguments (direct enqueue) or, in a replayed graph, from the slot's pinned
@@ -306,6 +309,7 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(dmalloc(&db->d_idx_from, MAXT));
   CK(dmalloc(&db->d_su, MAXT));
   CK(dmalloc(&db->d_wprefix, (n + 31) / 32 + 1));
+  CK(dmalloc(&db->d_coop, 4096));
   CK(cudaMemset(db->d_su, 0, MAXT * sizeof(uint16_t)));
   CK(dmalloc(&db->d_dense_live, 1));
   CK(cudaMemset(db->d_dense_live, 0, sizeof(uint32_t)));
@@ -394,7 +398,7 @@ void ltpg_destroy_db(ltpg_db* db) {
   cudaDeviceSynchronize();
   for (int t = 0; t < MAXT; ++t) free_table(db->h_tab[t]);
   void* bufs[] = {db->d_tab, db->d_nrows, db->d_reserve, db->d_dense_live, db->d_ptrs, db->d_scan,
-                  db->d_idx_from, db->d_su, db->d_wprefix};
+                  db->d_idx_from, db->d_su, db->d_wprefix, db->d_coop};
   for (void* p : bufs)
     if (p) cudaFree(p);
   for (Slot& S : db->slots) {
@@ -936,10 +940,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (fused) {  // validate + warp-local division + execute; INSERTs after their claims
           launch_ops_fused(db->n_tables, x, filter, s);
           if (evp) CK(tmark(evp[2], s));  // ms_group = the fused kernel; ms_exec = INSERT tail
-          scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
-          launch_capacity_check(db->n_tables, x.ins_tables, x.txn_ins + n, x.base, x.reserve, x.err, s);
-          launch_ops_claim(x, s);
-          launch_ops_exec_inserts(x, filter, s);
+          launch_ops_insert_tail(db->n_tables, x, filter, db->d_coop, s);  // one launch; no INSERT: returns
         } else {
           launch_ops_validate_group(db->n_tables, x, grouped, s);
           scan_exclusive_u32(x.txn_ins, x.txn_ins, n, db->d_scan, s, x.ins_tables);  // skipped: no INSERT
@@ -1004,8 +1005,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       k_sum_res<<<148 * 8, 256, 0, s>>>(db->d_ptrs + 128, L, n_reads, res_out);
       note_launch();
     }
-    for (uint32_t p = 0; p < L; ++p) {  // errors raised during write-back reach the caller too
-      k_or_err<<<1, 1, 0, s>>>(pb[p].err, S.d_small);
+    for (uint32_t p = 0; p < L && L > 1; ++p) {  // errors raised during write-back reach the caller
+      k_or_err<<<1, 1, 0, s>>>(pb[p].err, S.d_small);  // too (one partition: k_publish ORs it in)
       note_launch();
     }
     CK(cudaStreamWaitEvent(s, db->fin_done, 0));
@@ -1082,7 +1083,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const cudaMemcpyKind out_kind = S.host_out ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
   // error word, counters and abort count: one tiny kernel stores them into mapped host memory
   // (cheaper than a D2H copy in stream order); device outputs were written in place
-  k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17);
+  k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17, L == 1 ? db->parts[0].small : nullptr);
   note_launch();
   if (n && S.host_out) {
     if (res->status) CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));

@@ -643,16 +643,7 @@ void launch_build_index(uint32_t t, uint64_t row0, uint64_t n, uint32_t* err,
 // n_rows + base + [0, total); base is this partition's offset in the batch reservation.
 __global__ void k_capacity(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
                            unsigned long long* base, unsigned long long* reserve, uint32_t* err) {
-  const uint32_t m = *ins_tables;
-  const uint64_t tot = *total;
-  for (uint32_t t = 0; t < n_tables; ++t) {
-    base[t] = reserve[t];
-    if ((m >> t) & 1u) {
-      const DevTable& T = c_tabs[t];
-      reserve[t] += tot;
-      if (*T.n_rows + reserve[t] > T.capacity || *T.n_rows + reserve[t] > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
-    }
-  }
+  capacity_body(n_tables, ins_tables, total, base, reserve, err);
 }
 
 void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,

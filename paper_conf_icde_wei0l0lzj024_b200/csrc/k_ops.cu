@@ -7,7 +7,13 @@
 //            slots, epoch-tagged atomicMin marks per conflict unit (a4, a5)
 //  K-detect  rcheck / wcheck: per-txn OR of the RAW/WAW test (a6)
 //  K-wb      getStatus -> writeMem: committed write sets only (a7)
+#include <cooperative_groups.h>
+
+#include <algorithm>
+
 #include "ltpg_internal.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace ltpg {
 
@@ -191,7 +197,7 @@ void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool groupe
 
 // ---- K-claim: INSERT keys claim their slot; provisional row = n_rows + rank of the
 //      insert in (rank, op) order; atomicMin makes the earliest inserter own the unit ----
-__global__ void __launch_bounds__(256) k_ops_claim(BatchDev b) {
+__device__ __forceinline__ void ops_claim_body(const BatchDev& b) {
   if (*b.err) return;
   const uint32_t n = b.kcount[LTPG_INSERT];
   const unsigned long long* list = b.items + (uint64_t)LTPG_INSERT * b.max_ops;
@@ -210,6 +216,7 @@ __global__ void __launch_bounds__(256) k_ops_claim(BatchDev b) {
     atomicMin(&sl->claim, prov);
   }
 }
+__global__ void __launch_bounds__(256) k_ops_claim(BatchDev b) { ops_claim_body(b); }
 
 void launch_ops_claim(const BatchDev& b, cudaStream_t s) {
   k_ops_claim<<<148 * 4, 256, 0, s>>>(b);
@@ -314,7 +321,7 @@ __device__ __forceinline__ void exec_one(const BatchDev& b, uint32_t oi, uint32_
 }
 
 template <bool GROUPED>
-__global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
+__device__ __forceinline__ void ops_exec_body(const BatchDev& b, bool filter) {
   if (*b.err) return;
   const uint32_t dmask = *b.dense_live & ~*b.insdel;
   const int lane = threadIdx.x & 31;
@@ -341,6 +348,8 @@ __global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) {
     exec_one(b, oi, r, o, filter, dmask);
   }
 }
+template <bool GROUPED>
+__global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) { ops_exec_body<GROUPED>(b, filter); }
 
 // ---- K-fused: a1 + warp-local kind division + a4/a5 in one pass ------------
 // Each warp validates its 32 txns from shared memory, orders its own ops by kind and runs
@@ -452,6 +461,98 @@ void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStr
 
 void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s) {
   k_ops_exec<true><<<148 * 2, 256, 0, s>>>(b, filter);  // only the INSERT list is populated
+  note_launch();
+}
+
+// The fused front end's INSERT tail in ONE cooperative launch (grid-wide barriers between the
+// steps): exclusive scan of the per-txn insert counts -> capacity check and the partition's row
+// base -> index claims -> execution of the INSERT list.  A batch without INSERTs (YCSB A/B/C, the
+// common case) leaves after one load of the insert-table mask -- instead of the six dependent
+// launches (3-kernel scan, capacity, claim, exec) it paid before.
+__global__ void __launch_bounds__(256) k_ops_insert_tail(uint32_t n_tables, BatchDev b, bool filter,
+                                                         uint32_t* partials) {
+  cg::grid_group grid = cg::this_grid();
+  const uint32_t n = b.n_txns;
+  if (*(volatile uint32_t*)b.ins_tables == 0) {  // uniform: written by the previous kernel
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      b.txn_ins[n] = 0;
+      for (uint32_t t = 0; t < n_tables; ++t) b.base[t] = b.reserve[t];  // (k_capacity with no inserts)
+    }
+    return;
+  }
+  // exclusive scan of txn_ins[0, n) in place, total in txn_ins[n]: block chunks, their sums, offsets
+  __shared__ uint32_t wsum[8];
+  __shared__ uint32_t carry;
+  const uint32_t per = (n + gridDim.x - 1) / gridDim.x, lo = min(n, blockIdx.x * per), hi = min(n, lo + per);
+  uint32_t part = 0;
+  for (uint32_t i = lo + threadIdx.x; i < hi; i += blockDim.x) part += b.txn_ins[i];
+  part = __reduce_add_sync(0xffffffffu, part);
+  if ((threadIdx.x & 31) == 0) wsum[threadIdx.x >> 5] = part;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < 8; ++w) t += wsum[w];
+    partials[blockIdx.x] = t;
+  }
+  grid.sync();
+  if (threadIdx.x == 0) {
+    uint32_t off = 0;
+    for (uint32_t q = 0; q < blockIdx.x; ++q) off += partials[q];
+    carry = off;
+    if (blockIdx.x == gridDim.x - 1) {
+      uint32_t tot = off;
+      for (uint32_t q = blockIdx.x; q < gridDim.x; ++q) tot += partials[q];
+      b.txn_ins[n] = tot;
+    }
+  }
+  __syncthreads();
+  const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = lo; base < hi; base += blockDim.x) {  // 256 at a time, carried across rounds
+    const uint32_t i = base + threadIdx.x;
+    const uint32_t v = i < hi ? b.txn_ins[i] : 0u;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= (uint32_t)o) x += y;
+    }
+    __syncthreads();
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    uint32_t before = carry, round = 0;
+    for (uint32_t w = 0; w < 8; ++w) {
+      if (w < wid) before += wsum[w];
+      round += wsum[w];
+    }
+    if (i < hi) b.txn_ins[i] = before + x - v;
+    __syncthreads();
+    if (threadIdx.x == 0) carry += round;
+  }
+  grid.sync();
+  if (blockIdx.x == 0 && threadIdx.x == 0)
+    capacity_body(n_tables, b.ins_tables, b.txn_ins + n, b.base, b.reserve, b.err);
+  grid.sync();
+  ops_claim_body(b);
+  grid.sync();
+  ops_exec_body<true>(b, filter);  // only the INSERT list is populated
+}
+
+void launch_ops_insert_tail(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials, cudaStream_t s) {
+  static int per_sm = 0, sms = 0;
+  if (!per_sm) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_ops_insert_tail, 256, 0) != cudaSuccess || per_sm < 1)
+      per_sm = 1;
+  }
+  const uint32_t want = std::max<uint32_t>(1, (b.n_txns + 1023) / 1024);
+  const uint32_t grid = std::min<uint32_t>(std::min<uint32_t>(want, (uint32_t)(per_sm * sms)), 4096);  // partials[4096]
+  uint32_t nt = n_tables;
+  BatchDev bb = b;
+  bool f = filter;
+  void* args[] = {&nt, &bb, &f, &partials};
+  cudaLaunchCooperativeKernel((const void*)k_ops_insert_tail, dim3(grid), dim3(256), args, 0, s);
   note_launch();
 }
 

@@ -1253,35 +1253,59 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
   // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
   constexpr uint32_t ORD = PH == PH_DETECT ? (2u | SL_DLW << 4 | 0u << 8 | SL_DLT << 12 | 1u << 16 | 4u << 20)
                                            : (0u | 1u << 4 | 2u << 8 | SL_DLW << 12 | SL_DLT << 16 | 4u << 20);  // slot j -> type
-  uint32_t cnt[NSLOT], pre[NSLOT + 1];
-  pre[0] = 0;
-#pragma unroll
-  for (int j = 0; j < NSLOT; ++j) {
-    const uint32_t t = (ORD >> (4 * j)) & 15u;
-    const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
-    cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : tp.counts[t]));
-    const uint32_t lp = 5 - (__ffs(lanes_of(t, PH, b.nparts, reorder)) - 1);  // log2(txns per warp slot)
-    pre[j + 1] = pre[j] + ((cnt[j] + (1u << lp) - 1) >> lp);
+  // slot counts and warp-slot prefixes per slot type, in shared memory (computed once per block;
+  // as register arrays they cost every thread 12 registers for the whole kernel)
+  __shared__ uint32_t cnt[NSLOT], pre[NSLOT + 1];
+  if (threadIdx.x == 0) {
+    pre[0] = 0;
+    for (int j = 0; j < NSLOT; ++j) {
+      const uint32_t t = (ORD >> (4 * j)) & 15u;
+      const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
+      cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : tp.counts[t]));
+      const uint32_t lp = 5 - (__ffs(lanes_of(t, PH, b.nparts, reorder)) - 1);  // log2(txns per warp slot)
+      pre[j + 1] = pre[j] + ((cnt[j] + (1u << lp) - 1) >> lp);
+    }
   }
+  __syncthreads();
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib; w < pre[NSLOT]; w += nwarps) {
-    uint32_t j = 0, lw = w, ct = cnt[0];
+  // warp slot w -> slot type t, this lane's list position k and sub-lane (warp-uniform type)
+  const auto decode = [&](uint32_t w, uint32_t& t, uint32_t& k, uint32_t& sub, uint32_t& ct) {
+    uint32_t j = 0, lw = w;
+    ct = cnt[0];
 #pragma unroll
     for (int jj = 1; jj < NSLOT; ++jj)
-      if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }  // warp-uniform slot type
-    const uint32_t t = (ORD >> (4 * j)) & 15u;
-    const uint32_t L = lanes_of(t, PH, b.nparts, reorder);  // a power of two
-    const uint32_t ll = __ffs(L) - 1;
-    const uint32_t k = (lw << (5 - ll)) + (lane >> ll);
-    const uint32_t sub = lane & (L - 1);
+      if (w >= pre[jj]) { j = jj; lw = w - pre[jj]; ct = cnt[jj]; }
+    t = (ORD >> (4 * j)) & 15u;
+    const uint32_t ll = __ffs(lanes_of(t, PH, b.nparts, reorder)) - 1;  // lanes per txn: a power of two
+    k = (lw << (5 - ll)) + (lane >> ll);
+    sub = lane & ((1u << ll) - 1u);
+  };
+  // the list entry of a warp's NEXT slot is loaded before the current slot runs: the list ->
+  // parameters -> rows chain of each slot starts one load later than its list read
+  const auto list_entry = [&](uint32_t w) -> uint32_t {
+    uint32_t t, k, sub, ct;
+    decode(w, t, k, sub, ct);
+    return (t != SL_DLW && k < ct) ? tp.list[(uint64_t)t * tp.max_txns + k] : 0u;
+  };
+  uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib;
+  uint32_t r_next = w < pre[NSLOT] ? list_entry(w) : 0u;
+  for (; w < pre[NSLOT]; w += nwarps) {
+    uint32_t t, k, sub, ct;
+    decode(w, t, k, sub, ct);
+    const uint32_t L = lanes_of(t, PH, b.nparts, reorder);
     bool active = k < ct;
-    uint32_t r = 0;
+#ifdef LTPG_NO_PREFETCH
+    uint32_t r = list_entry(w);
+#else
+    uint32_t r = r_next;
+    if (w + nwarps < pre[NSLOT]) r_next = list_entry(w + nwarps);
+#endif
     if (t == SL_DLW) {  // warehouse k + 1's Delivery leader (write-back: only if it committed)
       r = active ? tp.dl_min[k + 1] : ~0u;
       active = r != ~0u && (PH != PH_WB || b.status[r] == LTPG_ST_COMMIT);
       if (!active) r = 0;
-    } else if (active) {
-      r = tp.list[(uint64_t)t * tp.max_txns + k];
+    } else if (!active) {
+      r = 0;
     }
     const uint32_t gr = active ? grank_of(b, r) : 0u;  // conflict TID (global rank of a sharded batch)
     Tx x{dmask, gr, b_epoch(b), epoch_tag(b_epoch(b)) | gr, !(b.flags & LTPG_FLAG_NO_MARK_FILTER), 0u, b.err, reorder,

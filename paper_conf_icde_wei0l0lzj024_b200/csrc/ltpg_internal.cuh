@@ -439,6 +439,23 @@ __device__ __forceinline__ void block_reserve(const uint32_t (&cnt)[NK], uint32_
   for (int k = 0; k < NK; ++k) base[k] = gbase[k] + wsum[k][wid] + incl[k] - cnt[k];
 }
 
+// ECAPACITY before anything mutates (one thread).  The partition's inserts take provisional rows
+// n_rows + base + [0, total); base is this partition's offset in the batch reservation.  (Table
+// metadata: the calling translation unit's c_tabs.)
+__device__ __forceinline__ void capacity_body(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
+                                              unsigned long long* base, unsigned long long* reserve, uint32_t* err) {
+  const uint32_t m = *ins_tables;
+  const uint64_t tot = *total;
+  for (uint32_t t = 0; t < n_tables; ++t) {
+    base[t] = reserve[t];
+    if ((m >> t) & 1u) {
+      const DevTable& T = c_tabs[t];
+      reserve[t] += tot;
+      if (*T.n_rows + reserve[t] > T.capacity || *T.n_rows + reserve[t] > 0xFFFFFFF0ull) atomicOr(err, ERR_ECAPACITY);
+    }
+  }
+}
+
 // ---- ownership (contiguous ranges) -------------------------------------------------------
 __host__ __device__ __forceinline__ uint32_t part_of_w(uint32_t w, uint32_t nw, uint32_t np) {
   return np <= 1 || !nw ? 0u : (uint32_t)(((uint64_t)(w - 1) * np) / nw);
@@ -470,6 +487,8 @@ void launch_ops_claim(const BatchDev& b, cudaStream_t s);
 void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t s);
 void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStream_t s);
 void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s);
+// scan + capacity + claim + INSERT execution of the fused front end, one cooperative launch
+void launch_ops_insert_tail(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials, cudaStream_t s);
 void launch_ops_detect(const BatchDev& b, cudaStream_t s);
 void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cudaStream_t s);
 void launch_capacity_check(uint32_t n_tables, const uint32_t* ins_tables, const uint32_t* total,
