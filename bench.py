@@ -233,7 +233,8 @@ def exec_algorithmic_bytes(batch, sparse=False):
 def tpcc_exec_algorithmic_bytes(batch, mode):
     """Algorithmic bytes of the TPC-C execute kernel: 128 B parameter block,
     32 B per random column read or index probe of a sparse-keyed table, 64 B per mark (atomic
-    sector RMW), contiguous order lines at element size, 32 B result + 4 B per logged row.
+    sector RMW) outside the per-block shared-memory WAREHOUSE / DISTRICT marks, contiguous order
+    lines at element size, 32 B result + 4 B per logged row.
     W/D/C/I/S rows are found by arithmetic (dense keys); ORDER_LINE rows from ORDER.
     Delivery / StockLevel use the expected line counts (10 / 190 distinct items) and are
     counted once per warehouse / district, as they are executed."""
@@ -244,9 +245,11 @@ def tpcc_exec_algorithmic_bytes(batch, mode):
     by_name = p[:, 3].astype(bool)
     b = np.zeros(len(ty), np.int64)
     no = ty == 0
-    b[no] = 128 + 3 * 32 + 64 + nl[no] * (32 + 64 * (1 + delayed) + 4) + 32 + 4
+    # (the WAREHOUSE / DISTRICT marks are aggregated per block in shared memory and flushed once
+    # per touched unit and block: not counted per txn)
+    b[no] = 128 + 3 * 32 + nl[no] * (32 + 64 * (1 + delayed) + 4) + 32 + 4
     pay = ty == 1
-    b[pay] = 128 + 3 * 64 + 32 * (not delayed) + 4 * by_name[pay] + 16 + 32
+    b[pay] = 128 + 64 + 32 * (not delayed) + 4 * by_name[pay] + 16 + 32
     b[ty == 2] = 128 + 2 * 32 + 32 + 2 * 32 + 4 + 10 * 8 + 32 + 68
     # Delivery is shared per warehouse (only its smallest rank executes): the
     # full cost once per warehouse, a parameter sector per other Delivery
@@ -567,12 +570,15 @@ def main():
         hb = b
         if w["kind"] == "tpcc":  # host leg ships compact TPC-C records (LTPG_BATCH_COMPACT_PARAMS)
             packed, offs = ltpg.pack_params_compact(b["type"], b["params"])
-            hb = {"tid": b["tid"], "type": b["type"], "params": packed, "offsets": offs}
+            # consecutive TIDs ship as the first one (LTPG_BATCH_TID_RANGE); a shard's are not consecutive
+            hb = {"tid": b["tid"] if sharded else b["tid"][:1].copy(), "type": b["type"], "params": packed,
+                  "offsets": offs}
             if sharded:
                 hb.update(grank=b["grank"], n_global=b["n_global"])
         pin_batches.append({k: to_t(v, True) for k, v in hb.items()})
         if w["kind"] == "tpcc":
             pin_batches[-1]["compact"] = True
+            pin_batches[-1]["tid_range"] = not sharded
 
     # result buffers allocated once (device for the resident leg, pinned host for e2e), so no
     # allocation ever lands inside a timed step
@@ -593,8 +599,12 @@ def main():
             return db.run_ops(inputs, stream=torch.cuda.current_stream().cuda_stream, want_reads=True,
                               device_out=device, stats=stats, n_txns=len(bh["tid"]), n_ops=len(bh["args"]),
                               out=out, wait=wait)
+        # host outputs: the commit bitmask, the abort list and the COMMITTED txns' result slots (written
+        # into pinned host memory by the kernel, LTPG_RESULT_COMMITTED_READS; the slots of aborted
+        # txns are snapshot reads recomputed on retry); status only for a shard (commit counting)
         return db.run_tpcc(inputs, clock, stream=torch.cuda.current_stream().cuda_stream, want_reads=True,
-                           device_out=device, stats=stats, n_txns=len(bh["tid"]), out=out, wait=wait)
+                           device_out=device, stats=stats, n_txns=len(bh["tid"]), out=out, wait=wait,
+                           committed_reads=not device, no_status=not device and not sharded)
 
     pin_of = {id(h): p for h, p in zip(host_batches, pin_batches)}
 
@@ -803,7 +813,10 @@ def main():
             else:
                 e_commits.append(int(np.bitwise_count(cb[:(n + 31) // 32].view(np.uint32)).sum()))
             nreads = n_reads if w["kind"] == "ycsb" else 4 * n
-            d2h += n + 4 * ((n + 31) // 32) + 4 * n + 8 * nreads + 68
+            if w["kind"] == "tpcc":  # bitmask, abort list (copied at capacity), committed slots, counters
+                d2h += 4 * ((n + 31) // 32) + 4 * n + 32 * e_commits[-1] + 68 + (n if sharded else 0)
+            else:
+                d2h += n + 4 * ((n + 31) // 32) + 4 * n + 8 * nreads + 68
 
         for s in range(args.steps):
             i = (args.warmup + s) % n_distinct
@@ -832,8 +845,12 @@ def main():
         e2e = {"value": e_c / e_s, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                "d2h_bytes_per_step": d2h // args.steps, "ms_per_step": 1000 * e_s / args.steps,
                "pipeline": "3 batches in flight (LTPG_BATCH_ASYNC): H2D / kernels / D2H overlapped",
-               "input": ("compact TPC-C records (LTPG_BATCH_COMPACT_PARAMS), expanded on the GPU"
-                         if w["kind"] == "tpcc" else "16-byte op records + i64 args")}
+               "input": ("compact TPC-C records (LTPG_BATCH_COMPACT_PARAMS) expanded on the GPU, consecutive "
+                         "TIDs as their first one (LTPG_BATCH_TID_RANGE)"
+                         if w["kind"] == "tpcc" else "16-byte op records + i64 args"),
+               "output": ("commit bitmask + abort list + the committed txns' result slots "
+                          "(LTPG_RESULT_COMMITTED_READS | LTPG_RESULT_NO_STATUS)" if w["kind"] == "tpcc"
+                          else "status + bitmask + abort list + every op's result slot")}
 
     if not os.environ.get("LTPG_NO_CLOCKS"):
         clk.__exit__(None, None, None)

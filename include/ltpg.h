@@ -279,6 +279,10 @@ typedef struct {
  * this batch is submitted.  EINVAL: OPS mode, device inputs, a graph db, or no completed previous
  * batch, or n_carried + n_txns > max_txns. */
 #define LTPG_BATCH_CARRY_ABORTS 4u
+/* Consecutive TIDs (host inputs): `tid` points to ONE u64, the TID of the first given txn; the
+ * i-th given txn has TID tid[0] + i (filled on the device, 8 bytes per txn less over PCIe).
+ * With LTPG_BATCH_CARRY_ABORTS the carried txns keep their own TIDs (tid[0] must exceed them). */
+#define LTPG_BATCH_TID_RANGE 8u
 
 typedef struct {
   float ms_upload, ms_group, ms_exec, ms_detect, ms_exchange, ms_writeback, ms_download;

@@ -134,6 +134,7 @@ ltpg_pending_aborts = _lib.ltpg_pending_aborts
 LTPG_BATCH_ASYNC = 1
 LTPG_BATCH_COMPACT_PARAMS = 2
 LTPG_BATCH_CARRY_ABORTS = 4
+LTPG_BATCH_TID_RANGE = 8
 LTPG_RESULT_COMMITTED_READS, LTPG_RESULT_NO_STATUS, LTPG_RESULT_NO_ABORT_LIST = 1, 2, 4
 
 EXPORTED = ["ltpg_create_db", "ltpg_load_table", "ltpg_run_batch", "ltpg_wait_batch", "ltpg_dump_table",
@@ -310,7 +311,8 @@ class Database:
         records with compact=True (see pack_params_compact).  A rank's shard of a global batch
         (route_tpcc) also carries grank u32[n] and n_global.  carry=True: the batch is the previous
         batch's conflict aborts (kept on the device) followed by these txns
-        (LTPG_BATCH_CARRY_ABORTS); the outputs cover pending_aborts() + n txns.  committed_reads:
+        (LTPG_BATCH_CARRY_ABORTS); the outputs cover pending_aborts() + n txns.  tid_range=True in
+        the batch dict: tid holds only the first TID, the others are consecutive (LTPG_BATCH_TID_RANGE).  committed_reads:
         reads = the result slots of the committed txns only, in rank order (host outputs must
         then be pinned memory); no_status / no_abort_list skip those outputs."""
         tid, ty, params = batch["tid"], batch["type"], batch["params"]
@@ -325,7 +327,8 @@ class Database:
                         proc_params=_ptr(params), batch_clock=int(clock), inputs_on_device=int(on_dev),
                         stream=c_vp(stream) if stream else None, proc_offsets=_ptr(offsets),
                         flags=(LTPG_BATCH_COMPACT_PARAMS if batch.get("compact") else 0) |
-                        (LTPG_BATCH_CARRY_ABORTS if carry else 0),
+                        (LTPG_BATCH_CARRY_ABORTS if carry else 0) |
+                        (LTPG_BATCH_TID_RANGE if batch.get("tid_range") else 0),
                         grank=_ptr(grank), n_global=int(batch.get("n_global", 0)))
         rflags = ((LTPG_RESULT_COMMITTED_READS if committed_reads else 0) | (LTPG_RESULT_NO_STATUS if no_status else 0)
                   | (LTPG_RESULT_NO_ABORT_LIST if no_abort_list else 0))

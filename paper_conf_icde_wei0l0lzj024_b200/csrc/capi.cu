@@ -689,6 +689,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
                 !db->carry_ok || db->carry_seq != db->submitted))
     return fail(db, LTPG_EINVAL, "LTPG_BATCH_CARRY_ABORTS: TPCC host inputs on a single-rank, non-graph db, after "
                                  "the previous batch completed");
+  const bool tid_range = (b->flags & LTPG_BATCH_TID_RANGE) != 0;
+  if (tid_range && b->inputs_on_device) return fail(db, LTPG_EINVAL, "LTPG_BATCH_TID_RANGE: host inputs only");
+  const unsigned long long tid0 = tid_range && nf ? (unsigned long long)b->tid[0] : 0ull;
   const uint32_t nc = carry ? db->carry_n : 0u;  // carried conflict aborts of the previous batch
   const uint32_t n = nc + nf;
   if ((uint64_t)nc + nf > db->cfg.max_txns) return fail(db, LTPG_EINVAL, "n_txns > max_txns"); 
@@ -769,7 +772,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     // the slot's staging buffers are free once its previous batch's kernels are done
     CK(cudaStreamWaitEvent(db->h2d, S.comp_done, 0));
     // (carried txns: positions [0, nc) are filled on the device by k_carry; the given ones follow)
-    CK(cudaMemcpyAsync(S.d_tid + nc, b->tid, nf * sizeof(uint64_t), h2d, db->h2d));
+    if (!tid_range) CK(cudaMemcpyAsync(S.d_tid + nc, b->tid, nf * sizeof(uint64_t), h2d, db->h2d));
     bd.tid = S.d_tid;
     if (sharded) {
       CK(cudaMemcpyAsync(S.d_grank, b->grank, n * sizeof(uint32_t), h2d, db->h2d));
@@ -906,6 +909,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         CK(cudaMemsetAsync(P.lflag, 0, n, s));  // txns this partition does not touch: no verdict
       }
     }
+    if (tid_range) launch_fill_tid(S.d_tid + nc, nf, tid0, s);  // consecutive TIDs of the given txns
     if (nc) {  // a9 on the device: the previous batch's conflict aborts lead this batch
       const Slot& P = db->slots[db->carry_slot];
       launch_carry(P.eff_tid, P.eff_ptype, P.eff_params, P.eff_abort, nc, S.d_tid, S.d_ptype, S.d_params, s);
@@ -1018,7 +1022,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // Graph replay: the same shape's captured graph if this slot has one, else capture, instantiate
   // and keep it (least recently used of GRAPHS_PER_SLOT replaced).  Multi-rank dbs enqueue
   // directly (their exchange selects buffers by epoch parity on the host).
-  const bool use_graph = n && db->cfg.world == 1 && (db->cfg.flags & LTPG_FLAG_GRAPH) && !cr;
+  const bool use_graph = n && db->cfg.world == 1 && (db->cfg.flags & LTPG_FLAG_GRAPH) && !cr && !tid_range;
   if (use_graph) {
     GraphKey k;
     std::memset(&k, 0, sizeof(k));

@@ -451,6 +451,16 @@ void launch_committed_reads(const uint32_t* bits, uint32_t n, const long long* r
   note_launch(2);
 }
 
+// LTPG_BATCH_TID_RANGE: tid[i] = t0 + i
+__global__ void k_fill_tid(unsigned long long* tid, uint32_t n, unsigned long long t0) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) tid[i] = t0 + i;
+}
+void launch_fill_tid(unsigned long long* tid, uint32_t n, unsigned long long t0, cudaStream_t s) {
+  if (!n) return;
+  k_fill_tid<<<std::min<uint32_t>((n + 255) / 256, 148 * 8), 256, 0, s>>>(tid, n, t0);
+  note_launch();
+}
+
 // LTPG_BATCH_CARRY_ABORTS: the previous batch's conflict aborts (abort[0..nc), ascending ranks) ->
 // the first nc txns of this batch, with their original TIDs, types and 128-byte blocks.  One
 // warp per carried txn: lanes move the block as 32 coalesced 4-byte words.

@@ -85,6 +85,13 @@ __device__ __forceinline__ uint32_t rowof(const DevTable& T, uint32_t t, uint64_
 }
 __device__ __forceinline__ long long rd(const DevTable& T, uint32_t c, uint32_t row) { return *col_ptr(T, c, row); }
 __device__ __forceinline__ void wr(const DevTable& T, uint32_t c, uint32_t row, long long v) { *col_ptr(T, c, row) = v; }
+// STOCK's four counters side by side in one 32-byte row block (row-block layout: S_QUANTITY,
+// S_YTD, S_ORDER_CNT, S_REMOTE_CNT at consecutive words, 16-byte aligned rows)
+__device__ __forceinline__ bool stock_block_vec(const DevTable& T) {
+  return !T.columnar && T.stride[S_QUANTITY] == 4 && T.col[S_YTD] == T.col[S_QUANTITY] + 1 &&
+         T.col[S_ORDER_CNT] == T.col[S_QUANTITY] + 2 && T.col[S_REMOTE_CNT] == T.col[S_QUANTITY] + 3 &&
+         (reinterpret_cast<uintptr_t>(T.col[S_QUANTITY]) & 15u) == 0;
+}
 // write-back increment: an ADD-unit column may have several committed adders (atomic); a
 // WRITE-unit column has exactly one committed writer per batch (R1: WAW) -> plain RMW
 __device__ __forceinline__ void addv(const DevTable& T, uint32_t c, uint32_t row, long long v) {
@@ -238,7 +245,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     if (!active) return;
     uint32_t rows[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) rows[k] = log[4 * sub + k];
+    for (int k = 0; k < 4; ++k) rows[k] = log[sub + 4 * k];  // slot sub + 4k: the 4 lanes read 16 B together
     const uint32_t gq = col_group(TSt, S_QUANTITY), gy = col_group(TSt, S_YTD);
     const uint32_t go = col_group(TSt, S_ORDER_CNT), gr = col_group(TSt, S_REMOTE_CNT);
     const uint32_t ay = col_is_add(TSt, S_YTD) ? ACC_ADD : ACC_WRITE;
@@ -247,7 +254,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     uint32_t bits = 0;
 #pragma unroll
     for (int k = 0; k < 4; ++k) {  // same units as the general path below (unit_w / col_upd3)
-      if (rows[k] == ROW_NONE || 4 * sub + k == 15) continue;
+      if (rows[k] == ROW_NONE || sub + 4 * k == 15) continue;
       bits |= unit_bits(TSt, gq, rows[k], ACC_WRITE, x.r, x.epoch);
       if (gy != gq) bits |= unit_bits(TSt, gy, rows[k], ay, x.r, x.epoch);
       if (go != gq && go != gy) bits |= unit_bits(TSt, go, rows[k], ao, x.r, x.epoch);
@@ -259,10 +266,12 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     return;
   }
   if (PH == PH_EXEC && b.nparts <= 1) {
-    // 4 lanes per NewOrder (lanes_of): lane q takes lines 4q..4q+3 (lane 3: lines 12-14 and the
-    // header).  A lane's line records, row lookups (arithmetic on the dense W/D/C/I/S key
-    // ranges) and item-price loads are all issued before any is used: 8 txns per warp instead
-    // of 2, so a warp pays the parameter -> price dependency chain once for 4x the lines.
+    // 4 lanes per NewOrder (lanes_of): lane q takes lines q, q+4, q+8, q+12 (lane 3: lines 3, 7,
+    // 11 and the header) -- so for each k the txn's 4 lanes read 4 consecutive 8-byte line records
+    // (one sector) and write 4 consecutive log slots.  A lane's line records, row lookups
+    // (arithmetic on the dense W/D/C/I/S key ranges) and item-price loads are all issued before any
+    // is used: 8 txns per warp instead of 2, so a warp pays the parameter -> price dependency chain
+    // once for 4x the lines.
     long long amount = 0, w_tax = 0, d_tax = 0, disc = 0;
     uint32_t ua = 0;
     // line validation (k_tpcc_group reads only the 16-byte headers of unpartitioned batches):
@@ -274,12 +283,13 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     uint2 v[4];
     uint32_t h0 = 0, h1 = 0;
     if (active) {
-      h0 = *reinterpret_cast<const uint32_t*>(p);
-      h1 = *reinterpret_cast<const uint32_t*>(p + 4);
+      const uint2 h = *reinterpret_cast<const uint2*>(p);  // u16 w | u8 d | u8 n_lines | u16 c | ...
+      h0 = h.x;
+      h1 = h.y;
     }
 #pragma unroll
     for (uint32_t k = 0; k < 4; ++k) {
-      const uint32_t l = 4 * sub + k;
+      const uint32_t l = sub + 4 * k;
       v[k] = make_uint2(0, 0);
       if (active && l < 15) v[k] = *reinterpret_cast<const uint2*>(p + 8 + 8 * l);  // u32 i | u16 supply_w | u8 qty
     }
@@ -290,7 +300,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
                 n < 1 || n > 15 || (h1 & 0xFFFFu) < 1 || (h1 & 0xFFFFu) > 3000);
 #pragma unroll
     for (uint32_t k = 0; k < 4; ++k) {
-      const uint32_t l = 4 * sub + k;
+      const uint32_t l = sub + 4 * k;
       if (l >= n) v[k] = make_uint2(0, 0);
       // unused slots get ids no item has (and that never collide with each other)
       it[k] = (active && l < n) ? v[k].x : 0xFFFFFFF0u - l;
@@ -332,7 +342,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       uint32_t qt[4], ri[4], rs[4];
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
-        const uint32_t l = 4 * sub + k;
+        const uint32_t l = sub + 4 * k;
         qt[k] = (v[k].y >> 16) & 0xFFu;
         ri[k] = l < n ? rowof(TIt, TI, v[k].x, x.dmask) : ROW_NONE;
         rs[k] = l < n ? rowof(TSt, TS, kS(v[k].y & 0xFFFFu, v[k].x), x.dmask) : ROW_NONE;
@@ -357,7 +367,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
 #endif
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
-        const uint32_t l = 4 * sub + k;
+        const uint32_t l = sub + 4 * k;
         if (l >= 15) continue;
         uint32_t row_s = ROW_NONE;
         if (l < n) {
@@ -402,11 +412,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     ua |= __shfl_xor_sync(0xffffffffu, ua, 2);
     if (active && sub == 3) {
       if (ua) b.ua[r] = 1;
-      long long* res = b.res + 4ull * r;
-      res[0] = 0;  // o_id: assigned after detection if committed
-      res[1] = amount * (10000 - disc) * (10000 + w_tax + d_tax) / 100000000;
-      res[2] = amount;
-      res[3] = 0;
+      longlong2* res = reinterpret_cast<longlong2*>(b.res + 4ull * r);
+      // [o_id (assigned after detection if committed), total, sum of amounts, 0]
+      res[0] = make_longlong2(0, amount * (10000 - disc) * (10000 + w_tax + d_tax) / 100000000);
+      res[1] = make_longlong2(amount, 0);
     }
     return;
   }
@@ -415,8 +424,12 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
     // write 4 consecutive ORDER_LINE rows per store); a lane's line records, item prices and
     // stock rows are all loaded before any is used
     uint32_t remote = 0, w = 0, d = 0, n = 0, c = 0;
+    // the stock row block holds the four counters side by side (row-block layout, 32 B): read
+    // and written as two 16-byte vectors instead of four 8-byte accesses to the same sector
+    const bool svec = stock_block_vec(TSt);
     if (active) {
-      const uint32_t h0 = *reinterpret_cast<const uint32_t*>(p), h1 = *reinterpret_cast<const uint32_t*>(p + 4);
+      const uint2 hh = *reinterpret_cast<const uint2*>(p);
+      const uint32_t h0 = hh.x, h1 = hh.y;
       w = h0 & 0xFFFFu, d = (h0 >> 16) & 0xFFu, n = h0 >> 24, c = h1 & 0xFFFFu;
       uint2 v[4];
       uint32_t rs[4];
@@ -434,10 +447,16 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         const uint32_t ri = sub + 4 * k < n ? rowof(TIt, TI, v[k].x, x.dmask) : ROW_NONE;
         price[k] = ri != ROW_NONE ? rd(TIt, I_PRICE, ri) : 0;  // committed: every item exists
         const bool h = rs[k] != ROW_NONE;
-        sq[k] = h ? rd(TSt, S_QUANTITY, rs[k]) : 0;
-        sy[k] = h ? rd(TSt, S_YTD, rs[k]) : 0;
-        so[k] = h ? rd(TSt, S_ORDER_CNT, rs[k]) : 0;
-        sr[k] = h ? rd(TSt, S_REMOTE_CNT, rs[k]) : 0;
+        if (h && svec) {
+          const longlong2* sp = reinterpret_cast<const longlong2*>(col_ptr(TSt, S_QUANTITY, rs[k]));
+          const longlong2 a = sp[0], bq = sp[1];
+          sq[k] = a.x, sy[k] = a.y, so[k] = bq.x, sr[k] = bq.y;
+        } else {
+          sq[k] = h ? rd(TSt, S_QUANTITY, rs[k]) : 0;
+          sy[k] = h ? rd(TSt, S_YTD, rs[k]) : 0;
+          so[k] = h ? rd(TSt, S_ORDER_CNT, rs[k]) : 0;
+          sr[k] = h ? rd(TSt, S_REMOTE_CNT, rs[k]) : 0;
+        }
       }
       const long long o = b.res[4ull * r];
       const uint64_t okey = kO(w, d, (uint64_t)o);
@@ -456,7 +475,7 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         const uint32_t row_s = rs[k];
         if (row_s != ROW_NONE) {
           const long long q = sq[k];
-          wr(TSt, S_QUANTITY, row_s, q >= (long long)qty + 10 ? q - qty : q - qty + 91);
+          const long long nq = q >= (long long)qty + 10 ? q - qty : q - qty + 91;
           // the counters may be ADD columns (delayed mode), but only NewOrder touches STOCK and
           // every NewOrder writes the row's S_QUANTITY unit (WAW): this txn is the row's only
           // committed toucher in the batch (and its items are distinct, R10), so plain
@@ -464,9 +483,16 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
           const auto add = [](long long a, long long dv) {
             return (long long)((unsigned long long)a + (unsigned long long)dv);
           };
-          wr(TSt, S_YTD, row_s, add(sy[k], qty));
-          wr(TSt, S_ORDER_CNT, row_s, add(so[k], 1));
-          wr(TSt, S_REMOTE_CNT, row_s, add(sr[k], rem));
+          if (svec) {
+            longlong2* sp = reinterpret_cast<longlong2*>(col_ptr(TSt, S_QUANTITY, row_s));
+            sp[0] = make_longlong2(nq, add(sy[k], qty));
+            sp[1] = make_longlong2(add(so[k], 1), add(sr[k], rem));
+          } else {
+            wr(TSt, S_QUANTITY, row_s, nq);
+            wr(TSt, S_YTD, row_s, add(sy[k], qty));
+            wr(TSt, S_ORDER_CNT, row_s, add(so[k], 1));
+            wr(TSt, S_REMOTE_CNT, row_s, add(sr[k], rem));
+          }
         }
         const uint32_t row = (uint32_t)(ol0 + (pref >> 32) + l);  // ORDER_LINE row
         wr(TOL_, OL_I_ID, row, i);
@@ -664,15 +690,20 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
   const DevTable& TCu = c_tabs[TC];
   uint32_t* log = tp.log + (uint64_t)r * TLOG;
   if (PH == PH_DETECT && b.nparts <= 1) {  // unpartitioned detection: the logged rows suffice
-    col_upd<PH>(TWh, W_YTD, log[0], x, true);
-    col_upd<PH>(TDi, D_YTD, log[1], x, true);
-    col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, log[2], x);
+    const uint4 lg = *reinterpret_cast<const uint4*>(log);  // one 16-byte load (TLOG keeps rows aligned)
+    col_upd<PH>(TWh, W_YTD, lg.x, x, true);
+    col_upd<PH>(TDi, D_YTD, lg.y, x, true);
+    col_upd3<PH>(TCu, C_BALANCE, C_YTD_PAYMENT, C_PAYMENT_CNT, lg.z, x);
     return;
   }
+  // the parameter fields in two vector loads (one lane per Payment: field-by-field byte loads were
+  // 7 load instructions, each touching 32 different blocks)
   const uint8_t* p = b.params + 128ull * r;
-  const uint32_t w = p16(p, 0), d = p[2], by_name = p[3], cw = p16(p, 4), cd = p[6];
-  uint32_t cid = p16(p, 8);
-  const uint32_t clast = p16(p, 10);
+  const uint4 hv = *reinterpret_cast<const uint4*>(p);
+  const uint32_t w = hv.x & 0xFFFFu, d = (hv.x >> 16) & 0xFFu, by_name = hv.x >> 24, cw = hv.y & 0xFFFFu,
+                 cd = (hv.y >> 16) & 0xFFu;
+  uint32_t cid = hv.z & 0xFFFFu;
+  const uint32_t clast = hv.z >> 16;
   const long long amount = p64(p, 16);
   // partitioned (§8(e)): warehouse + district on the home partition, the customer (its
   // by-name lookup, result and HISTORY row) on the customer's owner
@@ -698,21 +729,17 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     if (cust) {
       row_c = cid ? rowof(TCu, TC, kC(cw, cd, cid), x.dmask) : ROW_NONE;
       if (row_c == ROW_NONE) { internal_error(x); return; }
-      long long* res = b.res + 4ull * r;
-      res[0] = cid;
-      res[1] = col_is_add(TCu, C_BALANCE) ? 0 : rd(TCu, C_BALANCE, row_c);  // pre-image (strict only)
-      res[2] = 0;
-      res[3] = 0;
+      longlong2* res = reinterpret_cast<longlong2*>(b.res + 4ull * r);
+      res[0] = make_longlong2(cid, col_is_add(TCu, C_BALANCE) ? 0 : rd(TCu, C_BALANCE, row_c));  // pre-image (strict only)
+      res[1] = make_longlong2(0, 0);
     }
-    log[0] = row_w;
-    log[1] = row_d;
-    log[2] = row_c;
-    log[3] = cid;
+    *reinterpret_cast<uint4*>(log) = make_uint4(row_w, row_d, row_c, cid);
   } else {
-    row_w = log[0];
-    row_d = log[1];
-    row_c = log[2];
-    cid = log[3];
+    const uint4 lg = *reinterpret_cast<const uint4*>(log);
+    row_w = lg.x;
+    row_d = lg.y;
+    row_c = lg.z;
+    cid = lg.w;
   }
   if (home) {
     col_upd<PH>(TWh, W_YTD, row_w, x, true);
@@ -817,7 +844,7 @@ __device__ void proc_orderstatus(const BatchDev& b, const TpccParams& tp, uint32
   uint32_t row_ol[4];
 #pragma unroll
   for (uint32_t k = 0; k < 4; ++k) {  // the lane's line rows: from ORDER.aux (contiguous) or probed
-    const uint32_t l = 4 * sub + k;
+    const uint32_t l = sub + 4 * k;  // the txn's 4 lanes: 4 consecutive lines per k
     row_ol[k] = ROW_NONE;
     if (!active || l >= cnt || l >= 15) continue;
     if (PH == PH_EXEC) {

@@ -504,6 +504,7 @@ void launch_compact(const uint32_t* flags, const uint32_t* offs, uint32_t n, uin
 void launch_scatter_col(long long* dst, uint32_t stride, const long long* src, uint64_t n, cudaStream_t s);
 void launch_committed_reads(const uint32_t* bits, uint32_t n, const long long* res, long long* out, uint32_t* pre,
                             cudaStream_t s);
+void launch_fill_tid(unsigned long long* tid, uint32_t n, unsigned long long t0, cudaStream_t s);
 void launch_carry(const unsigned long long* ptid, const uint8_t* ptype, const uint8_t* pparams, const uint32_t* abort,
                   uint32_t nc, unsigned long long* tid, uint8_t* type, uint8_t* params, cudaStream_t s);
 void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const uint8_t* types, uint32_t n,

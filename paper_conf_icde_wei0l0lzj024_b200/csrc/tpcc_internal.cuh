@@ -5,7 +5,8 @@
 namespace ltpg {
 
 constexpr int NTYPES = 5;
-constexpr int TLOG = 17;         // u32 row slots logged per txn by execute (NewOrder/Payment/OrderStatus)
+constexpr int TLOG = 20;         // u32 row slots logged per txn by execute (NewOrder 16, Payment 4,
+                                 // OrderStatus 17), padded to 80 B so every txn's log is 16-B aligned
 constexpr int NO_CHUNK = 1024;   // ranks per chunk of the o_id prefix computation
 
 // TPC-C schema (include/ltpg.h): table ids and column indices

@@ -104,3 +104,28 @@ def test_committed_reads_only(device_out):
         nc = int((st == 1).sum())
         assert (reads.reshape(-1)[:4 * nc].reshape(nc, 4) == res[st == 1]).all(), bno
     compare_tables(g, o)
+
+
+def test_tid_range_equals_explicit_tids():
+    """LTPG_BATCH_TID_RANGE: only the first TID crosses PCIe, the device fills the consecutive
+    rest; with carried aborts (LTPG_BATCH_CARRY_ABORTS) the carried txns keep their TIDs (HISTORY
+    rows store them) -- closed loop == the oracle on the host-composed batches."""
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=79, mode="strict", mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=2000, tables=tables, append_batches=5)
+    o = oracle.tpcc_db(wl, tables)
+    tid, prev = 100, None
+    for bno in range(4):
+        nc = g.pending_aborts() if prev is not None else 0
+        fresh = wl.batch(2000 - nc, tid, bno)
+        packed, offs = lib.pack_params_compact(fresh["type"], fresh["params"])
+        inp = {"tid": fresh["tid"][:1].copy(), "type": fresh["type"], "params": packed, "offsets": offs,
+               "compact": True, "tid_range": True}
+        out = g.run_tpcc(inp, 2 + bno, carry=prev is not None, n_txns=len(fresh["type"]))
+        tid += len(fresh["tid"])
+        batch = fresh if prev is None else {k: np.concatenate([prev[k][prev_ab], fresh[k]]) for k in fresh}
+        rc, st, res = o.run_tpcc(batch, 2 + bno)
+        assert rc == 0 and (out["status"] == st).all() and (out["reads"] == res).all(), bno
+        prev, prev_ab = batch, np.nonzero(st == ST_CONFLICT)[0]
+    compare_tables(g, o)
