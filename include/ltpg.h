@@ -143,7 +143,15 @@ enum { LTPG_ST_CONFLICT = 0, LTPG_ST_COMMIT = 1, LTPG_ST_USER_ABORT = 2 };
 #define LTPG_FLAG_GRAPH         (1u << 6)  /* run each batch's device work as a captured CUDA graph,
                                               replayed for later batches of the same shape
                                               (see ltpg_run_batch); result-identical          */
+#define LTPG_FLAG_L2_PERSIST_MARKS (1u << 7) /* keep the largest conflict-mark array L2-resident
+                                              across batches: an L2 access-policy window
+                                              (persisting set-aside sized from the device's L2)
+                                              on the batch stream; result-identical            */
 #define LTPG_FLAG_LOOPBACK_SHIFT 8         /* bits 8..11: logical partitions on one GPU   */
+#define LTPG_FLAG_NO_SINGLE_LAUNCH (1u << 12) /* A/B: small single-partition OPS batches (<= 16384
+                                              txns) normally run a2..a8 as ONE cooperative
+                                              kernel with grid-wide barriers between the stages;
+                                              this flag keeps them on the multi-kernel path     */
 
 typedef struct {
   int device;                   /* CUDA device ordinal                                  */

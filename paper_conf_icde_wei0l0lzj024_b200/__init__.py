@@ -36,6 +36,8 @@ LTPG_FLAG_REORDER = 1 << 2
 LTPG_FLAG_UNFUSED = 1 << 3
 LTPG_FLAG_LARGE_BUCKETS = 1 << 5
 LTPG_FLAG_GRAPH = 1 << 6
+LTPG_FLAG_L2_PERSIST_MARKS = 1 << 7
+LTPG_FLAG_NO_SINGLE_LAUNCH = 1 << 12
 LTPG_PEER_HANDLE_BYTES = 128
 LTPG_PARAM_BYTES = 128
 LTPG_LAYOUT_ROWBLOCK, LTPG_LAYOUT_COLUMNAR = 0, 1

@@ -127,6 +127,9 @@ struct ltpg_db {
   uint16_t* d_su = nullptr;                  // [MAXT] NEXT-3: this batch's bucket size per table
   uint32_t* d_wprefix = nullptr;             // LTPG_RESULT_COMMITTED_READS: commits before each bitmask word
   uint32_t* d_coop = nullptr;                // [4096] per-block partial sums of cooperative kernels
+  // LTPG_FLAG_L2_PERSIST_MARKS: the largest mark array (base, bytes) under an L2 persisting window
+  void* persist_base = nullptr;
+  size_t persist_bytes = 0;
   std::vector<Part> parts;
   void** d_ptrs = nullptr;                 // [3 * 64] partition pointer tables
   uint32_t* d_scan = nullptr;
@@ -463,6 +466,10 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
   CK(cudaSetDevice(db->device));
   CK(cudaDeviceSynchronize());
   DevTable& T = db->h_tab[t];
+  if (T.wmarks && T.wmarks == db->persist_base) {  // its marks go away: no window over freed memory
+    db->persist_base = nullptr;
+    db->persist_bytes = 0;
+  }
   free_table(T);
   const uint64_t cap = std::max<uint64_t>(d->capacity_rows, 1);
   T.n_cols = d->n_cols;
@@ -523,6 +530,10 @@ int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t 
       if (d->col_is_add[c] && d->col_group[c] != LTPG_STATIC) T.add_groups |= 1u << d->col_group[c];
     CK(dmalloc(&T.wmarks, cap * d->n_groups));
     CK(cudaMemset(T.wmarks, 0xFF, cap * d->n_groups * sizeof(mark_t)));
+    if ((db->cfg.flags & LTPG_FLAG_L2_PERSIST_MARKS) && cap * d->n_groups * sizeof(mark_t) > db->persist_bytes) {
+      db->persist_base = T.wmarks;  // (a table reloaded later keeps the old pointer: refreshed below)
+      db->persist_bytes = cap * d->n_groups * sizeof(mark_t);
+    }
     if (const uint32_t na = __builtin_popcount(T.add_groups)) {
       CK(dmalloc(&T.amarks, cap * na));
       CK(cudaMemset(T.amarks, 0xFF, cap * na * sizeof(mark_t)));
@@ -826,6 +837,30 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     upload_tables_tpcc(db->d_tab, s);
     g_uploaded[db->device % 64] = db->tab_version;
   }
+  if ((db->cfg.flags & LTPG_FLAG_L2_PERSIST_MARKS) && db->persist_base) {
+    // the largest mark array under a persisting L2 window (the set-aside is sized once from the
+    // device's L2; accesses beyond the hit ratio stream)
+    static size_t setaside = 0;
+    if (!setaside) {
+      int l2 = 0, maxw = 0;
+      cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, db->device);
+      cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxPersistingL2CacheSize, db->device);
+      setaside = std::min<size_t>((size_t)maxw, std::min<size_t>(db->persist_bytes, (size_t)l2 / 2));
+      if (setaside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside);
+    }
+    int maxwin = 0;
+    cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, db->device);
+    cudaStreamAttrValue av{};
+    av.accessPolicyWindow.base_ptr = db->persist_base;
+    av.accessPolicyWindow.num_bytes = std::min<size_t>(db->persist_bytes, (size_t)maxwin);
+    av.accessPolicyWindow.hitRatio =
+        setaside ? std::min(1.0f, (float)setaside / (float)av.accessPolicyWindow.num_bytes) : 0.0f;
+    av.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    av.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &av);
+    cudaStreamSetAttribute(db->cap, cudaStreamAttributeAccessPolicyWindow, &av);
+    cudaGetLastError();
+  }
   if (db->epoch / 255 != db->mark_window) {  // the epoch tag byte wraps 0 -> 254: clear every mark
     db->mark_window = db->epoch / 255;
     for (uint32_t t = 0; t < db->n_tables; ++t) {
@@ -890,8 +925,31 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   auto tmark = [](cudaEvent_t e, cudaStream_t st) { return record_stage(e, st); };
 
   // ---- the batch's device work (a2..a8), enqueued on `s` -- or captured into a graph ---------
+  // small single-partition OPS batches: a2..a8 in one cooperative launch (k_ops_small)
+  const bool small = ops_mode && fused && L == 1 && !partitioned && !db->p2p && n && n <= ops_small_max_txns() &&
+                     !(db->cfg.flags & (LTPG_FLAG_LARGE_BUCKETS | LTPG_FLAG_NO_SINGLE_LAUNCH));
   auto enqueue = [&](cudaStream_t s) -> int {
     static_assert(MAXT <= 32, "k_batch_init clears the reservations with one warp");
+    if (small) {
+      if (tid_range) launch_fill_tid(S.d_tid + nc, nf, tid0, s);
+      if (nc) {
+        const Slot& P = db->slots[db->carry_slot];
+        launch_carry(P.eff_tid, P.eff_ptype, P.eff_params, P.eff_abort, nc, S.d_tid, S.d_ptype, S.d_params, s);
+        CK(cudaEventRecord(db->slots[db->carry_slot].comp_done, s));
+      }
+      const bool timed = timing || capturing;
+      if (timed) CK(tmark(S.ev[1], s));
+      BatchDev& x = pb[0];
+      x.status = st_out;
+      launch_ops_small(db->n_tables, x, filter, db->d_coop, db->d_reserve, S.d_vars,
+                       capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock, bits_out, counts, abort_out,
+                       S.d_small + 16, S.host_out ? nullptr : res->n_aborted, s);
+      if (timed)  // one kernel: ms_group holds the whole batch
+        for (int e = 2; e <= 5; ++e) CK(tmark(S.ev[e], s));
+      if (cr) launch_committed_reads(bits_out, n, res_out, cr_dst, db->d_wprefix, s);
+      CK(cudaGetLastError());
+      return LTPG_OK;
+    }
     const uint32_t ib = std::min<uint32_t>(148u * 4u, std::max<uint32_t>(1u, (n / 16 + 255) / 256));
     k_batch_init<<<ib, 256, 0, s>>>(db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch,
                                     b->batch_clock, db->parts[0].small, db->parts[0].ua, n,

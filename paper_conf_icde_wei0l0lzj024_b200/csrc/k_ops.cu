@@ -357,10 +357,10 @@ __global__ void __launch_bounds__(256) k_ops_exec(BatchDev b, bool filter) { ops
 // the warp-division effect without the global lists' round trip through HBM.  INSERTs go
 // to the INSERT list (K-claim, then K-exec on that list); reads of keys absent from the
 // index carry UREF_RECHECK so K-detect finds claims made after this kernel.
-__global__ void __launch_bounds__(256) k_ops_fused(uint32_t n_tables, BatchDev b, bool filter) {
-  constexpr uint32_t STAGE = 320;  // YCSB: 32 txns x 10 ops; larger warps run unstaged
-  __shared__ __align__(16) ltpg_op stage[8][STAGE];
-  __shared__ uint16_t perm[8][STAGE];  // staged op index | lane << 9, ordered by kind
+constexpr uint32_t FUSED_STAGE = 320;  // YCSB: 32 txns x 10 ops; larger warps run unstaged
+__device__ __forceinline__ void ops_fused_body(uint32_t n_tables, const BatchDev& b, bool filter,
+                                               ltpg_op (*stage)[FUSED_STAGE], uint16_t (*perm)[FUSED_STAGE]) {
+  constexpr uint32_t STAGE = FUSED_STAGE;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t wib = threadIdx.x >> 5;
@@ -453,6 +453,11 @@ __global__ void __launch_bounds__(256) k_ops_fused(uint32_t n_tables, BatchDev b
     exec_one(b, w0 + li, r0 + (e >> 9), o, filter, dmask, true);
   }
 }
+__global__ void __launch_bounds__(256) k_ops_fused(uint32_t n_tables, BatchDev b, bool filter) {
+  __shared__ __align__(16) ltpg_op stage[8][FUSED_STAGE];
+  __shared__ uint16_t perm[8][FUSED_STAGE];  // staged op index | lane << 9, ordered by kind
+  ops_fused_body(n_tables, b, filter, stage, perm);
+}
 
 void launch_ops_fused(uint32_t n_tables, const BatchDev& b, bool filter, cudaStream_t s) {
   k_ops_fused<<<(b.n_txns + 255) / 256, 256, 0, s>>>(n_tables, b, filter);
@@ -469,9 +474,8 @@ void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s) {
 // base -> index claims -> execution of the INSERT list.  A batch without INSERTs (YCSB A/B/C, the
 // common case) leaves after one load of the insert-table mask -- instead of the six dependent
 // launches (3-kernel scan, capacity, claim, exec) it paid before.
-__global__ void __launch_bounds__(256) k_ops_insert_tail(uint32_t n_tables, BatchDev b, bool filter,
-                                                         uint32_t* partials) {
-  cg::grid_group grid = cg::this_grid();
+__device__ __forceinline__ void ops_insert_tail_body(uint32_t n_tables, const BatchDev& b, bool filter,
+                                                     uint32_t* partials, cg::grid_group& grid) {
   const uint32_t n = b.n_txns;
   if (*(volatile uint32_t*)b.ins_tables == 0) {  // uniform: written by the previous kernel
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -536,6 +540,11 @@ __global__ void __launch_bounds__(256) k_ops_insert_tail(uint32_t n_tables, Batc
   grid.sync();
   ops_exec_body<true>(b, filter);  // only the INSERT list is populated
 }
+__global__ void __launch_bounds__(256) k_ops_insert_tail(uint32_t n_tables, BatchDev b, bool filter,
+                                                         uint32_t* partials) {
+  cg::grid_group grid = cg::this_grid();
+  ops_insert_tail_body(n_tables, b, filter, partials, grid);
+}
 
 void launch_ops_insert_tail(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials, cudaStream_t s) {
   static int per_sm = 0, sms = 0;
@@ -572,12 +581,9 @@ void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t 
 // PART: partitioned -- only this partition's ops / keys are checked and the verdict goes
 // to lflag (conflict*2 | user_abort) for the exchange; otherwise it is final (status).
 template <bool PART>
-__global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
-  if (*b.err) return;
+__device__ __forceinline__ void ops_detect_txn(const BatchDev& b, uint32_t r) {
   const uint32_t dmask = *b.dense_live & ~*b.insdel;
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= b.n_txns) return;
   const uint32_t b0 = b.op_begin[r], b1 = b.op_begin[r + 1];
   uint32_t bits = 0;
   for (uint32_t i = b0; i < b1 && !conflict_of(bits, reorder); ++i) {
@@ -618,6 +624,12 @@ __global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
   const uint32_t flag = bits | (b.ua[r] ? CF_UA : 0u);
   if (PART) b.lflag[r] = (uint8_t)flag;
   else b.status[r] = status_of_bits(flag, reorder);
+}
+template <bool PART>
+__global__ void __launch_bounds__(256) k_ops_detect(BatchDev b) {
+  if (*b.err) return;
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < b.n_txns) ops_detect_txn<PART>(b, r);
 }
 
 void launch_ops_detect(const BatchDev& b, cudaStream_t s) {
@@ -695,6 +707,139 @@ void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cu
     k_ops_writeback<true><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b, n_tables);
   else
     k_ops_writeback<false><<<(b.n_txns + 255) / 256, 256, 0, s>>>(b, n_tables);
+  note_launch();
+}
+
+
+// ---- small batches: the whole a2..a8 pipeline in ONE cooperative launch ------------------
+// A batch of a few thousand txns runs each stage in a few microseconds, so the per-kernel launch
+// gaps of the stream (batch init, fused front end, INSERT tail, detect, finalize, write-back) were
+// most of its latency.  Here the stages are separated by grid-wide barriers instead: init ->
+// execute + marks (k_ops_fused's body) -> INSERT tail -> RAW/WAW test -> {a8 in block 0, a7 in
+// every block} -> cursor advance.  Same bodies as the multi-kernel path, hence result-identical.
+// Single partition only (no exchange), no large-sized buckets (their fold is its own pass).
+struct SmallOut {
+  unsigned long long* reserve;  // [MAXT] append reservations (cleared here)
+  BatchVars* vars;              // written here from (epoch, clock) or the slot's mapped host copy
+  const volatile BatchVars* host;
+  uint32_t epoch;
+  long long clock;
+  uint32_t* commit_bits;        // a8 outputs (as k_finalize_compact)
+  uint32_t* counts;             // [3] commit / conflict / user-abort (zeroed by the host)
+  uint32_t* abort_out;
+  uint32_t* n_out;
+  uint32_t* n_out2;             // or null
+};
+
+// a8 for n txns in one block: 32 txns per thread-word, block-wide scan of the conflict counts
+// per 256-word round (carried), abort list in ascending rank order
+__device__ __forceinline__ void finalize_block(const uint8_t* __restrict__ status, uint32_t n, const SmallOut& o) {
+  __shared__ uint32_t fw[8], fcarry, fred[3];
+  const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (threadIdx.x == 0) fcarry = 0;
+  if (threadIdx.x < 3) fred[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t nw = (n + 31) / 32;
+  for (uint32_t base = 0; base < nw; base += blockDim.x) {
+    const uint32_t w = base + threadIdx.x;
+    uint32_t cm = 0, am = 0, nu = 0;
+    if (w < nw) {
+      const uint32_t r0 = w * 32, m = min(32u, n - r0);
+#pragma unroll 8
+      for (uint32_t j = 0; j < m; ++j) {
+        const uint8_t st = status[r0 + j];
+        cm |= (st == LTPG_ST_COMMIT ? 1u : 0u) << j;
+        am |= (st == LTPG_ST_CONFLICT ? 1u : 0u) << j;
+        nu += st == LTPG_ST_USER_ABORT;
+      }
+      o.commit_bits[w] = cm;
+    }
+    const uint32_t na = __popc(am);
+    uint32_t x = na;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+      if (lane >= (uint32_t)d) x += y;
+    }
+    const uint32_t nbw = __reduce_add_sync(0xffffffffu, __popc(cm)), nuw = __reduce_add_sync(0xffffffffu, nu);
+    if (lane == 31) fw[wid] = x;
+    if (lane == 0) {
+      atomicAdd(fred + 0, nbw);
+      atomicAdd(fred + 2, nuw);
+    }
+    __syncthreads();
+    uint32_t before = fcarry, round = 0;
+#pragma unroll
+    for (uint32_t q = 0; q < 8; ++q) {
+      if (q < wid) before += fw[q];
+      round += fw[q];
+    }
+    uint32_t pos = before + x - na;
+    for (uint32_t m = am; m; m &= m - 1) o.abort_out[pos++] = w * 32 + (__ffs(m) - 1);
+    __syncthreads();
+    if (threadIdx.x == 0) fcarry += round;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    atomicAdd(o.counts + 0, fred[0]);
+    atomicAdd(o.counts + 1, fcarry);
+    atomicAdd(o.counts + 2, fred[2]);
+    *o.n_out = fcarry;
+    if (o.n_out2) *o.n_out2 = fcarry;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_ops_small(uint32_t n_tables, BatchDev b, bool filter, uint32_t* partials,
+                                                   SmallOut o) {
+  __shared__ __align__(16) ltpg_op stage[8][FUSED_STAGE];
+  __shared__ uint16_t perm[8][FUSED_STAGE];
+  cg::grid_group grid = cg::this_grid();
+  const uint32_t n = b.n_txns;
+  const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
+  // init (k_batch_init's work).  The batch scalars are read with ld.global.nc (b_epoch) after the
+  // barrier below: no SM has cached their line in this launch before it was written here.
+  if (blockIdx.x == 0) {
+    if (threadIdx.x < MAXT) o.reserve[threadIdx.x] = 0;
+    if (threadIdx.x < 16) b.err[threadIdx.x] = 0;  // the partition's small words (err .. done)
+    if (threadIdx.x == 0) {
+      o.vars->epoch = o.host ? o.host->epoch : o.epoch;
+      o.vars->clock = o.host ? o.host->clock : o.clock;
+    }
+  }
+  for (uint32_t i = gt; i < n; i += gs) b.ua[i] = 0;
+  __threadfence();
+  grid.sync();
+  ops_fused_body(n_tables, b, filter, stage, perm);  // a1 + warp division + a4/a5
+  grid.sync();
+  ops_insert_tail_body(n_tables, b, filter, partials, grid);  // no INSERT: returns at once
+  grid.sync();
+  const bool ok = *(volatile uint32_t*)b.err == 0;  // uniform after the barrier
+  if (ok)
+    for (uint32_t r = gt; r < n; r += gs) ops_detect_txn<false>(b, r);  // a6: status is final
+  grid.sync();
+  if (blockIdx.x == 0) finalize_block(b.status, n, o);  // a8 (reads status only)
+  if (ok)
+    for (uint32_t r = gt; r < n; r += gs) ops_writeback_txn(b, r);  // a7
+  grid.sync();
+  if (gt == 0 && !*(volatile uint32_t*)b.err) {  // cursors past this batch's reservations
+    for (uint32_t t = 0; t < n_tables; ++t) *c_tabs[t].n_rows += o.reserve[t];
+    *b.dense_live &= ~*b.insdel;
+  }
+}
+
+uint32_t ops_small_max_txns() { return 16384; }
+
+void launch_ops_small(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials,
+                      unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host, uint32_t epoch,
+                      long long clock, uint32_t* commit_bits, uint32_t* counts, uint32_t* abort_out,
+                      uint32_t* n_out, uint32_t* n_out2, cudaStream_t s) {
+  uint32_t nt = n_tables;
+  BatchDev bb = b;
+  bool f = filter;
+  SmallOut so{reserve, vars, host, epoch, clock, commit_bits, counts, abort_out, n_out, n_out2};
+  void* args[] = {&nt, &bb, &f, &partials, &so};
+  const uint32_t grid = std::max<uint32_t>(1, (b.n_txns + 255) / 256);  // <= 64 blocks: co-resident
+  cudaLaunchCooperativeKernel((const void*)k_ops_small, dim3(grid), dim3(256), args, 0, s);
   note_launch();
 }
 

@@ -342,3 +342,22 @@ def test_header_validation_every_type(ptype, off, val):
     assert e.value.rc == lib.LTPG_EINVAL
     compare_tables(g, o)
     compare(g, o, wl.batch(1000, 5000, 1), 3)
+
+
+def test_l2_persist_marks_result_identical():
+    """LTPG_FLAG_L2_PERSIST_MARKS (an L2 persisting window over the largest mark array) is a
+    cache hint only: a closed loop with it == oracle."""
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=37, mode="strict", mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=3000, tables=tables, append_batches=4, flags=lib.LTPG_FLAG_L2_PERSIST_MARKS)
+    o = oracle.tpcc_db(wl, tables)
+    pending, tid = None, 1
+    for bno in range(3):
+        fresh = wl.batch(3000 - (0 if pending is None else len(pending["tid"])), tid, bno)
+        tid += len(fresh["tid"])
+        batch = fresh if pending is None else {k: np.concatenate([pending[k], fresh[k]]) for k in fresh}
+        st = compare(g, o, batch, 2 + bno)
+        ab = np.nonzero(st == ST_CONFLICT)[0]
+        pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
+    compare_tables(g, o)

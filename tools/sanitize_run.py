@@ -45,7 +45,49 @@ def tpcc_c2(batches=2, mode="strict", flags=0):
     print("tpcc_c2 (%s, flags %d) ok" % (mode, flags))
 
 
-def multirank():
+def ycsb_e(batches=3):
+    """YCSB-E: INSERTs (the cooperative insert tail) and SCANs."""
+    import oracle
+    import paper_conf_icde_wei0l0lzj024_b200 as ltpg
+    from workloads.ycsb import ycsb_letter
+    wl = ycsb_letter("E", 20_000, seed=5)
+    g = ltpg.ycsb_database(wl, max_txns=2048, max_ops=20480, capacity=20_000 + 20480 * batches)
+    o = oracle.ycsb_db(wl)
+    for b in range(batches):
+        batch = wl.batch(2048, 1 + 2048 * b, b)
+        out = g.run_ops(batch)
+        rc, st, rd = o.run_ops(batch)
+        assert rc == 0 and (out["status"] == st).all() and (out["reads"] == rd).all()
+    print("ycsb_e ok")
+
+
+def carry(batches=3):
+    """TPC-C closed loop with the aborts carried on the device, consecutive TIDs, committed
+    result slots written into pinned host memory by the kernel."""
+    import oracle
+    import paper_conf_icde_wei0l0lzj024_b200 as ltpg
+    from workloads import tpcc
+    wl = tpcc.TpccWorkload(1, seed=3, mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = ltpg.tpcc_database(wl, max_txns=2048, tables=tables, append_batches=batches + 1)
+    o = oracle.tpcc_db(wl, tables)
+    tid, prev = 1, None
+    for b in range(batches):
+        nc = g.pending_aborts() if prev is not None else 0
+        fresh = wl.batch(2048 - nc, tid, b)
+        packed, offs = ltpg.pack_params_compact(fresh["type"], fresh["params"])
+        inp = {"tid": fresh["tid"][:1].copy(), "type": fresh["type"], "params": packed, "offsets": offs,
+               "compact": True, "tid_range": True}
+        out = g.run_tpcc(inp, 2 + b, carry=prev is not None, n_txns=len(fresh["type"]), committed_reads=True)
+        batch = fresh if prev is None else {k: np.concatenate([prev[k][pab], fresh[k]]) for k in fresh}
+        rc, st, res = o.run_tpcc(batch, 2 + b)
+        assert rc == 0 and (out["status"] == st).all() and (out["reads"] == res[st == 1]).all()
+        tid += len(fresh["tid"])
+        prev, pab = batch, np.nonzero(st == 0)[0]
+    print("carry ok")
+
+
+def multirank(sharded=False):
     import torch
     import torch.distributed as dist
     import oracle
@@ -60,9 +102,15 @@ def multirank():
     o = oracle.tpcc_db(wl, tables)
     for b in range(2):
         batch = wl.batch(2048, 1 + 2048 * b, b)
-        out = g.run_tpcc(batch, 2 + b)
         rc, st, res = o.run_tpcc(batch, 2 + b)
-        assert rc == 0 and (out["status"] == st).all() and (out["reads"] == res).all()
+        assert rc == 0
+        if sharded:  # this rank's shard only (route_tpcc): its statuses == the oracle's
+            shard = ltpg.route_tpcc(batch, wl.W, world, rank)
+            out = g.run_tpcc(shard, 2 + b)
+            assert (out["status"] == st[shard["grank"]]).all()
+        else:
+            out = g.run_tpcc(batch, 2 + b)
+            assert (out["status"] == st).all() and (out["reads"] == res).all()
     dist.barrier()
     g.close()
     dist.barrier()
@@ -74,5 +122,7 @@ if __name__ == "__main__":
     if what == "tpcc_c2":
         tpcc_c2()
         tpcc_c2(mode="delayed", flags=4)  # + NEXT-1 reordering
+    elif what == "multirank_sharded":
+        multirank(sharded=True)
     else:
         globals()[what]()
