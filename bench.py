@@ -637,8 +637,12 @@ def main():
         i = (args.warmup + s) % n_distinct
         flush.fill_(s & 0xFF)  # evict L2 between steps (outside the timed events)
         ev[s][0].record(stream)
-        out = run(dev_batches[i], host_batches[i], clock, True, False)
+        # submitted asynchronously and completed after the end event: the event pair brackets the
+        # batch's device work (its last node is the result publish), not the host's wake-up from
+        # the completion wait
+        pend = run(dev_batches[i], host_batches[i], clock, True, False, wait=False)
         ev[s][1].record(stream)
+        out = pend.wait()
         clock += 1
         n_s = len(host_batches[i]["tid"])
         if sharded:  # the commits of the txns this rank is home of (summed over ranks below)
@@ -710,8 +714,9 @@ def main():
             flush.fill_(s_ & 0xFF)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            outc = run(bd, cur, clock, True, False)
+            pend = run(bd, cur, clock, True, False, wait=False)
             e1.record(stream)
+            outc = pend.wait()
             clock += 1
             torch.cuda.synchronize()
             c_ms += e0.elapsed_time(e1)

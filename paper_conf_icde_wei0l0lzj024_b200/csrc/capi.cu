@@ -28,7 +28,10 @@ uint64_t g_uploaded[64] = {0};   // per device: version whose tables sit in __co
 // per device: recorded after every batch's device work (any db).  A db that re-uploads the
 // constant bank (another db's tables were there) first waits on it, so the kernels of the
 // previous owner -- possibly still running on another stream -- never see the new tables.
-cudaEvent_t g_const_users[64] = {nullptr};
+// the completion event (a slot's comp_done) of the last batch that ran with this device's
+// constant bank, and its db: a db uploading other tables waits for it.  Not owned.
+cudaEvent_t g_const_last[64] = {nullptr};
+const void* g_const_owner[64] = {nullptr};
 
 // per-partition scratch (one per logical partition handled by this process)
 struct Part {
@@ -49,6 +52,7 @@ struct Part {
 // (epoch, clock), which the graph copies from the slot's pinned host copy when it runs.
 struct GraphKey {
   uint32_t mode, n, n_ops, bflags, host_out, reads_dev, inputs_dev, packed;
+  uint32_t small_w0, pad;  // single-launch kernel writes its result word 0 (no index catch-up ahead)
   uint64_t tab_version;
   const void* in[7];   // tid, op_begin, ops, args, ptype, params, offsets (device inputs only)
   const void* out[5];  // status, bits, abort, n_aborted, reads
@@ -83,6 +87,7 @@ struct Slot {
   uint32_t* h_small_dev = nullptr;         // its device-side address (written by k_publish)
   cudaEvent_t ev[8]{};
   cudaEvent_t h2d_done = nullptr, comp_done = nullptr, out_done = nullptr;
+  cudaEvent_t out_ev = nullptr;  // the batch's last event: out_done, or comp_done when nothing follows it
   bool pending = false, timing = false, host_out = false, empty = false;
   ltpg_result* res = nullptr;
   uint64_t launches0 = 0;
@@ -146,7 +151,6 @@ struct ltpg_db {
   cudaStream_t cap = nullptr;              // batch graphs are captured here (never executes work)
   // batches execute in submission order even when the caller passes different streams:
   // each batch's first kernel waits on the previous batch's compute (they share scratch)
-  cudaEvent_t last_comp = nullptr;
   uint64_t graph_uses = 0;
   // a8 (commit bitmask, abort list) runs on its own stream once the verdicts are final,
   // concurrently with write-back; it has its own scan scratch
@@ -337,9 +341,10 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(cudaHostAlloc(reinterpret_cast<void**>(&S.h_small), 64 * sizeof(uint32_t), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S.h_small_dev), S.h_small, 0));
     for (auto& e : S.ev) CK(cudaEventCreate(&e));
-    CK(cudaEventCreate(&S.h2d_done));
-    CK(cudaEventCreate(&S.comp_done));
-    CK(cudaEventCreate(&S.out_done));
+    CK(cudaEventCreateWithFlags(&S.h2d_done, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&S.comp_done, cudaEventDisableTiming));
+    CK(cudaEventCreate(&S.out_done));  // (timed: ltpg_stats.ms_download)
+    S.out_ev = S.out_done;
     CK(dmalloc(&S.d_vars, 1));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&S.h_vars), sizeof(BatchVars), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S.h_vars_dev), S.h_vars, 0));
@@ -352,8 +357,6 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
   CK(cudaStreamCreateWithFlags(&db->cap, cudaStreamNonBlocking));
   CK(cudaEventCreateWithFlags(&db->status_ready, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&db->fin_done, cudaEventDisableTiming));
-  CK(cudaEventCreateWithFlags(&db->last_comp, cudaEventDisableTiming));
-  if (!g_const_users[cfg->device % 64]) CK(cudaEventCreateWithFlags(&g_const_users[cfg->device % 64], cudaEventDisableTiming));
   CK(dmalloc(&db->d_scan_fin, scan_scratch_words(n) + 16));
   CK(dmalloc(&db->d_fc_state, (n + 1023) / 1024 + 1));
   CK(cudaMemset(db->d_fc_state, 0, ((n + 1023) / 1024 + 1) * sizeof(unsigned long long)));
@@ -368,9 +371,10 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&P.items, m * NKINDS));
     CK(dmalloc(&P.txn_ins, n + 1));
     CK(dmalloc(&P.ua, n));
-    CK(dmalloc(&P.lflag, n));
+    CK(dmalloc(&P.lflag, n + 4));  // (k_ops_small ORs verdict bytes as 32-bit words)
     CK(dmalloc(&P.pmask, n));
-    CK(dmalloc(&P.small, 64));
+    CK(dmalloc(&P.small, 64));  // [0, 16) the partition's words; [16, 64) per-slot sets (k_ops_small)
+    CK(cudaMemset(P.small, 0, 64 * sizeof(uint32_t)));
     CK(dmalloc(&P.base, MAXT));
     int rc = tpcc_alloc(P.tpcc, cfg->max_txns, cfg->n_warehouses, p ? db->parts[0].tpcc.by_name : nullptr);
     if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
@@ -425,7 +429,10 @@ void ltpg_destroy_db(ltpg_db* db) {
   if (db->cap) cudaStreamDestroy(db->cap);
   if (db->status_ready) cudaEventDestroy(db->status_ready);
   if (db->fin_done) cudaEventDestroy(db->fin_done);
-  if (db->last_comp) cudaEventDestroy(db->last_comp);
+  if (g_const_owner[db->device % 64] == db) {  // (cudaFree below synchronizes the device)
+    g_const_last[db->device % 64] = nullptr;
+    g_const_owner[db->device % 64] = nullptr;
+  }
   if (db->d_scan_fin) cudaFree(db->d_scan_fin);
   if (db->d_fc_state) cudaFree(db->d_fc_state);
   if (db->d_fc_ctr) cudaFree(db->d_fc_ctr);
@@ -635,7 +642,7 @@ namespace {
 int finish_slot(ltpg_db* db, Slot& S) {
   S.pending = false;
   db->carry_ok = false;
-  CK(cudaEventSynchronize(S.out_done));
+  CK(cudaEventSynchronize(S.out_ev));
   const uint32_t err = S.h_small[0];
   if (err & ERR_EINTERNAL) return fail(db, LTPG_EINTERNAL, "device invariant violated");
   if (err & ERR_EINVAL) return fail(db, LTPG_EINVAL, "invalid batch (validated on device; nothing changed)");
@@ -746,6 +753,12 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool timing = res->stats != nullptr;
   const bool partitioned = db->nparts > 1;
   const uint32_t L = db->loopback;
+  const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
+  // small single-partition OPS batches: a1..a8 in one cooperative launch (k_ops_small), with the
+  // slot's own set of partition small words (published and cleared by the kernel's last block)
+  const bool small = ops_mode && grouped && L == 1 && !partitioned && !db->p2p && n && n <= ops_small_max_txns() &&
+                     !(db->cfg.flags & (LTPG_FLAG_LARGE_BUCKETS | LTPG_FLAG_NO_SINGLE_LAUNCH));
+  uint32_t* small_words = small ? db->parts[0].small + 16 * (1 + (&S - db->slots)) : nullptr;
   S.timing = timing;
   S.res = res;
   S.host_out = !res->outputs_on_device;
@@ -815,10 +828,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   }
   // kernels of this batch: after its upload, after the slot's previous outputs were read and
   // after the previous batch's compute (it may have run on another stream)
-  CK(cudaStreamWaitEvent(s, S.out_done, 0));
-  if (db->submitted > 1) CK(cudaStreamWaitEvent(s, db->last_comp, 0));
+  CK(cudaStreamWaitEvent(s, S.out_ev, 0));
+  if (db->submitted > 1) CK(cudaStreamWaitEvent(s, db->slots[(db->submitted - 2) % 3].comp_done, 0));
   if (timing) CK(cudaEventRecord(S.ev[0], s));
-  CK(cudaMemsetAsync(S.d_small, 0, 17 * sizeof(uint32_t), s));
+  // the slot's result words; the single-launch kernel writes them itself (word 0 too unless an
+  // index catch-up below may raise an error in it first)
+  const bool idx_catchup = db->idx_lag && (ops_mode || !db->olrow_ready);
+  if (!small || idx_catchup) CK(cudaMemsetAsync(S.d_small, 0, 17 * sizeof(uint32_t), s));
   if (!n && !S.host_out) CK(cudaMemsetAsync(res->n_aborted, 0, sizeof(uint32_t), s));
   if (!b->inputs_on_device) CK(cudaStreamWaitEvent(s, S.h2d_done, 0));
   const bool packed_params = !ops_mode && b->proc_offsets;
@@ -831,7 +847,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   // table metadata -> __constant__ (stream-ordered D2D; every TU holds its own copy);
   // skipped when this device's constant bank already holds this db's current tables
   if (g_uploaded[db->device % 64] != db->tab_version) {
-    CK(cudaStreamWaitEvent(s, g_const_users[db->device % 64], 0));  // the previous owner's kernels
+    if (g_const_last[db->device % 64])  // the previous owner's kernels
+      CK(cudaStreamWaitEvent(s, g_const_last[db->device % 64], 0));
     upload_tables_common(db->d_tab, s);
     upload_tables_ops(db->d_tab, s);
     upload_tables_tpcc(db->d_tab, s);
@@ -876,7 +893,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         if (T.sub[k]) CK(cudaMemsetAsync(T.sub[k], 0xFF, su_units[k] * T.su * sizeof(mark_t), s));
     }
   }
-  if (db->idx_lag && (ops_mode || !db->olrow_ready)) {  // key lookups ahead: catch the indexes up
+  if (idx_catchup) {  // key lookups ahead: catch the indexes up
     for (uint32_t t = 0; t < db->n_tables; ++t)
       if ((db->idx_lag >> t) & 1u) launch_build_index_tail(t, db->d_idx_from + t, S.d_small, s);
     db->idx_lag = 0;
@@ -889,7 +906,6 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     launch_note_rows(LTPG_T_ORDER_LINE, db->d_idx_from + LTPG_T_ORDER_LINE, s);  // first unindexed row
     db->idx_lag |= 1u << LTPG_T_ORDER_LINE;
   }
-  const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
   const bool filter = !(db->cfg.flags & LTPG_FLAG_NO_MARK_FILTER);
   const bool reorder = (db->cfg.flags & LTPG_FLAG_REORDER) != 0;
   // fused OPS front end; NEXT-1 needs min reader marks on claimed keys, so it keeps the lists
@@ -909,12 +925,13 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     x.txn_ins = P.txn_ins;
     x.ua = P.ua;
     x.lflag = P.lflag;
-    x.err = P.small + 0;
-    x.ins_tables = P.small + 1;
-    x.kcount = P.small + 2;
+    uint32_t* w = small ? small_words : P.small;
+    x.err = w + 0;
+    x.ins_tables = w + 1;
+    x.kcount = w + 2;
     x.base = P.base;
-    x.insdel = P.small + 12;
-    x.done = P.small + 14;
+    x.insdel = w + 12;
+    x.done = w + 14;
   }
   S.h_vars->epoch = db->epoch;  // the slot's previous batch (the copy's last reader) is complete
   S.h_vars->clock = b->batch_clock;
@@ -925,9 +942,6 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   auto tmark = [](cudaEvent_t e, cudaStream_t st) { return record_stage(e, st); };
 
   // ---- the batch's device work (a2..a8), enqueued on `s` -- or captured into a graph ---------
-  // small single-partition OPS batches: a2..a8 in one cooperative launch (k_ops_small)
-  const bool small = ops_mode && fused && L == 1 && !partitioned && !db->p2p && n && n <= ops_small_max_txns() &&
-                     !(db->cfg.flags & (LTPG_FLAG_LARGE_BUCKETS | LTPG_FLAG_NO_SINGLE_LAUNCH));
   auto enqueue = [&](cudaStream_t s) -> int {
     static_assert(MAXT <= 32, "k_batch_init clears the reservations with one warp");
     if (small) {
@@ -942,8 +956,8 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
       BatchDev& x = pb[0];
       x.status = st_out;
       launch_ops_small(db->n_tables, x, filter, db->d_coop, db->d_reserve, S.d_vars,
-                       capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock, bits_out, counts, abort_out,
-                       S.d_small + 16, S.host_out ? nullptr : res->n_aborted, s);
+                       capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock, bits_out, S.d_small,
+                       !idx_catchup, abort_out, S.host_out ? nullptr : res->n_aborted, S.h_small_dev, s);
       if (timed)  // one kernel: ms_group holds the whole batch
         for (int e = 2; e <= 5; ++e) CK(tmark(S.ev[e], s));
       if (cr) launch_committed_reads(bits_out, n, res_out, cr_dst, db->d_wprefix, s);
@@ -1087,6 +1101,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     k.mode = b->mode, k.n = n, k.n_ops = bd.n_ops, k.bflags = b->flags & LTPG_BATCH_COMPACT_PARAMS;
     k.host_out = S.host_out, k.reads_dev = reads_dev, k.inputs_dev = b->inputs_on_device != 0;
     k.packed = packed_params;
+    k.small_w0 = small && !idx_catchup;
     k.tab_version = db->tab_version;
     if (b->inputs_on_device) {
       const void* in[7] = {b->tid, b->op_begin, b->ops, b->op_arg, b->proc_type, b->proc_params, b->proc_offsets};
@@ -1136,17 +1151,19 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     if (rc) return rc;
   }
   if (timing) CK(cudaEventRecord(S.ev[6], s));
-  CK(cudaEventRecord(S.comp_done, s));
-  CK(cudaEventRecord(db->last_comp, s));
-  CK(cudaEventRecord(g_const_users[db->device % 64], s));
+  CK(cudaEventRecord(S.comp_done, s));  // (also the next batch's "previous compute" and the constants' last user)
+  g_const_last[db->device % 64] = S.comp_done;
+  g_const_owner[db->device % 64] = db;
   // ---- a8: results: D2H on the copy stream (overlaps the next batch's kernels) ------------------
   cudaStream_t os = S.host_out ? db->d2h : s;
   if (S.host_out) CK(cudaStreamWaitEvent(db->d2h, S.comp_done, 0));
   const cudaMemcpyKind out_kind = S.host_out ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
   // error word, counters and abort count: one tiny kernel stores them into mapped host memory
   // (cheaper than a D2H copy in stream order); device outputs were written in place
-  k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17, L == 1 ? db->parts[0].small : nullptr);
-  note_launch();
+  if (!small) {  // (the single-launch kernel's last block publishes them itself)
+    k_publish<<<1, 32, 0, os>>>(S.d_small, S.h_small_dev, 17, L == 1 ? db->parts[0].small : nullptr);
+    note_launch();
+  }
   if (n && S.host_out) {
     if (res->status) CK(cudaMemcpyAsync(res->status, S.d_status, n, out_kind, os));
     CK(cudaMemcpyAsync(res->commit_bits, S.d_bits, ((n + 31) / 32) * sizeof(uint32_t), out_kind, os));
@@ -1156,7 +1173,10 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   } else if (n && res->reads && !reads_dev && !cr) {
     CK(cudaMemcpyAsync(res->reads, res_out, n_reads * sizeof(int64_t), out_kind, os));
   }
-  CK(cudaEventRecord(S.out_done, os));
+  // nothing after comp_done (single launch, device outputs, no statistics): it is the last event
+  const bool tail = !small || S.host_out || timing || (n && res->reads && !reads_dev && !cr);
+  S.out_ev = tail ? S.out_done : S.comp_done;
+  if (tail) CK(cudaEventRecord(S.out_done, os));
   if (timing) res->stats->n_kernels = (uint32_t)(g_kernel_launches - S.launches0);
   S.eff_tid = bd.tid;
   S.eff_ptype = bd.ptype;

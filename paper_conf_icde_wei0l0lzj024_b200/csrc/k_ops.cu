@@ -10,6 +10,7 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <cstdio>
 
 #include "ltpg_internal.cuh"
 
@@ -116,12 +117,16 @@ __device__ __forceinline__ ltpg_op unpack_op(ulonglong2 v) {
 }
 
 // ---- K-group: validation + decomposition into per-kind lists (one thread per txn) ----
+constexpr uint32_t GROUP_STAGE = 352;  // ops per warp staged in shared memory (YCSB: 32 x 10 = 320)
 template <bool GROUPED>
-__global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
-                                                            BatchDev b) {
-  constexpr uint32_t STAGE = 352;  // ops per warp staged in shared memory (YCSB: 32 x 10 = 320)
-  __shared__ __align__(16) ltpg_op stage[8][STAGE];
+__device__ __forceinline__ void ops_validate_group_body(uint32_t n_tables, const BatchDev& b,
+                                                        ltpg_op (*stage)[GROUP_STAGE]) {
+  constexpr uint32_t STAGE = GROUP_STAGE;
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < b.n_txns) {  // validation's scalar loads, in flight while the op records are staged
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(b.tid + r));
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(b.op_begin + r));
+  }
   const int lane = threadIdx.x & 31;
   const uint32_t wib = threadIdx.x >> 5;
   bool bad = false;
@@ -174,7 +179,7 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
   block_reserve<NKINDS>(ck, b.kcount, pos);
   if (r < b.n_txns && !bad)
     for (uint32_t i = b0; i < b1; ++i) {
-      const ltpg_op o = load_op(b.ops, i);
+      const ltpg_op o = get(i);
       if (!op_touches(b, o)) continue;
       const uint8_t k = o.kind;
       uint32_t p = 0;
@@ -183,6 +188,11 @@ __global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables,
         if (kk == k) p = pos[kk]++;
       b.items[(uint64_t)k * b.max_ops + p] = (unsigned long long)i | ((unsigned long long)r << 32);
     }
+}
+template <bool GROUPED>
+__global__ void __launch_bounds__(256) k_ops_validate_group(uint32_t n_tables, BatchDev b) {
+  __shared__ __align__(16) ltpg_op stage[8][GROUP_STAGE];
+  ops_validate_group_body<GROUPED>(n_tables, b, stage);
 }
 
 void launch_ops_validate_group(uint32_t n_tables, const BatchDev& b, bool grouped,
@@ -474,8 +484,10 @@ void launch_ops_exec_inserts(const BatchDev& b, bool filter, cudaStream_t s) {
 // base -> index claims -> execution of the INSERT list.  A batch without INSERTs (YCSB A/B/C, the
 // common case) leaves after one load of the insert-table mask -- instead of the six dependent
 // launches (3-kernel scan, capacity, claim, exec) it paid before.
+// run_exec = false: ends after the claims' grid barrier (when there are INSERTs) -- the caller
+// executes every kind list itself
 __device__ __forceinline__ void ops_insert_tail_body(uint32_t n_tables, const BatchDev& b, bool filter,
-                                                     uint32_t* partials, cg::grid_group& grid) {
+                                                     uint32_t* partials, cg::grid_group& grid, bool run_exec = true) {
   const uint32_t n = b.n_txns;
   if (*(volatile uint32_t*)b.ins_tables == 0) {  // uniform: written by the previous kernel
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -538,7 +550,7 @@ __device__ __forceinline__ void ops_insert_tail_body(uint32_t n_tables, const Ba
   grid.sync();
   ops_claim_body(b);
   grid.sync();
-  ops_exec_body<true>(b, filter);  // only the INSERT list is populated
+  if (run_exec) ops_exec_body<true>(b, filter);  // (fused front end: only the INSERT list is populated)
 }
 __global__ void __launch_bounds__(256) k_ops_insert_tail(uint32_t n_tables, BatchDev b, bool filter,
                                                          uint32_t* partials) {
@@ -580,6 +592,43 @@ void launch_ops_exec(const BatchDev& b, bool grouped, bool filter, cudaStream_t 
 // ---- K-detect: per txn, OR of the unit tests over its ops ------------------------------
 // PART: partitioned -- only this partition's ops / keys are checked and the verdict goes
 // to lflag (conflict*2 | user_abort) for the exchange; otherwise it is final (status).
+// the RAW/WAW(/WAR) bits of op i of txn r (PART: only this partition's keys of a SCAN)
+template <bool PART>
+__device__ __forceinline__ uint32_t ops_detect_op(const BatchDev& b, uint32_t i, uint32_t r, uint32_t dmask) {
+  const uint64_t u = b.uref[i];
+  const uint64_t chk = u >> 62;
+  if (chk == CHK_NONE) return 0;
+  const uint32_t t = (u >> 40) & 0xFF;
+  const DevTable& T = c_tabs[t];
+  uint32_t bits = 0;
+  if (chk == CHK_SCAN) {  // phantom-safe: every key of the range is a read (R8)
+    const ltpg_op o = load_op(b.ops, i);
+    if (!T.n_groups) return 0;
+    const uint32_t gs = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
+    for (uint64_t k = o.key; k < o.key + o.aux && !(bits & CF_RAW); ++k) {
+      if (PART && !owns_key(b, T, k)) continue;
+      uint32_t row, claim;
+      lookup(T, t, dmask, k, row, claim);
+      if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b_epoch(b));
+      else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b));
+    }
+    return bits;
+  }
+  if (u & UREF_RECHECK) {  // absent at execution (fused path): an INSERT may have claimed it since
+    const ltpg_op o = load_op(b.ops, i);
+    uint32_t row, claim;
+    lookup(T, t, dmask, o.key, row, claim);
+    return claim != ROW_NONE ? unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b)) : 0u;
+  }
+  const uint32_t row = (uint32_t)u;
+  const uint32_t acc = chk == CHK_A ? ACC_ADD : (((u >> 59) & 1) ? ACC_WRITE : ACC_READ);
+  if ((u >> 61) & 1) {
+    for (uint32_t g = 0; g < T.n_groups; ++g) bits |= unit_bits(T, g, row, acc, r, b_epoch(b));
+  } else {
+    bits |= unit_bits(T, (u >> 32) & 0xFF, row, acc, r, b_epoch(b));
+  }
+  return bits;
+}
 template <bool PART>
 __device__ __forceinline__ void ops_detect_txn(const BatchDev& b, uint32_t r) {
   const uint32_t dmask = *b.dense_live & ~*b.insdel;
@@ -588,38 +637,7 @@ __device__ __forceinline__ void ops_detect_txn(const BatchDev& b, uint32_t r) {
   uint32_t bits = 0;
   for (uint32_t i = b0; i < b1 && !conflict_of(bits, reorder); ++i) {
     if (PART && !op_touches(b, load_op(b.ops, i))) continue;
-    const uint64_t u = b.uref[i];
-    const uint64_t chk = u >> 62;
-    if (chk == CHK_NONE) continue;
-    const uint32_t t = (u >> 40) & 0xFF;
-    const DevTable& T = c_tabs[t];
-    if (chk == CHK_SCAN) {  // phantom-safe: every key of the range is a read (R8)
-      const ltpg_op o = load_op(b.ops, i);
-      if (!T.n_groups) continue;
-      const uint32_t gs = (o.col != LTPG_COL_COUNT && col_group(T, o.col) != LTPG_STATIC) ? col_group(T, o.col) : 0;
-      for (uint64_t k = o.key; k < o.key + o.aux && !(bits & CF_RAW); ++k) {
-        if (PART && !owns_key(b, T, k)) continue;
-        uint32_t row, claim;
-        lookup(T, t, dmask, k, row, claim);
-        if (row != ROW_NONE) bits |= unit_bits(T, gs, row, ACC_READ, r, b_epoch(b));
-        else if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b));
-      }
-      continue;
-    }
-    if (u & UREF_RECHECK) {  // absent at execution (fused path): an INSERT may have claimed it since
-      const ltpg_op o = load_op(b.ops, i);
-      uint32_t row, claim;
-      lookup(T, t, dmask, o.key, row, claim);
-      if (claim != ROW_NONE) bits |= unit_bits(T, 0, claim, ACC_READ, r, b_epoch(b));
-      continue;
-    }
-    const uint32_t row = (uint32_t)u;
-    const uint32_t acc = chk == CHK_A ? ACC_ADD : (((u >> 59) & 1) ? ACC_WRITE : ACC_READ);
-    if ((u >> 61) & 1) {
-      for (uint32_t g = 0; g < T.n_groups; ++g) bits |= unit_bits(T, g, row, acc, r, b_epoch(b));
-    } else {
-      bits |= unit_bits(T, (u >> 32) & 0xFF, row, acc, r, b_epoch(b));
-    }
+    bits |= ops_detect_op<PART>(b, i, r, dmask);
   }
   const uint32_t flag = bits | (b.ua[r] ? CF_UA : 0u);
   if (PART) b.lflag[r] = (uint8_t)flag;
@@ -641,6 +659,54 @@ void launch_ops_detect(const BatchDev& b, cudaStream_t s) {
 }
 
 // ---- K-wb: apply committed write sets; every INSERT releases its claim ----------------
+// op i (of a committed txn, or an INSERT of any txn: its claim is released).  The ops of one txn
+// touch distinct keys (R10), so they may be applied in any order and by different threads.
+// EAGER: the result slot and argument are loaded together with the uref (one round trip instead
+// of two on the latency-bound small path; the large-batch path loads them only for UPDATE / ADD)
+template <bool EAGER = false>
+__device__ __forceinline__ void ops_writeback_op(const BatchDev& b, uint32_t i, const ltpg_op& o, bool commit) {
+  const uint64_t u = b.uref[i];
+  long long rv = 0, av = 0;
+  if (EAGER) rv = b.res[i], av = b.args[i];
+  if ((u >> 62) == CHK_NONE || (u >> 62) == CHK_SCAN) return;
+  const bool present = (u >> 60) & 1;
+  const uint32_t row = (uint32_t)u;
+  const DevTable& T = c_tabs[o.table];
+  if (o.kind == LTPG_INSERT) {
+    if (present) return;  // duplicate-key user abort: nothing claimed
+    IdxSlot* sl = idx_slot(T, o.key);
+    if (!sl) { atomicOr(b.err, ERR_EINTERNAL); return; }
+    if (commit) {
+      const long long arg = EAGER ? av : b.args[i];
+      for (uint32_t c = 0; c < T.n_cols; ++c)
+        *col_ptr_ops(T, c, row) = (long long)((unsigned long long)arg + c);
+      T.rowkey[row] = o.key;
+      T.valid[row] = 1;
+      sl->row = row;
+    }
+    sl->claim = ROW_NONE;
+    return;
+  }
+  if (!present) return;
+  switch (o.kind) {
+    case LTPG_UPDATE:
+      *col_ptr_ops(T, o.col, row) = (long long)((unsigned long long)(EAGER ? rv : b.res[i]) +
+                                                (unsigned long long)(EAGER ? av : b.args[i]));
+      break;
+    case LTPG_ADD:  // delayed update: commutative, order-free and exact
+      atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr_ops(T, o.col, row)),
+                (unsigned long long)(EAGER ? av : b.args[i]));
+      break;
+    case LTPG_DELETE: {
+      T.valid[row] = 0;
+      IdxSlot* sl = idx_slot(T, o.key);
+      if (sl) sl->row = ROW_NONE;
+      break;
+    }
+    default:
+      break;
+  }
+}
 __device__ __forceinline__ void ops_writeback_txn(const BatchDev& b, uint32_t r) {
   const bool commit = b.status[r] == LTPG_ST_COMMIT;  // final verdict (after the exchange)
   if (!commit && b.txn_ins[r + 1] == b.txn_ins[r]) return;  // aborted, no claims to release
@@ -649,43 +715,7 @@ __device__ __forceinline__ void ops_writeback_txn(const BatchDev& b, uint32_t r)
     const ltpg_op o = load_op(b.ops, i);
     if (!commit && o.kind != LTPG_INSERT) continue;
     if (!op_touches(b, o)) continue;  // another partition's op: its uref is not ours
-    const uint64_t u = b.uref[i];
-    if ((u >> 62) == CHK_NONE || (u >> 62) == CHK_SCAN) continue;
-    const bool present = (u >> 60) & 1;
-    const uint32_t row = (uint32_t)u;
-    const DevTable& T = c_tabs[o.table];
-    if (o.kind == LTPG_INSERT) {
-      if (present) continue;  // duplicate-key user abort: nothing claimed
-      IdxSlot* sl = idx_slot(T, o.key);
-      if (!sl) { atomicOr(b.err, ERR_EINTERNAL); continue; }
-      if (commit) {
-        const long long arg = b.args[i];
-        for (uint32_t c = 0; c < T.n_cols; ++c)
-          *col_ptr_ops(T, c, row) = (long long)((unsigned long long)arg + c);
-        T.rowkey[row] = o.key;
-        T.valid[row] = 1;
-        sl->row = row;
-      }
-      sl->claim = ROW_NONE;
-      continue;
-    }
-    if (!present) continue;
-    switch (o.kind) {
-      case LTPG_UPDATE:
-        *col_ptr_ops(T, o.col, row) = (long long)((unsigned long long)b.res[i] + (unsigned long long)b.args[i]);
-        break;
-      case LTPG_ADD:  // delayed update: commutative, order-free and exact
-        atomicAdd(reinterpret_cast<unsigned long long*>(col_ptr_ops(T, o.col, row)), (unsigned long long)b.args[i]);
-        break;
-      case LTPG_DELETE: {
-        T.valid[row] = 0;
-        IdxSlot* sl = idx_slot(T, o.key);
-        if (sl) sl->row = ROW_NONE;
-        break;
-      }
-      default:
-        break;
-    }
+    ops_writeback_op(b, i, o, commit);
   }
 }
 // ADV (single-partition batches): the grid's last block also advances the append cursors past
@@ -711,13 +741,25 @@ void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cu
 }
 
 
-// ---- small batches: the whole a2..a8 pipeline in ONE cooperative launch ------------------
-// A batch of a few thousand txns runs each stage in a few microseconds, so the per-kernel launch
-// gaps of the stream (batch init, fused front end, INSERT tail, detect, finalize, write-back) were
-// most of its latency.  Here the stages are separated by grid-wide barriers instead: init ->
-// execute + marks (k_ops_fused's body) -> INSERT tail -> RAW/WAW test -> {a8 in block 0, a7 in
-// every block} -> cursor advance.  Same bodies as the multi-kernel path, hence result-identical.
+// ---- small batches: the whole a1..a8 pipeline in ONE cooperative launch ------------------
+// A batch of a few thousand txns runs each stage in a few microseconds, so per-kernel launch
+// gaps were most of its latency, and one thread per txn left each thread a serial chain of its
+// ops' dependent loads.  Here the stages are separated by grid-wide barriers and the op-level
+// stages run one thread per op (from the per-kind lists), so a stage costs about one dependent
+// memory round trip:
+//   a1 validate + per-kind lists (K-group; + the batch's clears) -> INSERT tail (scan, capacity,
+//   K-claim; only with INSERTs) -> a4/a5 execute every list (K-exec) -> a6 per-op RAW/WAW(/WAR)
+//   bits, OR-ed into the txn's verdict byte -> {a6 status + a7 per op + cursor advance; a8 in
+//   the grid's last block}.
+// Same per-op code as the multi-kernel unfused path (the verdict is the OR of the ops' bits:
+// conflict_of / status_of_bits are monotone in the bits), hence result-identical.  A thread
+// keeps its op (list entry + record) in registers across the op stages when the grid covers
+// every op.  The partition's small words (error, counters) are a per-slot set that the batch's
+// result publish (k_publish) reads and clears, so they need no clearing barrier here.
 // Single partition only (no exchange), no large-sized buckets (their fold is its own pass).
+#ifdef LTPG_SMALL_TS
+__device__ unsigned long long g_small_we[8];  // per phase: the latest end of a thread's work
+#endif
 struct SmallOut {
   unsigned long long* reserve;  // [MAXT] append reservations (cleared here)
   BatchVars* vars;              // written here from (epoch, clock) or the slot's mapped host copy
@@ -725,15 +767,17 @@ struct SmallOut {
   uint32_t epoch;
   long long clock;
   uint32_t* commit_bits;        // a8 outputs (as k_finalize_compact)
-  uint32_t* counts;             // [3] commit / conflict / user-abort (zeroed by the host)
+  uint32_t* dsmall;             // the slot's words: [0] err (written iff write0) [8..10] counts [16] n
   uint32_t* abort_out;
-  uint32_t* n_out;
   uint32_t* n_out2;             // or null
+  volatile uint32_t* host_small;  // the slot's mapped host words: [0..16] of dsmall, err ORed into [0]
+  bool write0;
 };
 
 // a8 for n txns in one block: 32 txns per thread-word, block-wide scan of the conflict counts
-// per 256-word round (carried), abort list in ascending rank order
-__device__ __forceinline__ void finalize_block(const uint8_t* __restrict__ status, uint32_t n, const SmallOut& o) {
+// per 256-word round (carried), abort list in ascending rank order.  st_of(r) = txn r's status.
+template <class St>
+__device__ __forceinline__ void finalize_block(uint32_t n, const SmallOut& o, St st_of) {
   __shared__ uint32_t fw[8], fcarry, fred[3];
   const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   if (threadIdx.x == 0) fcarry = 0;
@@ -747,7 +791,7 @@ __device__ __forceinline__ void finalize_block(const uint8_t* __restrict__ statu
       const uint32_t r0 = w * 32, m = min(32u, n - r0);
 #pragma unroll 8
       for (uint32_t j = 0; j < m; ++j) {
-        const uint8_t st = status[r0 + j];
+        const uint8_t st = st_of(r0 + j);
         cm |= (st == LTPG_ST_COMMIT ? 1u : 0u) << j;
         am |= (st == LTPG_ST_CONFLICT ? 1u : 0u) << j;
         nu += st == LTPG_ST_USER_ABORT;
@@ -780,65 +824,232 @@ __device__ __forceinline__ void finalize_block(const uint8_t* __restrict__ statu
     if (threadIdx.x == 0) fcarry += round;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    atomicAdd(o.counts + 0, fred[0]);
-    atomicAdd(o.counts + 1, fcarry);
-    atomicAdd(o.counts + 2, fred[2]);
-    *o.n_out = fcarry;
-    if (o.n_out2) *o.n_out2 = fcarry;
+  if (threadIdx.x < 17) {  // the slot's result words (the host memset of them is skipped)
+    const uint32_t t = threadIdx.x;
+    const uint32_t v = t == 8 ? fred[0] : t == 9 ? fcarry : t == 10 ? fred[2] : t == 16 ? fcarry : 0u;
+    if (t || o.write0) o.dsmall[t] = v;
   }
+  if (threadIdx.x == 0 && o.n_out2) *o.n_out2 = fcarry;
+}
+
+__device__ __forceinline__ void prefetch_l2(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
+
+// Grid-wide barrier of a co-resident grid on a counter that is zero at launch: barrier k waits
+// for k * gridDim.x arrivals (one release-add per block, acquire polling by thread 0).  About
+// half the cost of cg::grid_group::sync on B200 (tools/launchcost.cu).
+__device__ __forceinline__ void grid_barrier(uint32_t* ctr, uint32_t k) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
+    const uint32_t target = k * gridDim.x;
+    uint32_t v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+    } while (v < target);
+  }
+  __syncthreads();
+}
+
+// Warm-up by the blocks that hold no txns during K-group: read the op records (so K-group's
+// staging loads find them in L2) and fetch every point op's row word, write mark (or index
+// home slot) and argument into L2 for the op stages that follow.  Loads and prefetches only.
+__device__ __forceinline__ void small_warm(const BatchDev& b, uint32_t t0, uint32_t nt) {
+  const uint32_t live = *b.dense_live;
+  for (uint32_t i = t0; i < b.n_ops; i += nt) {
+    const ltpg_op o = load_op(b.ops, i);
+    if (o.table >= MAXT || o.kind == LTPG_SCAN) continue;
+    const DevTable& T = c_tabs[o.table];
+    if (!T.defined) continue;
+    if (o.kind != LTPG_SELECT) prefetch_l2(b.args + i);
+    if (o.kind == LTPG_INSERT) continue;
+    if (((live >> o.table) & 1u) && o.key - T.key_base < T.dense_n) {
+      const uint32_t row = (uint32_t)(o.key - T.key_base);
+      if (o.col < T.n_cols) prefetch_l2(col_ptr_ops(T, o.col, row));
+      if (T.wmarks) {
+        const uint32_t g = o.col < T.n_cols && col_group(T, o.col) != LTPG_STATIC ? col_group(T, o.col) : 0;
+        prefetch_l2(wmark_ptr(T, g < T.n_groups ? g : 0, row));
+      }
+    } else if (T.idx) {
+      prefetch_l2(T.idx + idx_hash(o.key, T.idx_shift));
+    }
+  }
+}
+
+// the p-th entry of the concatenated per-kind lists (kinds in order)
+__device__ __forceinline__ unsigned long long list_entry(const BatchDev& b, uint32_t p, const uint32_t (&cnt)[NKINDS]) {
+  uint32_t k = 0;
+#pragma unroll
+  for (int kk = 0; kk < NKINDS - 1; ++kk)
+    if (k == (uint32_t)kk && p >= cnt[kk]) { p -= cnt[kk]; k = kk + 1; }
+  return b.items[(uint64_t)k * b.max_ops + p];
 }
 
 __global__ void __launch_bounds__(256) k_ops_small(uint32_t n_tables, BatchDev b, bool filter, uint32_t* partials,
                                                    SmallOut o) {
-  __shared__ __align__(16) ltpg_op stage[8][FUSED_STAGE];
-  __shared__ uint16_t perm[8][FUSED_STAGE];
-  cg::grid_group grid = cg::this_grid();
+  __shared__ __align__(16) ltpg_op stage[8][GROUP_STAGE];
+  cg::grid_group grid = cg::this_grid();  // (the INSERT tail's barriers)
+  uint32_t* bar = b.err + 15;  // a free partition word: zero at launch, cleared by the last block
   const uint32_t n = b.n_txns;
-  const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
-  // init (k_batch_init's work).  The batch scalars are read with ld.global.nc (b_epoch) after the
-  // barrier below: no SM has cached their line in this launch before it was written here.
+  const bool fin_block = blockIdx.x == gridDim.x - 1;  // a8 only; no op work
+  const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = (gridDim.x - 1) * blockDim.x;
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
+#ifdef LTPG_SMALL_TS  // phase timestamps (diagnostic builds only): printed by thread 0
+  unsigned long long ts[8];
+  int nts = 0;
+#define SMALL_TS() \
+  if (gt == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ts[nts++]))
+#define WORK_END(k)                                                    \
+  {                                                                    \
+    __syncthreads();                                                   \
+    unsigned long long t_;                                             \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));             \
+    if (threadIdx.x == 0) atomicMax(g_small_we + (k), t_);             \
+  }
+#else
+#define SMALL_TS()
+#define WORK_END(k)
+#endif
+  SMALL_TS();
+  WORK_END(7);  // the last block's start
+  // a1 + per-kind lists, one thread per txn (blocks [0, ceil(n/256)) cover the batch), and the
+  // batch's clears for the later stages: reservations, batch scalars (read with ld.global.nc by
+  // b_epoch after the barrier below -- no SM cached their line in this launch before), user-abort
+  // flags, verdict bytes
   if (blockIdx.x == 0) {
     if (threadIdx.x < MAXT) o.reserve[threadIdx.x] = 0;
-    if (threadIdx.x < 16) b.err[threadIdx.x] = 0;  // the partition's small words (err .. done)
     if (threadIdx.x == 0) {
       o.vars->epoch = o.host ? o.host->epoch : o.epoch;
       o.vars->clock = o.host ? o.host->clock : o.clock;
     }
   }
-  for (uint32_t i = gt; i < n; i += gs) b.ua[i] = 0;
-  __threadfence();
-  grid.sync();
-  ops_fused_body(n_tables, b, filter, stage, perm);  // a1 + warp division + a4/a5
-  grid.sync();
-  ops_insert_tail_body(n_tables, b, filter, partials, grid);  // no INSERT: returns at once
-  grid.sync();
-  const bool ok = *(volatile uint32_t*)b.err == 0;  // uniform after the barrier
-  if (ok)
-    for (uint32_t r = gt; r < n; r += gs) ops_detect_txn<false>(b, r);  // a6: status is final
-  grid.sync();
-  if (blockIdx.x == 0) finalize_block(b.status, n, o);  // a8 (reads status only)
-  if (ok)
-    for (uint32_t r = gt; r < n; r += gs) ops_writeback_txn(b, r);  // a7
-  grid.sync();
-  if (gt == 0 && !*(volatile uint32_t*)b.err) {  // cursors past this batch's reservations
-    for (uint32_t t = 0; t < n_tables; ++t) *c_tabs[t].n_rows += o.reserve[t];
-    *b.dense_live &= ~*b.insdel;
+  if (gt < n) b.ua[gt] = 0;
+  if (gt < (n + 3) / 4) reinterpret_cast<uint32_t*>(b.lflag)[gt] = 0;
+  const uint32_t txn_blocks = (n + blockDim.x - 1) / blockDim.x;
+#ifndef LTPG_SMALL_NO_WARM
+  if (blockIdx.x >= txn_blocks)
+    small_warm(b, (blockIdx.x - txn_blocks) * blockDim.x + threadIdx.x, (gridDim.x - txn_blocks) * blockDim.x);
+#endif
+  ops_validate_group_body<true>(n_tables, b, stage);
+  WORK_END(0);
+  grid_barrier(bar, 1);
+  SMALL_TS();
+  ops_insert_tail_body(n_tables, b, filter, partials, grid, false);  // INSERTs: scan, capacity, claims
+  SMALL_TS();
+  uint32_t cnt[NKINDS], total = 0;
+#pragma unroll
+  for (int k = 0; k < NKINDS; ++k) total += (cnt[k] = *(volatile uint32_t*)(b.kcount + k));
+  const bool ok = *(volatile uint32_t*)b.err == 0;  // uniform: raised before the last barrier
+  const uint32_t dmask = *b.dense_live & ~*b.insdel;
+  const bool one = total <= gs;  // every op has its own thread: keep it in registers
+  unsigned long long it1 = 0;
+  ltpg_op op1{};
+  if (ok && !fin_block) {  // a4/a5: one thread per op
+    if (one) {
+      if (gt < total) {
+        it1 = list_entry(b, gt, cnt);
+        op1 = load_op(b.ops, (uint32_t)it1);
+        exec_one(b, (uint32_t)it1, (uint32_t)(it1 >> 32), op1, filter, dmask);
+      }
+    } else {
+      for (uint32_t p = gt; p < total; p += gs) {
+        const unsigned long long it = list_entry(b, p, cnt);
+        exec_one(b, (uint32_t)it, (uint32_t)(it >> 32), load_op(b.ops, (uint32_t)it), filter, dmask);
+      }
+    }
   }
+  WORK_END(2);
+  grid_barrier(bar, 2);
+  SMALL_TS();
+  if (ok && !fin_block)  // a6: one thread per op, OR into the txn's byte
+    for (uint32_t p = gt; p < total; p += gs) {
+      const unsigned long long it = one ? it1 : list_entry(b, p, cnt);
+      const uint32_t r = (uint32_t)(it >> 32);
+      const uint32_t bits = ops_detect_op<false>(b, (uint32_t)it, r, dmask);
+      if (bits) atomicOr(reinterpret_cast<uint32_t*>(b.lflag) + (r >> 2), bits << (8 * (r & 3)));
+    }
+  WORK_END(3);
+  grid_barrier(bar, 3);
+  SMALL_TS();
+  auto st_of = [&](uint32_t r) { return status_of_bits(b.lflag[r] | (b.ua[r] ? CF_UA : 0u), reorder); };
+  if (fin_block) {
+    if (ok) finalize_block(n, o, st_of);  // a8
+  } else if (ok) {
+    for (uint32_t p = gt; p < total; p += gs) {  // a7: one thread per op
+      const unsigned long long it = one ? it1 : list_entry(b, p, cnt);
+      const uint32_t oi = (uint32_t)it;
+      const ltpg_op op = one ? op1 : load_op(b.ops, oi);
+      const bool commit = st_of((uint32_t)(it >> 32)) == LTPG_ST_COMMIT;
+      if (commit || op.kind == LTPG_INSERT) ops_writeback_op<true>(b, oi, op, commit);
+    }
+    for (uint32_t r = gt; r < n; r += gs) b.status[r] = st_of(r);
+    // cursors past this batch's reservations (nothing of a7 reads them; an error raised by a7
+    // is internal and poisons the db)
+    if (gt == 0) {
+      for (uint32_t t = 0; t < n_tables; ++t)
+        if (o.reserve[t]) *c_tabs[t].n_rows += o.reserve[t];
+      if (*b.insdel) *b.dense_live &= ~*b.insdel;
+    }
+  }
+  WORK_END(fin_block ? 5 : 4);
+  if (!ok && fin_block && threadIdx.x < 17 && (threadIdx.x || o.write0))
+    o.dsmall[threadIdx.x] = 0;  // failed batch (the error is in the partition's word): no counts
+  // the last block to finish publishes the result words into the slot's mapped host words (what
+  // k_publish does after the multi-kernel path) and clears the partition words for the slot's
+  // next batch (which is stream-ordered after this kernel)
+  __shared__ bool last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(b.done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last) {
+    __threadfence();
+    if (threadIdx.x < 17)
+      o.host_small[threadIdx.x] = reinterpret_cast<volatile uint32_t*>(o.dsmall)[threadIdx.x] |
+                                  (threadIdx.x == 0 ? *reinterpret_cast<volatile uint32_t*>(b.err) : 0u);
+    __syncthreads();
+    if (threadIdx.x < 16) b.err[threadIdx.x] = 0;  // err .. done, barrier counter
+  }
+#ifdef LTPG_SMALL_TS
+  SMALL_TS();
+  if (gt == 0) {
+    volatile unsigned long long* we = g_small_we;
+    printf("k_ops_small n=%u ops=%u grid=%u ns: group %llu ins %llu exec %llu detect %llu fin+wb %llu | "
+           "last block start +%lld | work: group %lld exec %lld detect %lld wb %lld fin %lld\n", n, total,
+           gridDim.x, ts[1] - ts[0], ts[2] - ts[1], ts[3] - ts[2], ts[4] - ts[3], ts[5] - ts[4],
+           (long long)(we[7] - ts[0]), (long long)(we[0] - ts[0]), (long long)(we[2] - ts[2]),
+           (long long)(we[3] - ts[3]), (long long)(we[4] - ts[4]), (long long)(we[5] - ts[4]));
+    for (int k = 0; k < 8; ++k) we[k] = 0;
+  }
+#endif
+#undef SMALL_TS
+#undef WORK_END
 }
 
 uint32_t ops_small_max_txns() { return 16384; }
 
 void launch_ops_small(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials,
                       unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host, uint32_t epoch,
-                      long long clock, uint32_t* commit_bits, uint32_t* counts, uint32_t* abort_out,
-                      uint32_t* n_out, uint32_t* n_out2, cudaStream_t s) {
+                      long long clock, uint32_t* commit_bits, uint32_t* dsmall, bool write0, uint32_t* abort_out,
+                      uint32_t* n_out2, volatile uint32_t* host_small, cudaStream_t s) {
+  static int per_sm = 0, sms = 0;
+  if (!per_sm) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_ops_small, 256, 0) != cudaSuccess || per_sm < 1)
+      per_sm = 1;
+  }
   uint32_t nt = n_tables;
   BatchDev bb = b;
   bool f = filter;
-  SmallOut so{reserve, vars, host, epoch, clock, commit_bits, counts, abort_out, n_out, n_out2};
+  SmallOut so{reserve, vars, host, epoch, clock, commit_bits, dsmall, abort_out, n_out2, host_small, write0};
   void* args[] = {&nt, &bb, &f, &partials, &so};
-  const uint32_t grid = std::max<uint32_t>(1, (b.n_txns + 255) / 256);  // <= 64 blocks: co-resident
+  // one thread per txn for K-group, one per op for the op stages (grid-stride beyond), + the a8
+  // block; co-resident
+  const uint32_t want = std::max<uint32_t>((b.n_txns + 255) / 256, (b.n_ops + 255) / 256) + 1;
+  const uint32_t grid = std::max<uint32_t>(2, std::min<uint32_t>(want, (uint32_t)(per_sm * sms)));
   cudaLaunchCooperativeKernel((const void*)k_ops_small, dim3(grid), dim3(256), args, 0, s);
   note_launch();
 }

@@ -36,14 +36,18 @@ def test_single_launch_ycsb_equals_oracle(n):
         check_batch(g, o, batch, tables)
 
 
+@pytest.mark.parametrize("flags", [0, 2, 4])  # (+ no mark filter, + NEXT-1 reordering)
 @pytest.mark.parametrize("seed", range(8))
-def test_single_launch_equals_multi_kernel(seed):
+def test_single_launch_equals_multi_kernel(seed, flags):
     """Every op kind (incl. duplicate-key INSERT user aborts, DELETE, SCAN over absent keys):
     the single launch and the multi-kernel path give the same verdicts, reads and tables."""
     rng = np.random.default_rng(7100 + seed)
     tables = opscases.rand_tables(rng)
-    g1, o = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048)
-    g2, _ = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048, flags=L().LTPG_FLAG_NO_SINGLE_LAUNCH)
+    g1, o = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048, flags=flags)
+    g2, _ = make_pair(opscases.RAND_DESCS, tables, 64, 256, extra_rows=2048,
+                      flags=flags | L().LTPG_FLAG_NO_SINGLE_LAUNCH)
+    if flags & 4:
+        o.set_reorder(True)
     for b in range(8):
         batch = opscases.rand_batch(rng, int(rng.integers(1, 60)), tid_start=1 + 100 * b)
         st = check_batch(g1, o, batch, tables)
