@@ -123,6 +123,8 @@ struct ltpg_db {
   unsigned long long* d_reserve = nullptr; // [MAXT]
   uint32_t* d_dense_live = nullptr;        // bitmask: tables whose dense key->row mapping is valid
   bool olrow_ready = false;                // TPC-C ORDER -> first ORDER_LINE row map built
+  bool tpcc_small_clean = false;           // partition 0's TPC-C batch scratch is in k_tpcc_small's
+                                           // rest state (set by it; a multi-kernel batch clears it)
   // Deferred PK index maintenance: TPC-C reaches new ORDER_LINE rows through ORDER.aux only,
   // so their write-back skips the hash insert; rows >= d_idx_from[t] of a table in idx_lag
   // are indexed in one pass before anything else could look them up by key (an OPS batch,
@@ -373,8 +375,10 @@ int ltpg_create_db(const ltpg_config* cfg, ltpg_db** out) {
     CK(dmalloc(&P.ua, n));
     CK(dmalloc(&P.lflag, n + 4));  // (k_ops_small ORs verdict bytes as 32-bit words)
     CK(dmalloc(&P.pmask, n));
-    CK(dmalloc(&P.small, 64));  // [0, 16) the partition's words; [16, 64) per-slot sets (k_ops_small)
-    CK(cudaMemset(P.small, 0, 64 * sizeof(uint32_t)));
+    // [0, 16) the partition's words; [16, 64) per-slot sets (single-launch kernels); [64 + 32 k]
+    // slot k's grid-barrier counter (one 128-byte line each)
+    CK(dmalloc(&P.small, 64 + 3 * 32));
+    CK(cudaMemset(P.small, 0, (64 + 3 * 32) * sizeof(uint32_t)));
     CK(dmalloc(&P.base, MAXT));
     int rc = tpcc_alloc(P.tpcc, cfg->max_txns, cfg->n_warehouses, p ? db->parts[0].tpcc.by_name : nullptr);
     if (rc) return fail(db, rc, "tpcc scratch allocation failed (n_warehouses <= 1000)");
@@ -754,11 +758,15 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   const bool partitioned = db->nparts > 1;
   const uint32_t L = db->loopback;
   const bool grouped = !(db->cfg.flags & LTPG_FLAG_NO_GROUPING);
-  // small single-partition OPS batches: a1..a8 in one cooperative launch (k_ops_small), with the
-  // slot's own set of partition small words (published and cleared by the kernel's last block)
-  const bool small = ops_mode && grouped && L == 1 && !partitioned && !db->p2p && n && n <= ops_small_max_txns() &&
+  // small single-partition batches: a1..a8 in one cooperative launch (k_ops_small, k_tpcc_small),
+  // with the slot's own set of partition small words (published and cleared by the kernel's last
+  // block)
+  const bool small = (ops_mode ? grouped && n <= ops_small_max_txns()
+                               : n <= tpcc_small_max_txns() && tpcc_small_fits(db->parts[0].tpcc)) &&
+                     L == 1 && !partitioned && !db->p2p && n &&
                      !(db->cfg.flags & (LTPG_FLAG_LARGE_BUCKETS | LTPG_FLAG_NO_SINGLE_LAUNCH));
   uint32_t* small_words = small ? db->parts[0].small + 16 * (1 + (&S - db->slots)) : nullptr;
+  uint32_t* small_bar = small ? db->parts[0].small + 64 + 32 * (&S - db->slots) : nullptr;
   S.timing = timing;
   S.res = res;
   S.host_out = !res->outputs_on_device;
@@ -951,13 +959,32 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
         launch_carry(P.eff_tid, P.eff_ptype, P.eff_params, P.eff_abort, nc, S.d_tid, S.d_ptype, S.d_params, s);
         CK(cudaEventRecord(db->slots[db->carry_slot].comp_done, s));
       }
+      BatchDev& x = pb[0];
+      if (!ops_mode) {
+        if (packed_params) {  // expand packed parameter blocks into 128-byte blocks (errors -> the slot's word)
+          const uint8_t* packed = b->inputs_on_device ? b->proc_params : S.d_packed;
+          const uint32_t* offs = b->inputs_on_device ? b->proc_offsets : S.d_offsets;
+          uint8_t* dst = S.d_params + (size_t)nc * LTPG_PARAM_BYTES;
+          if (b->flags & LTPG_BATCH_COMPACT_PARAMS) launch_unpack_compact(packed, offs, bd.ptype + nc, nf, dst, x.err, s);
+          else launch_unpack_params(packed, offs, nf, dst, x.err, s);
+        }
+        // the batch scratch's rest state (a captured graph always carries the clears: it may be
+        // replayed after a multi-kernel batch)
+        if (!db->tpcc_small_clean || capturing) tpcc_small_clear(db->parts[0].tpcc, s);
+      }
       const bool timed = timing || capturing;
       if (timed) CK(tmark(S.ev[1], s));
-      BatchDev& x = pb[0];
       x.status = st_out;
-      launch_ops_small(db->n_tables, x, filter, db->d_coop, db->d_reserve, S.d_vars,
-                       capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock, bits_out, S.d_small,
-                       !idx_catchup, abort_out, S.host_out ? nullptr : res->n_aborted, S.h_small_dev, s);
+      if (ops_mode) {
+        launch_ops_small(db->n_tables, x, filter, db->d_coop, db->d_reserve, S.d_vars,
+                         capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock, bits_out, S.d_small,
+                         !idx_catchup, abort_out, S.host_out ? nullptr : res->n_aborted, S.h_small_dev, small_bar, s);
+      } else {
+        const SmallOut so{db->d_reserve, S.d_vars, capturing ? S.h_vars_dev : nullptr, db->epoch, b->batch_clock,
+                          bits_out, S.d_small, abort_out, S.host_out ? nullptr : res->n_aborted, S.h_small_dev,
+                          !idx_catchup, small_bar};
+        if (launch_tpcc_small(db->parts[0].tpcc, x, so, s)) return fail(db, LTPG_ECUDA, "k_tpcc_small launch failed");
+      }
       if (timed)  // one kernel: ms_group holds the whole batch
         for (int e = 2; e <= 5; ++e) CK(tmark(S.ev[e], s));
       if (cr) launch_committed_reads(bits_out, n, res_out, cr_dst, db->d_wprefix, s);
@@ -1150,6 +1177,7 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
     const int rc = enqueue(s);
     if (rc) return rc;
   }
+  if (!ops_mode && n) db->tpcc_small_clean = small;  // a multi-kernel batch leaves its scratch dirty
   if (timing) CK(cudaEventRecord(S.ev[6], s));
   CK(cudaEventRecord(S.comp_done, s));  // (also the next batch's "previous compute" and the constants' last user)
   g_const_last[db->device % 64] = S.comp_done;

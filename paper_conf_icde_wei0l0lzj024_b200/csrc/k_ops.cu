@@ -13,6 +13,7 @@
 #include <cstdio>
 
 #include "ltpg_internal.cuh"
+#include "small.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -760,96 +761,6 @@ void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cu
 #ifdef LTPG_SMALL_TS
 __device__ unsigned long long g_small_we[8];  // per phase: the latest end of a thread's work
 #endif
-struct SmallOut {
-  unsigned long long* reserve;  // [MAXT] append reservations (cleared here)
-  BatchVars* vars;              // written here from (epoch, clock) or the slot's mapped host copy
-  const volatile BatchVars* host;
-  uint32_t epoch;
-  long long clock;
-  uint32_t* commit_bits;        // a8 outputs (as k_finalize_compact)
-  uint32_t* dsmall;             // the slot's words: [0] err (written iff write0) [8..10] counts [16] n
-  uint32_t* abort_out;
-  uint32_t* n_out2;             // or null
-  volatile uint32_t* host_small;  // the slot's mapped host words: [0..16] of dsmall, err ORed into [0]
-  bool write0;
-};
-
-// a8 for n txns in one block: 32 txns per thread-word, block-wide scan of the conflict counts
-// per 256-word round (carried), abort list in ascending rank order.  st_of(r) = txn r's status.
-template <class St>
-__device__ __forceinline__ void finalize_block(uint32_t n, const SmallOut& o, St st_of) {
-  __shared__ uint32_t fw[8], fcarry, fred[3];
-  const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if (threadIdx.x == 0) fcarry = 0;
-  if (threadIdx.x < 3) fred[threadIdx.x] = 0;
-  __syncthreads();
-  const uint32_t nw = (n + 31) / 32;
-  for (uint32_t base = 0; base < nw; base += blockDim.x) {
-    const uint32_t w = base + threadIdx.x;
-    uint32_t cm = 0, am = 0, nu = 0;
-    if (w < nw) {
-      const uint32_t r0 = w * 32, m = min(32u, n - r0);
-#pragma unroll 8
-      for (uint32_t j = 0; j < m; ++j) {
-        const uint8_t st = st_of(r0 + j);
-        cm |= (st == LTPG_ST_COMMIT ? 1u : 0u) << j;
-        am |= (st == LTPG_ST_CONFLICT ? 1u : 0u) << j;
-        nu += st == LTPG_ST_USER_ABORT;
-      }
-      o.commit_bits[w] = cm;
-    }
-    const uint32_t na = __popc(am);
-    uint32_t x = na;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
-      if (lane >= (uint32_t)d) x += y;
-    }
-    const uint32_t nbw = __reduce_add_sync(0xffffffffu, __popc(cm)), nuw = __reduce_add_sync(0xffffffffu, nu);
-    if (lane == 31) fw[wid] = x;
-    if (lane == 0) {
-      atomicAdd(fred + 0, nbw);
-      atomicAdd(fred + 2, nuw);
-    }
-    __syncthreads();
-    uint32_t before = fcarry, round = 0;
-#pragma unroll
-    for (uint32_t q = 0; q < 8; ++q) {
-      if (q < wid) before += fw[q];
-      round += fw[q];
-    }
-    uint32_t pos = before + x - na;
-    for (uint32_t m = am; m; m &= m - 1) o.abort_out[pos++] = w * 32 + (__ffs(m) - 1);
-    __syncthreads();
-    if (threadIdx.x == 0) fcarry += round;
-  }
-  __syncthreads();
-  if (threadIdx.x < 17) {  // the slot's result words (the host memset of them is skipped)
-    const uint32_t t = threadIdx.x;
-    const uint32_t v = t == 8 ? fred[0] : t == 9 ? fcarry : t == 10 ? fred[2] : t == 16 ? fcarry : 0u;
-    if (t || o.write0) o.dsmall[t] = v;
-  }
-  if (threadIdx.x == 0 && o.n_out2) *o.n_out2 = fcarry;
-}
-
-__device__ __forceinline__ void prefetch_l2(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
-
-// Grid-wide barrier of a co-resident grid on a counter that is zero at launch: barrier k waits
-// for k * gridDim.x arrivals (one release-add per block, acquire polling by thread 0).  About
-// half the cost of cg::grid_group::sync on B200 (tools/launchcost.cu).
-__device__ __forceinline__ void grid_barrier(uint32_t* ctr, uint32_t k) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
-    const uint32_t target = k * gridDim.x;
-    uint32_t v;
-    do {
-      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-    } while (v < target);
-  }
-  __syncthreads();
-}
-
 // Warm-up by the blocks that hold no txns during K-group: read the op records (so K-group's
 // staging loads find them in L2) and fetch every point op's row word, write mark (or index
 // home slot) and argument into L2 for the op stages that follow.  Loads and prefetches only.
@@ -888,7 +799,7 @@ __global__ void __launch_bounds__(256) k_ops_small(uint32_t n_tables, BatchDev b
                                                    SmallOut o) {
   __shared__ __align__(16) ltpg_op stage[8][GROUP_STAGE];
   cg::grid_group grid = cg::this_grid();  // (the INSERT tail's barriers)
-  uint32_t* bar = b.err + 15;  // a free partition word: zero at launch, cleared by the last block
+  uint32_t* bar = o.bar;  // zero at launch, cleared by the last block
   const uint32_t n = b.n_txns;
   const bool fin_block = blockIdx.x == gridDim.x - 1;  // a8 only; no op work
   const uint32_t gt = blockIdx.x * blockDim.x + threadIdx.x, gs = (gridDim.x - 1) * blockDim.x;
@@ -1009,7 +920,8 @@ __global__ void __launch_bounds__(256) k_ops_small(uint32_t n_tables, BatchDev b
       o.host_small[threadIdx.x] = reinterpret_cast<volatile uint32_t*>(o.dsmall)[threadIdx.x] |
                                   (threadIdx.x == 0 ? *reinterpret_cast<volatile uint32_t*>(b.err) : 0u);
     __syncthreads();
-    if (threadIdx.x < 16) b.err[threadIdx.x] = 0;  // err .. done, barrier counter
+    if (threadIdx.x < 16) b.err[threadIdx.x] = 0;  // err .. done
+    if (threadIdx.x == 0) *o.bar = 0;
   }
 #ifdef LTPG_SMALL_TS
   SMALL_TS();
@@ -1032,7 +944,7 @@ uint32_t ops_small_max_txns() { return 16384; }
 void launch_ops_small(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials,
                       unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host, uint32_t epoch,
                       long long clock, uint32_t* commit_bits, uint32_t* dsmall, bool write0, uint32_t* abort_out,
-                      uint32_t* n_out2, volatile uint32_t* host_small, cudaStream_t s) {
+                      uint32_t* n_out2, volatile uint32_t* host_small, uint32_t* bar, cudaStream_t s) {
   static int per_sm = 0, sms = 0;
   if (!per_sm) {
     int dev = 0;
@@ -1044,7 +956,7 @@ void launch_ops_small(uint32_t n_tables, const BatchDev& b, bool filter, uint32_
   uint32_t nt = n_tables;
   BatchDev bb = b;
   bool f = filter;
-  SmallOut so{reserve, vars, host, epoch, clock, commit_bits, dsmall, abort_out, n_out2, host_small, write0};
+  SmallOut so{reserve, vars, host, epoch, clock, commit_bits, dsmall, abort_out, n_out2, host_small, write0, bar};
   void* args[] = {&nt, &bb, &f, &partials, &so};
   // one thread per txn for K-group, one per op for the op stages (grid-stride beyond), + the a8
   // block; co-resident

@@ -16,6 +16,7 @@
 // NewOrder's fetch-ADD of D_NEXT_O_ID (R12, delayed-update prefix sum P:241) is
 // resolved after detection by a per-district prefix count in rank order.
 #include <algorithm>
+#include <cstdio>
 #include <map>
 #include <vector>
 
@@ -26,6 +27,29 @@ namespace ltpg {
 LTPG_DEFINE_TABLE_UPLOAD(upload_tables_tpcc)
 
 enum { PH_EXEC = 0, PH_DETECT = 1, PH_WB = 2 };
+
+#ifdef LTPG_SMALL_TS  // diagnostic builds: per-stage times, printed by the last block
+__device__ unsigned long long g_tsm[2][10];  // [0][k]: block 0 passed barrier k; [1][k]: latest work end of stage k
+#define TSM_PASS(k) \
+  if (blockIdx.x == 0 && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g_tsm[0][k]))
+#define TSM_AT(k)                                                \
+  {                                                              \
+    unsigned long long t_;                                       \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));       \
+    atomicMax(&g_tsm[1][k], t_);                                 \
+  }
+#define TSM_WORK(k)                                              \
+  {                                                              \
+    __syncthreads();                                             \
+    unsigned long long t_;                                       \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));       \
+    if (threadIdx.x == 0) atomicMax(&g_tsm[1][k], t_);           \
+  }
+#else
+#define TSM_PASS(k)
+#define TSM_WORK(k)
+#define TSM_AT(k)
+#endif
 
 __device__ __forceinline__ uint32_t p16(const uint8_t* p, int off) { return *reinterpret_cast<const uint16_t*>(p + off); }
 __device__ __forceinline__ uint32_t p32(const uint8_t* p, int off) { return *reinterpret_cast<const uint32_t*>(p + off); }
@@ -212,6 +236,16 @@ __device__ void tpcc_advance_tail(const BatchDev& b, const TpccParams& tp) {
   *c_tabs[TNO].n_rows += (uint32_t)tot;
   *c_tabs[TOL].n_rows += tot >> 32;
   *c_tabs[TH].n_rows += __ldcg(tp.misc + M_HIST);
+}
+
+// a committed NewOrder's o_id (the fetch-ADD pre-image of D_NEXT_O_ID, R12): assigned by k_no_assign
+// into its first result slot, or -- single-launch path (oid_inline, 32-rank chunks) -- the
+// district's snapshot value + committed NewOrders of the district in earlier chunks (column
+// scan) + those of smaller rank in the txn's own chunk (dk_of, written by no_chunk32_body)
+__device__ __forceinline__ long long no_oid(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t w, uint32_t d) {
+  if (!tp.oid_inline) return b.res[4ull * r];
+  const uint32_t dk = (uint32_t)kD(w, d);
+  return tp.dist_base[dk] + tp.chunk_cnt[(uint64_t)dk * tp.n_chunks + (r >> tp.chunk_shift)] + tp.dk_of[r];
 }
 
 // ---- NewOrder (TPC-C 2.4; SURVEY §8(c) procedure table) --------------------------------
@@ -458,12 +492,12 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
           sr[k] = h ? rd(TSt, S_REMOTE_CNT, rs[k]) : 0;
         }
       }
-      const long long o = b.res[4ull * r];
+      const long long o = no_oid(b, tp, r, w, d);
       const uint64_t okey = kO(w, d, (uint64_t)o);
       const DevTable& TOL_ = c_tabs[TOL];
       // append position: chunk base + in-chunk prefix of committed NewOrders (k_no_chunk); the
       // row counter is read before any store (a store could alias it and force a reload)
-      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
+      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r >> tp.chunk_shift];
       const unsigned long long ol0 = *TOL_.n_rows;
 #pragma unroll
       for (uint32_t k = 0; k < 4; ++k) {
@@ -510,9 +544,10 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
       const DevTable& TOr = c_tabs[TO];
       const DevTable& TOL_ = c_tabs[TOL];
       const DevTable& TNw = c_tabs[TNO];
-      const long long o = b.res[4ull * r];
+      const long long o = no_oid(b, tp, r, w, d);
+      if (tp.oid_inline) b.res[4ull * r] = o;
       const uint64_t okey = kO(w, d, (uint64_t)o);
-      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r / NO_CHUNK];
+      const unsigned long long pref = tp.no_pref[r] + tp.chunk_tot[r >> tp.chunk_shift];
       const unsigned long long nr_o = *TOr.n_rows, nr_ol = *TOL_.n_rows, nr_no = *TNw.n_rows;  // before stores
       const long long clock = b_clock(b);
       const uint32_t orow = (uint32_t)(nr_o + (uint32_t)pref);
@@ -1028,8 +1063,8 @@ __global__ void __launch_bounds__(256) k_sl_claim(BatchDev b, TpccParams tp, SlS
 }
 
 // one warp per listed district: window, distinct items, S_QUANTITY prefix table; NEXT-1 minR
-__global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
-  if (*b.err) return;
+__device__ __forceinline__ void sl_district_body(const BatchDev& b, const SlScratch& sl, uint32_t vb, uint32_t nvb) {
+  if (*(volatile uint32_t*)b.err) return;
   __shared__ uint32_t items_s[8][SL_SLOTS];
   __shared__ uint32_t set_s[8][SL_HASH];
   __shared__ uint32_t hist_s[8][SL_T + 1];
@@ -1043,9 +1078,9 @@ __global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
   uint32_t* hist = hist_s[wib];
   const uint32_t dmask = *b.dense_live;
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
-  const uint32_t nd_total = *sl.cnt;
-  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t idx = blockIdx.x * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
+  const uint32_t nd_total = *(volatile uint32_t*)sl.cnt;
+  const uint32_t nwarps = nvb * (blockDim.x >> 5);
+  for (uint32_t idx = vb * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
     const uint32_t dk = sl.dk[idx];
     uint32_t w = dk / 10, d = dk % 10;
     if (d == 0) { d = 10; w -= 1; }  // kD(w, 10) == kD(w + 1, 0)
@@ -1165,17 +1200,20 @@ __global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
     __syncwarp();
   }
 }
+__global__ void __launch_bounds__(256) k_sl_district(BatchDev b, SlScratch sl) {
+  sl_district_body(b, sl, blockIdx.x, gridDim.x);
+}
 
 // detection, one warp per listed district: M = smallest write / add rank over its unit set
-__global__ void __launch_bounds__(256) k_sl_detect(BatchDev b, SlScratch sl) {
-  if (*b.err) return;
+__device__ __forceinline__ void sl_detect_body(const BatchDev& b, const SlScratch& sl, uint32_t vb, uint32_t nvb) {
+  if (*(volatile uint32_t*)b.err) return;
   const DevTable& TDi = c_tabs[TD];
   const DevTable& TSt = c_tabs[TS];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t nd_total = *sl.cnt;
-  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  const uint32_t nd_total = *(volatile uint32_t*)sl.cnt;
+  const uint32_t nwarps = nvb * (blockDim.x >> 5);
   const uint32_t gq = col_group(TSt, S_QUANTITY), gd = col_group(TDi, D_NEXT_O_ID);
-  for (uint32_t idx = blockIdx.x * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
+  for (uint32_t idx = vb * (blockDim.x >> 5) + wib; idx < nd_total; idx += nwarps) {
     const uint32_t nd = sl.nd[idx];
     uint32_t m = 0xFFFFFFFFu;
     auto wa = [&](const DevTable& T, uint32_t g, uint32_t row) {
@@ -1189,14 +1227,16 @@ __global__ void __launch_bounds__(256) k_sl_detect(BatchDev b, SlScratch sl) {
     if (lane == 0) sl.m[idx] = m;
   }
 }
+__global__ void __launch_bounds__(256) k_sl_detect(BatchDev b, SlScratch sl) { sl_detect_body(b, sl, blockIdx.x, gridDim.x); }
 
 // per StockLevel txn: result from the district's table, RAW verdict from its M
-__global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScratch sl) {
-  if (*b.err) return;
-  const uint32_t n = tp.counts[4];
+__device__ __forceinline__ void sl_txn_body(const BatchDev& b, const TpccParams& tp, const SlScratch& sl, uint32_t vb,
+                                            uint32_t nvb) {
+  if (*(volatile uint32_t*)b.err) return;
+  const uint32_t n = *(volatile const uint32_t*)(tp.counts + 4);
   const uint32_t* list = tp.list + 4ull * tp.max_txns;
   const bool reorder = b.flags & LTPG_FLAG_REORDER;
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+  for (uint32_t i = vb * blockDim.x + threadIdx.x; i < n; i += nvb * blockDim.x) {
     const uint32_t r = list[i];
     const uint8_t* p = b.params + 128ull * r;
     const uint32_t idx = sl.slot[kD(p16(p, 0), p[2])];
@@ -1210,6 +1250,9 @@ __global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScr
     if (b.nparts > 1) b.lflag[r] = (uint8_t)flag;
     else b.status[r] = status_of_bits(flag, reorder);
   }
+}
+__global__ void __launch_bounds__(256) k_sl_txn(BatchDev b, TpccParams tp, SlScratch sl) {
+  sl_txn_body(b, tp, sl, blockIdx.x, gridDim.x);
 }
 
 // ---- the phase kernel: type-homogeneous warps over the per-type txn lists -------------------------
@@ -1231,7 +1274,6 @@ __device__ __forceinline__ uint32_t lanes_of(uint32_t t, int PH, uint32_t nparts
                           : (t == 4 ? 32u
                                     : (t == 2 || (t == 0 && nparts <= 1 && (PH != PH_DETECT || !reorder)) ? 4u : 16u));
 }  // NewOrder, Payment, OrderStatus, Delivery (StockLevel: k_sl_*)
-template <int PH, uint32_t TMASK>
 // minimum resident blocks per phase (register cap): detection is a chain of dependent
 // loads (params -> log -> marks) and gains most from occupancy (measured: 8 -> 32 regs);
 // write-back keeps every stock column of a lane's lines in registers (one load wave instead of
@@ -1246,18 +1288,43 @@ template <int PH, uint32_t TMASK>
 #ifndef LTPG_WB_MINB
 #define LTPG_WB_MINB 3
 #endif
-__global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
-    k_tpcc_phase(BatchDev b, TpccParams tp) {
-  // one read of the error word per block: the kernel has block barriers, and the word can be
-  // raised by other blocks of this grid while this one starts
-  __shared__ uint32_t s_err;
-  if (threadIdx.x == 0) s_err = *(volatile uint32_t*)b.err;
+// the phase body over (virtual) blocks vb of nvb; FUSED (single-launch path): the write-back's
+// row-counter advance is left to the caller
+template <int PH, uint32_t TMASK, bool FUSED>
+__device__ __forceinline__ void tpcc_phase_body(const BatchDev& b, const TpccParams& tp, uint32_t vb, uint32_t nvb) {
+  const bool reorder = b.flags & LTPG_FLAG_REORDER;
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
+  // NewOrder, Payment), so that the grid's tail is made of short Payment warps (0.088 -> 0.077
+  // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
+  constexpr uint32_t ORD = PH == PH_DETECT ? (2u | SL_DLW << 4 | 0u << 8 | SL_DLT << 12 | 1u << 16 | 4u << 20)
+                                           : (0u | 1u << 4 | 2u << 8 | SL_DLW << 12 | SL_DLT << 16 | 4u << 20);  // slot j -> type
+  // One read of the error word per block (the kernel has block barriers, and the word can be
+  // raised by other blocks of this grid while this one starts), issued together with the list
+  // lengths: slot counts and warp-slot prefixes per slot type, in shared memory (computed once
+  // per block; as register arrays they cost every thread 12 registers for the whole kernel)
+  __shared__ uint32_t s_err, cnt[NSLOT], pre[NSLOT + 1];
+  const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
+  if (threadIdx.x == 0) {
+    uint32_t c5[NTYPES];
+#pragma unroll
+    for (int t = 0; t < NTYPES; ++t) c5[t] = (TMASK >> t) & 1u ? tp.counts[t] : 0u;
+    s_err = *(volatile uint32_t*)b.err;
+    pre[0] = 0;
+#pragma unroll
+    for (int j = 0; j < NSLOT; ++j) {
+      const uint32_t t = (ORD >> (4 * j)) & 15u;
+      const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
+      cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : c5[t]));
+      const uint32_t lp = 5 - (__ffs(lanes_of(t, PH, b.nparts, reorder)) - 1);  // log2(txns per warp slot)
+      pre[j + 1] = pre[j] + ((cnt[j] + (1u << lp) - 1) >> lp);
+    }
+  }
   __syncthreads();
   if (s_err) return;  // (write-back: the row counters then stay put -- no last block runs)
   // ECAPACITY before anything is written back: the grouping counts are final here (a block
   // barrier + fence + counter per grouping block for a "last block" cost 22% of that kernel)
-  if (PH == PH_EXEC && TMASK == TM_MAIN && blockIdx.x == 0 && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
-  const uint32_t dmask = *b.dense_live;  // procedures never insert into / delete from W, D, C, I, S
+  if (PH == PH_EXEC && TMASK == TM_MAIN && vb == 0 && threadIdx.x == 0) tpcc_capacity_tail(b, tp);
   // write-back with delayed W_YTD / D_YTD (ADD columns): the block's committed Payments add
   // into shared-memory deltas per warehouse (and district), flushed with one atomic per touched
   // row at the end -- hundreds of thousands of same-row atomics at the L2 become a few per block
@@ -1273,28 +1340,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     for (uint32_t i = threadIdx.x; i < tp.hot_words; i += blockDim.x) hm[i] = 0xFFFFFFFFu;
     __syncthreads();
   }
-  const bool reorder = b.flags & LTPG_FLAG_REORDER;
-  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
-  // NewOrder, Payment), so that the grid's tail is made of short Payment warps (0.088 -> 0.077
-  // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
-  constexpr uint32_t ORD = PH == PH_DETECT ? (2u | SL_DLW << 4 | 0u << 8 | SL_DLT << 12 | 1u << 16 | 4u << 20)
-                                           : (0u | 1u << 4 | 2u << 8 | SL_DLW << 12 | SL_DLT << 16 | 4u << 20);  // slot j -> type
-  // slot counts and warp-slot prefixes per slot type, in shared memory (computed once per block;
-  // as register arrays they cost every thread 12 registers for the whole kernel)
-  __shared__ uint32_t cnt[NSLOT], pre[NSLOT + 1];
-  if (threadIdx.x == 0) {
-    pre[0] = 0;
-    for (int j = 0; j < NSLOT; ++j) {
-      const uint32_t t = (ORD >> (4 * j)) & 15u;
-      const bool on = (TMASK >> (t == SL_DLW ? SL_DLT : t)) & 1u;
-      cnt[j] = !on ? 0u : (t == SL_DLW ? tp.nw : (t == SL_DLT && PH != PH_DETECT ? 0u : tp.counts[t]));
-      const uint32_t lp = 5 - (__ffs(lanes_of(t, PH, b.nparts, reorder)) - 1);  // log2(txns per warp slot)
-      pre[j + 1] = pre[j] + ((cnt[j] + (1u << lp) - 1) >> lp);
-    }
-  }
-  __syncthreads();
-  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  const uint32_t nwarps = nvb * (blockDim.x >> 5);
   // warp slot w -> slot type t, this lane's list position k and sub-lane (warp-uniform type)
   const auto decode = [&](uint32_t w, uint32_t& t, uint32_t& k, uint32_t& sub, uint32_t& ct) {
     uint32_t j = 0, lw = w;
@@ -1314,7 +1360,7 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
     decode(w, t, k, sub, ct);
     return (t != SL_DLW && k < ct) ? tp.list[(uint64_t)t * tp.max_txns + k] : 0u;
   };
-  uint32_t w = blockIdx.x * (blockDim.x >> 5) + wib;
+  uint32_t w = vb * (blockDim.x >> 5) + wib;
   uint32_t r_next = w < pre[NSLOT] ? list_entry(w) : 0u;
   for (; w < pre[NSLOT]; w += nwarps) {
     uint32_t t, k, sub, ct;
@@ -1394,8 +1440,13 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
       addv(T, isw ? W_YTD : D_YTD, row, v);
     }
   }
-  if (PH == PH_WB && TMASK == TM_MAIN && last_block(tp.misc + M_DONE_WB) && threadIdx.x == 0)
+  if (!FUSED && PH == PH_WB && TMASK == TM_MAIN && last_block(tp.misc + M_DONE_WB) && threadIdx.x == 0)
     tpcc_advance_tail(b, tp);
+}
+template <int PH, uint32_t TMASK>
+__global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
+    k_tpcc_phase(BatchDev b, TpccParams tp) {
+  tpcc_phase_body<PH, TMASK, false>(b, tp, blockIdx.x, gridDim.x);
 }
 
 // ---- K-tgroup: validation + per-type lists (warp-aggregated appends) ----------------------------
@@ -1404,15 +1455,18 @@ __global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == P
 // first 16 bytes of each block are read: every field but the NewOrder lines sits there, and the
 // lines are validated by execute, which reads them anyway (proc_neworder; an invalid line
 // raises ERR_EINVAL there, before anything is written back).  134 -> 16 MB read per 2^20 txns.
-template <bool FULL>
-__global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
+// CLAIM (single-launch path, !FULL): k_sl_claim folded in -- a StockLevel's district is claimed
+// here (smallest rank per district, the first claimer lists it).  vb: the (virtual) block index.
+template <bool FULL, bool CLAIM>
+__device__ __forceinline__ void tpcc_group_body(const BatchDev& b, const TpccParams& tp, uint32_t vb,
+                                                const SlScratch& sl) {
   // FULL: the warp's 32 parameter blocks (4 KB, contiguous) staged through shared memory with
   // coalesced 16-byte loads; each lane then parses its own block.  Rows are padded to 33
   // words: with a 128-byte stride every lane's field would sit in the same bank (32-way
   // conflicts measured at 45% short-scoreboard stalls)
   constexpr uint32_t SROW = 132;
   __shared__ __align__(16) uint8_t stage[FULL ? 8 : 1][FULL ? 32 * SROW : 16];
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t r = vb * blockDim.x + threadIdx.x;
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = r - lane;
   uint8_t* sw = stage[FULL ? wib : 0];
@@ -1522,6 +1576,14 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
     uint32_t* m = tp.dl_min + (FULL ? p16(sw + SROW * lane, 0) : (head.x & 0xFFFFu));
     if (r < *m) atomicMin(m, r);
   }
+  if (CLAIM && !FULL && t == 4 && touch) {  // StockLevel: the district's smallest rank (k_sl_claim)
+    const uint32_t dk = (uint32_t)kD(head.x & 0xFFFFu, (head.x >> 16) & 0xFFu);
+    if (atomicMin(sl.minr + dk, r) == 0xFFFFFFFFu) {
+      const uint32_t idx = atomicAdd(sl.cnt, 1u);
+      sl.dk[idx] = dk;
+      sl.slot[dk] = idx;
+    }
+  }
   // block-aggregated counters and per-type list positions (one atomic per block and list)
   // slots 0..4: the per-type list flags (b.kcount), 5..7: misc[M_NO_LINES], misc[M_PAY],
   // misc[M_NO]; every slot but the line count is a 0/1 flag (ballot scans), one barrier pair
@@ -1536,6 +1598,10 @@ __global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
 #pragma unroll
   for (uint32_t k = 0; k < NTYPES; ++k)
     if (cnt[k]) tp.list[(uint64_t)k * tp.max_txns + base[k]] = r;
+}
+template <bool FULL>
+__global__ void __launch_bounds__(256) k_tpcc_group(BatchDev b, TpccParams tp) {
+  tpcc_group_body<FULL, false>(b, tp, blockIdx.x, SlScratch{});
 }
 
 // committed entries of every per-type list -> clist (order inside a list is irrelevant)
@@ -1569,22 +1635,23 @@ __global__ void __launch_bounds__(256) k_tpcc_relist(BatchDev b, TpccParams tp) 
 // total (chunk_tot; scanned by the last block of k_no_colscan).
 // RELIST (unpartitioned batches, where every txn touches this partition): also the committed
 // re-list of k_tpcc_relist, from the same status reads.
+// (StockLevel txns are not re-listed: write-back has nothing to do for them, and on the
+// single-launch path their verdicts are written concurrently with this pass)
 template <bool RELIST>
-__global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
-  extern __shared__ uint32_t hist[];
+__device__ __forceinline__ void no_chunk_body(const BatchDev& b, const TpccParams& tp, uint32_t chunk, uint32_t* hist) {
   __shared__ unsigned long long wsum[8];
-  if (*b.err) return;
+  if (*(volatile uint32_t*)b.err) return;
   for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) hist[i] = 0;
   __syncthreads();
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const uint32_t r0 = blockIdx.x * NO_CHUNK + 4 * threadIdx.x;
+  const uint32_t r0 = chunk * NO_CHUNK + 4 * threadIdx.x;
   unsigned long long v[4], tsum = 0;
   uint32_t dk[4], ty[4], cm[4];
 #pragma unroll
   for (uint32_t j = 0; j < 4; ++j) {
     const uint32_t r = r0 + j;
     ty[j] = r < b.n_txns ? b.ptype[r] : 0xFFu;
-    cm[j] = r < b.n_txns && b.status[r] == LTPG_ST_COMMIT;
+    cm[j] = r < b.n_txns && ty[j] != 4 && b.status[r] == LTPG_ST_COMMIT;
   }
   if (RELIST) {
     uint32_t cnt[NTYPES], base[NTYPES];
@@ -1639,9 +1706,55 @@ __global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
     }
     ex += v[j];
   }
-  if (threadIdx.x == 0) tp.chunk_tot[blockIdx.x] = total;
+  if (threadIdx.x == 0) tp.chunk_tot[chunk] = total;
   __syncthreads();
-  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i] = hist[i];
+  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)chunk * tp.dsz + i] = hist[i];
+  __syncthreads();  // (hist is reused by the caller's next chunk)
+}
+template <bool RELIST>
+__global__ void __launch_bounds__(256) k_no_chunk(BatchDev b, TpccParams tp) {
+  extern __shared__ uint32_t hist[];
+  no_chunk_body<RELIST>(b, tp, blockIdx.x, hist);
+}
+
+// Single-launch path: the same per-chunk quantities for 32-rank chunks, one (virtual) block of
+// 256 ranks = 8 chunks, one thread per rank: committed re-lists (block-aggregated), each warp's
+// district counts (every district's word of the chunk, zeros included, district-major for the
+// column scan's coalesced rows), the in-chunk rank among the district's committed NewOrders (dk_of: write-back adds it
+// to the district's chunk base, no assignment pass) and the in-chunk prefix of (lines << 32 | 1).
+__device__ __forceinline__ void no_chunk32_body(const BatchDev& b, const TpccParams& tp, uint32_t vb) {
+  if (*(volatile uint32_t*)b.err) return;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t r = vb * blockDim.x + threadIdx.x, c = r >> 5;
+  const uint32_t ty = r < b.n_txns ? b.ptype[r] : 0xFFu;
+  const bool cm = r < b.n_txns && ty != 4 && b.status[r] == LTPG_ST_COMMIT;
+  uint32_t cnt[NTYPES], base[NTYPES];
+#pragma unroll
+  for (uint32_t k = 0; k < NTYPES; ++k) cnt[k] = (cm && ty == k) ? 1u : 0u;
+  block_reserve<NTYPES, (1u << NTYPES) - 1u>(cnt, tp.misc + M_CCOUNT, base);
+#pragma unroll
+  for (uint32_t k = 0; k < NTYPES; ++k)
+    if (cnt[k]) tp.clist[(uint64_t)k * tp.max_txns + base[k]] = r;
+  bool no = cm && ty == 0;
+  uint32_t hdr = 0;
+  if (no) hdr = *reinterpret_cast<const uint32_t*>(b.params + 128ull * r);  // u16 w | u8 d | u8 n_lines
+  const uint32_t dk = no ? (uint32_t)kD(hdr & 0xFFFFu, (hdr >> 16) & 0xFFu) : ~0u;
+  const uint32_t m = __match_any_sync(0xffffffffu, dk);
+  if (c * 32 < b.n_txns) {  // district-major: [dk][chunk] (the column scan reads whole rows)
+    for (uint32_t i = lane; i < tp.dsz; i += 32) tp.chunk_cnt[(uint64_t)i * tp.n_chunks + c] = 0;
+    __syncwarp();
+    if (no && lane == (uint32_t)(__ffs(m) - 1)) tp.chunk_cnt[(uint64_t)dk * tp.n_chunks + c] = __popc(m);
+  }
+  if (r < b.n_txns) tp.dk_of[r] = no ? __popc(m & ((1u << lane) - 1u)) : 0u;
+  const unsigned long long v = no ? ((unsigned long long)(hdr >> 24) << 32 | 1ull) : 0ull;
+  unsigned long long x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  if (r < b.n_txns) tp.no_pref[r] = x - v;
+  if (lane == 31 && c * 32 < b.n_txns) tp.chunk_tot[c] = x;
 }
 
 // chunk totals -> exclusive chunk bases (in place) and the batch total in no_pref[n]
@@ -1651,6 +1764,7 @@ __device__ void chunk_total_scan(const BatchDev& b, const TpccParams& tp) {
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t c0 = threadIdx.x * per;
   unsigned long long tsum = 0;
+#pragma unroll 4
   for (uint32_t c = c0; c < c0 + per && c < nc; ++c) tsum += tp.chunk_tot[c];
   unsigned long long x = tsum;
 #pragma unroll
@@ -1675,13 +1789,14 @@ __device__ void chunk_total_scan(const BatchDev& b, const TpccParams& tp) {
 
 // Column scan of chunk_cnt ([chunk][district] -> exclusive prefix over chunks, in place), plus
 // the district bases and the final D_NEXT_O_ID: one warp per district key
-__global__ void k_no_colscan(BatchDev b, TpccParams tp) {
-  if (*b.err) return;
-  if (blockIdx.x == gridDim.x - 1) {  // the extra last block: chunk bases
+// vb of nvb = (dsz + 7) / 8 + 1 blocks (the last one scans the chunk totals)
+__device__ __forceinline__ void no_colscan_body(const BatchDev& b, const TpccParams& tp, uint32_t vb, uint32_t nvb) {
+  if (*(volatile uint32_t*)b.err) return;
+  if (vb == nvb - 1) {  // the extra last block: chunk bases
     chunk_total_scan(b, tp);
     return;
   }
-  const uint32_t dk = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const uint32_t dk = vb * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
   constexpr uint32_t PER = 32;  // chunks per lane held in registers; 1024 chunks per pass
@@ -1718,9 +1833,42 @@ __global__ void k_no_colscan(BatchDev b, TpccParams tp) {
     atomicOr(b.err, ERR_EINTERNAL);
     return;
   }
-  const long long base = rd(TDi, D_NEXT_O_ID, row_d);
-  tp.dist_base[dk] = base;
+  tp.dist_base[dk] = rd(TDi, D_NEXT_O_ID, row_d);
   addv(TDi, D_NEXT_O_ID, row_d, run_all);  // final value: snapshot + committed NewOrders (delayed add)
+}
+__global__ void k_no_colscan(BatchDev b, TpccParams tp) { no_colscan_body(b, tp, blockIdx.x, gridDim.x); }
+
+// Single-launch path: one warp per district over its district-major row of <= 512 32-rank chunk
+// counts (coalesced: lane l holds chunks l, l + 32, ...; 16 warp scans with a carry) -> exclusive
+// prefixes in place; D_NEXT_O_ID advanced (the snapshot was read into dist_base before).  The
+// caller checked the error word.
+static_assert(16384 / SMALL_CHUNK <= 16 * 32, "no_colscan32_body: 16 chunks per lane");
+__device__ __forceinline__ void no_colscan32_body(const BatchDev& b, const TpccParams& tp, uint32_t dk) {
+  const uint32_t lane = threadIdx.x & 31, nc = tp.n_chunks;
+  uint32_t* row = tp.chunk_cnt + (uint64_t)dk * nc;
+  uint32_t v[16];
+#pragma unroll
+  for (uint32_t k = 0; k < 16; ++k) v[k] = k * 32 + lane < nc ? row[k * 32 + lane] : 0u;
+  uint32_t carry = 0;
+#pragma unroll
+  for (uint32_t k = 0; k < 16; ++k) {
+    uint32_t x = v[k];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= (uint32_t)o) x += y;
+    }
+    if (k * 32 + lane < nc) row[k * 32 + lane] = carry + x - v[k];
+    carry += __shfl_sync(0xffffffffu, x, 31);
+  }
+  if (!carry || lane) return;
+  const DevTable& TDi = c_tabs[TD];
+  const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
+  if (row_d == ROW_NONE) {
+    atomicOr(b.err, ERR_EINTERNAL);
+    return;
+  }
+  addv(TDi, D_NEXT_O_ID, row_d, carry);  // final value: snapshot + committed NewOrders (delayed add)
 }
 
 // Column scan for many districts (tpcc_c5: 5131 district keys): 8 districts per block, tiles of
@@ -1787,12 +1935,16 @@ __global__ void __launch_bounds__(256) k_no_colscan_tiled(BatchDev b, TpccParams
   addv(TDi, D_NEXT_O_ID, row_d, run_all);  // final value: snapshot + committed NewOrders (delayed add)
 }
 
-__global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk, ranks in order
-  extern __shared__ uint32_t cntd[];
-  if (*b.err) return;
-  const uint32_t lane = threadIdx.x;
-  for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.chunk_cnt[(uint64_t)blockIdx.x * tp.dsz + i];
-  const uint32_t r0 = blockIdx.x * NO_CHUNK;
+// one warp per chunk, ranks in order; cntd: the warp's dsz shared-memory words, each district's
+// next o_id (snapshot D_NEXT_O_ID + committed NewOrders of smaller rank in earlier chunks: the
+// walk below then touches shared memory only -- with the district base read from global memory
+// in the walk, every step waited for an L2 round trip)
+__device__ __forceinline__ void no_assign_body(const BatchDev& b, const TpccParams& tp, uint32_t chunk, long long* cntd) {
+  if (*(volatile uint32_t*)b.err) return;
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t i = lane; i < tp.dsz; i += 32)  // (dist_base of a district without commits: unused)
+    cntd[i] = tp.dist_base[i] + tp.chunk_cnt[(uint64_t)chunk * tp.dsz + i];
+  const uint32_t r0 = chunk * NO_CHUNK;
   uint32_t dks[NO_CHUNK / 32];
 #pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {  // all of the chunk's loads in flight first
@@ -1808,12 +1960,16 @@ __global__ void k_no_assign(BatchDev b, TpccParams tp) {  // one warp per chunk,
     const uint32_t m = __match_any_sync(0xffffffffu, dk);
     if (dk != ~0u) {
       const uint32_t before = __popc(m & ((1u << lane) - 1));
-      b.res[4ull * r] = tp.dist_base[dk] + cntd[dk] + before;
+      b.res[4ull * r] = cntd[dk] + before;
     }
     __syncwarp();
     if (dk != ~0u && lane == (uint32_t)(__ffs(m) - 1)) cntd[dk] += __popc(m);
     __syncwarp();
   }
+}
+__global__ void k_no_assign(BatchDev b, TpccParams tp) {
+  extern __shared__ long long cntd[];
+  no_assign_body(b, tp, blockIdx.x, cntd);
 }
 
 
@@ -1854,7 +2010,9 @@ int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t nw, int* shared_by_name) 
   if (!nw) return 0;
   if (nw > 1000) return LTPG_EINVAL;
   t.dsz = nw * 10 + 11;
-  const uint64_t chunks = (max_txns + NO_CHUNK - 1) / NO_CHUNK;
+  // (the single-launch path counts in 32-rank chunks: up to 16384 / 32 of them)
+  const uint64_t chunks = std::max<uint64_t>((max_txns + NO_CHUNK - 1) / NO_CHUNK,
+                                             (std::min<uint64_t>(max_txns, 16384) + SMALL_CHUNK - 1) / SMALL_CHUNK);
   t.owns_by_name = shared_by_name == nullptr;
   if (shared_by_name) t.by_name = shared_by_name;
   else if (dm(&t.by_name, (uint64_t)t.dsz * 1000)) return LTPG_ENOMEM;
@@ -1935,7 +2093,8 @@ static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists)
   return TpccParams{t.clist, committed_lists ? t.clist : t.list, committed_lists ? t.misc + M_CCOUNT : b.kcount, t.log,
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min,
-                    committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u, committed_lists ? 0u : hot_words(t, b)};
+                    committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u, committed_lists ? 0u : hot_words(t, b),
+                    10u, false};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -2021,10 +2180,183 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
     k_no_colscan_tiled<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   else
     k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
-  k_no_assign<<<tp.n_chunks, 32, smem, s>>>(b, tp);
+  if (2 * smem > 48 * 1024) {  // (n_warehouses <= 1000: at most 80 KB)
+    static size_t set = 0;
+    if (set < 2 * smem && cudaFuncSetAttribute(k_no_assign, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               (int)(2 * smem)) == cudaSuccess)
+      set = 2 * smem;
+  }
+  k_no_assign<<<tp.n_chunks, 32, 2 * smem, s>>>(b, tp);
   note_launch(3);
   k_tpcc_phase<PH_WB, TM_MAIN><<<resident_grid<PH_WB>(n, wb_smem(t)), 256, wb_smem(t), s>>>(b, params_of(t, b, true));  // + row counters
   note_launch(1);
+  return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
+}
+
+
+// ---- small batches: a1..a8 in ONE cooperative launch ---------------------------------------
+// A single-partition batch of <= 16384 txns (BASELINE configs[1]: 1 warehouse, 16k NewOrder /
+// Payment) runs each stage in a few microseconds, so the ~14 kernel boundaries of the multi-kernel
+// path (and the StockLevel side-stream joins) were most of its latency.  Here the same stage
+// bodies run in one co-resident grid separated by grid-wide barriers:
+//   S1 a1/a2 validation + per-type lists (+ the StockLevel district claims, the batch's clears)
+//   S2 a4/a5 execute + marks; StockLevel districts          S3 a6 detection; StockLevel M
+//   S4 StockLevel verdicts; committed re-lists + o_id counts per 32-rank chunk
+//   S5 o_id column scans + chunk bases   (the a8 block: commit bitmask, counts, abort list)
+//   S6 a7 write-back, each committed NewOrder's o_id = district base + chunk prefix + in-chunk rank
+// then the last block to finish advances the append-row counters, publishes the slot's result
+// words into mapped host memory and returns the batch scratch to its rest state (misc counters,
+// Delivery minima, StockLevel claims, the slot's small words: the next single-launch batch needs
+// no clearing pass; capi.cu clears them once after a multi-kernel batch).  Same device code as
+// the multi-kernel path (the bodies above), hence result-identical.  Work stages run on blocks
+// [0, G-1); block G-1 only computes a8 (it leaves the barrier protocol after S4).
+__global__ void __launch_bounds__(256, 2) k_tpcc_small(BatchDev b, TpccParams tx, TpccParams tw, SlScratch sl,
+                                                       SmallOut o) {
+  TSM_PASS(0);
+  uint32_t* bar = o.bar;  // zero at launch, cleared at the end
+  const uint32_t G = gridDim.x, W = G - 1;
+  const bool fin = blockIdx.x == G - 1;
+  const uint32_t n = b.n_txns;
+  // S1: the batch's clears for the later stages (append reservations, batch scalars -- read with
+  // ld.global.nc by b_epoch after the barrier, no SM cached their line before -- user-abort flags)
+  if (blockIdx.x == 0) {
+    if (threadIdx.x < MAXT) o.reserve[threadIdx.x] = 0;
+    if (threadIdx.x == 0) {
+      o.vars->epoch = o.host ? o.host->epoch : o.epoch;
+      o.vars->clock = o.host ? o.host->clock : o.clock;
+    }
+  }
+  if (!fin) {
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += W * blockDim.x) b.ua[i] = 0;
+    for (uint32_t vb = blockIdx.x; vb < (n + blockDim.x - 1) / blockDim.x; vb += W)
+      tpcc_group_body<false, true>(b, tx, vb, sl);
+  }
+  TSM_WORK(1);
+  grid_barrier_to(bar, G);
+  TSM_PASS(1);
+  if (!fin) {  // S2
+    tpcc_phase_body<PH_EXEC, TM_MAIN, true>(b, tx, blockIdx.x, W);
+    sl_district_body(b, sl, blockIdx.x, W);
+  }
+  TSM_WORK(2);
+  grid_barrier_to(bar, 2 * G);
+  TSM_PASS(2);
+  if (!fin) {  // S3
+    tpcc_phase_body<PH_DETECT, TM_MAIN, true>(b, tx, blockIdx.x, W);
+    sl_detect_body(b, sl, blockIdx.x, W);
+  }
+  TSM_WORK(3);
+  grid_barrier_to(bar, 3 * G);
+  TSM_PASS(3);
+  if (!fin) {  // S4
+    sl_txn_body(b, tx, sl, blockIdx.x, W);
+    for (uint32_t vb = blockIdx.x; vb < (n + blockDim.x - 1) / blockDim.x; vb += W) no_chunk32_body(b, tx, vb);
+  } else {  // every district's snapshot D_NEXT_O_ID (the o_id bases; S5 then only adds)
+    const DevTable& TDi = c_tabs[TD];
+    const uint32_t dmask = *b.dense_live;
+    for (uint32_t dk = 11 + threadIdx.x; dk < tx.dsz; dk += blockDim.x) {  // kD(1, 1) = 11
+      const uint32_t row_d = rowof(TDi, TD, dk, dmask);
+      if (row_d != ROW_NONE) tx.dist_base[dk] = rd(TDi, D_NEXT_O_ID, row_d);
+    }
+  }
+  TSM_WORK(4);
+  grid_barrier_to(bar, 4 * G);  // every verdict is final
+  TSM_PASS(4);
+  const bool ok = *(volatile uint32_t*)b.err == 0;  // uniform: raised before the last barrier
+  if (fin) {  // a8
+    if (ok) finalize_block(n, o, [&](uint32_t r) { return b.status[r]; });
+    else if (threadIdx.x < 17 && (threadIdx.x || o.write0)) o.dsmall[threadIdx.x] = 0;  // failed batch: no counts
+    TSM_WORK(8);
+  } else {
+    const uint32_t ncs = (tx.dsz + 7) / 8 + 1;  // S5
+    if (ok)
+      for (uint32_t vb = blockIdx.x; vb < ncs; vb += W) {
+        if (vb == ncs - 1) chunk_total_scan(b, tx);  // chunk bases
+        else if (vb * 8 + (threadIdx.x >> 5) < tx.dsz) no_colscan32_body(b, tx, vb * 8 + (threadIdx.x >> 5));
+      }
+    TSM_WORK(5);
+    grid_barrier_to(bar, 4 * G + W);
+    TSM_PASS(5);
+    TSM_PASS(6);
+    tpcc_phase_body<PH_WB, TM_MAIN, true>(b, tw, blockIdx.x, W);  // S6 (o_ids computed inline)
+    TSM_WORK(7);
+  }
+  __shared__ bool last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(b.done, 1u) == G - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  if (threadIdx.x == 0) tpcc_advance_tail(b, tw);  // (nothing when the batch failed)
+  if (threadIdx.x < 17)
+    o.host_small[threadIdx.x] = reinterpret_cast<volatile uint32_t*>(o.dsmall)[threadIdx.x] |
+                                (threadIdx.x == 0 ? *reinterpret_cast<volatile uint32_t*>(b.err) : 0u);
+  const uint32_t nsl = *(volatile uint32_t*)sl.cnt;
+  for (uint32_t i = threadIdx.x; i < nsl; i += blockDim.x) sl.minr[sl.dk[i]] = 0xFFFFFFFFu;
+  for (uint32_t w = threadIdx.x; w <= tx.nw; w += blockDim.x) tx.dl_min[w] = ~0u;
+  __syncthreads();
+  if (threadIdx.x < 16) {
+    b.err[threadIdx.x] = 0;  // err .. done
+    tx.misc[threadIdx.x] = 0;
+  }
+  if (threadIdx.x == 0) *bar = 0;
+  if (threadIdx.x == 0) *sl.cnt = 0;
+#ifdef LTPG_SMALL_TS
+  if (threadIdx.x == 0) {
+    unsigned long long t_;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));
+    volatile unsigned long long* p = g_tsm[0];
+    volatile unsigned long long* w = g_tsm[1];
+    printf("k_tpcc_small n=%u G=%u ns from start: pass B1 %lld B2 %lld B3 %lld B4 %lld B5 %lld B6 %lld end %lld | "
+           "work end S1 %lld S2 %lld S3 %lld S4 %lld S5 %lld S5-districts %lld S7 %lld a8 %lld S5-chunks %lld\n", n, G,
+           (long long)(p[1] - p[0]), (long long)(p[2] - p[0]), (long long)(p[3] - p[0]), (long long)(p[4] - p[0]),
+           (long long)(p[5] - p[0]), (long long)(p[6] - p[0]), (long long)(t_ - p[0]), (long long)(w[1] - p[0]),
+           (long long)(w[2] - p[0]), (long long)(w[3] - p[0]), (long long)(w[4] - p[0]), (long long)(w[5] - p[0]),
+           (long long)(w[6] - p[0]), (long long)(w[7] - p[0]), (long long)(w[8] - p[0]), (long long)(w[9] - p[0]));
+    for (int k = 0; k < 10; ++k) w[k] = 0;
+  }
+#endif
+}
+
+uint32_t tpcc_small_max_txns() { return 16384; }
+bool tpcc_small_fits(const TpccDev& t) { return t.nw >= 1 && t.nw <= TPCC_SMALL_MAX_W; }
+
+void tpcc_small_clear(TpccDev& t, cudaStream_t s) {
+  cudaMemsetAsync(t.misc, 0, 16 * sizeof(uint32_t), s);
+  cudaMemsetAsync(t.dl_min, 0xFF, (t.nw + 1) * sizeof(uint32_t), s);
+  cudaMemsetAsync(t.sl.minr, 0xFF, (size_t)t.dsz * sizeof(uint32_t), s);
+  cudaMemsetAsync(t.sl.cnt, 0, sizeof(uint32_t), s);
+}
+
+int launch_tpcc_small(TpccDev& t, const BatchDev& b, const SmallOut& o, cudaStream_t s) {
+  TpccParams tx = params_of(t, b, false), tw = params_of(t, b, true);
+  tx.n_chunks = tw.n_chunks = (b.n_txns + SMALL_CHUNK - 1) / SMALL_CHUNK;
+  tx.chunk_shift = tw.chunk_shift = 5;
+  static_assert(SMALL_CHUNK == 32, "one warp per chunk");
+  tw.oid_inline = true;
+  const size_t smem = std::max((size_t)tx.hot_words * sizeof(mark_t), wb_smem(t));  // execute's hm / write-back's agg
+  static int ps = 0, sms = 0;  // co-resident blocks per SM at the last dynamic shared memory size
+  static size_t ps_smem = ~(size_t)0;
+  if (smem != ps_smem) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ps, k_tpcc_small, 256, smem) != cudaSuccess || ps < 1) ps = 1;
+    ps_smem = smem;
+  }
+  // about 8 txns per warp (execute's NewOrder slots) + the a8 block; co-resident
+  const uint32_t want = (b.n_txns + 63) / 64 + 1;
+  const uint32_t grid = std::max<uint32_t>(2, std::min<uint32_t>(want, (uint32_t)(ps * sms)));
+  BatchDev bb = b;
+  TpccParams a = tx, c = tw;
+  SlScratch sl = t.sl;
+  SmallOut so = o;
+  void* args[] = {&bb, &a, &c, &sl, &so};
+  cudaLaunchCooperativeKernel((const void*)k_tpcc_small, dim3(grid), dim3(256), args, smem, s);
+  note_launch();
   return cudaGetLastError() == cudaSuccess ? 0 : LTPG_ECUDA;
 }
 

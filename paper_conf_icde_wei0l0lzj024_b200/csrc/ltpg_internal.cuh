@@ -492,7 +492,7 @@ uint32_t ops_small_max_txns();
 void launch_ops_small(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials,
                       unsigned long long* reserve, BatchVars* vars, const volatile BatchVars* host, uint32_t epoch,
                       long long clock, uint32_t* commit_bits, uint32_t* dsmall, bool write0, uint32_t* abort_out,
-                      uint32_t* n_out2, volatile uint32_t* host_small, cudaStream_t s);
+                      uint32_t* n_out2, volatile uint32_t* host_small, uint32_t* bar, cudaStream_t s);
 void launch_ops_insert_tail(uint32_t n_tables, const BatchDev& b, bool filter, uint32_t* partials, cudaStream_t s);
 void launch_ops_detect(const BatchDev& b, cudaStream_t s);
 void launch_ops_writeback(const BatchDev& b, uint32_t n_tables, bool advance, cudaStream_t s);

@@ -1,6 +1,7 @@
 // TPC-C PROC-mode scratch and launchers (pre-compiled stored procedures).
 #pragma once
 #include "ltpg_internal.cuh"
+#include "small.cuh"
 
 namespace ltpg {
 
@@ -8,6 +9,7 @@ constexpr int NTYPES = 5;
 constexpr int TLOG = 20;         // u32 row slots logged per txn by execute (NewOrder 16, Payment 4,
                                  // OrderStatus 17), padded to 80 B so every txn's log is 16-B aligned
 constexpr int NO_CHUNK = 1024;   // ranks per chunk of the o_id prefix computation
+constexpr int SMALL_CHUNK = 32;  // the same on the single-launch path (k_tpcc_small)
 
 // TPC-C schema (include/ltpg.h): table ids and column indices
 enum { TW = 0, TD = 1, TC = 2, TH = 3, TNO = 4, TO = 5, TOL = 6, TI = 7, TS = 8 };
@@ -83,6 +85,8 @@ struct TpccParams {
   uint32_t* dl_min;
   uint32_t agg_dsz;             // write-back: DISTRICT D_YTD deltas aggregated per block (0: not)
   uint32_t hot_words;           // execute: shared-memory marks of the W / D units (nw + 30 nw; 0: off)
+  uint32_t chunk_shift;         // log2 ranks per o_id chunk (NO_CHUNK; SMALL_CHUNK on the single-launch path)
+  bool oid_inline;              // write-back computes the o_id (single-launch path, no k_no_assign)
 };
 
 int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);
@@ -92,6 +96,15 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
 // front: validate + lists, capacity, execute, detect;  back: o_id prefix, write-back, cursors
 int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cleared);
 int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s);
+// single-launch path for small single-partition batches (k_tpcc_small): n_txns <= max_txns()
+// and n_warehouses <= TPCC_SMALL_MAX_W (the per-warp o_id counters live in shared memory);
+// tpcc_small_clear puts the batch scratch into the rest state the kernel expects (after a
+// multi-kernel batch, which leaves it dirty)
+constexpr uint32_t TPCC_SMALL_MAX_W = 64;
+uint32_t tpcc_small_max_txns();
+bool tpcc_small_fits(const TpccDev& t);
+void tpcc_small_clear(TpccDev& t, cudaStream_t s);
+int launch_tpcc_small(TpccDev& t, const BatchDev& b, const SmallOut& o, cudaStream_t s);
 // ORDER.aux[row] = first row of the order's ORDER_LINE rows when they are contiguous
 void tpcc_build_olrow(cudaStream_t s);
 
