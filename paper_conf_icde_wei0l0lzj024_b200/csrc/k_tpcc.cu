@@ -238,6 +238,13 @@ __device__ void tpcc_advance_tail(const BatchDev& b, const TpccParams& tp) {
   *c_tabs[TH].n_rows += __ldcg(tp.misc + M_HIST);
 }
 
+// chunk_cnt[chunk][district] word: district-major ([dk][chunk]) up to CC_DM_DSZ district keys --
+// the column scan then reads whole rows coalesced (chunk-major, its strided column reads cost
+// 16.5 us on tpcc_c4) -- chunk-major above (512 warehouses: per-chunk rows of 5131 words, whose
+// scattered district-major stores cost more than the tiled column scan, k_no_colscan_tiled)
+__device__ __forceinline__ uint64_t cc_at(const TpccParams& tp, uint32_t dk, uint32_t c) {
+  return tp.cc_dm ? (uint64_t)dk * tp.n_chunks + c : (uint64_t)c * tp.dsz + dk;
+}
 // a committed NewOrder's o_id (the fetch-ADD pre-image of D_NEXT_O_ID, R12): assigned by k_no_assign
 // into its first result slot, or -- single-launch path (oid_inline, 32-rank chunks) -- the
 // district's snapshot value + committed NewOrders of the district in earlier chunks (column
@@ -245,7 +252,7 @@ __device__ void tpcc_advance_tail(const BatchDev& b, const TpccParams& tp) {
 __device__ __forceinline__ long long no_oid(const BatchDev& b, const TpccParams& tp, uint32_t r, uint32_t w, uint32_t d) {
   if (!tp.oid_inline) return b.res[4ull * r];
   const uint32_t dk = (uint32_t)kD(w, d);
-  return tp.dist_base[dk] + tp.chunk_cnt[(uint64_t)dk * tp.n_chunks + (r >> tp.chunk_shift)] + tp.dk_of[r];
+  return tp.dist_base[dk] + tp.chunk_cnt[cc_at(tp, dk, r >> tp.chunk_shift)] + tp.dk_of[r];
 }
 
 // ---- NewOrder (TPC-C 2.4; SURVEY §8(c) procedure table) --------------------------------
@@ -1708,7 +1715,7 @@ __device__ __forceinline__ void no_chunk_body(const BatchDev& b, const TpccParam
   }
   if (threadIdx.x == 0) tp.chunk_tot[chunk] = total;
   __syncthreads();
-  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[(uint64_t)chunk * tp.dsz + i] = hist[i];
+  for (uint32_t i = threadIdx.x; i < tp.dsz; i += blockDim.x) tp.chunk_cnt[cc_at(tp, i, chunk)] = hist[i];
   __syncthreads();  // (hist is reused by the caller's next chunk)
 }
 template <bool RELIST>
@@ -1741,9 +1748,9 @@ __device__ __forceinline__ void no_chunk32_body(const BatchDev& b, const TpccPar
   const uint32_t dk = no ? (uint32_t)kD(hdr & 0xFFFFu, (hdr >> 16) & 0xFFu) : ~0u;
   const uint32_t m = __match_any_sync(0xffffffffu, dk);
   if (c * 32 < b.n_txns) {  // district-major: [dk][chunk] (the column scan reads whole rows)
-    for (uint32_t i = lane; i < tp.dsz; i += 32) tp.chunk_cnt[(uint64_t)i * tp.n_chunks + c] = 0;
+    for (uint32_t i = lane; i < tp.dsz; i += 32) tp.chunk_cnt[cc_at(tp, i, c)] = 0;
     __syncwarp();
-    if (no && lane == (uint32_t)(__ffs(m) - 1)) tp.chunk_cnt[(uint64_t)dk * tp.n_chunks + c] = __popc(m);
+    if (no && lane == (uint32_t)(__ffs(m) - 1)) tp.chunk_cnt[cc_at(tp, dk, c)] = __popc(m);
   }
   if (r < b.n_txns) tp.dk_of[r] = no ? __popc(m & ((1u << lane) - 1u)) : 0u;
   const unsigned long long v = no ? ((unsigned long long)(hdr >> 24) << 32 | 1ull) : 0ull;
@@ -1787,11 +1794,40 @@ __device__ void chunk_total_scan(const BatchDev& b, const TpccParams& tp) {
   if (threadIdx.x == 0) tp.no_pref[b.n_txns] = total;
 }
 
-// Column scan of chunk_cnt ([chunk][district] -> exclusive prefix over chunks, in place), plus
-// the district bases and the final D_NEXT_O_ID: one warp per district key
-// vb of nvb = (dsz + 7) / 8 + 1 blocks (the last one scans the chunk totals)
+// Exclusive prefix over chunks of one district's row of chunk counts (district-major, in place):
+// lane l holds chunks t0 + 32 k + l of a 1024-chunk tile (coalesced loads and stores), 32 warp
+// scans per tile with a running carry.  Returns the district's total.
+__device__ __forceinline__ uint32_t chunk_row_scan(uint32_t* row, uint32_t nc) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t carry = 0;
+  for (uint32_t t0 = 0; t0 < nc; t0 += 1024) {
+    uint32_t v[32];
+#pragma unroll
+    for (uint32_t k = 0; k < 32; ++k) v[k] = t0 + k * 32 + lane < nc ? row[t0 + k * 32 + lane] : 0u;
+#pragma unroll
+    for (uint32_t k = 0; k < 32; ++k) {
+      if (t0 + k * 32 >= nc) break;  // (warp-uniform)
+      uint32_t x = v[k];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      if (t0 + k * 32 + lane < nc) row[t0 + k * 32 + lane] = carry + x - v[k];
+      carry += __shfl_sync(0xffffffffu, x, 31);
+    }
+  }
+  return carry;
+}
+
+// Column scan of chunk_cnt ([district][chunk] -> exclusive prefix over chunks, in place), plus
+// the district bases and the final D_NEXT_O_ID: one warp per district key.  SNAP (single-launch
+// path): the caller checked the error word and dist_base already holds every district's snapshot
+// D_NEXT_O_ID (read in the previous stage by the otherwise idle a8 block).
+// vb of nvb = (dsz + 7) / 8 + 1 blocks (the last one scans the chunk totals).
+template <bool SNAP>
 __device__ __forceinline__ void no_colscan_body(const BatchDev& b, const TpccParams& tp, uint32_t vb, uint32_t nvb) {
-  if (*(volatile uint32_t*)b.err) return;
+  if (!SNAP && *(volatile uint32_t*)b.err) return;
   if (vb == nvb - 1) {  // the extra last block: chunk bases
     chunk_total_scan(b, tp);
     return;
@@ -1799,33 +1835,7 @@ __device__ __forceinline__ void no_colscan_body(const BatchDev& b, const TpccPar
   const uint32_t dk = vb * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
-  constexpr uint32_t PER = 32;  // chunks per lane held in registers; 1024 chunks per pass
-  uint32_t run_all = 0;
-  for (uint32_t base = 0; base < tp.n_chunks; base += 32 * PER) {
-    uint32_t v[PER];
-#pragma unroll
-    for (uint32_t k = 0; k < PER; ++k) {  // lane owns chunks base + [lane*PER, lane*PER+PER): loads in flight
-      const uint32_t ch = base + lane * PER + k;
-      v[k] = ch < tp.n_chunks ? tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] : 0u;
-    }
-    uint32_t tot = 0;
-#pragma unroll
-    for (uint32_t k = 0; k < PER; ++k) tot += v[k];
-    uint32_t x = tot;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= (uint32_t)o) x += y;
-    }
-    uint32_t run = run_all + x - tot;  // exclusive prefix of this lane's first chunk
-    run_all += __shfl_sync(0xffffffffu, x, 31);
-#pragma unroll
-    for (uint32_t k = 0; k < PER; ++k) {
-      const uint32_t ch = base + lane * PER + k;
-      if (ch < tp.n_chunks) tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] = run;
-      run += v[k];
-    }
-  }
+  const uint32_t run_all = chunk_row_scan(tp.chunk_cnt + (uint64_t)dk * tp.n_chunks, tp.n_chunks);  // (cc_dm)
   if (!run_all || lane) return;
   const DevTable& TDi = c_tabs[TD];
   const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
@@ -1833,42 +1843,11 @@ __device__ __forceinline__ void no_colscan_body(const BatchDev& b, const TpccPar
     atomicOr(b.err, ERR_EINTERNAL);
     return;
   }
-  tp.dist_base[dk] = rd(TDi, D_NEXT_O_ID, row_d);
+  if (!SNAP) tp.dist_base[dk] = rd(TDi, D_NEXT_O_ID, row_d);
   addv(TDi, D_NEXT_O_ID, row_d, run_all);  // final value: snapshot + committed NewOrders (delayed add)
 }
-__global__ void k_no_colscan(BatchDev b, TpccParams tp) { no_colscan_body(b, tp, blockIdx.x, gridDim.x); }
-
-// Single-launch path: one warp per district over its district-major row of <= 512 32-rank chunk
-// counts (coalesced: lane l holds chunks l, l + 32, ...; 16 warp scans with a carry) -> exclusive
-// prefixes in place; D_NEXT_O_ID advanced (the snapshot was read into dist_base before).  The
-// caller checked the error word.
-static_assert(16384 / SMALL_CHUNK <= 16 * 32, "no_colscan32_body: 16 chunks per lane");
-__device__ __forceinline__ void no_colscan32_body(const BatchDev& b, const TpccParams& tp, uint32_t dk) {
-  const uint32_t lane = threadIdx.x & 31, nc = tp.n_chunks;
-  uint32_t* row = tp.chunk_cnt + (uint64_t)dk * nc;
-  uint32_t v[16];
-#pragma unroll
-  for (uint32_t k = 0; k < 16; ++k) v[k] = k * 32 + lane < nc ? row[k * 32 + lane] : 0u;
-  uint32_t carry = 0;
-#pragma unroll
-  for (uint32_t k = 0; k < 16; ++k) {
-    uint32_t x = v[k];
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= (uint32_t)o) x += y;
-    }
-    if (k * 32 + lane < nc) row[k * 32 + lane] = carry + x - v[k];
-    carry += __shfl_sync(0xffffffffu, x, 31);
-  }
-  if (!carry || lane) return;
-  const DevTable& TDi = c_tabs[TD];
-  const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
-  if (row_d == ROW_NONE) {
-    atomicOr(b.err, ERR_EINTERNAL);
-    return;
-  }
-  addv(TDi, D_NEXT_O_ID, row_d, carry);  // final value: snapshot + committed NewOrders (delayed add)
+__global__ void __launch_bounds__(256) k_no_colscan(BatchDev b, TpccParams tp) {
+  no_colscan_body<false>(b, tp, blockIdx.x, gridDim.x);
 }
 
 // Column scan for many districts (tpcc_c5: 5131 district keys): 8 districts per block, tiles of
@@ -1942,8 +1921,6 @@ __global__ void __launch_bounds__(256) k_no_colscan_tiled(BatchDev b, TpccParams
 __device__ __forceinline__ void no_assign_body(const BatchDev& b, const TpccParams& tp, uint32_t chunk, long long* cntd) {
   if (*(volatile uint32_t*)b.err) return;
   const uint32_t lane = threadIdx.x & 31;
-  for (uint32_t i = lane; i < tp.dsz; i += 32)  // (dist_base of a district without commits: unused)
-    cntd[i] = tp.dist_base[i] + tp.chunk_cnt[(uint64_t)chunk * tp.dsz + i];
   const uint32_t r0 = chunk * NO_CHUNK;
   uint32_t dks[NO_CHUNK / 32];
 #pragma unroll
@@ -1951,6 +1928,11 @@ __device__ __forceinline__ void no_assign_body(const BatchDev& b, const TpccPara
     const uint32_t r = r0 + it * 32 + lane;
     dks[it] = r < b.n_txns ? tp.dk_of[r] : ~0u;
   }
+  // only the districts of the chunk's committed NewOrders (a few dozen of dsz) are initialised
+  // (a lane writing a district another lane writes too stores the same value)
+#pragma unroll
+  for (uint32_t it = 0; it < NO_CHUNK / 32; ++it)
+    if (dks[it] != ~0u) cntd[dks[it]] = tp.dist_base[dks[it]] + tp.chunk_cnt[cc_at(tp, dks[it], chunk)];
   __syncwarp();
 #pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {
@@ -2074,7 +2056,6 @@ int tpcc_build_secondary(TpccDev& t, const uint64_t* keys, const int64_t* cols, 
 }
 
 constexpr uint32_t AGG_DSZ_MAX = 4096;  // per-block D_YTD aggregation up to ~400 warehouses (32 KB)
-constexpr uint32_t COLSCAN_TILED_DSZ = 2048;  // above: k_no_colscan_tiled
 static size_t wb_smem(const TpccDev& t) {
   return ((size_t)t.nw + 1 + (t.dsz <= AGG_DSZ_MAX ? t.dsz : 0)) * sizeof(long long);
 }
@@ -2094,7 +2075,7 @@ static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists)
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min,
                     committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u, committed_lists ? 0u : hot_words(t, b),
-                    10u, false};
+                    10u, false, t.dsz <= CC_DM_DSZ};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -2176,10 +2157,10 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
     k_no_chunk<false><<<tp.n_chunks, 256, smem, s>>>(b, tp);
     note_launch();
   }
-  if (t.dsz > COLSCAN_TILED_DSZ)
-    k_no_colscan_tiled<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
-  else
+  if (tp.cc_dm)
     k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
+  else
+    k_no_colscan_tiled<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   if (2 * smem > 48 * 1024) {  // (n_warehouses <= 1000: at most 80 KB)
     static size_t set = 0;
     if (set < 2 * smem && cudaFuncSetAttribute(k_no_assign, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2270,10 +2251,7 @@ __global__ void __launch_bounds__(256, 2) k_tpcc_small(BatchDev b, TpccParams tx
   } else {
     const uint32_t ncs = (tx.dsz + 7) / 8 + 1;  // S5
     if (ok)
-      for (uint32_t vb = blockIdx.x; vb < ncs; vb += W) {
-        if (vb == ncs - 1) chunk_total_scan(b, tx);  // chunk bases
-        else if (vb * 8 + (threadIdx.x >> 5) < tx.dsz) no_colscan32_body(b, tx, vb * 8 + (threadIdx.x >> 5));
-      }
+      for (uint32_t vb = blockIdx.x; vb < ncs; vb += W) no_colscan_body<true>(b, tx, vb, ncs);
     TSM_WORK(5);
     grid_barrier_to(bar, 4 * G + W);
     TSM_PASS(5);
@@ -2337,6 +2315,7 @@ int launch_tpcc_small(TpccDev& t, const BatchDev& b, const SmallOut& o, cudaStre
   tx.chunk_shift = tw.chunk_shift = 5;
   static_assert(SMALL_CHUNK == 32, "one warp per chunk");
   tw.oid_inline = true;
+  tx.cc_dm = tw.cc_dm = true;  // (<= 64 warehouses)
   const size_t smem = std::max((size_t)tx.hot_words * sizeof(mark_t), wb_smem(t));  // execute's hm / write-back's agg
   static int ps = 0, sms = 0;  // co-resident blocks per SM at the last dynamic shared memory size
   static size_t ps_smem = ~(size_t)0;
