@@ -238,10 +238,12 @@ __device__ void tpcc_advance_tail(const BatchDev& b, const TpccParams& tp) {
   *c_tabs[TH].n_rows += __ldcg(tp.misc + M_HIST);
 }
 
-// chunk_cnt[chunk][district] word: district-major ([dk][chunk]) up to CC_DM_DSZ district keys --
-// the column scan then reads whole rows coalesced (chunk-major, its strided column reads cost
-// 16.5 us on tpcc_c4) -- chunk-major above (512 warehouses: per-chunk rows of 5131 words, whose
-// scattered district-major stores cost more than the tiled column scan, k_no_colscan_tiled)
+// chunk_cnt[chunk][district] word: district-major ([dk][chunk]) up to COLSCAN_TILED_DSZ district
+// keys and on the single-launch path -- the column scan reads whole rows coalesced (chunk-major,
+// a warp reading one word per 2.6 KB row: 16.5 us on tpcc_c4; tpcc_c2 single launch 9 -> 5 us;
+// tpcc_c4 write-back 0.128 -> 0.124 ms, profiles/ab_r02_assign.txt) -- chunk-major above (512
+// warehouses: the per-chunk histogram's 5131 scattered stores per chunk would cost more than the
+// tiled column scan, k_no_colscan_tiled, that transposes through shared memory)
 __device__ __forceinline__ uint64_t cc_at(const TpccParams& tp, uint32_t dk, uint32_t c) {
   return tp.cc_dm ? (uint64_t)dk * tp.n_chunks + c : (uint64_t)c * tp.dsz + dk;
 }
@@ -1835,7 +1837,37 @@ __device__ __forceinline__ void no_colscan_body(const BatchDev& b, const TpccPar
   const uint32_t dk = vb * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const uint32_t lane = threadIdx.x & 31;
   if (dk >= tp.dsz) return;
-  const uint32_t run_all = chunk_row_scan(tp.chunk_cnt + (uint64_t)dk * tp.n_chunks, tp.n_chunks);  // (cc_dm)
+  uint32_t run_all = 0;
+  if (tp.cc_dm) {
+    run_all = chunk_row_scan(tp.chunk_cnt + (uint64_t)dk * tp.n_chunks, tp.n_chunks);
+  } else {  // chunk-major: a column walk, 32 chunks per lane held in registers, 1024 per pass
+    constexpr uint32_t PER = 32;
+    for (uint32_t base = 0; base < tp.n_chunks; base += 32 * PER) {
+      uint32_t v[PER];
+#pragma unroll
+      for (uint32_t k = 0; k < PER; ++k) {  // lane owns chunks base + [lane*PER, lane*PER+PER): loads in flight
+        const uint32_t ch = base + lane * PER + k;
+        v[k] = ch < tp.n_chunks ? tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] : 0u;
+      }
+      uint32_t tot = 0;
+#pragma unroll
+      for (uint32_t k = 0; k < PER; ++k) tot += v[k];
+      uint32_t x = tot;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      uint32_t run = run_all + x - tot;  // exclusive prefix of this lane's first chunk
+      run_all += __shfl_sync(0xffffffffu, x, 31);
+#pragma unroll
+      for (uint32_t k = 0; k < PER; ++k) {
+        const uint32_t ch = base + lane * PER + k;
+        if (ch < tp.n_chunks) tp.chunk_cnt[(uint64_t)ch * tp.dsz + dk] = run;
+        run += v[k];
+      }
+    }
+  }
   if (!run_all || lane) return;
   const DevTable& TDi = c_tabs[TD];
   const uint32_t row_d = rowof(TDi, TD, dk, *b.dense_live);
@@ -1928,11 +1960,19 @@ __device__ __forceinline__ void no_assign_body(const BatchDev& b, const TpccPara
     const uint32_t r = r0 + it * 32 + lane;
     dks[it] = r < b.n_txns ? tp.dk_of[r] : ~0u;
   }
-  // only the districts of the chunk's committed NewOrders (a few dozen of dsz) are initialised
-  // (a lane writing a district another lane writes too stores the same value)
+  // Many districts (> COLSCAN_TILED_DSZ keys, chunk-major): only the districts of the chunk's
+  // committed NewOrders (a few dozen of the 5131 at 512 warehouses; tpcc_c5 write-back 0.432 ->
+  // 0.411 ms).  Otherwise the whole row (district-major gathers / one coalesced row; tpcc_c4
+  // write-back 0.132 (per-district) -> 0.124 ms, profiles/ab_r02_assign.txt).  (A lane writing a
+  // district another lane writes too stores the same value; dist_base of a district without
+  // commits is never read.)
+  if (tp.dsz > COLSCAN_TILED_DSZ) {
 #pragma unroll
-  for (uint32_t it = 0; it < NO_CHUNK / 32; ++it)
-    if (dks[it] != ~0u) cntd[dks[it]] = tp.dist_base[dks[it]] + tp.chunk_cnt[cc_at(tp, dks[it], chunk)];
+    for (uint32_t it = 0; it < NO_CHUNK / 32; ++it)
+      if (dks[it] != ~0u) cntd[dks[it]] = tp.dist_base[dks[it]] + tp.chunk_cnt[cc_at(tp, dks[it], chunk)];
+  } else {
+    for (uint32_t i = lane; i < tp.dsz; i += 32) cntd[i] = tp.dist_base[i] + tp.chunk_cnt[cc_at(tp, i, chunk)];
+  }
   __syncwarp();
 #pragma unroll
   for (uint32_t it = 0; it < NO_CHUNK / 32; ++it) {
@@ -2075,7 +2115,7 @@ static TpccParams params_of(TpccDev& t, const BatchDev& b, bool committed_lists)
                     t.no_pref, t.dk_of, t.chunk_cnt, t.dist_base, t.misc, t.by_name,
                     t.nw, t.dsz, t.max_txns, (n + NO_CHUNK - 1) / NO_CHUNK, t.chunk_tot, t.dl_min,
                     committed_lists && t.dsz <= AGG_DSZ_MAX ? t.dsz : 0u, committed_lists ? 0u : hot_words(t, b),
-                    10u, false, t.dsz <= CC_DM_DSZ};
+                    10u, false, t.dsz <= COLSCAN_TILED_DSZ};
 }
 static uint32_t phase_grid(uint32_t n) {
   const uint64_t warps = (uint64_t)n + NTYPES;  // upper bound (StockLevel: 1 warp/txn)
@@ -2157,10 +2197,10 @@ int tpcc_back(TpccDev& t, BatchDev& b, uint32_t* scan_scratch, cudaStream_t s) {
     k_no_chunk<false><<<tp.n_chunks, 256, smem, s>>>(b, tp);
     note_launch();
   }
-  if (tp.cc_dm)
-    k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
-  else
+  if (t.dsz > COLSCAN_TILED_DSZ && !tp.cc_dm)
     k_no_colscan_tiled<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
+  else
+    k_no_colscan<<<(t.dsz + 7) / 8 + 1, 256, 0, s>>>(b, tp);
   if (2 * smem > 48 * 1024) {  // (n_warehouses <= 1000: at most 80 KB)
     static size_t set = 0;
     if (set < 2 * smem && cudaFuncSetAttribute(k_no_assign, cudaFuncAttributeMaxDynamicSharedMemorySize,

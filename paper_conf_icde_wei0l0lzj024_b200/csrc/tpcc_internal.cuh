@@ -87,9 +87,9 @@ struct TpccParams {
   uint32_t hot_words;           // execute: shared-memory marks of the W / D units (nw + 30 nw; 0: off)
   uint32_t chunk_shift;         // log2 ranks per o_id chunk (NO_CHUNK; SMALL_CHUNK on the single-launch path)
   bool oid_inline;              // write-back computes the o_id (single-launch path, no k_no_assign)
-  bool cc_dm;                   // chunk_cnt district-major (dsz <= CC_DM_DSZ), else chunk-major
+  bool cc_dm;                   // chunk_cnt district-major (dsz <= COLSCAN_TILED_DSZ, single-launch path)
 };
-constexpr uint32_t CC_DM_DSZ = 2048;
+constexpr uint32_t COLSCAN_TILED_DSZ = 2048;  // above: chunk-major chunk counts, k_no_colscan_tiled
 
 int tpcc_alloc(TpccDev& t, uint32_t max_txns, uint32_t n_warehouses, int* shared_by_name);
 void tpcc_free(TpccDev& t);
