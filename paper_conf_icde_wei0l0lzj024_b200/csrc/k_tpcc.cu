@@ -759,15 +759,11 @@ __device__ void proc_payment(const BatchDev& b, const TpccParams& tp, uint32_t r
     return;
   }
   if (PH == PH_EXEC) {
-    PP pw{}, pd{};
-    if (home) {  // warehouse + district lookups and the by-name lookup in flight together
-      pw = pp_issue(TWh, TW, w, x.dmask);
-      pd = pp_issue(TDi, TD, kD(w, d), x.dmask);
-    }
     if (cust && by_name) cid = (uint32_t)tp.by_name[kD(cw, cd) * 1000 + clast];  // static secondary index
-    if (home) {
-      row_w = pp_finish(TWh, pw);
-      row_d = pp_finish(TDi, pd);
+    if (home) {  // (dense W / D keys: arithmetic; two in-flight probes (pp_issue) cost execute 16
+                 // registers and spills of its slot loop for a case no TPC-C table layout hits)
+      row_w = rowof(TWh, TW, w, x.dmask);
+      row_d = rowof(TDi, TD, kD(w, d), x.dmask);
       if (row_w == ROW_NONE || row_d == ROW_NONE) { internal_error(x); return; }
     }
     if (cust) {
