@@ -417,7 +417,9 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
           if (ri[k] == ROW_NONE) {
             ua = 1;  // unused item id: NewOrder rollback (R11)
           } else {
+#ifdef LTPG_AMOUNT_IN_LOOP
             amount += (long long)qt[k] * price[k];
+#endif
             row_s = rs[k];
             if (row_s == ROW_NONE) internal_error(x);
           }
@@ -430,6 +432,12 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
         }
       }
       (void)it;
+#ifndef LTPG_AMOUNT_IN_LOOP
+      // the amounts after every mark and log store of the lane were issued: the item-price round
+      // trip overlaps them instead of holding them back (price[k] == 0 for unused slots and items)
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) amount += (long long)qt[k] * price[k];
+#endif
       if (sub == 3) {  // header: warehouse / district / customer reads, fetch-ADD of D_NEXT_O_ID
 #ifdef LTPG_NO_HDR_EARLY
         const uint32_t row_w = rowof(TWh, TW, w, x.dmask), row_d = rowof(TDi, TD, kD(w, d), x.dmask),
