@@ -8,8 +8,10 @@ fast enough to compute every output of these batches, so the comparison is compl
 batches (a fresh batch, then its aborted txns + fresh txns, with the state of the first
 carried over), then every table's canonical dump -- bit-exact.
 
-configs[2] (YCSB 10M rows, 2^20 x 10 ops, zipf 0.99) and configs[3] (TPC-C 64 warehouses,
-full mix, 2^20) against the oracle; configs[4] (512 warehouses, 2^20) by the partition
+configs[0] (YCSB 10k rows, 1024 x 4 ops) and configs[1] (TPC-C 1 warehouse, 16k; strict and
+delayed + NEXT-1) -- one cooperative launch each in the bench --, configs[2] (YCSB 10M rows, 2^20
+x 10 ops, zipf 0.99) and configs[3] (TPC-C 64 warehouses, full mix, 2^20; strict, delayed,
+delayed + NEXT-1) against the oracle; configs[4] (512 warehouses, 2^20) by the partition
 invariance PIN-8 at full size (one partition vs eight loopback partitions, every output and the
 WAREHOUSE / DISTRICT state equal) plus CC1, and -- opt-in, LTPG_FULL_C5=1 on a box with the host
 RAM for it -- against the oracle like the others.
@@ -102,7 +104,10 @@ def _c5_enabled():
         return False
 
 
-@pytest.mark.parametrize("name", ["ycsb_c3", "tpcc_c4", "tpcc_c4_opt",
+# (ycsb_c1 / tpcc_c2 / tpcc_c2_opt: BASELINE configs[0] and [1], which the bench runs as ONE
+# cooperative launch -- the single-launch path in the bench's own launch configuration)
+@pytest.mark.parametrize("name", ["ycsb_c1", "tpcc_c2", "tpcc_c2_opt", "ycsb_c3", "tpcc_c4", "tpcc_c4_delayed",
+                                  "tpcc_c4_opt",
                                   pytest.param("tpcc_c5", marks=pytest.mark.skipif(
                                       not _c5_enabled(), reason="opt-in: LTPG_FULL_C5=1 and > 100 GB host RAM"))])
 def test_full_size_equals_oracle(name):
