@@ -168,7 +168,7 @@ __device__ __forceinline__ void unit_w(const DevTable& T, uint32_t g, uint32_t r
     if (h) atomicMin(h, x.tag);
     else mark_unit(T, MK_W, g, row, x.tag, x.filter && hot);
   }
-  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_WRITE, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits_lim(T, g, row, ACC_WRITE, x.tag);
 }
 template <int PH>
 __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
@@ -177,13 +177,13 @@ __device__ __forceinline__ void unit_a(const DevTable& T, uint32_t g, uint32_t r
     if (h) atomicMin(h, x.tag);
     else mark_unit(T, MK_A, g, row, x.tag, x.filter && hot);
   }
-  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_ADD, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits_lim(T, g, row, ACC_ADD, x.tag);
 }
 template <int PH>
 __device__ __forceinline__ void unit_r(const DevTable& T, uint32_t g, uint32_t row, Tx& x, bool hot = false) {
   if (g == LTPG_STATIC) return;
   if (PH == PH_EXEC && T.rmarks) mark_unit(T, MK_R, g, row, x.tag, x.filter && hot);  // NEXT-1 minR
-  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits(T, g, row, ACC_READ, x.r, x.epoch);
+  if (PH == PH_DETECT && !x.done()) x.bits |= unit_bits_lim(T, g, row, ACC_READ, x.tag);
 }
 // update of column c (strict: WRITE unit of its group; delayed: ADD unit)
 template <int PH>
@@ -298,13 +298,13 @@ __device__ void proc_neworder(const BatchDev& b, const TpccParams& tp, uint32_t 
 #pragma unroll
     for (int k = 0; k < 4; ++k) {  // same units as the general path below (unit_w / col_upd3)
       if (rows[k] == ROW_NONE || sub + 4 * k == 15) continue;
-      bits |= unit_bits(TSt, gq, rows[k], ACC_WRITE, x.r, x.epoch);
-      if (gy != gq) bits |= unit_bits(TSt, gy, rows[k], ay, x.r, x.epoch);
-      if (go != gq && go != gy) bits |= unit_bits(TSt, go, rows[k], ao, x.r, x.epoch);
-      if (gr != gq && gr != gy && gr != go) bits |= unit_bits(TSt, gr, rows[k], ar, x.r, x.epoch);
+      bits |= unit_bits_lim(TSt, gq, rows[k], ACC_WRITE, x.tag);
+      if (gy != gq) bits |= unit_bits_lim(TSt, gy, rows[k], ay, x.tag);
+      if (go != gq && go != gy) bits |= unit_bits_lim(TSt, go, rows[k], ao, x.tag);
+      if (gr != gq && gr != gy && gr != go) bits |= unit_bits_lim(TSt, gr, rows[k], ar, x.tag);
     }
     if (sub == 3 && rows[3] != ROW_NONE)  // slot 15: the district row (fetch-ADD of D_NEXT_O_ID)
-      bits |= unit_bits(TDi, col_group(TDi, D_NEXT_O_ID), rows[3], ACC_ADD, x.r, x.epoch);
+      bits |= unit_bits_lim(TDi, col_group(TDi, D_NEXT_O_ID), rows[3], ACC_ADD, x.tag);
     x.bits |= bits;
     return;
   }

@@ -274,16 +274,24 @@ __device__ __forceinline__ uint8_t status_of_bits(uint32_t bits, bool reorder) {
 //   READ  -> RAW if a smaller rank wrote or added
 //   WRITE -> WAW if a smaller rank wrote or added; WAR if a smaller rank read (reorder only)
 //   ADD   -> WAW if a smaller rank plainly wrote;  WAR if a smaller rank read (reorder only)
+// The same on raw mark words: lim = epoch_tag(epoch) | r.  Within a mark window (capi.cu resets
+// every mark when epoch / 255 changes) a live mark's tag byte is this epoch's or an older epoch's,
+// i.e. >= this epoch's byte, so  mark_rank(v, epoch) < r  <=>  v < lim  (an older epoch's mark and
+// the unmarked 0xFFFFFFFF compare above lim; r < 2^24) -- one compare per mark, no tag extraction.
+__device__ __forceinline__ uint32_t unit_bits_lim(const DevTable& T, uint32_t g, uint32_t row, uint32_t acc,
+                                                  mark_t lim) {
+  const mark_t w = *wmark_ptr(T, g, row);
+  const mark_t a = ((T.add_groups >> g) & 1u) ? *amark_ptr(T, g, row) : 0xFFFFFFFFu;
+  const mark_t wa = w < a ? w : a;
+  uint32_t bits = 0;
+  if (acc == ACC_READ) return wa < lim ? CF_RAW : 0u;
+  if ((acc == ACC_WRITE ? wa : w) < lim) bits |= CF_WAW;
+  if (T.rmarks && *rmark_ptr(T, g, row) < lim) bits |= CF_WAR;
+  return bits;
+}
 __device__ __forceinline__ uint32_t unit_bits(const DevTable& T, uint32_t g, uint32_t row, uint32_t acc, uint32_t r,
                                               uint32_t epoch) {
-  const uint32_t w = mark_rank(*wmark_ptr(T, g, row), epoch);
-  const uint32_t a = ((T.add_groups >> g) & 1u) ? mark_rank(*amark_ptr(T, g, row), epoch) : 0xFFFFFFFFu;
-  const uint32_t wa = w < a ? w : a;
-  uint32_t bits = 0;
-  if (acc == ACC_READ) return wa < r ? CF_RAW : 0u;
-  if ((acc == ACC_WRITE ? wa : w) < r) bits |= CF_WAW;
-  if (T.rmarks && mark_rank(*rmark_ptr(T, g, row), epoch) < r) bits |= CF_WAR;
-  return bits;
+  return unit_bits_lim(T, g, row, acc, epoch_tag(epoch) | r);
 }
 __device__ __forceinline__ bool unit_conflicts(const DevTable& T, uint32_t g, uint32_t row, uint64_t chk,
                                                uint32_t r, uint32_t epoch) {
