@@ -268,11 +268,12 @@ typedef struct {
  * must stay valid (and unmodified) until then.  Batches still execute in submission order. */
 #define LTPG_BATCH_ASYNC 1u
 /* Compact TPC-C records (with proc_offsets; txn r's record is bytes [off[r], off[r+1])),
- * expanded to 128-byte blocks on the device -- ~1/3 fewer host->device bytes than used prefixes:
+ * expanded to 128-byte blocks on the device -- ~1/2 the host->device bytes of used prefixes:
  * NewOrder   : u16 w | u8 d | u8 n_lines | u16 c | u8 rbk | u8 n_remote |
- *              n_lines x u32 { i (bits 0-16) | qty-1 (bits 17-20) | remote (bit 21) } |
- *              n_remote x u16 supply_w (of the remote lines, in line order; other lines
- *              are supplied by w)                          = 8 + 4 n_lines + 2 n_remote bytes
+ *              n_lines x 22-bit line { i (bits 0-16) | qty-1 (bits 17-20) | remote (bit 21) },
+ *              a little-endian bit stream (line l at bits 22 l .. 22 l + 21; ceil(22 n_lines / 8)
+ *              bytes) | n_remote x u16 supply_w (of the remote lines, in line order; other
+ *              lines are supplied by w)          = 8 + ceil(22 n_lines / 8) + 2 n_remote bytes
  * Payment    : bytes 0-11 of the block | u32 amount (0 <= amount < 2^32)  = 16 bytes
  * other types: the used prefix of the block (as without this flag).
  * A record whose length does not match its header is LTPG_EINVAL (nothing changed). */

@@ -378,8 +378,9 @@ def pack_params(types, params):
 
 
 def pack_params_compact(types, params):
-    """Compact TPC-C records (include/ltpg.h LTPG_BATCH_COMPACT_PARAMS): NewOrder lines as u32
-    (item, qty, remote flag) plus the supply warehouses of remote lines, Payment amounts as u32.
+    """Compact TPC-C records (include/ltpg.h LTPG_BATCH_COMPACT_PARAMS): NewOrder lines as 22-bit
+    fields (item, qty, remote flag) in a little-endian bit stream plus the supply warehouses of
+    remote lines, Payment amounts as u32.
     Client-side encoding (vectorised); returns (packed u8[total], offsets u32[n+1])."""
     types = np.asarray(types)
     params = np.ascontiguousarray(params, dtype=np.uint8).reshape(len(types), 128)
@@ -405,19 +406,25 @@ def pack_params_compact(types, params):
             raise ValueError("NewOrder line not representable compactly (item >= 2^17 or qty outside 1..16)")
         remote = live & (sw != w[:, None])
         v = np.where(live, item | ((qty - 1) << 17) | (remote.astype(np.uint32) << 21), 0).astype(np.uint32)
-        C = np.zeros((len(no), 128), np.uint8)
+        C = np.zeros((len(no), 132), np.uint8)  # (+4: the last line's 4-byte window)
         C[:, :7] = P[:, :7]
         nrem = remote.sum(axis=1)
         C[:, 7] = nrem
-        C[:, 8:68] = v.view(np.uint8).reshape(len(no), 60)
-        # supply warehouses of remote lines at 8 + 4 nl + 2 k (k-th remote line)
+        # 22-bit lines, little-endian bit stream: line l at bits 22 l .. 22 l + 21
+        for l in range(15):
+            bit = 22 * l
+            x = v[:, l].astype(np.uint64) << np.uint64(bit & 7)
+            for j in range(4):
+                C[:, 8 + (bit >> 3) + j] |= ((x >> np.uint64(8 * j)) & np.uint64(0xFF)).astype(np.uint8)
+        lb = (22 * nl + 7) // 8
+        # supply warehouses of remote lines at 8 + lb + 2 k (k-th remote line)
         k = np.cumsum(remote, axis=1) - 1
         ri, li = np.nonzero(remote)
-        pos = 8 + 4 * nl[ri] + 2 * k[ri, li]
+        pos = 8 + lb[ri] + 2 * k[ri, li]
         C[ri, pos] = (sw[ri, li] & 0xFF).astype(np.uint8)
         C[ri, pos + 1] = (sw[ri, li] >> 8).astype(np.uint8)
-        comp[no] = C
-        used[no] = 8 + 4 * nl + 2 * nrem
+        comp[no] = C[:, :128]
+        used[no] = 8 + lb + 2 * nrem
     pay = np.nonzero(types == 1)[0]
     if len(pay):
         amount = params[pay, 16:24].copy().view(np.int64)[:, 0]

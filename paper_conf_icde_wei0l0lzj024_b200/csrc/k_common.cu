@@ -346,20 +346,23 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
     const uint32_t len = b1 - b0;
     if (b1 < b0 || b0 < lo || b1 > hi || len > 128) {
       bad = true;
-    } else if (types[r] == 0) {  // NewOrder: 8-byte header, u32 lines, u16 supply warehouses
+    } else if (types[r] == 0) {  // NewOrder: 8-byte header, 22-bit lines, u16 supply warehouses
       const uint32_t nl = len >= 8 ? q[3] : 0, nrem = len >= 8 ? q[7] : 0;
-      if (len < 8 || nl > 15 || len != 8 + 4 * nl + 2 * nrem) {
+      const uint32_t lb = (22 * nl + 7) / 8;  // bytes of the line bit stream
+      if (len < 8 || nl > 15 || len != 8 + lb + 2 * nrem) {
         bad = true;
       } else {
         for (int k = 0; k < 7; ++k) o[k] = q[k];
         const uint32_t w = ld_u16(q);
         uint32_t k = 0;
         for (uint32_t l = 0; l < nl; ++l) {
-          const uint8_t* L = q + 8 + 4 * l;
-          const uint32_t v = ld_u16(L) | ld_u16(L + 2) << 16;
+          // line l: bits 22 l .. 22 l + 21, inside the 4 bytes from byte 22 l / 8 (bytes past the
+          // record are staged too -- the stage keeps 32 bytes of slack -- and masked off here)
+          const uint8_t* L = q + 8 + (22 * l >> 3);
+          const uint32_t v = ((ld_u16(L) | ld_u16(L + 2) << 16) >> ((22 * l) & 7)) & 0x3FFFFFu;
           uint32_t sw = w;
           if ((v >> 21) & 1u) {
-            if (k < nrem) sw = ld_u16(q + 8 + 4 * nl + 2 * k);
+            if (k < nrem) sw = ld_u16(q + 8 + lb + 2 * k);
             ++k;
           }
           const uint32_t i = v & 0x1FFFFu;
