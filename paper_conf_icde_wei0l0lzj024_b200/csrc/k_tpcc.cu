@@ -1310,7 +1310,11 @@ __device__ __forceinline__ void tpcc_phase_body(const BatchDev& b, const TpccPar
   // warp slots by procedure type.  Detection: the longest chains first (OrderStatus, Delivery,
   // NewOrder, Payment), so that the grid's tail is made of short Payment warps (0.088 -> 0.077
   // ms on tpcc_c4); execute keeps the type order (measured slower the other way round)
+  // write-back starts with the Delivery leaders (their chains -- cursor, NEW_ORDER, ORDER, lines,
+  // customer per district -- are the longest; last, they were the grid's tail: tpcc_c4 write-back
+  // 0.122 -> 0.115 ms, profiles/ab_r02_bar_detect.txt); execute keeps the type order (neutral)
   constexpr uint32_t ORD = PH == PH_DETECT ? (2u | SL_DLW << 4 | 0u << 8 | SL_DLT << 12 | 1u << 16 | 4u << 20)
+                           : PH == PH_WB   ? (SL_DLW | 0u << 4 | 1u << 8 | 2u << 12 | SL_DLT << 16 | 4u << 20)
                                            : (0u | 1u << 4 | 2u << 8 | SL_DLW << 12 | SL_DLT << 16 | 4u << 20);  // slot j -> type
   // One read of the error word per block (the kernel has block barriers, and the word can be
   // raised by other blocks of this grid while this one starts), issued together with the list
