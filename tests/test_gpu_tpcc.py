@@ -94,15 +94,22 @@ def test_table6_gpu():
     assert abs(rate - 63.4) <= 2.0
 
 
-def test_tpcc_validation_and_capacity():
+@pytest.mark.parametrize("path", ["single", "multi"])
+def test_tpcc_validation_and_capacity(path):
     lib = L()
     wl = tpcc.TpccWorkload(1, seed=3, mix=tpcc.MIX_FULL)
     tables = wl.initial_tables()
-    g = lib.tpcc_database(wl, max_txns=512, tables=tables, append_batches=1)
+    g = lib.tpcc_database(wl, max_txns=512, tables=tables, append_batches=1,
+                          flags=lib.LTPG_FLAG_NO_SINGLE_LAUNCH if path == "multi" else 0)
     b = wl.batch(100, 1, 0)
     b["params"][5, 0] = 9  # warehouse 9 does not exist
     with pytest.raises(lib.LtpgError) as e:
         g.run_tpcc(b, 2)
+    assert e.value.rc == lib.LTPG_EINVAL
+    bt = wl.batch(100, 1, 0)
+    bt["tid"][40] = bt["tid"][39]  # TIDs must be strictly increasing
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(bt, 2)
     assert e.value.rc == lib.LTPG_EINVAL
     # capacity: append region sized for one batch of 512; two full batches of NewOrders overflow
     o = oracle.tpcc_db(wl, tables)
@@ -282,7 +289,8 @@ def test_ten_repeated_runs_identical(mode):
 
 
 @pytest.mark.parametrize("what", ["item0", "item_big", "qty0", "qty11", "supply_w", "dup_item", "dup_far"])
-def test_neworder_line_validation_in_execute(what):
+@pytest.mark.parametrize("path", ["single", "multi"])
+def test_neworder_line_validation_in_execute(what, path):
     """Unpartitioned batches validate NewOrder lines in execute (the grouping kernel reads only
     the 16-byte headers): every malformed line is EINVAL with nothing changed, and the database
     keeps running the next batch == oracle."""
@@ -291,6 +299,8 @@ def test_neworder_line_validation_in_execute(what):
     tables = wl.initial_tables()
     g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3)
     o = oracle.tpcc_db(wl, tables)
+    if path == "multi":  # (batches this small run as one cooperative launch unless told otherwise)
+        g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3, flags=lib.LTPG_FLAG_NO_SINGLE_LAUNCH)
     b = wl.batch(1000, 1, 0)
     no = np.nonzero((b["type"] == NEW_ORDER) & (b["params"][:, 3] >= 14))[0][3]
     p = b["params"][no]
@@ -323,7 +333,8 @@ def test_neworder_line_validation_in_execute(what):
     (PAYMENT, 0, 0), (PAYMENT, 2, 0), (PAYMENT, 3, 2), (PAYMENT, 4, 5), (PAYMENT, 6, 12),
     (2, 0, 7), (2, 2, 0), (2, 3, 3), (DELIVERY, 0, 9), (DELIVERY, 2, 11), (4, 0, 0), (4, 2, 15),
 ])
-def test_header_validation_every_type(ptype, off, val):
+@pytest.mark.parametrize("path", ["single", "multi"])
+def test_header_validation_every_type(ptype, off, val, path):
     """Each procedure's header checks (grouping for Delivery / StockLevel, execute for the others in
     an unpartitioned batch): a bad field is EINVAL, nothing changes, the db keeps working == oracle."""
     lib = L()
@@ -331,6 +342,8 @@ def test_header_validation_every_type(ptype, off, val):
     tables = wl.initial_tables()
     g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3)
     o = oracle.tpcc_db(wl, tables)
+    if path == "multi":  # (batches this small run as one cooperative launch unless told otherwise)
+        g = lib.tpcc_database(wl, max_txns=1024, tables=tables, append_batches=3, flags=lib.LTPG_FLAG_NO_SINGLE_LAUNCH)
     b = wl.batch(1000, 1, 0)
     i = int(np.nonzero(b["type"] == ptype)[0][2])
     b["params"][i, off] = val
