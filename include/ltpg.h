@@ -311,6 +311,10 @@ typedef struct {
   int outputs_on_device;        /* 1: the pointers above are device pointers             */
   ltpg_stats* stats;            /* optional host struct: per-stage device times           */
   uint32_t flags;               /* LTPG_RESULT_*                                          */
+  uint64_t reads_cap;           /* capacity of `reads` in int64 slots (0: not checked); a
+                                   batch that needs more (OPS: n_ops; TPCC: 4 x the txns it
+                                   outputs, carried ones included) is LTPG_EINVAL before any
+                                   state change                                           */
 } ltpg_result;
 
 /* Result options.  COMMITTED_READS (TPC-C): `reads` receives the 4 result slots of the COMMITTED

@@ -79,7 +79,7 @@ class ltpg_stats(ctypes.Structure):
 class ltpg_result(ctypes.Structure):
     _fields_ = [("commit_bits", c_vp), ("status", c_vp), ("abort_idx", c_vp), ("n_aborted", c_vp),
                 ("reads", c_vp), ("outputs_on_device", c_int), ("stats", ctypes.POINTER(ltpg_stats)),
-                ("flags", c_u32)]
+                ("flags", c_u32), ("reads_cap", c_u64)]
 
 
 _lib.ltpg_create_db.restype = c_int
@@ -148,6 +148,10 @@ class LtpgError(RuntimeError):
     def __init__(self, rc, msg):
         super().__init__("%s (%d): %s" % (ERR_NAMES.get(rc, "?"), rc, msg))
         self.rc = rc
+
+
+def _numel(x):
+    return int(x.numel()) if hasattr(x, "numel") else int(np.asarray(x).size)
 
 
 def _ptr(x):
@@ -259,7 +263,8 @@ class Database:
                           n_aborted=_ptr(out["n_aborted"]),
                           reads=_ptr(out["reads"]) if want_reads else None,
                           outputs_on_device=int(device_out),
-                          stats=ctypes.pointer(st) if st is not None else None, flags=rflags)
+                          stats=ctypes.pointer(st) if st is not None else None, flags=rflags,
+                          reads_cap=_numel(out["reads"]) if want_reads else 0)
         if not wait:
             bt.flags |= LTPG_BATCH_ASYNC
             self._check(ltpg_run_batch(self.h, ctypes.byref(bt), ctypes.byref(res)))

@@ -727,6 +727,9 @@ int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (db->p2p && !db->connected) return fail(db, LTPG_EINVAL, "world > 1: ltpg_connect_peers first");
   if (!ops_mode && b->proc_offsets && !b->inputs_on_device && b->proc_offsets[nf] > (uint64_t)nf * LTPG_PARAM_BYTES)
     return fail(db, LTPG_EINVAL, "packed params too large");
+  if (res->reads && res->reads_cap &&
+      res->reads_cap < (ops_mode ? (uint64_t)b->n_ops : (uint64_t)n * LTPG_PROC_RESULTS))
+    return fail(db, LTPG_EINVAL, "reads buffer smaller than the batch's result slots (reads_cap)");
   // LTPG_RESULT_COMMITTED_READS: the gather kernel writes the caller's buffer directly
   const bool cr = (res->flags & LTPG_RESULT_COMMITTED_READS) != 0;
   long long* cr_dst = nullptr;

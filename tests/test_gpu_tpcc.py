@@ -374,3 +374,19 @@ def test_l2_persist_marks_result_identical():
         ab = np.nonzero(st == ST_CONFLICT)[0]
         pending = {k: v[ab] for k, v in batch.items()} if len(ab) else None
     compare_tables(g, o)
+
+
+def test_reads_cap_einval():
+    """ltpg_result.reads_cap: a reads buffer smaller than the batch's result slots is EINVAL
+    before any state change; the db keeps working == oracle."""
+    lib = L()
+    wl, g, o = pair(1, "strict", tpcc.MIX_FULL, 512, 3, seed=31)
+    b = wl.batch(300, 1, 0)
+    out = g._outputs(300, 4 * 300, False)
+    out["reads"] = np.empty(4 * 300 - 1, np.int64)
+    with pytest.raises(lib.LtpgError) as e:
+        g.run_tpcc(b, 2, out=out)
+    assert e.value.rc == lib.LTPG_EINVAL
+    compare_tables(g, o)
+    compare(g, o, b, 2)
+    compare_tables(g, o)
