@@ -313,7 +313,10 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
                                                                   const uint8_t* __restrict__ types, uint32_t n,
                                                                   uint8_t* __restrict__ params, uint32_t* err) {
   __shared__ __align__(16) uint8_t in[UC_WARPS][32 * 128 + 32];
-  __shared__ __align__(16) uint8_t out[UC_WARPS][32 * 128];
+  // decoded blocks, rows padded to 144 bytes: with a 128-byte stride every lane's row started
+  // in the same bank (32-way conflicts on each decode store)
+  constexpr uint32_t OROW = 144;
+  __shared__ __align__(16) uint8_t out[UC_WARPS][32 * OROW];
   const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t r0 = (blockIdx.x * UC_WARPS + wib) * 32;
   if (r0 >= n) return;
@@ -334,7 +337,7 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
       for (uint32_t k = 0; k < 16; ++k) in[wib][16 * c + k] = at + k < end ? packed[at + k] : 0;
     }
   }
-  uint4* ob = reinterpret_cast<uint4*>(out[wib] + 128 * lane);
+  uint4* ob = reinterpret_cast<uint4*>(out[wib] + OROW * lane);
 #pragma unroll
   for (int k = 0; k < 8; ++k) ob[k] = make_uint4(0, 0, 0, 0);
   __syncwarp();
@@ -342,7 +345,7 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
   if (lane < cnt) {
     const uint32_t r = r0 + lane, b0 = offs[r], b1 = offs[r + 1];
     const uint8_t* q = in[wib] + (b0 - a0);
-    uint8_t* o = out[wib] + 128 * lane;
+    uint8_t* o = out[wib] + OROW * lane;
     const uint32_t len = b1 - b0;
     if (b1 < b0 || b0 < lo || b1 > hi || len > 128) {
       bad = true;
@@ -352,7 +355,12 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
       if (len < 8 || nl > 15 || len != 8 + lb + 2 * nrem) {
         bad = true;
       } else {
-        for (int k = 0; k < 7; ++k) o[k] = q[k];
+        {  // header bytes 0-6 (byte 7 stays 0) as one 8-byte store
+          unsigned long long h = 0;
+#pragma unroll
+          for (int k = 0; k < 7; ++k) h |= (unsigned long long)q[k] << (8 * k);
+          *reinterpret_cast<unsigned long long*>(o) = h;
+        }
         const uint32_t w = ld_u16(q);
         uint32_t k = 0;
         for (uint32_t l = 0; l < nl; ++l) {
@@ -365,10 +373,8 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
             if (k < nrem) sw = ld_u16(q + 8 + lb + 2 * k);
             ++k;
           }
-          const uint32_t i = v & 0x1FFFFu;
-          uint8_t* D = o + 8 + 8 * l;
-          D[0] = i & 0xFF, D[1] = (i >> 8) & 0xFF, D[2] = i >> 16, D[3] = 0;
-          D[4] = sw & 0xFF, D[5] = sw >> 8, D[6] = ((v >> 17) & 15u) + 1, D[7] = 0;
+          // u32 i | u16 supply_w | u8 qty | 0, one 8-byte store
+          *reinterpret_cast<uint2*>(o + 8 + 8 * l) = make_uint2(v & 0x1FFFFu, (sw & 0xFFFFu) | (((v >> 17) & 15u) + 1) << 16);
         }
         if (k != nrem) bad = true;
       }
@@ -386,7 +392,8 @@ __global__ void __launch_bounds__(32 * UC_WARPS) k_unpack_compact(const uint8_t*
   if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, ERR_EINVAL);
   __syncwarp();
   for (uint32_t c = lane; c < cnt * 8; c += 32)
-    *reinterpret_cast<uint4*>(params + 128ull * r0 + 16 * c) = *reinterpret_cast<const uint4*>(out[wib] + 16 * c);
+    *reinterpret_cast<uint4*>(params + 128ull * r0 + 16 * c) =
+        *reinterpret_cast<const uint4*>(out[wib] + OROW * (c >> 3) + 16 * (c & 7));
 }
 
 void launch_unpack_compact(const uint8_t* packed, const uint32_t* offs, const uint8_t* types, uint32_t n,
