@@ -14,9 +14,19 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "ltpg_internal.cuh"
 #include "tpcc_internal.cuh"
 #include "xchg.cuh"
+
+// NVTX ranges around the C-ABI calls (SURVEY §5 tracing): nsys timelines and `ncu --nvtx
+// --nvtx-include "ltpg_run_batch/"` (header-only nvtx3: no cost without an attached tool)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 
 using namespace ltpg;
 
@@ -456,6 +466,7 @@ void ltpg_destroy_db(ltpg_db* db) {
 int ltpg_load_table(ltpg_db* db, uint32_t t, const ltpg_table_desc* d, uint64_t n_rows, const uint64_t* keys,
                     const int64_t* cols) {
   if (!db) return LTPG_EINVAL;
+  NvtxRange nvtx_range("ltpg_load_table");
   if (db->poisoned) return LTPG_EPOISONED;
   if (!d || t >= db->n_tables || d->n_cols > MAXC || (d->n_cols && (!d->col_group || !d->col_is_add)) ||
       n_rows > d->capacity_rows || d->capacity_rows >= 0xFFFFFFF0ull || (n_rows && d->n_cols && !cols) ||
@@ -692,6 +703,7 @@ int ltpg_pending_aborts(ltpg_db* db, uint32_t* n) {
 
 int ltpg_wait_batch(ltpg_db* db, ltpg_result* res) {
   if (!db || !res) return LTPG_EINVAL;
+  NvtxRange nvtx_range("ltpg_wait_batch");
   for (Slot& S : db->slots)
     if (S.pending && S.res == res) return finish_slot(db, S);
   return fail(db, LTPG_EINVAL, "no batch in flight for this result");
@@ -699,6 +711,7 @@ int ltpg_wait_batch(ltpg_db* db, ltpg_result* res) {
 
 int ltpg_run_batch(ltpg_db* db, const ltpg_batch* b, ltpg_result* res) {
   if (!db) return LTPG_EINVAL;
+  NvtxRange nvtx_range("ltpg_run_batch");
   if (db->poisoned) return LTPG_EPOISONED;
   if (!b || !res || !b->tid || !res->commit_bits || !res->n_aborted ||
       (!res->status && !(res->flags & LTPG_RESULT_NO_STATUS)) ||
