@@ -1,6 +1,7 @@
 #!/usr/bin/env python
-"""Small end-to-end runs of the library for compute-sanitizer (memcheck / racecheck /
-synccheck), each checked against the oracle:  python tools/sanitize_run.py ycsb_c1|tpcc_c2|multirank
+"""Test harness, not product code: small end-to-end runs of the library for compute-sanitizer
+(memcheck / racecheck / synccheck), each checked against the oracle:
+python tests/sanitize_run.py ycsb_c1|tpcc_c2|multirank
 (multirank: 2 ranks on one GPU over CUDA IPC, gloo bootstrap; run under torch.distributed.run)."""
 import os
 import sys
