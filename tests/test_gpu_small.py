@@ -189,3 +189,26 @@ def test_single_launch_tpcc_einval_applies_nothing():
         g.run_tpcc(bad, 2)
     compare(g, o, batch, 2)
     compare_tables(g, o)
+
+
+def test_single_launch_dispatch_rule():
+    """The documented dispatch: single-partition TPC-C / OPS batches of <= 16384 txns run as ONE
+    kernel launch (ltpg_stats.n_kernels == 1); larger batches and LTPG_FLAG_NO_SINGLE_LAUNCH run
+    the multi-kernel path."""
+    from workloads import tpcc
+    lib = L()
+    wl = tpcc.TpccWorkload(2, seed=0x5A15, mode="strict", mix=tpcc.MIX_FULL)
+    tables = wl.initial_tables()
+    g = lib.tpcc_database(wl, max_txns=SMALL_MAX + 64, tables=tables, append_batches=4)
+    g2 = lib.tpcc_database(wl, max_txns=SMALL_MAX + 64, tables=tables, append_batches=4,
+                           flags=lib.LTPG_FLAG_NO_SINGLE_LAUNCH)
+    g.run_tpcc(wl.batch(1000, 1, 0), 2)  # (a db's first TPC-C batch also builds the ORDER -> lines map)
+    assert g.run_tpcc(wl.batch(1000, 1001, 5), 2, stats=True)["stats"]["n_kernels"] == 1
+    assert g.run_tpcc(wl.batch(SMALL_MAX, 2001, 1), 3, stats=True)["stats"]["n_kernels"] == 1
+    assert g.run_tpcc(wl.batch(SMALL_MAX + 1, 30000, 2), 4, stats=True)["stats"]["n_kernels"] > 5
+    assert g2.run_tpcc(wl.batch(1000, 1, 0), 2, stats=True)["stats"]["n_kernels"] > 5
+    y = YcsbWorkload(10_000, theta=0.5, ops_per_txn=4, seed=0x17C0)
+    keys, cols = y.initial_table()
+    gy, _ = make_pair({0: tuple(y.table_desc()[:3])}, {0: (keys, cols)}, 2048, 8192)
+    gy.run_ops(y.batch(1024, 1, 0))
+    assert gy.run_ops(y.batch(1024, 1025, 1), stats=True)["stats"]["n_kernels"] == 1
