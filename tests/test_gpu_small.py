@@ -212,3 +212,13 @@ def test_single_launch_dispatch_rule():
     gy, _ = make_pair({0: tuple(y.table_desc()[:3])}, {0: (keys, cols)}, 2048, 8192)
     gy.run_ops(y.batch(1024, 1, 0))
     assert gy.run_ops(y.batch(1024, 1025, 1), stats=True)["stats"]["n_kernels"] == 1
+
+
+def test_single_launch_graph_replay_after_multi_kernel_batch():
+    """LTPG_FLAG_GRAPH: a captured single-launch batch is replayed after a multi-kernel batch left
+    the batch scratch dirty (the captured graph carries the scratch clears) -- == oracle."""
+    from tests.test_gpu_tpcc import compare_tables
+    from workloads import tpcc
+    wl, _, g, o = _tpcc_pair(2, "strict", tpcc.MIX_FULL, 20000, 8, seed=0x5A16, flags=L().LTPG_FLAG_GRAPH)
+    _tpcc_loop(wl, g, o, [700, 700, 17000, 700, 700, 17000, 700])
+    compare_tables(g, o)
