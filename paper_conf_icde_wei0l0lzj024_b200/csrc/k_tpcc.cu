@@ -1461,7 +1461,12 @@ __device__ __forceinline__ void tpcc_phase_body(const BatchDev& b, const TpccPar
     tpcc_advance_tail(b, tp);
 }
 template <int PH, uint32_t TMASK>
-__global__ void __launch_bounds__(256, (PH == PH_EXEC ? LTPG_EXEC_MINB : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
+#ifndef LTPG_EXEC_THREADS
+#define LTPG_EXEC_THREADS 256
+#endif
+__global__ void __launch_bounds__(PH == PH_EXEC ? LTPG_EXEC_THREADS : 256,
+                                  (PH == PH_EXEC ? LTPG_EXEC_MINB * 256 / LTPG_EXEC_THREADS
+                                                 : PH == PH_DETECT ? LTPG_DETECT_MINB : LTPG_WB_MINB))
     k_tpcc_phase(BatchDev b, TpccParams tp) {
   tpcc_phase_body<PH, TMASK, false>(b, tp, blockIdx.x, gridDim.x);
 }
@@ -2208,7 +2213,8 @@ template <int PH>
 static uint32_t resident_grid(uint32_t n, size_t smem) {
   static int per_sm[3][2] = {{0, 0}, {0, 0}, {0, 0}};  // by phase, by dynamic shared memory or not
   int& b = per_sm[PH][smem ? 1 : 0];
-  if (!b && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_tpcc_phase<PH, TM_MAIN>, 256, smem) != cudaSuccess)
+  if (!b && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_tpcc_phase<PH, TM_MAIN>,
+                                                          PH == PH_EXEC ? LTPG_EXEC_THREADS : 256, smem) != cudaSuccess)
     b = 2;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -2242,7 +2248,7 @@ int tpcc_front(TpccDev& t, BatchDev& b, cudaStream_t s, cudaEvent_t* ev, bool cl
   k_sl_claim<<<148 * 2, 256, 0, t.side>>>(b, tp, sl);
   k_sl_district<<<148 * 2, 256, 0, t.side>>>(b, sl);
   cudaEventRecord(t.join[0], t.side);
-  k_tpcc_phase<PH_EXEC, TM_MAIN><<<resident_grid<PH_EXEC>(n, tp.hot_words * sizeof(mark_t)), 256,
+  k_tpcc_phase<PH_EXEC, TM_MAIN><<<resident_grid<PH_EXEC>(n, tp.hot_words * sizeof(mark_t)), LTPG_EXEC_THREADS,
                                    tp.hot_words * sizeof(mark_t), s>>>(b, tp);
   cudaStreamWaitEvent(s, t.join[0], 0);  // detection reads the marks of every execute warp
   note_launch(3);
